@@ -1,0 +1,367 @@
+#!/usr/bin/env python3
+"""Benchmark of the B200 state-vector hot path (BASELINE.json metric).
+
+Metric: RQC circuit time in seconds (lower is better) and the apply kernels'
+achieved HBM bandwidth.  N=1 workload: BASELINE.json configs[1], the paper's
+30-qubit RQC at depth 14 with max_fused = 4 (the paper's
+optimum, L189).  A "step" is one pass of the whole hot path:
+|0..0> init, every fused-gate apply of the circuit, and drawing 10^6 samples.
+
+  value  -- device time per step with the fused circuit already resident
+            (sv_circuit_run_device + sv_sample_device), CUDA events on the
+            library's stream, max over ranks.
+  e2e    -- the same step through the public C ABI with host buffers:
+            sv_reset + sv_run_circuit (host gates -> fusion -> upload ->
+            kernels) + sv_sample into host memory.
+
+N>1 (torchrun): the multi-process sharded mode (one shard per GPU, P2P
+exchanges), weak scaling with 2^30 amplitudes per GPU (n = 30 + log2 N)
+unless --qubits is given (e.g. --qubits 36 for the north star's 36q run).
+
+--impl reference: the CPU oracle (oracle/sv_ref.c, complex128, unfused,
+OpenMP on the host cores) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from workloads import rqc as W  # noqa: E402
+
+N_SAMPLES = 1_000_000
+REASON_BITS = {
+    0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+    0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+    0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--qubits", type=int, default=0)
+    ap.add_argument("--depth", type=int, default=14)
+    ap.add_argument("--max-fused", type=int, default=4)
+    ap.add_argument("--seed", type=int, default=2023)
+    ap.add_argument("--samples", type=int, default=N_SAMPLES)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    return ap.parse_args()
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured"
+    return 6650.0, "fallback"
+
+
+def load_traffic(kernel_class: str):
+    """Per-launch dram bytes of the dominant kernel from the committed ncu
+    summary (profiles/ncu_summary.json), if present."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        return d.get("traffic_per_launch", {}).get(kernel_class)
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index),
+                 "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 3:
+                try:
+                    self.rows.append((float(parts[0]), float(parts[1]), int(parts[2], 16)))
+                except ValueError:
+                    pass
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        load = [r for r in self.rows if not (r[2] & 0x1)] or self.rows
+        reasons = set()
+        for r in load:
+            for bit, name in REASON_BITS.items():
+                if r[2] & bit and bit != 0x1:
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(r[0] for r in load), "sm_max_mhz": max(r[1] for r in self.rows),
+                "reasons": sorted(reasons), "samples": len(load)}
+
+
+# ----------------------------------------------------------------------------- CPU oracle
+def cpu_oracle_sample(n: int, gates, seconds: float):
+    """Time the oracle (unfused complex128 C simulator) on the first gates of
+    the workload circuit; extrapolate to seconds per circuit."""
+    import psutil
+
+    from oracle import ref_c
+    n_eff = n
+    avail = psutil.virtual_memory().available
+    while n_eff > 20 and (16 << n_eff) > 0.6 * avail:
+        n_eff -= 1
+    sub = W.rqc(n_eff, 14, 2023) if n_eff != n else gates
+    done, sec = ref_c.time_gates(n_eff, sub, max_seconds=seconds)
+    per_gate = sec / done
+    scale = 2.0 ** (n - n_eff)
+    value = per_gate * len(gates) * scale
+    sample = (f"first {done} of {len(sub)} unfused gates of the {n_eff}q depth-14 RQC in {sec:.1f} s "
+              f"({per_gate * 1e3:.1f} ms/gate), extrapolated x{len(gates)} gates"
+              + (f" x{scale:.0f} (2^{n - n_eff}: host RAM too small for 2^{n} complex128)" if scale > 1 else ""))
+    return {"value": value, "unit": "s", "cores": ref_c.threads(), "kind": "oracle", "sample": sample}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n = args.qubits or (30 if args.gpus == 1 else 30 + (args.gpus.bit_length() - 1))
+    gates = W.rqc(n, args.depth, args.seed)
+    vals = []
+    last = None
+    for _ in range(args.warmup):
+        cpu_oracle_sample(n, gates, min(3.0, args.cpu_seconds))
+    for _ in range(args.steps):
+        last = cpu_oracle_sample(n, gates, args.cpu_seconds)
+        vals.append(last["value"])
+    v = statistics.mean(vals)
+    cfg = {"workload": f"rqc_{n}q_d{args.depth}_f{args.max_fused}", "n_qubits": n, "depth": args.depth,
+           "max_fused": args.max_fused, "seed": args.seed}
+    last["value"] = v
+    out = {"impl": "reference", "metric": f"rqc_circuit_time_{n}q_d{args.depth}", "value": v, "unit": "s",
+           "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": v * 1e3,
+           "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic", "config": cfg, "cpu_baseline": last,
+           "e2e": {"value": v, "unit": "s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# ----------------------------------------------------------------------------- ours
+def run_ours(args):
+    import torch
+
+    import paper_conf_sc_markidis23_b200 as sv
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n = args.qubits or (30 if world == 1 else 30 + (world.bit_length() - 1))
+    gates = W.rqc(n, args.depth, args.seed)
+    stream = torch.cuda.Stream()
+    if world == 1:
+        h = sv.sv_create_ex(n, cuda_stream=stream.cuda_stream)
+    else:
+        h = sv.sv_create_ex(n, world=world, rank=rank, virtual_shards=False, cuda_stream=stream.cuda_stream)
+        blob = sv.sv_ipc_handle(h)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, blob)
+        sv.sv_attach_peers(h, blobs)
+    samples_dev = torch.empty(args.samples, dtype=torch.int64, device="cuda")
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # ---- device step: fused circuit resident
+    circ = sv.sv_circuit_create(h, gates, args.max_fused)
+    cst = sv.sv_circuit_stats(circ)
+
+    def device_step():
+        sv.sv_reset(h)
+        sv.sv_circuit_run_device(h, circ)
+        sv.sv_sample_device(h, 1, args.samples, samples_dev.data_ptr())
+
+    for _ in range(max(args.warmup, 1)):
+        device_step()
+    sv.sv_synchronize(h)
+    barrier()
+    sv.sv_set_timing(h, True)
+    sv.sv_last_stats(h)  # drain
+    t_apply = t_high = t_low = t_exch = t_other = 0.0
+    n_high = n_low = n_other = 0
+    bytes_apply = 0
+    flops = 0
+    bytes_exch = 0
+    with ClockSampler(local) as clk:
+        start = torch.cuda.Event(enable_timing=True)
+        end = torch.cuda.Event(enable_timing=True)
+        barrier()
+        start.record(stream)
+        for _ in range(args.steps):
+            device_step()
+            st = sv.sv_last_stats(h)  # syncs + collects per-launch event times of this step
+            t_high += st["t_apply_high_dev_s"]
+            t_low += st["t_apply_low_dev_s"]
+            t_exch += st["t_exchange_dev_s"]
+            t_other += st["t_other_dev_s"]
+            n_high += st["n_launch_high"]
+            n_low += st["n_launch_low"]
+            n_other += st["n_launch_other"]
+            bytes_apply += st["bytes_apply"]
+            flops += st["flops_apply"]
+            bytes_exch += st["bytes_exchange"]
+        end.record(stream)
+        barrier()
+    sv.sv_set_timing(h, False)
+    ms = start.elapsed_time(end) / args.steps
+    # the per-step sv_last_stats sync adds a host round trip per step; report
+    # the device-side sum of our launches as well
+    t_apply = t_high + t_low
+    ms_t = torch.tensor([ms], device="cuda")
+    if dist is not None:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms = float(ms_t.item())
+
+    # ---- end-to-end through the public API with host buffers
+    host_samples = np.empty(args.samples, dtype=np.uint64)
+    g_arr = sv.as_gates(gates)
+
+    def e2e_step():
+        sv.sv_reset(h)
+        sv.sv_run_circuit(h, g_arr, args.max_fused)
+        out = sv.sv_sample(h, 1, args.samples)
+        host_samples[:] = out
+
+    e2e_step()
+    barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e2e_steps = max(1, min(args.steps, 3))
+    e0.record(stream)
+    for _ in range(e2e_steps):
+        e2e_step()
+    e1.record(stream)
+    barrier()
+    e2e_ms = e0.elapsed_time(e1) / e2e_steps
+    et = torch.tensor([e2e_ms], device="cuda")
+    if dist is not None:
+        dist.all_reduce(et, op=dist.ReduceOp.MAX)
+    e2e_ms = float(et.item())
+    h2d = int(sum(8 * (1 << (2 * k)) * c for k, c in enumerate(cst["fused_hist"])))
+
+    peak, peak_src = load_peaks()
+    launches_apply = n_high + n_low
+    avg_launch = t_apply / max(launches_apply, 1)
+    bytes_per_launch = 16 * (1 << (n - (world.bit_length() - 1)))
+    achieved = bytes_per_launch / avg_launch / 1e9 if avg_launch > 0 else None
+    frac = achieved / peak if achieved else None
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            cpu = cpu_oracle_sample(n, gates, args.cpu_seconds)
+        except Exception as ex:  # host RAM / build issues must not kill the bench line
+            cpu = {"value": None, "unit": "s", "cores": os.cpu_count(), "kind": "oracle",
+                   "sample": f"failed: {ex}"}
+    if rank == 0:
+        sv_fused = cst["n_fused"]
+        out = {
+            "metric": f"rqc_circuit_time_{n}q_d{args.depth}_f{args.max_fused}",
+            "value": ms / 1e3,
+            "unit": "s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": ms,
+            "higher_is_better": False,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "f32",
+            "data": "synthetic",
+            "config": {
+                "workload": f"rqc_{n}q_d{args.depth}_f{args.max_fused}",
+                "n_qubits": n, "depth": args.depth, "max_fused": args.max_fused, "seed": args.seed,
+                "gates": len(gates), "n_fused": sv_fused, "fused_hist": cst["fused_hist"],
+                "samples_per_step": args.samples,
+                "step": "sv_reset + all fused-gate applies + sv_sample_device(1e6)",
+                "l2": f"inputs larger than L2 (state {8 << n >> 30} GiB per circuit)",
+                "parallelism": "single GPU" if world == 1 else f"sharded x{world} (P2P exchange)",
+                "apply_ms_per_step": 1e3 * t_apply / args.steps,
+                "apply_high_ms_per_step": 1e3 * t_high / args.steps,
+                "apply_low_ms_per_step": 1e3 * t_low / args.steps,
+                "exchange_ms_per_step": 1e3 * t_exch / args.steps,
+                "other_ms_per_step": 1e3 * t_other / args.steps,
+                "apply_gbs_high": (16 << (n - (world.bit_length() - 1))) * n_high / t_high / 1e9 if t_high else None,
+                "apply_gbs_low": (16 << (n - (world.bit_length() - 1))) * n_low / t_low / 1e9 if t_low else None,
+                "apply_tflops": flops / t_apply / 1e12 if t_apply else None,
+                "fuse_plan_upload_s": cst["t_fuse_s"] + cst["t_plan_s"] + cst["t_upload_s"],
+            },
+            "roofline": {"bound": "hbm", "kernel": "apply_high+apply_low", "achieved": achieved, "peak": peak,
+                         "peak_source": peak_src, "unit": "GB/s", "frac": frac,
+                         "frac_of_8tbs": achieved / 8000.0 if achieved else None,
+                         "algorithmic_bytes_per_launch": bytes_per_launch,
+                         "traffic": load_traffic("apply")},
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_ms / 1e3, "unit": "s", "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": 8 * args.samples},
+            "gpu_launches": (n_high + n_low + n_other),
+            "clocks": clk.summary(),
+        }
+        print(json.dumps(out), flush=True)
+    sv.sv_circuit_destroy(circ)
+    sv.sv_destroy(h)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,206 @@
+/*
+ * sv.h -- C ABI of the B200 state-vector hot path (libsvb200.so).
+ *
+ * What the library computes (citations: /root/reference/PAPER.md line Lnnn):
+ *   - a state of n qubits is 2^n complex amplitudes; |c_i|^2 is the
+ *     probability of |i> (L69, §2.2);
+ *   - a gate G acts as psi' = G psi, applied matrix-free and in place
+ *     (L71-93, §2.2, Figs. 3-4); the 2^n outputs split into 2^(n-k)
+ *     independent groups of a 2^k x 2^k complex matvec (L93);
+ *   - gates are fused in space (tensor product) and time (ordered matrix
+ *     product) up to a "maximum of fused gates" (L98-104, Fig. 5);
+ *   - gates on high qubits and on low qubits run in different kernels
+ *     (L110-112, §2.3);
+ *   - amplitudes can be read and measurement outcomes sampled (L131-132, §3).
+ *
+ * Conventions (SURVEY.md §8c readings Q1/Q3):
+ *   - qubit q is bit q of the basis index (little-endian, qubit 0 = stride 1);
+ *   - amplitudes are interleaved complex64 (sv_c64 == cuFloatComplex ==
+ *     torch.complex64), fp32 arithmetic on the device;
+ *   - a k-qubit matrix is row-major 2^k x 2^k; bit b of its row/column index
+ *     belongs to qubits[b]; qubits[] may be in any order.
+ *
+ * Errors: every call returns int; SV_OK = 0, negative = error.  Nothing
+ * throws or exits.  sv_last_error() returns a thread-local message for the
+ * last failing call on this thread.  Arguments are validated before any side
+ * effect.  After a failed asynchronous device operation a handle is sticky
+ * SV_EBADSTATE until sv_destroy().
+ *
+ * Ownership: every input array is caller-owned and fully consumed (copied)
+ * before the call returns; the library keeps no caller pointers except a
+ * caller-provided device buffer (sv_config.dev_buf), which the caller must
+ * keep alive until sv_destroy().  Output arrays are caller-allocated host
+ * memory.
+ *
+ * Streams / sync: all device work of a handle runs on its stream (its own, or
+ * sv_config.cuda_stream).  sv_apply_fused and sv_circuit_run_device are
+ * asynchronous w.r.t. the host; sv_run_circuit, sv_amplitudes, sv_sample and
+ * sv_get_state synchronise the stream before returning.
+ *
+ * Threading: a handle is not thread-safe; distinct handles are independent.
+ *
+ * Sharded mode (north star; PAPER.md L209/L229 name multi-GPU as future
+ * work): the 2^n state is split into P = 2^g shards of 2^(n-g) amplitudes by
+ * the top g PHYSICAL qubits.  Either all P shards live on this GPU
+ * (virtual_shards = 1, used to test the exchange path on one device) or each
+ * of P processes owns one shard and the processes exchange peer-memory
+ * handles with sv_ipc_handle / sv_attach_peers (one GPU per process, NVLink
+ * P2P).  In multi-process mode every rank makes the same calls with the same
+ * arguments (collective semantics) and receives identical results.
+ */
+#ifndef SV_B200_H
+#define SV_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SV_OK 0
+#define SV_EINVAL (-1)        /* bad argument (range, NULL with count>0, dup qubit, ...) */
+#define SV_ENOMEM (-2)        /* device or host allocation failed                          */
+#define SV_ECUDA (-3)         /* CUDA runtime error (message in sv_last_error)            */
+#define SV_ECOMM (-4)         /* peer attach / P2P error in sharded mode                   */
+#define SV_EUNSUPPORTED (-5)  /* world not a power of two, shard too small, ...          */
+#define SV_EBADSTATE (-6)     /* handle poisoned by an earlier asynchronous failure        */
+
+#define SV_MAX_QUBITS 40      /* per handle (all shards) */
+#define SV_MAX_FUSED 6        /* k <= 6: dense 64 x 64 fused matrices */
+
+typedef struct sv_state sv_state;       /* opaque: device state + qubit map */
+typedef struct sv_circuit sv_circuit;   /* opaque: fused, planned and uploaded circuit */
+
+typedef struct { float re, im; } sv_c64;
+typedef struct { double re, im; } sv_c128;
+
+/* One input gate (1 or 2 qubits).  m is row-major 2^nq x 2^nq (a 1-qubit gate
+ * uses m[0..3]); bit b of the matrix index <-> q[b].  fp64 so that fusion
+ * (in fp64) rounds to complex64 once per fused gate. */
+typedef struct {
+    int32_t nq;
+    int32_t q[2];
+    int32_t pad_;
+    sv_c128 m[16];
+} sv_gate;
+
+/* Statistics of the last sv_run_circuit / sv_circuit_run_device.  Host times
+ * are wall-clock; t_apply_*_dev / t_exchange_dev / t_sample_dev are summed
+ * CUDA-event durations around each launch and are filled only when timing is
+ * enabled with sv_set_timing(s, 1).  Bytes are ALGORITHMIC: 16 B per
+ * amplitude per apply pass, sent bytes per exchange. */
+typedef struct {
+    int32_t n_fused;            /* fused gates in the plan                       */
+    int32_t n_exchanges;        /* exchange events (sharded)                     */
+    int32_t fused_hist[7];      /* fused gates by size k = 0..6                  */
+    int32_t n_launch_high;      /* high-qubit apply launches                     */
+    int32_t n_launch_low;       /* low/mixed-qubit apply launches                */
+    int32_t n_launch_other;     /* reset / permute / exchange / sample launches  */
+    double t_fuse_s, t_plan_s, t_upload_s, t_total_s;
+    double t_apply_high_dev_s, t_apply_low_dev_s, t_exchange_dev_s, t_other_dev_s;
+    uint64_t bytes_apply;       /* per shard */
+    uint64_t bytes_exchange;    /* sent per shard */
+    uint64_t flops_apply;       /* (8*2^k - 2) per amplitude per fused gate, per shard */
+} sv_stats;
+
+typedef struct {
+    int32_t n_qubits;        /* total qubits n, 1..SV_MAX_QUBITS                          */
+    int32_t world;           /* P = number of shards (power of two); 0 or 1 = unsharded   */
+    int32_t rank;            /* this process's shard in multi-process mode, else 0        */
+    int32_t virtual_shards;  /* 1: all P shards on this GPU (single process)              */
+    int32_t exchange_vmin;   /* planner victim floor (S4); < 0 = default 5                */
+    int32_t device;          /* CUDA device ordinal; < 0 = current device                 */
+    void* dev_buf;           /* optional caller-owned device buffer for the state, or NULL */
+    size_t buf_bytes;        /* size of dev_buf: >= 8 * 2^n / (world if multi-process)    */
+    void* cuda_stream;       /* optional cudaStream_t; NULL = library-owned stream        */
+} sv_config;
+
+/* ---- lifetime ------------------------------------------------------------- */
+/* 1 GPU (current device), state = |0...0>.  n in [1, SV_MAX_QUBITS]. */
+int sv_create(int n_qubits, sv_state** out);
+/* General form (sharded / caller-owned buffer / caller stream). */
+int sv_create_ex(const sv_config* cfg, sv_state** out);
+int sv_destroy(sv_state* s);
+/* |0...0> and the identity qubit map. Asynchronous. */
+int sv_reset(sv_state* s);
+
+/* ---- the hot path ----------------------------------------------------------- */
+/* Apply one dense k-qubit matrix (1 <= k <= 6) in place.  qubits distinct and
+ * < n in any order; matrix row-major 2^k x 2^k complex64, bit b <-> qubits[b]
+ * (logical qubits: in sharded mode an exchange is inserted when needed).
+ * Asynchronous: the matrix is staged before return. */
+int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix);
+
+/* Fuse (max_fused in [0,6]; 0 = no fusion), plan (sharded), upload and apply a
+ * whole circuit of 1-2 qubit gates, synchronising before return.  stats may be
+ * NULL. Equivalent to sv_circuit_create + sv_circuit_run + sv_circuit_destroy. */
+int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_stats* stats);
+
+/* Prepared circuits: fusion, planning and the single H2D upload of all fused
+ * matrices happen in sv_circuit_create; sv_circuit_run_device only launches
+ * kernels (asynchronous; the timed "device" step of bench.py). */
+int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out);
+int sv_circuit_run_device(sv_state* s, const sv_circuit* c);
+int sv_circuit_stats(const sv_circuit* c, sv_stats* stats);
+int sv_circuit_destroy(sv_circuit* c);
+
+/* Read `count` amplitudes at LOGICAL indices idx[] into out[] (host). */
+int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out);
+
+/* Draw n_samples basis states (LOGICAL indices) with the integer fixed-point
+ * sampler: bit-identical for a given complex64 state and
+ * seed under any parallel decomposition.  SV_EINVAL if the total weight is 0
+ * or sum |c|^2 >= 3.99.  out[] is host memory of n_samples uint64. */
+int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out);
+/* Device form: writes n_samples uint64 into device memory dev_out
+ * (asynchronous; the bench's device step). */
+int sv_sample_device(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* dev_out);
+
+/* ---- whole-state access (tests, debugging) ------------------------------ */
+/* Copy 2^n amplitudes in LOGICAL order from host (set) / to host (get). In
+ * multi-process mode each rank passes/receives the FULL vector. */
+int sv_set_state(sv_state* s, const sv_c64* host, size_t count);
+int sv_get_state(sv_state* s, sv_c64* host, size_t count);
+/* Device pointer of shard `shard` (virtual mode) / of this rank's shard. */
+int sv_device_ptr(sv_state* s, int shard, void** out);
+
+/* ---- pure host helpers (no GPU needed) ------------------------------------ */
+/* Fusion plan as a flat int32 stream: per fused gate
+ *   k, q_0..q_{k-1} (ascending), n_mem, mem_0..mem_{n_mem-1} (ascending).
+ * *need gets the required length; if cap < *need returns SV_EINVAL and
+ * writes nothing to buf.  (SURVEY.md §8b / §8c-S3.) */
+int sv_fusion_plan(const sv_gate* gates, size_t n_gates, int max_fused, int32_t* buf, size_t cap, size_t* need);
+/* Fused matrix of fused gate `index` of that plan, complex128 row-major over
+ * the ascending qubit list (computed in fp64). out holds 4^k entries. */
+int sv_fused_matrix(const sv_gate* gates, size_t n_gates, int max_fused, size_t index, sv_c128* out, size_t cap);
+/* Sharded plan (S4) for fused qubit sets given as the sv_fusion_plan stream.
+ * Output stream: per event  X: -1, s, P_0, p_0, ...;  A: i, k, phys_0..phys_{k-1}.
+ * final_pos (n entries, may be NULL) receives logical -> physical positions. */
+int sv_shard_plan(const int32_t* fusion_stream, size_t len, int n_qubits, int log2_world, int vmin,
+                  int32_t* buf, size_t cap, size_t* need, int32_t* final_pos);
+/* Current logical -> physical qubit map (n entries). */
+int sv_qubit_map(const sv_state* s, int32_t* pos);
+
+/* ---- sharded multi-process plumbing --------------------------------------- */
+/* Opaque bytes describing this rank's shard and control block for peers
+ * (CUDA IPC handles). *need gets the size; cap < *need -> SV_EINVAL. */
+int sv_ipc_handle(sv_state* s, void* out, size_t cap, size_t* need);
+/* handles: world blobs of `each` bytes in rank order (from an all-gather). */
+int sv_attach_peers(sv_state* s, const void* handles, size_t each);
+
+/* ---- misc ------------------------------------------------------------------- */
+/* 1: record CUDA events around every launch and fill the *_dev_s stats. */
+int sv_set_timing(sv_state* s, int enable);
+/* Stats of the most recent run on this handle. */
+int sv_last_stats(const sv_state* s, sv_stats* out);
+/* Synchronise the handle's stream. */
+int sv_synchronize(sv_state* s);
+const char* sv_last_error(void);
+/* Library version string. */
+const char* sv_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SV_B200_H */

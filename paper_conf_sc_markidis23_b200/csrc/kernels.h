@@ -1,0 +1,82 @@
+// kernels.h -- launch descriptors and launchers of the device kernels
+// (internal to libsvb200; host code never sees a template).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <vector>
+
+#include "sv_internal.h"
+
+namespace svb {
+
+// Qubit-class split (qsim splits at log2(32) = 5 for a
+// 32-lane warp of 1 amplitude/lane).  On B200 a lane moves 16 B (2 amps) and
+// 8 lanes fill a 128 B line, so a gate is "high" when none of its qubits is
+// 1, 2 or 3 (qubit 0 lives inside a lane's float4).  Everything else is
+// "low" and goes through a shared-memory tile.
+constexpr uint64_t kLowMask = 0xEull;  // qubits {1,2,3}
+
+struct ApplyDesc {
+    int k = 0;
+    int q[SV_MAX_FUSED] = {0};        // ascending physical qubits (within a shard)
+    std::vector<cf> m;                // 2^k x 2^k row-major over ascending q, complex64
+    bool high = false;                // kernel class
+    // low-kernel tile plan (host-computed once)
+    int T = 0, r = 0;                 // tile bits, run bits
+    // device copy of m for k == 6 (owned by the circuit / state scratch)
+    const float2* dev_m = nullptr;
+};
+
+// Decide high/low and the tile plan for a gate on `n` local qubits.
+void plan_apply(int n_local, ApplyDesc& d);
+
+// Launch one fused-gate apply on a shard of 2^n_local amplitudes.
+cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);
+
+// |0...0> on a shard (one=true puts 1 at index 0).
+cudaError_t launch_reset(float2* psi, uint64_t n_amps, bool one, cudaStream_t st);
+
+// out[i] = psi_shard[ phys_index[i] ] for entries owned by this shard
+// (owner[i] == shard), others untouched.
+cudaError_t launch_gather(const float2* psi, const uint64_t* phys, const int32_t* owner, int shard,
+                          uint64_t count, float2* out, cudaStream_t st);
+
+// ---- sampling (S5) ----------------------------------------------------------
+constexpr int kSampleBinBits = 5;  // 32 amplitudes per fine bin
+// bins[b] = sum over the 32 amplitudes of bin b of floor(p * 2^62)
+cudaError_t launch_bin_weights(const float2* psi, uint64_t n_amps, uint64_t* bins, cudaStream_t st);
+// inclusive prefix sum in place over `count` uint64 (scratch: >= scan_scratch_elems(count))
+size_t scan_scratch_elems(uint64_t count);
+cudaError_t launch_inclusive_scan(uint64_t* data, uint64_t count, uint64_t* scratch, cudaStream_t st);
+// Resolve samples s in [0, n_samples): t_s = (splitmix64#(s+1)(seed) * T) >> 64
+// with T = *total_dev (+ global offset); samples whose t falls into this
+// shard's range [range_lo, range_lo + local_total) are written as
+// logical index = index_base + local index.  Others untouched.
+cudaError_t launch_sample_resolve(const float2* psi, uint64_t n_amps, const uint64_t* cum_bins, uint64_t n_bins,
+                                  const uint64_t* range_lo_dev, const uint64_t* total_dev, uint64_t seed,
+                                  uint64_t n_samples, uint64_t index_base, uint64_t* out, cudaStream_t st);
+
+// offsets of shard totals in LOGICAL shard order: lo[d] = sum of totals of
+// shards whose logical index sigma[d'] < sigma[d]; *total = sum of all.
+// totals_src[d] points at shard d's total (last inclusive-prefix element).
+cudaError_t launch_shard_offsets(const uint64_t* const* totals_src_dev, const int32_t* sigma_dev, int world,
+                                 uint64_t* lo_dev, uint64_t* total_dev, cudaStream_t st);
+// out[i] = min over r < world of src[r][i] (merge of per-rank partial results)
+cudaError_t launch_merge_min(const uint64_t* const* src_dev, int world, uint64_t count, uint64_t* out, cudaStream_t st);
+// device-side barrier over P2P-mapped flag words (multi-process sharded mode)
+cudaError_t launch_barrier(uint64_t* const* flags_dev, int world, int me, uint64_t epoch, cudaStream_t st);
+
+// ---- sharded exchange (S4 semantics) -----------------------------------------
+struct ExchangeDesc {
+    int l = 0;                       // local bits
+    int s = 0;                       // number of pairs
+    int P[8] = {0}, p[8] = {0};      // global positions (>= l) and local positions
+};
+// Swap chunks among shards: shards[d] points at shard d's amplitudes (local or
+// peer-mapped).  Work is split so that rank `me` of `world` does its share of
+// every pair (all pairs of all shards when me < 0: virtual mode).
+cudaError_t launch_exchange(float2* const* shards_dev, int world, int me, const ExchangeDesc& x, cudaStream_t st);
+
+}  // namespace svb

@@ -1,0 +1,1090 @@
+// sv_api.cpp -- the C ABI of include/sv.h: validation, error handling, the
+// dispatcher that turns a circuit into kernel launches (SURVEY.md §8 rows
+// a0-a9, b), and the sharded-mode plumbing.
+//
+// PAPER.md §3 (L128-135) describes the layering this replaces: an app reads
+// a circuit and "maximum number of fused gates" (L128), a simulator class
+// applies gates and launches the kernels (L129-130), a state-space class
+// sets states, gets amplitudes and samples (L131-132).  Here all of it sits
+// behind plain C calls; PyTorch is only a possible owner of the buffer and
+// stream.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+#include "sv_internal.h"
+
+using namespace svb;
+
+namespace svb {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string& msg) { g_err = msg; }
+int fail(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+
+}  // namespace svb
+
+namespace {
+
+double now_s() {
+    return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+struct Ctrl {               // per-rank control block (device memory, IPC-shared)
+    uint64_t flags[64];     // barrier epochs written by each rank
+    uint64_t total;         // this rank's sampling total
+    uint64_t pad[63];
+};
+
+constexpr size_t kXferBytes = 64ull << 20;  // per-rank exchange area for samples / amplitudes
+
+enum class LaunchClass { HIGH = 0, LOW = 1, EXCH = 2, OTHER = 3 };
+
+}  // namespace
+
+struct sv_state {
+    int n = 0, g = 0, l = 0;
+    int world = 1;            // P
+    int rank = 0;
+    bool virt = true;         // all shards on this GPU
+    int device = 0;
+    int vmin = 5;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    std::vector<float2*> shard;        // shard pointers (local or peer-mapped)
+    float2** shard_dev = nullptr;      // device copy of shard pointers
+    void* alloc = nullptr;             // library-owned state allocation
+    std::vector<int> pos;              // logical -> physical
+    int sticky = SV_OK;
+    // scratch
+    uint64_t* bins = nullptr;          // world_local * n_bins
+    uint64_t* scan_scratch = nullptr;
+    uint64_t* misc = nullptr;          // [0..63] lo, [64] total, [65..] totals ptrs area
+    uint64_t** totals_ptr_dev = nullptr;
+    int32_t* sigma_dev = nullptr;
+    float2* kmat = nullptr;            // k=6 matrix for sv_apply_fused
+    // multi-process
+    Ctrl* ctrl = nullptr;
+    uint64_t* xfer = nullptr;          // kXferBytes
+    std::vector<Ctrl*> peer_ctrl;
+    std::vector<uint64_t*> peer_xfer;
+    uint64_t** flags_dev = nullptr;
+    uint64_t** xfer_dev = nullptr;
+    uint64_t epoch = 0;
+    bool attached = false;
+    std::vector<void*> ipc_opened;
+    // timing
+    bool timing = false;
+    struct Rec {
+        LaunchClass cls;
+        cudaEvent_t a, b;
+    };
+    std::vector<Rec> recs;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    sv_stats stats{};
+    // reusable device buffers
+    uint64_t* idx_dev = nullptr;
+    size_t idx_cap = 0;
+    float2* amp_dev = nullptr;
+    size_t amp_cap = 0;
+    uint64_t* samp_dev = nullptr;
+    size_t samp_cap = 0;
+
+    uint64_t local_amps() const { return 1ull << l; }
+    int local_shards() const { return virt ? world : 1; }
+};
+
+struct sv_circuit {
+    sv_state* owner = nullptr;
+    std::vector<int> pos_in, pos_out;
+    struct Step {
+        Event::Type type;
+        ApplyDesc apply;
+        ExchangeDesc exch;
+        std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
+    };
+    std::vector<Step> steps;
+    float2* dev_mats = nullptr;
+    sv_stats stats{};
+};
+
+namespace {
+
+int cuda_fail(sv_state* s, cudaError_t e, const char* what) {
+    if (s) s->sticky = SV_EBADSTATE;
+    return fail(SV_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(s, expr)                                             \
+    do {                                                        \
+        cudaError_t e__ = (expr);                               \
+        if (e__ != cudaSuccess) return cuda_fail((s), e__, #expr); \
+    } while (0)
+
+int check_state(sv_state* s) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    if (s->sticky != SV_OK) return fail(SV_EBADSTATE, "state poisoned by an earlier device failure");
+    return SV_OK;
+}
+
+cudaEvent_t next_event(sv_state* s) {
+    if (s->ev_used == s->ev_pool.size()) {
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        s->ev_pool.push_back(e);
+    }
+    return s->ev_pool[s->ev_used++];
+}
+
+// Launch wrapper: records events around the launch when timing is on.
+template <class F>
+int launch(sv_state* s, LaunchClass cls, F&& f) {
+    cudaEvent_t a = nullptr, b = nullptr;
+    if (s->timing) {
+        a = next_event(s);
+        b = next_event(s);
+        cudaEventRecord(a, s->stream);
+    }
+    cudaError_t e = f();
+    if (e != cudaSuccess) return cuda_fail(s, e, "kernel launch");
+    if (s->timing) {
+        cudaEventRecord(b, s->stream);
+        s->recs.push_back({cls, a, b});
+    }
+    switch (cls) {
+        case LaunchClass::HIGH: s->stats.n_launch_high++; break;
+        case LaunchClass::LOW: s->stats.n_launch_low++; break;
+        default: s->stats.n_launch_other++; break;
+    }
+    return SV_OK;
+}
+
+void reset_stats(sv_state* s) {
+    s->stats = sv_stats{};
+    s->recs.clear();
+    s->ev_used = 0;
+}
+
+// Sum recorded event intervals into stats (requires the stream to be done).
+void collect_timing(sv_state* s) {
+    for (auto& r : s->recs) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, r.a, r.b) != cudaSuccess) continue;
+        const double sec = ms * 1e-3;
+        switch (r.cls) {
+            case LaunchClass::HIGH: s->stats.t_apply_high_dev_s += sec; break;
+            case LaunchClass::LOW: s->stats.t_apply_low_dev_s += sec; break;
+            case LaunchClass::EXCH: s->stats.t_exchange_dev_s += sec; break;
+            default: s->stats.t_other_dev_s += sec; break;
+        }
+    }
+    s->recs.clear();
+    s->ev_used = 0;
+}
+
+int sync(sv_state* s) {
+    CK(s, cudaStreamSynchronize(s->stream));
+    if (s->timing) collect_timing(s);
+    return SV_OK;
+}
+
+template <class T>
+int ensure(sv_state* s, T*& p, size_t& cap, size_t need) {
+    if (need <= cap) return SV_OK;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    cudaError_t e = cudaMalloc(&p, std::max<size_t>(need, 1) * sizeof(T));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    cap = need;
+    return SV_OK;
+}
+
+// ---- multi-process barrier ---------------------------------------------------
+int barrier(sv_state* s) {
+    if (s->virt || s->world == 1) return SV_OK;
+    if (!s->attached) return fail(SV_ECOMM, "sharded multi-process state used before sv_attach_peers");
+    ++s->epoch;
+    return launch(s, LaunchClass::OTHER,
+                  [&] { return launch_barrier(s->flags_dev, s->world, s->rank, s->epoch, s->stream); });
+}
+
+// ---- building launch descriptors -------------------------------------------
+void make_apply(int l, int k, const int* phys_in_order, const cd* M /* bit b <-> phys_in_order[b] */, ApplyDesc& d) {
+    std::vector<cd> Ms((size_t)1 << (2 * k));
+    int sq[SV_MAX_FUSED];
+    sort_matrix_qubits<cd>(k, phys_in_order, M, sq, Ms.data());
+    d.k = k;
+    for (int b = 0; b < k; ++b) d.q[b] = sq[b];
+    d.m.resize(Ms.size());
+    for (size_t i = 0; i < Ms.size(); ++i) d.m[i] = cf((float)Ms[i].real(), (float)Ms[i].imag());
+    plan_apply(l, d);
+}
+
+// PERMUTE (data at local bit b moves to bit perm[b]) as passes of disjoint
+// transpositions, <= 3 per pass (a 2t-qubit permutation matrix; exact).
+void lower_permute(int l, const std::vector<int>& perm, std::vector<ApplyDesc>& out) {
+    // current[b] = which original bit's data sits at bit b; target: bit perm[b] holds original b
+    std::vector<int> where(l);  // where[orig] = current position of orig's data
+    for (int b = 0; b < l; ++b) where[b] = b;
+    std::vector<std::pair<int, int>> swaps;
+    for (int b = 0; b < l; ++b) {
+        // want orig b's data at perm[b]
+        int cur = where[b];
+        int dst = perm[b];
+        if (cur == dst) continue;
+        // which orig currently sits at dst?
+        int other = -1;
+        for (int o = 0; o < l; ++o)
+            if (where[o] == dst) other = o;
+        swaps.push_back({cur, dst});
+        where[b] = dst;
+        where[other] = cur;
+    }
+    size_t i = 0;
+    while (i < swaps.size()) {
+        std::vector<std::pair<int, int>> pass;
+        uint64_t used = 0;
+        while (i < swaps.size() && pass.size() < 3) {
+            const auto sw = swaps[i];
+            const uint64_t m = (1ull << sw.first) | (1ull << sw.second);
+            if (used & m) break;  // keep order: a later swap touching these bits goes to the next pass
+            used |= m;
+            pass.push_back(sw);
+            ++i;
+        }
+        const int k = 2 * (int)pass.size();
+        int qs[SV_MAX_FUSED];
+        for (size_t t = 0; t < pass.size(); ++t) {
+            qs[2 * t] = pass[t].first;
+            qs[2 * t + 1] = pass[t].second;
+        }
+        // matrix over qs (bit 2t <-> first, 2t+1 <-> second): swaps bit pairs
+        const int D = 1 << k;
+        std::vector<cd> M((size_t)D * D, cd(0));
+        for (int c = 0; c < D; ++c) {
+            int r = c;
+            for (size_t t = 0; t < pass.size(); ++t) {
+                const int b0 = (c >> (2 * t)) & 1, b1 = (c >> (2 * t + 1)) & 1;
+                r &= ~(3 << (2 * t));
+                r |= (b1 << (2 * t)) | (b0 << (2 * t + 1));
+            }
+            M[(size_t)r * D + c] = 1.0;
+        }
+        ApplyDesc d;
+        make_apply(l, k, qs, M.data(), d);
+        out.push_back(std::move(d));
+    }
+}
+
+int run_apply(sv_state* s, const ApplyDesc& d) {
+    for (int sh = 0; sh < s->local_shards(); ++sh) {
+        float2* psi = s->virt ? s->shard[sh] : s->shard[s->rank];
+        int rc = launch(s, d.high ? LaunchClass::HIGH : LaunchClass::LOW,
+                        [&] { return launch_apply(psi, s->l, d, s->stream); });
+        if (rc) return rc;
+    }
+    const int k = d.k;
+    s->stats.bytes_apply += 16ull << s->l;
+    s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
+    return SV_OK;
+}
+
+int run_exchange(sv_state* s, const ExchangeDesc& x) {
+    int rc = barrier(s);
+    if (rc) return rc;
+    rc = launch(s, LaunchClass::EXCH,
+                [&] { return launch_exchange(s->shard_dev, s->world, s->virt ? -1 : s->rank, x, s->stream); });
+    if (rc) return rc;
+    s->stats.bytes_exchange += (uint64_t)((1.0 - 1.0 / (1 << x.s)) * 8.0 * (double)(1ull << s->l));
+    s->stats.n_exchanges++;
+    return barrier(s);
+}
+
+void apply_event_pairs(sv_state* s, const std::vector<std::pair<int, int>>& pairs) {
+    std::vector<int> inv(s->n);
+    for (int q = 0; q < s->n; ++q) inv[s->pos[q]] = q;
+    for (auto& pr : pairs) {
+        const int a = inv[pr.first], b = inv[pr.second];
+        s->pos[a] = pr.second;
+        s->pos[b] = pr.first;
+        inv[pr.first] = b;
+        inv[pr.second] = a;
+    }
+}
+
+ExchangeDesc make_exchange(int l, const std::vector<std::pair<int, int>>& pairs) {
+    ExchangeDesc x;
+    x.l = l;
+    x.s = (int)pairs.size();
+    for (int j = 0; j < x.s; ++j) {
+        x.P[j] = pairs[j].first;
+        x.p[j] = pairs[j].second;
+    }
+    return x;
+}
+
+// Bring the state to a canonical map (local part identity) -- needed before
+// sampling / whole-state reads in sharded mode.
+int canonicalize(sv_state* s) {
+    if (s->g == 0) return SV_OK;
+    std::vector<Event> ev;
+    std::vector<int> pos = s->pos;
+    plan_canonicalize(s->n, s->g, pos, ev);
+    for (auto& e : ev) {
+        if (e.type == Event::EXCHANGE) {
+            int rc = run_exchange(s, make_exchange(s->l, e.pairs));
+            if (rc) return rc;
+            apply_event_pairs(s, e.pairs);
+        } else if (e.type == Event::PERMUTE) {
+            std::vector<ApplyDesc> passes;
+            lower_permute(s->l, e.perm, passes);
+            for (auto& d : passes) {
+                int rc = run_apply(s, d);
+                if (rc) return rc;
+            }
+            for (int p = 0; p < s->l; ++p) s->pos[e.perm[p]] = e.perm[p];
+        }
+    }
+    return SV_OK;
+}
+
+// logical shard index of physical shard d
+int sigma_of(const sv_state* s, int d) {
+    int sg = 0;
+    for (int q = s->l; q < s->n; ++q) sg |= ((d >> (s->pos[q] - s->l)) & 1) << (q - s->l);
+    return sg;
+}
+
+uint64_t phys_of(const sv_state* s, uint64_t i) {
+    uint64_t p = 0;
+    for (int q = 0; q < s->n; ++q) p |= ((i >> q) & 1ull) << s->pos[q];
+    return p;
+}
+
+int alloc_scratch(sv_state* s) {
+    const uint64_t nb_local = (s->local_amps() + 31) >> 5;
+    const uint64_t nb = nb_local * s->local_shards();
+    cudaError_t e = cudaMalloc(&s->bins, nb * sizeof(uint64_t));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(bins) failed");
+    e = cudaMalloc(&s->scan_scratch, scan_scratch_elems(nb_local) * sizeof(uint64_t));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(scan scratch) failed");
+    e = cudaMalloc(&s->misc, 256 * sizeof(uint64_t));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(misc) failed");
+    e = cudaMalloc(&s->totals_ptr_dev, 64 * sizeof(uint64_t*));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
+    e = cudaMalloc(&s->sigma_dev, 64 * sizeof(int32_t));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
+    e = cudaMalloc(&s->kmat, 64 * 64 * sizeof(float2));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
+    return SV_OK;
+}
+
+void destroy_state(sv_state* s) {
+    if (!s) return;
+    if (s->stream) cudaStreamSynchronize(s->stream);
+    for (void* p : s->ipc_opened) cudaIpcCloseMemHandle(p);
+    if (s->alloc) cudaFree(s->alloc);
+    for (void* p : {(void*)s->shard_dev, (void*)s->bins, (void*)s->scan_scratch, (void*)s->misc,
+                    (void*)s->totals_ptr_dev, (void*)s->sigma_dev, (void*)s->kmat, (void*)s->ctrl, (void*)s->xfer,
+                    (void*)s->flags_dev, (void*)s->xfer_dev, (void*)s->idx_dev, (void*)s->amp_dev,
+                    (void*)s->samp_dev})
+        if (p) cudaFree(p);
+    for (auto e : s->ev_pool) cudaEventDestroy(e);
+    if (s->own_stream && s->stream) cudaStreamDestroy(s->stream);
+    delete s;
+}
+
+int upload_shard_table(sv_state* s) {
+    CK(s, cudaMemcpyAsync(s->shard_dev, s->shard.data(), sizeof(float2*) * s->world, cudaMemcpyHostToDevice,
+                          s->stream));
+    return SV_OK;
+}
+
+}  // namespace
+
+// =============================================================================
+extern "C" {
+
+const char* sv_last_error(void) { return g_err.c_str(); }
+const char* sv_version(void) { return "svb200 0.1 (sm_100a)"; }
+
+int sv_create(int n_qubits, sv_state** out) {
+    sv_config c{};
+    c.n_qubits = n_qubits;
+    c.world = 1;
+    c.exchange_vmin = -1;
+    c.device = -1;
+    return sv_create_ex(&c, out);
+}
+
+int sv_create_ex(const sv_config* cfg, sv_state** out) {
+    if (!cfg || !out) return fail(SV_EINVAL, "cfg/out is NULL");
+    *out = nullptr;
+    const int n = cfg->n_qubits;
+    if (n < 1 || n > SV_MAX_QUBITS) return fail(SV_EINVAL, "n_qubits out of range [1, 40]");
+    const int world = cfg->world <= 1 ? 1 : cfg->world;
+    if (world & (world - 1)) return fail(SV_EUNSUPPORTED, "world must be a power of two");
+    if (world > 64) return fail(SV_EUNSUPPORTED, "world > 64");
+    int g = 0;
+    while ((1 << g) < world) ++g;
+    const int l = n - g;
+    if (world > 1 && l < std::max(SV_MAX_FUSED, 2) + 2)
+        return fail(SV_EUNSUPPORTED, "shard too small: need n - log2(world) >= 8");
+    const bool virt = world == 1 || cfg->virtual_shards != 0;
+    if (!virt && (cfg->rank < 0 || cfg->rank >= world)) return fail(SV_EINVAL, "rank out of range");
+    const size_t shard_bytes = (size_t)8 << l;
+    const size_t need_bytes = shard_bytes * (virt ? world : 1);
+    if (cfg->dev_buf && cfg->buf_bytes < need_bytes) return fail(SV_EINVAL, "buf_bytes too small for the state");
+    if (cfg->dev_buf && !virt) return fail(SV_EUNSUPPORTED, "multi-process mode owns its buffers (dev_buf must be NULL)");
+
+    std::unique_ptr<sv_state, void (*)(sv_state*)> s(new sv_state(), destroy_state);
+    s->n = n;
+    s->g = g;
+    s->l = l;
+    s->world = world;
+    s->rank = virt ? 0 : cfg->rank;
+    s->virt = virt;
+    s->vmin = cfg->exchange_vmin < 0 ? 5 : cfg->exchange_vmin;
+    if (cfg->device >= 0) CK(nullptr, cudaSetDevice(cfg->device));
+    CK(nullptr, cudaGetDevice(&s->device));
+    if (cfg->cuda_stream) {
+        s->stream = (cudaStream_t)cfg->cuda_stream;
+    } else {
+        CK(nullptr, cudaStreamCreateWithFlags(&s->stream, cudaStreamNonBlocking));
+        s->own_stream = true;
+    }
+    char* base = nullptr;
+    if (cfg->dev_buf) {
+        base = (char*)cfg->dev_buf;
+    } else {
+        size_t free_b = 0, total_b = 0;
+        cudaMemGetInfo(&free_b, &total_b);
+        if (need_bytes + (need_bytes >> 5) + (64ull << 20) > free_b)
+            return fail(SV_ENOMEM, "state does not fit in free device memory");
+        cudaError_t e = cudaMalloc(&s->alloc, need_bytes);
+        if (e != cudaSuccess) return fail(SV_ENOMEM, std::string("cudaMalloc(state): ") + cudaGetErrorString(e));
+        base = (char*)s->alloc;
+    }
+    s->shard.assign(world, nullptr);
+    if (virt) {
+        for (int d = 0; d < world; ++d) s->shard[d] = (float2*)(base + shard_bytes * d);
+    } else {
+        s->shard[s->rank] = (float2*)base;
+        cudaError_t e = cudaMalloc(&s->ctrl, sizeof(Ctrl));
+        if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(ctrl)");
+        CK(nullptr, cudaMemset(s->ctrl, 0, sizeof(Ctrl)));
+        e = cudaMalloc(&s->xfer, kXferBytes);
+        if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(xfer)");
+        CK(nullptr, cudaMalloc(&s->flags_dev, sizeof(uint64_t*) * world));
+        CK(nullptr, cudaMalloc(&s->xfer_dev, sizeof(uint64_t*) * world));
+    }
+    CK(nullptr, cudaMalloc(&s->shard_dev, sizeof(float2*) * world));
+    int rc = alloc_scratch(s.get());
+    if (rc) return rc;
+    rc = upload_shard_table(s.get());
+    if (rc) return rc;
+    s->pos.resize(n);
+    for (int q = 0; q < n; ++q) s->pos[q] = q;
+    rc = sv_reset(s.get());
+    if (rc) return rc;
+    CK(nullptr, cudaStreamSynchronize(s->stream));
+    *out = s.release();
+    return SV_OK;
+}
+
+int sv_destroy(sv_state* s) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    destroy_state(s);
+    return SV_OK;
+}
+
+int sv_reset(sv_state* s) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    if (s->sticky) return fail(SV_EBADSTATE, "state poisoned by an earlier device failure");
+    for (int q = 0; q < s->n; ++q) s->pos[q] = q;
+    for (int d = 0; d < s->local_shards(); ++d) {
+        const int shard = s->virt ? d : s->rank;
+        float2* psi = s->shard[shard];
+        int rc = launch(s, LaunchClass::OTHER,
+                        [&] { return launch_reset(psi, s->local_amps(), shard == 0, s->stream); });
+        if (rc) return rc;
+    }
+    return SV_OK;
+}
+
+int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
+    if (!qubits || !matrix) return fail(SV_EINVAL, "qubits/matrix is NULL");
+    uint64_t mask = 0;
+    for (int b = 0; b < k; ++b) {
+        if (qubits[b] < 0 || qubits[b] >= s->n) return fail(SV_EINVAL, "qubit out of range");
+        if ((mask >> qubits[b]) & 1) return fail(SV_EINVAL, "duplicate qubit");
+        mask |= 1ull << qubits[b];
+    }
+    if (s->g > 0 && k > s->l - 1) return fail(SV_EUNSUPPORTED, "gate wider than a shard allows");
+    const int D = 1 << k;
+    std::vector<cd> M((size_t)D * D);
+    for (int i = 0; i < D * D; ++i) M[i] = cd(matrix[i].re, matrix[i].im);
+    std::vector<int> q(qubits, qubits + k);
+    // sharded: bring global qubits local (one S4 step for this gate alone)
+    if (s->g > 0) {
+        std::vector<std::vector<int>> fq(1, q);
+        std::vector<Event> ev;
+        std::vector<int> pos = s->pos;
+        plan_sharded(fq, s->n, s->g, s->vmin, ev, pos);
+        for (auto& e : ev)
+            if (e.type == Event::EXCHANGE) {
+                rc = run_exchange(s, make_exchange(s->l, e.pairs));
+                if (rc) return rc;
+                apply_event_pairs(s, e.pairs);
+            }
+    }
+    std::vector<int> phys(k);
+    for (int b = 0; b < k; ++b) phys[b] = s->pos[q[b]];
+    ApplyDesc d;
+    make_apply(s->l, k, phys.data(), M.data(), d);
+    if (k == 6) {
+        // matrix staged in device memory before return (stream-ordered)
+        CK(s, cudaMemcpyAsync(s->kmat, d.m.data(), 64 * 64 * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
+        CK(s, cudaStreamSynchronize(s->stream));
+        d.dev_m = s->kmat;
+    }
+    return run_apply(s, d);
+}
+
+int sv_fusion_plan(const sv_gate* gates, size_t n_gates, int max_fused, int32_t* buf, size_t cap, size_t* need) {
+    if (!need) return fail(SV_EINVAL, "need is NULL");
+    if (max_fused < 0 || max_fused > SV_MAX_FUSED) return fail(SV_EINVAL, "max_fused must be in [0, 6]");
+    int rc = validate_gates(gates, n_gates, -1);
+    if (rc) return rc;
+    std::vector<FusedGate> plan;
+    fuse_plan(gates, n_gates, max_fused, plan);
+    size_t len = 0;
+    for (auto& f : plan) len += 2 + f.k + f.mem.size();
+    *need = len;
+    if (cap < len) return fail(SV_EINVAL, "cap too small");
+    if (len && !buf) return fail(SV_EINVAL, "buf is NULL");
+    size_t o = 0;
+    for (auto& f : plan) {
+        buf[o++] = f.k;
+        for (int b = 0; b < f.k; ++b) buf[o++] = f.q[b];
+        buf[o++] = (int32_t)f.mem.size();
+        for (int32_t m : f.mem) buf[o++] = m;
+    }
+    return SV_OK;
+}
+
+int sv_fused_matrix(const sv_gate* gates, size_t n_gates, int max_fused, size_t index, sv_c128* out, size_t cap) {
+    if (max_fused < 0 || max_fused > SV_MAX_FUSED) return fail(SV_EINVAL, "max_fused must be in [0, 6]");
+    int rc = validate_gates(gates, n_gates, -1);
+    if (rc) return rc;
+    std::vector<FusedGate> plan;
+    fuse_plan(gates, n_gates, max_fused, plan);
+    if (index >= plan.size()) return fail(SV_EINVAL, "index out of range");
+    FusedGate& f = plan[index];
+    build_fused_matrix(gates, f);
+    if (!out || cap < f.M.size()) return fail(SV_EINVAL, "out too small");
+    for (size_t i = 0; i < f.M.size(); ++i) out[i] = sv_c128{f.M[i].real(), f.M[i].imag()};
+    return SV_OK;
+}
+
+static void write_events(const std::vector<Event>& ev, std::vector<int32_t>& o) {
+    for (auto& e : ev) {
+        if (e.type == Event::EXCHANGE) {
+            o.push_back(-1);
+            o.push_back((int32_t)e.pairs.size());
+            for (auto& pr : e.pairs) {
+                o.push_back(pr.first);
+                o.push_back(pr.second);
+            }
+        } else if (e.type == Event::APPLY) {
+            o.push_back(e.fused);
+            o.push_back(e.k);
+            for (int b = 0; b < e.k; ++b) o.push_back(e.phys[b]);
+        } else {
+            o.push_back(-2);
+            o.push_back((int32_t)e.perm.size());
+            for (int v : e.perm) o.push_back(v);
+        }
+    }
+}
+
+int sv_shard_plan(const int32_t* fs, size_t len, int n, int g, int vmin, int32_t* buf, size_t cap, size_t* need,
+                  int32_t* final_pos) {
+    if (!need) return fail(SV_EINVAL, "need is NULL");
+    if (n < 1 || n > SV_MAX_QUBITS || g < 0 || g >= n) return fail(SV_EINVAL, "bad n / log2_world");
+    if (len && !fs) return fail(SV_EINVAL, "fusion stream is NULL");
+    std::vector<std::vector<int>> fq;
+    size_t o = 0;
+    while (o < len) {
+        const int k = fs[o++];
+        if (k < 1 || k > SV_MAX_FUSED || o + k + 1 > len) return fail(SV_EINVAL, "malformed fusion stream");
+        std::vector<int> q(fs + o, fs + o + k);
+        for (int x : q)
+            if (x < 0 || x >= n) return fail(SV_EINVAL, "qubit out of range in fusion stream");
+        if (k > n - g) return fail(SV_EUNSUPPORTED, "fused gate wider than a shard");
+        o += k;
+        const int nm = fs[o++];
+        if (nm < 0 || o + nm > len) return fail(SV_EINVAL, "malformed fusion stream");
+        o += nm;
+        fq.push_back(q);
+    }
+    std::vector<Event> ev;
+    std::vector<int> pos;
+    plan_sharded(fq, n, g, vmin < 0 ? 5 : vmin, ev, pos);
+    std::vector<int32_t> outv;
+    write_events(ev, outv);
+    *need = outv.size();
+    if (cap < outv.size()) return fail(SV_EINVAL, "cap too small");
+    if (!outv.empty() && !buf) return fail(SV_EINVAL, "buf is NULL");
+    std::copy(outv.begin(), outv.end(), buf);
+    if (final_pos)
+        for (int q = 0; q < n; ++q) final_pos[q] = pos[q];
+    return SV_OK;
+}
+
+int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (!out) return fail(SV_EINVAL, "out is NULL");
+    if (max_fused < 0 || max_fused > SV_MAX_FUSED) return fail(SV_EINVAL, "max_fused must be in [0, 6]");
+    rc = validate_gates(gates, n_gates, s->n);
+    if (rc) return rc;
+    if (s->g > 0 && std::max(max_fused, 2) > s->l - 1) return fail(SV_EUNSUPPORTED, "fused gates wider than a shard allows");
+    std::unique_ptr<sv_circuit> c(new sv_circuit());
+    c->owner = s;
+    const double t0 = now_s();
+    std::vector<FusedGate> plan;
+    fuse_plan(gates, n_gates, max_fused, plan);
+    for (auto& f : plan) build_fused_matrix(gates, f);
+    const double t1 = now_s();
+    c->stats.t_fuse_s = t1 - t0;
+    c->stats.n_fused = (int)plan.size();
+    for (auto& f : plan) c->stats.fused_hist[f.k]++;
+    // plan (sharded) or trivial apply list
+    std::vector<Event> ev;
+    c->pos_in = s->pos;
+    std::vector<int> pos = s->pos;
+    if (s->g > 0) {
+        std::vector<std::vector<int>> fq;
+        for (auto& f : plan) fq.emplace_back(f.q, f.q + f.k);
+        plan_sharded(fq, s->n, s->g, s->vmin, ev, pos);
+        plan_canonicalize(s->n, s->g, pos, ev);
+    } else {
+        for (size_t i = 0; i < plan.size(); ++i) {
+            Event a;
+            a.type = Event::APPLY;
+            a.fused = (int)i;
+            a.k = plan[i].k;
+            for (int b = 0; b < a.k; ++b) a.phys[b] = plan[i].q[b];
+            ev.push_back(a);
+        }
+    }
+    c->pos_out = pos;
+    const double t2 = now_s();
+    c->stats.t_plan_s = t2 - t1;
+    // lower events to launch descriptors
+    size_t n6 = 0;
+    for (auto& e : ev) {
+        sv_circuit::Step st;
+        st.type = e.type;
+        if (e.type == Event::APPLY) {
+            make_apply(s->l, e.k, e.phys, plan[e.fused].M.data(), st.apply);
+            if (e.k == 6) ++n6;
+        } else if (e.type == Event::EXCHANGE) {
+            st.exch = make_exchange(s->l, e.pairs);
+            c->stats.n_exchanges++;
+        } else {
+            lower_permute(s->l, e.perm, st.perm_applies);
+        }
+        c->steps.push_back(std::move(st));
+    }
+    // one H2D upload of all k = 6 matrices (smaller ones travel as kernel params)
+    if (n6) {
+        cudaError_t e = cudaMalloc(&c->dev_mats, n6 * 64 * 64 * sizeof(float2));
+        if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(fused matrices)");
+        std::vector<float2> host(n6 * 64 * 64);
+        size_t i6 = 0;
+        for (auto& st : c->steps)
+            if (st.type == Event::APPLY && st.apply.k == 6) {
+                std::memcpy(&host[i6 * 4096], st.apply.m.data(), 4096 * sizeof(float2));
+                st.apply.dev_m = c->dev_mats + i6 * 4096;
+                ++i6;
+            }
+        CK(s, cudaMemcpyAsync(c->dev_mats, host.data(), host.size() * sizeof(float2), cudaMemcpyHostToDevice,
+                              s->stream));
+        CK(s, cudaStreamSynchronize(s->stream));
+    }
+    c->stats.t_upload_s = now_s() - t2;
+    *out = c.release();
+    return SV_OK;
+}
+
+int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (!c || c->owner != s) return fail(SV_EINVAL, "circuit is NULL or belongs to another state");
+    if (s->pos != c->pos_in) return fail(SV_EINVAL, "state qubit map differs from the circuit's (sv_reset first)");
+    const sv_stats keep = c->stats;
+    reset_stats(s);
+    s->stats.t_fuse_s = keep.t_fuse_s;
+    s->stats.t_plan_s = keep.t_plan_s;
+    s->stats.t_upload_s = keep.t_upload_s;
+    s->stats.n_fused = keep.n_fused;
+    for (int k = 0; k < 7; ++k) s->stats.fused_hist[k] = keep.fused_hist[k];
+    for (auto& st : c->steps) {
+        if (st.type == Event::APPLY) {
+            rc = run_apply(s, st.apply);
+        } else if (st.type == Event::EXCHANGE) {
+            rc = run_exchange(s, st.exch);
+        } else {
+            for (auto& d : st.perm_applies) {
+                rc = run_apply(s, d);
+                if (rc) break;
+            }
+        }
+        if (rc) return rc;
+    }
+    s->pos = c->pos_out;
+    return SV_OK;
+}
+
+int sv_circuit_stats(const sv_circuit* c, sv_stats* st) {
+    if (!c || !st) return fail(SV_EINVAL, "NULL argument");
+    *st = c->stats;
+    return SV_OK;
+}
+
+int sv_circuit_destroy(sv_circuit* c) {
+    if (!c) return fail(SV_EINVAL, "circuit is NULL");
+    if (c->dev_mats) {
+        if (c->owner && c->owner->stream) cudaStreamSynchronize(c->owner->stream);
+        cudaFree(c->dev_mats);
+    }
+    delete c;
+    return SV_OK;
+}
+
+int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_stats* stats) {
+    const double t0 = now_s();
+    sv_circuit* c = nullptr;
+    int rc = sv_circuit_create(s, gates, n_gates, max_fused, &c);
+    if (rc) return rc;
+    rc = sv_circuit_run_device(s, c);
+    if (rc == SV_OK) rc = sync(s);
+    sv_circuit_destroy(c);
+    if (rc) return rc;
+    s->stats.t_total_s = now_s() - t0;
+    if (stats) *stats = s->stats;
+    return SV_OK;
+}
+
+// ---- amplitudes ----------------------------------------------------------------
+int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count == 0) return SV_OK;
+    if (!idx || !out) return fail(SV_EINVAL, "idx/out is NULL");
+    const uint64_t dim = 1ull << s->n;
+    std::vector<uint64_t> loc(count);
+    std::vector<int32_t> own(count);
+    for (size_t i = 0; i < count; ++i) {
+        if (idx[i] >= dim) return fail(SV_EINVAL, "amplitude index out of range");
+        const uint64_t p = phys_of(s, idx[i]);
+        loc[i] = p & (s->local_amps() - 1);
+        own[i] = (int32_t)(p >> s->l);
+    }
+    const size_t chunk = s->virt ? count : std::min<size_t>(count, kXferBytes / 8);
+    for (size_t o = 0; o < count; o += chunk) {
+        const size_t cnt = std::min(chunk, count - o);
+        rc = ensure(s, s->idx_dev, s->idx_cap, 2 * cnt);
+        if (rc) return rc;
+        rc = ensure(s, s->amp_dev, s->amp_cap, cnt);
+        if (rc) return rc;
+        CK(s, cudaMemcpyAsync(s->idx_dev, loc.data() + o, cnt * 8, cudaMemcpyHostToDevice, s->stream));
+        int32_t* own_dev = reinterpret_cast<int32_t*>(s->idx_dev + cnt);
+        CK(s, cudaMemcpyAsync(own_dev, own.data() + o, cnt * 4, cudaMemcpyHostToDevice, s->stream));
+        if (s->virt) {
+            for (int d = 0; d < s->world; ++d) {
+                rc = launch(s, LaunchClass::OTHER, [&] {
+                    return launch_gather(s->shard[d], s->idx_dev, s->world > 1 ? own_dev : nullptr, d, cnt,
+                                         s->amp_dev, s->stream);
+                });
+                if (rc) return rc;
+            }
+        } else {
+            // owner writes into its xfer area; everyone merges (min over ~0-filled areas)
+            CK(s, cudaMemsetAsync(s->xfer, 0xff, cnt * 8, s->stream));
+            rc = launch(s, LaunchClass::OTHER, [&] {
+                return launch_gather(s->shard[s->rank], s->idx_dev, own_dev, s->rank, cnt,
+                                     reinterpret_cast<float2*>(s->xfer), s->stream);
+            });
+            if (rc) return rc;
+            rc = barrier(s);
+            if (rc) return rc;
+            rc = launch(s, LaunchClass::OTHER, [&] {
+                return launch_merge_min(s->xfer_dev, s->world, cnt, reinterpret_cast<uint64_t*>(s->amp_dev),
+                                        s->stream);
+            });
+            if (rc) return rc;
+            rc = barrier(s);
+            if (rc) return rc;
+        }
+        CK(s, cudaMemcpyAsync(out + o, s->amp_dev, cnt * 8, cudaMemcpyDeviceToHost, s->stream));
+        rc = sync(s);
+        if (rc) return rc;
+    }
+    return SV_OK;
+}
+
+// ---- sampling --------------------------------------------------------------------
+static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) {
+    int rc = canonicalize(s);
+    if (rc) return rc;
+    const uint64_t La = s->local_amps();
+    const uint64_t nb = (La + 31) >> 5;
+    const int nloc = s->local_shards();
+    // per local shard: bin weights + inclusive scan
+    for (int i = 0; i < nloc; ++i) {
+        const int d = s->virt ? i : s->rank;
+        uint64_t* bins = s->bins + (size_t)i * nb;
+        rc = launch(s, LaunchClass::OTHER, [&] { return launch_bin_weights(s->shard[d], La, bins, s->stream); });
+        if (rc) return rc;
+        rc = launch(s, LaunchClass::OTHER, [&] { return launch_inclusive_scan(bins, nb, s->scan_scratch, s->stream); });
+        if (rc) return rc;
+    }
+    // totals pointers (shard d's total = last element of its prefix) and sigma
+    std::vector<const uint64_t*> tp(s->world);
+    std::vector<int32_t> sig(s->world);
+    for (int d = 0; d < s->world; ++d) sig[d] = sigma_of(s, d);
+    if (s->virt) {
+        for (int d = 0; d < s->world; ++d) tp[d] = s->bins + (size_t)d * nb + (nb - 1);
+    } else {
+        CK(s, cudaMemcpyAsync(&s->ctrl->total, s->bins + (nb - 1), 8, cudaMemcpyDeviceToDevice, s->stream));
+        rc = barrier(s);
+        if (rc) return rc;
+        for (int d = 0; d < s->world; ++d) tp[d] = &s->peer_ctrl[d]->total;
+    }
+    CK(s, cudaMemcpyAsync(s->totals_ptr_dev, tp.data(), sizeof(void*) * s->world, cudaMemcpyHostToDevice, s->stream));
+    CK(s, cudaMemcpyAsync(s->sigma_dev, sig.data(), sizeof(int32_t) * s->world, cudaMemcpyHostToDevice, s->stream));
+    uint64_t* lo = s->misc;
+    uint64_t* total = s->misc + 64;
+    rc = launch(s, LaunchClass::OTHER, [&] {
+        return launch_shard_offsets(s->totals_ptr_dev, s->sigma_dev, s->world, lo, total, s->stream);
+    });
+    if (rc) return rc;
+    // check total weight on the host (argument validation of the result)
+    uint64_t T = 0;
+    CK(s, cudaMemcpyAsync(&T, total, 8, cudaMemcpyDeviceToHost, s->stream));
+    rc = sync(s);
+    if (rc) return rc;
+    if (T == 0) return fail(SV_EINVAL, "state has zero total weight");
+    if ((double)T >= 3.99 * 4611686018427387904.0) return fail(SV_EINVAL, "sum |c|^2 >= 3.99 (uint64 overflow risk)");
+    if (s->virt) {
+        for (int d = 0; d < s->world; ++d) {
+            const uint64_t base = (uint64_t)sig[d] << s->l;
+            rc = launch(s, LaunchClass::OTHER, [&] {
+                return launch_sample_resolve(s->shard[d], La, s->bins + (size_t)d * nb, nb, lo + d, total, seed, N,
+                                             base, dev_out, s->stream);
+            });
+            if (rc) return rc;
+        }
+    } else {
+        const size_t chunk = kXferBytes / 8;
+        for (size_t o = 0; o < N; o += chunk) {
+            const size_t cnt = std::min(chunk, N - o);
+            CK(s, cudaMemsetAsync(s->xfer, 0xff, cnt * 8, s->stream));
+            const uint64_t base = (uint64_t)sig[s->rank] << s->l;
+            // resolve samples o..o+cnt: shift the counter by o through the seed stream
+            rc = launch(s, LaunchClass::OTHER, [&] {
+                return launch_sample_resolve(s->shard[s->rank], La, s->bins, nb, lo + s->rank, total,
+                                             seed + (uint64_t)o * 0x9E3779B97F4A7C15ull, cnt, base, s->xfer, s->stream);
+            });
+            if (rc) return rc;
+            rc = barrier(s);
+            if (rc) return rc;
+            rc = launch(s, LaunchClass::OTHER,
+                        [&] { return launch_merge_min(s->xfer_dev, s->world, cnt, dev_out + o, s->stream); });
+            if (rc) return rc;
+            rc = barrier(s);
+            if (rc) return rc;
+        }
+    }
+    return SV_OK;
+}
+
+int sv_sample_device(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* dev_out) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (n_samples == 0) return SV_OK;
+    if (!dev_out) return fail(SV_EINVAL, "dev_out is NULL");
+    return sample_impl(s, seed, n_samples, dev_out);
+}
+
+int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (n_samples == 0) return SV_OK;
+    if (!out) return fail(SV_EINVAL, "out is NULL");
+    rc = ensure(s, s->samp_dev, s->samp_cap, n_samples);
+    if (rc) return rc;
+    rc = sample_impl(s, seed, n_samples, s->samp_dev);
+    if (rc) return rc;
+    CK(s, cudaMemcpyAsync(out, s->samp_dev, n_samples * 8, cudaMemcpyDeviceToHost, s->stream));
+    return sync(s);
+}
+
+// ---- whole state ------------------------------------------------------------------
+int sv_set_state(sv_state* s, const sv_c64* host, size_t count) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
+    for (int q = 0; q < s->n; ++q) s->pos[q] = q;
+    for (int i = 0; i < s->local_shards(); ++i) {
+        const int d = s->virt ? i : s->rank;
+        CK(s, cudaMemcpyAsync(s->shard[d], host + ((size_t)d << s->l), (size_t)8 << s->l, cudaMemcpyHostToDevice,
+                              s->stream));
+    }
+    rc = sync(s);
+    if (rc) return rc;
+    return barrier(s) ? fail(SV_ECOMM, "barrier failed") : sync(s);
+}
+
+int sv_get_state(sv_state* s, sv_c64* host, size_t count) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
+    rc = canonicalize(s);
+    if (rc) return rc;
+    rc = barrier(s);
+    if (rc) return rc;
+    rc = sync(s);
+    if (rc) return rc;
+    for (int d = 0; d < s->world; ++d) {
+        const int sg = sigma_of(s, d);
+        CK(s, cudaMemcpyAsync(host + ((size_t)sg << s->l), s->shard[d], (size_t)8 << s->l, cudaMemcpyDeviceToHost,
+                              s->stream));
+    }
+    rc = sync(s);
+    if (rc) return rc;
+    rc = barrier(s);
+    if (rc) return rc;
+    return sync(s);
+}
+
+int sv_device_ptr(sv_state* s, int shard, void** out) {
+    if (!s || !out) return fail(SV_EINVAL, "NULL argument");
+    if (shard < 0 || shard >= s->world || !s->shard[shard]) return fail(SV_EINVAL, "shard not available here");
+    *out = s->shard[shard];
+    return SV_OK;
+}
+
+int sv_qubit_map(const sv_state* s, int32_t* pos) {
+    if (!s || !pos) return fail(SV_EINVAL, "NULL argument");
+    for (int q = 0; q < s->n; ++q) pos[q] = s->pos[q];
+    return SV_OK;
+}
+
+// ---- multi-process plumbing -------------------------------------------------------
+struct IpcBlob {
+    int32_t magic, rank, world, l;
+    cudaIpcMemHandle_t state, ctrl, xfer;
+};
+
+int sv_ipc_handle(sv_state* s, void* out, size_t cap, size_t* need) {
+    if (!s || !need) return fail(SV_EINVAL, "NULL argument");
+    *need = sizeof(IpcBlob);
+    if (s->virt) return fail(SV_EINVAL, "not a multi-process sharded state");
+    if (cap < sizeof(IpcBlob) || !out) return fail(SV_EINVAL, "cap too small");
+    IpcBlob b{};
+    b.magic = 0x53564232;
+    b.rank = s->rank;
+    b.world = s->world;
+    b.l = s->l;
+    CK(s, cudaIpcGetMemHandle(&b.state, s->alloc));
+    CK(s, cudaIpcGetMemHandle(&b.ctrl, s->ctrl));
+    CK(s, cudaIpcGetMemHandle(&b.xfer, s->xfer));
+    std::memcpy(out, &b, sizeof(b));
+    return SV_OK;
+}
+
+int sv_attach_peers(sv_state* s, const void* handles, size_t each) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (s->virt) return fail(SV_EINVAL, "not a multi-process sharded state");
+    if (!handles || each < sizeof(IpcBlob)) return fail(SV_EINVAL, "bad handle blobs");
+    s->peer_ctrl.assign(s->world, nullptr);
+    s->peer_xfer.assign(s->world, nullptr);
+    for (int r = 0; r < s->world; ++r) {
+        IpcBlob b;
+        std::memcpy(&b, (const char*)handles + each * r, sizeof(b));
+        if (b.magic != 0x53564232 || b.rank != r || b.world != s->world || b.l != s->l)
+            return fail(SV_ECOMM, "peer handle blob mismatch");
+        if (r == s->rank) {
+            s->peer_ctrl[r] = s->ctrl;
+            s->peer_xfer[r] = s->xfer;
+            continue;
+        }
+        void* p = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&p, b.state, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) return fail(SV_ECOMM, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+        s->ipc_opened.push_back(p);
+        s->shard[r] = (float2*)p;
+        e = cudaIpcOpenMemHandle(&p, b.ctrl, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) return fail(SV_ECOMM, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+        s->ipc_opened.push_back(p);
+        s->peer_ctrl[r] = (Ctrl*)p;
+        e = cudaIpcOpenMemHandle(&p, b.xfer, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) return fail(SV_ECOMM, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+        s->ipc_opened.push_back(p);
+        s->peer_xfer[r] = (uint64_t*)p;
+    }
+    std::vector<uint64_t*> fl(s->world);
+    for (int r = 0; r < s->world; ++r) fl[r] = s->peer_ctrl[r]->flags;
+    CK(s, cudaMemcpy(s->flags_dev, fl.data(), sizeof(void*) * s->world, cudaMemcpyHostToDevice));
+    CK(s, cudaMemcpy(s->xfer_dev, s->peer_xfer.data(), sizeof(void*) * s->world, cudaMemcpyHostToDevice));
+    rc = upload_shard_table(s);
+    if (rc) return rc;
+    s->attached = true;
+    rc = barrier(s);
+    if (rc) return rc;
+    return sync(s);
+}
+
+int sv_set_timing(sv_state* s, int enable) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    s->timing = enable != 0;
+    return SV_OK;
+}
+
+int sv_last_stats(const sv_state* s_, sv_stats* out) {
+    sv_state* s = const_cast<sv_state*>(s_);
+    if (!s || !out) return fail(SV_EINVAL, "NULL argument");
+    if (s->timing && !s->recs.empty()) {
+        int rc = sync(s);
+        if (rc) return rc;
+    }
+    *out = s->stats;
+    return SV_OK;
+}
+
+int sv_synchronize(sv_state* s) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    return sync(s);
+}
+
+}  // extern "C"

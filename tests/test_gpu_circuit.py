@@ -1,0 +1,169 @@
+"""GPU parity of whole circuits (fuser + dispatcher + kernels), sampling,
+amplitudes and the virtual-shard exchange path, against the oracle.
+
+Tolerances are the north star's (BASELINE.json): fidelity
+|<psi_gpu|psi_ref>|^2 >= 1 - 1e-5 and max |psi_gpu - psi_ref| <=
+1e-5 * 2^(-n/2) * depth.  Sampling is bit-exact against oracle/sample.py on a
+seeded complex64 state (S5 is integer arithmetic).
+"""
+import numpy as np
+import pytest
+
+import paper_conf_sc_markidis23_b200 as sv
+from oracle import ref_c
+from oracle import sample as osample
+from oracle import sv as osv
+from workloads import rqc as W
+
+pytestmark = pytest.mark.gpu
+
+
+def _run(n, gates, F, world=1):
+    h = sv.sv_create_ex(n, world=world, virtual_shards=True) if world > 1 else sv.sv_create(n)
+    try:
+        st = sv.sv_run_circuit(h, gates, F)
+        return sv.sv_get_state(h, n), st
+    finally:
+        sv.sv_destroy(h)
+
+
+def _check(n, depth, got, ref):
+    got = got.astype(np.complex128)
+    fid = osv.fidelity(got, ref)
+    err = np.abs(got - ref).max()
+    assert fid >= 1 - 1e-5, fid
+    assert err <= osv.max_abs_bound(n, depth), (err, osv.max_abs_bound(n, depth))
+
+
+@pytest.mark.parametrize("F", range(7))
+def test_rqc12_all_fusion_sizes(F):
+    gates = W.rqc(12, 14)
+    got, st = _run(12, gates, F)
+    _check(12, 14, got, osv.simulate(12, gates))
+    assert st["n_fused"] == [121, 85, 34, 19, 15, 11, 8][F]
+
+
+@pytest.mark.parametrize("n,d,F", [(16, 14, 2), (20, 14, 4), (22, 16, 3), (24, 14, 5), (25, 14, 6), (26, 14, 4)])
+def test_rqc_medium(n, d, F):
+    gates = W.rqc(n, d, seed=n)
+    got, _ = _run(n, gates, F)
+    _check(n, d, got, ref_c.run(n, gates))
+
+
+def test_random_circuit_unsorted_two_qubit_gates():
+    n = 18
+    gates = W.random_circuit(n, 150, 9, two_qubit_frac=0.5)
+    ref = ref_c.run(n, gates)
+    for F in (0, 2, 4, 6):
+        got, _ = _run(n, gates, F)
+        _check(n, 10, got, ref)
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+@pytest.mark.parametrize("F", [2, 4])
+def test_virtual_shards_match_oracle(world, F):
+    n = 16
+    gates = W.rqc(n, 14, seed=world)
+    got, st = _run(n, gates, F, world=world)
+    _check(n, 14, got, ref_c.run(n, gates))
+    assert st["n_exchanges"] >= 1
+
+
+def test_amplitudes_match_state():
+    n = 20
+    gates = W.rqc(n, 12)
+    h = sv.sv_create(n)
+    try:
+        sv.sv_run_circuit(h, gates, 4)
+        full = sv.sv_get_state(h, n)
+        idx = np.random.default_rng(0).integers(0, 1 << n, size=1000).astype(np.uint64)
+        assert np.array_equal(sv.sv_amplitudes(h, idx), full[idx.astype(np.int64)])
+        with pytest.raises(sv.SVError):
+            sv.sv_amplitudes(h, np.array([1 << n], dtype=np.uint64))
+    finally:
+        sv.sv_destroy(h)
+
+
+@pytest.mark.parametrize("n", [2, 3, 5, 6, 11, 20])
+def test_sampler_bit_exact(n):
+    psi = W.random_state_c64(n, 50 + n)
+    ref, _ = osample.sample(psi, 1234, 5000)
+    h = sv.sv_create(n)
+    try:
+        sv.sv_set_state(h, psi)
+        got = sv.sv_sample(h, 1234, 5000)
+    finally:
+        sv.sv_destroy(h)
+    assert np.array_equal(got, ref)
+
+
+def test_sampler_rqc12_appendix_c_state():
+    """Sample the oracle's fp64 RQC-12 state rounded to complex64 (S5 vectors)."""
+    psi = osv.simulate(12, W.rqc(12, 14)).astype(np.complex64)
+    h = sv.sv_create(12)
+    try:
+        sv.sv_set_state(h, psi)
+        got = sv.sv_sample(h, 1, 8)
+    finally:
+        sv.sv_destroy(h)
+    assert [int(x) for x in got] == [2318, 3050, 3966, 1826, 1826, 3132, 3597, 2133]
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_sampler_sharded_bit_exact(world):
+    n = 14
+    psi = W.random_state_c64(n, 77)
+    ref, _ = osample.sample(psi, 99, 3000)
+    h = sv.sv_create_ex(n, world=world, virtual_shards=True)
+    try:
+        sv.sv_set_state(h, psi)
+        got = sv.sv_sample(h, 99, 3000)
+    finally:
+        sv.sv_destroy(h)
+    assert np.array_equal(got, ref)
+
+
+def test_sampler_after_sharded_circuit_statistics():
+    n, d = 14, 12
+    gates = W.rqc(n, d)
+    p = osample.exact_probabilities(ref_c.run(n, gates))
+    h = sv.sv_create_ex(n, world=4, virtual_shards=True)
+    try:
+        sv.sv_run_circuit(h, gates, 4)
+        s = sv.sv_sample(h, 5, 200000)
+    finally:
+        sv.sv_destroy(h)
+    cnt = np.bincount(s.astype(np.int64), minlength=1 << n)
+    # chi-square on the 64 coarse bins of the top 6 bits
+    P = p.reshape(64, -1).sum(1)
+    C = cnt.reshape(64, -1).sum(1)
+    chi2 = float(np.sum((C - s.size * P) ** 2 / (s.size * P)))
+    assert chi2 < 63 + 6 * np.sqrt(2 * 63)
+
+
+def test_sampler_rejects_zero_state():
+    h = sv.sv_create(6)
+    try:
+        sv.sv_set_state(h, np.zeros(64, np.complex64))
+        with pytest.raises(sv.SVError) as e:
+            sv.sv_sample(h, 1, 10)
+        assert e.value.code == sv.SV_EINVAL
+    finally:
+        sv.sv_destroy(h)
+
+
+def test_prepared_circuit_and_reset():
+    n = 18
+    gates = W.rqc(n, 14)
+    ref = ref_c.run(n, gates)
+    h = sv.sv_create(n)
+    try:
+        c = sv.sv_circuit_create(h, gates, 4)
+        for _ in range(2):
+            sv.sv_reset(h)
+            sv.sv_circuit_run_device(h, c)
+            sv.sv_synchronize(h)
+            _check(n, 14, sv.sv_get_state(h, n), ref)
+        sv.sv_circuit_destroy(c)
+    finally:
+        sv.sv_destroy(h)

@@ -1,0 +1,112 @@
+"""CPU-only checks of the C-ABI library (no GPU needed):
+
+* libsvb200.so loads and exports every function include/sv.h declares;
+* the host fuser (sv_fusion_plan) reproduces the oracle's S3 plan bit for bit
+  and its fp64 fused matrices (sv_fused_matrix) within 1e-12;
+* the host planner (sv_shard_plan) reproduces the oracle's S4 events bit for
+  bit;
+* argument validation returns the documented error codes before any device
+  work.
+"""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_sc_markidis23_b200 as sv
+from oracle import fuse as ofuse
+from oracle import plan as oplan
+from workloads import rqc as W
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    from paper_conf_sc_markidis23_b200.build import build
+    build()
+
+
+def test_exports_match_header():
+    hdr = open(os.path.join(ROOT, "include", "sv.h")).read()
+    declared = set(re.findall(r"^(?:int|const char\*)\s+(sv_\w+)\s*\(", hdr, flags=re.M))
+    assert declared, "no declarations parsed"
+    L = sv.lib()
+    for name in declared:
+        assert hasattr(L, name), name
+    assert declared == set(sv.EXPORTED)
+    assert sv.sv_version().startswith("svb200")
+
+
+def _circuits():
+    yield "rqc12", W.rqc(12, 14)
+    yield "rqc30", W.rqc(30, 14)
+    yield "rqc36", W.rqc(36, 20)
+    yield "rand", W.random_circuit(11, 200, 5, two_qubit_frac=0.4)
+
+
+@pytest.mark.parametrize("F", range(7))
+def test_fusion_plan_bit_exact(F):
+    for name, gates in _circuits():
+        got = sv.sv_fusion_plan(gates, F)
+        ref = ofuse.plan_stream(ofuse.fuse_plan([g.qubits for g in gates], F))
+        assert np.array_equal(got, ref), (name, F)
+
+
+@pytest.mark.parametrize("F", [1, 2, 4, 6])
+def test_fused_matrices_fp64(F):
+    gates = W.random_circuit(9, 60, 100 + F, two_qubit_frac=0.4)
+    plan = ofuse.fuse(gates, F)
+    for i, (Q, mem, M) in enumerate(plan):
+        got = sv.sv_fused_matrix(gates, F, i, len(Q))
+        assert np.abs(got - M).max() < 1e-12
+        # rounding to complex64 agrees to within one ulp
+        a, b = got.astype(np.complex64), M.astype(np.complex64)
+        assert np.all(np.abs(a - b) <= np.spacing(np.maximum(np.abs(a.real), np.abs(a.imag))).max() + 0)
+
+
+@pytest.mark.parametrize("n,d,g,F,vmin", [(12, 14, 1, 4, 5), (20, 14, 2, 4, 5), (30, 14, 3, 2, 5),
+                                           (34, 20, 1, 4, 5), (34, 20, 2, 4, 5), (36, 20, 3, 4, 5),
+                                           (36, 20, 2, 6, 5), (16, 14, 3, 3, 0), (14, 14, 2, 5, 2)])
+def test_shard_plan_bit_exact(n, d, g, F, vmin):
+    gates = W.rqc(n, d)
+    fs = sv.sv_fusion_plan(gates, F)
+    fq = [Q for Q, _ in ofuse.fuse_plan([x.qubits for x in gates], F)]
+    ev, pos = oplan.plan_sharded(fq, n, g, vmin)
+    got, gpos = sv.sv_shard_plan(fs, n, g, vmin)
+    assert np.array_equal(got, oplan.plan_stream(ev))
+    assert list(gpos) == list(pos)
+
+
+def test_error_codes():
+    gates = W.rqc(12, 14)
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_fusion_plan(gates, 7)
+    assert e.value.code == sv.SV_EINVAL
+    bad = sv.as_gates(gates[:3])
+    bad["nq"][1] = 3
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_fusion_plan(bad, 2)
+    assert e.value.code == sv.SV_EINVAL
+    bad = sv.as_gates(gates[12:14])
+    bad["q"][0] = [5, 5]
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_fusion_plan(bad, 2)
+    assert e.value.code == sv.SV_EINVAL
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_shard_plan(np.array([2, 0, 40, 1, 0], np.int32), 12, 1)
+    assert e.value.code == sv.SV_EINVAL
+    # sv_create validates n before touching the device
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_create(0)
+    assert e.value.code == sv.SV_EINVAL
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_create_ex(20, world=3)
+    assert e.value.code == sv.SV_EUNSUPPORTED
+
+
+def test_gate_struct_layout():
+    g = sv.as_gates([W.Gate(0, "cz", (3, 1), W.GATE_CZ)])
+    assert g.itemsize == 272 and g["nq"][0] == 2 and list(g["q"][0]) == [3, 1]
+    assert g["m"][0][15] == -1 and g["m"][0][0] == 1
