@@ -89,6 +89,7 @@ def run(n: int, gates, psi: np.ndarray | None = None) -> np.ndarray:
 def time_gates(n: int, gates, max_seconds: float = 20.0):
     """Bounded timing sample for the CPU baseline: apply gates in order on a
     fresh 2^n state until max_seconds elapse.  Returns (gates_done, seconds)."""
+    from workloads.rqc import gate_arrays
     psi = zero_state(n)
     nq, qq, mat = gate_arrays(gates)
     L = lib()

@@ -20,7 +20,8 @@ from typing import Sequence
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libsvb200.so")
+# SVB200_LIB selects an alternative in-tree build (A/B kernel variants)
+LIB_PATH = os.environ.get("SVB200_LIB") or os.path.join(HERE, "libsvb200.so")
 
 SV_OK = 0
 SV_EINVAL = -1

@@ -42,6 +42,24 @@ def _compile(src: str, verbose: bool) -> str:
     return obj
 
 
+def build_variant(name: str, defines) -> str:
+    """Build an A/B variant library (extra -D flags) next to the main one."""
+    out = os.path.join(HERE, "_variants", f"libsvb200_{name}.so")
+    bdir = os.path.join(HERE, "_variants", name)
+    os.makedirs(bdir, exist_ok=True)
+    extra = [f"-D{d}" for d in defines]
+
+    def comp(src):
+        obj = os.path.join(bdir, src + ".o")
+        subprocess.check_call([NVCC] + ARCH + COMMON + extra + ["-c", os.path.join(CSRC, src), "-o", obj])
+        return obj
+
+    with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
+        objs = list(ex.map(comp, SOURCES))
+    subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", out] + objs + ["-Xcompiler", "-fPIC"])
+    return out
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest_input():
         return LIB
@@ -58,5 +76,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="--verbose" in sys.argv)
-    print(LIB)
+    if len(sys.argv) > 2 and sys.argv[1] == "--variant":
+        print(build_variant(sys.argv[2], sys.argv[3:]))
+    else:
+        build(force="--force" in sys.argv, verbose="--verbose" in sys.argv)
+        print(LIB)

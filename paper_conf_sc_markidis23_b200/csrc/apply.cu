@@ -35,7 +35,6 @@ namespace svb {
 
 namespace {
 
-constexpr int kThreads = 256;
 
 __device__ __forceinline__ uint64_t insert_zeros(uint64_t x, const int* pos, int npos) {
 #pragma unroll
@@ -81,49 +80,58 @@ __device__ __forceinline__ void cmac(float2& y, const float2 m, const float2 a) 
     y.y = fmaf(m.y, a.x, y.y);
 }
 
+// Fused matrix as three real planes for the 3-multiplication complex product
+// (Gauss): with m = p + iq and a = x + iy,
+//   A = sum_c p_c (x_c + y_c),  B = sum_c (p_c + q_c) y_c,  C = sum_c (q_c - p_c) x_c,
+//   Re y = A - B,  Im y = A + C.
+// 3 FMAs per complex multiply-add instead of 4 (k <= 5, planes in the kernel
+// parameters).  k = 6 keeps the plain 4-FMA form with the matrix in shared
+// memory (3 planes of 64 x 64 would not fit next to the tile).
 template <int K>
 struct MatStore {
-    float2 m[1 << K][1 << K];
+    alignas(16) float P[1 << K][1 << K];
+    alignas(16) float S[1 << K][1 << K];
+    alignas(16) float Q[1 << K][1 << K];
 };
 template <>
-struct MatStore<6> {  // 32 KB: does not fit the 32764 B parameter space
+struct MatStore<6> {  // 32 KB complex: does not fit the 32764 B parameter space
     const float2* dev;
 };
 
-template <int K>
-__device__ __forceinline__ float2 mat_elem(const MatStore<K>& M, const float2* sm, int r, int c) {
-    return M.m[r][c];
-}
-template <>
-__device__ __forceinline__ float2 mat_elem<6>(const MatStore<6>&, const float2* sm, int r, int c) {
-    return sm[r * 64 + c];
-}
-
-// Rows unrolled fully for k <= 4 (matrix from the constant bank as FFMA
-// operands); k = 5/6 loop over rows to bound code size.
-template <int K>
-struct RowUnroll {
-    static constexpr int value = (K <= 4) ? (1 << K) : 1;
-    static constexpr int half = (K <= 4) ? (1 << (K - 1)) : 1;
-};
+#ifndef SV_ROWS
+#define SV_ROWS 1  // output rows per (non-unrolled) row-loop iteration
+#endif
 
 // ------------------------------------------------------------------ kernels
-// One tile per CTA iteration: the 2^nH runs of 2^r contiguous amplitudes that
-// share every bit outside {0..r-1} u H (H = gate qubits >= r).  The tile holds
-// complete groups, so the gate is applied entirely inside shared memory.
+// A tile is the set of 2^nH runs of 2^r contiguous amplitudes that share
+// every bit outside {0..r-1} u H (H = gate qubits >= r); it holds complete
+// groups, so the gate is applied entirely inside shared memory.  Tile index
+// t (0 <= t < 2^T) maps to the global offset dep(t) = (t mod 2^r) + deposit of
+// (t >> r) into H, and to the swizzled shared-memory slot phys(t); both maps
+// are additive/XOR-linear over disjoint bits, so per-unit offsets are
+// precomputed on the host and a thread adds/XORs them to its own base.
 template <int K>
-struct TileParams {
+struct alignas(16) TileParams {
+    MatStore<K> M;                     // first: 16 B aligned in the constant bank (LDCU.128)
     float2* psi;
     uint64_t n_tiles;
     int T, r;                          // tile bits, run bits
     int nH;
     int Hpos[SV_MAX_FUSED];            // gate qubits >= r (ascending, global positions)
-    uint64_t offH[1 << SV_MAX_FUSED];  // amplitude offset of run h (deposit of h into Hpos)
     int nzt;
     int ztpos[SV_MAX_FUSED];           // tile-local gate bit positions, ascending
     uint32_t swz[3];                   // phys bit (i+1) ^= parity(t & swz[i])
-    uint32_t loc[1 << K];              // swizzled tile offsets of the gathers
-    MatStore<K> M;
+    int upt;                           // 16-byte units per thread per tile
+    int iters;                         // compute iterations per thread per tile
+    uint64_t goff[64];                 // dep(2 * nthreads * i)
+    uint32_t soff[64];                 // phys(2 * nthreads * i)
+    uint32_t loc[1 << K];              // phys offsets of the gathers (members / member pairs)
+    uint32_t gsec;                     // phys offset of the second group of a pair (PAIR, 2 groups)
+    // monomial matrices (one nonzero per row: permutations, diagonals, identity)
+    int mono;
+    uint32_t mloc[1 << K];             // phys offset of member r (output slot of row r)
+    uint32_t ploc[1 << K];             // phys offset of the source member of row r
+    float2 mdiag[1 << K];              // the nonzero of row r
 };
 
 __device__ __forceinline__ uint32_t swizzle(uint32_t t, const uint32_t* swz) {
@@ -135,117 +143,341 @@ __device__ __forceinline__ void cp_async16(uint32_t saddr, const void* g) {
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
-constexpr int kStages = 2;
-
-// Issue the asynchronous global->shared copies of tile u (16 B per lane,
-// swizzled destination; consecutive lanes read consecutive 16 B of a run).
-template <int K>
-__device__ __forceinline__ void tile_load(const TileParams<K>& p, uint64_t u, uint32_t sbuf) {
-    const uint64_t tbase = insert_zeros(u << p.r, p.Hpos, p.nH);
-    const uint32_t units = 1u << (p.T - 1);
-    const uint32_t rmask = (1u << p.r) - 1u;
-    for (uint32_t v = threadIdx.x; v < units; v += blockDim.x) {
-        const uint32_t t = v << 1;
-        const uint64_t g = tbase + p.offH[t >> p.r] + (t & rmask);
-        cp_async16(sbuf + (swizzle(t, p.swz) << 3), p.psi + g);
-    }
-}
-
-template <int K>
-__device__ __forceinline__ void tile_store(const TileParams<K>& p, uint64_t u, uint32_t sbuf) {
-    const uint64_t tbase = insert_zeros(u << p.r, p.Hpos, p.nH);
-    const uint32_t units = 1u << (p.T - 1);
-    const uint32_t rmask = (1u << p.r) - 1u;
-    for (uint32_t v = threadIdx.x; v < units; v += blockDim.x) {
-        const uint32_t t = v << 1;
-        const uint64_t g = tbase + p.offH[t >> p.r] + (t & rmask);
-        st_stream(reinterpret_cast<float4*>(p.psi + g), lds4(sbuf + (swizzle(t, p.swz) << 3)));
-    }
-}
-
-// y = M a for every group of the tile, in place in shared memory.
-// PAIR: qubit 0 is a gate qubit -> 16 B gathers hold members 2j, 2j+1.
-template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* sm) {
+// Gauss form of output rows [r0, r0 + R) for one group (s[c] = x_c + y_c).
+// The row loop of the callers is NOT unrolled: each iteration is a scheduling
+// fence, so ptxas cannot interleave all rows (which needs 6 accumulators per
+// row live at once and spills at k >= 4).  Matrix operands are warp-uniform
+// constant-bank loads (LDCU) feeding FFMA uniform-register operands.
+template <int K, int R>
+__device__ __forceinline__ void gauss_block(const MatStore<K>& M, int r0, const float2* a, const float* s, float2* y) {
     constexpr int D = 1 << K;
-    const uint32_t ngroups = 1u << (p.T - K);
-    for (uint32_t gidx = threadIdx.x; gidx < ngroups; gidx += blockDim.x) {
-        const uint32_t bt = (uint32_t)insert_zeros(gidx, p.ztpos, p.nzt);
-        const uint32_t pb = swizzle(bt, p.swz);
-        if constexpr (PAIR) {
-            float4 v[D / 2];
 #pragma unroll
-            for (int j = 0; j < D / 2; ++j) v[j] = lds4(sbuf + ((pb ^ p.loc[j]) << 3));
-#pragma unroll RowUnroll<K>::half
-            for (int r2 = 0; r2 < D / 2; ++r2) {
-                float2 y0 = make_float2(0.f, 0.f), y1 = make_float2(0.f, 0.f);
+    for (int i = 0; i < R; ++i) {
+        float A = 0.f, B = 0.f, C = 0.f;
 #pragma unroll
-                for (int c = 0; c < D; ++c) {
-                    const float2 a = (c & 1) ? make_float2(v[c >> 1].z, v[c >> 1].w)
-                                             : make_float2(v[c >> 1].x, v[c >> 1].y);
-                    cmac(y0, mat_elem<K>(p.M, sm, 2 * r2, c), a);
-                    cmac(y1, mat_elem<K>(p.M, sm, 2 * r2 + 1, c), a);
-                }
-                sts4(sbuf + ((pb ^ p.loc[r2]) << 3), make_float4(y0.x, y0.y, y1.x, y1.y));
+        for (int c = 0; c < D; ++c) {
+            A = fmaf(M.P[r0 + i][c], s[c], A);
+            B = fmaf(M.S[r0 + i][c], a[c].y, B);
+            C = fmaf(M.Q[r0 + i][c], a[c].x, C);
+        }
+        y[i] = make_float2(A - B, A + C);
+    }
+}
+
+template <int K, int R>
+__device__ __forceinline__ void gauss_block2(const MatStore<K>& M, int r0, const float2* a0, const float* s0,
+                                             const float2* a1, const float* s1, float2* y0, float2* y1) {
+    constexpr int D = 1 << K;
+#pragma unroll
+    for (int i = 0; i < R; ++i) {
+        float A0 = 0.f, B0 = 0.f, C0 = 0.f, A1 = 0.f, B1 = 0.f, C1 = 0.f;
+#pragma unroll
+        for (int c = 0; c < D; ++c) {
+            const float p = M.P[r0 + i][c], sq = M.S[r0 + i][c], q = M.Q[r0 + i][c];
+            A0 = fmaf(p, s0[c], A0);
+            A1 = fmaf(p, s1[c], A1);
+            B0 = fmaf(sq, a0[c].y, B0);
+            B1 = fmaf(sq, a1[c].y, B1);
+            C0 = fmaf(q, a0[c].x, C0);
+            C1 = fmaf(q, a1[c].x, C1);
+        }
+        y0[i] = make_float2(A0 - B0, A0 + C0);
+        y1[i] = make_float2(A1 - B1, A1 + C1);
+    }
+}
+
+// One group, rows one by one (small-state fallback).
+template <int K, class Emit>
+__device__ __forceinline__ void gauss_rows(const MatStore<K>& M, const float2* a, Emit&& emit) {
+    constexpr int D = 1 << K;
+    float s[D];
+#pragma unroll
+    for (int c = 0; c < D; ++c) s[c] = a[c].x + a[c].y;
+#pragma unroll 1
+    for (int r = 0; r < D; ++r) {
+        float2 y;
+        gauss_block<K, 1>(M, r, a, s, &y);
+        emit(r, y);
+    }
+}
+
+// GPT (groups per thread) = 2 for k <= 4, else 1.  PAIR: tile bit 0 is a gate
+// bit, so a 16 B shared-memory word holds members 2j, 2j+1 of one group;
+// otherwise (GPT = 2) it holds the same member of two neighbouring groups.
+// y_r = m_r * a_{perm(r)}: exact for entries in {+-1, +-i} (identity,
+// permutation and CZ-like matrices).  All sources are read before any output
+// is written (in place).
+__device__ __forceinline__ float2 cmul(float2 m, float2 a) {
+    return make_float2(fmaf(m.x, a.x, -(m.y * a.y)), fmaf(m.x, a.y, m.y * a.x));
+}
+
+template <int K, bool PAIR>
+__device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32_t sbuf) {
+    constexpr int D = 1 << K;
+    constexpr int GPT = (K <= 4) ? 2 : 1;
+    for (int j = 0; j < p.iters; ++j) {
+        const uint32_t gidx = threadIdx.x + (uint32_t)j * blockDim.x;
+        if constexpr (GPT == 2 && !PAIR) {
+            const uint32_t pb = swizzle((uint32_t)insert_zeros((uint64_t)gidx << 1, p.ztpos, p.nzt), p.swz);
+            float4 v[D];
+#pragma unroll
+            for (int r = 0; r < D; ++r) v[r] = lds4(sbuf + ((pb ^ p.ploc[r]) << 3));
+#pragma unroll
+            for (int r = 0; r < D; ++r) {
+                const float2 y0 = cmul(p.mdiag[r], make_float2(v[r].x, v[r].y));
+                const float2 y1 = cmul(p.mdiag[r], make_float2(v[r].z, v[r].w));
+                sts4(sbuf + ((pb ^ p.mloc[r]) << 3), make_float4(y0.x, y0.y, y1.x, y1.y));
             }
         } else {
-            float2 v[D];
+            const uint32_t pb = (GPT == 2) ? swizzle((uint32_t)insert_zeros((uint64_t)gidx << 1, p.ztpos, p.nzt), p.swz)
+                                           : swizzle((uint32_t)insert_zeros(gidx, p.ztpos, p.nzt), p.swz);
 #pragma unroll
-            for (int j = 0; j < D; ++j) v[j] = lds2(sbuf + ((pb ^ p.loc[j]) << 3));
-#pragma unroll RowUnroll<K>::value
-            for (int r = 0; r < D; ++r) {
-                float2 y = make_float2(0.f, 0.f);
+            for (int gg = 0; gg < GPT; ++gg) {
+                const uint32_t b = gg ? (pb ^ p.gsec) : pb;
+                float2 v[D];
 #pragma unroll
-                for (int c = 0; c < D; ++c) cmac(y, mat_elem<K>(p.M, sm, r, c), v[c]);
-                sts2(sbuf + ((pb ^ p.loc[r]) << 3), y);
+                for (int r = 0; r < D; ++r) v[r] = lds2(sbuf + ((b ^ p.ploc[r]) << 3));
+#pragma unroll
+                for (int r = 0; r < D; ++r) sts2(sbuf + ((b ^ p.mloc[r]) << 3), cmul(p.mdiag[r], v[r]));
             }
         }
     }
 }
 
-// Persistent, double-buffered: the copies of tile i+1 are in flight while
-// tile i is transformed and written back.
 template <int K, bool PAIR>
+__device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* smat) {
+    constexpr int D = 1 << K;
+    constexpr int GPT = (K <= 4) ? 2 : 1;
+    for (int j = 0; j < p.iters; ++j) {
+        const uint32_t gidx = threadIdx.x + (uint32_t)j * blockDim.x;
+        if constexpr (GPT == 2) {
+            const uint32_t pb = swizzle((uint32_t)insert_zeros((uint64_t)gidx << 1, p.ztpos, p.nzt), p.swz);
+            float2 a0[D], a1[D];
+            float s0[D], s1[D];
+            if constexpr (PAIR) {
+#pragma unroll
+                for (int jj = 0; jj < D / 2; ++jj) {
+                    const float4 v0 = lds4(sbuf + ((pb ^ p.loc[jj]) << 3));
+                    const float4 v1 = lds4(sbuf + ((pb ^ p.gsec ^ p.loc[jj]) << 3));
+                    a0[2 * jj] = make_float2(v0.x, v0.y);
+                    a0[2 * jj + 1] = make_float2(v0.z, v0.w);
+                    a1[2 * jj] = make_float2(v1.x, v1.y);
+                    a1[2 * jj + 1] = make_float2(v1.z, v1.w);
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < D; ++c) {
+                    const float4 v = lds4(sbuf + ((pb ^ p.loc[c]) << 3));
+                    a0[c] = make_float2(v.x, v.y);
+                    a1[c] = make_float2(v.z, v.w);
+                }
+            }
+#pragma unroll
+            for (int c = 0; c < D; ++c) {
+                s0[c] = a0[c].x + a0[c].y;
+                s1[c] = a1[c].x + a1[c].y;
+            }
+            if constexpr (PAIR) {
+#pragma unroll 1
+                for (int r2 = 0; r2 < D / 2; ++r2) {
+                    float2 y0[2], y1[2];
+                    gauss_block2<K, 2>(p.M, 2 * r2, a0, s0, a1, s1, y0, y1);
+                    sts4(sbuf + ((pb ^ p.loc[r2]) << 3), make_float4(y0[0].x, y0[0].y, y0[1].x, y0[1].y));
+                    sts4(sbuf + ((pb ^ p.gsec ^ p.loc[r2]) << 3), make_float4(y1[0].x, y1[0].y, y1[1].x, y1[1].y));
+                }
+            } else {
+#pragma unroll 1
+                for (int r = 0; r < D; r += SV_ROWS) {
+                    float2 y0[SV_ROWS], y1[SV_ROWS];
+                    gauss_block2<K, SV_ROWS>(p.M, r, a0, s0, a1, s1, y0, y1);
+#pragma unroll
+                    for (int i = 0; i < SV_ROWS; ++i)
+                        sts4(sbuf + ((pb ^ p.loc[r + i]) << 3), make_float4(y0[i].x, y0[i].y, y1[i].x, y1[i].y));
+                }
+            }
+        } else {
+            const uint32_t pb = swizzle((uint32_t)insert_zeros(gidx, p.ztpos, p.nzt), p.swz);
+            float2 a[D];
+            if constexpr (PAIR) {
+#pragma unroll
+                for (int jj = 0; jj < D / 2; ++jj) {
+                    const float4 v = lds4(sbuf + ((pb ^ p.loc[jj]) << 3));
+                    a[2 * jj] = make_float2(v.x, v.y);
+                    a[2 * jj + 1] = make_float2(v.z, v.w);
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < D; ++c) a[c] = lds2(sbuf + ((pb ^ p.loc[c]) << 3));
+            }
+            if constexpr (K <= 5) {
+                float s[D];
+#pragma unroll
+                for (int c = 0; c < D; ++c) s[c] = a[c].x + a[c].y;
+                if constexpr (PAIR) {
+#pragma unroll 1
+                    for (int r2 = 0; r2 < D / 2; ++r2) {
+                        float2 y[2];
+                        gauss_block<K, 2>(p.M, 2 * r2, a, s, y);
+                        sts4(sbuf + ((pb ^ p.loc[r2]) << 3), make_float4(y[0].x, y[0].y, y[1].x, y[1].y));
+                    }
+                } else {
+#pragma unroll 1
+                    for (int r = 0; r < D; ++r) {
+                        float2 y;
+                        gauss_block<K, 1>(p.M, r, a, s, &y);
+                        sts2(sbuf + ((pb ^ p.loc[r]) << 3), y);
+                    }
+                }
+            } else {
+                // k = 6: rows in a loop, matrix rows broadcast from shared memory
+#pragma unroll 1
+                for (int r2 = 0; r2 < D / 2; ++r2) {
+                    float2 y0 = make_float2(0.f, 0.f), y1 = make_float2(0.f, 0.f);
+                    const float4* m0 = reinterpret_cast<const float4*>(smat + (2 * r2) * D);
+                    const float4* m1 = reinterpret_cast<const float4*>(smat + (2 * r2 + 1) * D);
+#pragma unroll
+                    for (int c2 = 0; c2 < D / 2; ++c2) {
+                        const float4 u0 = m0[c2], u1 = m1[c2];
+                        cmac(y0, make_float2(u0.x, u0.y), a[2 * c2]);
+                        cmac(y0, make_float2(u0.z, u0.w), a[2 * c2 + 1]);
+                        cmac(y1, make_float2(u1.x, u1.y), a[2 * c2]);
+                        cmac(y1, make_float2(u1.z, u1.w), a[2 * c2 + 1]);
+                    }
+                    if constexpr (PAIR) {
+                        sts4(sbuf + ((pb ^ p.loc[r2]) << 3), make_float4(y0.x, y0.y, y1.x, y1.y));
+                    } else {
+                        sts2(sbuf + ((pb ^ p.loc[2 * r2]) << 3), y0);
+                        sts2(sbuf + ((pb ^ p.loc[2 * r2 + 1]) << 3), y1);
+                    }
+                }
+            }
+        }
+    }
+}
+
+// Persistent loop over tiles.  STAGES = 2: the copies of tile i+1 are in
+// flight while tile i is transformed and written back.
+template <int K, bool PAIR, bool MONO, int STAGES>
 __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
     extern __shared__ float4 dsm[];
     const uint32_t tile_bytes = 8u << p.T;
     const uint32_t s0 = smem_addr(dsm);
-    const float2* sm = nullptr;
+    const float2* smat = nullptr;
     if constexpr (K == 6) {
-        float2* smat = reinterpret_cast<float2*>(reinterpret_cast<char*>(dsm) + kStages * tile_bytes);
-        for (int i = threadIdx.x; i < 64 * 64; i += blockDim.x) smat[i] = p.M.dev[i];
-        sm = smat;
+        float2* sm = reinterpret_cast<float2*>(reinterpret_cast<char*>(dsm) + STAGES * tile_bytes);
+        for (int i = threadIdx.x; i < 64 * 64; i += blockDim.x) sm[i] = p.M.dev[i];
+        smat = sm;
         __syncthreads();
     }
+    // per-thread bases of the unit maps (t = 2*tid + 2*nthreads*i)
+    const uint32_t t0 = 2u * threadIdx.x;
+    const uint32_t rmask = (1u << p.r) - 1u;
+    uint64_t dthr = t0 & rmask;
+    {
+        const uint32_t h = t0 >> p.r;
+        for (int b = 0; b < p.nH; ++b)
+            if ((h >> b) & 1u) dthr += 1ull << p.Hpos[b];
+    }
+    const uint32_t sthr = swizzle(t0, p.swz);
+    const int upt = p.upt;
+    auto load = [&](uint64_t u, uint32_t sbuf) {
+        const float2* g = p.psi + insert_zeros(u << p.r, p.Hpos, p.nH) + dthr;
+        for (int i = 0; i < upt; ++i) cp_async16(sbuf + ((sthr ^ p.soff[i]) << 3), g + p.goff[i]);
+    };
+    auto store = [&](uint64_t u, uint32_t sbuf) {
+        float2* g = p.psi + insert_zeros(u << p.r, p.Hpos, p.nH) + dthr;
+        for (int i = 0; i < upt; ++i)
+            st_stream(reinterpret_cast<float4*>(g + p.goff[i]), lds4(sbuf + ((sthr ^ p.soff[i]) << 3)));
+    };
     uint64_t u = blockIdx.x;
-    if (u < p.n_tiles) tile_load<K>(p, u, s0);
-    cp_async_commit();
-    for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
-        const uint32_t cur = s0 + (uint32_t)(it & 1) * tile_bytes;
-        const uint32_t nxt = s0 + (uint32_t)((it + 1) & 1) * tile_bytes;
-        const uint64_t un = u + gridDim.x;
-        __syncthreads();  // buffer `nxt` was drained by the previous iteration's store
-        if (un < p.n_tiles) tile_load<K>(p, un, nxt);
+    if constexpr (STAGES == 2) {
+        if (u < p.n_tiles) load(u, s0);
         cp_async_commit();
-        cp_async_wait1();  // this thread's copies of tile u have landed
-        __syncthreads();   // ... and everyone else's
-        tile_compute<K, PAIR>(p, cur, sm);
-        __syncthreads();
-        tile_store<K>(p, u, cur);
+        for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
+            const uint32_t cur = s0 + (uint32_t)(it & 1) * tile_bytes;
+            const uint32_t nxt = s0 + (uint32_t)((it + 1) & 1) * tile_bytes;
+            const uint64_t un = u + gridDim.x;
+            __syncthreads();  // buffer `nxt` was drained by the previous iteration's store
+            if (un < p.n_tiles) load(un, nxt);
+            cp_async_commit();
+            cp_async_wait1();  // this thread's copies of tile u have landed
+            __syncthreads();   // ... and everyone else's
+            if constexpr (MONO) tile_compute_mono<K, PAIR>(p, cur);
+            else tile_compute<K, PAIR>(p, cur, smat);
+            __syncthreads();
+            store(u, cur);
+        }
+    } else {
+        for (; u < p.n_tiles; u += gridDim.x) {
+            __syncthreads();
+            load(u, s0);
+            cp_async_commit();
+            cp_async_wait0();
+            __syncthreads();
+            if constexpr (MONO) tile_compute_mono<K, PAIR>(p, s0);
+            else tile_compute<K, PAIR>(p, s0, smat);
+            __syncthreads();
+            store(u, s0);
+        }
     }
 }
 
+__host__ __device__ constexpr int stages_for(int K) { return K == 6 ? 1 : 2; }
+
 // The paper's two kernel classes (L110-112).  Same tile engine; "high" gates
-// (no qubit in {1,2,3}) need no swizzle and have runs of >= 16 amplitudes
-// per member, "low" gates carry their partners inside a 128 B line.
-template <int K, bool PAIR>
-__global__ void __launch_bounds__(kThreads) apply_high(const __grid_constant__ TileParams<K> p) {
-    tile_loop<K, PAIR>(p);
+// (no qubit in {1,2,3}) need no swizzle and read whole 128 B lines per
+// member, "low" gates carry partners inside one 128 B line.
+// MONO: the matrix has one nonzero per row (permutation x diagonal) -> the
+// exact y_r = m_r a_perm(r) path, a separate instantiation so the dense path
+// carries no branch.
+template <int K, bool PAIR, bool MONO>
+__global__ void __launch_bounds__(256) apply_high(const __grid_constant__ TileParams<K> p) {
+    tile_loop<K, PAIR, MONO, stages_for(K)>(p);
 }
-template <int K, bool PAIR>
-__global__ void __launch_bounds__(kThreads) apply_low(const __grid_constant__ TileParams<K> p) {
-    tile_loop<K, PAIR>(p);
+template <int K, bool PAIR, bool MONO>
+__global__ void __launch_bounds__(256) apply_low(const __grid_constant__ TileParams<K> p) {
+    tile_loop<K, PAIR, MONO, stages_for(K)>(p);
+}
+
+// Tiny states (fewer amplitudes than one tile can split into thread work):
+// one thread per group, direct global accesses.  Only used when n is small.
+template <int K>
+struct SmallParams {
+    float2* psi;
+    uint64_t n_groups;
+    int q[SV_MAX_FUSED];
+    MatStore<K> M;
+};
+template <int K>
+__global__ void __launch_bounds__(256) apply_small(const __grid_constant__ SmallParams<K> p) {
+    constexpr int D = 1 << K;
+    const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (g >= p.n_groups) return;
+    const uint64_t base = insert_zeros(g, p.q, K);
+    uint64_t off[D];
+    float2 a[D];
+#pragma unroll
+    for (int c = 0; c < D; ++c) {
+        uint64_t o = 0;
+#pragma unroll
+        for (int b = 0; b < K; ++b)
+            if ((c >> b) & 1) o |= 1ull << p.q[b];
+        off[c] = base | o;
+        a[c] = p.psi[off[c]];
+    }
+    if constexpr (K <= 5) {
+        gauss_rows<K>(p.M, a, [&](int r, float2 y) { p.psi[off[r]] = y; });
+    } else {
+        float2 y[D];
+        for (int r = 0; r < D; ++r) {
+            float2 acc = make_float2(0.f, 0.f);
+            for (int c = 0; c < D; ++c) cmac(acc, p.M.dev[r * D + c], a[c]);
+            y[r] = acc;
+        }
+        for (int r = 0; r < D; ++r) p.psi[off[r]] = y[r];
+    }
 }
 
 int g_num_sms = 0;
@@ -261,7 +493,14 @@ int num_sms() {
 
 template <int K>
 void fill_matrix(MatStore<K>& M, const ApplyDesc& d) {
-    std::memcpy(M.m, d.m.data(), sizeof(M.m));
+    constexpr int D = 1 << K;
+    for (int r = 0; r < D; ++r)
+        for (int c = 0; c < D; ++c) {
+            const cf m = d.m[(size_t)r * D + c];
+            M.P[r][c] = m.real();
+            M.S[r][c] = m.real() + m.imag();
+            M.Q[r][c] = m.imag() - m.real();
+        }
 }
 template <>
 void fill_matrix<6>(MatStore<6>& M, const ApplyDesc& d) {
@@ -270,6 +509,7 @@ void fill_matrix<6>(MatStore<6>& M, const ApplyDesc& d) {
 
 template <int K>
 cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t st) {
+    constexpr int GPT = (K <= 4) ? 2 : 1;
     TileParams<K> p;
     std::memset(&p, 0, sizeof(p));
     p.psi = psi;
@@ -277,8 +517,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     p.T = d.T;
     p.r = d.r;
     const bool pair = d.q[0] == 0;
-    // tile-local gate positions
-    int tl[SV_MAX_FUSED];
+    int tl[SV_MAX_FUSED];  // tile-local gate positions
     for (int b = 0; b < K; ++b) {
         if (d.q[b] < p.r) {
             tl[b] = d.q[b];
@@ -287,55 +526,125 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
             p.Hpos[p.nH++] = d.q[b];
         }
     }
-    for (int h = 0; h < (1 << p.nH); ++h) {
-        uint64_t o = 0;
-        for (int b = 0; b < p.nH; ++b)
-            if ((h >> b) & 1) o |= 1ull << p.Hpos[b];
-        p.offH[h] = o;
-    }
     p.nzt = K;
     for (int b = 0; b < K; ++b) p.ztpos[b] = tl[b];
-    // swizzle: the lanes of one shared-memory phase run over the lowest W
-    // non-gate tile bits; each gate bit f in {1,2,3} (fixed within a gather)
-    // is XORed with one of those lane bits >= 4, so the W lanes hit W distinct
-    // 8/16 B bank slots.  Linear over GF(2), so phys(base ^ off) = phys(base) ^ phys(off).
     uint32_t gmask = 0;
     for (int b = 0; b < K; ++b) gmask |= 1u << tl[b];
-    const int W = pair ? 3 : 4;
-    int hl[8], nhl = 0, nl = 0;
-    for (int t = 0; t < p.T && nl < W; ++t)
-        if (!((gmask >> t) & 1)) {
-            ++nl;
-            if (t >= 4) hl[nhl++] = t;
-        }
-    int j = 0;
+    int ng[32], nng = 0;  // non-gate tile bits, ascending
+    for (int t = 0; t < p.T; ++t)
+        if (!((gmask >> t) & 1)) ng[nng++] = t;
+    // Bank-conflict-free gathers: one shared-memory phase is 8 lanes of 16 B
+    // (or 16 lanes of 8 B when GPT = 1 and bit 0 is free).  Lanes run over the
+    // non-gate bits `lane`; every bit in {1,2,3} that is fixed within one gather
+    // (a gate bit, or the pair-of-groups bit) is XORed with one lane bit >= 4.
+    std::vector<int> lane;
+    uint32_t fixed = gmask;
+    if (GPT == 2) {
+        // ng[0] selects the group of the pair (bit 0 when free -> inside the 16 B word)
+        if (pair) fixed |= 1u << ng[0];
+        for (int i = 1; i < nng && (int)lane.size() < 3; ++i) lane.push_back(ng[i]);
+    } else {
+        const int W = pair ? 3 : 4;
+        for (int i = 0; i < nng && (int)lane.size() < W; ++i) lane.push_back(ng[i]);
+    }
+    std::vector<int> hl;
+    for (int t : lane)
+        if (t >= 4) hl.push_back(t);
+    size_t jh = 0;
     for (int f = 1; f <= 3; ++f)
-        if (((gmask >> f) & 1) && j < nhl) p.swz[f - 1] = 1u << hl[j++];
+        if (((fixed >> f) & 1) && jh < hl.size()) p.swz[f - 1] = 1u << hl[jh++];
     auto sw = [&](uint32_t t) {
         return t ^ ((__builtin_popcount(t & p.swz[0]) & 1) << 1) ^ ((__builtin_popcount(t & p.swz[1]) & 1) << 2) ^
                ((__builtin_popcount(t & p.swz[2]) & 1) << 3);
     };
-    const int ng = pair ? (1 << (K - 1)) : (1 << K);
-    for (int m = 0; m < ng; ++m) {
+    auto dep = [&](uint64_t t) {
+        uint64_t g = t & ((1ull << p.r) - 1);
+        const uint64_t h = t >> p.r;
+        for (int b = 0; b < p.nH; ++b)
+            if ((h >> b) & 1) g += 1ull << p.Hpos[b];
+        return g;
+    };
+    const int nloc = pair ? (1 << (K - 1)) : (1 << K);
+    for (int m = 0; m < nloc; ++m) {
         const int mm = pair ? (m << 1) : m;
         uint32_t o = 0;
         for (int b = 0; b < K; ++b)
             if ((mm >> b) & 1) o |= 1u << tl[b];
         p.loc[m] = sw(o);
     }
+    if (GPT == 2 && pair) p.gsec = sw(1u << ng[0]);
+    {
+        // monomial detection on the complex64 matrix (exact zeros)
+        constexpr int D = 1 << K;
+        int src[D];
+        bool mono = true;
+        uint64_t used = 0;
+        for (int r = 0; r < D && mono; ++r) {
+            int cnt = 0;
+            for (int c = 0; c < D; ++c) {
+                const cf m = d.m[(size_t)r * D + c];
+                if (m.real() != 0.f || m.imag() != 0.f) {
+                    ++cnt;
+                    src[r] = c;
+                }
+            }
+            if (cnt != 1 || ((used >> src[r]) & 1)) mono = false;
+            else used |= 1ull << src[r];
+        }
+        p.mono = mono ? 1 : 0;
+        if (mono) {
+            for (int r = 0; r < D; ++r) {
+                uint32_t o = 0, oc = 0;
+                for (int b = 0; b < K; ++b) {
+                    if ((r >> b) & 1) o |= 1u << tl[b];
+                    if ((src[r] >> b) & 1) oc |= 1u << tl[b];
+                }
+                p.mloc[r] = sw(o);
+                p.ploc[r] = sw(oc);
+                const cf m = d.m[(size_t)r * D + src[r]];
+                p.mdiag[r] = make_float2(m.real(), m.imag());
+            }
+        }
+    }
+    // threads: one (GPT = 1) or two (GPT = 2) groups each per compute step
+    const int wbits = p.T - K - (GPT == 2 ? 1 : 0);
+    const uint32_t work = wbits >= 0 ? (1u << wbits) : 0u;
+    const uint32_t nthr = std::min<uint32_t>(256, std::max<uint32_t>(32, work));
+    p.iters = (int)std::max<uint32_t>(1, work / nthr);
+    const uint32_t units = 1u << (p.T - 1);
+    p.upt = (int)(units / nthr);
+    if (p.T < K + (GPT == 2 ? 1 : 0) || work < 32 || p.upt < 1 || p.upt > 64 || work < nthr) {
+        SmallParams<K> sp;
+        std::memset(&sp, 0, sizeof(sp));
+        sp.psi = psi;
+        sp.n_groups = 1ull << (n - K);
+        for (int b = 0; b < K; ++b) sp.q[b] = d.q[b];
+        fill_matrix<K>(sp.M, d);
+        apply_small<K><<<(unsigned)((sp.n_groups + 255) / 256), 256, 0, st>>>(sp);
+        return cudaGetLastError();
+    }
+    for (int i = 0; i < p.upt; ++i) {
+        p.goff[i] = dep(2ull * nthr * i);
+        p.soff[i] = sw(2u * nthr * i);
+    }
     p.n_tiles = 1ull << (n - p.T);
-    size_t smem = (size_t)kStages * ((size_t)8 << p.T);
+    constexpr int STG = stages_for(K);
+    size_t smem = (size_t)STG * ((size_t)8 << p.T);
     if (K == 6) smem += 64 * 64 * 8;
-    const int per_sm = std::max(1, (int)((220 * 1024) / (smem + 1024)));
-    const uint64_t grid = std::max<uint64_t>(1, std::min<uint64_t>(p.n_tiles, (uint64_t)num_sms() * per_sm));
+    const int per_sm_smem = std::max(1, (int)((227 * 1024) / (smem + 1024)));
+    const uint64_t grid = std::max<uint64_t>(1, std::min<uint64_t>(p.n_tiles, (uint64_t)num_sms() * per_sm_smem));
     auto go = [&](auto kern) -> cudaError_t {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        kern<<<(unsigned)grid, kThreads, smem, st>>>(p);
+        kern<<<(unsigned)grid, nthr, smem, st>>>(p);
         return cudaGetLastError();
     };
-    if (d.high) return pair ? go(apply_high<K, true>) : go(apply_high<K, false>);
-    return pair ? go(apply_low<K, true>) : go(apply_low<K, false>);
+    if (p.mono) {
+        if (d.high) return pair ? go(apply_high<K, true, true>) : go(apply_high<K, false, true>);
+        return pair ? go(apply_low<K, true, true>) : go(apply_low<K, false, true>);
+    }
+    if (d.high) return pair ? go(apply_high<K, true, false>) : go(apply_high<K, false, false>);
+    return pair ? go(apply_low<K, true, false>) : go(apply_low<K, false, false>);
 }
 
 }  // namespace
@@ -346,7 +655,7 @@ void plan_apply(int n, ApplyDesc& d) {
     d.high = (gm & kLowMask) == 0;
     // tile: runs of >= 16 amplitudes (128 B); grow the run until the tile
     // reaches the target size (32 KB for k <= 4).
-    const int target = std::min(n, d.k <= 4 ? 12 : 13);
+    const int target = std::min(n, d.k <= 5 ? 12 : 14);
     auto tile_bits = [&](int rr) {
         int t = rr;
         for (int b = 0; b < d.k; ++b)

@@ -233,7 +233,8 @@ void make_apply(int l, int k, const int* phys_in_order, const cd* M /* bit b <->
 }
 
 // PERMUTE (data at local bit b moves to bit perm[b]) as passes of disjoint
-// transpositions, <= 3 per pass (a 2t-qubit permutation matrix; exact).
+// transpositions, <= 2 per pass (a 4-qubit permutation matrix carried in the
+// kernel parameters; the FMA chain of a 0/1 matrix is exact).
 void lower_permute(int l, const std::vector<int>& perm, std::vector<ApplyDesc>& out) {
     // current[b] = which original bit's data sits at bit b; target: bit perm[b] holds original b
     std::vector<int> where(l);  // where[orig] = current position of orig's data
@@ -256,7 +257,7 @@ void lower_permute(int l, const std::vector<int>& perm, std::vector<ApplyDesc>& 
     while (i < swaps.size()) {
         std::vector<std::pair<int, int>> pass;
         uint64_t used = 0;
-        while (i < swaps.size() && pass.size() < 3) {
+        while (i < swaps.size() && pass.size() < 2) {
             const auto sw = swaps[i];
             const uint64_t m = (1ull << sw.first) | (1ull << sw.second);
             if (used & m) break;  // keep order: a later swap touching these bits goes to the next pass
