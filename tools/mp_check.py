@@ -1,0 +1,87 @@
+"""Multi-process sharded mode check (one process per shard).
+
+Launched by tests/test_gpu_multiproc.py as
+  python -m torch.distributed.run --nproc-per-node P --master-addr 127.0.0.1 ... tools/mp_check.py N
+Every rank owns one shard (sv_create_ex(world=P, rank, virtual_shards=0));
+the shards are cross-mapped with CUDA IPC handles exchanged through
+torch.distributed (gloo all_gather_object -- plumbing only).  Ranks map onto
+cuda:(local_rank % device_count), so P processes can share one GPU.
+
+Rank 0 checks the sharded results against the oracle and prints OK.
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+import paper_conf_sc_markidis23_b200 as sv
+from oracle import ref_c
+from oracle import sample as osample
+from oracle import sv as osv
+from workloads import rqc as W
+
+
+def main():
+    n = int(sys.argv[1]) if len(sys.argv) > 1 else 14
+    dist.init_process_group("gloo")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dev = local % torch.cuda.device_count()
+    torch.cuda.set_device(dev)
+    h = sv.sv_create_ex(n, world=world, rank=rank, virtual_shards=False, device=dev)
+    blobs = [None] * world
+    dist.all_gather_object(blobs, sv.sv_ipc_handle(h))
+    sv.sv_attach_peers(h, blobs)
+    ok = True
+    msgs = []
+    # 1. circuit through exchanges
+    gates = W.rqc(n, 14, seed=3)
+    st = sv.sv_run_circuit(h, gates, 4)
+    psi = sv.sv_get_state(h, n)
+    ref = ref_c.run(n, gates)
+    fid = osv.fidelity(psi.astype(np.complex128), ref)
+    err = float(np.abs(psi.astype(np.complex128) - ref).max())
+    if not (fid >= 1 - 1e-5 and err <= osv.max_abs_bound(n, 14) and st["n_exchanges"] >= 1):
+        ok = False
+        msgs.append(f"circuit fid={fid} err={err} exch={st['n_exchanges']}")
+    # 2. amplitudes
+    idx = np.random.default_rng(1).integers(0, 1 << n, size=200).astype(np.uint64)
+    amps = sv.sv_amplitudes(h, idx)
+    if not np.array_equal(amps, psi[idx.astype(np.int64)]):
+        ok = False
+        msgs.append("amplitudes mismatch")
+    # 3. sampling on a seeded state: bit-exact vs the oracle
+    s0 = W.random_state_c64(n, 11)
+    sv.sv_set_state(h, s0)
+    got = sv.sv_sample(h, 42, 4000)
+    exp, _ = osample.sample(s0, 42, 4000)
+    if not np.array_equal(got, exp):
+        ok = False
+        msgs.append("sampling mismatch")
+    # 4. single apply touching a global qubit (exchange inside sv_apply_fused)
+    sv.sv_set_state(h, s0)
+    M = W.haar_unitary(4, np.random.default_rng(5)).astype(np.complex64)
+    sv.sv_apply_fused(h, [n - 1, 2], M)
+    got = sv.sv_get_state(h, n).astype(np.complex128)
+    exp = osv.apply_gate(s0.astype(np.complex128), n, [n - 1, 2], M.astype(np.complex128))
+    if np.abs(got - exp).max() > 1e-6:
+        ok = False
+        msgs.append(f"apply with global qubit err={np.abs(got - exp).max()}")
+    flags = [None] * world
+    dist.all_gather_object(flags, (ok, msgs))
+    sv.sv_destroy(h)
+    dist.barrier()
+    if rank == 0:
+        if all(f[0] for f in flags):
+            print(f"MP_OK world={world} n={n}")
+        else:
+            print("MP_FAIL", flags)
+    dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
