@@ -23,6 +23,8 @@ struct ApplyDesc {
     int q[SV_MAX_FUSED] = {0};        // ascending physical qubits (within a shard)
     std::vector<cf> m;                // 2^k x 2^k row-major over ascending q, complex64
     bool high = false;                // kernel class
+    bool mono = false;                // one nonzero per row (exact permutation/diagonal path)
+    bool tc = false;                  // tensor-core path (tc.cu)
     // low-kernel tile plan (host-computed once)
     int T = 0, r = 0;                 // tile bits, run bits
     // device copy of m for k == 6 (owned by the circuit / state scratch)
@@ -31,6 +33,10 @@ struct ApplyDesc {
 
 // Decide high/low and the tile plan for a gate on `n` local qubits.
 void plan_apply(int n_local, ApplyDesc& d);
+
+// Dense k = 4, 5 gates run on the tensor cores (tcgen05, TF32 x3) when the
+// shard has at least 2^13 amplitudes.
+bool tc_supported(int n_local, const ApplyDesc& d);
 
 // Launch one fused-gate apply on a shard of 2^n_local amplitudes.
 cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);
