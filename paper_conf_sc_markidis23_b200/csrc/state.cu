@@ -63,17 +63,31 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
     return v;
 }
 
-// One warp per 32-amplitude bin.
+// 8 lanes per 32-amplitude bin, 4 amplitudes (two 16 B loads) per lane.
 __global__ void bin_weights_kernel(const float2* __restrict__ psi, uint64_t n_amps, uint64_t* __restrict__ bins,
                                    uint64_t n_bins) {
-    const int lane = threadIdx.x & 31;
-    const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t b = warp; b < n_bins; b += nwarps) {
-        const uint64_t i = (b << kSampleBinBits) + lane;
-        uint64_t w = (i < n_amps) ? weight(__ldcs(psi + i)) : 0ull;
-        w = warp_sum_u64(w);
-        if (lane == 0) bins[b] = w;
+    const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;  // multiple of 32
+    const int sub = threadIdx.x & 7;
+    const uint64_t full_bins = n_amps >> kSampleBinBits;  // bins with all 32 amplitudes
+    // warp-uniform loop (4 bins per warp per trip) so the shuffles see all lanes
+    for (uint64_t b0 = (tid >> 5) << 2; b0 < n_bins; b0 += (nthr >> 5) << 2) {
+        const uint64_t b = b0 + ((threadIdx.x & 31) >> 3);
+        uint64_t w = 0;
+        const uint64_t i0 = (b << kSampleBinBits) + 4 * sub;
+        if (b < full_bins) {
+            const float4 u = __ldcs(reinterpret_cast<const float4*>(psi + i0));
+            const float4 v = __ldcs(reinterpret_cast<const float4*>(psi + i0 + 2));
+            w = weight(make_float2(u.x, u.y)) + weight(make_float2(u.z, u.w)) + weight(make_float2(v.x, v.y)) +
+                weight(make_float2(v.z, v.w));
+        } else if (b < n_bins) {
+            for (int j = 0; j < 4; ++j)
+                if (i0 + j < n_amps) w += weight(psi[i0 + j]);
+        }
+        w += __shfl_xor_sync(0xffffffffu, w, 1);
+        w += __shfl_xor_sync(0xffffffffu, w, 2);
+        w += __shfl_xor_sync(0xffffffffu, w, 4);
+        if (sub == 0 && b < n_bins) bins[b] = w;
     }
 }
 
@@ -189,47 +203,56 @@ struct XParams {
     int pj[8];     // pj[t] = j of the t-th smallest position
 };
 
-// Thread z in [0, 2^l) of shard d: chunk c = bits of z at p_j, x = remaining
-// bits.  Partner e = d with device bits (P_j - l) := c_j; partner chunk cd =
-// d's device bits (P_j - l).  The pair {(d,c),(e,cd)} is split in halves of x:
-// the lower shard of the pair swaps x < half, the other x >= half, so P ranks
-// share the work evenly and every element pair is swapped exactly once.
+// Shard d swaps, for every chunk c != c_d, its chunk c with chunk c_d of
+// shard e (e = d with device bits (P_j - l) := c_j, c_d = d's device bits);
+// the 2^(l-s) elements x of a chunk pair are split in halves: the lower shard
+// of the pair swaps x < half, the other x >= half, so P ranks share the work
+// evenly and every element pair is swapped exactly once.  Work item w of
+// shard d enumerates only the elements it swaps: (chunk index, x in its half);
+// VEC: all p_j >= 1, so x is handled in pairs of neighbouring amplitudes (16 B).
+template <bool VEC>
 __global__ void exchange_kernel(const __grid_constant__ XParams xp) {
-    const uint64_t nloc = 1ull << xp.l;
-    const uint64_t half = 1ull << (xp.l - xp.s - 1);
-    const uint64_t total = (uint64_t)(xp.d1 - xp.d0) * nloc;
+    const int l = xp.l, s = xp.s;
+    const int hb = l - s - 1 - (VEC ? 1 : 0);  // bits of the per-chunk work index
+    const uint64_t per_chunk = 1ull << hb;
+    const uint64_t per_shard = per_chunk * (uint64_t)((1 << s) - 1);
+    const uint64_t total = per_shard * (uint64_t)(xp.d1 - xp.d0);
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t gz = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; gz < total; gz += stride) {
-        const int d = xp.d0 + (int)(gz >> xp.l);
-        const uint64_t z = gz & (nloc - 1);
-        uint32_t c = 0, cd = 0;
+    const uint64_t half = 1ull << (l - s - 1);
+    for (uint64_t gw = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; gw < total; gw += stride) {
+        const int d = xp.d0 + (int)(gw / per_shard);
+        const uint64_t w = gw % per_shard;
+        uint32_t cd = 0;
+        for (int j = 0; j < s; ++j) cd |= (uint32_t)((d >> (xp.P[j] - l)) & 1) << j;
+        uint32_t c = (uint32_t)(w >> hb);
+        if (c >= cd) ++c;  // skip the self chunk
         int e = d;
-        for (int j = 0; j < xp.s; ++j) {
-            c |= (uint32_t)((z >> xp.p[j]) & 1ull) << j;
-            const int gb = xp.P[j] - xp.l;
-            cd |= (uint32_t)((d >> gb) & 1) << j;
+        for (int j = 0; j < s; ++j) {
+            const int gb = xp.P[j] - l;
             e = (e & ~(1 << gb)) | (int)(((c >> j) & 1u) << gb);
         }
-        if (e == d) continue;  // c == cd: self-swap
-        // remove the chunk bits (descending positions) -> x
-        uint64_t x = z;
-        for (int t = xp.s - 1; t >= 0; --t) {
+        uint64_t x = (w & (per_chunk - 1)) << (VEC ? 1 : 0);
+        if (d > e) x += half;
+        uint64_t za = x, zb = x;
+        for (int t = 0; t < s; ++t) {
             const int q = xp.ps[t];
-            x = ((x >> (q + 1)) << q) | (x & ((1ull << q) - 1ull));
-        }
-        if ((d < e) != (x < half)) continue;
-        // partner offset: insert cd's bits at ascending positions
-        uint64_t zb = x;
-        for (int t = 0; t < xp.s; ++t) {
-            const int q = xp.ps[t];
-            zb = ((zb >> q) << (q + 1)) | ((uint64_t)((cd >> xp.pj[t]) & 1u) << q) | (zb & ((1ull << q) - 1ull));
+            const uint64_t lo_a = za & ((1ull << q) - 1ull), lo_b = zb & ((1ull << q) - 1ull);
+            za = ((za >> q) << (q + 1)) | ((uint64_t)((c >> xp.pj[t]) & 1u) << q) | lo_a;
+            zb = ((zb >> q) << (q + 1)) | ((uint64_t)((cd >> xp.pj[t]) & 1u) << q) | lo_b;
         }
         float2* A = xp.shards[d];
         float2* B = xp.shards[e];
-        const float2 va = A[z];
-        const float2 vb = B[zb];
-        A[z] = vb;
-        B[zb] = va;
+        if constexpr (VEC) {
+            float4* pa = reinterpret_cast<float4*>(A + za);
+            float4* pb = reinterpret_cast<float4*>(B + zb);
+            const float4 va = *pa, vb = *pb;
+            *pa = vb;
+            *pb = va;
+        } else {
+            const float2 va = A[za], vb = B[zb];
+            A[za] = vb;
+            B[zb] = va;
+        }
     }
 }
 
@@ -251,7 +274,8 @@ cudaError_t launch_gather(const float2* psi, const uint64_t* phys, const int32_t
 
 cudaError_t launch_bin_weights(const float2* psi, uint64_t n_amps, uint64_t* bins, cudaStream_t st) {
     const uint64_t n_bins = (n_amps + (1u << kSampleBinBits) - 1) >> kSampleBinBits;
-    bin_weights_kernel<<<grid_cap(n_bins * 32, 256, 16), 256, 0, st>>>(psi, n_amps, bins, n_bins);
+    // whole warps per loop trip (the 8-lane shuffles need all lanes): round the grid to warps
+    bin_weights_kernel<<<grid_cap(n_bins * 8, 256, 16), 256, 0, st>>>(psi, n_amps, bins, n_bins);
     return cudaGetLastError();
 }
 
@@ -304,8 +328,12 @@ cudaError_t launch_exchange(float2* const* shards_dev, int world, int me, const 
     }
     std::sort(p.pj, p.pj + x.s, [&](int a, int b) { return x.p[a] < x.p[b]; });
     for (int t = 0; t < x.s; ++t) p.ps[t] = x.p[p.pj[t]];
-    const uint64_t total = (uint64_t)(p.d1 - p.d0) << x.l;
-    exchange_kernel<<<grid_cap(total, 256, 16), 256, 0, st>>>(p);
+    bool vec = x.l - x.s - 1 >= 1;
+    for (int j = 0; j < x.s; ++j)
+        if (x.p[j] < 1) vec = false;
+    const uint64_t total = ((uint64_t)(p.d1 - p.d0) * (((1ull << x.s) - 1) << (x.l - x.s - 1))) >> (vec ? 1 : 0);
+    if (vec) exchange_kernel<true><<<grid_cap(total, 256, 16), 256, 0, st>>>(p);
+    else exchange_kernel<false><<<grid_cap(total, 256, 16), 256, 0, st>>>(p);
     return cudaGetLastError();
 }
 
