@@ -38,6 +38,17 @@ void plan_apply(int n_local, ApplyDesc& d);
 // shard has at least 2^13 amplitudes.
 bool tc_supported(int n_local, const ApplyDesc& d);
 
+// Whole circuit in one CTA with the state in shared memory (n <= 13).
+constexpr int kSmallCircuitMaxQubits = 13;
+struct SmallGateDesc {
+    int k;
+    int q[SV_MAX_FUSED];  // ascending
+    uint32_t mat_off;     // offset (complex elements) of the 2^k x 2^k matrix
+};
+size_t small_circuit_smem(int n);
+cudaError_t launch_small_circuit(float2* psi, int n, int ngates, const SmallGateDesc* gates_dev,
+                                 const float2* mats_dev, cudaStream_t st);
+
 // Launch one fused-gate apply on a shard of 2^n_local amplitudes.
 cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);
 

@@ -116,6 +116,11 @@ struct sv_circuit {
     };
     std::vector<Step> steps;
     float2* dev_mats = nullptr;
+    // small states (n <= 13, unsharded): whole circuit in one CTA (small.cu)
+    bool small = false;
+    int n_small = 0;
+    SmallGateDesc* small_gates = nullptr;
+    float2* small_mats = nullptr;
     sv_stats stats{};
 };
 
@@ -730,6 +735,30 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
                               s->stream));
         CK(s, cudaStreamSynchronize(s->stream));
     }
+    if (s->g == 0 && s->n <= kSmallCircuitMaxQubits) {
+        std::vector<SmallGateDesc> gd;
+        std::vector<float2> mats;
+        for (auto& st : c->steps) {
+            SmallGateDesc g{};
+            g.k = st.apply.k;
+            for (int b = 0; b < g.k; ++b) g.q[b] = st.apply.q[b];
+            g.mat_off = (uint32_t)mats.size();
+            for (const cf& m : st.apply.m) mats.push_back(make_float2(m.real(), m.imag()));
+            gd.push_back(g);
+        }
+        c->n_small = (int)gd.size();
+        if (c->n_small > 0) {
+            cudaError_t e = cudaMalloc(&c->small_gates, gd.size() * sizeof(SmallGateDesc));
+            if (e == cudaSuccess) e = cudaMalloc(&c->small_mats, mats.size() * sizeof(float2));
+            if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(small circuit)");
+            CK(s, cudaMemcpyAsync(c->small_gates, gd.data(), gd.size() * sizeof(SmallGateDesc), cudaMemcpyHostToDevice,
+                                  s->stream));
+            CK(s, cudaMemcpyAsync(c->small_mats, mats.data(), mats.size() * sizeof(float2), cudaMemcpyHostToDevice,
+                                  s->stream));
+            CK(s, cudaStreamSynchronize(s->stream));
+        }
+        c->small = true;
+    }
     c->stats.t_upload_s = now_s() - t2;
     *out = c.release();
     return SV_OK;
@@ -747,6 +776,20 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     s->stats.t_upload_s = keep.t_upload_s;
     s->stats.n_fused = keep.n_fused;
     for (int k = 0; k < 7; ++k) s->stats.fused_hist[k] = keep.fused_hist[k];
+    if (c->small) {
+        if (c->n_small > 0) {
+            rc = launch(s, LaunchClass::HIGH, [&] {
+                return launch_small_circuit(s->shard[0], s->n, c->n_small, c->small_gates, c->small_mats, s->stream);
+            });
+            if (rc) return rc;
+            for (auto& st : c->steps) {
+                s->stats.bytes_apply += 16ull << s->l;
+                s->stats.flops_apply += (uint64_t)((8 << st.apply.k) - 2) << s->l;
+            }
+        }
+        s->pos = c->pos_out;
+        return SV_OK;
+    }
     for (auto& st : c->steps) {
         if (st.type == Event::APPLY) {
             rc = run_apply(s, st.apply);
@@ -772,9 +815,11 @@ int sv_circuit_stats(const sv_circuit* c, sv_stats* st) {
 
 int sv_circuit_destroy(sv_circuit* c) {
     if (!c) return fail(SV_EINVAL, "circuit is NULL");
-    if (c->dev_mats) {
+    if (c->dev_mats || c->small_gates || c->small_mats) {
         if (c->owner && c->owner->stream) cudaStreamSynchronize(c->owner->stream);
-        cudaFree(c->dev_mats);
+        if (c->dev_mats) cudaFree(c->dev_mats);
+        if (c->small_gates) cudaFree(c->small_gates);
+        if (c->small_mats) cudaFree(c->small_mats);
     }
     delete c;
     return SV_OK;
