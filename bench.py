@@ -59,6 +59,7 @@ def parse():
     ap.add_argument("--max-fused", type=int, default=4)
     ap.add_argument("--seed", type=int, default=2023)
     ap.add_argument("--samples", type=int, default=N_SAMPLES)
+    ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
@@ -206,6 +207,8 @@ def run_ours(args):
         blobs = [None] * world
         dist.all_gather_object(blobs, blob)
         sv.sv_attach_peers(h, blobs)
+    if args.block_bits >= 0:
+        sv.sv_set_blocking(h, args.block_bits)
     samples_dev = torch.empty(args.samples, dtype=torch.int64, device="cuda")
 
     def barrier():
@@ -335,6 +338,8 @@ def run_ours(args):
                 "apply_gbs_low": (16 << (n - (world.bit_length() - 1))) * n_low / t_low / 1e9 if t_low else None,
                 "apply_tflops": flops / t_apply / 1e12 if t_apply else None,
                 "fuse_plan_upload_s": cst["t_fuse_s"] + cst["t_plan_s"] + cst["t_upload_s"],
+                "apply_launches_per_step": launches_apply // max(args.steps, 1),
+                "block_bits": args.block_bits,
             },
             "roofline": {"bound": "hbm", "kernel": "apply_high+apply_low", "achieved": achieved, "peak": peak,
                          "peak_source": peak_src, "unit": "GB/s", "frac": frac,

@@ -190,6 +190,14 @@ int sv_ipc_handle(sv_state* s, void* out, size_t cap, size_t* need);
 int sv_attach_peers(sv_state* s, const void* handles, size_t each);
 
 /* ---- misc ------------------------------------------------------------------- */
+/* Cache-blocked circuit execution (related work [12],
+ * PAPER.md L221): sv_circuit_create on an unsharded state with max_fused in
+ * [1,4] groups the fused gates into passes whose qubits all lie in one set of
+ * tile_bits qubits; each pass is ONE HBM read + write of the state with all its
+ * gates applied in shared memory.  tile_bits in [10,13]; 0 disables (one launch
+ * per fused gate).  Default 0 (off: on B200 the per-gate path is faster today,
+ * DESIGN.md).  Takes effect for circuits created afterwards. */
+int sv_set_blocking(sv_state* s, int tile_bits);
 /* 1: record CUDA events around every launch and fill the *_dev_s stats. */
 int sv_set_timing(sv_state* s, int enable);
 /* Stats of the most recent run on this handle. */

@@ -112,6 +112,7 @@ _SIGS = {
     "sv_qubit_map": ([_vp, _i32p], ctypes.c_int),
     "sv_ipc_handle": ([_vp, _vp, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_attach_peers": ([_vp, _vp, _sz], ctypes.c_int),
+    "sv_set_blocking": ([_vp, ctypes.c_int], ctypes.c_int),
     "sv_set_timing": ([_vp, ctypes.c_int], ctypes.c_int),
     "sv_last_stats": ([_vp, ctypes.POINTER(sv_stats)], ctypes.c_int),
     "sv_synchronize": ([_vp], ctypes.c_int),
@@ -313,6 +314,10 @@ def sv_attach_peers(h: int, blobs: Sequence[bytes]) -> None:
 
 
 # ---- misc ----------------------------------------------------------------------------
+def sv_set_blocking(h: int, tile_bits: int) -> None:
+    _check(lib().sv_set_blocking(h, tile_bits), "sv_set_blocking")
+
+
 def sv_set_timing(h: int, enable: bool) -> None:
     _check(lib().sv_set_timing(h, 1 if enable else 0), "sv_set_timing")
 

@@ -49,6 +49,24 @@ size_t small_circuit_smem(int n);
 cudaError_t launch_small_circuit(float2* psi, int n, int ngates, const SmallGateDesc* gates_dev,
                                  const float2* mats_dev, cudaStream_t st);
 
+// Cache-blocked pass (blocked.cu): all gates of the pass act on qubits in S
+// (|S| = tile bits, contains 0..r-1); one HBM read + write per pass.
+constexpr int kPassMaxGates = 64;
+constexpr int kPassPlaneFloats = 6144;
+struct PassGate {
+    int k;          // 1..4
+    int pos[4];     // tile-local positions (rank of the qubit in sorted S), ascending
+    uint32_t poff;  // offset (floats) of the gate's planes P, S, Q (3 x 4^k floats)
+};
+struct PassDesc {
+    std::vector<int> S;  // qubits of the tile
+    int r = 0;           // run bits (S[0..r) == 0..r-1)
+    std::vector<PassGate> gates;
+    std::vector<float> planes;
+};
+void plan_pass_tile(PassDesc& pd);
+cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
+
 // Launch one fused-gate apply on a shard of 2^n_local amplitudes.
 cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);
 

@@ -59,6 +59,7 @@ struct sv_state {
     bool virt = true;         // all shards on this GPU
     int device = 0;
     int vmin = 5;
+    int block_bits = 0;       // cache-blocked passes: tile qubits (0 = off; opt-in)
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     std::vector<float2*> shard;        // shard pointers (local or peer-mapped)
@@ -110,7 +111,9 @@ struct sv_circuit {
     std::vector<int> pos_in, pos_out;
     struct Step {
         Event::Type type;
+        bool block = false;                   // APPLY of a cache-blocked pass (pass below)
         ApplyDesc apply;
+        PassDesc pass;
         ExchangeDesc exch;
         std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
     };
@@ -701,8 +704,85 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
     }
     c->pos_out = pos;
+    // Cache-blocked passes (unsharded, large states, k <= 4): the S4 planner
+    // with "local" = the tile's T slots cuts the fused list into passes; a
+    // remap only changes the tile's qubit set S (no data movement).
+    const int T = s->block_bits;
+    bool blocked = s->g == 0 && T >= 10 && s->n >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
+                   max_fused >= 1;
+    std::vector<PassDesc> passes;
+    if (blocked) {
+        std::vector<std::vector<int>> fq;
+        for (auto& f : plan) fq.emplace_back(f.q, f.q + f.k);
+        std::vector<Event> bev;
+        std::vector<int> bpos;
+        plan_sharded(fq, s->n, s->n - T, 5, bev, bpos);
+        std::vector<int> ppos(s->n), inv(s->n);
+        for (int q = 0; q < s->n; ++q) ppos[q] = inv[q] = q;
+        auto new_pass = [&]() {
+            PassDesc pd;
+            for (int p = 0; p < T; ++p) pd.S.push_back(inv[p]);
+            plan_pass_tile(pd);
+            return pd;
+        };
+        PassDesc cur = new_pass();
+        for (auto& e : bev) {
+            if (e.type == Event::EXCHANGE) {
+                for (auto& pr : e.pairs) {
+                    const int a = inv[pr.first], b = inv[pr.second];
+                    ppos[a] = pr.second;
+                    ppos[b] = pr.first;
+                    inv[pr.first] = b;
+                    inv[pr.second] = a;
+                }
+                if (!cur.gates.empty()) passes.push_back(std::move(cur));
+                cur = new_pass();
+                continue;
+            }
+            const FusedGate& f = plan[e.fused];
+            const int D = 1 << f.k;
+            if ((int)cur.gates.size() == kPassMaxGates || cur.planes.size() + 3 * D * D > (size_t)kPassPlaneFloats) {
+                passes.push_back(cur);
+                cur.gates.clear();
+                cur.planes.clear();
+            }
+            PassGate pg{};
+            pg.k = f.k;
+            for (int b = 0; b < f.k; ++b)
+                pg.pos[b] = (int)(std::find(cur.S.begin(), cur.S.end(), f.q[b]) - cur.S.begin());
+            pg.poff = (uint32_t)cur.planes.size();
+            std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
+            for (int i = 0; i < D * D; ++i) {
+                const float re = (float)f.M[i].real(), im = (float)f.M[i].imag();
+                Pp[i] = re;
+                Sp[i] = re + im;
+                Qp[i] = im - re;
+            }
+            cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
+            cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
+            cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
+            cur.gates.push_back(pg);
+        }
+        if (!cur.gates.empty()) passes.push_back(std::move(cur));
+        // tiles need contiguous runs of >= 16 amplitudes (T - 5 >= 4 >= k keeps
+        // the planner from evicting qubits 0..4; checked, else run unblocked)
+        for (auto& pd : passes)
+            if (pd.r < 4) blocked = false;
+    }
     const double t2 = now_s();
     c->stats.t_plan_s = t2 - t1;
+    if (blocked) {
+        for (auto& pd : passes) {
+            sv_circuit::Step st;
+            st.type = Event::APPLY;
+            st.block = true;
+            st.pass = std::move(pd);
+            c->steps.push_back(std::move(st));
+        }
+        c->stats.t_upload_s = now_s() - t2;
+        *out = c.release();
+        return SV_OK;
+    }
     // lower events to launch descriptors
     size_t n6 = 0;
     for (auto& e : ev) {
@@ -791,6 +871,13 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
         return SV_OK;
     }
     for (auto& st : c->steps) {
+        if (st.block) {
+            rc = launch(s, LaunchClass::HIGH, [&] { return launch_pass(s->shard[0], s->l, st.pass, s->stream); });
+            if (rc) return rc;
+            s->stats.bytes_apply += 16ull << s->l;
+            for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
+            continue;
+        }
         if (st.type == Event::APPLY) {
             rc = run_apply(s, st.apply);
         } else if (st.type == Event::EXCHANGE) {
@@ -1109,6 +1196,14 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each) {
     rc = barrier(s);
     if (rc) return rc;
     return sync(s);
+}
+
+int sv_set_blocking(sv_state* s, int tile_bits) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    if (tile_bits != 0 && (tile_bits < 10 || tile_bits > 13))
+        return fail(SV_EINVAL, "tile_bits must be 0 (off) or in [10, 13]");
+    s->block_bits = tile_bits;
+    return SV_OK;
 }
 
 int sv_set_timing(sv_state* s, int enable) {

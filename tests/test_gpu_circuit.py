@@ -69,6 +69,25 @@ def test_virtual_shards_match_oracle(world, F):
     assert st["n_exchanges"] >= 1
 
 
+@pytest.mark.parametrize("bits", [0, 10, 12, 13])
+@pytest.mark.parametrize("F", [1, 2, 4])
+def test_blocked_passes_match_oracle(bits, F):
+    """Cache-blocked passes (sv_set_blocking) against the oracle."""
+    n, d = 20, 14
+    gates = W.rqc(n, d, seed=F + bits)
+    h = sv.sv_create(n)
+    try:
+        sv.sv_set_blocking(h, bits)
+        c = sv.sv_circuit_create(h, gates, F)
+        sv.sv_circuit_run_device(h, c)
+        sv.sv_synchronize(h)
+        got = sv.sv_get_state(h, n)
+        sv.sv_circuit_destroy(c)
+    finally:
+        sv.sv_destroy(h)
+    _check(n, d, got, ref_c.run(n, gates))
+
+
 def test_amplitudes_match_state():
     n = 20
     gates = W.rqc(n, 12)
