@@ -60,6 +60,7 @@ def parse():
     ap.add_argument("--seed", type=int, default=2023)
     ap.add_argument("--samples", type=int, default=N_SAMPLES)
     ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
+    ap.add_argument("--precision", type=int, default=32, choices=[32, 64], help="complex64 (32) or complex128 (64) state")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
@@ -199,8 +200,10 @@ def run_ours(args):
     n = args.qubits or (30 if world == 1 else 30 + (world.bit_length() - 1))
     gates = W.rqc(n, args.depth, args.seed)
     stream = torch.cuda.Stream()
+    fp64 = args.precision == 64
+    elem = 16 if fp64 else 8
     if world == 1:
-        h = sv.sv_create_ex(n, cuda_stream=stream.cuda_stream)
+        h = sv.sv_create_ex(n, cuda_stream=stream.cuda_stream, precision=1 if fp64 else 0)
     else:
         h = sv.sv_create_ex(n, world=world, rank=rank, virtual_shards=False, cuda_stream=stream.cuda_stream)
         blob = sv.sv_ipc_handle(h)
@@ -296,7 +299,7 @@ def run_ours(args):
     peak, peak_src = load_peaks()
     launches_apply = n_high + n_low
     avg_launch = t_apply / max(launches_apply, 1)
-    bytes_per_launch = 16 * (1 << (n - (world.bit_length() - 1)))
+    bytes_per_launch = 2 * elem * (1 << (n - (world.bit_length() - 1)))
     achieved = bytes_per_launch / avg_launch / 1e9 if avg_launch > 0 else None
     frac = achieved / peak if achieved else None
     cpu = None
@@ -309,7 +312,7 @@ def run_ours(args):
     if rank == 0:
         sv_fused = cst["n_fused"]
         out = {
-            "metric": f"rqc_circuit_time_{n}q_d{args.depth}_f{args.max_fused}",
+            "metric": f"rqc_circuit_time_{n}q_d{args.depth}_f{args.max_fused}" + ("_c128" if fp64 else ""),
             "value": ms / 1e3,
             "unit": "s",
             "n_gpus": world,
@@ -319,7 +322,7 @@ def run_ours(args):
             "higher_is_better": False,
             "scaling": "weak",
             "vs_baseline": None,
-            "dtype": "f32",
+            "dtype": "f64" if fp64 else "f32",
             "data": "synthetic",
             "config": {
                 "workload": f"rqc_{n}q_d{args.depth}_f{args.max_fused}",
@@ -327,15 +330,15 @@ def run_ours(args):
                 "gates": len(gates), "n_fused": sv_fused, "fused_hist": cst["fused_hist"],
                 "samples_per_step": args.samples,
                 "step": "sv_reset + all fused-gate applies + sv_sample_device(1e6)",
-                "l2": f"inputs larger than L2 (state {8 << n >> 30} GiB per circuit)",
+                "l2": f"inputs larger than L2 (state {elem << n >> 30} GiB per circuit)",
                 "parallelism": "single GPU" if world == 1 else f"sharded x{world} (P2P exchange)",
                 "apply_ms_per_step": 1e3 * t_apply / args.steps,
                 "apply_high_ms_per_step": 1e3 * t_high / args.steps,
                 "apply_low_ms_per_step": 1e3 * t_low / args.steps,
                 "exchange_ms_per_step": 1e3 * t_exch / args.steps,
                 "other_ms_per_step": 1e3 * t_other / args.steps,
-                "apply_gbs_high": (16 << (n - (world.bit_length() - 1))) * n_high / t_high / 1e9 if t_high else None,
-                "apply_gbs_low": (16 << (n - (world.bit_length() - 1))) * n_low / t_low / 1e9 if t_low else None,
+                "apply_gbs_high": bytes_per_launch * n_high / t_high / 1e9 if t_high else None,
+                "apply_gbs_low": bytes_per_launch * n_low / t_low / 1e9 if t_low else None,
                 "apply_tflops": flops / t_apply / 1e12 if t_apply else None,
                 "fuse_plan_upload_s": cst["t_fuse_s"] + cst["t_plan_s"] + cst["t_upload_s"],
                 "apply_launches_per_step": launches_apply // max(args.steps, 1),

@@ -1,4 +1,3 @@
 python -c "import __graft_entry__ as g; g.build()" > /dev/null
-timeout 900 python -m pytest tests/test_gpu_circuit.py -q -x -k "blocked" 2>&1 | grep -E "Error|error|assert" | head -10
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:apply_pass -s 3 -c 1 -o gpurun_out/prof_pass python bench.py --steps 1 --warmup 1 --no-cpu-baseline --max-fused 3 --block-bits 12 --samples 1000 > /dev/null 2>&1
-ls gpurun_out/
+timeout 900 python -m pytest tests -q -m gpu 2>&1 | tail -6
+for F in 2 4 5; do timeout 300 python bench.py --steps 3 --warmup 2 --no-cpu-baseline --max-fused $F --precision 64 --samples 100000 | cut -c1-250; done

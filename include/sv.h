@@ -114,6 +114,9 @@ typedef struct {
     void* dev_buf;           /* optional caller-owned device buffer for the state, or NULL */
     size_t buf_bytes;        /* size of dev_buf: >= 8 * 2^n / (world if multi-process)    */
     void* cuda_stream;       /* optional cudaStream_t; NULL = library-owned stream        */
+    int32_t precision;       /* 0: complex64 (fp32, default); 1: complex128 (fp64, NEXT-1;
+                                PAPER.md L191 Fig. 8) -- single shard, fused k <= 5      */
+    int32_t reserved_;
 } sv_config;
 
 /* ---- lifetime ------------------------------------------------------------- */
@@ -132,6 +135,10 @@ int sv_reset(sv_state* s);
  * Asynchronous: the matrix is staged before return. */
 int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix);
 
+/* Same with a complex128 matrix (no rounding on complex128 states; rounded to
+ * complex64 on complex64 states). */
+int sv_apply_fused_c128(sv_state* s, int k, const int32_t* qubits, const sv_c128* matrix);
+
 /* Fuse (max_fused in [0,6]; 0 = no fusion), plan (sharded), upload and apply a
  * whole circuit of 1-2 qubit gates, synchronising before return.  stats may be
  * NULL. Equivalent to sv_circuit_create + sv_circuit_run + sv_circuit_destroy. */
@@ -148,10 +155,14 @@ int sv_circuit_destroy(sv_circuit* c);
 /* Read `count` amplitudes at LOGICAL indices idx[] into out[] (host). */
 int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out);
 
+/* complex128 output (exact on complex128 states). */
+int sv_amplitudes_c128(sv_state* s, const uint64_t* idx, size_t count, sv_c128* out);
+
 /* Draw n_samples basis states (LOGICAL indices) with the integer fixed-point
  * sampler: bit-identical for a given complex64 state and
  * seed under any parallel decomposition.  SV_EINVAL if the total weight is 0
- * or sum |c|^2 >= 3.99.  out[] is host memory of n_samples uint64. */
+ * or sum |c|^2 >= 3.99.  out[] is host memory of n_samples uint64.  On
+ * complex128 states p = fl(fl(re^2) + fl(im^2)) (reading R5). */
 int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out);
 /* Device form: writes n_samples uint64 into device memory dev_out
  * (asynchronous; the bench's device step). */
@@ -162,6 +173,9 @@ int sv_sample_device(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* dev
  * multi-process mode each rank passes/receives the FULL vector. */
 int sv_set_state(sv_state* s, const sv_c64* host, size_t count);
 int sv_get_state(sv_state* s, sv_c64* host, size_t count);
+/* complex128 forms (converting on complex64 states). */
+int sv_set_state_c128(sv_state* s, const sv_c128* host, size_t count);
+int sv_get_state_c128(sv_state* s, sv_c128* host, size_t count);
 /* Device pointer of shard `shard` (virtual mode) / of this rank's shard. */
 int sv_device_ptr(sv_state* s, int shard, void** out);
 

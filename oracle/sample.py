@@ -22,19 +22,26 @@ from workloads.rqc import splitmix64_nth
 TWO62 = float(2 ** 62)
 
 
-def weights(psi_c64: np.ndarray) -> np.ndarray:
-    """w_i = floor(p_i * 2^62) with p_i computed in fp64 from complex64 parts."""
-    psi = np.asarray(psi_c64, dtype=np.complex64)
+def weights(psi: np.ndarray) -> np.ndarray:
+    """w_i = floor(p_i * 2^62) with p_i computed in fp64.
+
+    complex64 input: both products are exact in fp64, one rounding in the sum
+    (S5).  complex128 input (NEXT-1, reading R5): p = fl(fl(re^2) + fl(im^2)),
+    three separately rounded operations (numpy ufuncs do not contract)."""
+    psi = np.asarray(psi)
+    if psi.dtype != np.complex128:
+        psi = psi.astype(np.complex64)
     re = psi.real.astype(np.float64)
     im = psi.imag.astype(np.float64)
     p = re * re + im * im
     return np.floor(p * TWO62).astype(np.uint64)
 
 
-def sample(psi_c64: np.ndarray, seed: int, n_samples: int):
-    """S5 on a complex64 state in logical order.  Returns (indices uint64, T)."""
-    w = weights(psi_c64)
-    psi = np.asarray(psi_c64, dtype=np.complex64)
+def sample(psi_in: np.ndarray, seed: int, n_samples: int):
+    """S5 on a complex64 (or complex128) state in logical order.
+    Returns (indices uint64, T)."""
+    w = weights(psi_in)
+    psi = np.asarray(psi_in)
     psum = float(np.sum(psi.real.astype(np.float64) ** 2 + psi.imag.astype(np.float64) ** 2))
     T = int(w.sum(dtype=np.uint64)) if w.size else 0
     if T == 0 or psum >= 3.99:

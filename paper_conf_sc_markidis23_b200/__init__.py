@@ -79,6 +79,8 @@ class sv_config(ctypes.Structure):
         ("dev_buf", ctypes.c_void_p),
         ("buf_bytes", ctypes.c_size_t),
         ("cuda_stream", ctypes.c_void_p),
+        ("precision", ctypes.c_int32),
+        ("reserved_", ctypes.c_int32),
     ]
 
 
@@ -94,16 +96,20 @@ _SIGS = {
     "sv_destroy": ([_vp], ctypes.c_int),
     "sv_reset": ([_vp], ctypes.c_int),
     "sv_apply_fused": ([_vp, ctypes.c_int, _i32p, _vp], ctypes.c_int),
+    "sv_apply_fused_c128": ([_vp, ctypes.c_int, _i32p, _vp], ctypes.c_int),
     "sv_run_circuit": ([_vp, _vp, _sz, ctypes.c_int, ctypes.POINTER(sv_stats)], ctypes.c_int),
     "sv_circuit_create": ([_vp, _vp, _sz, ctypes.c_int, ctypes.POINTER(_vp)], ctypes.c_int),
     "sv_circuit_run_device": ([_vp, _vp], ctypes.c_int),
     "sv_circuit_stats": ([_vp, ctypes.POINTER(sv_stats)], ctypes.c_int),
     "sv_circuit_destroy": ([_vp], ctypes.c_int),
     "sv_amplitudes": ([_vp, _u64p, _sz, _vp], ctypes.c_int),
+    "sv_amplitudes_c128": ([_vp, _u64p, _sz, _vp], ctypes.c_int),
     "sv_sample": ([_vp, ctypes.c_uint64, _sz, _u64p], ctypes.c_int),
     "sv_sample_device": ([_vp, ctypes.c_uint64, _sz, _vp], ctypes.c_int),
     "sv_set_state": ([_vp, _vp, _sz], ctypes.c_int),
     "sv_get_state": ([_vp, _vp, _sz], ctypes.c_int),
+    "sv_set_state_c128": ([_vp, _vp, _sz], ctypes.c_int),
+    "sv_get_state_c128": ([_vp, _vp, _sz], ctypes.c_int),
     "sv_device_ptr": ([_vp, ctypes.c_int, ctypes.POINTER(_vp)], ctypes.c_int),
     "sv_fusion_plan": ([_vp, _sz, ctypes.c_int, _i32p, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_fused_matrix": ([_vp, _sz, ctypes.c_int, _sz, _vp, _sz], ctypes.c_int),
@@ -170,9 +176,10 @@ def sv_create(n_qubits: int) -> int:
 
 def sv_create_ex(n_qubits: int, world: int = 1, rank: int = 0, virtual_shards: bool = True,
                  exchange_vmin: int = -1, device: int = -1, dev_buf: int = 0, buf_bytes: int = 0,
-                 cuda_stream: int = 0) -> int:
+                 cuda_stream: int = 0, precision: int = 0) -> int:
+    """precision: 0 = complex64 (default), 1 = complex128."""
     cfg = sv_config(n_qubits, world, rank, 1 if virtual_shards else 0, exchange_vmin, device,
-                    dev_buf or None, buf_bytes, cuda_stream or None)
+                    dev_buf or None, buf_bytes, cuda_stream or None, precision, 0)
     h = _vp()
     _check(lib().sv_create_ex(ctypes.byref(cfg), ctypes.byref(h)), "sv_create_ex")
     return h.value
@@ -194,6 +201,14 @@ def sv_apply_fused(h: int, qubits: Sequence[int], matrix) -> None:
     if m.size != (1 << (2 * k)):
         raise ValueError("matrix must be 2^k x 2^k")
     _check(lib().sv_apply_fused(h, k, q.ctypes.data_as(_i32p), _ptr(m)), "sv_apply_fused")
+
+
+def sv_apply_fused_c128(h: int, qubits: Sequence[int], matrix) -> None:
+    q = np.ascontiguousarray(qubits, dtype=np.int32)
+    m = np.ascontiguousarray(matrix, dtype=np.complex128)
+    if m.size != (1 << (2 * q.size)):
+        raise ValueError("matrix must be 2^k x 2^k")
+    _check(lib().sv_apply_fused_c128(h, q.size, q.ctypes.data_as(_i32p), _ptr(m)), "sv_apply_fused_c128")
 
 
 def sv_run_circuit(h: int, gates, max_fused: int) -> dict:
@@ -231,6 +246,13 @@ def sv_amplitudes(h: int, idx) -> np.ndarray:
     return out
 
 
+def sv_amplitudes_c128(h: int, idx) -> np.ndarray:
+    i = np.ascontiguousarray(idx, dtype=np.uint64)
+    out = np.empty(i.size, dtype=np.complex128)
+    _check(lib().sv_amplitudes_c128(h, i.ctypes.data_as(_u64p), i.size, _ptr(out)), "sv_amplitudes_c128")
+    return out
+
+
 def sv_sample(h: int, seed: int, n_samples: int) -> np.ndarray:
     out = np.empty(n_samples, dtype=np.uint64)
     _check(lib().sv_sample(h, seed, n_samples, out.ctypes.data_as(_u64p)), "sv_sample")
@@ -249,6 +271,17 @@ def sv_set_state(h: int, psi) -> None:
 def sv_get_state(h: int, n_qubits: int) -> np.ndarray:
     out = np.empty(1 << n_qubits, dtype=np.complex64)
     _check(lib().sv_get_state(h, _ptr(out), out.size), "sv_get_state")
+    return out
+
+
+def sv_set_state_c128(h: int, psi) -> None:
+    a = np.ascontiguousarray(psi, dtype=np.complex128)
+    _check(lib().sv_set_state_c128(h, _ptr(a), a.size), "sv_set_state_c128")
+
+
+def sv_get_state_c128(h: int, n_qubits: int) -> np.ndarray:
+    out = np.empty(1 << n_qubits, dtype=np.complex128)
+    _check(lib().sv_get_state_c128(h, _ptr(out), out.size), "sv_get_state_c128")
     return out
 
 

@@ -38,6 +38,19 @@ void plan_apply(int n_local, ApplyDesc& d);
 // shard has at least 2^13 amplitudes.
 bool tc_supported(int n_local, const ApplyDesc& d);
 
+// ---- complex128 states (apply64.cu, NEXT-1) --------------------------------
+struct Apply64Desc {
+    int k = 0;
+    int q[SV_MAX_FUSED] = {0};          // ascending
+    std::vector<cd> m;                  // 2^k x 2^k row-major over ascending q (fp64)
+    const double* dev_planes = nullptr; // planes P, S, Q on the device (k = 6 and tiny states)
+    const void* small_scratch = nullptr;  // device int[6] with q (tiny states)
+};
+void pack_planes64(const Apply64Desc& d, double* out);  // 3 * 4^k doubles
+cudaError_t launch_apply64(double2* psi, int n, const Apply64Desc& d, cudaStream_t st);
+cudaError_t launch_reset64(double2* psi, uint64_t n_amps, bool one, cudaStream_t st);
+cudaError_t launch_gather64(const double2* psi, const uint64_t* phys, uint64_t count, double2* out, cudaStream_t st);
+
 // Whole circuit in one CTA with the state in shared memory (n <= 13).
 constexpr int kSmallCircuitMaxQubits = 13;
 struct SmallGateDesc {
@@ -81,7 +94,7 @@ cudaError_t launch_gather(const float2* psi, const uint64_t* phys, const int32_t
 // ---- sampling (S5) ----------------------------------------------------------
 constexpr int kSampleBinBits = 5;  // 32 amplitudes per fine bin
 // bins[b] = sum over the 32 amplitudes of bin b of floor(p * 2^62)
-cudaError_t launch_bin_weights(const float2* psi, uint64_t n_amps, uint64_t* bins, cudaStream_t st);
+cudaError_t launch_bin_weights(const void* psi, bool fp64, uint64_t n_amps, uint64_t* bins, cudaStream_t st);
 // inclusive prefix sum in place over `count` uint64 (scratch: >= scan_scratch_elems(count))
 size_t scan_scratch_elems(uint64_t count);
 cudaError_t launch_inclusive_scan(uint64_t* data, uint64_t count, uint64_t* scratch, cudaStream_t st);
@@ -89,9 +102,10 @@ cudaError_t launch_inclusive_scan(uint64_t* data, uint64_t count, uint64_t* scra
 // with T = *total_dev (+ global offset); samples whose t falls into this
 // shard's range [range_lo, range_lo + local_total) are written as
 // logical index = index_base + local index.  Others untouched.
-cudaError_t launch_sample_resolve(const float2* psi, uint64_t n_amps, const uint64_t* cum_bins, uint64_t n_bins,
-                                  const uint64_t* range_lo_dev, const uint64_t* total_dev, uint64_t seed,
-                                  uint64_t n_samples, uint64_t index_base, uint64_t* out, cudaStream_t st);
+cudaError_t launch_sample_resolve(const void* psi, bool fp64, uint64_t n_amps, const uint64_t* cum_bins,
+                                  uint64_t n_bins, const uint64_t* range_lo_dev, const uint64_t* total_dev,
+                                  uint64_t seed, uint64_t n_samples, uint64_t index_base, uint64_t* out,
+                                  cudaStream_t st);
 
 // offsets of shard totals in LOGICAL shard order: lo[d] = sum of totals of
 // shards whose logical index sigma[d'] < sigma[d]; *total = sum of all.

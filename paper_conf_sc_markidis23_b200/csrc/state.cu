@@ -57,14 +57,33 @@ __device__ __forceinline__ uint64_t weight(float2 a) {
     return __double2ull_rz(p * 0x1p62);           // floor for p >= 0 (exact scaling)
 }
 
+// complex128 states: p = fl(fl(re*re) + fl(im*im)) with explicit roundings
+// (no FMA contraction), the reading R5 shared with oracle/sample.py.
+__device__ __forceinline__ uint64_t weight(double2 a) {
+    const double p = __dadd_rn(__dmul_rn(a.x, a.x), __dmul_rn(a.y, a.y));
+    return __double2ull_rz(p * 0x1p62);
+}
+
+__device__ __forceinline__ void load4w(const float2* psi, uint64_t i0, uint64_t& w) {
+    const float4 u = __ldcs(reinterpret_cast<const float4*>(psi + i0));
+    const float4 v = __ldcs(reinterpret_cast<const float4*>(psi + i0 + 2));
+    w = weight(make_float2(u.x, u.y)) + weight(make_float2(u.z, u.w)) + weight(make_float2(v.x, v.y)) +
+        weight(make_float2(v.z, v.w));
+}
+__device__ __forceinline__ void load4w(const double2* psi, uint64_t i0, uint64_t& w) {
+    w = weight(__ldcs(psi + i0)) + weight(__ldcs(psi + i0 + 1)) + weight(__ldcs(psi + i0 + 2)) +
+        weight(__ldcs(psi + i0 + 3));
+}
+
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
     return v;
 }
 
-// 8 lanes per 32-amplitude bin, 4 amplitudes (two 16 B loads) per lane.
-__global__ void bin_weights_kernel(const float2* __restrict__ psi, uint64_t n_amps, uint64_t* __restrict__ bins,
+// 8 lanes per 32-amplitude bin, 4 amplitudes per lane.
+template <class E>
+__global__ void bin_weights_kernel(const E* __restrict__ psi, uint64_t n_amps, uint64_t* __restrict__ bins,
                                    uint64_t n_bins) {
     const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;  // multiple of 32
@@ -76,10 +95,7 @@ __global__ void bin_weights_kernel(const float2* __restrict__ psi, uint64_t n_am
         uint64_t w = 0;
         const uint64_t i0 = (b << kSampleBinBits) + 4 * sub;
         if (b < full_bins) {
-            const float4 u = __ldcs(reinterpret_cast<const float4*>(psi + i0));
-            const float4 v = __ldcs(reinterpret_cast<const float4*>(psi + i0 + 2));
-            w = weight(make_float2(u.x, u.y)) + weight(make_float2(u.z, u.w)) + weight(make_float2(v.x, v.y)) +
-                weight(make_float2(v.z, v.w));
+            load4w(psi, i0, w);
         } else if (b < n_bins) {
             for (int j = 0; j < 4; ++j)
                 if (i0 + j < n_amps) w += weight(psi[i0 + j]);
@@ -162,7 +178,8 @@ __device__ __forceinline__ uint64_t splitmix64_at(uint64_t seed, uint64_t s) {
     return z ^ (z >> 31);
 }
 
-__global__ void sample_resolve_kernel(const float2* __restrict__ psi, const uint64_t* __restrict__ cum,
+template <class E>
+__global__ void sample_resolve_kernel(const E* __restrict__ psi, const uint64_t* __restrict__ cum,
                                       uint64_t n_bins, const uint64_t* range_lo_dev, const uint64_t* total_dev,
                                       uint64_t seed, uint64_t n_samples, uint64_t index_base, uint64_t n_amps,
                                       uint64_t* out) {
@@ -272,10 +289,15 @@ cudaError_t launch_gather(const float2* psi, const uint64_t* phys, const int32_t
     return cudaGetLastError();
 }
 
-cudaError_t launch_bin_weights(const float2* psi, uint64_t n_amps, uint64_t* bins, cudaStream_t st) {
+cudaError_t launch_bin_weights(const void* psi, bool fp64, uint64_t n_amps, uint64_t* bins, cudaStream_t st) {
     const uint64_t n_bins = (n_amps + (1u << kSampleBinBits) - 1) >> kSampleBinBits;
-    // whole warps per loop trip (the 8-lane shuffles need all lanes): round the grid to warps
-    bin_weights_kernel<<<grid_cap(n_bins * 8, 256, 16), 256, 0, st>>>(psi, n_amps, bins, n_bins);
+    // whole warps per loop trip (the 8-lane shuffles need all lanes)
+    if (fp64)
+        bin_weights_kernel<double2><<<grid_cap(n_bins * 8, 256, 16), 256, 0, st>>>((const double2*)psi, n_amps, bins,
+                                                                                     n_bins);
+    else
+        bin_weights_kernel<float2><<<grid_cap(n_bins * 8, 256, 16), 256, 0, st>>>((const float2*)psi, n_amps, bins,
+                                                                                    n_bins);
     return cudaGetLastError();
 }
 
@@ -304,12 +326,17 @@ cudaError_t launch_inclusive_scan(uint64_t* data, uint64_t count, uint64_t* scra
     return cudaGetLastError();
 }
 
-cudaError_t launch_sample_resolve(const float2* psi, uint64_t n_amps, const uint64_t* cum_bins, uint64_t n_bins,
-                                  const uint64_t* range_lo_dev, const uint64_t* total_dev, uint64_t seed,
-                                  uint64_t n_samples, uint64_t index_base, uint64_t* out, cudaStream_t st) {
+cudaError_t launch_sample_resolve(const void* psi, bool fp64, uint64_t n_amps, const uint64_t* cum_bins,
+                                  uint64_t n_bins, const uint64_t* range_lo_dev, const uint64_t* total_dev,
+                                  uint64_t seed, uint64_t n_samples, uint64_t index_base, uint64_t* out,
+                                  cudaStream_t st) {
     if (n_samples == 0) return cudaSuccess;
-    sample_resolve_kernel<<<(unsigned)((n_samples + 255) / 256), 256, 0, st>>>(
-        psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out);
+    if (fp64)
+        sample_resolve_kernel<double2><<<(unsigned)((n_samples + 255) / 256), 256, 0, st>>>(
+            (const double2*)psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out);
+    else
+        sample_resolve_kernel<float2><<<(unsigned)((n_samples + 255) / 256), 256, 0, st>>>(
+            (const float2*)psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out);
     return cudaGetLastError();
 }
 

@@ -60,6 +60,10 @@ struct sv_state {
     int device = 0;
     int vmin = 5;
     int block_bits = 0;       // cache-blocked passes: tile qubits (0 = off; opt-in)
+    bool fp64 = false;        // complex128 amplitudes (NEXT-1)
+    size_t elem = 8;          // bytes per amplitude
+    double* planes64 = nullptr;   // fp64 scratch: planes of one gate (sv_apply_fused on fp64 states)
+    int* q64 = nullptr;           // fp64 scratch: qubits of one gate (tiny states)
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     std::vector<float2*> shard;        // shard pointers (local or peer-mapped)
@@ -113,12 +117,15 @@ struct sv_circuit {
         Event::Type type;
         bool block = false;                   // APPLY of a cache-blocked pass (pass below)
         ApplyDesc apply;
+        Apply64Desc a64;  // complex128 states
         PassDesc pass;
         ExchangeDesc exch;
         std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
     };
     std::vector<Step> steps;
     float2* dev_mats = nullptr;
+    double* planes64 = nullptr;  // complex128 states: planes of every gate
+    int* q64 = nullptr;          // complex128 states: qubits of every gate (int[6] each)
     // small states (n <= 13, unsharded): whole circuit in one CTA (small.cu)
     bool small = false;
     int n_small = 0;
@@ -408,7 +415,7 @@ void destroy_state(sv_state* s) {
     for (void* p : {(void*)s->shard_dev, (void*)s->bins, (void*)s->scan_scratch, (void*)s->misc,
                     (void*)s->totals_ptr_dev, (void*)s->sigma_dev, (void*)s->kmat, (void*)s->ctrl, (void*)s->xfer,
                     (void*)s->flags_dev, (void*)s->xfer_dev, (void*)s->idx_dev, (void*)s->amp_dev,
-                    (void*)s->samp_dev})
+                    (void*)s->samp_dev, (void*)s->planes64, (void*)s->q64})
         if (p) cudaFree(p);
     for (auto e : s->ev_pool) cudaEventDestroy(e);
     if (s->own_stream && s->stream) cudaStreamDestroy(s->stream);
@@ -453,7 +460,10 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
         return fail(SV_EUNSUPPORTED, "shard too small: need n - log2(world) >= 8");
     const bool virt = world == 1 || cfg->virtual_shards != 0;
     if (!virt && (cfg->rank < 0 || cfg->rank >= world)) return fail(SV_EINVAL, "rank out of range");
-    const size_t shard_bytes = (size_t)8 << l;
+    if (cfg->precision != 0 && cfg->precision != 1) return fail(SV_EINVAL, "precision must be 0 (complex64) or 1 (complex128)");
+    const bool fp64 = cfg->precision == 1;
+    if (fp64 && world > 1) return fail(SV_EUNSUPPORTED, "complex128 states are single-shard in this version");
+    const size_t shard_bytes = (size_t)(fp64 ? 16 : 8) << l;
     const size_t need_bytes = shard_bytes * (virt ? world : 1);
     if (cfg->dev_buf && cfg->buf_bytes < need_bytes) return fail(SV_EINVAL, "buf_bytes too small for the state");
     if (cfg->dev_buf && !virt) return fail(SV_EUNSUPPORTED, "multi-process mode owns its buffers (dev_buf must be NULL)");
@@ -466,6 +476,8 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
     s->rank = virt ? 0 : cfg->rank;
     s->virt = virt;
     s->vmin = cfg->exchange_vmin < 0 ? 5 : cfg->exchange_vmin;
+    s->fp64 = fp64;
+    s->elem = fp64 ? 16 : 8;
     if (cfg->device >= 0) CK(nullptr, cudaSetDevice(cfg->device));
     CK(nullptr, cudaGetDevice(&s->device));
     if (cfg->cuda_stream) {
@@ -502,6 +514,11 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
     CK(nullptr, cudaMalloc(&s->shard_dev, sizeof(float2*) * world));
     int rc = alloc_scratch(s.get());
     if (rc) return rc;
+    if (fp64) {
+        cudaError_t e = cudaMalloc(&s->planes64, 3 * 4096 * sizeof(double));
+        if (e == cudaSuccess) e = cudaMalloc(&s->q64, 8 * sizeof(int));
+        if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(fp64 scratch)");
+    }
     rc = upload_shard_table(s.get());
     if (rc) return rc;
     s->pos.resize(n);
@@ -526,18 +543,41 @@ int sv_reset(sv_state* s) {
     for (int d = 0; d < s->local_shards(); ++d) {
         const int shard = s->virt ? d : s->rank;
         float2* psi = s->shard[shard];
-        int rc = launch(s, LaunchClass::OTHER,
-                        [&] { return launch_reset(psi, s->local_amps(), shard == 0, s->stream); });
+        int rc = launch(s, LaunchClass::OTHER, [&] {
+            return s->fp64 ? launch_reset64(reinterpret_cast<double2*>(psi), s->local_amps(), shard == 0, s->stream)
+                           : launch_reset(psi, s->local_amps(), shard == 0, s->stream);
+        });
         if (rc) return rc;
     }
     return SV_OK;
 }
+
+static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::vector<cd>& M);
 
 int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix) {
     int rc = check_state(s);
     if (rc) return rc;
     if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
     if (!qubits || !matrix) return fail(SV_EINVAL, "qubits/matrix is NULL");
+    const int D = 1 << k;
+    std::vector<cd> M((size_t)D * D);
+    for (int i = 0; i < D * D; ++i) M[i] = cd(matrix[i].re, matrix[i].im);
+    return apply_matrix(s, k, qubits, M);
+}
+
+int sv_apply_fused_c128(sv_state* s, int k, const int32_t* qubits, const sv_c128* matrix) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
+    if (!qubits || !matrix) return fail(SV_EINVAL, "qubits/matrix is NULL");
+    const int D = 1 << k;
+    std::vector<cd> M((size_t)D * D);
+    for (int i = 0; i < D * D; ++i) M[i] = cd(matrix[i].re, matrix[i].im);
+    return apply_matrix(s, k, qubits, M);
+}
+
+static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::vector<cd>& Min) {
+    int rc = SV_OK;
     uint64_t mask = 0;
     for (int b = 0; b < k; ++b) {
         if (qubits[b] < 0 || qubits[b] >= s->n) return fail(SV_EINVAL, "qubit out of range");
@@ -545,10 +585,32 @@ int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matr
         mask |= 1ull << qubits[b];
     }
     if (s->g > 0 && k > s->l - 1) return fail(SV_EUNSUPPORTED, "gate wider than a shard allows");
-    const int D = 1 << k;
-    std::vector<cd> M((size_t)D * D);
-    for (int i = 0; i < D * D; ++i) M[i] = cd(matrix[i].re, matrix[i].im);
+    std::vector<cd> M = Min;
     std::vector<int> q(qubits, qubits + k);
+    if (s->fp64 && k > 5) return fail(SV_EUNSUPPORTED, "complex128 states support fused gates with k <= 5");
+    if (s->fp64) {
+        Apply64Desc d;
+        d.k = k;
+        std::vector<cd> Ms(M.size());
+        sort_matrix_qubits<cd>(k, q.data(), M.data(), d.q, Ms.data());
+        d.m = Ms;
+        std::vector<double> planes(3 * M.size());
+        pack_planes64(d, planes.data());
+        CK(s, cudaStreamSynchronize(s->stream));  // the previous launch may still read the scratch
+        CK(s, cudaMemcpyAsync(s->planes64, planes.data(), planes.size() * sizeof(double), cudaMemcpyHostToDevice,
+                              s->stream));
+        CK(s, cudaMemcpyAsync(s->q64, d.q, sizeof(int) * SV_MAX_FUSED, cudaMemcpyHostToDevice, s->stream));
+        CK(s, cudaStreamSynchronize(s->stream));
+        d.dev_planes = s->planes64;
+        d.small_scratch = s->q64;
+        rc = launch(s, LaunchClass::HIGH, [&] {
+            return launch_apply64(reinterpret_cast<double2*>(s->shard[0]), s->l, d, s->stream);
+        });
+        if (rc) return rc;
+        s->stats.bytes_apply += 32ull << s->l;
+        s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
+        return SV_OK;
+    }
     // sharded: bring global qubits local (one S4 step for this gate alone)
     if (s->g > 0) {
         std::vector<std::vector<int>> fq(1, q);
@@ -674,6 +736,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     rc = validate_gates(gates, n_gates, s->n);
     if (rc) return rc;
     if (s->g > 0 && std::max(max_fused, 2) > s->l - 1) return fail(SV_EUNSUPPORTED, "fused gates wider than a shard allows");
+    if (s->fp64 && max_fused > 5) return fail(SV_EUNSUPPORTED, "complex128 states support max_fused <= 5");
     std::unique_ptr<sv_circuit> c(new sv_circuit());
     c->owner = s;
     const double t0 = now_s();
@@ -708,7 +771,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     // with "local" = the tile's T slots cuts the fused list into passes; a
     // remap only changes the tile's qubit set S (no data movement).
     const int T = s->block_bits;
-    bool blocked = s->g == 0 && T >= 10 && s->n >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
+    bool blocked = !s->fp64 && s->g == 0 && T >= 10 && s->n >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
                    max_fused >= 1;
     std::vector<PassDesc> passes;
     if (blocked) {
@@ -783,6 +846,42 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         *out = c.release();
         return SV_OK;
     }
+    if (s->fp64) {
+        // complex128: one apply64 launch per fused gate; all planes and qubit
+        // lists uploaded once (row a4)
+        std::vector<double> planes;
+        std::vector<int> qs;
+        std::vector<size_t> poff;
+        for (auto& e : ev) {
+            sv_circuit::Step st;
+            st.type = Event::APPLY;
+            const FusedGate& f = plan[e.fused];
+            st.a64.k = f.k;
+            for (int b = 0; b < f.k; ++b) st.a64.q[b] = f.q[b];
+            st.a64.m = f.M;  // fp64, ascending qubits: no rounding to complex64
+            poff.push_back(planes.size());
+            planes.resize(planes.size() + 3 * f.M.size());
+            pack_planes64(st.a64, planes.data() + poff.back());
+            for (int b = 0; b < SV_MAX_FUSED; ++b) qs.push_back(st.a64.q[b]);
+            c->steps.push_back(std::move(st));
+        }
+        if (!planes.empty()) {
+            cudaError_t e = cudaMalloc(&c->planes64, planes.size() * sizeof(double));
+            if (e == cudaSuccess) e = cudaMalloc(&c->q64, qs.size() * sizeof(int));
+            if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(fp64 circuit)");
+            CK(s, cudaMemcpyAsync(c->planes64, planes.data(), planes.size() * sizeof(double), cudaMemcpyHostToDevice,
+                                  s->stream));
+            CK(s, cudaMemcpyAsync(c->q64, qs.data(), qs.size() * sizeof(int), cudaMemcpyHostToDevice, s->stream));
+            CK(s, cudaStreamSynchronize(s->stream));
+            for (size_t i = 0; i < c->steps.size(); ++i) {
+                c->steps[i].a64.dev_planes = c->planes64 + poff[i];
+                c->steps[i].a64.small_scratch = c->q64 + SV_MAX_FUSED * i;
+            }
+        }
+        c->stats.t_upload_s = now_s() - t2;
+        *out = c.release();
+        return SV_OK;
+    }
     // lower events to launch descriptors
     size_t n6 = 0;
     for (auto& e : ev) {
@@ -815,7 +914,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
                               s->stream));
         CK(s, cudaStreamSynchronize(s->stream));
     }
-    if (s->g == 0 && s->n <= kSmallCircuitMaxQubits) {
+    if (s->g == 0 && s->n <= kSmallCircuitMaxQubits && !s->fp64) {
         std::vector<SmallGateDesc> gd;
         std::vector<float2> mats;
         for (auto& st : c->steps) {
@@ -870,6 +969,18 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
         s->pos = c->pos_out;
         return SV_OK;
     }
+    if (s->fp64) {
+        for (auto& st : c->steps) {
+            rc = launch(s, LaunchClass::HIGH, [&] {
+                return launch_apply64(reinterpret_cast<double2*>(s->shard[0]), s->l, st.a64, s->stream);
+            });
+            if (rc) return rc;
+            s->stats.bytes_apply += 32ull << s->l;
+            s->stats.flops_apply += (uint64_t)((8 << st.a64.k) - 2) << s->l;
+        }
+        s->pos = c->pos_out;
+        return SV_OK;
+    }
     for (auto& st : c->steps) {
         if (st.block) {
             rc = launch(s, LaunchClass::HIGH, [&] { return launch_pass(s->shard[0], s->l, st.pass, s->stream); });
@@ -902,8 +1013,10 @@ int sv_circuit_stats(const sv_circuit* c, sv_stats* st) {
 
 int sv_circuit_destroy(sv_circuit* c) {
     if (!c) return fail(SV_EINVAL, "circuit is NULL");
-    if (c->dev_mats || c->small_gates || c->small_mats) {
+    if (c->dev_mats || c->small_gates || c->small_mats || c->planes64 || c->q64) {
         if (c->owner && c->owner->stream) cudaStreamSynchronize(c->owner->stream);
+        if (c->planes64) cudaFree(c->planes64);
+        if (c->q64) cudaFree(c->q64);
         if (c->dev_mats) cudaFree(c->dev_mats);
         if (c->small_gates) cudaFree(c->small_gates);
         if (c->small_mats) cudaFree(c->small_mats);
@@ -927,11 +1040,50 @@ int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fu
 }
 
 // ---- amplitudes ----------------------------------------------------------------
+// complex128 states (single shard): gather into double2, D2H
+static int amplitudes64(sv_state* s, const uint64_t* idx, size_t count, sv_c128* out) {
+    const uint64_t dim = 1ull << s->n;
+    for (size_t i = 0; i < count; ++i)
+        if (idx[i] >= dim) return fail(SV_EINVAL, "amplitude index out of range");
+    int rc = ensure(s, s->idx_dev, s->idx_cap, count);
+    if (rc) return rc;
+    rc = ensure(s, s->amp_dev, s->amp_cap, 2 * count);
+    if (rc) return rc;
+    CK(s, cudaMemcpyAsync(s->idx_dev, idx, count * 8, cudaMemcpyHostToDevice, s->stream));
+    rc = launch(s, LaunchClass::OTHER, [&] {
+        return launch_gather64(reinterpret_cast<const double2*>(s->shard[0]), s->idx_dev, count,
+                               reinterpret_cast<double2*>(s->amp_dev), s->stream);
+    });
+    if (rc) return rc;
+    CK(s, cudaMemcpyAsync(out, s->amp_dev, count * 16, cudaMemcpyDeviceToHost, s->stream));
+    return sync(s);
+}
+
+int sv_amplitudes_c128(sv_state* s, const uint64_t* idx, size_t count, sv_c128* out) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count == 0) return SV_OK;
+    if (!idx || !out) return fail(SV_EINVAL, "idx/out is NULL");
+    if (s->fp64) return amplitudes64(s, idx, count, out);
+    std::vector<sv_c64> tmp(count);
+    rc = sv_amplitudes(s, idx, count, tmp.data());
+    if (rc) return rc;
+    for (size_t i = 0; i < count; ++i) out[i] = sv_c128{tmp[i].re, tmp[i].im};
+    return SV_OK;
+}
+
 int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
     int rc = check_state(s);
     if (rc) return rc;
     if (count == 0) return SV_OK;
     if (!idx || !out) return fail(SV_EINVAL, "idx/out is NULL");
+    if (s->fp64) {
+        std::vector<sv_c128> tmp(count);
+        rc = amplitudes64(s, idx, count, tmp.data());
+        if (rc) return rc;
+        for (size_t i = 0; i < count; ++i) out[i] = sv_c64{(float)tmp[i].re, (float)tmp[i].im};
+        return SV_OK;
+    }
     const uint64_t dim = 1ull << s->n;
     std::vector<uint64_t> loc(count);
     std::vector<int32_t> own(count);
@@ -995,7 +1147,8 @@ static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) 
     for (int i = 0; i < nloc; ++i) {
         const int d = s->virt ? i : s->rank;
         uint64_t* bins = s->bins + (size_t)i * nb;
-        rc = launch(s, LaunchClass::OTHER, [&] { return launch_bin_weights(s->shard[d], La, bins, s->stream); });
+        rc = launch(s, LaunchClass::OTHER,
+                    [&] { return launch_bin_weights(s->shard[d], s->fp64, La, bins, s->stream); });
         if (rc) return rc;
         rc = launch(s, LaunchClass::OTHER, [&] { return launch_inclusive_scan(bins, nb, s->scan_scratch, s->stream); });
         if (rc) return rc;
@@ -1031,7 +1184,7 @@ static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) 
         for (int d = 0; d < s->world; ++d) {
             const uint64_t base = (uint64_t)sig[d] << s->l;
             rc = launch(s, LaunchClass::OTHER, [&] {
-                return launch_sample_resolve(s->shard[d], La, s->bins + (size_t)d * nb, nb, lo + d, total, seed, N,
+                return launch_sample_resolve(s->shard[d], s->fp64, La, s->bins + (size_t)d * nb, nb, lo + d, total, seed, N,
                                              base, dev_out, s->stream);
             });
             if (rc) return rc;
@@ -1044,7 +1197,7 @@ static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) 
             const uint64_t base = (uint64_t)sig[s->rank] << s->l;
             // resolve samples o..o+cnt: shift the counter by o through the seed stream
             rc = launch(s, LaunchClass::OTHER, [&] {
-                return launch_sample_resolve(s->shard[s->rank], La, s->bins, nb, lo + s->rank, total,
+                return launch_sample_resolve(s->shard[s->rank], s->fp64, La, s->bins, nb, lo + s->rank, total,
                                              seed + (uint64_t)o * 0x9E3779B97F4A7C15ull, cnt, base, s->xfer, s->stream);
             });
             if (rc) return rc;
@@ -1082,41 +1235,79 @@ int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out) {
 }
 
 // ---- whole state ------------------------------------------------------------------
-int sv_set_state(sv_state* s, const sv_c64* host, size_t count) {
-    int rc = check_state(s);
-    if (rc) return rc;
-    if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
+static int set_state_bytes(sv_state* s, const void* host) {
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
+    const size_t sb = s->elem << s->l;
     for (int i = 0; i < s->local_shards(); ++i) {
         const int d = s->virt ? i : s->rank;
-        CK(s, cudaMemcpyAsync(s->shard[d], host + ((size_t)d << s->l), (size_t)8 << s->l, cudaMemcpyHostToDevice,
-                              s->stream));
+        CK(s, cudaMemcpyAsync(s->shard[d], (const char*)host + sb * d, sb, cudaMemcpyHostToDevice, s->stream));
     }
-    rc = sync(s);
+    int rc = sync(s);
     if (rc) return rc;
     return barrier(s) ? fail(SV_ECOMM, "barrier failed") : sync(s);
 }
 
-int sv_get_state(sv_state* s, sv_c64* host, size_t count) {
+int sv_set_state(sv_state* s, const sv_c64* host, size_t count) {
     int rc = check_state(s);
     if (rc) return rc;
     if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
-    rc = canonicalize(s);
+    if (!s->fp64) return set_state_bytes(s, host);
+    std::vector<sv_c128> up(count);
+    for (size_t i = 0; i < count; ++i) up[i] = sv_c128{host[i].re, host[i].im};
+    return set_state_bytes(s, up.data());
+}
+
+int sv_set_state_c128(sv_state* s, const sv_c128* host, size_t count) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
+    if (s->fp64) return set_state_bytes(s, host);
+    std::vector<sv_c64> dn(count);
+    for (size_t i = 0; i < count; ++i) dn[i] = sv_c64{(float)host[i].re, (float)host[i].im};
+    return set_state_bytes(s, dn.data());
+}
+
+static int get_state_bytes(sv_state* s, void* host) {
+    int rc = canonicalize(s);
     if (rc) return rc;
     rc = barrier(s);
     if (rc) return rc;
     rc = sync(s);
     if (rc) return rc;
+    const size_t sb = s->elem << s->l;
     for (int d = 0; d < s->world; ++d) {
         const int sg = sigma_of(s, d);
-        CK(s, cudaMemcpyAsync(host + ((size_t)sg << s->l), s->shard[d], (size_t)8 << s->l, cudaMemcpyDeviceToHost,
-                              s->stream));
+        CK(s, cudaMemcpyAsync((char*)host + sb * sg, s->shard[d], sb, cudaMemcpyDeviceToHost, s->stream));
     }
     rc = sync(s);
     if (rc) return rc;
     rc = barrier(s);
     if (rc) return rc;
     return sync(s);
+}
+
+int sv_get_state(sv_state* s, sv_c64* host, size_t count) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
+    if (!s->fp64) return get_state_bytes(s, host);
+    std::vector<sv_c128> full(count);
+    rc = get_state_bytes(s, full.data());
+    if (rc) return rc;
+    for (size_t i = 0; i < count; ++i) host[i] = sv_c64{(float)full[i].re, (float)full[i].im};
+    return SV_OK;
+}
+
+int sv_get_state_c128(sv_state* s, sv_c128* host, size_t count) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (count != (1ull << s->n) || !host) return fail(SV_EINVAL, "count must be 2^n and host non-NULL");
+    if (s->fp64) return get_state_bytes(s, host);
+    std::vector<sv_c64> low(count);
+    rc = get_state_bytes(s, low.data());
+    if (rc) return rc;
+    for (size_t i = 0; i < count; ++i) host[i] = sv_c128{low[i].re, low[i].im};
+    return SV_OK;
 }
 
 int sv_device_ptr(sv_state* s, int shard, void** out) {

@@ -1,0 +1,101 @@
+"""complex128 (fp64) states -- SURVEY.md §8f NEXT-1, the paper's Fig. 8
+experiment (double precision shows no substantial state
+differences).  Parity against the complex128 oracle with the fp64 analogue
+of the kernel error bound, |dy_r| <= (4 (2^k + 1) + 2) 2^-53 sum_c |M_rc||a_c|;
+circuits with fidelity 1 - 1e-12; sampling bit-exact (reading R5)."""
+import numpy as np
+import pytest
+
+import paper_conf_sc_markidis23_b200 as sv
+from oracle import ref_c
+from oracle import sample as osample
+from oracle import sv as osv
+from workloads import rqc as W
+
+pytestmark = pytest.mark.gpu
+U64 = 2.0 ** -53
+
+
+def _state128(n, seed):
+    rs = np.random.default_rng(seed)
+    psi = rs.standard_normal(1 << n) + 1j * rs.standard_normal(1 << n)
+    return psi / np.linalg.norm(psi)
+
+
+@pytest.mark.parametrize("k,qs_list", [(1, [(0,), (2,), (9,)]), (2, [(0, 5), (1, 2), (7, 3)]),
+                                        (3, [(0, 1, 2), (4, 8, 10), (2, 9, 5)]),
+                                        (4, [(0, 1, 2, 3), (3, 6, 9, 12), (13, 1, 7, 4)]),
+                                        (5, [(0, 2, 4, 6, 8), (5, 9, 10, 11, 13), (1, 3, 12, 7, 0)])])
+def test_apply_fp64_parity(k, qs_list):
+    n = 14
+    for i, qs in enumerate(qs_list):
+        rs = np.random.default_rng(10 * k + i)
+        M = W.haar_unitary(1 << k, rs)
+        psi = _state128(n, 3 + i)
+        h = sv.sv_create_ex(n, precision=1)
+        try:
+            sv.sv_set_state_c128(h, psi)
+            sv.sv_apply_fused_c128(h, list(qs), M)
+            got = sv.sv_get_state_c128(h, n)
+        finally:
+            sv.sv_destroy(h)
+        ref = osv.apply_gate(psi, n, list(qs), M)
+        bound = osv.apply_gate(np.abs(psi).astype(np.complex128), n, list(qs), np.abs(M).astype(np.complex128)).real
+        assert np.all(np.abs(got - ref) <= (4 * ((1 << k) + 1) + 2) * U64 * bound + 1e-300), qs
+
+
+@pytest.mark.parametrize("n,F", [(12, 0), (12, 4), (16, 2), (20, 4), (20, 5)])
+def test_rqc_fp64_matches_oracle(n, F):
+    gates = W.rqc(n, 14, seed=n)
+    ref = ref_c.run(n, gates)
+    h = sv.sv_create_ex(n, precision=1)
+    try:
+        sv.sv_run_circuit(h, gates, F)
+        got = sv.sv_get_state_c128(h, n)
+    finally:
+        sv.sv_destroy(h)
+    assert osv.fidelity(got, ref) >= 1 - 1e-12
+    assert np.abs(got - ref).max() <= 1e-12 * 2.0 ** (-n / 2) * 14
+
+
+def test_fp64_vs_fp32_no_substantial_disparity():
+    """fp64 and fp32 states agree (here: fidelity 1 - 1e-5)."""
+    n = 20
+    gates = W.rqc(n, 14)
+    out = {}
+    for prec in (0, 1):
+        h = sv.sv_create_ex(n, precision=prec)
+        try:
+            sv.sv_run_circuit(h, gates, 4)
+            out[prec] = sv.sv_get_state_c128(h, n)
+        finally:
+            sv.sv_destroy(h)
+    assert osv.fidelity(out[0], out[1]) >= 1 - 1e-5
+
+
+@pytest.mark.parametrize("n", [3, 10, 17])
+def test_sampler_fp64_bit_exact(n):
+    psi = _state128(n, 40 + n)
+    ref, _ = osample.sample(psi, 77, 3000)
+    h = sv.sv_create_ex(n, precision=1)
+    try:
+        sv.sv_set_state_c128(h, psi)
+        got = sv.sv_sample(h, 77, 3000)
+        idx = np.arange(0, 1 << n, 7, dtype=np.uint64)
+        assert np.array_equal(sv.sv_amplitudes_c128(h, idx), psi[idx.astype(np.int64)])
+    finally:
+        sv.sv_destroy(h)
+    assert np.array_equal(got, ref)
+
+
+def test_fp64_limits():
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_create_ex(16, world=2, precision=1)
+    assert e.value.code == sv.SV_EUNSUPPORTED
+    h = sv.sv_create_ex(10, precision=1)
+    try:
+        with pytest.raises(sv.SVError) as e:
+            sv.sv_apply_fused_c128(h, list(range(6)), np.eye(64))
+        assert e.value.code == sv.SV_EUNSUPPORTED
+    finally:
+        sv.sv_destroy(h)

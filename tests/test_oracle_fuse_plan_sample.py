@@ -161,6 +161,22 @@ def test_sampler_matches_definition(n, seed):
     assert T == Tr and [int(x) for x in got] == ref
 
 
+def test_sampler_complex128_matches_definition():
+    """Reading R5: complex128 weights use p = fl(fl(re^2) + fl(im^2)), i.e.
+    Python float arithmetic."""
+    rs = np.random.default_rng(8)
+    n = 7
+    psi = rs.standard_normal(1 << n) + 1j * rs.standard_normal(1 << n)
+    psi /= np.linalg.norm(psi)
+    w_ref = [math.floor((a.real * a.real + a.imag * a.imag) * 2.0 ** 62) for a in psi]
+    assert [int(x) for x in sample.weights(psi)] == w_ref
+    got, T = sample.sample(psi, 5, 200)
+    C = np.cumsum(np.array(w_ref, dtype=object))
+    for s_, x in enumerate(got):
+        t = (W.splitmix64_nth(5, s_) * sum(w_ref)) >> 64
+        assert int(x) == next(i for i, c in enumerate(C) if c > t)
+
+
 def test_sampler_enumeration_n2():
     # probabilities exactly 1/2, 0, 1/4, 1/4: w = 2^61, 0, 2^60, 2^60
     psi = np.array([0.5 + 0.5j, 0, 0.5, 0.5j], dtype=np.complex64)
