@@ -135,6 +135,15 @@ int sv_reset(sv_state* s);
  * Asynchronous: the matrix is staged before return. */
 int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix);
 
+/* Controlled gate (qsim ApplyControlledGate; SURVEY.md
+ * NEXT-4): the k-qubit matrix acts on targets[] only where every one of the
+ * n_ctrl control qubits is 1 (0 <= n_ctrl <= 6, all qubits distinct).  On
+ * unsharded complex64 states with no control on qubit 0 only the
+ * control-1 subspace (2^-n_ctrl of the state) is read and written; otherwise
+ * the block matrix over targets ++ controls is applied (k + n_ctrl <= 6). */
+int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k, const int32_t* targets,
+                        const sv_c64* matrix);
+
 /* Same with a complex128 matrix (no rounding on complex128 states; rounded to
  * complex64 on complex64 states). */
 int sv_apply_fused_c128(sv_state* s, int k, const int32_t* qubits, const sv_c128* matrix);

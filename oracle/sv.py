@@ -43,6 +43,42 @@ def apply_gate(psi: np.ndarray, n: int, qubits: Sequence[int], g: np.ndarray) ->
     return np.ascontiguousarray(res).reshape(-1)
 
 
+def apply_controlled(psi: np.ndarray, n: int, controls: Sequence[int], targets: Sequence[int],
+                     g: np.ndarray) -> np.ndarray:
+    """Controlled gate (qsim's ApplyControlledGate): G acts
+    on `targets` in the subspace where every control qubit is 1; amplitudes
+    with any control 0 are unchanged.  Written as that definition: take the
+    sub-tensor with the control axes fixed to 1 and apply G to it."""
+    controls = list(controls)
+    targets = list(targets)
+    assert not set(controls) & set(targets)
+    t = np.asarray(psi, dtype=np.complex128).reshape((2,) * n).copy()
+    idx = [slice(None)] * n
+    for c in controls:
+        idx[n - 1 - c] = 1
+    sub = t[tuple(idx)]  # remaining axes: qubits not in controls, descending
+    rest = sorted((q for q in range(n) if q not in controls), reverse=True)
+    m = len(rest)
+    # qubit q -> position in the sub-state (little-endian over the remaining qubits)
+    sub_pos = {q: m - 1 - i for i, q in enumerate(rest)}
+    new = apply_gate(sub.reshape(-1), m, [sub_pos[q] for q in targets], g).reshape(sub.shape)
+    t[tuple(idx)] = new
+    return t.reshape(-1)
+
+
+def controlled_full_matrix(n: int, controls: Sequence[int], targets: Sequence[int], g: np.ndarray) -> np.ndarray:
+    """Brute force: |all-controls-1><..| (x) G + (I - that projector) (x) I as a
+    2^n x 2^n matrix (n <= 10)."""
+    u = full_gate_matrix(n, list(targets), g)
+    idx = np.arange(1 << n)
+    on = np.ones(1 << n, dtype=bool)
+    for c in controls:
+        on &= ((idx >> c) & 1) == 1
+    full = np.eye(1 << n, dtype=np.complex128)
+    full[np.ix_(on, on)] = u[np.ix_(on, on)]
+    return full
+
+
 def simulate(n: int, gates, psi0: np.ndarray | None = None) -> np.ndarray:
     """U_m ... U_1 |psi0> (default |0..0>), unfused, in circuit order (S0)."""
     psi = zero_state(n) if psi0 is None else np.asarray(psi0, dtype=np.complex128).copy()

@@ -97,6 +97,7 @@ _SIGS = {
     "sv_reset": ([_vp], ctypes.c_int),
     "sv_apply_fused": ([_vp, ctypes.c_int, _i32p, _vp], ctypes.c_int),
     "sv_apply_fused_c128": ([_vp, ctypes.c_int, _i32p, _vp], ctypes.c_int),
+    "sv_apply_controlled": ([_vp, ctypes.c_int, _i32p, ctypes.c_int, _i32p, _vp], ctypes.c_int),
     "sv_run_circuit": ([_vp, _vp, _sz, ctypes.c_int, ctypes.POINTER(sv_stats)], ctypes.c_int),
     "sv_circuit_create": ([_vp, _vp, _sz, ctypes.c_int, ctypes.POINTER(_vp)], ctypes.c_int),
     "sv_circuit_run_device": ([_vp, _vp], ctypes.c_int),
@@ -201,6 +202,16 @@ def sv_apply_fused(h: int, qubits: Sequence[int], matrix) -> None:
     if m.size != (1 << (2 * k)):
         raise ValueError("matrix must be 2^k x 2^k")
     _check(lib().sv_apply_fused(h, k, q.ctypes.data_as(_i32p), _ptr(m)), "sv_apply_fused")
+
+
+def sv_apply_controlled(h: int, controls: Sequence[int], targets: Sequence[int], matrix) -> None:
+    c = np.ascontiguousarray(controls, dtype=np.int32)
+    t = np.ascontiguousarray(targets, dtype=np.int32)
+    m = np.ascontiguousarray(matrix, dtype=np.complex64)
+    if m.size != (1 << (2 * t.size)):
+        raise ValueError("matrix must be 2^k x 2^k over the targets")
+    _check(lib().sv_apply_controlled(h, c.size, c.ctypes.data_as(_i32p), t.size, t.ctypes.data_as(_i32p), _ptr(m)),
+           "sv_apply_controlled")
 
 
 def sv_apply_fused_c128(h: int, qubits: Sequence[int], matrix) -> None:

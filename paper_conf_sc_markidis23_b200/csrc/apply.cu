@@ -90,6 +90,9 @@ struct alignas(16) TileParams {
     int nzt;
     int ztpos[SV_MAX_FUSED];           // tile-local gate bit positions, ascending
     uint32_t swz[3];                   // phys bit (i+1) ^= parity(t & swz[i])
+    int nZ;                            // tile-base zero insertions: H and control qubits, ascending
+    int Zpos[2 * SV_MAX_FUSED];
+    uint64_t ones;                     // control qubits forced to 1 in the tile base
     int upt;                           // 16-byte units per thread per tile
     int iters;                         // compute iterations per thread per tile
     uint64_t goff[64];                 // dep(2 * nthreads * i)
@@ -535,6 +538,18 @@ __device__ __forceinline__ void tile_compute_tc(const TileParams<K>& p, uint32_t
 
 // Persistent loop over tiles.  STAGES = 2: the copies of tile i+1 are in
 // flight while tile i is transformed and written back.
+// Global index of tile u's first amplitude: zeros at the tile's high gate
+// qubits and at the control qubits, then the controls set to 1.
+template <int K>
+__device__ __forceinline__ uint64_t tile_base(const TileParams<K>& p, uint64_t u) {
+    uint64_t x = u << p.r;
+    for (int b = 0; b < p.nZ; ++b) {
+        const int q = p.Zpos[b];
+        x = ((x >> q) << (q + 1)) | (x & ((1ull << q) - 1ull));
+    }
+    return x | p.ones;
+}
+
 template <int K, bool PAIR, int MODE, int STAGES>
 __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
     extern __shared__ float4 dsm[];
@@ -565,11 +580,11 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
     const uint32_t sthr = swizzle(t0, p.swz);
     const int upt = p.upt;
     auto load = [&](uint64_t u, uint32_t sbuf) {
-        const float2* g = p.psi + insert_zeros(u << p.r, p.Hpos, p.nH) + dthr;
+        const float2* g = p.psi + tile_base(p, u) + dthr;
         for (int i = 0; i < upt; ++i) cp_async16(sbuf + ((sthr ^ p.soff[i]) << 3), g + p.goff[i]);
     };
     auto store = [&](uint64_t u, uint32_t sbuf) {
-        float2* g = p.psi + insert_zeros(u << p.r, p.Hpos, p.nH) + dthr;
+        float2* g = p.psi + tile_base(p, u) + dthr;
         for (int i = 0; i < upt; ++i)
             st_stream(reinterpret_cast<float4*>(g + p.goff[i]), lds4(sbuf + ((sthr ^ p.soff[i]) << 3)));
     };
@@ -636,6 +651,9 @@ struct SmallParams {
     float2* psi;
     uint64_t n_groups;
     int q[SV_MAX_FUSED];
+    int nz;                        // gate + control qubits, ascending (zero insertion)
+    int zpos[2 * SV_MAX_FUSED];
+    uint64_t ones;                 // control qubits set to 1
     MatStore<K> M;
 };
 template <int K>
@@ -643,7 +661,12 @@ __global__ void __launch_bounds__(256) apply_small(const __grid_constant__ Small
     constexpr int D = 1 << K;
     const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (g >= p.n_groups) return;
-    const uint64_t base = insert_zeros(g, p.q, K);
+    uint64_t base = g;
+    for (int b = 0; b < p.nz; ++b) {
+        const int q = p.zpos[b];
+        base = ((base >> q) << (q + 1)) | (base & ((1ull << q) - 1ull));
+    }
+    base |= p.ones;
     uint64_t off[D];
     float2 a[D];
 #pragma unroll
@@ -807,8 +830,16 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         SmallParams<K> sp;
         std::memset(&sp, 0, sizeof(sp));
         sp.psi = psi;
-        sp.n_groups = 1ull << (n - K);
+        sp.n_groups = 1ull << (n - K - d.nc);
         for (int b = 0; b < K; ++b) sp.q[b] = d.q[b];
+        std::vector<int> z(d.q, d.q + K);
+        for (int c = 0; c < d.nc; ++c) {
+            z.push_back(d.cq[c]);
+            sp.ones |= 1ull << d.cq[c];
+        }
+        std::sort(z.begin(), z.end());
+        sp.nz = (int)z.size();
+        for (size_t i = 0; i < z.size(); ++i) sp.zpos[i] = z[i];
         fill_matrix<K>(sp.M, d);
         apply_small<K><<<(unsigned)((sp.n_groups + 255) / 256), 256, 0, st>>>(sp);
         return cudaGetLastError();
@@ -817,7 +848,17 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         p.goff[i] = dep(2ull * nthr * i);
         p.soff[i] = sw(2u * nthr * i);
     }
-    p.n_tiles = 1ull << (n - p.T);
+    {
+        std::vector<int> z(p.Hpos, p.Hpos + p.nH);
+        for (int c = 0; c < d.nc; ++c) {
+            z.push_back(d.cq[c]);
+            p.ones |= 1ull << d.cq[c];
+        }
+        std::sort(z.begin(), z.end());
+        p.nZ = (int)z.size();
+        for (size_t i = 0; i < z.size(); ++i) p.Zpos[i] = z[i];
+    }
+    p.n_tiles = 1ull << (n - p.T - d.nc);
     const int STG = d.tc ? 2 : stages_for(K);
     size_t smem = (size_t)STG * ((size_t)8 << p.T);
     if (K == 6) smem += 64 * 64 * 8;
@@ -876,7 +917,7 @@ void plan_apply(int n, ApplyDesc& d) {
             const char* e = std::getenv("SVB200_TC");
             return e && e[0] == '1';
         }();
-        d.tc = !mono && use_tc && tc_supported(n, d);
+        d.tc = !mono && use_tc && d.nc == 0 && tc_supported(n, d);
     }
     uint64_t gm = 0;
     for (int b = 0; b < d.k; ++b) gm |= 1ull << d.q[b];
@@ -890,8 +931,11 @@ void plan_apply(int n, ApplyDesc& d) {
             if (d.q[b] >= rr) ++t;
         return t;
     };
-    int r = std::min(n, 4);
-    while (r < n && tile_bits(r) < target) ++r;
+    int minc = n;
+    for (int c = 0; c < d.nc; ++c) minc = std::min(minc, d.cq[c]);
+    const int nfree = n - d.nc;  // qubits a tile may span
+    int r = std::min(std::min(nfree, 4), minc);
+    while (r < n && r < minc && tile_bits(r) < std::min(target, nfree)) ++r;
     d.r = r;
     d.T = tile_bits(r);
 }

@@ -24,6 +24,8 @@ struct ApplyDesc {
     std::vector<cf> m;                // 2^k x 2^k row-major over ascending q, complex64
     bool high = false;                // kernel class
     bool mono = false;                // one nonzero per row (exact permutation/diagonal path)
+    int nc = 0;                       // control qubits (controlled gate, NEXT-4): only the
+    int cq[SV_MAX_FUSED] = {0};       //   amplitudes with every control bit 1 are transformed
     bool tc = false;                  // tensor-core path (tc.cu)
     // low-kernel tile plan (host-computed once)
     int T = 0, r = 0;                 // tile bits, run bits

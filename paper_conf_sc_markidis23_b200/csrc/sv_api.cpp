@@ -637,6 +637,65 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
     return run_apply(s, d);
 }
 
+int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k, const int32_t* targets,
+                        const sv_c64* matrix) {
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
+    if (n_ctrl < 0 || n_ctrl > SV_MAX_FUSED) return fail(SV_EINVAL, "n_ctrl must be in [0, 6]");
+    if (!targets || !matrix || (n_ctrl > 0 && !controls)) return fail(SV_EINVAL, "NULL argument");
+    uint64_t mask = 0;
+    for (int b = 0; b < k + n_ctrl; ++b) {
+        const int q = b < k ? targets[b] : controls[b - k];
+        if (q < 0 || q >= s->n) return fail(SV_EINVAL, "qubit out of range");
+        if ((mask >> q) & 1) return fail(SV_EINVAL, "duplicate qubit");
+        mask |= 1ull << q;
+    }
+    if (n_ctrl == 0) return sv_apply_fused(s, k, targets, matrix);
+    const int D = 1 << k;
+    std::vector<cd> M((size_t)D * D);
+    for (int i = 0; i < D * D; ++i) M[i] = cd(matrix[i].re, matrix[i].im);
+    int minc = s->n;
+    for (int c = 0; c < n_ctrl; ++c) minc = std::min(minc, (int)controls[c]);
+    if (!s->fp64 && s->g == 0 && minc >= 1) {
+        // tile engine over the control-1 subspace only: 2^-n_ctrl of the state
+        ApplyDesc d;
+        make_apply(s->l, k, targets, M.data(), d);
+        d.nc = n_ctrl;
+        for (int c = 0; c < n_ctrl; ++c) d.cq[c] = controls[c];
+        d.tc = false;
+        plan_apply(s->l, d);
+        d.tc = false;
+        if (k == 6) {
+            CK(s, cudaMemcpyAsync(s->kmat, d.m.data(), 64 * 64 * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
+            CK(s, cudaStreamSynchronize(s->stream));
+            d.dev_m = s->kmat;
+        }
+        rc = launch(s, d.high ? LaunchClass::HIGH : LaunchClass::LOW,
+                    [&] { return launch_apply(s->shard[0], s->l, d, s->stream); });
+        if (rc) return rc;
+        s->stats.bytes_apply += 16ull << (s->l - n_ctrl);
+        s->stats.flops_apply += (uint64_t)((8 << k) - 2) << (s->l - n_ctrl);
+        return SV_OK;
+    }
+    if (k + n_ctrl > SV_MAX_FUSED)
+        return fail(SV_EUNSUPPORTED, "controlled gate needs k + n_ctrl <= 6 here (control on qubit 0, sharded or fp64)");
+    // dense block expansion over targets ++ controls: U on the all-ones control block, identity elsewhere
+    const int kk = k + n_ctrl, DD = 1 << kk;
+    std::vector<int32_t> qs(targets, targets + k);
+    for (int c = 0; c < n_ctrl; ++c) qs.push_back(controls[c]);
+    std::vector<cd> F((size_t)DD * DD, cd(0));
+    const int call = ((1 << n_ctrl) - 1) << k;
+    for (int r = 0; r < DD; ++r) {
+        if ((r & call) == call) {
+            for (int c = 0; c < D; ++c) F[(size_t)r * DD + (call | c)] = M[(size_t)(r & (D - 1)) * D + c];
+        } else {
+            F[(size_t)r * DD + r] = 1.0;
+        }
+    }
+    return apply_matrix(s, kk, qs.data(), F);
+}
+
 int sv_fusion_plan(const sv_gate* gates, size_t n_gates, int max_fused, int32_t* buf, size_t cap, size_t* need) {
     if (!need) return fail(SV_EINVAL, "need is NULL");
     if (max_fused < 0 || max_fused > SV_MAX_FUSED) return fail(SV_EINVAL, "max_fused must be in [0, 6]");

@@ -97,6 +97,28 @@ def test_rqc12_unitary_brute_force():
     assert np.abs(u.conj().T @ u - np.eye(1 << 10)).max() < 1e-12
 
 
+# -------------------------------------------------------- controlled gates
+def test_controlled_gate_vs_brute_force():
+    rs = np.random.default_rng(21)
+    n = 7
+    for controls, targets in (([0], [1]), ([3], [0]), ([6, 2], [4]), ([1, 5], [0, 3]), ([0, 1, 2], [6]),
+                              ([4], [2, 5, 6])):
+        g = W.haar_unitary(1 << len(targets), rs)
+        psi = W.random_state_c64(n, 5).astype(np.complex128)
+        ref = sv.controlled_full_matrix(n, controls, targets, g) @ psi
+        assert np.abs(sv.apply_controlled(psi, n, controls, targets, g) - ref).max() < 1e-14
+
+
+def test_controlled_x_is_cx_and_controls_commute():
+    psi = W.random_state_c64(5, 2).astype(np.complex128)
+    # CX (qubits[0] = control) == controlled-X
+    assert np.abs(sv.apply_controlled(psi, 5, [1], [3], W.GATE_X) - sv.apply_gate(psi, 5, [1, 3], W.GATE_CX)).max() == 0
+    # CZ is symmetric: control 0 target 2 == control 2 target 0
+    a = sv.apply_controlled(psi, 5, [0], [2], W.GATE_Z)
+    b = sv.apply_controlled(psi, 5, [2], [0], W.GATE_Z)
+    assert np.abs(a - b).max() == 0
+
+
 # ------------------------------------------------------------- closed forms
 @pytest.mark.parametrize("n", [1, 5, 12])
 def test_hadamard_layer_uniform(n):
