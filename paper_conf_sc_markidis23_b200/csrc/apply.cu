@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
 
@@ -99,6 +100,7 @@ struct alignas(16) TileParams {
     uint32_t soff[64];                 // phys(2 * nthreads * i)
     uint32_t loc[1 << K];              // phys offsets of the gathers (members / member pairs)
     uint32_t gsec;                     // phys offset of the second group of a pair (PAIR, 2 groups)
+    const uint8_t* wi8;                // tensor-core int8 path: W slices + column exponents (device)
     // monomial matrices (one nonzero per row: permutations, diagonals, identity)
     int mono;
     uint32_t mloc[1 << K];             // phys offset of member r (output slot of row r)
@@ -360,6 +362,18 @@ __device__ __forceinline__ void tmem_st8(uint32_t taddr, const float* v) {
                  "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7]))
                  : "memory");
 }
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t* v) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+                 : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+        : "r"(taddr));
+}
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* v) {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
@@ -536,6 +550,271 @@ __device__ __forceinline__ void tile_compute_tc(const TileParams<K>& p, uint32_t
     tc_fence_before();
 }
 
+// ------------------------------------------ tensor cores, exact accumulation
+// The TF32 path above is biased (its accumulation truncates toward zero).
+// Here the contraction Out = In . W runs on tcgen05.mma.kind::i8 with exact
+// s32 accumulation: every real input of a group row is scaled by a
+// power-of-two row scale 2^(22 - e_r) to an integer |xi| <= 2^22 written in
+// balanced signed base-256 digits
+//   xi = a0 2^16 + a1 2^8 + a2     (a1, a2 in [-128, 127], |a0| <= 65),
+// every column n of W likewise with 2^(22 - f_n) into b0, b1, b2, and
+//   sum_kk xi wi ~= 2^16 (S32 2^16 + S24 2^8 + S16),
+//   S32 = a0.b0, S24 = a0.b1 + a1.b0, S16 = a0.b2 + a1.b1 + a2.b0
+// (6 int8 MMAs per K-step of 32).  The dropped cross terms (a1.b2, a2.b1,
+// a2.b2) are below 2^-21 of the row x column scale and zero-mean (balanced
+// digits), so no bias.  The three s32 sums are exact; they are combined in
+// int64, converted to fp32 with a single correctly rounded conversion and
+// scaled by 2^(e_r + f_n - 28) (exact).
+// Operand A (slices) and B (W slices) live in shared memory in the K-major
+// SWIZZLE_NONE canonical layout (core matrix 8 rows x 16 B), D in TMEM.
+template <int K>
+struct TciShape {
+    static constexpr int D = 1 << K;
+    static constexpr int KR = 2 * D;                  // MMA K (reals per group)
+    static constexpr int N = 2 * D;                   // MMA N
+    static constexpr int MB = (1 << (12 - K)) / 128;  // M-blocks of 128 groups per 2^12 tile
+    static constexpr int KS = KR / 32;                // int8 MMA K-steps (K = 32)
+    static constexpr uint32_t SBO = KR * 8;           // byte distance between row octets (KR/16 chunks x 128 B)
+    static constexpr uint32_t A_SLICE = 128u * MB * KR;  // bytes of one A slice
+    static constexpr uint32_t B_SLICE = (uint32_t)N * KR;
+    static constexpr uint32_t ROWMAX = 2 * 128 * MB * 4;  // half-row maxima exchange
+    static constexpr uint32_t SMEM = 3 * A_SLICE + 3 * B_SLICE + N * 4 + ROWMAX + 64;
+    static constexpr int NACC = 3;                    // S32, S24, S16
+    static constexpr int COLS = NACC * N * MB;
+    static constexpr int ALLOC = COLS <= 32 ? 32 : COLS <= 64 ? 64 : COLS <= 128 ? 128 : COLS <= 256 ? 256 : 512;
+};
+
+__host__ __device__ constexpr uint32_t umma_idesc_i8(int N, bool a_signed, bool b_signed) {
+    return (2u << 4) | ((a_signed ? 1u : 0u) << 7) | ((b_signed ? 1u : 0u) << 10) | ((uint32_t)(N >> 3) << 17) |
+           ((uint32_t)(128 >> 4) << 24);
+}
+__device__ __forceinline__ void mma_i8_ss(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc)
+        : "memory");
+}
+
+struct TciState {
+    uint32_t tmem, sA, sB, sF, sM, bar, phase;
+};
+
+template <int K>
+__device__ __forceinline__ TciState tci_setup(const TileParams<K>& p, uint32_t sBase) {
+    using S = TciShape<K>;
+    TciState t;
+    t.sA = sBase;
+    t.sB = sBase + 3 * S::A_SLICE;
+    t.sF = t.sB + 3 * S::B_SLICE;
+    t.sM = t.sF + S::N * 4;
+    t.bar = t.sM + S::ROWMAX;
+    const uint32_t slot = t.bar + 8;
+    // B slices (canonical layout, prepared on the host) + column exponents
+    const uint4* src = reinterpret_cast<const uint4*>(p.wi8);
+    for (uint32_t i = threadIdx.x; i < (3 * S::B_SLICE + S::N * 4) / 16; i += blockDim.x) {
+        const uint4 v = src[i];
+        asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(t.sB + 16 * i), "r"(v.x), "r"(v.y), "r"(v.z),
+                     "r"(v.w)
+                     : "memory");
+    }
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(t.bar) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if ((threadIdx.x >> 5) == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(slot), "n"(S::ALLOC)
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t.tmem) : "r"(slot) : "memory");
+    t.phase = 0;
+    return t;
+}
+
+template <int K>
+__device__ __forceinline__ void tci_teardown(const TciState& t) {
+    using S = TciShape<K>;
+    tc_fence_before();
+    __syncthreads();
+    if ((threadIdx.x >> 5) == 0)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(t.tmem), "n"(S::ALLOC) : "memory");
+}
+
+// 16 reals -> one 16 B chunk of each of the three slices.
+// v = x * scale + 1.5 * 2^23 rounds x * scale to the nearest integer xi
+// (|xi| <= 2^22) and leaves bits(v) = 0x4B400000 + xi.  The balanced digits
+// are d2 = low byte of xi, d1 = byte 1 of xi + 2^7, d0 = byte 2 of
+// xi + 2^15 + 2^7, i.e. bytes of bits(v) plus constants (the additions only
+// carry upward, so the low bytes of 0x4B400000 + ... are those of xi + ...).
+__device__ __forceinline__ void slice16(const float* x, float scale, uint4& s0, uint4& s1, uint4& s2) {
+    uint32_t w0[4], w1[4], w2[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        uint32_t b2[4], b1[4], b0[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            const uint32_t v = __float_as_uint(fmaf(x[4 * q + e], scale, 12582912.0f));
+            b2[e] = v;
+            b1[e] = v + 128u;
+            b0[e] = v + (32896u - 0x400000u);
+        }
+        w2[q] = __byte_perm(__byte_perm(b2[0], b2[1], 0x0040), __byte_perm(b2[2], b2[3], 0x0040), 0x5410);
+        w1[q] = __byte_perm(__byte_perm(b1[0], b1[1], 0x0051), __byte_perm(b1[2], b1[3], 0x0051), 0x5410);
+        w0[q] = __byte_perm(__byte_perm(b0[0], b0[1], 0x0062), __byte_perm(b0[2], b0[3], 0x0062), 0x5410);
+    }
+    s0 = make_uint4(w0[0], w0[1], w0[2], w0[3]);
+    s1 = make_uint4(w1[0], w1[1], w1[2], w1[3]);
+    s2 = make_uint4(w2[0], w2[1], w2[2], w2[3]);
+}
+
+__device__ __forceinline__ void sts128u(uint32_t a, uint4 v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+
+// Two threads per MMA row (256 threads): thread h = threadIdx.x / 128 of row
+// r = threadIdx.x % 128 gathers and slices members [h D/2, (h+1) D/2) and
+// later combines output columns [h N/2, (h+1) N/2); warps 4..7 read the same
+// TMEM lane quarters as warps 0..3.
+template <int K, bool PAIR>
+__device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_t sbuf, TciState& t) {
+    using S = TciShape<K>;
+    constexpr int D = S::D;
+    constexpr int HM = D / 2;  // members per thread
+    const int half = threadIdx.x >> 7;
+    const uint32_t row = threadIdx.x & 127u;
+    const uint32_t lane_base = (uint32_t)(((threadIdx.x >> 5) & 3) * 32) << 16;
+    float srow[S::MB];
+    float x[S::MB][2 * HM];
+    uint32_t pbs[S::MB];
+    // 1a. gather this thread's half row, publish the half maximum
+#pragma unroll
+    for (int mb = 0; mb < S::MB; ++mb) {
+        const uint32_t g = (uint32_t)mb * 128u + row;
+        const uint32_t pb = swizzle((uint32_t)insert_zeros(g, p.ztpos, p.nzt), p.swz);
+        pbs[mb] = pb;
+#pragma unroll
+        for (int j = 0; j < HM / 2; ++j) {
+            const int jj = half * (HM / 2) + j;  // member pair (2jj, 2jj+1)
+            if constexpr (PAIR) {
+                const float4 v = lds4(sbuf + ((pb ^ p.loc[jj]) << 3));
+                x[mb][4 * j] = v.x; x[mb][4 * j + 1] = v.y; x[mb][4 * j + 2] = v.z; x[mb][4 * j + 3] = v.w;
+            } else {
+                const float2 u = lds2(sbuf + ((pb ^ p.loc[2 * jj]) << 3));
+                const float2 w = lds2(sbuf + ((pb ^ p.loc[2 * jj + 1]) << 3));
+                x[mb][4 * j] = u.x; x[mb][4 * j + 1] = u.y; x[mb][4 * j + 2] = w.x; x[mb][4 * j + 3] = w.y;
+            }
+        }
+        float mx = 0.f;
+#pragma unroll
+        for (int i = 0; i < 2 * HM; ++i) mx = fmaxf(mx, fabsf(x[mb][i]));
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(t.sM + 4u * ((uint32_t)mb * 256u + threadIdx.x)), "f"(mx)
+                     : "memory");
+    }
+    __syncthreads();
+    // 1b. row scale 2^(22 - e) with max|x| < 2^e; slice into A (shared memory)
+#pragma unroll
+    for (int mb = 0; mb < S::MB; ++mb) {
+        float m0, m1;
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(m0) : "r"(t.sM + 4u * ((uint32_t)mb * 256u + row)));
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(m1) : "r"(t.sM + 4u * ((uint32_t)mb * 256u + 128u + row)));
+        const float mx = fmaxf(m0, m1);
+        const int e = max(((int)(__float_as_uint(mx) >> 23) & 0xFF) - 126, -100);  // mx < 2^e
+        srow[mb] = __uint_as_float((uint32_t)(127 + e - 14) << 23);                 // 2^(e - 14)
+        const float scale = __uint_as_float((uint32_t)(127 + 22 - e) << 23);
+        const uint32_t rbase = (uint32_t)mb * 128u * S::KR + (row >> 3) * S::SBO + (row & 7) * 16u;
+#pragma unroll
+        for (int c = 0; c < HM / 8; ++c) {  // 16 reals per chunk
+            uint4 s0, s1, s2;
+            slice16(x[mb] + 16 * c, scale, s0, s1, s2);
+            const uint32_t a = t.sA + rbase + (uint32_t)(half * (HM / 8) + c) * 128u;
+            sts128u(a, s0);
+            sts128u(a + S::A_SLICE, s1);
+            sts128u(a + 2 * S::A_SLICE, s2);
+        }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    // 2. eight int8 MMAs per K-step into four exact s32 accumulators
+    if (threadIdx.x == 0) {
+        constexpr uint32_t i_ss = umma_idesc_i8(S::N, true, true);
+#pragma unroll
+        for (int mb = 0; mb < S::MB; ++mb) {
+            const uint32_t d0 = t.tmem + (uint32_t)(mb * S::NACC * S::N);
+            const uint32_t d32 = d0, d24 = d0 + S::N, d16 = d0 + 2 * S::N;
+#pragma unroll
+            for (int ks = 0; ks < S::KS; ++ks) {
+                const uint32_t ao = t.sA + (uint32_t)mb * 128u * S::KR + (uint32_t)ks * 256u;
+                const uint32_t bo = t.sB + (uint32_t)ks * 256u;
+                const uint64_t a0 = umma_desc(ao, 128, S::SBO), a1 = umma_desc(ao + S::A_SLICE, 128, S::SBO),
+                               a2 = umma_desc(ao + 2 * S::A_SLICE, 128, S::SBO);
+                const uint64_t b0 = umma_desc(bo, 128, S::SBO), b1 = umma_desc(bo + S::B_SLICE, 128, S::SBO),
+                               b2 = umma_desc(bo + 2 * S::B_SLICE, 128, S::SBO);
+                const uint32_t acc = ks > 0 ? 1u : 0u;
+                mma_i8_ss(d32, a0, b0, i_ss, acc);
+                mma_i8_ss(d24, a0, b1, i_ss, acc);
+                mma_i8_ss(d24, a1, b0, i_ss, 1u);
+                mma_i8_ss(d16, a0, b2, i_ss, acc);
+                mma_i8_ss(d16, a1, b1, i_ss, 1u);
+                mma_i8_ss(d16, a2, b0, i_ss, 1u);
+            }
+        }
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(t.bar)
+                     : "memory");
+    }
+    mbar_wait(t.bar, t.phase);
+    t.phase ^= 1u;
+    tc_fence_after();
+    // 3. exact recombination of this thread's half of the columns, one rounding
+#pragma unroll
+    for (int mb = 0; mb < S::MB; ++mb) {
+        const uint32_t pb = pbs[mb];
+        const uint32_t d0 = t.tmem + lane_base + (uint32_t)(mb * S::NACC * S::N);
+#pragma unroll 1
+        for (int c0 = half * (S::N / 2); c0 < (half + 1) * (S::N / 2); c0 += 8) {
+            uint32_t v32[8], v24[8], v16[8];
+            tmem_ld8(d0 + (uint32_t)c0, v32);
+            tmem_ld8(d0 + (uint32_t)(S::N + c0), v24);
+            tmem_ld8(d0 + (uint32_t)(2 * S::N + c0), v16);
+            float fc[8];
+#pragma unroll
+            for (int q = 0; q < 2; ++q)
+                asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
+                             : "=f"(fc[4 * q]), "=f"(fc[4 * q + 1]), "=f"(fc[4 * q + 2]), "=f"(fc[4 * q + 3])
+                             : "r"(t.sF + 4u * (uint32_t)(c0 + 4 * q)));
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+            float o[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                // exact integer combination (|S24 2^8 + S16| < 2^30), ONE
+                // correctly rounded int64 -> fp32 conversion, then the exact
+                // power-of-two scaling 2^(e - 14) 2^(f - 14) (each factor normal)
+                const int lo = (int)v24[i] * 256 + (int)v16[i];
+                const long long tt = (long long)(int)v32[i] * 65536ll + (long long)lo;
+                o[i] = __ll2float_rn(tt) * srow[mb] * fc[i];
+            }
+#pragma unroll
+            for (int i = 0; i < 2; ++i) {
+                const int j = c0 / 4 + i;
+                if constexpr (PAIR) {
+                    sts4(sbuf + ((pb ^ p.loc[j]) << 3), make_float4(o[4 * i], o[4 * i + 1], o[4 * i + 2], o[4 * i + 3]));
+                } else {
+                    sts2(sbuf + ((pb ^ p.loc[2 * j]) << 3), make_float2(o[4 * i], o[4 * i + 1]));
+                    sts2(sbuf + ((pb ^ p.loc[2 * j + 1]) << 3), make_float2(o[4 * i + 2], o[4 * i + 3]));
+                }
+            }
+        }
+    }
+    tc_fence_before();
+}
+
 // Persistent loop over tiles.  STAGES = 2: the copies of tile i+1 are in
 // flight while tile i is transformed and written back.
 // Global index of tile u's first amplitude: zeros at the tile's high gate
@@ -562,6 +841,8 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
         smat = sm;
         __syncthreads();
     }
+    TciState tis{};
+    if constexpr (MODE == 3 && K <= 5) tis = tci_setup<K>(p, s0 + STAGES * tile_bytes);
     TcState tcs{};
     if constexpr (MODE == 2 && K <= 5) {
         const uint32_t sW = s0 + STAGES * tile_bytes;
@@ -603,11 +884,13 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             __syncthreads();   // ... and everyone else's
             if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, cur);
             else if constexpr (MODE == 2 && K <= 5) tile_compute_tc<K, PAIR>(p, cur, tcs);
+            else if constexpr (MODE == 3 && K <= 5) tile_compute_tci<K, PAIR>(p, cur, tis);
             else tile_compute<K, PAIR>(p, cur, smat);
             __syncthreads();
             store(u, cur);
         }
         if constexpr (MODE == 2 && K <= 5) tc_teardown<K>(tcs);
+        if constexpr (MODE == 3 && K <= 5) tci_teardown<K>(tis);
     } else {
         for (; u < p.n_tiles; u += gridDim.x) {
             __syncthreads();
@@ -642,6 +925,10 @@ __global__ void __launch_bounds__(256) apply_low(const __grid_constant__ TilePar
 template <int K, bool PAIR>
 __global__ void __launch_bounds__(128, 1) apply_tc(const __grid_constant__ TileParams<K> p) {
     tile_loop<K, PAIR, 2, 2>(p);
+}
+template <int K, bool PAIR>
+__global__ void __launch_bounds__(256, 2) apply_tci(const __grid_constant__ TileParams<K> p) {
+    tile_loop<K, PAIR, 3, 2>(p);
 }
 
 // Tiny states (fewer amplitudes than one tile can split into thread work):
@@ -822,11 +1109,11 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     // threads: one (GPT = 1) or two (GPT = 2) groups each per compute step
     const int wbits = p.T - K - (gpt == 2 ? 1 : 0);
     const uint32_t work = wbits >= 0 ? (1u << wbits) : 0u;
-    const uint32_t nthr = d.tc ? 128u : std::min<uint32_t>(256, std::max<uint32_t>(32, work));
+    const uint32_t nthr = d.tc ? (d.tci ? 256u : 128u) : std::min<uint32_t>(256, std::max<uint32_t>(32, work));
     p.iters = (int)std::max<uint32_t>(1, work / nthr);
     const uint32_t units = 1u << (p.T - 1);
     p.upt = (int)(units / nthr);
-    if (p.T < K + (gpt == 2 ? 1 : 0) || work < 32 || p.upt < 1 || p.upt > 64 || work < nthr) {
+    if (p.T < K + (gpt == 2 ? 1 : 0) || work < 32 || p.upt < 1 || p.upt > 64 || (work < nthr && !d.tci)) {
         SmallParams<K> sp;
         std::memset(&sp, 0, sizeof(sp));
         sp.psi = psi;
@@ -863,7 +1150,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     size_t smem = (size_t)STG * ((size_t)8 << p.T);
     if (K == 6) smem += 64 * 64 * 8;
     if constexpr (K == 4 || K == 5) {
-        if (d.tc) smem += 2 * TcShape<K>::W_BYTES + 64;
+        if (d.tc) smem += d.tci ? TciShape<K>::SMEM : 2 * TcShape<K>::W_BYTES + 64;
     }
     const int per_sm_smem = std::max(1, (int)((227 * 1024) / (smem + 1024)));
     const uint64_t grid = std::max<uint64_t>(1, std::min<uint64_t>(p.n_tiles, (uint64_t)num_sms() * per_sm_smem));
@@ -875,7 +1162,11 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     };
     if constexpr (K == 4 || K == 5) {
         if (d.tc) {
-            if (p.T != 12 || nthr != 128) return cudaErrorInvalidConfiguration;
+            if (p.T != 12) return cudaErrorInvalidConfiguration;
+            if (d.tci) {
+                p.wi8 = d.dev_wi8;
+                return pair ? go(apply_tci<K, true>) : go(apply_tci<K, false>);
+            }
             return pair ? go(apply_tc<K, true>) : go(apply_tc<K, false>);
         }
     }
@@ -888,6 +1179,46 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
 }
 
 }  // namespace
+
+size_t wi8_bytes(int k) {
+    const int D = 1 << k, KR = 2 * D, N = 2 * D;
+    return (size_t)3 * N * KR + (size_t)N * 4;
+}
+
+void pack_wi8(const ApplyDesc& d, uint8_t* out) {
+    const int D = 1 << d.k, KR = 2 * D, N = 2 * D;
+    const uint32_t SBO = KR * 8, BS = (uint32_t)N * KR;
+    std::memset(out, 0, wi8_bytes(d.k));
+    float* fcol = reinterpret_cast<float*>(out + 3 * BS);
+    for (int n = 0; n < N; ++n) {
+        const int r = n >> 1, ni = n & 1;
+        double w[128];
+        double mx = 0.0;
+        for (int kk = 0; kk < KR; ++kk) {
+            const int c = kk >> 1, ki = kk & 1;
+            const cf m = d.m[(size_t)r * D + c];
+            w[kk] = (ni == 0) ? (ki == 0 ? m.real() : -m.imag()) : (ki == 0 ? m.imag() : m.real());
+            mx = std::max(mx, std::fabs(w[kk]));
+        }
+        int f = 0;
+        std::frexp(mx, &f);  // mx < 2^f
+        f = std::max(f, -100);
+        fcol[n] = std::ldexp(1.0f, f - 14);  // column half of the output scale 2^(e + f - 28)
+        for (int kk = 0; kk < KR; ++kk) {
+            const int32_t wi = (int32_t)std::nearbyint(std::ldexp(w[kk], 22 - f));
+            // balanced signed base-256 digits (as the kernel slices the state)
+            const int32_t d2 = (int32_t)(int8_t)(wi & 0xFF);
+            const int32_t r1 = (wi - d2) >> 8;
+            const int32_t d1 = (int32_t)(int8_t)(r1 & 0xFF);
+            const int32_t d0 = (r1 - d1) >> 8;
+            const uint32_t off = (uint32_t)(n >> 3) * SBO + (uint32_t)(kk >> 4) * 128u + (uint32_t)(n & 7) * 16u +
+                                 (uint32_t)(kk & 15);
+            out[off] = (uint8_t)(d0 & 0xFF);
+            out[BS + off] = (uint8_t)(d1 & 0xFF);
+            out[2 * BS + off] = (uint8_t)(d2 & 0xFF);
+        }
+    }
+}
 
 bool tc_supported(int n_local, const ApplyDesc& d) { return (d.k == 4 || d.k == 5) && n_local >= 13; }
 
@@ -909,15 +1240,19 @@ void plan_apply(int n, ApplyDesc& d) {
             else used |= 1ull << src;
         }
         d.mono = mono;
-        // Opt-in (SVB200_TC=1): the TF32x3 tensor-core path is 2x faster at
-        // k = 5 but its accumulation truncates toward zero, shrinking the norm
-        // by ~4u (k = 4) / ~7u (k = 5) per apply -- over a 40+ gate circuit that
-        // breaks the 1 - 1e-5 fidelity bar.
-        static const bool use_tc = [] {
+        // Tensor cores for dense k = 4, 5 gates.  SVB200_TC selects the path:
+        //   "i8" (exact int8 slices, s32 accumulation; unbiased), "tf32" (TF32x3:
+        //   its accumulation truncates toward zero, shrinking the norm by
+        //   ~4u / ~7u per apply), anything else: SIMT only.
+        static const int tc_mode = [] {
             const char* e = std::getenv("SVB200_TC");
-            return e && e[0] == '1';
+            if (!e) return 0;
+            if (std::strcmp(e, "tf32") == 0 || std::strcmp(e, "1") == 0) return 1;
+            if (std::strcmp(e, "i8") == 0) return 2;
+            return 0;
         }();
-        d.tc = !mono && use_tc && d.nc == 0 && tc_supported(n, d);
+        d.tc = !mono && tc_mode != 0 && d.nc == 0 && tc_supported(n, d);
+        d.tci = d.tc && tc_mode == 2;
     }
     uint64_t gm = 0;
     for (int b = 0; b < d.k; ++b) gm |= 1ull << d.q[b];

@@ -26,7 +26,9 @@ struct ApplyDesc {
     bool mono = false;                // one nonzero per row (exact permutation/diagonal path)
     int nc = 0;                       // control qubits (controlled gate, NEXT-4): only the
     int cq[SV_MAX_FUSED] = {0};       //   amplitudes with every control bit 1 are transformed
-    bool tc = false;                  // tensor-core path (tc.cu)
+    bool tc = false;                  // tensor-core path
+    bool tci = false;                 //   ... exact int8-slice variant (needs dev_wi8)
+    const uint8_t* dev_wi8 = nullptr; // int8 W slices + column exponents (pack_wi8), device
     // low-kernel tile plan (host-computed once)
     int T = 0, r = 0;                 // tile bits, run bits
     // device copy of m for k == 6 (owned by the circuit / state scratch)
@@ -39,6 +41,8 @@ void plan_apply(int n_local, ApplyDesc& d);
 // Dense k = 4, 5 gates run on the tensor cores (tcgen05, TF32 x3) when the
 // shard has at least 2^13 amplitudes.
 bool tc_supported(int n_local, const ApplyDesc& d);
+size_t wi8_bytes(int k);
+void pack_wi8(const ApplyDesc& d, uint8_t* out);
 
 // ---- complex128 states (apply64.cu, NEXT-1) --------------------------------
 struct Apply64Desc {

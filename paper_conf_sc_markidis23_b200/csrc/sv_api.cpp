@@ -63,6 +63,7 @@ struct sv_state {
     bool fp64 = false;        // complex128 amplitudes (NEXT-1)
     size_t elem = 8;          // bytes per amplitude
     double* planes64 = nullptr;   // fp64 scratch: planes of one gate (sv_apply_fused on fp64 states)
+    uint8_t* wi8 = nullptr;       // int8 tensor-core scratch: W slices of one gate (sv_apply_fused)
     int* q64 = nullptr;           // fp64 scratch: qubits of one gate (tiny states)
     cudaStream_t stream = nullptr;
     bool own_stream = false;
@@ -125,6 +126,7 @@ struct sv_circuit {
     std::vector<Step> steps;
     float2* dev_mats = nullptr;
     double* planes64 = nullptr;  // complex128 states: planes of every gate
+    uint8_t* wi8 = nullptr;      // int8 tensor-core W slices of every tensor-core gate
     int* q64 = nullptr;          // complex128 states: qubits of every gate (int[6] each)
     // small states (n <= 13, unsharded): whole circuit in one CTA (small.cu)
     bool small = false;
@@ -404,6 +406,8 @@ int alloc_scratch(sv_state* s) {
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
     e = cudaMalloc(&s->kmat, 64 * 64 * sizeof(float2));
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
+    e = cudaMalloc(&s->wi8, wi8_bytes(5));
+    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
     return SV_OK;
 }
 
@@ -415,7 +419,7 @@ void destroy_state(sv_state* s) {
     for (void* p : {(void*)s->shard_dev, (void*)s->bins, (void*)s->scan_scratch, (void*)s->misc,
                     (void*)s->totals_ptr_dev, (void*)s->sigma_dev, (void*)s->kmat, (void*)s->ctrl, (void*)s->xfer,
                     (void*)s->flags_dev, (void*)s->xfer_dev, (void*)s->idx_dev, (void*)s->amp_dev,
-                    (void*)s->samp_dev, (void*)s->planes64, (void*)s->q64})
+                    (void*)s->samp_dev, (void*)s->planes64, (void*)s->q64, (void*)s->wi8})
         if (p) cudaFree(p);
     for (auto e : s->ev_pool) cudaEventDestroy(e);
     if (s->own_stream && s->stream) cudaStreamDestroy(s->stream);
@@ -633,6 +637,14 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
         CK(s, cudaMemcpyAsync(s->kmat, d.m.data(), 64 * 64 * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
         CK(s, cudaStreamSynchronize(s->stream));
         d.dev_m = s->kmat;
+    }
+    if (d.tci) {
+        std::vector<uint8_t> w(wi8_bytes(k));
+        pack_wi8(d, w.data());
+        CK(s, cudaStreamSynchronize(s->stream));  // the previous tensor-core launch may still read the scratch
+        CK(s, cudaMemcpyAsync(s->wi8, w.data(), w.size(), cudaMemcpyHostToDevice, s->stream));
+        CK(s, cudaStreamSynchronize(s->stream));
+        d.dev_wi8 = s->wi8;
     }
     return run_apply(s, d);
 }
@@ -957,6 +969,30 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
         c->steps.push_back(std::move(st));
     }
+    // int8 tensor-core W slices of every tensor-core gate: one H2D upload
+    {
+        size_t total = 0;
+        for (auto& st : c->steps)
+            if (st.type == Event::APPLY && st.apply.tci) total += wi8_bytes(st.apply.k);
+        if (total) {
+            std::vector<uint8_t> host(total);
+            std::vector<size_t> offs;
+            size_t o = 0;
+            for (auto& st : c->steps)
+                if (st.type == Event::APPLY && st.apply.tci) {
+                    pack_wi8(st.apply, host.data() + o);
+                    offs.push_back(o);
+                    o += wi8_bytes(st.apply.k);
+                }
+            cudaError_t e = cudaMalloc(&c->wi8, total);
+            if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(int8 W slices)");
+            CK(s, cudaMemcpyAsync(c->wi8, host.data(), total, cudaMemcpyHostToDevice, s->stream));
+            CK(s, cudaStreamSynchronize(s->stream));
+            size_t i = 0;
+            for (auto& st : c->steps)
+                if (st.type == Event::APPLY && st.apply.tci) st.apply.dev_wi8 = c->wi8 + offs[i++];
+        }
+    }
     // one H2D upload of all k = 6 matrices (smaller ones travel as kernel params)
     if (n6) {
         cudaError_t e = cudaMalloc(&c->dev_mats, n6 * 64 * 64 * sizeof(float2));
@@ -1072,8 +1108,9 @@ int sv_circuit_stats(const sv_circuit* c, sv_stats* st) {
 
 int sv_circuit_destroy(sv_circuit* c) {
     if (!c) return fail(SV_EINVAL, "circuit is NULL");
-    if (c->dev_mats || c->small_gates || c->small_mats || c->planes64 || c->q64) {
+    if (c->dev_mats || c->small_gates || c->small_mats || c->planes64 || c->q64 || c->wi8) {
         if (c->owner && c->owner->stream) cudaStreamSynchronize(c->owner->stream);
+        if (c->wi8) cudaFree(c->wi8);
         if (c->planes64) cudaFree(c->planes64);
         if (c->q64) cudaFree(c->q64);
         if (c->dev_mats) cudaFree(c->dev_mats);

@@ -1,6 +1,7 @@
-"""Opt-in tensor-core path check (run with SVB200_TC=1): single-apply parity
-for k = 4, 5 against the oracle with the TF32x3 error bound, and the
-measured per-apply norm change (the documented truncation bias)."""
+"""Tensor-core path check (run with SVB200_TC=tf32 or SVB200_TC=i8): single
+apply parity for k = 4, 5 against the oracle and the per-apply norm change.
+The int8 path's slicing error is relative to the group-row / column maximum,
+so its bound adds 2^(k+1) 2^-21 max_c|a| max|M| to the SIMT bound."""
 import os
 import sys
 
@@ -28,7 +29,29 @@ for k, cases in ((4, [(4, 5, 6, 7), (0, 1, 2, 3), (1, 6, 8, 11), (10, 0, 3, 5)])
         sv.sv_destroy(h)
         ref = osv.apply_gate(psi.astype(np.complex128), n, list(qs), M.astype(np.complex128))
         bound = osv.apply_gate(np.abs(psi).astype(np.complex128), n, list(qs), np.abs(M).astype(np.complex128)).real
-        ratio = float((np.abs(got - ref) / (U * bound + 1e-30)).max())
-        worst = max(worst, ratio / (4 * ((1 << k) + 1) + 2))
+        # per-group maximum |a| broadcast back onto the group's members
+        t = np.abs(psi).astype(np.float64).reshape((2,) * n)
+        axes = tuple(n - 1 - q for q in qs)
+        gmax = np.broadcast_to(t.max(axis=axes, keepdims=True) if False else np.max(t, axis=axes, keepdims=True),
+                               t.shape).reshape(-1)
+        slack = (4 * ((1 << k) + 1) + 2) * U * bound + (2 << k) * 2.0 ** -21 * gmax * np.abs(M).max()
+        worst = max(worst, float((np.abs(got - ref) / (slack + 1e-30)).max()))
         drift.append(float(np.vdot(got, got).real - np.vdot(ref, ref).real))
 print(f"TC_CHECK worst_error_over_bound={worst:.3f} mean_norm_change_per_apply={np.mean(drift):+.3e}")
+
+# whole circuits from |0..0> (many all-zero group rows early on) at F = 4, 5
+from oracle import ref_c
+
+cworst = 0.0
+for nq, depth, F in ((20, 14, 5), (20, 14, 4), (18, 20, 5)):
+    gates = W.rqc(nq, depth, 2023)
+    ref = ref_c.run(nq, gates)
+    h = sv.sv_create(nq)
+    sv.sv_run_circuit(h, gates, F)
+    got = sv.sv_get_state(h, nq).astype(np.complex128)
+    sv.sv_destroy(h)
+    fid = osv.fidelity(got, ref)
+    err = float(np.abs(got - ref).max())
+    cworst = max(cworst, err / osv.max_abs_bound(nq, depth))
+    assert np.isfinite(got).all() and fid >= 1 - 1e-5, (nq, F, fid)
+print(f"TC_CIRCUIT worst_error_over_northstar_bound={cworst:.3f}")
