@@ -1,4 +1,4 @@
 python -c "import __graft_entry__ as g; g.build()" > /dev/null
-SVB200_TC=i8 python tools/tc_check.py
-SVB200_TC=i8 timeout 300 python tools/prof_apply.py 30 5 h4 l4 q0 h5 l5 2>&1
-SVB200_TC=i8 timeout 600 ncu --set full --import-source on --clock-control none -k regex:apply_tci -s 1 -c 1 -o gpurun_out/prof_tci python tools/prof_apply.py 30 1 h5 > /dev/null 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -5
+for F in 4 5; do timeout 300 python bench.py --max-fused $F --no-cpu-baseline --steps 5 --warmup 3 2>&1 | tail -1; done
+timeout 300 python bench.py --qubits 32 --depth 20 --max-fused 5 --no-cpu-baseline --steps 3 --warmup 3 2>&1 | tail -1

@@ -96,7 +96,7 @@ struct alignas(16) TileParams {
     uint64_t ones;                     // control qubits forced to 1 in the tile base
     int upt;                           // 16-byte units per thread per tile
     int iters;                         // compute iterations per thread per tile
-    uint64_t goff[64];                 // dep(2 * nthreads * i)
+    uint64_t goff[64];                 // 8 * dep(2 * nthreads * i)  (bytes)
     uint32_t soff[64];                 // phys(2 * nthreads * i)
     uint32_t loc[1 << K];              // phys offsets of the gathers (members / member pairs)
     uint32_t gsec;                     // phys offset of the second group of a pair (PAIR, 2 groups)
@@ -860,25 +860,35 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
     }
     const uint32_t sthr = swizzle(t0, p.swz);
     const int upt = p.upt;
-    auto load = [&](uint64_t u, uint32_t sbuf) {
-        const float2* g = p.psi + tile_base(p, u) + dthr;
-        for (int i = 0; i < upt; ++i) cp_async16(sbuf + ((sthr ^ p.soff[i]) << 3), g + p.goff[i]);
-    };
-    auto store = [&](uint64_t u, uint32_t sbuf) {
-        float2* g = p.psi + tile_base(p, u) + dthr;
+    // byte address of this thread's first unit of tile u (computed once per
+    // tile: the same address serves the load and the store)
+    auto gaddr = [&](uint64_t u) { return reinterpret_cast<const char*>(p.psi + tile_base(p, u) + dthr); };
+    auto load = [&](const char* g, uint32_t sbuf) {
         for (int i = 0; i < upt; ++i)
-            st_stream(reinterpret_cast<float4*>(g + p.goff[i]), lds4(sbuf + ((sthr ^ p.soff[i]) << 3)));
+            cp_async16(sbuf + ((sthr ^ p.soff[i]) << 3), reinterpret_cast<const float2*>(g + p.goff[i]));
+    };
+    auto store = [&](const char* g, uint32_t sbuf) {
+        for (int i = 0; i < upt; ++i)
+            st_stream(reinterpret_cast<float4*>(const_cast<char*>(g) + p.goff[i]), lds4(sbuf + ((sthr ^ p.soff[i]) << 3)));
     };
     uint64_t u = blockIdx.x;
     if constexpr (STAGES == 2) {
-        if (u < p.n_tiles) load(u, s0);
+        const char* gcur = nullptr;
+        if (u < p.n_tiles) {
+            gcur = gaddr(u);
+            load(gcur, s0);
+        }
         cp_async_commit();
         for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
             const uint32_t cur = s0 + (uint32_t)(it & 1) * tile_bytes;
             const uint32_t nxt = s0 + (uint32_t)((it + 1) & 1) * tile_bytes;
             const uint64_t un = u + gridDim.x;
+            const char* gnext = nullptr;
             __syncthreads();  // buffer `nxt` was drained by the previous iteration's store
-            if (un < p.n_tiles) load(un, nxt);
+            if (un < p.n_tiles) {
+                gnext = gaddr(un);
+                load(gnext, nxt);
+            }
             cp_async_commit();
             cp_async_wait1();  // this thread's copies of tile u have landed
             __syncthreads();   // ... and everyone else's
@@ -887,21 +897,23 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             else if constexpr (MODE == 3 && K <= 5) tile_compute_tci<K, PAIR>(p, cur, tis);
             else tile_compute<K, PAIR>(p, cur, smat);
             __syncthreads();
-            store(u, cur);
+            store(gcur, cur);
+            gcur = gnext;
         }
         if constexpr (MODE == 2 && K <= 5) tc_teardown<K>(tcs);
         if constexpr (MODE == 3 && K <= 5) tci_teardown<K>(tis);
     } else {
         for (; u < p.n_tiles; u += gridDim.x) {
             __syncthreads();
-            load(u, s0);
+            const char* g = gaddr(u);
+            load(g, s0);
             cp_async_commit();
             cp_async_wait0();
             __syncthreads();
             if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, s0);
             else tile_compute<K, PAIR>(p, s0, smat);
             __syncthreads();
-            store(u, s0);
+            store(g, s0);
         }
     }
 }
@@ -1132,7 +1144,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         return cudaGetLastError();
     }
     for (int i = 0; i < p.upt; ++i) {
-        p.goff[i] = dep(2ull * nthr * i);
+        p.goff[i] = 8ull * dep(2ull * nthr * i);
         p.soff[i] = sw(2u * nthr * i);
     }
     {
@@ -1241,18 +1253,22 @@ void plan_apply(int n, ApplyDesc& d) {
         }
         d.mono = mono;
         // Tensor cores for dense k = 4, 5 gates.  SVB200_TC selects the path:
-        //   "i8" (exact int8 slices, s32 accumulation; unbiased), "tf32" (TF32x3:
-        //   its accumulation truncates toward zero, shrinking the norm by
-        //   ~4u / ~7u per apply), anything else: SIMT only.
+        //   unset / "auto": k = 5 on the exact int8-slice tensor-core path
+        //     (2.2x faster than SIMT k = 5, which is FP32-issue bound), k <= 4
+        //     SIMT (HBM-bound or close to it);
+        //   "i8": the int8 path for k = 4 and 5; "tf32": TF32x3 for k = 4, 5
+        //     (its accumulation truncates toward zero, shrinking the norm by
+        //     ~4u / ~7u per apply); "simt" / "0": SIMT only.
         static const int tc_mode = [] {
             const char* e = std::getenv("SVB200_TC");
-            if (!e) return 0;
+            if (!e || std::strcmp(e, "auto") == 0) return 3;
             if (std::strcmp(e, "tf32") == 0 || std::strcmp(e, "1") == 0) return 1;
             if (std::strcmp(e, "i8") == 0) return 2;
             return 0;
         }();
-        d.tc = !mono && tc_mode != 0 && d.nc == 0 && tc_supported(n, d);
-        d.tci = d.tc && tc_mode == 2;
+        const bool want = tc_mode == 1 || tc_mode == 2 || (tc_mode == 3 && d.k == 5);
+        d.tc = !mono && want && d.nc == 0 && tc_supported(n, d);
+        d.tci = d.tc && tc_mode != 1;
     }
     uint64_t gm = 0;
     for (int b = 0; b < d.k; ++b) gm |= 1ull << d.q[b];
