@@ -62,6 +62,8 @@ def parse():
     ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
     ap.add_argument("--precision", type=int, default=32, choices=[32, 64], help="complex64 (32) or complex128 (64) state")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true",
+                    help="skip the max_fused = 1..6 sweep (N = 1) that reports the optimal fusion")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
 
@@ -296,6 +298,31 @@ def run_ours(args):
     e2e_ms = float(et.item())
     h2d = int(sum(8 * (1 << (2 * k)) * c for k, c in enumerate(cst["fused_hist"])))
 
+    # ---- fusion sweep (N = 1): the same device step for max_fused = 1..6,
+    # CUDA events on the launching stream, 1 warm-up + 3 timed steps each
+    sweep = None
+    if world == 1 and not args.no_sweep and not fp64:
+        sweep = {}
+        for f in range(1, 7):
+            c = sv.sv_circuit_create(h, gates, f)
+
+            def st_f():
+                sv.sv_reset(h)
+                sv.sv_circuit_run_device(h, c)
+                sv.sv_sample_device(h, 1, args.samples, samples_dev.data_ptr())
+
+            st_f()
+            barrier()
+            a0 = torch.cuda.Event(enable_timing=True)
+            a1 = torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            for _ in range(3):
+                st_f()
+            a1.record(stream)
+            barrier()
+            sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
+            sv.sv_circuit_destroy(c)
+
     peak, peak_src = load_peaks()
     launches_apply = n_high + n_low
     avg_launch = t_apply / max(launches_apply, 1)
@@ -353,6 +380,9 @@ def run_ours(args):
             "e2e": {"value": e2e_ms / 1e3, "unit": "s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": 8 * args.samples},
             "gpu_launches": (n_high + n_low + n_other),
+            "fusion_sweep_s": sweep,
+            "optimal_fusion": (None if not sweep else
+                               {"max_fused": int(min(sweep, key=sweep.get)), "value": min(sweep.values()), "unit": "s"}),
             "clocks": clk.summary(),
         }
         print(json.dumps(out), flush=True)

@@ -1,4 +1,5 @@
 python -c "import __graft_entry__ as g; g.build()" > /dev/null
-timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -5
-for F in 4 5; do timeout 300 python bench.py --max-fused $F --no-cpu-baseline --steps 5 --warmup 3 2>&1 | tail -1; done
-timeout 300 python bench.py --qubits 32 --depth 20 --max-fused 5 --no-cpu-baseline --steps 3 --warmup 3 2>&1 | tail -1
+timeout 600 python tools/tc_check.py
+timeout 300 python tools/prof_apply.py 30 5 h5 h6 l6 2>&1
+SVB200_TC=simt timeout 300 python tools/prof_apply.py 30 3 h6 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:apply_tci -s 1 -c 1 -o gpurun_out/prof_tci6 python tools/prof_apply.py 30 1 h6 > /dev/null 2>&1

@@ -567,18 +567,28 @@ __device__ __forceinline__ void tile_compute_tc(const TileParams<K>& p, uint32_t
 // scaled by 2^(e_r + f_n - 28) (exact).
 // Operand A (slices) and B (W slices) live in shared memory in the K-major
 // SWIZZLE_NONE canonical layout (core matrix 8 rows x 16 B), D in TMEM.
+__host__ __device__ constexpr int tci_threads(int K) { return K == 6 ? 512 : 256; }
+
 template <int K>
 struct TciShape {
     static constexpr int D = 1 << K;
     static constexpr int KR = 2 * D;                  // MMA K (reals per group)
     static constexpr int N = 2 * D;                   // MMA N
-    static constexpr int MB = (1 << (12 - K)) / 128;  // M-blocks of 128 groups per 2^12 tile
+    static constexpr int T = K == 6 ? 13 : 12;        // tile bits
+    static constexpr int MB = (1 << (T - K)) / 128;   // M-blocks of 128 groups per tile
+    static constexpr int TPR = K == 6 ? 4 : 2;        // threads per MMA row (k = 6: 1 CTA/SM -> 16 warps)
+    static constexpr int THREADS = 128 * TPR;
+    static_assert(THREADS == tci_threads(K), "thread count");
+    // k = 6: the A slices are written into the current tile buffer once its
+    // amplitudes are in registers (the MMA is complete before the epilogue
+    // writes the outputs there), saving 48 KB of shared memory
+    static constexpr bool A_IN_TILE = K == 6;
     static constexpr int KS = KR / 32;                // int8 MMA K-steps (K = 32)
     static constexpr uint32_t SBO = KR * 8;           // byte distance between row octets (KR/16 chunks x 128 B)
     static constexpr uint32_t A_SLICE = 128u * MB * KR;  // bytes of one A slice
     static constexpr uint32_t B_SLICE = (uint32_t)N * KR;
-    static constexpr uint32_t ROWMAX = 2 * 128 * MB * 4;  // half-row maxima exchange
-    static constexpr uint32_t SMEM = 3 * A_SLICE + 3 * B_SLICE + N * 4 + ROWMAX + 64;
+    static constexpr uint32_t ROWMAX = 4 * 128 * MB * 4;  // part-row maxima exchange (TPR <= 4)
+    static constexpr uint32_t SMEM = (A_IN_TILE ? 0u : 3 * A_SLICE) + 3 * B_SLICE + N * 4 + ROWMAX + 64;
     static constexpr int NACC = 3;                    // S32, S24, S16
     static constexpr int COLS = NACC * N * MB;
     static constexpr int ALLOC = COLS <= 32 ? 32 : COLS <= 64 ? 64 : COLS <= 128 ? 128 : COLS <= 256 ? 256 : 512;
@@ -597,6 +607,7 @@ __device__ __forceinline__ void mma_i8_ss(uint32_t d_tmem, uint64_t adesc, uint6
         : "memory");
 }
 
+
 struct TciState {
     uint32_t tmem, sA, sB, sF, sM, bar, phase;
 };
@@ -606,7 +617,7 @@ __device__ __forceinline__ TciState tci_setup(const TileParams<K>& p, uint32_t s
     using S = TciShape<K>;
     TciState t;
     t.sA = sBase;
-    t.sB = sBase + 3 * S::A_SLICE;
+    t.sB = sBase + (S::A_IN_TILE ? 0u : 3 * S::A_SLICE);
     t.sF = t.sB + 3 * S::B_SLICE;
     t.sM = t.sF + S::N * 4;
     t.bar = t.sM + S::ROWMAX;
@@ -677,22 +688,28 @@ __device__ __forceinline__ void sts128u(uint32_t a, uint4 v) {
     asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
-// Two threads per MMA row (256 threads): thread h = threadIdx.x / 128 of row
-// r = threadIdx.x % 128 gathers and slices members [h D/2, (h+1) D/2) and
-// later combines output columns [h N/2, (h+1) N/2); warps 4..7 read the same
-// TMEM lane quarters as warps 0..3.
+// TPR threads per MMA row (128 TPR threads; TPR = 2 for k <= 5 -- 4 measured
+// slower there -- and 4 for k = 6): thread part p = threadIdx.x / 128
+// of row r = threadIdx.x % 128 gathers and slices members [p D/TPR,
+// (p+1) D/TPR) and later combines output columns [p N/TPR, (p+1) N/TPR);
+// warps w and w + 4j read the same TMEM lane quarter (w % 4).
 template <int K, bool PAIR>
 __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_t sbuf, TciState& t) {
     using S = TciShape<K>;
+    constexpr int TPR = S::TPR;
     constexpr int D = S::D;
-    constexpr int HM = D / 2;  // members per thread
-    const int half = threadIdx.x >> 7;
+    const uint32_t sA = S::A_IN_TILE ? sbuf : t.sA;
+    constexpr int HM = D / TPR;   // members per thread
+    constexpr int RPT = 2 * HM;   // reals per thread (8 or 16)
+    constexpr int NPT = S::N / TPR;  // output columns per thread
+    static_assert(RPT == 8 || RPT % 16 == 0, "slice granularity");
+    const int part = threadIdx.x >> 7;
     const uint32_t row = threadIdx.x & 127u;
     const uint32_t lane_base = (uint32_t)(((threadIdx.x >> 5) & 3) * 32) << 16;
     float srow[S::MB];
-    float x[S::MB][2 * HM];
+    float x[S::MB][RPT];
     uint32_t pbs[S::MB];
-    // 1a. gather this thread's half row, publish the half maximum
+    // 1a. gather this thread's part of the row, publish the part maximum
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
         const uint32_t g = (uint32_t)mb * 128u + row;
@@ -700,7 +717,7 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
         pbs[mb] = pb;
 #pragma unroll
         for (int j = 0; j < HM / 2; ++j) {
-            const int jj = half * (HM / 2) + j;  // member pair (2jj, 2jj+1)
+            const int jj = part * (HM / 2) + j;  // member pair (2jj, 2jj+1)
             if constexpr (PAIR) {
                 const float4 v = lds4(sbuf + ((pb ^ p.loc[jj]) << 3));
                 x[mb][4 * j] = v.x; x[mb][4 * j + 1] = v.y; x[mb][4 * j + 2] = v.z; x[mb][4 * j + 3] = v.w;
@@ -712,37 +729,55 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
         }
         float mx = 0.f;
 #pragma unroll
-        for (int i = 0; i < 2 * HM; ++i) mx = fmaxf(mx, fabsf(x[mb][i]));
-        asm volatile("st.shared.f32 [%0], %1;" ::"r"(t.sM + 4u * ((uint32_t)mb * 256u + threadIdx.x)), "f"(mx)
+        for (int i = 0; i < RPT; ++i) mx = fmaxf(mx, fabsf(x[mb][i]));
+        asm volatile("st.shared.f32 [%0], %1;" ::"r"(t.sM + 4u * ((uint32_t)mb * (128u * TPR) + threadIdx.x)), "f"(mx)
                      : "memory");
     }
     __syncthreads();
     // 1b. row scale 2^(22 - e) with max|x| < 2^e; slice into A (shared memory)
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
-        float m0, m1;
-        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(m0) : "r"(t.sM + 4u * ((uint32_t)mb * 256u + row)));
-        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(m1) : "r"(t.sM + 4u * ((uint32_t)mb * 256u + 128u + row)));
-        const float mx = fmaxf(m0, m1);
+        float mx = 0.f;
+#pragma unroll
+        for (int q = 0; q < TPR; ++q) {
+            float m;
+            asm volatile("ld.shared.f32 %0, [%1];"
+                         : "=f"(m)
+                         : "r"(t.sM + 4u * ((uint32_t)mb * (128u * TPR) + (uint32_t)q * 128u + row)));
+            mx = fmaxf(mx, m);
+        }
         const int e = max(((int)(__float_as_uint(mx) >> 23) & 0xFF) - 126, -100);  // mx < 2^e
         srow[mb] = __uint_as_float((uint32_t)(127 + e - 14) << 23);                 // 2^(e - 14)
         const float scale = __uint_as_float((uint32_t)(127 + 22 - e) << 23);
         const uint32_t rbase = (uint32_t)mb * 128u * S::KR + (row >> 3) * S::SBO + (row & 7) * 16u;
-#pragma unroll
-        for (int c = 0; c < HM / 8; ++c) {  // 16 reals per chunk
+        if constexpr (RPT == 8) {
             uint4 s0, s1, s2;
-            slice16(x[mb] + 16 * c, scale, s0, s1, s2);
-            const uint32_t a = t.sA + rbase + (uint32_t)(half * (HM / 8) + c) * 128u;
-            sts128u(a, s0);
-            sts128u(a + S::A_SLICE, s1);
-            sts128u(a + 2 * S::A_SLICE, s2);
+            float xx[16];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) { xx[i] = x[mb][i]; xx[8 + i] = 0.f; }
+            slice16(xx, scale, s0, s1, s2);
+            const uint32_t a = sA + rbase + (uint32_t)(part >> 1) * 128u + (uint32_t)(part & 1) * 8u;
+            asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(a), "r"(s0.x), "r"(s0.y) : "memory");
+            asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(a + S::A_SLICE), "r"(s1.x), "r"(s1.y) : "memory");
+            asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(a + 2 * S::A_SLICE), "r"(s2.x), "r"(s2.y)
+                         : "memory");
+        } else {
+#pragma unroll
+            for (int c = 0; c < RPT / 16; ++c) {  // 16 reals per chunk
+                uint4 s0, s1, s2;
+                slice16(x[mb] + 16 * c, scale, s0, s1, s2);
+                const uint32_t a = sA + rbase + (uint32_t)(part * (RPT / 16) + c) * 128u;
+                sts128u(a, s0);
+                sts128u(a + S::A_SLICE, s1);
+                sts128u(a + 2 * S::A_SLICE, s2);
+            }
         }
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
-    // 2. eight int8 MMAs per K-step into four exact s32 accumulators
+    // 2. six int8 MMAs per K-step into three exact s32 accumulators
     if (threadIdx.x == 0) {
         constexpr uint32_t i_ss = umma_idesc_i8(S::N, true, true);
 #pragma unroll
@@ -751,7 +786,7 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
             const uint32_t d32 = d0, d24 = d0 + S::N, d16 = d0 + 2 * S::N;
 #pragma unroll
             for (int ks = 0; ks < S::KS; ++ks) {
-                const uint32_t ao = t.sA + (uint32_t)mb * 128u * S::KR + (uint32_t)ks * 256u;
+                const uint32_t ao = sA + (uint32_t)mb * 128u * S::KR + (uint32_t)ks * 256u;
                 const uint32_t bo = t.sB + (uint32_t)ks * 256u;
                 const uint64_t a0 = umma_desc(ao, 128, S::SBO), a1 = umma_desc(ao + S::A_SLICE, 128, S::SBO),
                                a2 = umma_desc(ao + 2 * S::A_SLICE, 128, S::SBO);
@@ -772,13 +807,13 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
     mbar_wait(t.bar, t.phase);
     t.phase ^= 1u;
     tc_fence_after();
-    // 3. exact recombination of this thread's half of the columns, one rounding
+    // 3. exact recombination of this thread's columns, one rounding
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
         const uint32_t pb = pbs[mb];
         const uint32_t d0 = t.tmem + lane_base + (uint32_t)(mb * S::NACC * S::N);
 #pragma unroll 1
-        for (int c0 = half * (S::N / 2); c0 < (half + 1) * (S::N / 2); c0 += 8) {
+        for (int c0 = part * NPT; c0 < (part + 1) * NPT; c0 += 8) {
             uint32_t v32[8], v24[8], v16[8];
             tmem_ld8(d0 + (uint32_t)c0, v32);
             tmem_ld8(d0 + (uint32_t)(S::N + c0), v24);
@@ -835,14 +870,14 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
     const uint32_t tile_bytes = 8u << p.T;
     const uint32_t s0 = smem_addr(dsm);
     const float2* smat = nullptr;
-    if constexpr (K == 6) {
+    if constexpr (K == 6 && MODE != 3) {
         float2* sm = reinterpret_cast<float2*>(reinterpret_cast<char*>(dsm) + STAGES * tile_bytes);
         for (int i = threadIdx.x; i < 64 * 64; i += blockDim.x) sm[i] = p.M.dev[i];
         smat = sm;
         __syncthreads();
     }
     TciState tis{};
-    if constexpr (MODE == 3 && K <= 5) tis = tci_setup<K>(p, s0 + STAGES * tile_bytes);
+    if constexpr (MODE == 3) tis = tci_setup<K>(p, s0 + STAGES * tile_bytes);
     TcState tcs{};
     if constexpr (MODE == 2 && K <= 5) {
         const uint32_t sW = s0 + STAGES * tile_bytes;
@@ -894,14 +929,14 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             __syncthreads();   // ... and everyone else's
             if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, cur);
             else if constexpr (MODE == 2 && K <= 5) tile_compute_tc<K, PAIR>(p, cur, tcs);
-            else if constexpr (MODE == 3 && K <= 5) tile_compute_tci<K, PAIR>(p, cur, tis);
+            else if constexpr (MODE == 3) tile_compute_tci<K, PAIR>(p, cur, tis);
             else tile_compute<K, PAIR>(p, cur, smat);
             __syncthreads();
             store(gcur, cur);
             gcur = gnext;
         }
         if constexpr (MODE == 2 && K <= 5) tc_teardown<K>(tcs);
-        if constexpr (MODE == 3 && K <= 5) tci_teardown<K>(tis);
+        if constexpr (MODE == 3) tci_teardown<K>(tis);
     } else {
         for (; u < p.n_tiles; u += gridDim.x) {
             __syncthreads();
@@ -939,7 +974,7 @@ __global__ void __launch_bounds__(128, 1) apply_tc(const __grid_constant__ TileP
     tile_loop<K, PAIR, 2, 2>(p);
 }
 template <int K, bool PAIR>
-__global__ void __launch_bounds__(256, 2) apply_tci(const __grid_constant__ TileParams<K> p) {
+__global__ void __launch_bounds__(TciShape<K>::THREADS, K == 6 ? 1 : 2) apply_tci(const __grid_constant__ TileParams<K> p) {
     tile_loop<K, PAIR, 3, 2>(p);
 }
 
@@ -1121,7 +1156,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     // threads: one (GPT = 1) or two (GPT = 2) groups each per compute step
     const int wbits = p.T - K - (gpt == 2 ? 1 : 0);
     const uint32_t work = wbits >= 0 ? (1u << wbits) : 0u;
-    const uint32_t nthr = d.tc ? (d.tci ? 256u : 128u) : std::min<uint32_t>(256, std::max<uint32_t>(32, work));
+    const uint32_t nthr = d.tc ? (d.tci ? tci_threads(K) : 128u) : std::min<uint32_t>(256, std::max<uint32_t>(32, work));
     p.iters = (int)std::max<uint32_t>(1, work / nthr);
     const uint32_t units = 1u << (p.T - 1);
     p.upt = (int)(units / nthr);
@@ -1160,9 +1195,12 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     p.n_tiles = 1ull << (n - p.T - d.nc);
     const int STG = d.tc ? 2 : stages_for(K);
     size_t smem = (size_t)STG * ((size_t)8 << p.T);
-    if (K == 6) smem += 64 * 64 * 8;
+    if (K == 6 && !d.tci) smem += 64 * 64 * 8;
+    if constexpr (K >= 4) {
+        if (d.tci) smem += TciShape<K>::SMEM;
+    }
     if constexpr (K == 4 || K == 5) {
-        if (d.tc) smem += d.tci ? TciShape<K>::SMEM : 2 * TcShape<K>::W_BYTES + 64;
+        if (d.tc && !d.tci) smem += 2 * TcShape<K>::W_BYTES + 64;
     }
     const int per_sm_smem = std::max(1, (int)((227 * 1024) / (smem + 1024)));
     const uint64_t grid = std::max<uint64_t>(1, std::min<uint64_t>(p.n_tiles, (uint64_t)num_sms() * per_sm_smem));
@@ -1172,13 +1210,16 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         kern<<<(unsigned)grid, nthr, smem, st>>>(p);
         return cudaGetLastError();
     };
+    if constexpr (K >= 4) {
+        if (d.tci) {
+            if (p.T != TciShape<K>::T) return cudaErrorInvalidConfiguration;
+            p.wi8 = d.dev_wi8;
+            return pair ? go(apply_tci<K, true>) : go(apply_tci<K, false>);
+        }
+    }
     if constexpr (K == 4 || K == 5) {
         if (d.tc) {
             if (p.T != 12) return cudaErrorInvalidConfiguration;
-            if (d.tci) {
-                p.wi8 = d.dev_wi8;
-                return pair ? go(apply_tci<K, true>) : go(apply_tci<K, false>);
-            }
             return pair ? go(apply_tc<K, true>) : go(apply_tc<K, false>);
         }
     }
@@ -1232,7 +1273,9 @@ void pack_wi8(const ApplyDesc& d, uint8_t* out) {
     }
 }
 
-bool tc_supported(int n_local, const ApplyDesc& d) { return (d.k == 4 || d.k == 5) && n_local >= 13; }
+bool tc_supported(int n_local, const ApplyDesc& d) {
+    return ((d.k == 4 || d.k == 5) && n_local >= 13) || (d.k == 6 && n_local >= 14);
+}
 
 void plan_apply(int n, ApplyDesc& d) {
     {
@@ -1253,10 +1296,10 @@ void plan_apply(int n, ApplyDesc& d) {
         }
         d.mono = mono;
         // Tensor cores for dense k = 4, 5 gates.  SVB200_TC selects the path:
-        //   unset / "auto": k = 5 on the exact int8-slice tensor-core path
-        //     (2.2x faster than SIMT k = 5, which is FP32-issue bound), k <= 4
-        //     SIMT (HBM-bound or close to it);
-        //   "i8": the int8 path for k = 4 and 5; "tf32": TF32x3 for k = 4, 5
+        //   unset / "auto": k = 5, 6 on the exact int8-slice tensor-core path
+        //     (SIMT k = 5, 6 are FP32-issue bound), k <= 4 SIMT (HBM-bound or
+        //     close to it);
+        //   "i8": the int8 path for k = 4..6; "tf32": TF32x3 for k = 4, 5
         //     (its accumulation truncates toward zero, shrinking the norm by
         //     ~4u / ~7u per apply); "simt" / "0": SIMT only.
         static const int tc_mode = [] {
@@ -1266,7 +1309,7 @@ void plan_apply(int n, ApplyDesc& d) {
             if (std::strcmp(e, "i8") == 0) return 2;
             return 0;
         }();
-        const bool want = tc_mode == 1 || tc_mode == 2 || (tc_mode == 3 && d.k == 5);
+        const bool want = (tc_mode == 1 && d.k <= 5) || tc_mode == 2 || (tc_mode == 3 && d.k >= 5);
         d.tc = !mono && want && d.nc == 0 && tc_supported(n, d);
         d.tci = d.tc && tc_mode != 1;
     }
@@ -1275,7 +1318,7 @@ void plan_apply(int n, ApplyDesc& d) {
     d.high = (gm & kLowMask) == 0;
     // tile: runs of >= 16 amplitudes (128 B); grow the run until the tile
     // reaches the target size (32 KB for k <= 4).
-    const int target = std::min(n, d.k <= 5 ? 12 : 14);
+    const int target = std::min(n, d.k <= 5 ? 12 : (d.tci ? 13 : 14));
     auto tile_bits = [&](int rr) {
         int t = rr;
         for (int b = 0; b < d.k; ++b)

@@ -406,7 +406,7 @@ int alloc_scratch(sv_state* s) {
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
     e = cudaMalloc(&s->kmat, 64 * 64 * sizeof(float2));
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
-    e = cudaMalloc(&s->wi8, wi8_bytes(5));
+    e = cudaMalloc(&s->wi8, wi8_bytes(6));
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
     return SV_OK;
 }

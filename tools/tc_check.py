@@ -1,5 +1,6 @@
-"""Tensor-core path check (run with SVB200_TC=tf32 or SVB200_TC=i8): single
-apply parity for k = 4, 5 against the oracle and the per-apply norm change.
+"""Tensor-core path check (run with SVB200_TC=tf32, i8 or auto): single
+apply parity for k = 4, 5, 6 against the oracle and the per-apply norm change
+(k = 6 runs on the tensor cores with i8 / auto only; with tf32 it is SIMT).
 The int8 path's slicing error is relative to the group-row / column maximum,
 so its bound adds 2^(k+1) 2^-21 max_c|a| max|M| to the SIMT bound."""
 import os
@@ -17,7 +18,8 @@ n = 16
 worst = 0.0
 drift = []
 for k, cases in ((4, [(4, 5, 6, 7), (0, 1, 2, 3), (1, 6, 8, 11), (10, 0, 3, 5)]),
-                 (5, [(4, 5, 6, 8, 10), (0, 1, 2, 3, 4), (11, 0, 6, 2, 8)])):
+                 (5, [(4, 5, 6, 8, 10), (0, 1, 2, 3, 4), (11, 0, 6, 2, 8)]),
+                 (6, [(4, 5, 6, 7, 8, 9), (0, 1, 2, 3, 4, 5), (13, 0, 7, 2, 9, 4), (1, 3, 8, 10, 12, 15)])):
     for i, qs in enumerate(cases):
         rs = np.random.default_rng(100 + 10 * k + i)
         M = W.haar_unitary(1 << k, rs).astype(np.complex64)
@@ -47,7 +49,7 @@ if os.environ.get("SVB200_TC") in ("1", "tf32"):
     sys.exit(0)
 
 cworst = 0.0
-for nq, depth, F in ((20, 14, 5), (20, 14, 4), (18, 20, 5)):
+for nq, depth, F in ((20, 14, 5), (20, 14, 4), (18, 20, 5), (20, 14, 6), (18, 20, 6)):
     gates = W.rqc(nq, depth, 2023)
     ref = ref_c.run(nq, gates)
     h = sv.sv_create(nq)
