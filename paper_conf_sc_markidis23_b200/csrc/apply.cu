@@ -579,10 +579,13 @@ struct TciShape {
     static constexpr int TPR = K == 6 ? 4 : 2;        // threads per MMA row (k = 6: 1 CTA/SM -> 16 warps)
     static constexpr int THREADS = 128 * TPR;
     static_assert(THREADS == tci_threads(K), "thread count");
-    // k = 6: the A slices are written into the current tile buffer once its
+    // The A slices are written into the current tile buffer once its
     // amplitudes are in registers (the MMA is complete before the epilogue
-    // writes the outputs there), saving 48 KB of shared memory
-    static constexpr bool A_IN_TILE = K == 6;
+    // writes the outputs there): 3 x 128 MB KR bytes <= 3/4 of the tile.
+    static constexpr bool A_IN_TILE = true;
+    // k <= 5: three tile buffers (store of tile i-1 overlaps the MMAs of tile
+    // i, load of tile i+2 in flight); k = 6 (64 KB tiles): two.
+    static constexpr int STAGES = K == 6 ? 2 : 3;
     static constexpr int KS = KR / 32;                // int8 MMA K-steps (K = 32)
     static constexpr uint32_t SBO = KR * 8;           // byte distance between row octets (KR/16 chunks x 128 B)
     static constexpr uint32_t A_SLICE = 128u * MB * KR;  // bytes of one A slice
@@ -693,28 +696,33 @@ __device__ __forceinline__ void sts128u(uint32_t a, uint4 v) {
 // of row r = threadIdx.x % 128 gathers and slices members [p D/TPR,
 // (p+1) D/TPR) and later combines output columns [p N/TPR, (p+1) N/TPR);
 // warps w and w + 4j read the same TMEM lane quarter (w % 4).
+template <int MB>
+struct TciRows {
+    float srow[MB];    // 2^(e - 14) per M-block row
+    uint32_t pbs[MB];  // phys offset of the row's group
+};
+
+// Phase A: gather, slice, issue the MMAs (asynchronous; completion is
+// signalled on t.bar).
 template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_t sbuf, TciState& t) {
+__device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbuf, TciState& t,
+                                            TciRows<TciShape<K>::MB>& rw) {
     using S = TciShape<K>;
     constexpr int TPR = S::TPR;
     constexpr int D = S::D;
     const uint32_t sA = S::A_IN_TILE ? sbuf : t.sA;
     constexpr int HM = D / TPR;   // members per thread
     constexpr int RPT = 2 * HM;   // reals per thread (8 or 16)
-    constexpr int NPT = S::N / TPR;  // output columns per thread
     static_assert(RPT == 8 || RPT % 16 == 0, "slice granularity");
     const int part = threadIdx.x >> 7;
     const uint32_t row = threadIdx.x & 127u;
-    const uint32_t lane_base = (uint32_t)(((threadIdx.x >> 5) & 3) * 32) << 16;
-    float srow[S::MB];
     float x[S::MB][RPT];
-    uint32_t pbs[S::MB];
     // 1a. gather this thread's part of the row, publish the part maximum
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
         const uint32_t g = (uint32_t)mb * 128u + row;
         const uint32_t pb = swizzle((uint32_t)insert_zeros(g, p.ztpos, p.nzt), p.swz);
-        pbs[mb] = pb;
+        rw.pbs[mb] = pb;
 #pragma unroll
         for (int j = 0; j < HM / 2; ++j) {
             const int jj = part * (HM / 2) + j;  // member pair (2jj, 2jj+1)
@@ -747,7 +755,7 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
             mx = fmaxf(mx, m);
         }
         const int e = max(((int)(__float_as_uint(mx) >> 23) & 0xFF) - 126, -100);  // mx < 2^e
-        srow[mb] = __uint_as_float((uint32_t)(127 + e - 14) << 23);                 // 2^(e - 14)
+        rw.srow[mb] = __uint_as_float((uint32_t)(127 + e - 14) << 23);                 // 2^(e - 14)
         const float scale = __uint_as_float((uint32_t)(127 + 22 - e) << 23);
         const uint32_t rbase = (uint32_t)mb * 128u * S::KR + (row >> 3) * S::SBO + (row & 7) * 16u;
         if constexpr (RPT == 8) {
@@ -804,39 +812,58 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(t.bar)
                      : "memory");
     }
+}
+
+// Phase B: wait for the MMAs, exact recombination of this thread's columns
+// (one rounding), outputs written back into the tile.
+template <int K, bool PAIR>
+__device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbuf, TciState& t,
+                                            const TciRows<TciShape<K>::MB>& rw) {
+    using S = TciShape<K>;
+    constexpr int TPR = S::TPR;
+    constexpr int NPT = S::N / TPR;
+    constexpr int CW = K == 6 ? 8 : 16;  // columns per TMEM-load round (16 at k = 6 measured slower)
+    const int part = threadIdx.x >> 7;
+    const uint32_t lane_base = (uint32_t)(((threadIdx.x >> 5) & 3) * 32) << 16;
     mbar_wait(t.bar, t.phase);
     t.phase ^= 1u;
     tc_fence_after();
     // 3. exact recombination of this thread's columns, one rounding
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
-        const uint32_t pb = pbs[mb];
+        const uint32_t pb = rw.pbs[mb];
         const uint32_t d0 = t.tmem + lane_base + (uint32_t)(mb * S::NACC * S::N);
 #pragma unroll 1
-        for (int c0 = part * NPT; c0 < (part + 1) * NPT; c0 += 8) {
-            uint32_t v32[8], v24[8], v16[8];
-            tmem_ld8(d0 + (uint32_t)c0, v32);
-            tmem_ld8(d0 + (uint32_t)(S::N + c0), v24);
-            tmem_ld8(d0 + (uint32_t)(2 * S::N + c0), v16);
-            float fc[8];
+        for (int c0 = part * NPT; c0 < (part + 1) * NPT; c0 += CW) {
+            uint32_t v32[CW], v24[CW], v16[CW];
+            if constexpr (CW == 16) {
+                tmem_ld16(d0 + (uint32_t)c0, v32);
+                tmem_ld16(d0 + (uint32_t)(S::N + c0), v24);
+                tmem_ld16(d0 + (uint32_t)(2 * S::N + c0), v16);
+            } else {
+                tmem_ld8(d0 + (uint32_t)c0, v32);
+                tmem_ld8(d0 + (uint32_t)(S::N + c0), v24);
+                tmem_ld8(d0 + (uint32_t)(2 * S::N + c0), v16);
+            }
+            float fc[CW];
 #pragma unroll
-            for (int q = 0; q < 2; ++q)
+            for (int q = 0; q < CW / 4; ++q)
                 asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
                              : "=f"(fc[4 * q]), "=f"(fc[4 * q + 1]), "=f"(fc[4 * q + 2]), "=f"(fc[4 * q + 3])
                              : "r"(t.sF + 4u * (uint32_t)(c0 + 4 * q)));
             asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-            float o[8];
+            float o[CW];
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
+            for (int i = 0; i < CW; ++i) {
                 // exact integer combination (|S24 2^8 + S16| < 2^30), ONE
                 // correctly rounded int64 -> fp32 conversion, then the exact
                 // power-of-two scaling 2^(e - 14) 2^(f - 14) (each factor normal)
                 const int lo = (int)v24[i] * 256 + (int)v16[i];
                 const long long tt = (long long)(int)v32[i] * 65536ll + (long long)lo;
-                o[i] = __ll2float_rn(tt) * srow[mb] * fc[i];
+                o[i] = __ll2float_rn(tt) * rw.srow[mb] * fc[i];
             }
 #pragma unroll
-            for (int i = 0; i < 2; ++i) {
+            for (int i = 0; i < CW / 4; ++i) {
                 const int j = c0 / 4 + i;
                 if constexpr (PAIR) {
                     sts4(sbuf + ((pb ^ p.loc[j]) << 3), make_float4(o[4 * i], o[4 * i + 1], o[4 * i + 2], o[4 * i + 3]));
@@ -848,6 +875,13 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
         }
     }
     tc_fence_before();
+}
+
+template <int K, bool PAIR>
+__device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_t sbuf, TciState& t) {
+    TciRows<TciShape<K>::MB> rw;
+    tci_phase_a<K, PAIR>(p, sbuf, t, rw);
+    tci_phase_b<K, PAIR>(p, sbuf, t, rw);
 }
 
 // Persistent loop over tiles.  STAGES = 2: the copies of tile i+1 are in
@@ -907,7 +941,52 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             st_stream(reinterpret_cast<float4*>(const_cast<char*>(g) + p.goff[i]), lds4(sbuf + ((sthr ^ p.soff[i]) << 3)));
     };
     uint64_t u = blockIdx.x;
-    if constexpr (STAGES == 2) {
+    if constexpr (MODE == 3 && STAGES == 3) {
+        // Three buffers, tile i in buf[i % 3]:
+        //   wait load(i) | phase A(i): gather, slice, issue MMAs |
+        //   store(i-1) while the MMAs run | load(i+2) into the drained buffer |
+        //   phase B(i): wait MMAs, epilogue into buf[i % 3]
+        const uint64_t G = gridDim.x;
+        // global addresses / buffers of tiles it-1 (prv), it (cur), it+1 (nxt)
+        const char* gprv = nullptr;
+        const char* gcur = nullptr;
+        const char* gnxt = nullptr;
+        uint32_t bprv = s0 + 2 * tile_bytes, bcur = s0, bnxt = s0 + tile_bytes;
+        if (u < p.n_tiles) {
+            gcur = gaddr(u);
+            load(gcur, bcur);
+        }
+        cp_async_commit();
+        if (u + G < p.n_tiles) {
+            gnxt = gaddr(u + G);
+            load(gnxt, bnxt);
+        }
+        cp_async_commit();
+        for (int it = 0; u < p.n_tiles; u += G, ++it) {
+            cp_async_wait1();  // this thread's copies of tile it have landed
+            __syncthreads();   // ... and everyone else's; epilogue(it-1) writes are visible
+            TciRows<TciShape<K>::MB> rw;
+            tci_phase_a<K, PAIR>(p, bcur, tis, rw);
+            if (it > 0) store(gprv, bprv);
+            __syncthreads();  // buffer of tile it-1 drained
+            const uint64_t u2 = u + 2 * G;
+            const char* gnew = nullptr;
+            if (u2 < p.n_tiles) {
+                gnew = gaddr(u2);
+                load(gnew, bprv);
+            }
+            cp_async_commit();
+            tci_phase_b<K, PAIR>(p, bcur, tis, rw);
+            const uint32_t bfree = bprv;
+            gprv = gcur; bprv = bcur;
+            gcur = gnxt; bcur = bnxt;
+            gnxt = gnew; bnxt = bfree;
+        }
+        __syncthreads();  // last epilogue complete
+        if (u != blockIdx.x) store(gprv, bprv);
+        cp_async_wait0();
+        tci_teardown<K>(tis);
+    } else if constexpr (STAGES == 2) {
         const char* gcur = nullptr;
         if (u < p.n_tiles) {
             gcur = gaddr(u);
@@ -975,7 +1054,7 @@ __global__ void __launch_bounds__(128, 1) apply_tc(const __grid_constant__ TileP
 }
 template <int K, bool PAIR>
 __global__ void __launch_bounds__(TciShape<K>::THREADS, K == 6 ? 1 : 2) apply_tci(const __grid_constant__ TileParams<K> p) {
-    tile_loop<K, PAIR, 3, 2>(p);
+    tile_loop<K, PAIR, 3, TciShape<K>::STAGES>(p);
 }
 
 // Tiny states (fewer amplitudes than one tile can split into thread work):
@@ -1193,7 +1272,10 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         for (size_t i = 0; i < z.size(); ++i) p.Zpos[i] = z[i];
     }
     p.n_tiles = 1ull << (n - p.T - d.nc);
-    const int STG = d.tc ? 2 : stages_for(K);
+    int STG = d.tc ? 2 : stages_for(K);
+    if constexpr (K >= 4) {
+        if (d.tci) STG = TciShape<K>::STAGES;
+    }
     size_t smem = (size_t)STG * ((size_t)8 << p.T);
     if (K == 6 && !d.tci) smem += 64 * 64 * 8;
     if constexpr (K >= 4) {
