@@ -1,10 +1,11 @@
 """Summarise ncu output into profiles/ (committed evidence).
 
-usage: python tools/summarize_ncu.py <launches.csv> <full_raw.csv> <round_tag>
+usage: python tools/summarize_ncu.py <launches.csv> <full_raw.csv>[,<full_raw2.csv>...] <round_tag>
 
 launches.csv : ncu --metrics gpu__time_duration.sum --csv launch list of a
                bench.py run (cold-cache, serialised -> compare shares)
-full_raw.csv : ncu -i <full .ncu-rep> --page raw --csv of the apply kernel
+full_raw.csv : ncu -i <full .ncu-rep> --page raw --csv of the apply kernel(s)
+               (comma-separated list: the first is the headline kernel)
 Writes profiles/ncu_summary.json (read by bench.py for roofline.traffic)
 and profiles/<round_tag>_ncu_summary.md.
 """
@@ -18,6 +19,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def kclass(name: str) -> str:
+    if "apply_tci" in name or "apply_tc" in name:
+        return "apply_tc"
     if "apply_high" in name or "apply_low" in name or "apply_small" in name:
         return "apply"
     if "exchange" in name:
@@ -62,6 +65,29 @@ def to_bytes(v, unit):
     return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(unit, 1)
 
 
+KEEP = ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
+        "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
+        "smsp__inst_executed.sum", "smsp__issue_active.avg.pct_of_peak_sustained_active",
+        "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum", "sm__cycles_elapsed.avg.per_second")
+TSCALE = {"nsecond": 1e-9, "ns": 1e-9, "usecond": 1e-6, "us": 1e-6, "msecond": 1e-3, "ms": 1e-3, "second": 1.0, "s": 1.0}
+
+
+def captures(path):
+    hdr, units, res = full_raw(path)
+    ui = dict(zip(hdr, units))
+    out = []
+    for d in res:
+        rb = to_bytes(d["dram__bytes_read.sum"], ui["dram__bytes_read.sum"])
+        wb = to_bytes(d["dram__bytes_write.sum"], ui["dram__bytes_write.sum"])
+        dur = float(d["gpu__time_duration.sum"].replace(",", "")) * TSCALE.get(ui["gpu__time_duration.sum"], 1e-9)
+        keep = {k: d[k] for k in KEEP if k in d}
+        out.append({"kernel": d.get("Kernel Name", "")[:120], "dram_read_bytes": rb, "dram_write_bytes": wb,
+                    "traffic_bytes": rb + wb, "duration_s": dur, "dram_GBps": (rb + wb) / dur / 1e9, **keep})
+    return out
+
+
 def main():
     lp, fp, tag = sys.argv[1], sys.argv[2], sys.argv[3]
     L = launches(lp)
@@ -78,26 +104,13 @@ def main():
     summary = {"round": tag, "launch_list": os.path.basename(lp), "classes": {}, "traffic_per_launch": {}}
     for c, (cnt, t) in sorted(by.items()):
         summary["classes"][c] = {"launches": cnt, "time_s": t, "share_of_our_kernels": (t / tot_ours) if c != "other" and tot_ours else None}
-    hdr, units, res = full_raw(fp)
-    ui = dict(zip(hdr, units))
-    caps = []
-    for d in res:
-        rb = to_bytes(d["dram__bytes_read.sum"], ui["dram__bytes_read.sum"])
-        wb = to_bytes(d["dram__bytes_write.sum"], ui["dram__bytes_write.sum"])
-        dur = float(d["gpu__time_duration.sum"].replace(",", "")) * {"nsecond": 1e-9, "ns": 1e-9, "usecond": 1e-6, "us": 1e-6, "msecond": 1e-3, "ms": 1e-3, "second": 1.0, "s": 1.0}.get(ui["gpu__time_duration.sum"], 1e-9)
-        keep = {}
-        for k in ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
-                  "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
-                  "smsp__inst_executed.sum", "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
-                  "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
-                  "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum", "sm__cycles_elapsed.avg.per_second"):
-            if k in d:
-                keep[k] = d[k]
-        caps.append({"kernel": d.get("Kernel Name", "")[:120], "dram_read_bytes": rb, "dram_write_bytes": wb,
-                     "traffic_bytes": rb + wb, "duration_s": dur, "dram_GBps": (rb + wb) / dur / 1e9, **keep})
+    caps = [c for one in fp.split(",") for c in captures(one)]
     if caps:
         summary["full_capture"] = caps
         summary["traffic_per_launch"]["apply"] = caps[0]["traffic_bytes"]
+        for c in caps:
+            if "apply_tci" in c["kernel"]:
+                summary["traffic_per_launch"].setdefault("apply_tci", c["traffic_bytes"])
     json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
     md = [f"# ncu summary ({tag})", "", f"Launch list: `{os.path.basename(lp)}` (ncu --metrics gpu__time_duration.sum "
           "--clock-control none; cold-cache, serialised: compare shares, not absolutes)", "",
@@ -109,7 +122,7 @@ def main():
     for n, (cnt, t) in sorted(names.items(), key=lambda x: -x[1][1])[:20]:
         md.append(f"| `{n}` | {cnt} | {t:.4f} |")
     if caps:
-        md += ["", "Full capture (--set full) of the dominant apply kernel:", ""]
+        md += ["", "Full captures (--set full, one launch each, 30 qubits): the headline kernel first:", ""]
         for c in caps:
             md.append(f"- `{c['kernel']}`: DRAM read {c['dram_read_bytes'] / 1e9:.3f} GB, write "
                       f"{c['dram_write_bytes'] / 1e9:.3f} GB per launch (algorithmic 16 B x 2^30 = 17.180 GB), "
