@@ -42,16 +42,20 @@ def _compile(src: str, verbose: bool) -> str:
     return obj
 
 
-def build_variant(name: str, defines) -> str:
-    """Build an A/B variant library (extra -D flags) next to the main one."""
+def build_variant(name: str, defines, csrc: str = CSRC, include: str = INCLUDE) -> str:
+    """Build an A/B variant library (extra -D flags, or another source tree,
+    e.g. a git ref extracted by tools/ab_ref.py) next to the main one."""
     out = os.path.join(HERE, "_variants", f"libsvb200_{name}.so")
     bdir = os.path.join(HERE, "_variants", name)
     os.makedirs(bdir, exist_ok=True)
     extra = [f"-D{d}" for d in defines]
+    common = [c for c in COMMON]
+    common[common.index(INCLUDE)] = include
+    common[common.index(CSRC)] = csrc
 
     def comp(src):
         obj = os.path.join(bdir, src + ".o")
-        subprocess.check_call([NVCC] + ARCH + COMMON + extra + ["-c", os.path.join(CSRC, src), "-o", obj])
+        subprocess.check_call([NVCC] + ARCH + common + extra + ["-c", os.path.join(csrc, src), "-o", obj])
         return obj
 
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:

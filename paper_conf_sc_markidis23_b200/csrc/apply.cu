@@ -90,9 +90,10 @@ struct alignas(16) TileParams {
     int Hpos[SV_MAX_FUSED];            // gate qubits >= r (ascending, global positions)
     int nzt;
     int ztpos[SV_MAX_FUSED];           // tile-local gate bit positions, ascending
+    uint32_t zthigh[SV_MAX_FUSED];     // ~0u << ztpos[b]
     uint32_t swz[3];                   // phys bit (i+1) ^= parity(t & swz[i])
     int nZ;                            // tile-base zero insertions: H and control qubits, ascending
-    int Zpos[2 * SV_MAX_FUSED];
+    uint64_t Zhigh[2 * SV_MAX_FUSED];  // ~0 << Zpos[b]: inserting a zero at q is x += x & (~0 << q)
     uint64_t ones;                     // control qubits forced to 1 in the tile base
     int upt;                           // 16-byte units per thread per tile
     int iters;                         // compute iterations per thread per tile
@@ -107,6 +108,16 @@ struct alignas(16) TileParams {
     uint32_t ploc[1 << K];             // phys offset of the source member of row r
     float2 mdiag[1 << K];              // the nonzero of row r
 };
+
+// Swizzled shared-memory slot of tile-local group index g: zeros inserted at
+// the K gate positions (ascending; inserting a zero at q is x += x & (~0 << q))
+// -- 2 instructions per position in 32-bit arithmetic.
+template <int K>
+__device__ __forceinline__ uint32_t slot_of(const TileParams<K>& p, uint32_t g) {
+#pragma unroll
+    for (int b = 0; b < K; ++b) g += g & p.zthigh[b];
+    return swizzle(g, p.swz);
+}
 
 // Gauss form of output rows [r0, r0 + R) for one group (s[c] = x_c + y_c).
 // The row loop of the callers is NOT unrolled: each iteration is a scheduling
@@ -177,13 +188,13 @@ __device__ __forceinline__ float2 cmul(float2 m, float2 a) {
 }
 
 template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32_t sbuf) {
+__device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32_t sbuf, uint32_t pb0) {
     constexpr int D = 1 << K;
     constexpr int GPT = (K <= 4) ? 2 : 1;
     for (int j = 0; j < p.iters; ++j) {
         const uint32_t gidx = threadIdx.x + (uint32_t)j * blockDim.x;
         if constexpr (GPT == 2 && !PAIR) {
-            const uint32_t pb = swizzle((uint32_t)insert_zeros((uint64_t)gidx << 1, p.ztpos, p.nzt), p.swz);
+            const uint32_t pb = j == 0 ? pb0 : slot_of<K>(p, gidx << 1);
             float4 v[D];
 #pragma unroll
             for (int r = 0; r < D; ++r) v[r] = lds4(sbuf + ((pb ^ p.ploc[r]) << 3));
@@ -194,8 +205,7 @@ __device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32
                 sts4(sbuf + ((pb ^ p.mloc[r]) << 3), make_float4(y0.x, y0.y, y1.x, y1.y));
             }
         } else {
-            const uint32_t pb = (GPT == 2) ? swizzle((uint32_t)insert_zeros((uint64_t)gidx << 1, p.ztpos, p.nzt), p.swz)
-                                           : swizzle((uint32_t)insert_zeros(gidx, p.ztpos, p.nzt), p.swz);
+            const uint32_t pb = j == 0 ? pb0 : (GPT == 2) ? slot_of<K>(p, gidx << 1) : slot_of<K>(p, gidx);
 #pragma unroll
             for (int gg = 0; gg < GPT; ++gg) {
                 const uint32_t b = gg ? (pb ^ p.gsec) : pb;
@@ -210,13 +220,13 @@ __device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32
 }
 
 template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* smat) {
+__device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* smat, uint32_t pb0) {
     constexpr int D = 1 << K;
     constexpr int GPT = (K <= 4) ? 2 : 1;
     for (int j = 0; j < p.iters; ++j) {
         const uint32_t gidx = threadIdx.x + (uint32_t)j * blockDim.x;
         if constexpr (GPT == 2) {
-            const uint32_t pb = swizzle((uint32_t)insert_zeros((uint64_t)gidx << 1, p.ztpos, p.nzt), p.swz);
+            const uint32_t pb = j == 0 ? pb0 : slot_of<K>(p, gidx << 1);
             float2 a0[D], a1[D];
             float s0[D], s1[D];
             if constexpr (PAIR) {
@@ -261,7 +271,7 @@ __device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sb
                 }
             }
         } else {
-            const uint32_t pb = swizzle((uint32_t)insert_zeros(gidx, p.ztpos, p.nzt), p.swz);
+            const uint32_t pb = j == 0 ? pb0 : slot_of<K>(p, gidx);
             float2 a[D];
             if constexpr (PAIR) {
 #pragma unroll
@@ -470,7 +480,7 @@ __device__ __forceinline__ void tile_compute_tc(const TileParams<K>& p, uint32_t
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
         const uint32_t g = (uint32_t)mb * 128u + threadIdx.x;
-        const uint32_t pb = swizzle((uint32_t)insert_zeros(g, p.ztpos, p.nzt), p.swz);
+        const uint32_t pb = slot_of<K>(p, g);
         const uint32_t thi = t.tmem + lane_base + (uint32_t)(mb * 2 * S::KR);
         const uint32_t tlo = thi + (uint32_t)S::KR;
 #pragma unroll
@@ -527,7 +537,7 @@ __device__ __forceinline__ void tile_compute_tc(const TileParams<K>& p, uint32_t
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
         const uint32_t g = (uint32_t)mb * 128u + threadIdx.x;
-        const uint32_t pb = swizzle((uint32_t)insert_zeros(g, p.ztpos, p.nzt), p.swz);
+        const uint32_t pb = slot_of<K>(p, g);
 #pragma unroll
         for (int c0 = 0; c0 < S::N; c0 += 32) {
             uint32_t v[32];
@@ -699,14 +709,24 @@ __device__ __forceinline__ void sts128u(uint32_t a, uint4 v) {
 template <int MB>
 struct TciRows {
     float srow[MB];    // 2^(e - 14) per M-block row
-    uint32_t pbs[MB];  // phys offset of the row's group
 };
+
+// Phys (swizzled) slot of this thread's group row in M-block mb: the same
+// for every tile, computed once per kernel.
+template <int K>
+__device__ __forceinline__ void tci_slots(const TileParams<K>& p, uint32_t (&pbs)[TciShape<K>::MB]) {
+#pragma unroll
+    for (int mb = 0; mb < TciShape<K>::MB; ++mb) {
+        const uint32_t g = (uint32_t)mb * 128u + (threadIdx.x & 127u);
+        pbs[mb] = slot_of<K>(p, g);
+    }
+}
 
 // Phase A: gather, slice, issue the MMAs (asynchronous; completion is
 // signalled on t.bar).
 template <int K, bool PAIR>
 __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbuf, TciState& t,
-                                            TciRows<TciShape<K>::MB>& rw) {
+                                            TciRows<TciShape<K>::MB>& rw, const uint32_t (&pbs)[TciShape<K>::MB]) {
     using S = TciShape<K>;
     constexpr int TPR = S::TPR;
     constexpr int D = S::D;
@@ -720,9 +740,7 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
     // 1a. gather this thread's part of the row, publish the part maximum
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
-        const uint32_t g = (uint32_t)mb * 128u + row;
-        const uint32_t pb = swizzle((uint32_t)insert_zeros(g, p.ztpos, p.nzt), p.swz);
-        rw.pbs[mb] = pb;
+        const uint32_t pb = pbs[mb];
 #pragma unroll
         for (int j = 0; j < HM / 2; ++j) {
             const int jj = part * (HM / 2) + j;  // member pair (2jj, 2jj+1)
@@ -818,7 +836,7 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
 // (one rounding), outputs written back into the tile.
 template <int K, bool PAIR>
 __device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbuf, TciState& t,
-                                            const TciRows<TciShape<K>::MB>& rw) {
+                                            const TciRows<TciShape<K>::MB>& rw, const uint32_t (&pbs)[TciShape<K>::MB]) {
     using S = TciShape<K>;
     constexpr int TPR = S::TPR;
     constexpr int NPT = S::N / TPR;
@@ -831,7 +849,7 @@ __device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbu
     // 3. exact recombination of this thread's columns, one rounding
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
-        const uint32_t pb = rw.pbs[mb];
+        const uint32_t pb = pbs[mb];
         const uint32_t d0 = t.tmem + lane_base + (uint32_t)(mb * S::NACC * S::N);
 #pragma unroll 1
         for (int c0 = part * NPT; c0 < (part + 1) * NPT; c0 += CW) {
@@ -878,10 +896,11 @@ __device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbu
 }
 
 template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_t sbuf, TciState& t) {
+__device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_t sbuf, TciState& t,
+                                                 const uint32_t (&pbs)[TciShape<K>::MB]) {
     TciRows<TciShape<K>::MB> rw;
-    tci_phase_a<K, PAIR>(p, sbuf, t, rw);
-    tci_phase_b<K, PAIR>(p, sbuf, t, rw);
+    tci_phase_a<K, PAIR>(p, sbuf, t, rw, pbs);
+    tci_phase_b<K, PAIR>(p, sbuf, t, rw, pbs);
 }
 
 // Persistent loop over tiles.  STAGES = 2: the copies of tile i+1 are in
@@ -891,10 +910,7 @@ __device__ __forceinline__ void tile_compute_tci(const TileParams<K>& p, uint32_
 template <int K>
 __device__ __forceinline__ uint64_t tile_base(const TileParams<K>& p, uint64_t u) {
     uint64_t x = u << p.r;
-    for (int b = 0; b < p.nZ; ++b) {
-        const int q = p.Zpos[b];
-        x = ((x >> q) << (q + 1)) | (x & ((1ull << q) - 1ull));
-    }
+    for (int b = 0; b < p.nZ; ++b) x += x & p.Zhigh[b];  // ascending positions: shift bits >= q up by one
     return x | p.ones;
 }
 
@@ -910,8 +926,14 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
         smat = sm;
         __syncthreads();
     }
+    // slot of this thread's first group (the same in every tile)
+    const uint32_t pb0 = slot_of<K>(p, K <= 4 ? (threadIdx.x << 1) : threadIdx.x);
     TciState tis{};
-    if constexpr (MODE == 3) tis = tci_setup<K>(p, s0 + STAGES * tile_bytes);
+    uint32_t tslot[MODE == 3 ? TciShape<K>::MB : 1];
+    if constexpr (MODE == 3) {
+        tis = tci_setup<K>(p, s0 + STAGES * tile_bytes);
+        tci_slots<K>(p, tslot);
+    }
     TcState tcs{};
     if constexpr (MODE == 2 && K <= 5) {
         const uint32_t sW = s0 + STAGES * tile_bytes;
@@ -966,7 +988,7 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             cp_async_wait1();  // this thread's copies of tile it have landed
             __syncthreads();   // ... and everyone else's; epilogue(it-1) writes are visible
             TciRows<TciShape<K>::MB> rw;
-            tci_phase_a<K, PAIR>(p, bcur, tis, rw);
+            tci_phase_a<K, PAIR>(p, bcur, tis, rw, tslot);
             if (it > 0) store(gprv, bprv);
             __syncthreads();  // buffer of tile it-1 drained
             const uint64_t u2 = u + 2 * G;
@@ -976,7 +998,7 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
                 load(gnew, bprv);
             }
             cp_async_commit();
-            tci_phase_b<K, PAIR>(p, bcur, tis, rw);
+            tci_phase_b<K, PAIR>(p, bcur, tis, rw, tslot);
             const uint32_t bfree = bprv;
             gprv = gcur; bprv = bcur;
             gcur = gnxt; bcur = bnxt;
@@ -1006,10 +1028,10 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             cp_async_commit();
             cp_async_wait1();  // this thread's copies of tile u have landed
             __syncthreads();   // ... and everyone else's
-            if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, cur);
+            if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, cur, pb0);
             else if constexpr (MODE == 2 && K <= 5) tile_compute_tc<K, PAIR>(p, cur, tcs);
-            else if constexpr (MODE == 3) tile_compute_tci<K, PAIR>(p, cur, tis);
-            else tile_compute<K, PAIR>(p, cur, smat);
+            else if constexpr (MODE == 3) tile_compute_tci<K, PAIR>(p, cur, tis, tslot);
+            else tile_compute<K, PAIR>(p, cur, smat, pb0);
             __syncthreads();
             store(gcur, cur);
             gcur = gnext;
@@ -1024,8 +1046,8 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             cp_async_commit();
             cp_async_wait0();
             __syncthreads();
-            if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, s0);
-            else tile_compute<K, PAIR>(p, s0, smat);
+            if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, s0, pb0);
+            else tile_compute<K, PAIR>(p, s0, smat, pb0);
             __syncthreads();
             store(g, s0);
         }
@@ -1152,7 +1174,10 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         }
     }
     p.nzt = K;
-    for (int b = 0; b < K; ++b) p.ztpos[b] = tl[b];
+    for (int b = 0; b < K; ++b) {
+        p.ztpos[b] = tl[b];
+        p.zthigh[b] = ~0u << tl[b];
+    }
     uint32_t gmask = 0;
     for (int b = 0; b < K; ++b) gmask |= 1u << tl[b];
     int ng[32], nng = 0;  // non-gate tile bits, ascending
@@ -1269,7 +1294,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         }
         std::sort(z.begin(), z.end());
         p.nZ = (int)z.size();
-        for (size_t i = 0; i < z.size(); ++i) p.Zpos[i] = z[i];
+        for (size_t i = 0; i < z.size(); ++i) p.Zhigh[i] = ~0ull << z[i];
     }
     p.n_tiles = 1ull << (n - p.T - d.nc);
     int STG = d.tc ? 2 : stages_for(K);
