@@ -578,6 +578,22 @@ __device__ __forceinline__ void tile_compute_tc(const TileParams<K>& p, uint32_t
 // Operand A (slices) and B (W slices) live in shared memory in the K-major
 // SWIZZLE_NONE canonical layout (core matrix 8 rows x 16 B), D in TMEM.
 __host__ __device__ constexpr int tci_threads(int K) { return K == 6 ? 512 : 256; }
+// Accumulators: S32, S24, S16 (+ S8 = a1 b2 + a2 b1).  Without S8 the
+// dropped products correlate with the output through the state's own middle
+// digit and leave a per-gate norm change of random sign (DESIGN.md §11:
+// -1.1e-6 over a 23-gate k = 6 circuit, 1.3e-7 over 25 k = 5 gates); S8 costs
+// 2 MMAs per K-step, one more TMEM load per column group and ~1 instruction
+// per output (+7 % at k = 4, 5, +13 % at k = 6).  k = 6 keeps S8.
+__host__ __device__ constexpr int tci_nacc(int K) {
+#ifdef SVB_TCI_NACC4
+    return 4 + 0 * K;
+#else
+    return K == 6 ? 4 : 3;
+#endif
+}
+// Output scale 2^(e + f - 2 SH) split as 2^(e - SH) 2^(f - SH): tt is
+// sum xi wi / 2^16 with three accumulators (SH = 14), / 2^8 with four (SH = 18).
+__host__ __device__ constexpr int tci_shift(int K) { return tci_nacc(K) == 4 ? 18 : 14; }
 
 template <int K>
 struct TciShape {
@@ -602,7 +618,7 @@ struct TciShape {
     static constexpr uint32_t B_SLICE = (uint32_t)N * KR;
     static constexpr uint32_t ROWMAX = 4 * 128 * MB * 4;  // part-row maxima exchange (TPR <= 4)
     static constexpr uint32_t SMEM = (A_IN_TILE ? 0u : 3 * A_SLICE) + 3 * B_SLICE + N * 4 + ROWMAX + 64;
-    static constexpr int NACC = 3;                    // S32, S24, S16
+    static constexpr int NACC = tci_nacc(K);          // S32, S24, S16 (, S8)
     static constexpr int COLS = NACC * N * MB;
     static constexpr int ALLOC = COLS <= 32 ? 32 : COLS <= 64 ? 64 : COLS <= 128 ? 128 : COLS <= 256 ? 256 : 512;
 };
@@ -773,7 +789,7 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
             mx = fmaxf(mx, m);
         }
         const int e = max(((int)(__float_as_uint(mx) >> 23) & 0xFF) - 126, -100);  // mx < 2^e
-        rw.srow[mb] = __uint_as_float((uint32_t)(127 + e - 14) << 23);                 // 2^(e - 14)
+        rw.srow[mb] = __uint_as_float((uint32_t)(127 + e - tci_shift(K)) << 23);      // 2^(e - SH)
         const float scale = __uint_as_float((uint32_t)(127 + 22 - e) << 23);
         const uint32_t rbase = (uint32_t)mb * 128u * S::KR + (row >> 3) * S::SBO + (row & 7) * 16u;
         if constexpr (RPT == 8) {
@@ -809,7 +825,8 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
 #pragma unroll
         for (int mb = 0; mb < S::MB; ++mb) {
             const uint32_t d0 = t.tmem + (uint32_t)(mb * S::NACC * S::N);
-            const uint32_t d32 = d0, d24 = d0 + S::N, d16 = d0 + 2 * S::N;
+            const uint32_t d32 = d0, d24 = d0 + S::N, d16 = d0 + 2 * S::N, d8 = d0 + 3 * S::N;
+            (void)d8;
 #pragma unroll
             for (int ks = 0; ks < S::KS; ++ks) {
                 const uint32_t ao = sA + (uint32_t)mb * 128u * S::KR + (uint32_t)ks * 256u;
@@ -825,6 +842,10 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
                 mma_i8_ss(d16, a0, b2, i_ss, acc);
                 mma_i8_ss(d16, a1, b1, i_ss, 1u);
                 mma_i8_ss(d16, a2, b0, i_ss, 1u);
+                if constexpr (S::NACC == 4) {
+                    mma_i8_ss(d8, a1, b2, i_ss, acc);
+                    mma_i8_ss(d8, a2, b1, i_ss, 1u);
+                }
             }
         }
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(t.bar)
@@ -853,15 +874,17 @@ __device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbu
         const uint32_t d0 = t.tmem + lane_base + (uint32_t)(mb * S::NACC * S::N);
 #pragma unroll 1
         for (int c0 = part * NPT; c0 < (part + 1) * NPT; c0 += CW) {
-            uint32_t v32[CW], v24[CW], v16[CW];
+            uint32_t v32[CW], v24[CW], v16[CW], v8[S::NACC == 4 ? CW : 1];
             if constexpr (CW == 16) {
                 tmem_ld16(d0 + (uint32_t)c0, v32);
                 tmem_ld16(d0 + (uint32_t)(S::N + c0), v24);
                 tmem_ld16(d0 + (uint32_t)(2 * S::N + c0), v16);
+                if constexpr (S::NACC == 4) tmem_ld16(d0 + (uint32_t)(3 * S::N + c0), v8);
             } else {
                 tmem_ld8(d0 + (uint32_t)c0, v32);
                 tmem_ld8(d0 + (uint32_t)(S::N + c0), v24);
                 tmem_ld8(d0 + (uint32_t)(2 * S::N + c0), v16);
+                if constexpr (S::NACC == 4) tmem_ld8(d0 + (uint32_t)(3 * S::N + c0), v8);
             }
             float fc[CW];
 #pragma unroll
@@ -876,9 +899,17 @@ __device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbu
                 // exact integer combination (|S24 2^8 + S16| < 2^30), ONE
                 // correctly rounded int64 -> fp32 conversion, then the exact
                 // power-of-two scaling 2^(e - 14) 2^(f - 14) (each factor normal)
-                const int lo = (int)v24[i] * 256 + (int)v16[i];
-                const long long tt = (long long)(int)v32[i] * 65536ll + (long long)lo;
-                o[i] = __ll2float_rn(tt) * rw.srow[mb] * fc[i];
+                if constexpr (S::NACC == 4) {
+                    // |S32 2^8 + S24| < 2^28, |S16 2^8 + S8| < 2^31
+                    const int hi = (int)v32[i] * 256 + (int)v24[i];
+                    const int lo = (int)v16[i] * 256 + (int)v8[i];
+                    const long long tt = (long long)hi * 65536ll + (long long)lo;
+                    o[i] = __ll2float_rn(tt) * rw.srow[mb] * fc[i];
+                } else {
+                    const int lo = (int)v24[i] * 256 + (int)v16[i];
+                    const long long tt = (long long)(int)v32[i] * 65536ll + (long long)lo;
+                    o[i] = __ll2float_rn(tt) * rw.srow[mb] * fc[i];
+                }
             }
 #pragma unroll
             for (int i = 0; i < CW / 4; ++i) {
@@ -1350,25 +1381,58 @@ void pack_wi8(const ApplyDesc& d, uint8_t* out) {
     const uint32_t SBO = KR * 8, BS = (uint32_t)N * KR;
     std::memset(out, 0, wi8_bytes(d.k));
     float* fcol = reinterpret_cast<float*>(out + 3 * BS);
+    const bool have64 = d.m64.size() == d.m.size();
     for (int n = 0; n < N; ++n) {
         const int r = n >> 1, ni = n & 1;
         double w[128];
         double mx = 0.0;
         for (int kk = 0; kk < KR; ++kk) {
             const int c = kk >> 1, ki = kk & 1;
-            const cf m = d.m[(size_t)r * D + c];
+            const std::complex<double> m =
+                have64 ? d.m64[(size_t)r * D + c] : std::complex<double>(d.m[(size_t)r * D + c]);
             w[kk] = (ni == 0) ? (ki == 0 ? m.real() : -m.imag()) : (ki == 0 ? m.imag() : m.real());
             mx = std::max(mx, std::fabs(w[kk]));
         }
         int f = 0;
         std::frexp(mx, &f);  // mx < 2^f
         f = std::max(f, -100);
-        fcol[n] = std::ldexp(1.0f, f - 14);  // column half of the output scale 2^(e + f - 28)
+        fcol[n] = std::ldexp(1.0f, f - tci_shift(d.k));  // column half of the output scale
+        // Round to 22-bit integers, then match the column's exact squared norm:
+        // plain rounding changes each column norm by ~2^-23, and for a unitary
+        // that is a systematic per-gate change of the state norm (DESIGN.md
+        // §11: ~1e-8 per apply, 1.8e-6 of fidelity over a 30-qubit circuit).
+        // Flipping the rounding direction of an entry (it stays within one
+        // unit of its exact value) changes the integer sum of squares by
+        // 2|wi| +- 1; entries are visited from the largest down, so the
+        // residual ends near the smallest entries' granularity.
+        int64_t wi[128];
+        double sx[128];
+        double target = 0.0, cur = 0.0;
         for (int kk = 0; kk < KR; ++kk) {
-            const int32_t wi = (int32_t)std::nearbyint(std::ldexp(w[kk], 22 - f));
+            sx[kk] = std::ldexp(w[kk], 22 - f);
+            wi[kk] = (int64_t)std::nearbyint(sx[kk]);
+            target += sx[kk] * sx[kk];
+            cur += (double)wi[kk] * (double)wi[kk];
+        }
+        int order[128];
+        for (int kk = 0; kk < KR; ++kk) order[kk] = kk;
+        std::sort(order, order + KR, [&](int a, int b) { return std::llabs(wi[a]) > std::llabs(wi[b]); });
+        for (int i = 0; i < KR; ++i) {
+            const int kk = order[i];
+            const double delta = target - cur;
+            const int64_t s = (sx[kk] > (double)wi[kk]) ? 1 : -1;  // the other rounding direction
+            if (std::fabs(sx[kk] - (double)(wi[kk] + s)) >= 1.0) continue;
+            const double change = (double)(2 * wi[kk] * s + 1);
+            if (std::fabs(delta - change) < std::fabs(delta)) {
+                wi[kk] += s;
+                cur += change;
+            }
+        }
+        for (int kk = 0; kk < KR; ++kk) {
+            const int32_t v = (int32_t)wi[kk];
             // balanced signed base-256 digits (as the kernel slices the state)
-            const int32_t d2 = (int32_t)(int8_t)(wi & 0xFF);
-            const int32_t r1 = (wi - d2) >> 8;
+            const int32_t d2 = (int32_t)(int8_t)(v & 0xFF);
+            const int32_t r1 = (v - d2) >> 8;
             const int32_t d1 = (int32_t)(int8_t)(r1 & 0xFF);
             const int32_t d0 = (r1 - d1) >> 8;
             const uint32_t off = (uint32_t)(n >> 3) * SBO + (uint32_t)(kk >> 4) * 128u + (uint32_t)(n & 7) * 16u +

@@ -22,6 +22,7 @@ struct ApplyDesc {
     int k = 0;
     int q[SV_MAX_FUSED] = {0};        // ascending physical qubits (within a shard)
     std::vector<cf> m;                // 2^k x 2^k row-major over ascending q, complex64
+    std::vector<std::complex<double>> m64;  // the same in complex128 (int8 tensor-core packer)
     bool high = false;                // kernel class
     bool mono = false;                // one nonzero per row (exact permutation/diagonal path)
     int nc = 0;                       // control qubits (controlled gate, NEXT-4): only the

@@ -246,6 +246,7 @@ void make_apply(int l, int k, const int* phys_in_order, const cd* M /* bit b <->
     for (int b = 0; b < k; ++b) d.q[b] = sq[b];
     d.m.resize(Ms.size());
     for (size_t i = 0; i < Ms.size(); ++i) d.m[i] = cf((float)Ms[i].real(), (float)Ms[i].imag());
+    d.m64 = Ms;
     plan_apply(l, d);
 }
 
