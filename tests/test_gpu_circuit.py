@@ -60,9 +60,10 @@ def test_random_circuit_unsorted_two_qubit_gates():
 
 
 @pytest.mark.parametrize("world", [2, 4, 8])
-@pytest.mark.parametrize("F", [2, 4])
-def test_virtual_shards_match_oracle(world, F):
-    n = 16
+@pytest.mark.parametrize("n,F", [(16, 2), (16, 4), (19, 5), (19, 6)])
+def test_virtual_shards_match_oracle(world, n, F):
+    """F = 5, 6 at 19 qubits: 16-18 local qubits, so the int8 tensor-core
+    apply runs inside the shards between exchanges."""
     gates = W.rqc(n, 14, seed=world)
     got, st = _run(n, gates, F, world=world)
     _check(n, 14, got, ref_c.run(n, gates))

@@ -48,10 +48,19 @@ def main():
     if not (fid >= 1 - 1e-5 and err <= osv.max_abs_bound(n, 14) and st["n_exchanges"] >= 1):
         ok = False
         msgs.append(f"circuit fid={fid} err={err} exch={st['n_exchanges']}")
+    # 1b. F = 5 (int8 tensor-core apply inside the shards when >= 13 local qubits)
+    sv.sv_reset(h)
+    st5 = sv.sv_run_circuit(h, gates, 5)
+    psi5 = sv.sv_get_state(h, n)
+    fid5 = osv.fidelity(psi5.astype(np.complex128), ref)
+    err5 = float(np.abs(psi5.astype(np.complex128) - ref).max())
+    if not (fid5 >= 1 - 1e-5 and err5 <= osv.max_abs_bound(n, 14)):
+        ok = False
+        msgs.append(f"circuit F=5 fid={fid5} err={err5} exch={st5['n_exchanges']}")
     # 2. amplitudes
     idx = np.random.default_rng(1).integers(0, 1 << n, size=200).astype(np.uint64)
     amps = sv.sv_amplitudes(h, idx)
-    if not np.array_equal(amps, psi[idx.astype(np.int64)]):
+    if not np.array_equal(amps, psi5[idx.astype(np.int64)]):
         ok = False
         msgs.append("amplitudes mismatch")
     # 3. sampling on a seeded state: bit-exact vs the oracle
