@@ -18,7 +18,7 @@ INCLUDE = os.path.join(ROOT, "include")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC]
+COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcudafe", "--diag_suppress=177", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC]
 
 SOURCES = ["apply.cu", "apply64.cu", "blocked.cu", "small.cu", "state.cu", "fuser.cpp", "planner.cpp", "sv_api.cpp"]
 HEADERS = ["kernels.h", "sv_internal.h", "device_util.cuh"]

@@ -71,6 +71,9 @@ struct MatStore<6> {  // 32 KB complex: does not fit the 32764 B parameter space
 #ifndef SV_ROWS
 #define SV_ROWS 1  // output rows per (non-unrolled) row-loop iteration
 #endif
+#ifndef SVB_SMEM_PLANES
+#define SVB_SMEM_PLANES 1  // dense k = 2, 3 SIMT: Gauss planes read from shared memory (LDS.128)
+#endif
 
 // ------------------------------------------------------------------ kernels
 // A tile is the set of 2^nH runs of 2^r contiguous amplitudes that share
@@ -142,11 +145,41 @@ __device__ __forceinline__ void gauss_block(const MatStore<K>& M, int r0, const 
 
 template <int K, int R>
 __device__ __forceinline__ void gauss_block2(const MatStore<K>& M, int r0, const float2* a0, const float* s0,
-                                             const float2* a1, const float* s1, float2* y0, float2* y1) {
+                                             const float2* a1, const float* s1, float2* y0, float2* y1,
+                                             uint32_t splanes = 0) {
     constexpr int D = 1 << K;
 #pragma unroll
     for (int i = 0; i < R; ++i) {
         float A0 = 0.f, B0 = 0.f, C0 = 0.f, A1 = 0.f, B1 = 0.f, C1 = 0.f;
+#if SVB_SMEM_PLANES
+        if constexpr (D >= 4 && D <= 8) {
+            // planes staged in shared memory: one broadcast LDS.128 per 4 operands
+            // (the constant-bank path issues LDCU.64, twice as many loads)
+            const uint32_t rowP = splanes + 4u * (uint32_t)((r0 + i) * D);
+#pragma unroll
+            for (int c4 = 0; c4 < D / 4; ++c4) {
+                const float4 pv = lds4(rowP + 16u * c4);
+                const float4 sv = lds4(rowP + 4u * D * D + 16u * c4);
+                const float4 qv = lds4(rowP + 8u * D * D + 16u * c4);
+                const float pp[4] = {pv.x, pv.y, pv.z, pv.w}, ss[4] = {sv.x, sv.y, sv.z, sv.w},
+                            qq[4] = {qv.x, qv.y, qv.z, qv.w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int c = 4 * c4 + j;
+                    A0 = fmaf(pp[j], s0[c], A0);
+                    A1 = fmaf(pp[j], s1[c], A1);
+                    B0 = fmaf(ss[j], a0[c].y, B0);
+                    B1 = fmaf(ss[j], a1[c].y, B1);
+                    C0 = fmaf(qq[j], a0[c].x, C0);
+                    C1 = fmaf(qq[j], a1[c].x, C1);
+                }
+            }
+            y0[i] = make_float2(A0 - B0, A0 + C0);
+            y1[i] = make_float2(A1 - B1, A1 + C1);
+            continue;
+        }
+#endif
+        (void)splanes;
 #pragma unroll
         for (int c = 0; c < D; ++c) {
             const float p = M.P[r0 + i][c], sq = M.S[r0 + i][c], q = M.Q[r0 + i][c];
@@ -220,7 +253,8 @@ __device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32
 }
 
 template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* smat, uint32_t pb0) {
+__device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* smat, uint32_t pb0,
+                                             uint32_t splanes) {
     constexpr int D = 1 << K;
     constexpr int GPT = (K <= 4) ? 2 : 1;
     for (int j = 0; j < p.iters; ++j) {
@@ -256,7 +290,7 @@ __device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sb
 #pragma unroll 1
                 for (int r2 = 0; r2 < D / 2; ++r2) {
                     float2 y0[2], y1[2];
-                    gauss_block2<K, 2>(p.M, 2 * r2, a0, s0, a1, s1, y0, y1);
+                    gauss_block2<K, 2>(p.M, 2 * r2, a0, s0, a1, s1, y0, y1, splanes);
                     sts4(sbuf + ((pb ^ p.loc[r2]) << 3), make_float4(y0[0].x, y0[0].y, y0[1].x, y0[1].y));
                     sts4(sbuf + ((pb ^ p.gsec ^ p.loc[r2]) << 3), make_float4(y1[0].x, y1[0].y, y1[1].x, y1[1].y));
                 }
@@ -264,7 +298,7 @@ __device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sb
 #pragma unroll 1
                 for (int r = 0; r < D; r += SV_ROWS) {
                     float2 y0[SV_ROWS], y1[SV_ROWS];
-                    gauss_block2<K, SV_ROWS>(p.M, r, a0, s0, a1, s1, y0, y1);
+                    gauss_block2<K, SV_ROWS>(p.M, r, a0, s0, a1, s1, y0, y1, splanes);
 #pragma unroll
                     for (int i = 0; i < SV_ROWS; ++i)
                         sts4(sbuf + ((pb ^ p.loc[r + i]) << 3), make_float4(y0[i].x, y0[i].y, y1[i].x, y1[i].y));
@@ -951,6 +985,23 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
     const uint32_t tile_bytes = 8u << p.T;
     const uint32_t s0 = smem_addr(dsm);
     const float2* smat = nullptr;
+    uint32_t splanes = 0;
+#if SVB_SMEM_PLANES
+    // k = 2, 3 only: at k = 4 it measured 19 % slower (3.70 vs 3.12 ms; the
+    // LDCU operands feed the FFMAs without occupying vector registers)
+    if constexpr (MODE == 0 && K >= 2 && K <= 3) {
+        // Gauss planes P, S, Q (3 x 2^k x 2^k fp32) after the tile buffers
+        constexpr int DD = (1 << K) * (1 << K);
+        float* sp = reinterpret_cast<float*>(reinterpret_cast<char*>(dsm) + STAGES * tile_bytes);
+        for (int i = threadIdx.x; i < DD; i += blockDim.x) {
+            sp[i] = (&p.M.P[0][0])[i];
+            sp[DD + i] = (&p.M.S[0][0])[i];
+            sp[2 * DD + i] = (&p.M.Q[0][0])[i];
+        }
+        splanes = s0 + STAGES * tile_bytes;
+        __syncthreads();
+    }
+#endif
     if constexpr (K == 6 && MODE != 3) {
         float2* sm = reinterpret_cast<float2*>(reinterpret_cast<char*>(dsm) + STAGES * tile_bytes);
         for (int i = threadIdx.x; i < 64 * 64; i += blockDim.x) sm[i] = p.M.dev[i];
@@ -1062,7 +1113,7 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, cur, pb0);
             else if constexpr (MODE == 2 && K <= 5) tile_compute_tc<K, PAIR>(p, cur, tcs);
             else if constexpr (MODE == 3) tile_compute_tci<K, PAIR>(p, cur, tis, tslot);
-            else tile_compute<K, PAIR>(p, cur, smat, pb0);
+            else tile_compute<K, PAIR>(p, cur, smat, pb0, splanes);
             __syncthreads();
             store(gcur, cur);
             gcur = gnext;
@@ -1078,7 +1129,7 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             cp_async_wait0();
             __syncthreads();
             if constexpr (MODE == 1) tile_compute_mono<K, PAIR>(p, s0, pb0);
-            else tile_compute<K, PAIR>(p, s0, smat, pb0);
+            else tile_compute<K, PAIR>(p, s0, smat, pb0, splanes);
             __syncthreads();
             store(g, s0);
         }
@@ -1334,6 +1385,9 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     }
     size_t smem = (size_t)STG * ((size_t)8 << p.T);
     if (K == 6 && !d.tci) smem += 64 * 64 * 8;
+#if SVB_SMEM_PLANES
+    if (K >= 2 && K <= 3 && !d.tc && !p.mono) smem += (size_t)3 * 4 << (2 * K);
+#endif
     if constexpr (K >= 4) {
         if (d.tci) smem += TciShape<K>::SMEM;
     }
