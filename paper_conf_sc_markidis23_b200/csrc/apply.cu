@@ -71,6 +71,9 @@ struct MatStore<6> {  // 32 KB complex: does not fit the 32764 B parameter space
 #ifndef SV_ROWS
 #define SV_ROWS 1  // output rows per (non-unrolled) row-loop iteration
 #endif
+#ifndef SVB_WS_STAGES
+#define SVB_WS_STAGES 2  // SIMT bulk-copy loop: tile buffers
+#endif
 #ifndef SVB_SMEM_PLANES
 #define SVB_SMEM_PLANES 1  // dense k = 2, 3 SIMT: Gauss planes read from shared memory (LDS.128)
 #endif
@@ -105,6 +108,7 @@ struct alignas(16) TileParams {
     uint32_t loc[1 << K];              // phys offsets of the gathers (members / member pairs)
     uint32_t gsec;                     // phys offset of the second group of a pair (PAIR, 2 groups)
     const uint8_t* wi8;                // tensor-core int8 path: W slices + column exponents (device)
+    uint64_t roff[64];                 // bulk-copy path: byte offset of run j (dep(j << r))
     // monomial matrices (one nonzero per row: permutations, diagonals, identity)
     int mono;
     uint32_t mloc[1 << K];             // phys offset of member r (output slot of row r)
@@ -221,11 +225,12 @@ __device__ __forceinline__ float2 cmul(float2 m, float2 a) {
 }
 
 template <int K, bool PAIR>
-__device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32_t sbuf, uint32_t pb0) {
+__device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32_t sbuf, uint32_t pb0,
+                                                  uint32_t nt = blockDim.x) {
     constexpr int D = 1 << K;
     constexpr int GPT = (K <= 4) ? 2 : 1;
     for (int j = 0; j < p.iters; ++j) {
-        const uint32_t gidx = threadIdx.x + (uint32_t)j * blockDim.x;
+        const uint32_t gidx = threadIdx.x + (uint32_t)j * nt;
         if constexpr (GPT == 2 && !PAIR) {
             const uint32_t pb = j == 0 ? pb0 : slot_of<K>(p, gidx << 1);
             float4 v[D];
@@ -254,11 +259,11 @@ __device__ __forceinline__ void tile_compute_mono(const TileParams<K>& p, uint32
 
 template <int K, bool PAIR>
 __device__ __forceinline__ void tile_compute(const TileParams<K>& p, uint32_t sbuf, const float2* smat, uint32_t pb0,
-                                             uint32_t splanes) {
+                                             uint32_t splanes, uint32_t nt = blockDim.x) {
     constexpr int D = 1 << K;
     constexpr int GPT = (K <= 4) ? 2 : 1;
     for (int j = 0; j < p.iters; ++j) {
-        const uint32_t gidx = threadIdx.x + (uint32_t)j * blockDim.x;
+        const uint32_t gidx = threadIdx.x + (uint32_t)j * nt;
         if constexpr (GPT == 2) {
             const uint32_t pb = j == 0 ? pb0 : slot_of<K>(p, gidx << 1);
             float2 a0[D], a1[D];
@@ -774,7 +779,15 @@ __device__ __forceinline__ void tci_slots(const TileParams<K>& p, uint32_t (&pbs
 
 // Phase A: gather, slice, issue the MMAs (asynchronous; completion is
 // signalled on t.bar).
-template <int K, bool PAIR>
+// Barrier among the MMA/compute threads only: in the warp-specialised loop
+// (WS) a producer warp does not take part (named barrier 1).
+template <int K, bool WS>
+__device__ __forceinline__ void tci_sync() {
+    if constexpr (WS) asm volatile("bar.sync 1, %0;" ::"n"(TciShape<K>::THREADS) : "memory");
+    else __syncthreads();
+}
+
+template <int K, bool PAIR, bool WS = false>
 __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbuf, TciState& t,
                                             TciRows<TciShape<K>::MB>& rw, const uint32_t (&pbs)[TciShape<K>::MB]) {
     using S = TciShape<K>;
@@ -809,7 +822,7 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
         asm volatile("st.shared.f32 [%0], %1;" ::"r"(t.sM + 4u * ((uint32_t)mb * (128u * TPR) + threadIdx.x)), "f"(mx)
                      : "memory");
     }
-    __syncthreads();
+    tci_sync<K, WS>();
     // 1b. row scale 2^(22 - e) with max|x| < 2^e; slice into A (shared memory)
 #pragma unroll
     for (int mb = 0; mb < S::MB; ++mb) {
@@ -851,7 +864,7 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     tc_fence_before();
-    __syncthreads();
+    tci_sync<K, WS>();
     tc_fence_after();
     // 2. six int8 MMAs per K-step into three exact s32 accumulators
     if (threadIdx.x == 0) {
@@ -889,7 +902,7 @@ __device__ __forceinline__ void tci_phase_a(const TileParams<K>& p, uint32_t sbu
 
 // Phase B: wait for the MMAs, exact recombination of this thread's columns
 // (one rounding), outputs written back into the tile.
-template <int K, bool PAIR>
+template <int K, bool PAIR, bool WS = false>
 __device__ __forceinline__ void tci_phase_b(const TileParams<K>& p, uint32_t sbuf, TciState& t,
                                             const TciRows<TciShape<K>::MB>& rw, const uint32_t (&pbs)[TciShape<K>::MB]) {
     using S = TciShape<K>;
@@ -1134,6 +1147,151 @@ __device__ __forceinline__ void tile_loop(const TileParams<K>& p) {
             store(g, s0);
         }
     }
+}
+
+// ------------------------------------- tensor cores, bulk-copy pipeline
+// For gates with no qubit in {1,2,3} the shared-memory tile is unswizzled
+// (slot = tile index), so each of its 2^nH runs of 2^r contiguous amplitudes
+// is one contiguous block in HBM and in shared memory: the tile moves with
+// 2^nH bulk copies (cp.async.bulk, the TMA engine's non-tensor copy) issued
+// by ONE producer thread instead of 16 B copies from every thread.  A
+// producer warp (warp THREADS/32) streams tiles into NB buffers (mbarrier
+// full[b], transaction-counted) and, once the compute threads have written a
+// tile's outputs (mbarrier done[b]), bulk-stores it and refills the buffer;
+// the compute threads only gather/slice, issue the MMAs and run the
+// epilogue, so a tile's store and the next loads overlap its neighbours'
+// compute.
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+                 "l"(src), "r"(bytes), "r"(bar)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, uint32_t src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Warp-specialised tile loop (bulk copies).  Shared memory: NB tile buffers,
+// then the mode's area (k = 2, 3 Gauss planes / tensor-core state), then
+// 2 NB mbarriers.  The first NT threads compute; warp NT/32 is the producer.
+template <int K, int MODE>
+__host__ __device__ constexpr uint32_t ws_mode_bytes() {
+    if constexpr (MODE == 3) return TciShape<K>::SMEM;
+    else if constexpr (MODE == 0 && K >= 2 && K <= 3) return 3u * 4u << (2 * K);
+    else return 0u;
+}
+template <int K, int MODE>
+__host__ __device__ constexpr int ws_stages() {
+    if constexpr (MODE == 3) return TciShape<K>::STAGES;
+    else return SVB_WS_STAGES;
+}
+
+template <int K, bool PAIR, int MODE>
+__device__ __forceinline__ void ws_loop(const TileParams<K>& p) {
+    constexpr int NB = ws_stages<K, MODE>();
+    extern __shared__ float4 dsm[];
+    const uint32_t NT = blockDim.x - 32u;  // compute threads
+    const uint32_t tile_bytes = 8u << p.T;
+    const uint32_t s0 = smem_addr(dsm);
+    const uint32_t sarea = s0 + NB * tile_bytes;
+    const uint32_t fullb = sarea + ws_mode_bytes<K, MODE>();  // NB x 8 B
+    const uint32_t doneb = fullb + 8u * NB;                   // NB x 8 B
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NB; ++b) {
+            mbar_init(fullb + 8u * b, 1);
+            mbar_init(doneb + 8u * b, 1);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    uint32_t splanes = 0;
+    if constexpr (MODE == 0 && K >= 2 && K <= 3) {
+        constexpr int DD = (1 << K) * (1 << K);
+        float* sp = reinterpret_cast<float*>(reinterpret_cast<char*>(dsm) + NB * tile_bytes);
+        for (int i = threadIdx.x; i < DD; i += blockDim.x) {
+            sp[i] = (&p.M.P[0][0])[i];
+            sp[DD + i] = (&p.M.S[0][0])[i];
+            sp[2 * DD + i] = (&p.M.Q[0][0])[i];
+        }
+        splanes = sarea;
+    }
+    TciState tis{};
+    if constexpr (MODE == 3) tis = tci_setup<K>(p, sarea);  // __syncthreads inside
+    else __syncthreads();
+    const uint64_t G = gridDim.x;
+    if (threadIdx.x >= NT) {
+        if (threadIdx.x == NT) {
+            // producer: refill buffer b once the compute threads are done with
+            // its previous tile and that tile's bulk store has read it
+            const uint32_t nrun = 1u << p.nH, rbytes = 8u << p.r;
+            char* gb[NB];
+            int i = 0;
+            for (uint64_t u = blockIdx.x; u < p.n_tiles; u += G, ++i) {
+                const int b = i % NB;
+                const uint32_t sb = s0 + (uint32_t)b * tile_bytes;
+                if (i >= NB) {
+                    mbar_wait(doneb + 8u * b, (uint32_t)(i / NB - 1) & 1u);
+                    for (uint32_t j = 0; j < nrun; ++j) bulk_store(gb[b] + p.roff[j], sb + j * rbytes, rbytes);
+                    bulk_commit();
+                    bulk_wait_read0();
+                }
+                gb[b] = reinterpret_cast<char*>(p.psi + tile_base(p, u));
+                mbar_expect_tx(fullb + 8u * b, tile_bytes);
+                for (uint32_t j = 0; j < nrun; ++j) bulk_load(sb + j * rbytes, gb[b] + p.roff[j], rbytes, fullb + 8u * b);
+            }
+            for (int t = i > NB ? i - NB : 0; t < i; ++t) {
+                const int b = t % NB;
+                mbar_wait(doneb + 8u * b, (uint32_t)(t / NB) & 1u);
+                for (uint32_t j = 0; j < nrun; ++j)
+                    bulk_store(gb[b] + p.roff[j], s0 + (uint32_t)b * tile_bytes + j * rbytes, rbytes);
+                bulk_commit();
+            }
+            bulk_wait0();
+        }
+    } else {
+        uint32_t tslot[MODE == 3 ? TciShape<K>::MB : 1];
+        if constexpr (MODE == 3) tci_slots<K>(p, tslot);
+        const uint32_t pb0 = slot_of<K>(p, K <= 4 ? (threadIdx.x << 1) : threadIdx.x);
+        int i = 0;
+        for (uint64_t u = blockIdx.x; u < p.n_tiles; u += G, ++i) {
+            const int b = i % NB;
+            const uint32_t sb = s0 + (uint32_t)b * tile_bytes;
+            mbar_wait(fullb + 8u * b, (uint32_t)(i / NB) & 1u);
+            if constexpr (MODE == 3) {
+                TciRows<TciShape<K>::MB> rw;
+                tci_phase_a<K, PAIR, true>(p, sb, tis, rw, tslot);
+                tci_phase_b<K, PAIR, true>(p, sb, tis, rw, tslot);
+            } else if constexpr (MODE == 1) {
+                tile_compute_mono<K, PAIR>(p, sb, pb0, NT);
+            } else {
+                tile_compute<K, PAIR>(p, sb, nullptr, pb0, splanes, NT);
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // outputs -> async proxy (bulk store)
+            asm volatile("bar.sync 1, %0;" ::"r"(NT) : "memory");
+            if (threadIdx.x == 0) mbar_arrive(doneb + 8u * b);
+        }
+    }
+    if constexpr (MODE == 3) tci_teardown<K>(tis);
+}
+
+template <int K, bool PAIR>
+__global__ void __launch_bounds__(TciShape<K>::THREADS + 32, K == 6 ? 1 : 2) apply_tci_ws(const __grid_constant__ TileParams<K> p) {
+    ws_loop<K, PAIR, 3>(p);
+}
+template <int K, bool PAIR, bool MONO>
+__global__ void __launch_bounds__(256 + 32) apply_high_ws(const __grid_constant__ TileParams<K> p) {
+    ws_loop<K, PAIR, MONO ? 1 : 0>(p);
 }
 
 __host__ __device__ constexpr int stages_for(int K) { return K == 6 ? 1 : 2; }
@@ -1391,21 +1549,36 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     if constexpr (K >= 4) {
         if (d.tci) smem += TciShape<K>::SMEM;
     }
+    // Bulk-copy (warp-specialised) loop: unswizzled tiles only, i.e. no
+    // gate qubit in {1,2,3}; the int8 tensor-core path and the SIMT path
+    // for k <= 5 (not the TF32 or small-state paths).
+    const bool unswz = p.swz[0] == 0 && p.swz[1] == 0 && p.swz[2] == 0 && p.nH <= 6;
+    const bool ws = unswz && std::getenv("SVB200_NO_WS") == nullptr && (d.tci || (!d.tc && K <= 5));
+    if (ws) {
+        for (uint32_t j = 0; j < (1u << p.nH); ++j) p.roff[j] = 8ull * dep((uint64_t)j << p.r);
+        const int nb = d.tci ? STG : SVB_WS_STAGES;
+        smem = (size_t)nb * ((size_t)8 << p.T) + 16u * nb;
+        if constexpr (K >= 4) {
+            if (d.tci) smem += TciShape<K>::SMEM;
+        }
+        if (!d.tci && !p.mono && K >= 2 && K <= 3) smem += (size_t)3 * 4 << (2 * K);
+    }
     if constexpr (K == 4 || K == 5) {
         if (d.tc && !d.tci) smem += 2 * TcShape<K>::W_BYTES + 64;
     }
     const int per_sm_smem = std::max(1, (int)((227 * 1024) / (smem + 1024)));
     const uint64_t grid = std::max<uint64_t>(1, std::min<uint64_t>(p.n_tiles, (uint64_t)num_sms() * per_sm_smem));
-    auto go = [&](auto kern) -> cudaError_t {
+    auto go = [&](auto kern, uint32_t threads = 0) -> cudaError_t {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        kern<<<(unsigned)grid, nthr, smem, st>>>(p);
+        kern<<<(unsigned)grid, threads ? threads : nthr, smem, st>>>(p);
         return cudaGetLastError();
     };
     if constexpr (K >= 4) {
         if (d.tci) {
             if (p.T != TciShape<K>::T) return cudaErrorInvalidConfiguration;
             p.wi8 = d.dev_wi8;
+            if (ws) return pair ? go(apply_tci_ws<K, true>, nthr + 32) : go(apply_tci_ws<K, false>, nthr + 32);
             return pair ? go(apply_tci<K, true>) : go(apply_tci<K, false>);
         }
     }
@@ -1413,6 +1586,12 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         if (d.tc) {
             if (p.T != 12) return cudaErrorInvalidConfiguration;
             return pair ? go(apply_tc<K, true>) : go(apply_tc<K, false>);
+        }
+    }
+    if constexpr (K <= 5) {
+        if (ws) {
+            if (p.mono) return pair ? go(apply_high_ws<K, true, true>, nthr + 32) : go(apply_high_ws<K, false, true>, nthr + 32);
+            return pair ? go(apply_high_ws<K, true, false>, nthr + 32) : go(apply_high_ws<K, false, false>, nthr + 32);
         }
     }
     if (p.mono) {
