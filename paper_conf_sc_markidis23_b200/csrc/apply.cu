@@ -24,6 +24,7 @@
 // The fused matrix (k <= 5) travels in the kernel parameters
 // (__grid_constant__), so the unrolled FMAs read it from the constant bank;
 // k = 6 (32 KB) is staged in shared memory once per CTA.
+#include <cuda.h>  // CUtensorMap (the encoder is fetched with cudaGetDriverEntryPoint)
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -87,7 +88,7 @@ struct MatStore<6> {  // 32 KB complex: does not fit the 32764 B parameter space
 // are additive/XOR-linear over disjoint bits, so per-unit offsets are
 // precomputed on the host and a thread adds/XORs them to its own base.
 template <int K>
-struct alignas(16) TileParams {
+struct alignas(64) TileParams {
     MatStore<K> M;                     // first: 16 B aligned in the constant bank (LDCU.128)
     float2* psi;
     uint64_t n_tiles;
@@ -109,6 +110,11 @@ struct alignas(16) TileParams {
     uint32_t gsec;                     // phys offset of the second group of a pair (PAIR, 2 groups)
     const uint8_t* wi8;                // tensor-core int8 path: W slices + column exponents (device)
     uint64_t roff[64];                 // bulk-copy path: byte offset of run j (dep(j << r))
+    int trank;                         // tensor-copy path: rank (0 = per-run bulk copies)
+    int tstart[5], tbits[5];           // dim d covers index bits [tstart[d], tstart[d] + tbits[d])
+    int tnx;                           // gate qubits left out of the box: 2^tnx copies per tile
+    int txpos[SV_MAX_FUSED];           // their positions (ascending)
+    CUtensorMap tmap;                  // tensor map of the state for this gate's tile shape
     // monomial matrices (one nonzero per row: permutations, diagonals, identity)
     int mono;
     uint32_t mloc[1 << K];             // phys offset of member r (output slot of row r)
@@ -1179,6 +1185,55 @@ __device__ __forceinline__ void bulk_store(void* dst, uint32_t src, uint32_t byt
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes)
                  : "memory");
 }
+// Tensor copies (rank 2..5): coordinates c[d] in elements of 8 B.
+__device__ __forceinline__ void tensor_load(int rank, uint32_t dst, const void* tmap, const int* c, uint32_t bar) {
+    const uint64_t m = reinterpret_cast<uint64_t>(tmap);
+    switch (rank) {
+        case 2:
+            asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                         ::"r"(dst), "l"(m), "r"(c[0]), "r"(c[1]), "r"(bar) : "memory");
+            break;
+        case 3:
+            asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
+                         ::"r"(dst), "l"(m), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(bar) : "memory");
+            break;
+        case 4:
+            asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];"
+                         ::"r"(dst), "l"(m), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]), "r"(bar) : "memory");
+            break;
+        default:
+            asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"
+                         ::"r"(dst), "l"(m), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]), "r"(c[4]), "r"(bar) : "memory");
+            break;
+    }
+}
+__device__ __forceinline__ void tensor_store(int rank, const void* tmap, const int* c, uint32_t src) {
+    const uint64_t m = reinterpret_cast<uint64_t>(tmap);
+    switch (rank) {
+        case 2:
+            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
+                         ::"l"(m), "r"(src), "r"(c[0]), "r"(c[1]) : "memory");
+            break;
+        case 3:
+            asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];"
+                         ::"l"(m), "r"(src), "r"(c[0]), "r"(c[1]), "r"(c[2]) : "memory");
+            break;
+        case 4:
+            asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];"
+                         ::"l"(m), "r"(src), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]) : "memory");
+            break;
+        default:
+            asm volatile("cp.async.bulk.tensor.5d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];"
+                         ::"l"(m), "r"(src), "r"(c[0]), "r"(c[1]), "r"(c[2]), "r"(c[3]), "r"(c[4]) : "memory");
+            break;
+    }
+}
+template <int K>
+__device__ __forceinline__ void tensor_coords(const TileParams<K>& p, uint64_t base, int* c) {
+#pragma unroll
+    for (int d = 0; d < 5; ++d)
+        c[d] = d < p.trank ? (int)((base >> p.tstart[d]) & ((1ull << p.tbits[d]) - 1ull)) : 0;
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
@@ -1231,33 +1286,78 @@ __device__ __forceinline__ void ws_loop(const TileParams<K>& p) {
     else __syncthreads();
     const uint64_t G = gridDim.x;
     if (threadIdx.x >= NT) {
-        if (threadIdx.x == NT) {
-            // producer: refill buffer b once the compute threads are done with
-            // its previous tile and that tile's bulk store has read it
-            const uint32_t nrun = 1u << p.nH, rbytes = 8u << p.r;
-            char* gb[NB];
-            int i = 0;
-            for (uint64_t u = blockIdx.x; u < p.n_tiles; u += G, ++i) {
-                const int b = i % NB;
-                const uint32_t sb = s0 + (uint32_t)b * tile_bytes;
-                if (i >= NB) {
-                    mbar_wait(doneb + 8u * b, (uint32_t)(i / NB - 1) & 1u);
-                    for (uint32_t j = 0; j < nrun; ++j) bulk_store(gb[b] + p.roff[j], sb + j * rbytes, rbytes);
+        // producer warp: its 32 lanes issue the runs' bulk copies round-robin
+        // (runs can be as small as 1 KB; one thread alone measured slower)
+        const uint32_t lane = threadIdx.x - NT;
+        const uint32_t nrun = 1u << p.nH, rbytes = 8u << p.r;
+        if (p.trank > 0) {
+            // one tensor copy per tile (loads) / per tile (stores)
+            if (lane == 0) {
+                const uint32_t nops = 1u << p.tnx, obytes = tile_bytes >> p.tnx;
+                auto xoff = [&](uint32_t o) {  // o's bits at the gate qubits left out of the box
+                    uint64_t x = 0;
+                    for (int e = 0; e < p.tnx; ++e) x |= (uint64_t)((o >> e) & 1u) << p.txpos[e];
+                    return x;
+                };
+                auto store_tile = [&](uint64_t base, uint32_t sb) {
+                    int c[5];
+                    for (uint32_t o = 0; o < nops; ++o) {
+                        tensor_coords(p, base | xoff(o), c);
+                        tensor_store(p.trank, &p.tmap, c, sb + o * obytes);
+                    }
                     bulk_commit();
-                    bulk_wait_read0();
+                };
+                uint64_t gbase[NB];
+                int i = 0;
+                for (uint64_t u = blockIdx.x; u < p.n_tiles; u += G, ++i) {
+                    const int b = i % NB;
+                    const uint32_t sb = s0 + (uint32_t)b * tile_bytes;
+                    if (i >= NB) {
+                        mbar_wait(doneb + 8u * b, (uint32_t)(i / NB - 1) & 1u);
+                        store_tile(gbase[b], sb);
+                        bulk_wait_read0();
+                    }
+                    gbase[b] = tile_base(p, u);
+                    mbar_expect_tx(fullb + 8u * b, tile_bytes);
+                    for (uint32_t o = 0; o < nops; ++o) {
+                        int c[5];
+                        tensor_coords(p, gbase[b] | xoff(o), c);
+                        tensor_load(p.trank, sb + o * obytes, &p.tmap, c, fullb + 8u * b);
+                    }
                 }
-                gb[b] = reinterpret_cast<char*>(p.psi + tile_base(p, u));
-                mbar_expect_tx(fullb + 8u * b, tile_bytes);
-                for (uint32_t j = 0; j < nrun; ++j) bulk_load(sb + j * rbytes, gb[b] + p.roff[j], rbytes, fullb + 8u * b);
+                for (int t = i > NB ? i - NB : 0; t < i; ++t) {
+                    const int b = t % NB;
+                    mbar_wait(doneb + 8u * b, (uint32_t)(t / NB) & 1u);
+                    store_tile(gbase[b], s0 + (uint32_t)b * tile_bytes);
+                }
+                bulk_wait0();
             }
-            for (int t = i > NB ? i - NB : 0; t < i; ++t) {
-                const int b = t % NB;
-                mbar_wait(doneb + 8u * b, (uint32_t)(t / NB) & 1u);
-                for (uint32_t j = 0; j < nrun; ++j)
-                    bulk_store(gb[b] + p.roff[j], s0 + (uint32_t)b * tile_bytes + j * rbytes, rbytes);
+        } else {
+        char* gb[NB];
+        int i = 0;
+        for (uint64_t u = blockIdx.x; u < p.n_tiles; u += G, ++i) {
+            const int b = i % NB;
+            const uint32_t sb = s0 + (uint32_t)b * tile_bytes;
+            if (i >= NB) {
+                mbar_wait(doneb + 8u * b, (uint32_t)(i / NB - 1) & 1u);
+                for (uint32_t j = lane; j < nrun; j += 32) bulk_store(gb[b] + p.roff[j], sb + j * rbytes, rbytes);
                 bulk_commit();
+                bulk_wait_read0();
+                __syncwarp();
             }
-            bulk_wait0();
+            gb[b] = reinterpret_cast<char*>(p.psi + tile_base(p, u));
+            if (lane == 0) mbar_expect_tx(fullb + 8u * b, tile_bytes);
+            __syncwarp();
+            for (uint32_t j = lane; j < nrun; j += 32) bulk_load(sb + j * rbytes, gb[b] + p.roff[j], rbytes, fullb + 8u * b);
+        }
+        for (int t = i > NB ? i - NB : 0; t < i; ++t) {
+            const int b = t % NB;
+            mbar_wait(doneb + 8u * b, (uint32_t)(t / NB) & 1u);
+            for (uint32_t j = lane; j < nrun; j += 32)
+                bulk_store(gb[b] + p.roff[j], s0 + (uint32_t)b * tile_bytes + j * rbytes, rbytes);
+            bulk_commit();
+        }
+        bulk_wait0();
         }
     } else {
         uint32_t tslot[MODE == 3 ? TciShape<K>::MB : 1];
@@ -1394,6 +1494,82 @@ void fill_matrix<6>(MatStore<6>& M, const ApplyDesc& d) {
     M.dev = d.dev_m;
 }
 
+// Tensor map of the state for a tile of 2^nH runs of 2^r amplitudes (run j
+// at dep(j << r)).  Dimension 0 covers index bits [0, H_0) with a box of 2^r
+// (the run); every maximal group of consecutive gate qubits H_g..H_g+m-1
+// opens a dimension covering bits [H_g, next group) with a box of 2^m (the
+// gate bits are its low bits, the tile base supplies the rest as the
+// coordinate).  The box is then exactly the tile in tile-index order, and
+// one tensor copy moves a whole tile (runs longer than 256 amplitudes take
+// two dimensions; groups beyond rank 5 are iterated: 2^nx copies per tile).
+// rank = 0 when it does not fit or the driver has no encoder: per-run copies.
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn tensor_map_encoder() {
+    static EncodeTiledFn fn = []() -> EncodeTiledFn {
+        void* f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            return nullptr;
+        return reinterpret_cast<EncodeTiledFn>(f);
+    }();
+    return fn;
+}
+void encode_tile_map(CUtensorMap& map, int& rank, int* tstart, int* tbits, int& nx, int* xpos, float2* psi, int n,
+                     int r, const int* H, int nH) {
+    rank = 0;
+    nx = 0;
+    if (r > 16) return;
+    // dimension(s) of the run: [0, min(8, r)) and, for r > 8, [8, H_0) with a box of 2^(r-8)
+    int start[12], hbits[12], nd = 0;
+    start[nd] = 0;
+    hbits[nd] = std::min(r, 8);
+    ++nd;
+    if (r > 8) {
+        start[nd] = 8;
+        hbits[nd] = r - 8;
+        ++nd;
+    }
+    int gfirst[SV_MAX_FUSED + 1], ng = 0;  // first H index of each group of consecutive gate qubits
+    for (int b = 0; b < nH; ++b)
+        if (b == 0 || H[b] != H[b - 1] + 1) gfirst[ng++] = b;
+    gfirst[ng] = nH;
+    const int keep = std::min(ng, 5 - nd);  // groups with their own dimension
+    for (int g = 0; g < keep; ++g) {
+        start[nd] = H[gfirst[g]];
+        hbits[nd] = gfirst[g + 1] - gfirst[g];
+        ++nd;
+    }
+    for (int b = gfirst[keep]; b < nH; ++b) xpos[nx++] = H[b];  // the rest: one copy per combination
+    if (nx > 4) return;
+    cuuint64_t gdim[5], gstride[4];
+    cuuint32_t box[5], estr[5];
+    for (int d = 0; d < nd; ++d) {
+        const int end = d + 1 < nd ? start[d + 1] : n;
+        const int bits = end - start[d];
+        if (bits > 31 || bits < hbits[d] || hbits[d] > 8) {
+            nx = 0;
+            return;
+        }
+        gdim[d] = 1ull << bits;
+        box[d] = 1u << hbits[d];
+        estr[d] = 1;
+        if (d > 0) gstride[d - 1] = 8ull << start[d];
+        tstart[d] = start[d];
+        tbits[d] = bits;
+    }
+    EncodeTiledFn enc = tensor_map_encoder();
+    if (!enc || enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)nd, psi, gdim, gstride, box, estr,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+        nx = 0;
+        return;
+    }
+    rank = nd;
+}
+
 template <int K>
 cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t st) {
     constexpr int GPT = (K <= 4) ? 2 : 1;
@@ -1444,6 +1620,34 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     size_t jh = 0;
     for (int f = 1; f <= 3; ++f)
         if (((fixed >> f) & 1) && jh < hl.size()) p.swz[f - 1] = 1u << hl[jh++];
+    // Bulk-copy (warp-specialised) loop: it needs an unswizzled tile.  Gates
+    // with no qubit in {1,2,3} are unswizzled anyway; for the others the
+    // swizzle is dropped (2-4-way bank conflicts on the gathers) where that
+    // measured faster at 30 qubits: SIMT k = 1, 2, 4 and the
+    // int8 tensor-core path k <= 5 (k = 6: 4-way conflicts, slower).
+    // k = 3 SIMT keeps the 16 B-copy loop (bulk copies measured 0.7 % slower).
+    bool ws = false;
+    {
+        const bool natural = p.swz[0] == 0 && p.swz[1] == 0 && p.swz[2] == 0;
+        const bool simt = !d.tc && K <= 5 && K != 3;
+        const bool low_ok = (simt && K != 5) || (d.tci && K <= 5);
+        const char* ev = std::getenv("SVB200_WS_UNSWZ");
+        const bool force = ev != nullptr && ev[0] == '1', never = ev != nullptr && ev[0] == '0';
+        // bulk copies of runs below ~2 KB measured slower than the 16 B-copy loop
+        const char* mr = std::getenv("SVB200_WS_MINRUN");
+        const uint32_t minrun = mr ? (uint32_t)std::atoi(mr) : 2048u;
+        // runs of <= 1 KB (and every k = 6 tensor-core tile) move as tensor
+        // copies (encode_tile_map): per-run bulk copies of 1 KB measured 10-40 %
+        // slower, tensor copies of >= 2 KB runs 1-5 % slower than bulk copies
+        const char* tm = std::getenv("SVB200_TMAP");
+        const bool tmap = tm ? tm[0] == '1' : (p.r <= 7 || (d.tci && K == 6) || (gpt == 2 && pair));
+        if ((simt || d.tci) && tmap)
+            encode_tile_map(p.tmap, p.trank, p.tstart, p.tbits, p.tnx, p.txpos, psi, n, p.r, p.Hpos, p.nH);
+        ws = std::getenv("SVB200_NO_WS") == nullptr && p.nH <= 6 && (simt || d.tci) &&
+             ((8u << p.r) >= minrun || p.trank > 0) &&
+             (natural || (!never && (low_ok || force)));
+        if (ws) p.swz[0] = p.swz[1] = p.swz[2] = 0;
+    }
     auto sw = [&](uint32_t t) {
         return t ^ ((__builtin_popcount(t & p.swz[0]) & 1) << 1) ^ ((__builtin_popcount(t & p.swz[1]) & 1) << 2) ^
                ((__builtin_popcount(t & p.swz[2]) & 1) << 3);
@@ -1549,11 +1753,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     if constexpr (K >= 4) {
         if (d.tci) smem += TciShape<K>::SMEM;
     }
-    // Bulk-copy (warp-specialised) loop: unswizzled tiles only, i.e. no
-    // gate qubit in {1,2,3}; the int8 tensor-core path and the SIMT path
-    // for k <= 5 (not the TF32 or small-state paths).
-    const bool unswz = p.swz[0] == 0 && p.swz[1] == 0 && p.swz[2] == 0 && p.nH <= 6;
-    const bool ws = unswz && std::getenv("SVB200_NO_WS") == nullptr && (d.tci || (!d.tc && K <= 5));
+    // bulk-copy loop: run offsets, and its shared memory (tiles, mode area, mbarriers)
     if (ws) {
         for (uint32_t j = 0; j < (1u << p.nH); ++j) p.roff[j] = 8ull * dep((uint64_t)j << p.r);
         const int nb = d.tci ? STG : SVB_WS_STAGES;
