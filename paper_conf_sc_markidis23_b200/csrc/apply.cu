@@ -1570,6 +1570,60 @@ void encode_tile_map(CUtensorMap& map, int& rank, int* tstart, int* tbits, int& 
     rank = nd;
 }
 
+// Bank-conflict factor (wavefronts / ideal) of the group gathers of warp 0 if
+// the tile is NOT swizzled: 16 B words are served per quarter warp, 8 B per
+// half warp; a phase costs as many wavefronts as the most distinct words in
+// one bank group.  gpt = 2: lane t gathers the group pair (2t, 2t+1) (or,
+// PAIR, groups 2t and its partner at bit ng0); gpt = 1: lane t one group.
+double unswizzled_conflicts(int K, int gpt, bool pair, const int* tl, int ng0) {
+    auto slot = [&](uint32_t g) {
+        for (int b = 0; b < K; ++b) g += g & (~0u << tl[b]);
+        return g;
+    };
+    auto locf = [&](int mm) {
+        uint32_t o = 0;
+        for (int b = 0; b < K; ++b)
+            if ((mm >> b) & 1) o |= 1u << tl[b];
+        return o;
+    };
+    int wf = 0, ideal = 0;
+    auto count = [&](const uint32_t* addr, int bytes) {
+        const int lpp = 128 / bytes;
+        for (int ph = 0; ph < 32; ph += lpp) {
+            int worst = 0;
+            for (int bank = 0; bank < lpp; ++bank) {
+                uint32_t seen[32];
+                int ns = 0;
+                for (int l = ph; l < ph + lpp; ++l) {
+                    if ((int)((addr[l] / bytes) % lpp) != bank) continue;
+                    bool dup = false;
+                    for (int s = 0; s < ns; ++s) dup |= seen[s] == addr[l];
+                    if (!dup) seen[ns++] = addr[l];
+                }
+                worst = std::max(worst, ns);
+            }
+            wf += worst;
+            ++ideal;
+        }
+    };
+    const int D = 1 << K;
+    uint32_t a[32];
+    if (gpt == 2) {
+        for (int m = 0; m < (pair ? D / 2 : D); ++m)
+            for (int h = 0; h < (pair ? 2 : 1); ++h) {
+                for (int t = 0; t < 32; ++t)
+                    a[t] = 8u * (slot(2u * t) ^ (h ? (1u << ng0) : 0u) ^ locf(pair ? 2 * m : m));
+                count(a, 16);
+            }
+    } else {
+        for (int m = 0; m < (pair ? D / 2 : D); ++m) {
+            for (int t = 0; t < 32; ++t) a[t] = 8u * (slot((uint32_t)t) ^ locf(pair ? 2 * m : m));
+            count(a, pair ? 16 : 8);
+        }
+    }
+    return ideal ? (double)wf / ideal : 1.0;
+}
+
 template <int K>
 cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t st) {
     constexpr int GPT = (K <= 4) ? 2 : 1;
@@ -1630,7 +1684,11 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     {
         const bool natural = p.swz[0] == 0 && p.swz[1] == 0 && p.swz[2] == 0;
         const bool simt = !d.tc && K <= 5 && K != 3;
-        const bool low_ok = (simt && K != 5) || (d.tci && K <= 5);
+        // ... and only where the unswizzled gathers are at most 2-way (tensor
+        // cores) / 4-way (SIMT) conflicted: 4-way measured 3 % faster on SIMT
+        // k = 4, 2 % slower on the k = 6 tensor-core path, 8-way much slower
+        const double cf = (simt || d.tci) ? unswizzled_conflicts(K, gpt, pair, tl, ng[0]) : 99.0;
+        const bool low_ok = (simt && K != 5 && cf <= 4.0) || (d.tci && K <= 5 && cf <= 2.0);
         const char* ev = std::getenv("SVB200_WS_UNSWZ");
         const bool force = ev != nullptr && ev[0] == '1', never = ev != nullptr && ev[0] == '0';
         // bulk copies of runs below ~2 KB measured slower than the 16 B-copy loop

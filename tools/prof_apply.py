@@ -16,7 +16,7 @@ from workloads import rqc as W
 CASES = {
     "h1": (20,), "l1": (2,), "h2": (10, 20), "l2": (1, 20), "h3": (5, 12, 25), "l3": (2, 12, 25),
     "h4": (6, 12, 18, 24), "l4": (2, 12, 18, 24), "l4b": (1, 2, 12, 24), "q0": (0, 12, 18, 24),
-    "r4": (10, 11, 12, 13), "r5": (10, 11, 12, 13, 14), "r6": (12, 13, 14, 15, 16, 17),
+    "p4": (0, 1, 2, 3), "p4b": (0, 6, 25, 26), "p4c": (0, 2, 6, 8), "r4": (10, 11, 12, 13), "r5": (10, 11, 12, 13, 14), "r6": (12, 13, 14, 15, 16, 17),
     "h5": (4, 8, 12, 18, 24), "l5": (1, 8, 12, 18, 24), "h6": (4, 8, 12, 16, 20, 24), "l6": (1, 3, 8, 12, 20, 24),
 }
 
