@@ -27,9 +27,11 @@ CASES = {
     1: {"high": (20,), "low": (2,), "q0": (0,)},
     2: {"high": (10, 20), "low": (1, 20), "q0": (0, 20)},
     3: {"high": (5, 12, 25), "low": (2, 12, 25), "q0": (0, 12, 25)},
-    4: {"high": (6, 12, 18, 24), "low": (2, 12, 18, 24), "q0": (0, 12, 18, 24), "low2": (1, 2, 12, 24)},
-    5: {"high": (4, 8, 12, 18, 24), "low": (1, 8, 12, 18, 24), "q0": (0, 8, 12, 18, 24)},
-    6: {"high": (4, 8, 12, 16, 20, 24), "low": (1, 3, 8, 12, 20, 24), "q0": (0, 4, 8, 12, 20, 24)},
+    4: {"high": (6, 12, 18, 24), "low": (2, 12, 18, 24), "q0": (0, 12, 18, 24), "low2": (1, 2, 12, 24),
+        "run2k": (10, 11, 12, 13), "q0123": (0, 1, 2, 3)},
+    5: {"high": (4, 8, 12, 18, 24), "low": (1, 8, 12, 18, 24), "q0": (0, 8, 12, 18, 24), "run1k": (10, 11, 12, 13, 14)},
+    6: {"high": (4, 8, 12, 16, 20, 24), "low": (1, 3, 8, 12, 20, 24), "q0": (0, 4, 8, 12, 20, 24),
+        "run1k": (12, 13, 14, 15, 16, 17)},
 }
 n = 30
 h = sv.sv_create(n)
