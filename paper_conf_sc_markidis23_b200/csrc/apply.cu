@@ -1259,7 +1259,7 @@ __device__ __forceinline__ void ws_loop(const TileParams<K>& p) {
     extern __shared__ float4 dsm[];
     const uint32_t NT = blockDim.x - 32u;  // compute threads
     const uint32_t tile_bytes = 8u << p.T;
-    const uint32_t s0 = smem_addr(dsm);
+    const uint32_t s0 = (smem_addr(dsm) + 1023u) & ~1023u;  // the 128 B swizzle repeats every 1 KB
     const uint32_t sarea = s0 + NB * tile_bytes;
     const uint32_t fullb = sarea + ws_mode_bytes<K, MODE>();  // NB x 8 B
     const uint32_t doneb = fullb + 8u * NB;                   // NB x 8 B
@@ -1273,7 +1273,7 @@ __device__ __forceinline__ void ws_loop(const TileParams<K>& p) {
     uint32_t splanes = 0;
     if constexpr (MODE == 0 && K >= 2 && K <= 3) {
         constexpr int DD = (1 << K) * (1 << K);
-        float* sp = reinterpret_cast<float*>(reinterpret_cast<char*>(dsm) + NB * tile_bytes);
+        float* sp = reinterpret_cast<float*>(reinterpret_cast<char*>(dsm) + (s0 - smem_addr(dsm)) + NB * tile_bytes);
         for (int i = threadIdx.x; i < DD; i += blockDim.x) {
             sp[i] = (&p.M.P[0][0])[i];
             sp[DD + i] = (&p.M.S[0][0])[i];
@@ -1518,18 +1518,20 @@ EncodeTiledFn tensor_map_encoder() {
     return fn;
 }
 void encode_tile_map(CUtensorMap& map, int& rank, int* tstart, int* tbits, int& nx, int* xpos, float2* psi, int n,
-                     int r, const int* H, int nH) {
+                     int r, const int* H, int nH, bool swz128) {
     rank = 0;
     nx = 0;
-    if (r > 16) return;
-    // dimension(s) of the run: [0, min(8, r)) and, for r > 8, [8, H_0) with a box of 2^(r-8)
+    // dimension(s) of the run: [0, c) and, for r > c, [c, H_0) with a box of 2^(r-c); c = 8
+    // (256 amplitudes, the box limit), or 4 (128 B rows) with the 128 B swizzle
+    const int c = swz128 ? 4 : 8;
+    if (r > c + 8 || (swz128 && r < c)) return;
     int start[12], hbits[12], nd = 0;
     start[nd] = 0;
-    hbits[nd] = std::min(r, 8);
+    hbits[nd] = std::min(r, c);
     ++nd;
-    if (r > 8) {
-        start[nd] = 8;
-        hbits[nd] = r - 8;
+    if (r > c) {
+        start[nd] = c;
+        hbits[nd] = r - c;
         ++nd;
     }
     int gfirst[SV_MAX_FUSED + 1], ng = 0;  // first H index of each group of consecutive gate qubits
@@ -1562,7 +1564,8 @@ void encode_tile_map(CUtensorMap& map, int& rank, int* tstart, int* tbits, int& 
     }
     EncodeTiledFn enc = tensor_map_encoder();
     if (!enc || enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)nd, psi, gdim, gstride, box, estr,
-                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, swz128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
         nx = 0;
         return;
@@ -1570,12 +1573,16 @@ void encode_tile_map(CUtensorMap& map, int& rank, int* tstart, int* tbits, int& 
     rank = nd;
 }
 
-// Bank-conflict factor (wavefronts / ideal) of the group gathers of warp 0 if
-// the tile is NOT swizzled: 16 B words are served per quarter warp, 8 B per
+// Bank-conflict factor (wavefronts / ideal) of the group gathers of warp 0 for
+// a tile laid out with XOR swizzle swz (phys bit i+1 ^= parity(t & swz[i])): 16 B words are served per quarter warp, 8 B per
 // half warp; a phase costs as many wavefronts as the most distinct words in
 // one bank group.  gpt = 2: lane t gathers the group pair (2t, 2t+1) (or,
 // PAIR, groups 2t and its partner at bit ng0); gpt = 1: lane t one group.
-double unswizzled_conflicts(int K, int gpt, bool pair, const int* tl, int ng0) {
+double gather_conflicts(int K, int gpt, bool pair, const int* tl, int ng0, const uint32_t* swz) {
+    auto phys = [&](uint32_t t) {
+        return t ^ ((__builtin_popcount(t & swz[0]) & 1) << 1) ^ ((__builtin_popcount(t & swz[1]) & 1) << 2) ^
+               ((__builtin_popcount(t & swz[2]) & 1) << 3);
+    };
     auto slot = [&](uint32_t g) {
         for (int b = 0; b < K; ++b) g += g & (~0u << tl[b]);
         return g;
@@ -1612,12 +1619,12 @@ double unswizzled_conflicts(int K, int gpt, bool pair, const int* tl, int ng0) {
         for (int m = 0; m < (pair ? D / 2 : D); ++m)
             for (int h = 0; h < (pair ? 2 : 1); ++h) {
                 for (int t = 0; t < 32; ++t)
-                    a[t] = 8u * (slot(2u * t) ^ (h ? (1u << ng0) : 0u) ^ locf(pair ? 2 * m : m));
+                    a[t] = 8u * phys(slot(2u * t) ^ (h ? (1u << ng0) : 0u) ^ locf(pair ? 2 * m : m));
                 count(a, 16);
             }
     } else {
         for (int m = 0; m < (pair ? D / 2 : D); ++m) {
-            for (int t = 0; t < 32; ++t) a[t] = 8u * (slot((uint32_t)t) ^ locf(pair ? 2 * m : m));
+            for (int t = 0; t < 32; ++t) a[t] = 8u * phys(slot((uint32_t)t) ^ locf(pair ? 2 * m : m));
             count(a, pair ? 16 : 8);
         }
     }
@@ -1674,37 +1681,58 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     size_t jh = 0;
     for (int f = 1; f <= 3; ++f)
         if (((fixed >> f) & 1) && jh < hl.size()) p.swz[f - 1] = 1u << hl[jh++];
-    // Bulk-copy (warp-specialised) loop: it needs an unswizzled tile.  Gates
-    // with no qubit in {1,2,3} are unswizzled anyway; for the others the
-    // swizzle is dropped (2-4-way bank conflicts on the gathers) where that
-    // measured faster at 30 qubits: SIMT k = 1, 2, 4 and the
-    // int8 tensor-core path k <= 5 (k = 6: 4-way conflicts, slower).
-    // k = 3 SIMT keeps the 16 B-copy loop (bulk copies measured 0.7 % slower).
-    bool ws = false;
+    // Bulk-copy (warp-specialised) loop.  A bulk copy cannot apply the 16 B XOR
+    // swizzle of the 16 B-copy loop, so its tiles are either unswizzled or
+    // laid out with the TMA's 128 B swizzle (16 B chunk bits 1..3 ^= amplitude
+    // bits 4..6, tensor copies only).  Gates with no qubit in {1,2,3} need no
+    // swizzle; for the others the layout with fewer bank conflicts on the group
+    // gathers is taken (host model, gather_conflicts) when it is at most 2-way
+    // (tensor cores) / 4-way (SIMT) conflicted -- measured at 30 qubits
+    // (DESIGN.md §11): 2-way always beats the swizzled 16 B-copy loop, 4-way
+    // breaks even on SIMT k = 4 and loses on the k = 6 tensor-core path,
+    // 8-way loses badly.  k = 3 SIMT keeps the 16 B-copy loop (0.7 % faster).
+    bool ws = false, swz128 = false;
     {
+        static const uint32_t kNone[3] = {0u, 0u, 0u}, k128[3] = {1u << 4, 1u << 5, 1u << 6};
         const bool natural = p.swz[0] == 0 && p.swz[1] == 0 && p.swz[2] == 0;
         const bool simt = !d.tc && K <= 5 && K != 3;
-        // ... and only where the unswizzled gathers are at most 2-way (tensor
-        // cores) / 4-way (SIMT) conflicted: 4-way measured 3 % faster on SIMT
-        // k = 4, 2 % slower on the k = 6 tensor-core path, 8-way much slower
-        const double cf = (simt || d.tci) ? unswizzled_conflicts(K, gpt, pair, tl, ng[0]) : 99.0;
-        const bool low_ok = (simt && K != 5 && cf <= 4.0) || (d.tci && K <= 5 && cf <= 2.0);
+        const bool eligible = std::getenv("SVB200_NO_WS") == nullptr && p.nH <= 6 && (simt || d.tci);
         const char* ev = std::getenv("SVB200_WS_UNSWZ");
         const bool force = ev != nullptr && ev[0] == '1', never = ev != nullptr && ev[0] == '0';
-        // bulk copies of runs below ~2 KB measured slower than the 16 B-copy loop
-        const char* mr = std::getenv("SVB200_WS_MINRUN");
-        const uint32_t minrun = mr ? (uint32_t)std::atoi(mr) : 2048u;
-        // runs of <= 1 KB (and every k = 6 tensor-core tile) move as tensor
-        // copies (encode_tile_map): per-run bulk copies of 1 KB measured 10-40 %
-        // slower, tensor copies of >= 2 KB runs 1-5 % slower than bulk copies
-        const char* tm = std::getenv("SVB200_TMAP");
-        const bool tmap = tm ? tm[0] == '1' : (p.r <= 7 || (d.tci && K == 6) || (gpt == 2 && pair));
-        if ((simt || d.tci) && tmap)
-            encode_tile_map(p.tmap, p.trank, p.tstart, p.tbits, p.tnx, p.txpos, psi, n, p.r, p.Hpos, p.nH);
-        ws = std::getenv("SVB200_NO_WS") == nullptr && p.nH <= 6 && (simt || d.tci) &&
-             ((8u << p.r) >= minrun || p.trank > 0) &&
-             (natural || (!never && (low_ok || force)));
-        if (ws) p.swz[0] = p.swz[1] = p.swz[2] = 0;
+        const char* e128 = std::getenv("SVB200_SWZ128");
+        double cf = 1.0;
+        if (eligible && !natural) {
+            cf = gather_conflicts(K, gpt, pair, tl, ng[0], kNone);
+            const double c128 = gather_conflicts(K, gpt, pair, tl, ng[0], k128);
+            // SIMT: the fewer conflicts win; tensor cores: unswizzled whenever it is
+            // at most 2-way (its >= 2 KB runs can use per-run bulk copies, which
+            // measured faster there than tensor copies: k = 5 2.86 vs 2.96 ms)
+            const bool better = d.tci ? (cf > 2.0 && c128 <= 2.0) : c128 < cf;
+            if (better && !(e128 && e128[0] == '0')) {
+                swz128 = true;
+                cf = c128;
+            }
+        }
+        const bool low_ok = (simt && K != 5 && cf <= 4.0) || (d.tci && cf <= 2.0);
+        if (eligible && (natural || (!never && (low_ok || force)))) {
+            // runs of <= 2 KB (and every k = 6 tensor-core tile) move as tensor
+            // copies (encode_tile_map): per-run bulk copies of 1 KB runs measured
+            // 10-40 % slower, of 2 KB runs 8 % slower inside a circuit; tensor
+            // copies of >= 4 KB runs 1-3 % slower than per-run bulk copies
+            const char* mr = std::getenv("SVB200_WS_MINRUN");
+            const uint32_t minrun = mr ? (uint32_t)std::atoi(mr) : 2048u;
+            const char* tm = std::getenv("SVB200_TMAP");
+            const bool tmap = swz128 || (tm ? tm[0] == '1' : (p.r <= 8 || (d.tci && K == 6) || (gpt == 2 && pair)));
+            if (tmap)
+                encode_tile_map(p.tmap, p.trank, p.tstart, p.tbits, p.tnx, p.txpos, psi, n, p.r, p.Hpos, p.nH, swz128);
+            ws = swz128 ? p.trank > 0 : ((8u << p.r) >= minrun || p.trank > 0);
+        }
+        if (!ws) {
+            swz128 = false;
+            p.trank = 0;
+        } else {
+            for (int i = 0; i < 3; ++i) p.swz[i] = swz128 ? k128[i] : 0u;
+        }
     }
     auto sw = [&](uint32_t t) {
         return t ^ ((__builtin_popcount(t & p.swz[0]) & 1) << 1) ^ ((__builtin_popcount(t & p.swz[1]) & 1) << 2) ^
@@ -1815,7 +1843,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
     if (ws) {
         for (uint32_t j = 0; j < (1u << p.nH); ++j) p.roff[j] = 8ull * dep((uint64_t)j << p.r);
         const int nb = d.tci ? STG : SVB_WS_STAGES;
-        smem = (size_t)nb * ((size_t)8 << p.T) + 16u * nb;
+        smem = (size_t)nb * ((size_t)8 << p.T) + 16u * nb + 1024u;  // + alignment of the tiles to 1 KB
         if constexpr (K >= 4) {
             if (d.tci) smem += TciShape<K>::SMEM;
         }
