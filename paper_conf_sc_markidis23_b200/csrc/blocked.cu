@@ -217,6 +217,248 @@ int pass_sms() {
     return n;
 }
 
+
+// ------------------------------------------------ register-blocked passes
+// apply_rpass<M, F2>: the same tiles and tile loop, but a gate is not one sweep
+// of the shared-memory tile.  The pass's gates (k <= 2) are grouped into
+// PHASES (host, plan_phases): sets of gates whose tile positions fit in a set
+// R of M positions, gates moved forward only past gates on disjoint qubits
+// (they commute).  In a phase every thread gathers the 2^M amplitudes whose
+// tile index varies over R (its other tile bits are fixed by the thread
+// index), applies all the phase's gates to them in registers -- a gate on
+// register bits MASK is a compile-time-indexed 2^k x 2^k complex matvec over
+// the 2^M / 2^k groups, each matrix element loaded once per gate -- and
+// scatters them back: one barrier per phase instead of one per gate.
+// Addresses are XOR-linear: slot = tbase ^ roff[j], swizzled on the host with
+// a fold swizzle (16 B chunk bits 1..3 ^= the XOR of tile bits 4..6, 7..9,
+// ...) and the thread -> position order chosen so that each quarter-warp
+// (LDS.128) / half-warp (LDS.64) gather is conflict-free.
+constexpr int kRpMaxPhases = 48;
+constexpr int kRpMaxGates = 64;
+constexpr int kRpMatFloats = kRpMaxGates * 32;
+
+struct RpPhase {
+    uint32_t roff[32];  // byte offsets of register index j (swizzled)
+    uint32_t tbw[10];   // byte offset contributed by thread-index bit i (swizzled)
+    uint16_t g0, g1;    // gates [g0, g1) in launch order
+    uint32_t b0;        // tile bit 0 is register bit 0: 16 B gathers
+};
+
+struct alignas(16) RpassParams {
+    float mats[kRpMatFloats];
+    float2* psi;
+    uint64_t n_tiles;
+    int T, r, nH, nph, tbits;
+    int Hpos[32];
+    uint64_t goff[16];
+    uint32_t soff[16];
+    uint32_t gcode[kRpMaxGates];  // register mask (low 8 bits) | matrix float offset << 8
+    RpPhase ph[kRpMaxPhases];
+};
+
+__host__ __device__ constexpr int pdep5(int v, int mask) {
+    int r = 0, b = 0;
+    for (int i = 0; i < 5; ++i)
+        if ((mask >> i) & 1) {
+            if ((v >> b) & 1) r |= 1 << i;
+            ++b;
+        }
+    return r;
+}
+__host__ __device__ constexpr int popc5(int m) { return (m & 1) + ((m >> 1) & 1) + ((m >> 2) & 1) + ((m >> 3) & 1) + ((m >> 4) & 1); }
+
+// packed fp32 pair FMA (FFMA2): d = a * b + c per lane
+__device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
+    unsigned long long d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;"
+        : "=l"(d)
+        : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)),
+          "l"(*reinterpret_cast<unsigned long long*>(&c)));
+    return *reinterpret_cast<float2*>(&d);
+}
+
+// F2: complex MAC y += m x as two FFMA2: y += (mr, mr) (xr, xi); y += (-mi, mi) (xi, xr)
+// (ptxas encodes the swapped pair and the per-lane sign as operand modifiers
+// and takes (mr, mr) / (mi, mi) from uniform registers).  Otherwise four FFMA.
+template <int M, int MASK, bool F2>
+__device__ __forceinline__ void reg_gate(float2 (&a)[1 << M], const float* __restrict__ mf) {
+    constexpr int K = popc5(MASK);
+    constexpr int D = 1 << K;
+    constexpr int REST = ((1 << M) - 1) & ~MASK;
+    float2 m[D * D];
+#pragma unroll
+    for (int i = 0; i < D * D / 2; ++i) {
+        const float4 v = reinterpret_cast<const float4*>(mf)[i];
+        m[2 * i] = make_float2(v.x, v.y);
+        m[2 * i + 1] = make_float2(v.z, v.w);
+    }
+#pragma unroll
+    for (int g = 0; g < (1 << M) / D; ++g) {
+        const int base = pdep5(g, REST);
+        float2 x[D];
+#pragma unroll
+        for (int c = 0; c < D; ++c) x[c] = a[base | pdep5(c, MASK)];
+#pragma unroll
+        for (int rr = 0; rr < D; ++rr) {
+            float2 y;
+            if constexpr (F2) {
+                y = make_float2(0.f, 0.f);
+#pragma unroll
+                for (int c = 0; c < D; ++c) {
+                    const float2 mc = m[rr * D + c];
+                    y = ffma2(make_float2(mc.x, mc.x), x[c], y);
+                    y = ffma2(make_float2(-mc.y, mc.y), make_float2(x[c].y, x[c].x), y);
+                }
+            } else {
+                float yr = m[rr * D].x * x[0].x, yi = m[rr * D].x * x[0].y;
+                yr = fmaf(-m[rr * D].y, x[0].y, yr);
+                yi = fmaf(m[rr * D].y, x[0].x, yi);
+#pragma unroll
+                for (int c = 1; c < D; ++c) {
+                    yr = fmaf(m[rr * D + c].x, x[c].x, yr);
+                    yr = fmaf(-m[rr * D + c].y, x[c].y, yr);
+                    yi = fmaf(m[rr * D + c].x, x[c].y, yi);
+                    yi = fmaf(m[rr * D + c].y, x[c].x, yi);
+                }
+                y = make_float2(yr, yi);
+            }
+            a[base | pdep5(rr, MASK)] = y;
+        }
+    }
+}
+
+template <int M, bool F2>
+__device__ __forceinline__ void reg_gate_dispatch(int mask, float2 (&a)[1 << M], const float* mf) {
+    if constexpr (M == 4) {
+        switch (mask) {
+            case 1: reg_gate<4, 1, F2>(a, mf); break;
+            case 2: reg_gate<4, 2, F2>(a, mf); break;
+            case 4: reg_gate<4, 4, F2>(a, mf); break;
+            case 8: reg_gate<4, 8, F2>(a, mf); break;
+            case 3: reg_gate<4, 3, F2>(a, mf); break;
+            case 5: reg_gate<4, 5, F2>(a, mf); break;
+            case 6: reg_gate<4, 6, F2>(a, mf); break;
+            case 9: reg_gate<4, 9, F2>(a, mf); break;
+            case 10: reg_gate<4, 10, F2>(a, mf); break;
+            default: reg_gate<4, 12, F2>(a, mf); break;
+        }
+    } else {
+        switch (mask) {
+            case 1: reg_gate<5, 1, F2>(a, mf); break;
+            case 2: reg_gate<5, 2, F2>(a, mf); break;
+            case 4: reg_gate<5, 4, F2>(a, mf); break;
+            case 8: reg_gate<5, 8, F2>(a, mf); break;
+            case 16: reg_gate<5, 16, F2>(a, mf); break;
+            case 3: reg_gate<5, 3, F2>(a, mf); break;
+            case 5: reg_gate<5, 5, F2>(a, mf); break;
+            case 6: reg_gate<5, 6, F2>(a, mf); break;
+            case 9: reg_gate<5, 9, F2>(a, mf); break;
+            case 10: reg_gate<5, 10, F2>(a, mf); break;
+            case 12: reg_gate<5, 12, F2>(a, mf); break;
+            case 17: reg_gate<5, 17, F2>(a, mf); break;
+            case 18: reg_gate<5, 18, F2>(a, mf); break;
+            case 20: reg_gate<5, 20, F2>(a, mf); break;
+            default: reg_gate<5, 24, F2>(a, mf); break;
+        }
+    }
+}
+
+template <int M, bool F2>
+__global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 128) apply_rpass(const __grid_constant__ RpassParams p) {
+    constexpr int NA = 1 << M;   // amplitudes per thread
+    constexpr int UPT = NA / 2;  // 16 B load/store units per thread
+    extern __shared__ float4 rsm[];
+    const uint32_t tile_bytes = 8u << p.T;
+    const uint32_t s0 = smem_addr(rsm);
+    const uint32_t t0 = 2u * threadIdx.x;
+    const uint32_t rmask = (1u << p.r) - 1u;
+    uint64_t dthr = t0 & rmask;
+    {
+        const uint32_t h = t0 >> p.r;
+        for (int b = 0; b < p.nH; ++b)
+            if ((h >> b) & 1u) dthr += 1ull << p.Hpos[b];
+    }
+    // unit i of this thread: tile index t0 + 2*nthr*i; its smem byte offset
+    // is fold(t0) ^ soff[i] (the fold swizzle is XOR-linear)
+    uint32_t sthr = 0;
+    {
+        uint32_t f = 0;
+        for (int q = 4; q < p.T; ++q)
+            if ((t0 >> q) & 1u) f ^= 1u << (1 + (q - 4) % 3);
+        sthr = (t0 ^ f) << 3;
+    }
+    auto tbase = [&](uint64_t u) {
+        uint64_t x = u << p.r;
+        for (int b = 0; b < p.nH; ++b) {
+            const int q = p.Hpos[b];
+            x = ((x >> q) << (q + 1)) | (x & ((1ull << q) - 1ull));
+        }
+        return x;
+    };
+    auto load = [&](const float2* g, uint32_t sbuf) {
+#pragma unroll
+        for (int i = 0; i < UPT; ++i) cp_async16(sbuf + (sthr ^ p.soff[i]), g + p.goff[i]);
+    };
+    auto store = [&](float2* g, uint32_t sbuf) {
+#pragma unroll
+        for (int i = 0; i < UPT; ++i) st_stream(reinterpret_cast<float4*>(g + p.goff[i]), lds4(sbuf + (sthr ^ p.soff[i])));
+    };
+    uint64_t u = blockIdx.x;
+    const float2* gcur = nullptr;
+    if (u < p.n_tiles) {
+        gcur = p.psi + tbase(u) + dthr;
+        load(gcur, s0);
+    }
+    cp_async_commit();
+    for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
+        const uint32_t cur = s0 + (uint32_t)(it & 1) * tile_bytes;
+        const uint32_t nxt = s0 + (uint32_t)((it + 1) & 1) * tile_bytes;
+        const uint64_t un = u + gridDim.x;
+        const float2* gnext = nullptr;
+        __syncthreads();  // buffer `nxt` drained by the previous store
+        if (un < p.n_tiles) {
+            gnext = p.psi + tbase(un) + dthr;
+            load(gnext, nxt);
+        }
+        cp_async_commit();
+        cp_async_wait1();
+        __syncthreads();
+        for (int ph = 0; ph < p.nph; ++ph) {
+            const RpPhase& P = p.ph[ph];
+            uint32_t tb = 0;
+            for (int i = 0; i < p.tbits; ++i)
+                if ((threadIdx.x >> i) & 1u) tb ^= P.tbw[i];
+            float2 a[NA];
+            if (P.b0) {
+#pragma unroll
+                for (int j = 0; j < NA / 2; ++j) {
+                    const float4 v = lds4(cur + (tb ^ P.roff[2 * j]));
+                    a[2 * j] = make_float2(v.x, v.y);
+                    a[2 * j + 1] = make_float2(v.z, v.w);
+                }
+            } else {
+#pragma unroll
+                for (int j = 0; j < NA; ++j) a[j] = lds2(cur + (tb ^ P.roff[j]));
+            }
+            for (int gi = P.g0; gi < P.g1; ++gi) {
+                const uint32_t code = p.gcode[gi];
+                reg_gate_dispatch<M, F2>((int)(code & 0xffu), a, p.mats + (code >> 8));
+            }
+            if (P.b0) {
+#pragma unroll
+                for (int j = 0; j < NA / 2; ++j)
+                    sts4(cur + (tb ^ P.roff[2 * j]), make_float4(a[2 * j].x, a[2 * j].y, a[2 * j + 1].x, a[2 * j + 1].y));
+            } else {
+#pragma unroll
+                for (int j = 0; j < NA; ++j) sts2(cur + (tb ^ P.roff[j]), a[j]);
+            }
+            __syncthreads();
+        }
+        store(const_cast<float2*>(gcur), cur);
+        gcur = gnext;
+    }
+}
+
 }  // namespace
 
 void plan_pass_tile(PassDesc& pd) {
@@ -274,6 +516,240 @@ cudaError_t launch_pass(float2* psi, int n, const PassDesc& pd, cudaStream_t st)
     }
     delete pp;
     return e;
+}
+
+}  // namespace svb
+
+// ---------------------------------------------- register-blocked pass (host)
+namespace svb {
+namespace {
+
+uint32_t fold_swz(uint32_t t, int T) {
+    uint32_t f = 0;
+    for (int q = 4; q < T; ++q)
+        if ((t >> q) & 1u) f ^= 1u << (1 + (q - 4) % 3);
+    return t ^ f;
+}
+// 16 B chunk bank bit (0..2) that tile position q moves under the fold swizzle
+int bank_class(int q) { return q == 0 ? -1 : (q <= 3 ? q - 1 : (q - 4) % 3); }
+
+struct RpPhaseHost {
+    std::vector<int> gates;  // pass gate indices, in application order
+    std::vector<int> R;      // M tile positions, ascending (register bit j <-> R[j])
+    std::vector<int> lanes;  // T-M positions: thread-index bit i <-> lanes[i]
+    bool b0;
+};
+
+uint32_t deposit(uint32_t v, const std::vector<int>& pos) {
+    uint32_t x = 0;
+    for (size_t b = 0; b < pos.size(); ++b)
+        if ((v >> b) & 1u) x |= 1u << pos[b];
+    return x;
+}
+
+int rpass_m() {
+    static int m = 0;
+    if (!m) {
+        const char* e = getenv("SVB200_RPASS_M");
+        m = (e && e[0] == '5') ? 5 : 4;
+    }
+    return m;
+}
+
+// Phases of gates [g0, g1): each phase takes, in order, every remaining gate
+// whose positions fit in the phase's M-set and that does not touch a position
+// of a gate skipped before it (so it only moves past gates it commutes with).
+std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, int M) {
+    const int T = (int)pd.S.size();
+    std::vector<RpPhaseHost> out;
+    std::vector<int> rem;
+    for (size_t g = g0; g < g1; ++g) rem.push_back((int)g);
+    auto gmask = [&](int g) {
+        uint32_t m = 0;
+        for (int b = 0; b < pd.gates[g].k; ++b) m |= 1u << pd.gates[g].pos[b];
+        return m;
+    };
+    while (!rem.empty()) {
+        RpPhaseHost ph;
+        uint32_t used = 0, blocked = 0;
+        std::vector<int> keep;
+        for (int g : rem) {
+            const uint32_t m = gmask(g);
+            if (!(m & blocked) && __builtin_popcount(used | m) <= M) {
+                used |= m;
+                ph.gates.push_back(g);
+            } else {
+                blocked |= m;
+                keep.push_back(g);
+            }
+        }
+        rem.swap(keep);
+        if (__builtin_popcount(used) < M) used |= 1u;  // tile bit 0 in registers: 16 B gathers
+        for (int q = T - 1; q >= 0 && __builtin_popcount(used) < M; --q) used |= 1u << q;
+        for (int q = 0; q < T; ++q)
+            if ((used >> q) & 1u) ph.R.push_back(q);
+        ph.b0 = (used & 1u) != 0;
+        // lanes: the first lanes of a quarter- (16 B) / half-warp (8 B) must
+        // move distinct bank bits
+        std::vector<int> rest;
+        for (int q = 0; q < T; ++q)
+            if (!((used >> q) & 1u)) rest.push_back(q);
+        std::vector<int> lanes;
+        if (!ph.b0) {
+            lanes.push_back(0);
+            rest.erase(rest.begin());
+        }
+        int have = 0;
+        for (size_t i = 0; i < rest.size() && have != 7;) {
+            const int c = bank_class(rest[i]);
+            if (c >= 0 && !((have >> c) & 1)) {
+                have |= 1 << c;
+                lanes.push_back(rest[i]);
+                rest.erase(rest.begin() + (long)i);
+            } else {
+                ++i;
+            }
+        }
+        lanes.insert(lanes.end(), rest.begin(), rest.end());
+        ph.lanes = lanes;
+        out.push_back(ph);
+    }
+    return out;
+}
+
+// worst bank-conflict degree of a phase's gathers (warp 0, every register j)
+int phase_conflicts(const RpPhaseHost& ph, int T, int M) {
+    int worst = 1;
+    for (uint32_t j = 0; j < (1u << M); j += ph.b0 ? 2 : 1) {
+        const int group = ph.b0 ? 8 : 16;
+        for (int l0 = 0; l0 < 32; l0 += group) {
+            int cnt[16] = {0};
+            for (int l = l0; l < l0 + group; ++l) {
+                const uint32_t slot = fold_swz(deposit(j, ph.R) | deposit((uint32_t)l, ph.lanes), T);
+                const int bank = ph.b0 ? (int)((slot >> 1) & 7) : (int)(slot & 15);
+                worst = std::max(worst, ++cnt[bank]);
+            }
+        }
+    }
+    return worst;
+}
+
+template <int M, bool F2>
+cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st) {
+    const int T = (int)pd.S.size();
+    const uint32_t nthr = 1u << (T - M);
+    const size_t smem = 2 * ((size_t)8 << T);
+    cudaError_t e = cudaFuncSetAttribute(apply_rpass<M, F2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    static int per_sm_cache[16] = {0};
+    if (!per_sm_cache[T]) {
+        int nb = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, apply_rpass<M, F2>, (int)nthr, smem);
+        if (e != cudaSuccess) return e;
+        per_sm_cache[T] = std::max(1, nb);
+    }
+    RpassParams* pp = new RpassParams;
+    RpassParams& p = *pp;
+    std::memset(&p, 0, sizeof(p));
+    p.psi = psi;
+    p.T = T;
+    p.r = pd.r;
+    p.nH = 0;
+    for (int i = pd.r; i < T; ++i) p.Hpos[p.nH++] = pd.S[i];
+    p.tbits = T - M;
+    auto dep = [&](uint64_t t) {
+        uint64_t g = t & ((1ull << p.r) - 1);
+        const uint64_t h = t >> p.r;
+        for (int b = 0; b < p.nH; ++b)
+            if ((h >> b) & 1) g += 1ull << p.Hpos[b];
+        return g;
+    };
+    for (int i = 0; i < (1 << (M - 1)); ++i) {
+        p.goff[i] = dep(2ull * nthr * i);
+        p.soff[i] = fold_swz(2u * nthr * i, T) << 3;
+    }
+    p.n_tiles = 1ull << (n - T);
+    const uint64_t grid = std::min<uint64_t>(p.n_tiles, (uint64_t)pass_sms() * per_sm_cache[T]);
+    // gates in chunks that fit the parameter block (one launch each)
+    const size_t ng = pd.gates.size();
+    size_t g0 = 0;
+    while (g0 < ng && e == cudaSuccess) {
+        size_t g1 = std::min(ng, g0 + (size_t)kRpMaxGates);
+        auto phs = plan_phases(pd, g0, g1, M);
+        if ((int)phs.size() > kRpMaxPhases) {
+            // keep the first kRpMaxPhases phases; their gates are a prefix
+            // only if no gate was moved past a later phase: re-plan a prefix
+            size_t cut = g1;
+            do {
+                cut = g0 + (cut - g0) / 2;
+                phs = plan_phases(pd, g0, cut, M);
+            } while ((int)phs.size() > kRpMaxPhases);
+            g1 = cut;
+        }
+        p.nph = (int)phs.size();
+        uint32_t moff = 0;
+        int li = 0;
+        for (int i = 0; i < p.nph; ++i) {
+            const RpPhaseHost& h = phs[i];
+            RpPhase& P = p.ph[i];
+            P.g0 = (uint16_t)li;
+            P.b0 = h.b0 ? 1u : 0u;
+            for (uint32_t j = 0; j < (1u << M); ++j) P.roff[j] = fold_swz(deposit(j, h.R), T) << 3;
+            for (int b = 0; b < p.tbits; ++b) P.tbw[b] = fold_swz(1u << h.lanes[b], T) << 3;
+            for (int g : h.gates) {
+                const PassGate& pg = pd.gates[g];
+                const int D = 1 << pg.k;
+                std::memcpy(p.mats + moff, pd.mats.data() + pg.moff, sizeof(float) * 2 * D * D);
+                uint32_t mask = 0;
+                for (int b = 0; b < pg.k; ++b)
+                    mask |= 1u << (int)(std::find(h.R.begin(), h.R.end(), pg.pos[b]) - h.R.begin());
+                p.gcode[li++] = mask | (moff << 8);
+                moff += 2 * D * D;
+            }
+            P.g1 = (uint16_t)li;
+        }
+        apply_rpass<M, F2><<<(unsigned)grid, nthr, smem, st>>>(p);
+        e = cudaGetLastError();
+        g0 = g1;
+    }
+    delete pp;
+    return e;
+}
+
+}  // namespace
+
+bool rpass_supported(const PassDesc& pd) {
+    static int env = -1;
+    if (env < 0) {
+        const char* e = getenv("SVB200_RPASS");
+        env = (e && e[0] == '0') ? 0 : 1;
+    }
+    if (!env) return false;
+    const int T = (int)pd.S.size();
+    if (T < 10 || T > 13 || pd.r < 4) return false;
+    for (auto& g : pd.gates)
+        if (g.k > 2) return false;
+    return true;
+}
+
+void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {
+    const int M = rpass_m();
+    auto ph = plan_phases(pd, 0, pd.gates.size(), M);
+    int w = 1;
+    for (auto& x : ph) w = std::max(w, phase_conflicts(x, (int)pd.S.size(), M));
+    if (n_phases) *n_phases = (int)ph.size();
+    if (worst_conflict) *worst_conflict = w;
+}
+
+cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st) {
+    static_assert(sizeof(RpassParams) <= 32764, "rpass params exceed the kernel parameter space");
+    static int f2 = -1;
+    if (f2 < 0) {
+        const char* e = getenv("SVB200_RPASS_F2");
+        f2 = (e && e[0] == '0') ? 0 : 1;
+    }
+    if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st) : launch_rpass_m<5, false>(psi, n, pd, st);
+    return f2 ? launch_rpass_m<4, true>(psi, n, pd, st) : launch_rpass_m<4, false>(psi, n, pd, st);
 }
 
 }  // namespace svb

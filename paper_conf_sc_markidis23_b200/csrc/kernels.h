@@ -77,15 +77,25 @@ struct PassGate {
     int k;          // 1..4
     int pos[4];     // tile-local positions (rank of the qubit in sorted S), ascending
     uint32_t poff;  // offset (floats) of the gate's planes P, S, Q (3 x 4^k floats)
+    uint32_t moff;  // offset (floats) of the gate's matrix in PassDesc::mats
 };
 struct PassDesc {
     std::vector<int> S;  // qubits of the tile
     int r = 0;           // run bits (S[0..r) == 0..r-1)
     std::vector<PassGate> gates;
     std::vector<float> planes;
+    std::vector<float> mats;  // per gate: 2^k x 2^k complex64, row-major (re, im pairs)
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
+// Register-blocked pass (k <= 2 gates, 10 <= T <= 13): each thread holds 32
+// amplitudes of the tile in registers and applies every gate of a phase
+// there; phases exchange through the shared-memory tile.
+bool rpass_supported(const PassDesc& pd);
+cudaError_t launch_rpass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
+// Host model of the rpass phase plan (tests / tools): number of phases and
+// the worst bank-conflict degree of their gathers.
+void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict);
 
 // Launch one fused-gate apply on a shard of 2^n_local amplitudes.
 cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);

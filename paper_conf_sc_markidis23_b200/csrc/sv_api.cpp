@@ -880,6 +880,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
                 passes.push_back(cur);
                 cur.gates.clear();
                 cur.planes.clear();
+                cur.mats.clear();
             }
             PassGate pg{};
             pg.k = f.k;
@@ -892,6 +893,11 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
                 Pp[i] = re;
                 Sp[i] = re + im;
                 Qp[i] = im - re;
+            }
+            pg.moff = (uint32_t)cur.mats.size();
+            for (int i = 0; i < D * D; ++i) {
+                cur.mats.push_back((float)f.M[i].real());
+                cur.mats.push_back((float)f.M[i].imag());
             }
             cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
             cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
@@ -1079,7 +1085,10 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     }
     for (auto& st : c->steps) {
         if (st.block) {
-            rc = launch(s, LaunchClass::HIGH, [&] { return launch_pass(s->shard[0], s->l, st.pass, s->stream); });
+            rc = launch(s, LaunchClass::HIGH, [&] {
+                return rpass_supported(st.pass) ? launch_rpass(s->shard[0], s->l, st.pass, s->stream)
+                                                : launch_pass(s->shard[0], s->l, st.pass, s->stream);
+            });
             if (rc) return rc;
             s->stats.bytes_apply += 16ull << s->l;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
