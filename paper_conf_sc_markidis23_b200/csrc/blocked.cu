@@ -14,6 +14,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "device_util.cuh"
@@ -235,7 +237,7 @@ int pass_sms() {
 // (LDS.128) / half-warp (LDS.64) gather is conflict-free.
 constexpr int kRpMaxPhases = 48;
 constexpr int kRpMaxGates = 64;
-constexpr int kRpMatFloats = kRpMaxGates * 32;
+constexpr int kRpMatFloats = kRpMaxGates * 64;  // 4 floats per element, k <= 2
 
 struct RpPhase {
     uint32_t roff[32];  // byte offsets of register index j (swizzled)
@@ -252,7 +254,7 @@ struct alignas(16) RpassParams {
     int Hpos[32];
     uint64_t goff[16];
     uint32_t soff[16];
-    uint32_t gcode[kRpMaxGates];  // register mask (low 8 bits) | matrix float offset << 8
+    uint32_t gcode[kRpMaxGates];  // register mask (bits 0..4) | kind << 5 | matrix float offset << 8
     RpPhase ph[kRpMaxPhases];
 };
 
@@ -277,94 +279,369 @@ __device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
     return *reinterpret_cast<float2*>(&d);
 }
 
-// F2: complex MAC y += m x as two FFMA2: y += (mr, mr) (xr, xi); y += (-mi, mi) (xi, xr)
-// (ptxas encodes the swapped pair and the per-lane sign as operand modifiers
-// and takes (mr, mr) / (mi, mi) from uniform registers).  Otherwise four FFMA.
+// Matrix element e of a gate is stored as 4 floats (mr, mr, -mi, mi).
+// F2: complex MAC y += m x as two packed FFMA2, y += (mr, mr) (xr, xi) and
+// y += (-mi, mi) (xi, xr) (ptxas encodes the swapped pair as an operand
+// modifier; both matrix pairs come straight from uniform registers,
+// LDCU.64).  Otherwise four FFMA.
+#ifndef SVB_RP_G
+#define SVB_RP_G 2  // groups transformed together (independent FFMA2 chains)
+#endif
 template <int M, int MASK, bool F2>
 __device__ __forceinline__ void reg_gate(float2 (&a)[1 << M], const float* __restrict__ mf) {
     constexpr int K = popc5(MASK);
     constexpr int D = 1 << K;
     constexpr int REST = ((1 << M) - 1) & ~MASK;
-    float2 m[D * D];
+    constexpr int NG = (1 << M) / D;
+    constexpr int G = SVB_RP_G < NG ? SVB_RP_G : NG;
+    float4 m[D * D];
 #pragma unroll
-    for (int i = 0; i < D * D / 2; ++i) {
-        const float4 v = reinterpret_cast<const float4*>(mf)[i];
-        m[2 * i] = make_float2(v.x, v.y);
-        m[2 * i + 1] = make_float2(v.z, v.w);
-    }
+    for (int i = 0; i < D * D; ++i) m[i] = reinterpret_cast<const float4*>(mf)[i];
 #pragma unroll
-    for (int g = 0; g < (1 << M) / D; ++g) {
-        const int base = pdep5(g, REST);
-        float2 x[D];
+    for (int g0 = 0; g0 < NG; g0 += G) {
+        float2 x[G][D];
 #pragma unroll
-        for (int c = 0; c < D; ++c) x[c] = a[base | pdep5(c, MASK)];
+        for (int h = 0; h < G; ++h)
+#pragma unroll
+            for (int c = 0; c < D; ++c) x[h][c] = a[pdep5(g0 + h, REST) | pdep5(c, MASK)];
 #pragma unroll
         for (int rr = 0; rr < D; ++rr) {
-            float2 y;
-            if constexpr (F2) {
-                y = make_float2(0.f, 0.f);
+            float2 y[G];
 #pragma unroll
-                for (int c = 0; c < D; ++c) {
-                    const float2 mc = m[rr * D + c];
-                    y = ffma2(make_float2(mc.x, mc.x), x[c], y);
-                    y = ffma2(make_float2(-mc.y, mc.y), make_float2(x[c].y, x[c].x), y);
+            for (int h = 0; h < G; ++h) {
+                if constexpr (F2) {
+                    y[h] = make_float2(0.f, 0.f);
+                } else {
+                    y[h] = make_float2(m[rr * D].x * x[h][0].x, m[rr * D].x * x[h][0].y);
+                    y[h].x = fmaf(m[rr * D].z, x[h][0].y, y[h].x);
+                    y[h].y = fmaf(m[rr * D].w, x[h][0].x, y[h].y);
+                }
+            }
+#pragma unroll
+            for (int c = F2 ? 0 : 1; c < D; ++c) {
+                const float4 mc = m[rr * D + c];
+#pragma unroll
+                for (int h = 0; h < G; ++h) {
+                    if constexpr (F2) {
+                        y[h] = ffma2(make_float2(mc.x, mc.y), x[h][c], y[h]);
+                        y[h] = ffma2(make_float2(mc.z, mc.w), make_float2(x[h][c].y, x[h][c].x), y[h]);
+                    } else {
+                        y[h].x = fmaf(mc.x, x[h][c].x, y[h].x);
+                        y[h].x = fmaf(mc.z, x[h][c].y, y[h].x);
+                        y[h].y = fmaf(mc.x, x[h][c].y, y[h].y);
+                        y[h].y = fmaf(mc.w, x[h][c].x, y[h].y);
+                    }
+                }
+            }
+#pragma unroll
+            for (int h = 0; h < G; ++h) a[pdep5(g0 + h, REST) | pdep5(rr, MASK)] = y[h];
+        }
+    }
+}
+
+__host__ __device__ constexpr int pext5(int v, int mask) {
+    int r = 0, b = 0;
+    for (int i = 0; i < 5; ++i)
+        if ((mask >> i) & 1) {
+            if ((v >> i) & 1) r |= 1 << b;
+            ++b;
+        }
+    return r;
+}
+
+// Diagonal gate on register bits MASK: a[j] *= d[e(j)], entries stored like
+// matrix elements (dr, dr, -di, di); one complex product = two FFMA2.
+template <int M, int MASK>
+__device__ __forceinline__ void reg_diag(float2 (&a)[1 << M], const float* __restrict__ mf) {
+    constexpr int D = 1 << popc5(MASK);
+#pragma unroll
+    for (int i = 0; i < D; ++i) {
+        const float4 e = reinterpret_cast<const float4*>(mf)[i];
+#pragma unroll
+        for (int j = 0; j < (1 << M); ++j) {
+            if (pext5(j, MASK) != i) continue;
+            const float2 x = a[j];
+            a[j] = ffma2(make_float2(e.z, e.w), make_float2(x.y, x.x), ffma2(make_float2(e.x, e.y), x, make_float2(0.f, 0.f)));
+        }
+    }
+}
+
+// CZ-like gate (diag(1, 1, 1, -1) on register bits MASK): sign flips only.
+template <int M, int MASK>
+__device__ __forceinline__ void reg_cz(float2 (&a)[1 << M]) {
+#pragma unroll
+    for (int j = 0; j < (1 << M); ++j)
+        if ((j & MASK) == MASK) a[j] = make_float2(-a[j].x, -a[j].y);
+}
+
+template <int M, bool F2>
+__device__ __forceinline__ void reg_gate_dispatch(int code, float2 (&a)[1 << M], const float* mf) {
+    // code = mask (bits 0..4) | kind << 5: 0 dense, 1 diagonal, 2 CZ-like.
+    // Balanced compare trees on the (warp-uniform) code: a switch becomes a
+    // BRX jump table on a vector register, and the matrices then load with
+    // LDC into vector registers instead of uniform registers
+    const int mask = code & 31, kind = code >> 5;
+    if constexpr (M == 4) {
+        if (kind == 0) {
+            if (mask < 6) {
+                if (mask < 3) {
+                    if (mask < 2) {
+                        reg_gate<4, 1, F2>(a, mf);
+                    } else {
+                        reg_gate<4, 2, F2>(a, mf);
+                    }
+                } else {
+                    if (mask < 4) {
+                        reg_gate<4, 3, F2>(a, mf);
+                    } else {
+                        if (mask < 5) {
+                            reg_gate<4, 4, F2>(a, mf);
+                        } else {
+                            reg_gate<4, 5, F2>(a, mf);
+                        }
+                    }
                 }
             } else {
-                float yr = m[rr * D].x * x[0].x, yi = m[rr * D].x * x[0].y;
-                yr = fmaf(-m[rr * D].y, x[0].y, yr);
-                yi = fmaf(m[rr * D].y, x[0].x, yi);
-#pragma unroll
-                for (int c = 1; c < D; ++c) {
-                    yr = fmaf(m[rr * D + c].x, x[c].x, yr);
-                    yr = fmaf(-m[rr * D + c].y, x[c].y, yr);
-                    yi = fmaf(m[rr * D + c].x, x[c].y, yi);
-                    yi = fmaf(m[rr * D + c].y, x[c].x, yi);
+                if (mask < 9) {
+                    if (mask < 8) {
+                        reg_gate<4, 6, F2>(a, mf);
+                    } else {
+                        reg_gate<4, 8, F2>(a, mf);
+                    }
+                } else {
+                    if (mask < 10) {
+                        reg_gate<4, 9, F2>(a, mf);
+                    } else {
+                        if (mask < 12) {
+                            reg_gate<4, 10, F2>(a, mf);
+                        } else {
+                            reg_gate<4, 12, F2>(a, mf);
+                        }
+                    }
                 }
-                y = make_float2(yr, yi);
             }
-            a[base | pdep5(rr, MASK)] = y;
-        }
-    }
-}
-
-template <int M, bool F2>
-__device__ __forceinline__ void reg_gate_dispatch(int mask, float2 (&a)[1 << M], const float* mf) {
-    if constexpr (M == 4) {
-        switch (mask) {
-            case 1: reg_gate<4, 1, F2>(a, mf); break;
-            case 2: reg_gate<4, 2, F2>(a, mf); break;
-            case 4: reg_gate<4, 4, F2>(a, mf); break;
-            case 8: reg_gate<4, 8, F2>(a, mf); break;
-            case 3: reg_gate<4, 3, F2>(a, mf); break;
-            case 5: reg_gate<4, 5, F2>(a, mf); break;
-            case 6: reg_gate<4, 6, F2>(a, mf); break;
-            case 9: reg_gate<4, 9, F2>(a, mf); break;
-            case 10: reg_gate<4, 10, F2>(a, mf); break;
-            default: reg_gate<4, 12, F2>(a, mf); break;
+        } else if (kind == 1) {
+            if (mask < 6) {
+                if (mask < 3) {
+                    if (mask < 2) {
+                        reg_diag<4, 1>(a, mf);
+                    } else {
+                        reg_diag<4, 2>(a, mf);
+                    }
+                } else {
+                    if (mask < 4) {
+                        reg_diag<4, 3>(a, mf);
+                    } else {
+                        if (mask < 5) {
+                            reg_diag<4, 4>(a, mf);
+                        } else {
+                            reg_diag<4, 5>(a, mf);
+                        }
+                    }
+                }
+            } else {
+                if (mask < 9) {
+                    if (mask < 8) {
+                        reg_diag<4, 6>(a, mf);
+                    } else {
+                        reg_diag<4, 8>(a, mf);
+                    }
+                } else {
+                    if (mask < 10) {
+                        reg_diag<4, 9>(a, mf);
+                    } else {
+                        if (mask < 12) {
+                            reg_diag<4, 10>(a, mf);
+                        } else {
+                            reg_diag<4, 12>(a, mf);
+                        }
+                    }
+                }
+            }
+        } else {
+            if (mask < 9) {
+                if (mask < 5) {
+                    reg_cz<4, 3>(a);
+                } else {
+                    if (mask < 6) {
+                        reg_cz<4, 5>(a);
+                    } else {
+                        reg_cz<4, 6>(a);
+                    }
+                }
+            } else {
+                if (mask < 10) {
+                    reg_cz<4, 9>(a);
+                } else {
+                    if (mask < 12) {
+                        reg_cz<4, 10>(a);
+                    } else {
+                        reg_cz<4, 12>(a);
+                    }
+                }
+            }
         }
     } else {
-        switch (mask) {
-            case 1: reg_gate<5, 1, F2>(a, mf); break;
-            case 2: reg_gate<5, 2, F2>(a, mf); break;
-            case 4: reg_gate<5, 4, F2>(a, mf); break;
-            case 8: reg_gate<5, 8, F2>(a, mf); break;
-            case 16: reg_gate<5, 16, F2>(a, mf); break;
-            case 3: reg_gate<5, 3, F2>(a, mf); break;
-            case 5: reg_gate<5, 5, F2>(a, mf); break;
-            case 6: reg_gate<5, 6, F2>(a, mf); break;
-            case 9: reg_gate<5, 9, F2>(a, mf); break;
-            case 10: reg_gate<5, 10, F2>(a, mf); break;
-            case 12: reg_gate<5, 12, F2>(a, mf); break;
-            case 17: reg_gate<5, 17, F2>(a, mf); break;
-            case 18: reg_gate<5, 18, F2>(a, mf); break;
-            case 20: reg_gate<5, 20, F2>(a, mf); break;
-            default: reg_gate<5, 24, F2>(a, mf); break;
+        if (kind == 0) {
+            if (mask < 9) {
+                if (mask < 4) {
+                    if (mask < 2) {
+                        reg_gate<5, 1, F2>(a, mf);
+                    } else {
+                        if (mask < 3) {
+                            reg_gate<5, 2, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 3, F2>(a, mf);
+                        }
+                    }
+                } else {
+                    if (mask < 6) {
+                        if (mask < 5) {
+                            reg_gate<5, 4, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 5, F2>(a, mf);
+                        }
+                    } else {
+                        if (mask < 8) {
+                            reg_gate<5, 6, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 8, F2>(a, mf);
+                        }
+                    }
+                }
+            } else {
+                if (mask < 17) {
+                    if (mask < 12) {
+                        if (mask < 10) {
+                            reg_gate<5, 9, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 10, F2>(a, mf);
+                        }
+                    } else {
+                        if (mask < 16) {
+                            reg_gate<5, 12, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 16, F2>(a, mf);
+                        }
+                    }
+                } else {
+                    if (mask < 20) {
+                        if (mask < 18) {
+                            reg_gate<5, 17, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 18, F2>(a, mf);
+                        }
+                    } else {
+                        if (mask < 24) {
+                            reg_gate<5, 20, F2>(a, mf);
+                        } else {
+                            reg_gate<5, 24, F2>(a, mf);
+                        }
+                    }
+                }
+            }
+        } else if (kind == 1) {
+            if (mask < 9) {
+                if (mask < 4) {
+                    if (mask < 2) {
+                        reg_diag<5, 1>(a, mf);
+                    } else {
+                        if (mask < 3) {
+                            reg_diag<5, 2>(a, mf);
+                        } else {
+                            reg_diag<5, 3>(a, mf);
+                        }
+                    }
+                } else {
+                    if (mask < 6) {
+                        if (mask < 5) {
+                            reg_diag<5, 4>(a, mf);
+                        } else {
+                            reg_diag<5, 5>(a, mf);
+                        }
+                    } else {
+                        if (mask < 8) {
+                            reg_diag<5, 6>(a, mf);
+                        } else {
+                            reg_diag<5, 8>(a, mf);
+                        }
+                    }
+                }
+            } else {
+                if (mask < 17) {
+                    if (mask < 12) {
+                        if (mask < 10) {
+                            reg_diag<5, 9>(a, mf);
+                        } else {
+                            reg_diag<5, 10>(a, mf);
+                        }
+                    } else {
+                        if (mask < 16) {
+                            reg_diag<5, 12>(a, mf);
+                        } else {
+                            reg_diag<5, 16>(a, mf);
+                        }
+                    }
+                } else {
+                    if (mask < 20) {
+                        if (mask < 18) {
+                            reg_diag<5, 17>(a, mf);
+                        } else {
+                            reg_diag<5, 18>(a, mf);
+                        }
+                    } else {
+                        if (mask < 24) {
+                            reg_diag<5, 20>(a, mf);
+                        } else {
+                            reg_diag<5, 24>(a, mf);
+                        }
+                    }
+                }
+            }
+        } else {
+            if (mask < 12) {
+                if (mask < 6) {
+                    if (mask < 5) {
+                        reg_cz<5, 3>(a);
+                    } else {
+                        reg_cz<5, 5>(a);
+                    }
+                } else {
+                    if (mask < 9) {
+                        reg_cz<5, 6>(a);
+                    } else {
+                        if (mask < 10) {
+                            reg_cz<5, 9>(a);
+                        } else {
+                            reg_cz<5, 10>(a);
+                        }
+                    }
+                }
+            } else {
+                if (mask < 18) {
+                    if (mask < 17) {
+                        reg_cz<5, 12>(a);
+                    } else {
+                        reg_cz<5, 17>(a);
+                    }
+                } else {
+                    if (mask < 20) {
+                        reg_cz<5, 18>(a);
+                    } else {
+                        if (mask < 24) {
+                            reg_cz<5, 20>(a);
+                        } else {
+                            reg_cz<5, 24>(a);
+                        }
+                    }
+                }
+            }
         }
     }
 }
 
 template <int M, bool F2>
-__global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 128) apply_rpass(const __grid_constant__ RpassParams p) {
+__global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 168) apply_rpass(const __grid_constant__ RpassParams p) {
     constexpr int NA = 1 << M;   // amplitudes per thread
     constexpr int UPT = NA / 2;  // 16 B load/store units per thread
     extern __shared__ float4 rsm[];
@@ -442,7 +719,7 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             }
             for (int gi = P.g0; gi < P.g1; ++gi) {
                 const uint32_t code = p.gcode[gi];
-                reg_gate_dispatch<M, F2>((int)(code & 0xffu), a, p.mats + (code >> 8));
+                reg_gate_dispatch<M, F2>((int)(code & 0x7fu), a, p.mats + (code >> 8));
             }
             if (P.b0) {
 #pragma unroll
@@ -551,7 +828,7 @@ int rpass_m() {
     static int m = 0;
     if (!m) {
         const char* e = getenv("SVB200_RPASS_M");
-        m = (e && e[0] == '5') ? 5 : 4;
+        m = (e && e[0] == '4') ? 4 : 5;
     }
     return m;
 }
@@ -699,14 +976,39 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             for (int g : h.gates) {
                 const PassGate& pg = pd.gates[g];
                 const int D = 1 << pg.k;
-                std::memcpy(p.mats + moff, pd.mats.data() + pg.moff, sizeof(float) * 2 * D * D);
+                const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
+                bool diag = true, cz = pg.k == 2;
+                for (int r = 0; r < D; ++r)
+                    for (int c = 0; c < D; ++c) {
+                        const float re = mg[2 * (r * D + c)], im = mg[2 * (r * D + c) + 1];
+                        if (r != c && (re != 0.f || im != 0.f)) diag = cz = false;
+                        if (r == c && (im != 0.f || re != (r == D - 1 ? -1.f : 1.f))) cz = false;
+                    }
+                const int kind = cz ? 2 : diag ? 1 : 0;
+                const int ne = kind == 1 ? D : kind == 2 ? 0 : D * D;
+                for (int e2 = 0; e2 < ne; ++e2) {
+                    const int src = kind == 1 ? e2 * D + e2 : e2;
+                    const float mr = mg[2 * src], mi = mg[2 * src + 1];
+                    p.mats[moff + 4 * e2 + 0] = mr;
+                    p.mats[moff + 4 * e2 + 1] = mr;
+                    p.mats[moff + 4 * e2 + 2] = -mi;
+                    p.mats[moff + 4 * e2 + 3] = mi;
+                }
                 uint32_t mask = 0;
                 for (int b = 0; b < pg.k; ++b)
                     mask |= 1u << (int)(std::find(h.R.begin(), h.R.end(), pg.pos[b]) - h.R.begin());
-                p.gcode[li++] = mask | (moff << 8);
-                moff += 2 * D * D;
+                p.gcode[li++] = mask | ((uint32_t)kind << 5) | (moff << 8);
+                moff += 4 * ne;
             }
             P.g1 = (uint16_t)li;
+        }
+        static const bool dbg = getenv("SVB200_RPASS_DEBUG") != nullptr;
+        if (dbg) {
+            int w = 1;
+            for (auto& x : phs) w = std::max(w, phase_conflicts(x, T, M));
+            fprintf(stderr, "rpass T=%d M=%d gates=%zu phases=%d worst_conflict=%d S=", T, M, g1 - g0, p.nph, w);
+            for (int q : pd.S) fprintf(stderr, "%d,", q);
+            fprintf(stderr, "\n");
         }
         apply_rpass<M, F2><<<(unsigned)grid, nthr, smem, st>>>(p);
         e = cudaGetLastError();

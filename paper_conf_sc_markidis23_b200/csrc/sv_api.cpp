@@ -839,74 +839,86 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
     }
     c->pos_out = pos;
-    // Cache-blocked passes (unsharded, large states, k <= 4): the S4 planner
-    // with "local" = the tile's T slots cuts the fused list into passes; a
-    // remap only changes the tile's qubit set S (no data movement).
+    // Cache-blocked passes (unsharded, large states, k <= 4).  Passes are
+    // formed like fused gates (the S3 greedy, one level up): a pass starts at
+    // the first unplaced fused gate and absorbs every later one whose qubits
+    // keep the pass within T - kPassPinned free tile qubits, provided it does
+    // not touch a qubit of a gate skipped before it (so it only moves past
+    // gates it commutes with).  Qubits 0..kPassPinned-1 are in every tile
+    // (runs of >= 128 B); the pass's tile set S is the pinned qubits, the
+    // pass's qubits, then the lowest remaining qubits (longer runs).  The
+    // state never moves: a pass only chooses which amplitudes share a tile.
     const int T = s->block_bits;
     bool blocked = !s->fp64 && s->g == 0 && T >= 10 && s->n >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
                    max_fused >= 1;
     std::vector<PassDesc> passes;
     if (blocked) {
-        std::vector<std::vector<int>> fq;
-        for (auto& f : plan) fq.emplace_back(f.q, f.q + f.k);
-        std::vector<Event> bev;
-        std::vector<int> bpos;
-        plan_sharded(fq, s->n, s->n - T, 5, bev, bpos);
-        std::vector<int> ppos(s->n), inv(s->n);
-        for (int q = 0; q < s->n; ++q) ppos[q] = inv[q] = q;
-        auto new_pass = [&]() {
-            PassDesc pd;
-            for (int p = 0; p < T; ++p) pd.S.push_back(inv[p]);
-            plan_pass_tile(pd);
-            return pd;
-        };
-        PassDesc cur = new_pass();
-        for (auto& e : bev) {
-            if (e.type == Event::EXCHANGE) {
-                for (auto& pr : e.pairs) {
-                    const int a = inv[pr.first], b = inv[pr.second];
-                    ppos[a] = pr.second;
-                    ppos[b] = pr.first;
-                    inv[pr.first] = b;
-                    inv[pr.second] = a;
-                }
-                if (!cur.gates.empty()) passes.push_back(std::move(cur));
-                cur = new_pass();
-                continue;
-            }
-            const FusedGate& f = plan[e.fused];
+        constexpr int kPassPinned = 4;
+        const uint64_t pin = (1ull << kPassPinned) - 1ull;
+        const int Fp = T - kPassPinned;
+        const size_t nf = plan.size();
+        std::vector<uint64_t> fm(nf, 0);
+        for (size_t i = 0; i < nf; ++i)
+            for (int b = 0; b < plan[i].k; ++b) fm[i] |= 1ull << plan[i].q[b];
+        std::vector<char> placed(nf, 0);
+        auto add_gate = [&](PassDesc& cur, size_t i) {
+            const FusedGate& f = plan[i];
             const int D = 1 << f.k;
-            if ((int)cur.gates.size() == kPassMaxGates || cur.planes.size() + 3 * D * D > (size_t)kPassPlaneFloats) {
-                passes.push_back(cur);
-                cur.gates.clear();
-                cur.planes.clear();
-                cur.mats.clear();
-            }
             PassGate pg{};
             pg.k = f.k;
             for (int b = 0; b < f.k; ++b)
                 pg.pos[b] = (int)(std::find(cur.S.begin(), cur.S.end(), f.q[b]) - cur.S.begin());
             pg.poff = (uint32_t)cur.planes.size();
-            std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
-            for (int i = 0; i < D * D; ++i) {
-                const float re = (float)f.M[i].real(), im = (float)f.M[i].imag();
-                Pp[i] = re;
-                Sp[i] = re + im;
-                Qp[i] = im - re;
-            }
             pg.moff = (uint32_t)cur.mats.size();
-            for (int i = 0; i < D * D; ++i) {
-                cur.mats.push_back((float)f.M[i].real());
-                cur.mats.push_back((float)f.M[i].imag());
+            for (int e = 0; e < D * D; ++e) {
+                cur.mats.push_back((float)f.M[e].real());
+                cur.mats.push_back((float)f.M[e].imag());
+            }
+            std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
+            for (int e = 0; e < D * D; ++e) {
+                const float re = (float)f.M[e].real(), im = (float)f.M[e].imag();
+                Pp[e] = re;
+                Sp[e] = re + im;
+                Qp[e] = im - re;
             }
             cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
             cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
             cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
             cur.gates.push_back(pg);
+        };
+        for (size_t i = 0; i < nf; ++i) {
+            if (placed[i]) continue;
+            std::vector<size_t> mem{i};
+            placed[i] = 1;
+            uint64_t Q = fm[i], B = 0;
+            size_t planes = 3ull << (2 * plan[i].k);
+            for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
+                if (placed[j]) continue;
+                const uint64_t Sj = fm[j];
+                const size_t pj = 3ull << (2 * plan[j].k);
+                if (Sj & B) {
+                    B |= Sj;
+                } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
+                    Q |= Sj;
+                    planes += pj;
+                    mem.push_back(j);
+                    placed[j] = 1;
+                } else {
+                    B |= Sj;
+                }
+            }
+            // tile qubits: pinned + the pass's + the lowest others, ascending
+            uint64_t tile = Q | pin;
+            for (int q = 0; q < s->n && __builtin_popcountll(tile) < T; ++q) tile |= 1ull << q;
+            PassDesc cur;
+            for (int q = 0; q < s->n; ++q)
+                if ((tile >> q) & 1ull) cur.S.push_back(q);
+            plan_pass_tile(cur);
+            for (size_t j : mem) add_gate(cur, j);
+            passes.push_back(std::move(cur));
         }
-        if (!cur.gates.empty()) passes.push_back(std::move(cur));
-        // tiles need contiguous runs of >= 16 amplitudes (T - 5 >= 4 >= k keeps
-        // the planner from evicting qubits 0..4; checked, else run unblocked)
+        // tiles need contiguous runs of >= 16 amplitudes (pinned qubits 0..3;
+        // checked, else run unblocked)
         for (auto& pd : passes)
             if (pd.r < 4) blocked = false;
     }
