@@ -255,6 +255,12 @@ struct alignas(16) RpassParams {
     uint64_t goff[16];
     uint32_t soff[16];
     uint32_t gcode[kRpMaxGates];  // register mask (bits 0..4) | kind << 5 | matrix float offset << 8
+    // direct store: the last phase writes its registers straight to HBM
+    // (16 B pairs; tile bit 0 in registers, tile bits 1..3 on lanes 0..2 so
+    // each quarter-warp writes one 128 B run) instead of through the tile
+    int direct;
+    uint64_t dgoff[16];   // amplitude offset of register pair j
+    uint64_t dgtbw[10];   // amplitude offset of thread-index bit i
     RpPhase ph[kRpMaxPhases];
 };
 
@@ -641,7 +647,13 @@ __device__ __forceinline__ void reg_gate_dispatch(int code, float2 (&a)[1 << M],
 }
 
 template <int M, bool F2>
-__global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 168) apply_rpass(const __grid_constant__ RpassParams p) {
+#ifndef SVB_RP_STAGES
+#define SVB_RP_STAGES 1  // tile buffers per CTA (1: four CTAs per SM at T = 12 measured faster than 2 with three)
+#endif
+#ifndef SVB_RP_MAXREG5
+#define SVB_RP_MAXREG5 128
+#endif
+__global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : SVB_RP_MAXREG5) apply_rpass(const __grid_constant__ RpassParams p) {
     constexpr int NA = 1 << M;   // amplitudes per thread
     constexpr int UPT = NA / 2;  // 16 B load/store units per thread
     extern __shared__ float4 rsm[];
@@ -680,25 +692,36 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
 #pragma unroll
         for (int i = 0; i < UPT; ++i) st_stream(reinterpret_cast<float4*>(g + p.goff[i]), lds4(sbuf + (sthr ^ p.soff[i])));
     };
+    uint64_t dgthr = 0;
+    for (int i = 0; i < p.tbits; ++i)
+        if ((threadIdx.x >> i) & 1u) dgthr += p.dgtbw[i];
     uint64_t u = blockIdx.x;
     const float2* gcur = nullptr;
+    const float2* gtile = nullptr;
     if (u < p.n_tiles) {
-        gcur = p.psi + tbase(u) + dthr;
+        gtile = p.psi + tbase(u);
+        gcur = gtile + dthr;
         load(gcur, s0);
     }
     cp_async_commit();
     for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
-        const uint32_t cur = s0 + (uint32_t)(it & 1) * tile_bytes;
-        const uint32_t nxt = s0 + (uint32_t)((it + 1) & 1) * tile_bytes;
+        const uint32_t cur = s0 + (SVB_RP_STAGES == 2 ? (uint32_t)(it & 1) * tile_bytes : 0u);
+        const uint32_t nxt = s0 + (SVB_RP_STAGES == 2 ? (uint32_t)((it + 1) & 1) * tile_bytes : 0u);
         const uint64_t un = u + gridDim.x;
         const float2* gnext = nullptr;
-        __syncthreads();  // buffer `nxt` drained by the previous store
+        const float2* gtile_next = nullptr;
         if (un < p.n_tiles) {
-            gnext = p.psi + tbase(un) + dthr;
-            load(gnext, nxt);
+            gtile_next = p.psi + tbase(un);
+            gnext = gtile_next + dthr;
         }
-        cp_async_commit();
-        cp_async_wait1();
+        if constexpr (SVB_RP_STAGES == 2) {
+            __syncthreads();  // buffer `nxt` drained by the previous store
+            if (gnext) load(gnext, nxt);
+            cp_async_commit();
+            cp_async_wait1();
+        } else {
+            cp_async_wait0();
+        }
         __syncthreads();
         for (int ph = 0; ph < p.nph; ++ph) {
             const RpPhase& P = p.ph[ph];
@@ -721,6 +744,14 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
                 const uint32_t code = p.gcode[gi];
                 reg_gate_dispatch<M, F2>((int)(code & 0x7fu), a, p.mats + (code >> 8));
             }
+            if (ph == p.nph - 1 && p.direct) {
+                float2* g = const_cast<float2*>(gtile) + dgthr;
+#pragma unroll
+                for (int j = 0; j < NA / 2; ++j)
+                    st_stream(reinterpret_cast<float4*>(g + p.dgoff[j]),
+                              make_float4(a[2 * j].x, a[2 * j].y, a[2 * j + 1].x, a[2 * j + 1].y));
+                break;  // the next iteration's first barrier guards `cur`
+            }
             if (P.b0) {
 #pragma unroll
                 for (int j = 0; j < NA / 2; ++j)
@@ -731,8 +762,14 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             }
             __syncthreads();
         }
-        store(const_cast<float2*>(gcur), cur);
+        if (!p.direct) store(const_cast<float2*>(gcur), cur);
+        if constexpr (SVB_RP_STAGES == 1) {
+            __syncthreads();  // every thread is done with the tile buffer
+            if (gnext) load(gnext, cur);
+            cp_async_commit();
+        }
         gcur = gnext;
+        gtile = gtile_next;
     }
 }
 
@@ -915,7 +952,7 @@ template <int M, bool F2>
 cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st) {
     const int T = (int)pd.S.size();
     const uint32_t nthr = 1u << (T - M);
-    const size_t smem = 2 * ((size_t)8 << T);
+    const size_t smem = SVB_RP_STAGES * ((size_t)8 << T);
     cudaError_t e = cudaFuncSetAttribute(apply_rpass<M, F2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     static int per_sm_cache[16] = {0};
@@ -1010,6 +1047,20 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             for (int q : pd.S) fprintf(stderr, "%d,", q);
             fprintf(stderr, "\n");
         }
+        {
+            static int denv = -1;
+            if (denv < 0) {
+                const char* e = getenv("SVB200_RPASS_DIRECT");
+                denv = (e && e[0] == '0') ? 0 : 1;
+            }
+            const RpPhaseHost& lp = phs.back();
+            p.direct = denv && lp.b0 && lp.lanes.size() >= 3 && lp.lanes[0] == 1 && lp.lanes[1] == 2 && lp.lanes[2] == 3;
+            if (p.direct) {
+                for (int j = 0; j < (1 << (M - 1)); ++j) p.dgoff[j] = dep(deposit(2u * j, lp.R));
+                for (int b = 0; b < p.tbits; ++b) p.dgtbw[b] = dep(1ull << lp.lanes[b]);
+            }
+        }
+        if (dbg) fprintf(stderr, "   direct=%d\n", p.direct);
         apply_rpass<M, F2><<<(unsigned)grid, nthr, smem, st>>>(p);
         e = cudaGetLastError();
         g0 = g1;
