@@ -3,9 +3,14 @@
 
 Metric: RQC circuit time in seconds (lower is better) and the apply kernels'
 achieved HBM bandwidth.  N=1 workload: BASELINE.json configs[1], the paper's
-30-qubit RQC at depth 14 with max_fused = 4 (the paper's
-optimum, L189).  A "step" is one pass of the whole hot path:
-|0..0> init, every fused-gate apply of the circuit, and drawing 10^6 samples.
+30-qubit RQC at depth 14 "with optimal fusion" (north star):
+the same device step is first timed for max_fused = 1..6 with the library's
+default execution path for each (register-blocked passes for max_fused <= 2,
+one launch per fused gate otherwise; `fusion_sweep_s`), and the fastest
+max_fused is the timed configuration (`--max-fused F` fixes it instead; the
+paper found 4 optimal on its GPUs, L189).  A "step" is one pass of the whole
+hot path: |0..0> init, every fused-gate apply of the
+circuit, and drawing 10^6 samples.
 
   value  -- device time per step with the fused circuit already resident
             (sv_circuit_run_device + sv_sample_device), CUDA events on the
@@ -56,7 +61,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--qubits", type=int, default=0)
     ap.add_argument("--depth", type=int, default=14)
-    ap.add_argument("--max-fused", type=int, default=4)
+    ap.add_argument("--max-fused", type=int, default=-1,
+                    help="-1 (default): optimal over 1..6 from the fusion sweep (N=1; 4 for N>1)")
     ap.add_argument("--seed", type=int, default=2023)
     ap.add_argument("--samples", type=int, default=N_SAMPLES)
     ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
@@ -221,6 +227,37 @@ def run_ours(args):
             dist.barrier()
         torch.cuda.synchronize()
 
+    # ---- fusion sweep (N = 1): the same device step for max_fused = 1..6,
+    # CUDA events on the launching stream, 1 warm-up + 3 timed steps each;
+    # the fastest max_fused becomes the timed configuration (max_fused = -1)
+    sweep = None
+    if world == 1 and not fp64 and (args.max_fused < 0 or not args.no_sweep):
+        sweep = {}
+        for f in range(1, 7):
+            c = sv.sv_circuit_create(h, gates, f)
+
+            def st_f():
+                sv.sv_reset(h)
+                sv.sv_circuit_run_device(h, c)
+                sv.sv_sample_device(h, 1, args.samples, samples_dev.data_ptr())
+
+            st_f()
+            barrier()
+            a0 = torch.cuda.Event(enable_timing=True)
+            a1 = torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            for _ in range(3):
+                st_f()
+            a1.record(stream)
+            barrier()
+            sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
+            sv.sv_circuit_destroy(c)
+    if args.max_fused < 0:
+        args.max_fused = int(min(sweep, key=sweep.get)) if sweep else 4
+        fusion_choice = "optimal over max_fused 1..6 (fusion_sweep_s)" if sweep else "4 (sharded / complex128 default)"
+    else:
+        fusion_choice = "fixed by --max-fused"
+
     # ---- device step: fused circuit resident
     circ = sv.sv_circuit_create(h, gates, args.max_fused)
     cst = sv.sv_circuit_stats(circ)
@@ -241,6 +278,7 @@ def run_ours(args):
     bytes_apply = 0
     flops = 0
     bytes_exch = 0
+    fma = 0
     with ClockSampler(local) as clk:
         start = torch.cuda.Event(enable_timing=True)
         end = torch.cuda.Event(enable_timing=True)
@@ -259,6 +297,7 @@ def run_ours(args):
             bytes_apply += st["bytes_apply"]
             flops += st["flops_apply"]
             bytes_exch += st["bytes_exchange"]
+            fma += st["fma_apply"]
         end.record(stream)
         barrier()
     sv.sv_set_timing(h, False)
@@ -298,31 +337,6 @@ def run_ours(args):
     e2e_ms = float(et.item())
     h2d = int(sum(8 * (1 << (2 * k)) * c for k, c in enumerate(cst["fused_hist"])))
 
-    # ---- fusion sweep (N = 1): the same device step for max_fused = 1..6,
-    # CUDA events on the launching stream, 1 warm-up + 3 timed steps each
-    sweep = None
-    if world == 1 and not args.no_sweep and not fp64:
-        sweep = {}
-        for f in range(1, 7):
-            c = sv.sv_circuit_create(h, gates, f)
-
-            def st_f():
-                sv.sv_reset(h)
-                sv.sv_circuit_run_device(h, c)
-                sv.sv_sample_device(h, 1, args.samples, samples_dev.data_ptr())
-
-            st_f()
-            barrier()
-            a0 = torch.cuda.Event(enable_timing=True)
-            a1 = torch.cuda.Event(enable_timing=True)
-            a0.record(stream)
-            for _ in range(3):
-                st_f()
-            a1.record(stream)
-            barrier()
-            sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
-            sv.sv_circuit_destroy(c)
-
     peak, peak_src = load_peaks()
     launches_apply = n_high + n_low
     avg_launch = t_apply / max(launches_apply, 1)
@@ -339,7 +353,7 @@ def run_ours(args):
     if rank == 0:
         sv_fused = cst["n_fused"]
         out = {
-            "metric": f"rqc_circuit_time_{n}q_d{args.depth}_f{args.max_fused}" + ("_c128" if fp64 else ""),
+            "metric": f"rqc_circuit_time_{n}q_d{args.depth}" + ("_c128" if fp64 else ""),
             "value": ms / 1e3,
             "unit": "s",
             "n_gpus": world,
@@ -353,7 +367,10 @@ def run_ours(args):
             "data": "synthetic",
             "config": {
                 "workload": f"rqc_{n}q_d{args.depth}_f{args.max_fused}",
-                "n_qubits": n, "depth": args.depth, "max_fused": args.max_fused, "seed": args.seed,
+                "n_qubits": n, "depth": args.depth, "max_fused": args.max_fused, "fusion": fusion_choice,
+                "execution": ("register-blocked passes (apply_rpass), tile qubits "
+                              f"{cst.get('block_bits', 12)}" if cst.get("n_passes", 0) else "one launch per fused gate"),
+                "seed": args.seed,
                 "gates": len(gates), "n_fused": sv_fused, "fused_hist": cst["fused_hist"],
                 "samples_per_step": args.samples,
                 "step": "sv_reset + all fused-gate applies + sv_sample_device(1e6)",
@@ -371,11 +388,21 @@ def run_ours(args):
                 "apply_launches_per_step": launches_apply // max(args.steps, 1),
                 "block_bits": args.block_bits,
             },
-            "roofline": {"bound": "hbm", "kernel": "apply_high+apply_low", "achieved": achieved, "peak": peak,
+            "roofline": {"bound": "hbm",
+                         "kernel": ("apply_rpass (register-blocked pass: all gates of a pass per HBM read+write)"
+                                    if cst["n_passes"] else "apply_high+apply_low (one launch per fused gate)"),
+                         "achieved": achieved, "peak": peak,
                          "peak_source": peak_src, "unit": "GB/s", "frac": frac,
                          "frac_of_8tbs": achieved / 8000.0 if achieved else None,
                          "algorithmic_bytes_per_launch": bytes_per_launch,
-                         "traffic": load_traffic("apply")},
+                         "traffic": load_traffic("rpass" if cst["n_passes"] else "apply"),
+                         # the blocked passes are bound by HBM and the FP32 pipe
+                         # together: the FMA-pipe share of the same launches
+                         # (fp32 FMAs executed / (148 SMs x 128 FMA/clk x max clock))
+                         "fma_pipe": ({"achieved_tfma_s": fma / t_apply / 1e12,
+                                       "peak_tfma_s": 148 * 128 * (clk.summary().get("sm_max_mhz") or 1965) * 1e6 / 1e12,
+                                       "frac": fma / t_apply / (148 * 128 * (clk.summary().get("sm_max_mhz") or 1965) * 1e6)}
+                                      if fma and t_apply else None)},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_ms / 1e3, "unit": "s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": 8 * args.samples},

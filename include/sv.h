@@ -102,6 +102,11 @@ typedef struct {
     uint64_t bytes_apply;       /* per shard */
     uint64_t bytes_exchange;    /* sent per shard */
     uint64_t flops_apply;       /* (8*2^k - 2) per amplitude per fused gate, per shard */
+    int32_t n_passes;           /* cache-blocked passes (0: one launch per fused gate) */
+    int32_t block_bits;         /* tile qubits of the blocked passes (0: not blocked)  */
+    uint64_t fma_apply;         /* fp32 FMAs the register-blocked passes execute (dense
+                                   2^k x 2^k: 4*2^k per amplitude, diagonal: 4, CZ: 0),
+                                   per shard; 0 for other kernels                       */
 } sv_stats;
 
 typedef struct {
@@ -214,12 +219,15 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each);
 
 /* ---- misc ------------------------------------------------------------------- */
 /* Cache-blocked circuit execution (related work [12],
- * PAPER.md L221): sv_circuit_create on an unsharded state with max_fused in
- * [1,4] groups the fused gates into passes whose qubits all lie in one set of
- * tile_bits qubits; each pass is ONE HBM read + write of the state with all its
- * gates applied in shared memory.  tile_bits in [10,13]; 0 disables (one launch
- * per fused gate).  Default 0 (off: on B200 the per-gate path is faster today,
- * DESIGN.md).  Takes effect for circuits created afterwards. */
+ * PAPER.md L221): sv_circuit_create on an unsharded complex64 state with
+ * max_fused in [1,4] groups the fused gates into passes whose qubits all lie
+ * in one set of tile_bits qubits (qubits 0..3 always included); each pass is
+ * ONE HBM read + write of the state.  Passes of gates with k <= 2 run in the
+ * register-blocked kernel (32 amplitudes per thread, gates applied in
+ * registers); others in the shared-memory pass kernel.
+ * tile_bits in [10,13]; 0 disables (one launch per fused gate); -1 (default)
+ * = auto: 12 when max_fused <= 2 and n >= 20, else off.  Takes effect for
+ * circuits created afterwards.  Errors: SV_EINVAL for other values. */
 int sv_set_blocking(sv_state* s, int tile_bits);
 /* 1: record CUDA events around every launch and fill the *_dev_s stats. */
 int sv_set_timing(sv_state* s, int enable);

@@ -60,6 +60,9 @@ class sv_stats(ctypes.Structure):
         ("bytes_apply", ctypes.c_uint64),
         ("bytes_exchange", ctypes.c_uint64),
         ("flops_apply", ctypes.c_uint64),
+        ("n_passes", ctypes.c_int32),
+        ("block_bits", ctypes.c_int32),
+        ("fma_apply", ctypes.c_uint64),
     ]
 
     def as_dict(self):

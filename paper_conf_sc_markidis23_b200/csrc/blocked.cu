@@ -948,6 +948,20 @@ int phase_conflicts(const RpPhaseHost& ph, int T, int M) {
     return worst;
 }
 
+// 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
+int gate_kind(const PassDesc& pd, const PassGate& pg) {
+    const int D = 1 << pg.k;
+    const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
+    bool diag = true, cz = pg.k == 2;
+    for (int r = 0; r < D; ++r)
+        for (int c = 0; c < D; ++c) {
+            const float re = mg[2 * (r * D + c)], im = mg[2 * (r * D + c) + 1];
+            if (r != c && (re != 0.f || im != 0.f)) diag = cz = false;
+            if (r == c && (im != 0.f || re != (r == D - 1 ? -1.f : 1.f))) cz = false;
+        }
+    return cz ? 2 : diag ? 1 : 0;
+}
+
 template <int M, bool F2>
 cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st) {
     const int T = (int)pd.S.size();
@@ -1014,14 +1028,7 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                 const PassGate& pg = pd.gates[g];
                 const int D = 1 << pg.k;
                 const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
-                bool diag = true, cz = pg.k == 2;
-                for (int r = 0; r < D; ++r)
-                    for (int c = 0; c < D; ++c) {
-                        const float re = mg[2 * (r * D + c)], im = mg[2 * (r * D + c) + 1];
-                        if (r != c && (re != 0.f || im != 0.f)) diag = cz = false;
-                        if (r == c && (im != 0.f || re != (r == D - 1 ? -1.f : 1.f))) cz = false;
-                    }
-                const int kind = cz ? 2 : diag ? 1 : 0;
+                const int kind = gate_kind(pd, pg);
                 const int ne = kind == 1 ? D : kind == 2 ? 0 : D * D;
                 for (int e2 = 0; e2 < ne; ++e2) {
                     const int src = kind == 1 ? e2 * D + e2 : e2;
@@ -1083,6 +1090,15 @@ bool rpass_supported(const PassDesc& pd) {
     for (auto& g : pd.gates)
         if (g.k > 2) return false;
     return true;
+}
+
+uint64_t rpass_fma_per_amp(const PassDesc& pd) {
+    uint64_t f = 0;
+    for (auto& g : pd.gates) {
+        const int kind = gate_kind(pd, g);
+        f += kind == 0 ? 4ull << g.k : kind == 1 ? 4 : 0;
+    }
+    return f;
 }
 
 void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {

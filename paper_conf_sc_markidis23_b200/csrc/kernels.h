@@ -85,6 +85,7 @@ struct PassDesc {
     std::vector<PassGate> gates;
     std::vector<float> planes;
     std::vector<float> mats;  // per gate: 2^k x 2^k complex64, row-major (re, im pairs)
+    uint64_t fma_per_amp = 0;  // rpass FMAs per amplitude (stats), set at circuit creation
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
@@ -92,6 +93,9 @@ cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream
 // amplitudes of the tile in registers and applies every gate of a phase
 // there; phases exchange through the shared-memory tile.
 bool rpass_supported(const PassDesc& pd);
+// fp32 FMAs per amplitude the rpass kernel executes for this pass (dense
+// 2^k x 2^k: 4 * 2^k, diagonal: 4, CZ-like: 0)
+uint64_t rpass_fma_per_amp(const PassDesc& pd);
 cudaError_t launch_rpass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
 // Host model of the rpass phase plan (tests / tools): number of phases and
 // the worst bank-conflict degree of their gathers.

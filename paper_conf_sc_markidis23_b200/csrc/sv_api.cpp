@@ -59,7 +59,7 @@ struct sv_state {
     bool virt = true;         // all shards on this GPU
     int device = 0;
     int vmin = 5;
-    int block_bits = 0;       // cache-blocked passes: tile qubits (0 = off; opt-in)
+    int block_bits = -1;      // cache-blocked passes: tile qubits (0 = off, -1 = auto: 12 when max_fused <= 2)
     bool fp64 = false;        // complex128 amplitudes (NEXT-1)
     size_t elem = 8;          // bytes per amplitude
     double* planes64 = nullptr;   // fp64 scratch: planes of one gate (sv_apply_fused on fp64 states)
@@ -848,7 +848,11 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     // (runs of >= 128 B); the pass's tile set S is the pinned qubits, the
     // pass's qubits, then the lowest remaining qubits (longer runs).  The
     // state never moves: a pass only chooses which amplitudes share a tile.
-    const int T = s->block_bits;
+    // auto (-1): register-blocked passes (rpass) win over one launch per fused
+    // gate when the fused gates are small (max_fused <= 2: 30q D14 F=1
+    // 0.078 s, F=2 0.084 s, per-gate F=5 0.099 s); for k >= 3 the per-gate
+    // kernels are faster
+    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->n >= 20 ? 12 : 0);
     bool blocked = !s->fp64 && s->g == 0 && T >= 10 && s->n >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
                    max_fused >= 1;
     std::vector<PassDesc> passes;
@@ -925,6 +929,12 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     const double t2 = now_s();
     c->stats.t_plan_s = t2 - t1;
     if (blocked) {
+        c->stats.n_passes = (int)passes.size();
+        c->stats.block_bits = T;
+        for (auto& pd : passes) {
+            pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
+            c->stats.fma_apply += pd.fma_per_amp << s->l;
+        }
         for (auto& pd : passes) {
             sv_circuit::Step st;
             st.type = Event::APPLY;
@@ -1104,6 +1114,9 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
             if (rc) return rc;
             s->stats.bytes_apply += 16ull << s->l;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
+            s->stats.fma_apply += st.pass.fma_per_amp << s->l;
+            s->stats.n_passes += 1;
+            s->stats.block_bits = (int)st.pass.S.size();
             continue;
         }
         if (st.type == Event::APPLY) {
@@ -1509,8 +1522,8 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each) {
 
 int sv_set_blocking(sv_state* s, int tile_bits) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
-    if (tile_bits != 0 && (tile_bits < 10 || tile_bits > 13))
-        return fail(SV_EINVAL, "tile_bits must be 0 (off) or in [10, 13]");
+    if (tile_bits != 0 && tile_bits != -1 && (tile_bits < 10 || tile_bits > 13))
+        return fail(SV_EINVAL, "tile_bits must be 0 (off), -1 (auto) or in [10, 13]");
     s->block_bits = tile_bits;
     return SV_OK;
 }

@@ -187,3 +187,63 @@ def test_prepared_circuit_and_reset():
         sv.sv_circuit_destroy(c)
     finally:
         sv.sv_destroy(h)
+
+
+def _mixed_circuit(n, m, seed):
+    """Dense 1q/2q Haar gates, diagonal gates (T, S, Z, CP(phi)), CZ and
+    permutations (CX, SWAP), biased towards qubits 0..4 so that the
+    register-blocked passes see tile bit 0 in and out of the register set,
+    all three gate kinds (dense, diagonal, CZ-like) and both store paths."""
+    rs = np.random.default_rng(seed)
+    fixed = {"t": W.GATE_T, "s": W.GATE_S, "z": W.GATE_Z, "cz": W.GATE_CZ, "cx": W.GATE_CX, "swap": W.GATE_SWAP}
+    gates = []
+    for i in range(m):
+        kind = rs.choice(["u1", "u2", "t", "s", "z", "cz", "cp", "cx", "swap"])
+        k = 2 if kind in ("u2", "cz", "cp", "cx", "swap") else 1
+        pool = np.arange(n) if rs.random() < 0.5 else np.arange(min(n, 6))
+        qs = tuple(int(x) for x in rs.choice(pool, size=k, replace=False))
+        if kind in ("u1", "u2"):
+            mat = W.haar_unitary(1 << k, rs)
+        elif kind == "cp":
+            mat = W.gate_cp(float(rs.uniform(0, 2 * np.pi)))
+        else:
+            mat = fixed[kind]
+        gates.append(W.Gate(i, str(kind), qs, mat))
+    return gates
+
+
+@pytest.mark.parametrize("bits", [10, 11, 12, 13])
+@pytest.mark.parametrize("F", [1, 2])
+def test_register_blocked_mixed_kinds(bits, F):
+    """Register-blocked passes (apply_rpass) on a circuit mixing dense,
+    diagonal and CZ-like fused gates, against the oracle."""
+    n, m = 18, 160
+    gates = _mixed_circuit(n, m, seed=100 * F + bits)
+    h = sv.sv_create(n)
+    try:
+        sv.sv_set_blocking(h, bits)
+        c = sv.sv_circuit_create(h, gates, F)
+        st = sv.sv_circuit_stats(c)
+        assert st["n_passes"] > 0 and st["block_bits"] == bits
+        sv.sv_circuit_run_device(h, c)
+        sv.sv_synchronize(h)
+        got = sv.sv_get_state(h, n)
+        sv.sv_circuit_destroy(c)
+    finally:
+        sv.sv_destroy(h)
+    _check(n, m, got, ref_c.run(n, gates))
+
+
+def test_blocking_auto_default():
+    """Default (-1 = auto): blocked passes for max_fused <= 2 at n >= 20,
+    one launch per fused gate otherwise."""
+    n = 20
+    gates = W.rqc(n, 10)
+    h = sv.sv_create(n)
+    try:
+        for F, blocked in [(1, True), (2, True), (3, False), (4, False)]:
+            c = sv.sv_circuit_create(h, gates, F)
+            assert (sv.sv_circuit_stats(c)["n_passes"] > 0) == blocked
+            sv.sv_circuit_destroy(c)
+    finally:
+        sv.sv_destroy(h)

@@ -2,9 +2,9 @@
 times (prepared circuit: sv_circuit_create + sv_reset + sv_circuit_run_device).
 
 * 30 q depth 14 (configs[1]): the whole complex128 oracle state (16 GiB,
-  oracle/sv_ref.c on all host cores) against the GPU state for max_fused = 4
-  (the headline: SIMT k=4), 5 (optimal fusion: int8 tensor cores, k=5) and 6
-  (int8 tensor cores, k=6) -- fidelity and max |delta| against the north-star
+  oracle/sv_ref.c on all host cores) against the GPU state for max_fused = 1
+  and 2 (register-blocked passes: the optimal fusion on B200), 4 (SIMT k=4),
+  5 (int8 tensor cores, k=5) and 6 (int8 tensor cores, k=6) -- fidelity and max |delta| against the north-star
   bounds, accumulated in fp64 chunk by chunk.  Sampling at 30 q is bit-exact
   against oracle/sample.py on the GPU's own complex64 state.
 * 34 q depth 20 (configs[3], 128 GiB in place; no host oracle fits): the
@@ -72,13 +72,16 @@ def ref30():
     return ref_c.run(30, W.rqc(30, 14, 2023))
 
 
-@pytest.mark.parametrize("F,kmax", [(4, 4), (5, 5), (6, 6)])
+@pytest.mark.parametrize("F,kmax", [(1, 2), (2, 2), (4, 4), (5, 5), (6, 6)])
 def test_30q_d14_state_vs_oracle(ref30, F, kmax):
+    """F = 1, 2: register-blocked passes (the library default for
+    max_fused <= 2, tile qubits 12); F >= 4: one launch per fused gate."""
     n, depth = 30, 14
     gates = W.rqc(n, depth, 2023)
     h, st = _run_prepared(n, gates, F)
     try:
         assert max(k for k, c in enumerate(st["fused_hist"]) if c) == kmax
+        assert (st["n_passes"] > 0) == (F <= 2)
         got = sv.sv_get_state(h, n)
     finally:
         sv.sv_destroy(h)

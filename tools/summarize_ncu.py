@@ -19,6 +19,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def kclass(name: str) -> str:
+    if "apply_rpass" in name or "apply_pass" in name:
+        return "rpass"
     if "apply_tci" in name or "apply_tc" in name:
         return "apply_tc"
     if "apply_high" in name or "apply_low" in name or "apply_small" in name:
@@ -107,11 +109,13 @@ def main():
     caps = [c for one in fp.split(",") for c in captures(one)]
     if caps:
         summary["full_capture"] = caps
-        summary["traffic_per_launch"]["apply"] = caps[0]["traffic_bytes"]
         for c in caps:
-            if "apply_tci" in c["kernel"]:
-                summary["traffic_per_launch"].setdefault("apply_tci", c["traffic_bytes"])
-    json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
+            summary["traffic_per_launch"].setdefault(kclass(c["kernel"]), c["traffic_bytes"])
+    old = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(old):  # keep per-class traffic of kernels not captured this time
+        for k, v in json.load(open(old)).get("traffic_per_launch", {}).items():
+            summary["traffic_per_launch"].setdefault(k, v)
+    json.dump(summary, open(old, "w"), indent=1)
     md = [f"# ncu summary ({tag})", "", f"Launch list: `{os.path.basename(lp)}` (ncu --metrics gpu__time_duration.sum "
           "--clock-control none; cold-cache, serialised: compare shares, not absolutes)", "",
           "| class | launches | time (s) | share of our kernels |", "|---|---|---|---|"]
