@@ -231,7 +231,7 @@ def run_ours(args):
     # CUDA events on the launching stream, 1 warm-up + 3 timed steps each;
     # the fastest max_fused becomes the timed configuration (max_fused = -1)
     sweep = None
-    if world == 1 and not fp64 and (args.max_fused < 0 or not args.no_sweep):
+    if not fp64 and (args.max_fused < 0 or (world == 1 and not args.no_sweep)):
         sweep = {}
         for f in range(1, 7):
             c = sv.sv_circuit_create(h, gates, f)
@@ -253,8 +253,11 @@ def run_ours(args):
             sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
             sv.sv_circuit_destroy(c)
     if args.max_fused < 0:
-        args.max_fused = int(min(sweep, key=sweep.get)) if sweep else 4
-        fusion_choice = "optimal over max_fused 1..6 (fusion_sweep_s)" if sweep else "4 (sharded / complex128 default)"
+        best = torch.tensor([int(min(sweep, key=sweep.get)) if sweep else 4], device="cuda")
+        if dist is not None:  # every rank runs rank 0's choice (collective calls)
+            dist.broadcast(best, 0)
+        args.max_fused = int(best.item())
+        fusion_choice = "optimal over max_fused 1..6 (fusion_sweep_s)" if sweep else "4 (complex128 default)"
     else:
         fusion_choice = "fixed by --max-fused"
 

@@ -800,6 +800,90 @@ int sv_shard_plan(const int32_t* fs, size_t len, int n, int g, int vmin, int32_t
     return SV_OK;
 }
 
+// One fused gate for build_passes: ascending local (physical) qubits and its
+// fp64 matrix over them.
+struct PassIn {
+    int k = 0;
+    int q[SV_MAX_FUSED] = {0};
+    std::vector<cd> M;
+};
+
+// Cache-blocked passes (reading R7).  Passes are formed like fused
+// gates (the S3 greedy, one level up): a pass starts at the first unplaced
+// gate and absorbs every later one whose qubits keep the pass within
+// T - kPassPinned free tile qubits, provided it does not touch a qubit of a
+// gate skipped before it (so it only moves past gates it commutes with).
+// Qubits 0..kPassPinned-1 are in every tile (runs of >= 128 B); the pass's
+// tile set S is the pinned qubits, the pass's qubits, then the lowest
+// remaining qubits (longer runs).  The state never moves: a pass only
+// chooses which amplitudes share a tile.
+std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
+    constexpr int kPassPinned = 4;
+    const uint64_t pin = (1ull << kPassPinned) - 1ull;
+    const int Fp = T - kPassPinned;
+    const size_t nf = in.size();
+    std::vector<uint64_t> fm(nf, 0);
+    for (size_t i = 0; i < nf; ++i)
+        for (int b = 0; b < in[i].k; ++b) fm[i] |= 1ull << in[i].q[b];
+    std::vector<char> placed(nf, 0);
+    std::vector<PassDesc> passes;
+    auto add_gate = [&](PassDesc& cur, size_t i) {
+        const PassIn& f = in[i];
+        const int D = 1 << f.k;
+        PassGate pg{};
+        pg.k = f.k;
+        for (int b = 0; b < f.k; ++b) pg.pos[b] = (int)(std::find(cur.S.begin(), cur.S.end(), f.q[b]) - cur.S.begin());
+        pg.poff = (uint32_t)cur.planes.size();
+        pg.moff = (uint32_t)cur.mats.size();
+        for (int e = 0; e < D * D; ++e) {
+            cur.mats.push_back((float)f.M[e].real());
+            cur.mats.push_back((float)f.M[e].imag());
+        }
+        std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
+        for (int e = 0; e < D * D; ++e) {
+            const float re = (float)f.M[e].real(), im = (float)f.M[e].imag();
+            Pp[e] = re;
+            Sp[e] = re + im;
+            Qp[e] = im - re;
+        }
+        cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
+        cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
+        cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
+        cur.gates.push_back(pg);
+    };
+    for (size_t i = 0; i < nf; ++i) {
+        if (placed[i]) continue;
+        std::vector<size_t> mem{i};
+        placed[i] = 1;
+        uint64_t Q = fm[i], B = 0;
+        size_t planes = 3ull << (2 * in[i].k);
+        for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
+            if (placed[j]) continue;
+            const uint64_t Sj = fm[j];
+            const size_t pj = 3ull << (2 * in[j].k);
+            if (Sj & B) {
+                B |= Sj;
+            } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
+                Q |= Sj;
+                planes += pj;
+                mem.push_back(j);
+                placed[j] = 1;
+            } else {
+                B |= Sj;
+            }
+        }
+        uint64_t tile = Q | pin;
+        for (int q = 0; q < 64 && __builtin_popcountll(tile) < T; ++q) tile |= 1ull << q;
+        PassDesc cur;
+        for (int q = 0; q < 64; ++q)
+            if ((tile >> q) & 1ull) cur.S.push_back(q);
+        plan_pass_tile(cur);
+        for (size_t j : mem) add_gate(cur, j);
+        passes.push_back(std::move(cur));
+    }
+    return passes;
+}
+
 int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out) {
     int rc = check_state(s);
     if (rc) return rc;
@@ -839,113 +923,14 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
     }
     c->pos_out = pos;
-    // Cache-blocked passes (unsharded, large states, k <= 4).  Passes are
-    // formed like fused gates (the S3 greedy, one level up): a pass starts at
-    // the first unplaced fused gate and absorbs every later one whose qubits
-    // keep the pass within T - kPassPinned free tile qubits, provided it does
-    // not touch a qubit of a gate skipped before it (so it only moves past
-    // gates it commutes with).  Qubits 0..kPassPinned-1 are in every tile
-    // (runs of >= 128 B); the pass's tile set S is the pinned qubits, the
-    // pass's qubits, then the lowest remaining qubits (longer runs).  The
-    // state never moves: a pass only chooses which amplitudes share a tile.
-    // auto (-1): register-blocked passes (rpass) win over one launch per fused
-    // gate when the fused gates are small (max_fused <= 2: 30q D14 F=1
-    // 0.078 s, F=2 0.084 s, per-gate F=5 0.099 s); for k >= 3 the per-gate
-    // kernels are faster
-    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->n >= 20 ? 12 : 0);
-    bool blocked = !s->fp64 && s->g == 0 && T >= 10 && s->n >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
-                   max_fused >= 1;
-    std::vector<PassDesc> passes;
-    if (blocked) {
-        constexpr int kPassPinned = 4;
-        const uint64_t pin = (1ull << kPassPinned) - 1ull;
-        const int Fp = T - kPassPinned;
-        const size_t nf = plan.size();
-        std::vector<uint64_t> fm(nf, 0);
-        for (size_t i = 0; i < nf; ++i)
-            for (int b = 0; b < plan[i].k; ++b) fm[i] |= 1ull << plan[i].q[b];
-        std::vector<char> placed(nf, 0);
-        auto add_gate = [&](PassDesc& cur, size_t i) {
-            const FusedGate& f = plan[i];
-            const int D = 1 << f.k;
-            PassGate pg{};
-            pg.k = f.k;
-            for (int b = 0; b < f.k; ++b)
-                pg.pos[b] = (int)(std::find(cur.S.begin(), cur.S.end(), f.q[b]) - cur.S.begin());
-            pg.poff = (uint32_t)cur.planes.size();
-            pg.moff = (uint32_t)cur.mats.size();
-            for (int e = 0; e < D * D; ++e) {
-                cur.mats.push_back((float)f.M[e].real());
-                cur.mats.push_back((float)f.M[e].imag());
-            }
-            std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
-            for (int e = 0; e < D * D; ++e) {
-                const float re = (float)f.M[e].real(), im = (float)f.M[e].imag();
-                Pp[e] = re;
-                Sp[e] = re + im;
-                Qp[e] = im - re;
-            }
-            cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
-            cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
-            cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
-            cur.gates.push_back(pg);
-        };
-        for (size_t i = 0; i < nf; ++i) {
-            if (placed[i]) continue;
-            std::vector<size_t> mem{i};
-            placed[i] = 1;
-            uint64_t Q = fm[i], B = 0;
-            size_t planes = 3ull << (2 * plan[i].k);
-            for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
-                if (placed[j]) continue;
-                const uint64_t Sj = fm[j];
-                const size_t pj = 3ull << (2 * plan[j].k);
-                if (Sj & B) {
-                    B |= Sj;
-                } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
-                    Q |= Sj;
-                    planes += pj;
-                    mem.push_back(j);
-                    placed[j] = 1;
-                } else {
-                    B |= Sj;
-                }
-            }
-            // tile qubits: pinned + the pass's + the lowest others, ascending
-            uint64_t tile = Q | pin;
-            for (int q = 0; q < s->n && __builtin_popcountll(tile) < T; ++q) tile |= 1ull << q;
-            PassDesc cur;
-            for (int q = 0; q < s->n; ++q)
-                if ((tile >> q) & 1ull) cur.S.push_back(q);
-            plan_pass_tile(cur);
-            for (size_t j : mem) add_gate(cur, j);
-            passes.push_back(std::move(cur));
-        }
-        // tiles need contiguous runs of >= 16 amplitudes (pinned qubits 0..3;
-        // checked, else run unblocked)
-        for (auto& pd : passes)
-            if (pd.r < 4) blocked = false;
-    }
+    // Cache-blocked passes (complex64, large shards, k <= 4; sharded or not):
+    // each maximal run of APPLY events between exchanges is cut into passes
+    // by build_passes (reading R7); exchanges and permutations stay as they are.
+    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? 12 : 0);
+    const bool blocked = !s->fp64 && T >= 10 && s->l >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
+                         max_fused >= 1;
     const double t2 = now_s();
     c->stats.t_plan_s = t2 - t1;
-    if (blocked) {
-        c->stats.n_passes = (int)passes.size();
-        c->stats.block_bits = T;
-        for (auto& pd : passes) {
-            pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
-            c->stats.fma_apply += pd.fma_per_amp << s->l;
-        }
-        for (auto& pd : passes) {
-            sv_circuit::Step st;
-            st.type = Event::APPLY;
-            st.block = true;
-            st.pass = std::move(pd);
-            c->steps.push_back(std::move(st));
-        }
-        c->stats.t_upload_s = now_s() - t2;
-        *out = c.release();
-        return SV_OK;
-    }
     if (s->fp64) {
         // complex128: one apply64 launch per fused gate; all planes and qubit
         // lists uploaded once (row a4)
@@ -984,7 +969,32 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     }
     // lower events to launch descriptors
     size_t n6 = 0;
+    std::vector<PassIn> run;
+    auto flush_passes = [&]() {
+        if (run.empty()) return;
+        for (auto& pd : build_passes(T, run)) {
+            pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
+            c->stats.fma_apply += pd.fma_per_amp << s->l;
+            c->stats.n_passes++;
+            sv_circuit::Step st;
+            st.type = Event::APPLY;
+            st.block = true;
+            st.pass = std::move(pd);
+            c->steps.push_back(std::move(st));
+        }
+        run.clear();
+    };
+    if (blocked) c->stats.block_bits = T;
     for (auto& e : ev) {
+        if (blocked && e.type == Event::APPLY) {
+            PassIn pi;
+            pi.k = e.k;
+            pi.M.resize((size_t)1 << (2 * e.k));
+            sort_matrix_qubits<cd>(e.k, e.phys, plan[e.fused].M.data(), pi.q, pi.M.data());
+            run.push_back(std::move(pi));
+            continue;
+        }
+        flush_passes();
         sv_circuit::Step st;
         st.type = e.type;
         if (e.type == Event::APPLY) {
@@ -998,6 +1008,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
         c->steps.push_back(std::move(st));
     }
+    flush_passes();
     // int8 tensor-core W slices of every tensor-core gate: one H2D upload
     {
         size_t total = 0;
@@ -1107,11 +1118,14 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     }
     for (auto& st : c->steps) {
         if (st.block) {
-            rc = launch(s, LaunchClass::HIGH, [&] {
-                return rpass_supported(st.pass) ? launch_rpass(s->shard[0], s->l, st.pass, s->stream)
-                                                : launch_pass(s->shard[0], s->l, st.pass, s->stream);
-            });
-            if (rc) return rc;
+            for (int sh = 0; sh < s->local_shards(); ++sh) {
+                float2* psi = s->virt ? s->shard[sh] : s->shard[s->rank];
+                rc = launch(s, LaunchClass::HIGH, [&] {
+                    return rpass_supported(st.pass) ? launch_rpass(psi, s->l, st.pass, s->stream)
+                                                    : launch_pass(psi, s->l, st.pass, s->stream);
+                });
+                if (rc) return rc;
+            }
             s->stats.bytes_apply += 16ull << s->l;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
             s->stats.fma_apply += st.pass.fma_per_amp << s->l;

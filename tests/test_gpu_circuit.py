@@ -247,3 +247,20 @@ def test_blocking_auto_default():
             sv.sv_circuit_destroy(c)
     finally:
         sv.sv_destroy(h)
+
+
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("F", [1, 2])
+def test_virtual_shards_blocked_passes(world, F):
+    """Register-blocked passes inside every shard between the exchanges."""
+    n = 18
+    gates = W.rqc(n, 14, seed=7 + world)
+    h = sv.sv_create_ex(n, world=world, virtual_shards=True)
+    try:
+        sv.sv_set_blocking(h, 11)
+        st = sv.sv_run_circuit(h, gates, F)
+        got = sv.sv_get_state(h, n)
+    finally:
+        sv.sv_destroy(h)
+    assert st["n_exchanges"] >= 1 and st["n_passes"] >= 1
+    _check(n, 14, got, ref_c.run(n, gates))

@@ -48,6 +48,17 @@ def main():
     if not (fid >= 1 - 1e-5 and err <= osv.max_abs_bound(n, 14) and st["n_exchanges"] >= 1):
         ok = False
         msgs.append(f"circuit fid={fid} err={err} exch={st['n_exchanges']}")
+    # 1c. register-blocked passes inside the shards between exchanges (F = 1, tile 10)
+    sv.sv_set_blocking(h, 10)
+    sv.sv_reset(h)
+    st1 = sv.sv_run_circuit(h, gates, 1)
+    psi1 = sv.sv_get_state(h, n)
+    sv.sv_set_blocking(h, -1)
+    fid1 = osv.fidelity(psi1.astype(np.complex128), ref)
+    err1 = float(np.abs(psi1.astype(np.complex128) - ref).max())
+    if not (fid1 >= 1 - 1e-5 and err1 <= osv.max_abs_bound(n, 14) and st1["n_passes"] >= 1):
+        ok = False
+        msgs.append(f"blocked F=1 fid={fid1} err={err1} passes={st1['n_passes']}")
     # 1b. F = 5 (int8 tensor-core apply inside the shards when >= 13 local qubits)
     sv.sv_reset(h)
     st5 = sv.sv_run_circuit(h, gates, 5)
