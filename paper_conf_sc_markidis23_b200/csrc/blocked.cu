@@ -261,6 +261,11 @@ struct alignas(16) RpassParams {
     int direct;
     uint64_t dgoff[16];   // amplitude offset of register pair j
     uint64_t dgtbw[10];   // amplitude offset of thread-index bit i
+    // direct load: the first phase reads its registers straight from HBM
+    // (same layout condition; one tile buffer only) instead of via the tile
+    int dload;
+    uint64_t lgoff[16];
+    uint64_t lgtbw[10];
     RpPhase ph[kRpMaxPhases];
 };
 
@@ -274,6 +279,12 @@ __host__ __device__ constexpr int pdep5(int v, int mask) {
     return r;
 }
 __host__ __device__ constexpr int popc5(int m) { return (m & 1) + ((m >> 1) & 1) + ((m >> 2) & 1) + ((m >> 3) & 1) + ((m >> 4) & 1); }
+
+__device__ __forceinline__ float4 ld_stream(const float4* p) {
+    float4 v;
+    asm volatile("ld.global.cs.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+    return v;
+}
 
 // packed fp32 pair FMA (FFMA2): d = a * b + c per lane
 __device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
@@ -692,16 +703,19 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
 #pragma unroll
         for (int i = 0; i < UPT; ++i) st_stream(reinterpret_cast<float4*>(g + p.goff[i]), lds4(sbuf + (sthr ^ p.soff[i])));
     };
-    uint64_t dgthr = 0;
+    uint64_t dgthr = 0, lgthr = 0;
     for (int i = 0; i < p.tbits; ++i)
-        if ((threadIdx.x >> i) & 1u) dgthr += p.dgtbw[i];
+        if ((threadIdx.x >> i) & 1u) {
+            dgthr += p.dgtbw[i];
+            lgthr += p.lgtbw[i];
+        }
     uint64_t u = blockIdx.x;
     const float2* gcur = nullptr;
     const float2* gtile = nullptr;
     if (u < p.n_tiles) {
         gtile = p.psi + tbase(u);
         gcur = gtile + dthr;
-        load(gcur, s0);
+        if (!p.dload) load(gcur, s0);
     }
     cp_async_commit();
     for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
@@ -729,7 +743,15 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             for (int i = 0; i < p.tbits; ++i)
                 if ((threadIdx.x >> i) & 1u) tb ^= P.tbw[i];
             float2 a[NA];
-            if (P.b0) {
+            if (ph == 0 && p.dload) {
+                const float2* g = gtile + lgthr;
+#pragma unroll
+                for (int j = 0; j < NA / 2; ++j) {
+                    const float4 v = ld_stream(reinterpret_cast<const float4*>(g + p.lgoff[j]));
+                    a[2 * j] = make_float2(v.x, v.y);
+                    a[2 * j + 1] = make_float2(v.z, v.w);
+                }
+            } else if (P.b0) {
 #pragma unroll
                 for (int j = 0; j < NA / 2; ++j) {
                     const float4 v = lds4(cur + (tb ^ P.roff[2 * j]));
@@ -764,9 +786,11 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
         }
         if (!p.direct) store(const_cast<float2*>(gcur), cur);
         if constexpr (SVB_RP_STAGES == 1) {
-            __syncthreads();  // every thread is done with the tile buffer
-            if (gnext) load(gnext, cur);
-            cp_async_commit();
+            if (!p.dload) {
+                __syncthreads();  // every thread is done with the tile buffer
+                if (gnext) load(gnext, cur);
+                cp_async_commit();
+            }
         }
         gcur = gnext;
         gtile = gtile_next;
@@ -885,21 +909,43 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
     };
     while (!rem.empty()) {
         RpPhaseHost ph;
-        uint32_t used = 0, blocked = 0;
-        std::vector<int> keep;
-        for (int g : rem) {
-            const uint32_t m = gmask(g);
-            if (!(m & blocked) && __builtin_popcount(used | m) <= M) {
-                used |= m;
-                ph.gates.push_back(g);
-            } else {
-                blocked |= m;
-                keep.push_back(g);
+        // R = the M-subset of tile positions that lets the most remaining
+        // gates run in this phase (a gate runs if its positions are in R and
+        // it touches no position of a gate skipped before it); ties prefer
+        // tile bit 0 in R (16 B gathers), then R free of bits 1..3 (lanes
+        // 0..2 = bits 1..3: direct-store layout)
+        uint32_t used = 0;
+        int best = -1;
+        for (uint32_t R = (1u << M) - 1u; R < (1u << T);) {
+            int cnt = 0;
+            uint32_t blocked = 0;
+            for (int g : rem) {
+                const uint32_t m = gmask(g);
+                if (!(m & blocked) && !(m & ~R)) ++cnt;
+                else blocked |= m;
             }
+            const int score = 4 * cnt + ((R & 1u) ? 2 : 0) + ((R & 0xEu) ? 0 : 1);
+            if (score > best) {
+                best = score;
+                used = R;
+            }
+            const uint32_t c = R & (0u - R), r = R + c;  // next subset of the same size (Gosper)
+            R = (((r ^ R) >> 2) / c) | r;
         }
-        rem.swap(keep);
-        if (__builtin_popcount(used) < M) used |= 1u;  // tile bit 0 in registers: 16 B gathers
-        for (int q = T - 1; q >= 0 && __builtin_popcount(used) < M; --q) used |= 1u << q;
+        {
+            uint32_t blocked = 0;
+            std::vector<int> keep;
+            for (int g : rem) {
+                const uint32_t m = gmask(g);
+                if (!(m & blocked) && !(m & ~used)) {
+                    ph.gates.push_back(g);
+                } else {
+                    blocked |= m;
+                    keep.push_back(g);
+                }
+            }
+            rem.swap(keep);
+        }
         for (int q = 0; q < T; ++q)
             if ((used >> q) & 1u) ph.R.push_back(q);
         ph.b0 = (used & 1u) != 0;
@@ -1060,14 +1106,30 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                 const char* e = getenv("SVB200_RPASS_DIRECT");
                 denv = (e && e[0] == '0') ? 0 : 1;
             }
+            auto coalesced = [](const RpPhaseHost& h) {
+                return h.b0 && h.lanes.size() >= 3 && h.lanes[0] == 1 && h.lanes[1] == 2 && h.lanes[2] == 3;
+            };
             const RpPhaseHost& lp = phs.back();
-            p.direct = denv && lp.b0 && lp.lanes.size() >= 3 && lp.lanes[0] == 1 && lp.lanes[1] == 2 && lp.lanes[2] == 3;
+            p.direct = denv && coalesced(lp);
             if (p.direct) {
                 for (int j = 0; j < (1 << (M - 1)); ++j) p.dgoff[j] = dep(deposit(2u * j, lp.R));
                 for (int b = 0; b < p.tbits; ++b) p.dgtbw[b] = dep(1ull << lp.lanes[b]);
             }
+            const RpPhaseHost& fp = phs.front();
+            // measured 1.5 % slower on 30q F=1 (the load latency is no longer
+            // hidden behind the other CTAs' phases): opt-in SVB200_RPASS_DLOAD=1
+            static int lenv = -1;
+            if (lenv < 0) {
+                const char* e = getenv("SVB200_RPASS_DLOAD");
+                lenv = (e && e[0] == '1') ? 1 : 0;
+            }
+            p.dload = lenv && SVB_RP_STAGES == 1 && coalesced(fp);
+            if (p.dload) {
+                for (int j = 0; j < (1 << (M - 1)); ++j) p.lgoff[j] = dep(deposit(2u * j, fp.R));
+                for (int b = 0; b < p.tbits; ++b) p.lgtbw[b] = dep(1ull << fp.lanes[b]);
+            }
         }
-        if (dbg) fprintf(stderr, "   direct=%d\n", p.direct);
+        if (dbg) fprintf(stderr, "   direct=%d dload=%d\n", p.direct, p.dload);
         apply_rpass<M, F2><<<(unsigned)grid, nthr, smem, st>>>(p);
         e = cudaGetLastError();
         g0 = g1;
@@ -1086,7 +1148,7 @@ bool rpass_supported(const PassDesc& pd) {
     }
     if (!env) return false;
     const int T = (int)pd.S.size();
-    if (T < 10 || T > 13 || pd.r < 4) return false;
+    if (T < 10 || T > 13 || pd.r < 1) return false;
     for (auto& g : pd.gates)
         if (g.k > 2) return false;
     return true;

@@ -818,7 +818,11 @@ struct PassIn {
 // remaining qubits (longer runs).  The state never moves: a pass only
 // chooses which amplitudes share a tile.
 std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
-    constexpr int kPassPinned = 4;
+    static int kPassPinned = 0;
+    if (!kPassPinned) {
+        const char* e = getenv("SVB200_PASS_PIN");
+        kPassPinned = (e && e[0] >= '1' && e[0] <= '6') ? e[0] - '0' : 4;
+    }
     const uint64_t pin = (1ull << kPassPinned) - 1ull;
     const int Fp = T - kPassPinned;
     const size_t nf = in.size();
