@@ -383,21 +383,26 @@ __device__ __forceinline__ void reg_diag(float2 (&a)[1 << M], const float* __res
     }
 }
 
-// CZ-like gate (diag(1, 1, 1, -1) on register bits MASK): sign flips only.
+// CZ-like gate (diag(1, 1, 1, -1)): sign flips only.  Its qubits need not be
+// register bits: MASK holds the ones that are, and `tp` (per thread) tells
+// whether the thread-index bits holding the others are all 1.
 template <int M, int MASK>
-__device__ __forceinline__ void reg_cz(float2 (&a)[1 << M]) {
+__device__ __forceinline__ void reg_cz(float2 (&a)[1 << M], bool tp) {
 #pragma unroll
     for (int j = 0; j < (1 << M); ++j)
-        if ((j & MASK) == MASK) a[j] = make_float2(-a[j].x, -a[j].y);
+        if ((j & MASK) == MASK) {
+            if (popc5(MASK) == 2 || tp) a[j] = make_float2(-a[j].x, -a[j].y);
+        }
 }
 
 template <int M, bool F2>
-__device__ __forceinline__ void reg_gate_dispatch(int code, float2 (&a)[1 << M], const float* mf) {
-    // code = mask (bits 0..4) | kind << 5: 0 dense, 1 diagonal, 2 CZ-like.
+__device__ __forceinline__ void reg_gate_dispatch(uint32_t code, float2 (&a)[1 << M], const float* mf) {
+    // code = register mask (bits 0..4) | kind << 5 (0 dense, 1 diagonal, 2 CZ-like)
+    //        | dense/diagonal: matrix float offset << 8; CZ: thread-index mask << 8.
     // Balanced compare trees on the (warp-uniform) code: a switch becomes a
     // BRX jump table on a vector register, and the matrices then load with
     // LDC into vector registers instead of uniform registers
-    const int mask = code & 31, kind = code >> 5;
+    const int mask = code & 31, kind = (code >> 5) & 3;
     if constexpr (M == 4) {
         if (kind == 0) {
             if (mask < 6) {
@@ -476,24 +481,46 @@ __device__ __forceinline__ void reg_gate_dispatch(int code, float2 (&a)[1 << M],
                 }
             }
         } else {
-            if (mask < 9) {
-                if (mask < 5) {
-                    reg_cz<4, 3>(a);
-                } else {
-                    if (mask < 6) {
-                        reg_cz<4, 5>(a);
+            const uint32_t tm = code >> 8;
+            const bool tp = (threadIdx.x & tm) == tm;
+            if (mask < 5) {
+                if (mask < 2) {
+                    if (mask < 1) {
+                        reg_cz<4, 0>(a, tp);
                     } else {
-                        reg_cz<4, 6>(a);
+                        reg_cz<4, 1>(a, tp);
+                    }
+                } else {
+                    if (mask < 3) {
+                        reg_cz<4, 2>(a, tp);
+                    } else {
+                        if (mask < 4) {
+                            reg_cz<4, 3>(a, tp);
+                        } else {
+                            reg_cz<4, 4>(a, tp);
+                        }
                     }
                 }
             } else {
-                if (mask < 10) {
-                    reg_cz<4, 9>(a);
-                } else {
-                    if (mask < 12) {
-                        reg_cz<4, 10>(a);
+                if (mask < 9) {
+                    if (mask < 6) {
+                        reg_cz<4, 5>(a, tp);
                     } else {
-                        reg_cz<4, 12>(a);
+                        if (mask < 8) {
+                            reg_cz<4, 6>(a, tp);
+                        } else {
+                            reg_cz<4, 8>(a, tp);
+                        }
+                    }
+                } else {
+                    if (mask < 10) {
+                        reg_cz<4, 9>(a, tp);
+                    } else {
+                        if (mask < 12) {
+                            reg_cz<4, 10>(a, tp);
+                        } else {
+                            reg_cz<4, 12>(a, tp);
+                        }
                     }
                 }
             }
@@ -616,39 +643,65 @@ __device__ __forceinline__ void reg_gate_dispatch(int code, float2 (&a)[1 << M],
                 }
             }
         } else {
-            if (mask < 12) {
-                if (mask < 6) {
-                    if (mask < 5) {
-                        reg_cz<5, 3>(a);
+            const uint32_t tm = code >> 8;
+            const bool tp = (threadIdx.x & tm) == tm;
+            if (mask < 9) {
+                if (mask < 4) {
+                    if (mask < 2) {
+                        if (mask < 1) {
+                            reg_cz<5, 0>(a, tp);
+                        } else {
+                            reg_cz<5, 1>(a, tp);
+                        }
                     } else {
-                        reg_cz<5, 5>(a);
+                        if (mask < 3) {
+                            reg_cz<5, 2>(a, tp);
+                        } else {
+                            reg_cz<5, 3>(a, tp);
+                        }
                     }
                 } else {
-                    if (mask < 9) {
-                        reg_cz<5, 6>(a);
-                    } else {
-                        if (mask < 10) {
-                            reg_cz<5, 9>(a);
+                    if (mask < 6) {
+                        if (mask < 5) {
+                            reg_cz<5, 4>(a, tp);
                         } else {
-                            reg_cz<5, 10>(a);
+                            reg_cz<5, 5>(a, tp);
+                        }
+                    } else {
+                        if (mask < 8) {
+                            reg_cz<5, 6>(a, tp);
+                        } else {
+                            reg_cz<5, 8>(a, tp);
                         }
                     }
                 }
             } else {
-                if (mask < 18) {
-                    if (mask < 17) {
-                        reg_cz<5, 12>(a);
+                if (mask < 17) {
+                    if (mask < 12) {
+                        if (mask < 10) {
+                            reg_cz<5, 9>(a, tp);
+                        } else {
+                            reg_cz<5, 10>(a, tp);
+                        }
                     } else {
-                        reg_cz<5, 17>(a);
+                        if (mask < 16) {
+                            reg_cz<5, 12>(a, tp);
+                        } else {
+                            reg_cz<5, 16>(a, tp);
+                        }
                     }
                 } else {
                     if (mask < 20) {
-                        reg_cz<5, 18>(a);
+                        if (mask < 18) {
+                            reg_cz<5, 17>(a, tp);
+                        } else {
+                            reg_cz<5, 18>(a, tp);
+                        }
                     } else {
                         if (mask < 24) {
-                            reg_cz<5, 20>(a);
+                            reg_cz<5, 20>(a, tp);
                         } else {
-                            reg_cz<5, 24>(a);
+                            reg_cz<5, 24>(a, tp);
                         }
                     }
                 }
@@ -657,13 +710,13 @@ __device__ __forceinline__ void reg_gate_dispatch(int code, float2 (&a)[1 << M],
     }
 }
 
-template <int M, bool F2>
 #ifndef SVB_RP_STAGES
 #define SVB_RP_STAGES 1  // tile buffers per CTA (1: four CTAs per SM at T = 12 measured faster than 2 with three)
 #endif
 #ifndef SVB_RP_MAXREG5
 #define SVB_RP_MAXREG5 128
 #endif
+template <int M, bool F2>
 __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : SVB_RP_MAXREG5) apply_rpass(const __grid_constant__ RpassParams p) {
     constexpr int NA = 1 << M;   // amplitudes per thread
     constexpr int UPT = NA / 2;  // 16 B load/store units per thread
@@ -764,7 +817,7 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             }
             for (int gi = P.g0; gi < P.g1; ++gi) {
                 const uint32_t code = p.gcode[gi];
-                reg_gate_dispatch<M, F2>((int)(code & 0x7fu), a, p.mats + (code >> 8));
+                reg_gate_dispatch<M, F2>(code, a, p.mats + (code >> 8));
             }
             if (ph == p.nph - 1 && p.direct) {
                 float2* g = const_cast<float2*>(gtile) + dgthr;
@@ -894,6 +947,20 @@ int rpass_m() {
     return m;
 }
 
+// 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
+int gate_kind(const PassDesc& pd, const PassGate& pg) {
+    const int D = 1 << pg.k;
+    const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
+    bool diag = true, cz = pg.k == 2;
+    for (int r = 0; r < D; ++r)
+        for (int c = 0; c < D; ++c) {
+            const float re = mg[2 * (r * D + c)], im = mg[2 * (r * D + c) + 1];
+            if (r != c && (re != 0.f || im != 0.f)) diag = cz = false;
+            if (r == c && (im != 0.f || re != (r == D - 1 ? -1.f : 1.f))) cz = false;
+        }
+    return cz ? 2 : diag ? 1 : 0;
+}
+
 // Phases of gates [g0, g1): each phase takes, in order, every remaining gate
 // whose positions fit in the phase's M-set and that does not touch a position
 // of a gate skipped before it (so it only moves past gates it commutes with).
@@ -907,6 +974,14 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
         for (int b = 0; b < pd.gates[g].k; ++b) m |= 1u << pd.gates[g].pos[b];
         return m;
     };
+    // CZ-like gates run in any layout (their qubits may be thread bits)
+    std::vector<char> anyl(pd.gates.size(), 0);
+    static int czfree = -1;
+    if (czfree < 0) {
+        const char* e = getenv("SVB200_RPASS_CZFREE");
+        czfree = (e && e[0] == '0') ? 0 : 1;
+    }
+    for (size_t g = g0; g < g1; ++g) anyl[g] = czfree && gate_kind(pd, pd.gates[g]) == 2;
     while (!rem.empty()) {
         RpPhaseHost ph;
         // R = the M-subset of tile positions that lets the most remaining
@@ -921,7 +996,7 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
             uint32_t blocked = 0;
             for (int g : rem) {
                 const uint32_t m = gmask(g);
-                if (!(m & blocked) && !(m & ~R)) ++cnt;
+                if (!(m & blocked) && (anyl[g] || !(m & ~R))) ++cnt;
                 else blocked |= m;
             }
             const int score = 4 * cnt + ((R & 1u) ? 2 : 0) + ((R & 0xEu) ? 0 : 1);
@@ -937,7 +1012,7 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
             std::vector<int> keep;
             for (int g : rem) {
                 const uint32_t m = gmask(g);
-                if (!(m & blocked) && !(m & ~used)) {
+                if (!(m & blocked) && (anyl[g] || !(m & ~used))) {
                     ph.gates.push_back(g);
                 } else {
                     blocked |= m;
@@ -992,20 +1067,6 @@ int phase_conflicts(const RpPhaseHost& ph, int T, int M) {
         }
     }
     return worst;
-}
-
-// 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
-int gate_kind(const PassDesc& pd, const PassGate& pg) {
-    const int D = 1 << pg.k;
-    const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
-    bool diag = true, cz = pg.k == 2;
-    for (int r = 0; r < D; ++r)
-        for (int c = 0; c < D; ++c) {
-            const float re = mg[2 * (r * D + c)], im = mg[2 * (r * D + c) + 1];
-            if (r != c && (re != 0.f || im != 0.f)) diag = cz = false;
-            if (r == c && (im != 0.f || re != (r == D - 1 ? -1.f : 1.f))) cz = false;
-        }
-    return cz ? 2 : diag ? 1 : 0;
 }
 
 template <int M, bool F2>
@@ -1084,10 +1145,13 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                     p.mats[moff + 4 * e2 + 2] = -mi;
                     p.mats[moff + 4 * e2 + 3] = mi;
                 }
-                uint32_t mask = 0;
-                for (int b = 0; b < pg.k; ++b)
-                    mask |= 1u << (int)(std::find(h.R.begin(), h.R.end(), pg.pos[b]) - h.R.begin());
-                p.gcode[li++] = mask | ((uint32_t)kind << 5) | (moff << 8);
+                uint32_t mask = 0, tmask = 0;
+                for (int b = 0; b < pg.k; ++b) {
+                    const auto it = std::find(h.R.begin(), h.R.end(), pg.pos[b]);
+                    if (it != h.R.end()) mask |= 1u << (int)(it - h.R.begin());
+                    else tmask |= 1u << (int)(std::find(h.lanes.begin(), h.lanes.end(), pg.pos[b]) - h.lanes.begin());
+                }
+                p.gcode[li++] = mask | ((uint32_t)kind << 5) | ((kind == 2 ? tmask : moff) << 8);
                 moff += 4 * ne;
             }
             P.g1 = (uint16_t)li;
@@ -1096,7 +1160,9 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
         if (dbg) {
             int w = 1;
             for (auto& x : phs) w = std::max(w, phase_conflicts(x, T, M));
-            fprintf(stderr, "rpass T=%d M=%d gates=%zu phases=%d worst_conflict=%d S=", T, M, g1 - g0, p.nph, w);
+            int nb0 = 0;
+            for (auto& x : phs) nb0 += x.b0;
+            fprintf(stderr, "rpass T=%d M=%d gates=%zu phases=%d b0=%d worst_conflict=%d S=", T, M, g1 - g0, p.nph, nb0, w);
             for (int q : pd.S) fprintf(stderr, "%d,", q);
             fprintf(stderr, "\n");
         }
