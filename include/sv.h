@@ -199,6 +199,16 @@ int sv_device_ptr(sv_state* s, int shard, void** out);
  * *need gets the required length; if cap < *need returns SV_EINVAL and
  * writes nothing to buf.  (SURVEY.md §8b / §8c-S3.) */
 int sv_fusion_plan(const sv_gate* gates, size_t n_gates, int max_fused, int32_t* buf, size_t cap, size_t* need);
+/* Cache-blocked pass plan (pure host; reading R7, §7) of the fusion
+ * plan for max_fused in [1,4] and tile_bits in [10,13], as a flat int32 stream:
+ * per pass  T, S_0..S_{T-1} (tile qubits, ascending), n, f_0..f_{n-1} (fused-
+ * gate indices of sv_fusion_plan, in pass order), n_phases, then per phase of
+ * the register-blocked kernel (0 phases when the pass has a gate with k > 2)
+ *   m, R_0..R_{m-1} (tile positions held in registers, ascending), g,
+ *   j_0..j_{g-1} (indices into the pass's f list, in application order).
+ * *need gets the length; cap < *need returns SV_EINVAL, writing nothing. */
+int sv_block_plan(const sv_gate* gates, size_t n_gates, int max_fused, int tile_bits, int32_t* buf, size_t cap,
+                  size_t* need);
 /* Fused matrix of fused gate `index` of that plan, complex128 row-major over
  * the ascending qubit list (computed in fp64). out holds 4^k entries. */
 int sv_fused_matrix(const sv_gate* gates, size_t n_gates, int max_fused, size_t index, sv_c128* out, size_t cap);

@@ -117,6 +117,7 @@ _SIGS = {
     "sv_device_ptr": ([_vp, ctypes.c_int, ctypes.POINTER(_vp)], ctypes.c_int),
     "sv_fusion_plan": ([_vp, _sz, ctypes.c_int, _i32p, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_fused_matrix": ([_vp, _sz, ctypes.c_int, _sz, _vp, _sz], ctypes.c_int),
+    "sv_block_plan": ([_vp, _sz, ctypes.c_int, ctypes.c_int, _i32p, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_shard_plan": ([_i32p, _sz, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i32p, _sz, ctypes.POINTER(_sz), _i32p],
                       ctypes.c_int),
     "sv_qubit_map": ([_vp, _i32p], ctypes.c_int),
@@ -316,6 +317,41 @@ def sv_fusion_plan(gates, max_fused: int) -> np.ndarray:
     _check(lib().sv_fusion_plan(_ptr(g), len(g), max_fused, buf.ctypes.data_as(_i32p), buf.size,
                                 ctypes.byref(need)), "sv_fusion_plan")
     return buf
+
+
+def sv_block_plan(gates, max_fused: int, tile_bits: int) -> list:
+    """Cache-blocked pass plan (pure host): a list of passes, each
+    {"S": tile qubits, "fused": fused-gate indices in pass order,
+     "phases": [(R tile positions, [indices into "fused"]), ...]}."""
+    g = as_gates(gates)
+    need = _sz()
+    rc = lib().sv_block_plan(_ptr(g), len(g), max_fused, tile_bits, None, 0, ctypes.byref(need))
+    if rc != SV_OK and need.value == 0:
+        _check(rc, "sv_block_plan")
+    buf = np.empty(need.value, dtype=np.int32)
+    _check(lib().sv_block_plan(_ptr(g), len(g), max_fused, tile_bits, buf.ctypes.data_as(_i32p), buf.size,
+                               ctypes.byref(need)), "sv_block_plan")
+    out, i = [], 0
+    b = buf.tolist()
+    while i < len(b):
+        T = b[i]
+        S = b[i + 1:i + 1 + T]
+        i += 1 + T
+        n = b[i]
+        fused = b[i + 1:i + 1 + n]
+        i += 1 + n
+        nph = b[i]
+        i += 1
+        phases = []
+        for _ in range(nph):
+            m = b[i]
+            R = b[i + 1:i + 1 + m]
+            i += 1 + m
+            ng = b[i]
+            phases.append((R, b[i + 1:i + 1 + ng]))
+            i += 1 + ng
+        out.append({"S": S, "fused": fused, "phases": phases})
+    return out
 
 
 def sv_fused_matrix(gates, max_fused: int, index: int, k: int) -> np.ndarray:

@@ -1229,6 +1229,16 @@ uint64_t rpass_fma_per_amp(const PassDesc& pd) {
     return f;
 }
 
+void rpass_phase_plan(const PassDesc& pd, std::vector<std::vector<int>>& R, std::vector<std::vector<int>>& gates) {
+    auto ph = plan_phases(pd, 0, pd.gates.size(), rpass_m());
+    R.clear();
+    gates.clear();
+    for (auto& x : ph) {
+        R.push_back(x.R);
+        gates.push_back(x.gates);
+    }
+}
+
 void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {
     const int M = rpass_m();
     auto ph = plan_phases(pd, 0, pd.gates.size(), M);

@@ -86,6 +86,7 @@ struct PassDesc {
     std::vector<float> planes;
     std::vector<float> mats;  // per gate: 2^k x 2^k complex64, row-major (re, im pairs)
     uint64_t fma_per_amp = 0;  // rpass FMAs per amplitude (stats), set at circuit creation
+    std::vector<int> src;      // index of each gate in the planner's input run (sv_block_plan)
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
@@ -100,6 +101,10 @@ cudaError_t launch_rpass(float2* psi, int n_local, const PassDesc& pd, cudaStrea
 // Host model of the rpass phase plan (tests / tools): number of phases and
 // the worst bank-conflict degree of their gathers.
 void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict);
+// The rpass phase plan of a whole pass (host; sv_block_plan): per phase its
+// register positions R (ascending tile positions) and its gates (pass-local
+// indices, in application order).
+void rpass_phase_plan(const PassDesc& pd, std::vector<std::vector<int>>& R, std::vector<std::vector<int>>& gates);
 
 // Launch one fused-gate apply on a shard of 2^n_local amplitudes.
 cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);

@@ -436,6 +436,101 @@ int upload_shard_table(sv_state* s) {
 }  // namespace
 
 // =============================================================================
+namespace {
+
+// One fused gate for build_passes: ascending local (physical) qubits and its
+// fp64 matrix over them.
+struct PassIn {
+    int k = 0;
+    int q[SV_MAX_FUSED] = {0};
+    std::vector<cd> M;
+};
+
+// Cache-blocked passes (reading R7, DESIGN.md).  Passes are formed like fused
+// gates (the S3 greedy, one level up): a pass starts at the first unplaced
+// gate and absorbs every later one whose qubits keep the pass within
+// T - kPassPinned free tile qubits, provided it does not touch a qubit of a
+// gate skipped before it (so it only moves past gates it commutes with).
+// Qubits 0..kPassPinned-1 are in every tile (runs of >= 128 B); the pass's
+// tile set S is the pinned qubits, the pass's qubits, then the lowest
+// remaining qubits (longer runs).  The state never moves: a pass only
+// chooses which amplitudes share a tile.
+std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
+    static int kPassPinned = 0;
+    if (!kPassPinned) {
+        const char* e = getenv("SVB200_PASS_PIN");
+        kPassPinned = (e && e[0] >= '1' && e[0] <= '6') ? e[0] - '0' : 4;
+    }
+    const uint64_t pin = (1ull << kPassPinned) - 1ull;
+    const int Fp = T - kPassPinned;
+    const size_t nf = in.size();
+    std::vector<uint64_t> fm(nf, 0);
+    for (size_t i = 0; i < nf; ++i)
+        for (int b = 0; b < in[i].k; ++b) fm[i] |= 1ull << in[i].q[b];
+    std::vector<char> placed(nf, 0);
+    std::vector<PassDesc> passes;
+    auto add_gate = [&](PassDesc& cur, size_t i) {
+        const PassIn& f = in[i];
+        const int D = 1 << f.k;
+        PassGate pg{};
+        pg.k = f.k;
+        for (int b = 0; b < f.k; ++b) pg.pos[b] = (int)(std::find(cur.S.begin(), cur.S.end(), f.q[b]) - cur.S.begin());
+        pg.poff = (uint32_t)cur.planes.size();
+        pg.moff = (uint32_t)cur.mats.size();
+        for (int e = 0; e < D * D; ++e) {
+            cur.mats.push_back((float)f.M[e].real());
+            cur.mats.push_back((float)f.M[e].imag());
+        }
+        std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
+        for (int e = 0; e < D * D; ++e) {
+            const float re = (float)f.M[e].real(), im = (float)f.M[e].imag();
+            Pp[e] = re;
+            Sp[e] = re + im;
+            Qp[e] = im - re;
+        }
+        cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
+        cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
+        cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
+        cur.gates.push_back(pg);
+    };
+    for (size_t i = 0; i < nf; ++i) {
+        if (placed[i]) continue;
+        std::vector<size_t> mem{i};
+        placed[i] = 1;
+        uint64_t Q = fm[i], B = 0;
+        size_t planes = 3ull << (2 * in[i].k);
+        for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
+            if (placed[j]) continue;
+            const uint64_t Sj = fm[j];
+            const size_t pj = 3ull << (2 * in[j].k);
+            if (Sj & B) {
+                B |= Sj;
+            } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
+                Q |= Sj;
+                planes += pj;
+                mem.push_back(j);
+                placed[j] = 1;
+            } else {
+                B |= Sj;
+            }
+        }
+        uint64_t tile = Q | pin;
+        for (int q = 0; q < 64 && __builtin_popcountll(tile) < T; ++q) tile |= 1ull << q;
+        PassDesc cur;
+        for (int q = 0; q < 64; ++q)
+            if ((tile >> q) & 1ull) cur.S.push_back(q);
+        plan_pass_tile(cur);
+        for (size_t j : mem) {
+            add_gate(cur, j);
+            cur.src.push_back((int)j);
+        }
+        passes.push_back(std::move(cur));
+    }
+    return passes;
+}
+
+}  // namespace
+
 extern "C" {
 
 const char* sv_last_error(void) { return g_err.c_str(); }
@@ -731,6 +826,47 @@ int sv_fusion_plan(const sv_gate* gates, size_t n_gates, int max_fused, int32_t*
     return SV_OK;
 }
 
+int sv_block_plan(const sv_gate* gates, size_t n_gates, int max_fused, int tile_bits, int32_t* buf, size_t cap,
+                  size_t* need) {
+    if (!need) return fail(SV_EINVAL, "need is NULL");
+    if (max_fused < 1 || max_fused > 4) return fail(SV_EINVAL, "max_fused must be in [1, 4] for blocked passes");
+    if (tile_bits < 10 || tile_bits > 13) return fail(SV_EINVAL, "tile_bits must be in [10, 13]");
+    int rc = validate_gates(gates, n_gates, -1);
+    if (rc) return rc;
+    std::vector<FusedGate> plan;
+    fuse_plan(gates, n_gates, max_fused, plan);
+    std::vector<PassIn> in;
+    for (auto& f : plan) {
+        build_fused_matrix(gates, f);
+        PassIn pi;
+        pi.k = f.k;
+        for (int b = 0; b < f.k; ++b) pi.q[b] = f.q[b];
+        pi.M = f.M;
+        in.push_back(std::move(pi));
+    }
+    std::vector<int32_t> o;
+    for (auto& pd : build_passes(tile_bits, in)) {
+        o.push_back((int32_t)pd.S.size());
+        for (int q : pd.S) o.push_back(q);
+        o.push_back((int32_t)pd.src.size());
+        for (int j : pd.src) o.push_back(j);
+        std::vector<std::vector<int>> R, G;
+        if (rpass_supported(pd)) rpass_phase_plan(pd, R, G);
+        o.push_back((int32_t)R.size());
+        for (size_t i = 0; i < R.size(); ++i) {
+            o.push_back((int32_t)R[i].size());
+            for (int r : R[i]) o.push_back(r);
+            o.push_back((int32_t)G[i].size());
+            for (int g : G[i]) o.push_back(g);
+        }
+    }
+    *need = o.size();
+    if (cap < o.size()) return fail(SV_EINVAL, "cap too small");
+    if (!o.empty() && !buf) return fail(SV_EINVAL, "buf is NULL");
+    std::copy(o.begin(), o.end(), buf);
+    return SV_OK;
+}
+
 int sv_fused_matrix(const sv_gate* gates, size_t n_gates, int max_fused, size_t index, sv_c128* out, size_t cap) {
     if (max_fused < 0 || max_fused > SV_MAX_FUSED) return fail(SV_EINVAL, "max_fused must be in [0, 6]");
     int rc = validate_gates(gates, n_gates, -1);
@@ -798,94 +934,6 @@ int sv_shard_plan(const int32_t* fs, size_t len, int n, int g, int vmin, int32_t
     if (final_pos)
         for (int q = 0; q < n; ++q) final_pos[q] = pos[q];
     return SV_OK;
-}
-
-// One fused gate for build_passes: ascending local (physical) qubits and its
-// fp64 matrix over them.
-struct PassIn {
-    int k = 0;
-    int q[SV_MAX_FUSED] = {0};
-    std::vector<cd> M;
-};
-
-// Cache-blocked passes (reading R7, DESIGN.md).  Passes are formed like fused
-// gates (the S3 greedy, one level up): a pass starts at the first unplaced
-// gate and absorbs every later one whose qubits keep the pass within
-// T - kPassPinned free tile qubits, provided it does not touch a qubit of a
-// gate skipped before it (so it only moves past gates it commutes with).
-// Qubits 0..kPassPinned-1 are in every tile (runs of >= 128 B); the pass's
-// tile set S is the pinned qubits, the pass's qubits, then the lowest
-// remaining qubits (longer runs).  The state never moves: a pass only
-// chooses which amplitudes share a tile.
-std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
-    static int kPassPinned = 0;
-    if (!kPassPinned) {
-        const char* e = getenv("SVB200_PASS_PIN");
-        kPassPinned = (e && e[0] >= '1' && e[0] <= '6') ? e[0] - '0' : 4;
-    }
-    const uint64_t pin = (1ull << kPassPinned) - 1ull;
-    const int Fp = T - kPassPinned;
-    const size_t nf = in.size();
-    std::vector<uint64_t> fm(nf, 0);
-    for (size_t i = 0; i < nf; ++i)
-        for (int b = 0; b < in[i].k; ++b) fm[i] |= 1ull << in[i].q[b];
-    std::vector<char> placed(nf, 0);
-    std::vector<PassDesc> passes;
-    auto add_gate = [&](PassDesc& cur, size_t i) {
-        const PassIn& f = in[i];
-        const int D = 1 << f.k;
-        PassGate pg{};
-        pg.k = f.k;
-        for (int b = 0; b < f.k; ++b) pg.pos[b] = (int)(std::find(cur.S.begin(), cur.S.end(), f.q[b]) - cur.S.begin());
-        pg.poff = (uint32_t)cur.planes.size();
-        pg.moff = (uint32_t)cur.mats.size();
-        for (int e = 0; e < D * D; ++e) {
-            cur.mats.push_back((float)f.M[e].real());
-            cur.mats.push_back((float)f.M[e].imag());
-        }
-        std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
-        for (int e = 0; e < D * D; ++e) {
-            const float re = (float)f.M[e].real(), im = (float)f.M[e].imag();
-            Pp[e] = re;
-            Sp[e] = re + im;
-            Qp[e] = im - re;
-        }
-        cur.planes.insert(cur.planes.end(), Pp.begin(), Pp.end());
-        cur.planes.insert(cur.planes.end(), Sp.begin(), Sp.end());
-        cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
-        cur.gates.push_back(pg);
-    };
-    for (size_t i = 0; i < nf; ++i) {
-        if (placed[i]) continue;
-        std::vector<size_t> mem{i};
-        placed[i] = 1;
-        uint64_t Q = fm[i], B = 0;
-        size_t planes = 3ull << (2 * in[i].k);
-        for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
-            if (placed[j]) continue;
-            const uint64_t Sj = fm[j];
-            const size_t pj = 3ull << (2 * in[j].k);
-            if (Sj & B) {
-                B |= Sj;
-            } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
-                Q |= Sj;
-                planes += pj;
-                mem.push_back(j);
-                placed[j] = 1;
-            } else {
-                B |= Sj;
-            }
-        }
-        uint64_t tile = Q | pin;
-        for (int q = 0; q < 64 && __builtin_popcountll(tile) < T; ++q) tile |= 1ull << q;
-        PassDesc cur;
-        for (int q = 0; q < 64; ++q)
-            if ((tile >> q) & 1ull) cur.S.push_back(q);
-        plan_pass_tile(cur);
-        for (size_t j : mem) add_gate(cur, j);
-        passes.push_back(std::move(cur));
-    }
-    return passes;
 }
 
 int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out) {
