@@ -259,7 +259,7 @@ struct alignas(16) RpassParams {
     // (16 B pairs; tile bit 0 in registers, tile bits 1..3 on lanes 0..2 so
     // each quarter-warp writes one 128 B run) instead of through the tile
     int direct;
-    uint64_t dgoff[16];   // amplitude offset of register pair j
+    uint64_t dgoff[32];   // amplitude offset of register pair j (16 B) / register j (8 B layout)
     uint64_t dgtbw[10];   // amplitude offset of thread-index bit i
     // direct load: the first phase reads its registers straight from HBM
     // (same layout condition; one tile buffer only) instead of via the tile
@@ -280,6 +280,9 @@ __host__ __device__ constexpr int pdep5(int v, int mask) {
 }
 __host__ __device__ constexpr int popc5(int m) { return (m & 1) + ((m >> 1) & 1) + ((m >> 2) & 1) + ((m >> 3) & 1) + ((m >> 4) & 1); }
 
+__device__ __forceinline__ void st_stream2(float2* p, float2 v) {
+    asm volatile("st.global.cs.v2.f32 [%0], {%1,%2};" ::"l"(p), "f"(v.x), "f"(v.y) : "memory");
+}
 __device__ __forceinline__ float4 ld_stream(const float4* p) {
     float4 v;
     asm volatile("ld.global.cs.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
@@ -821,10 +824,16 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             }
             if (ph == p.nph - 1 && p.direct) {
                 float2* g = const_cast<float2*>(gtile) + dgthr;
+                if (P.b0) {
 #pragma unroll
-                for (int j = 0; j < NA / 2; ++j)
-                    st_stream(reinterpret_cast<float4*>(g + p.dgoff[j]),
-                              make_float4(a[2 * j].x, a[2 * j].y, a[2 * j + 1].x, a[2 * j + 1].y));
+                    for (int j = 0; j < NA / 2; ++j)
+                        st_stream(reinterpret_cast<float4*>(g + p.dgoff[j]),
+                                  make_float4(a[2 * j].x, a[2 * j].y, a[2 * j + 1].x, a[2 * j + 1].y));
+                } else {
+                    // tile bits 0..3 on lanes 0..3: each half-warp writes one 128 B run
+#pragma unroll
+                    for (int j = 0; j < NA; ++j) st_stream2(g + p.dgoff[j], a[j]);
+                }
                 break;  // the next iteration's first barrier guards `cur`
             }
             if (P.b0) {
@@ -1175,10 +1184,17 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             auto coalesced = [](const RpPhaseHost& h) {
                 return h.b0 && h.lanes.size() >= 3 && h.lanes[0] == 1 && h.lanes[1] == 2 && h.lanes[2] == 3;
             };
+            auto coalesced8 = [](const RpPhaseHost& h) {
+                return !h.b0 && h.lanes.size() >= 4 && h.lanes[0] == 0 && h.lanes[1] == 1 && h.lanes[2] == 2 &&
+                       h.lanes[3] == 3;
+            };
             const RpPhaseHost& lp = phs.back();
-            p.direct = denv && coalesced(lp);
+            p.direct = denv && (coalesced(lp) || coalesced8(lp));
             if (p.direct) {
-                for (int j = 0; j < (1 << (M - 1)); ++j) p.dgoff[j] = dep(deposit(2u * j, lp.R));
+                if (lp.b0)
+                    for (int j = 0; j < (1 << (M - 1)); ++j) p.dgoff[j] = dep(deposit(2u * j, lp.R));
+                else
+                    for (int j = 0; j < (1 << M); ++j) p.dgoff[j] = dep(deposit((uint32_t)j, lp.R));
                 for (int b = 0; b < p.tbits; ++b) p.dgtbw[b] = dep(1ull << lp.lanes[b]);
             }
             const RpPhaseHost& fp = phs.front();
