@@ -200,11 +200,19 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    # one rank per GPU; more ranks than GPUs (functional checks of the sharded
+    # path on a small box) share devices round-robin
+    dev = local % max(torch.cuda.device_count(), 1)
+    torch.cuda.set_device(dev)
     dist = None
+    cdev = "cuda"  # device of the small tensors the collectives carry
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        shared = world > torch.cuda.device_count()
+        # NCCL refuses two ranks on one device: gloo carries the (tiny) control
+        # traffic then; the data path is our own P2P kernel either way
+        dist.init_process_group("gloo" if shared else "nccl", **({} if shared else {"device_id": torch.device("cuda", dev)}))
+        cdev = "cpu" if shared else "cuda"
     n = args.qubits or (30 if world == 1 else 30 + (world.bit_length() - 1))
     gates = W.rqc(n, args.depth, args.seed)
     stream = torch.cuda.Stream()
@@ -253,7 +261,7 @@ def run_ours(args):
             sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
             sv.sv_circuit_destroy(c)
     if args.max_fused < 0:
-        best = torch.tensor([int(min(sweep, key=sweep.get)) if sweep else 4], device="cuda")
+        best = torch.tensor([int(min(sweep, key=sweep.get)) if sweep else 4], device=cdev)
         if dist is not None:  # every rank runs rank 0's choice (collective calls)
             dist.broadcast(best, 0)
         args.max_fused = int(best.item())
@@ -282,7 +290,7 @@ def run_ours(args):
     flops = 0
     bytes_exch = 0
     fma = 0
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev) as clk:
         start = torch.cuda.Event(enable_timing=True)
         end = torch.cuda.Event(enable_timing=True)
         barrier()
@@ -308,7 +316,7 @@ def run_ours(args):
     # the per-step sv_last_stats sync adds a host round trip per step; report
     # the device-side sum of our launches as well
     t_apply = t_high + t_low
-    ms_t = torch.tensor([ms], device="cuda")
+    ms_t = torch.tensor([ms], device=cdev)
     if dist is not None:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms = float(ms_t.item())
@@ -334,7 +342,7 @@ def run_ours(args):
     e1.record(stream)
     barrier()
     e2e_ms = e0.elapsed_time(e1) / e2e_steps
-    et = torch.tensor([e2e_ms], device="cuda")
+    et = torch.tensor([e2e_ms], device=cdev)
     if dist is not None:
         dist.all_reduce(et, op=dist.ReduceOp.MAX)
     e2e_ms = float(et.item())
