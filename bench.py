@@ -180,8 +180,8 @@ def run_reference(args):
         last = cpu_oracle_sample(n, gates, args.cpu_seconds)
         vals.append(last["value"])
     v = statistics.mean(vals)
-    cfg = {"workload": f"rqc_{n}q_d{args.depth}_f{args.max_fused}", "n_qubits": n, "depth": args.depth,
-           "max_fused": args.max_fused, "seed": args.seed}
+    cfg = {"workload": f"rqc_{n}q_d{args.depth}", "n_qubits": n, "depth": args.depth,
+           "max_fused": "none (the oracle applies the gates unfused)", "seed": args.seed}
     last["value"] = v
     out = {"impl": "reference", "metric": f"rqc_circuit_time_{n}q_d{args.depth}", "value": v, "unit": "s",
            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": v * 1e3,
@@ -377,7 +377,7 @@ def run_ours(args):
             "dtype": "f64" if fp64 else "f32",
             "data": "synthetic",
             "config": {
-                "workload": f"rqc_{n}q_d{args.depth}_f{args.max_fused}",
+                "workload": f"rqc_{n}q_d{args.depth}",
                 "n_qubits": n, "depth": args.depth, "max_fused": args.max_fused, "fusion": fusion_choice,
                 "execution": ("register-blocked passes (apply_rpass), tile qubits "
                               f"{cst.get('block_bits', 12)}" if cst.get("n_passes", 0) else "one launch per fused gate"),
