@@ -107,15 +107,18 @@ def test_30q_sampling_bit_exact():
     assert np.array_equal(np.asarray(got, dtype=np.uint64), ref)
 
 
-def test_34q_d20_norm_and_inverse_roundtrip():
+@pytest.mark.parametrize("F", [1, 5])
+def test_34q_d20_norm_and_inverse_roundtrip(F):
+    """F = 1: register-blocked passes (the default); F = 5: int8 tensor cores."""
     n, depth = 34, 20
     if _gpu_free_gb() < 132:
         pytest.skip("needs a 128 GiB state in HBM")
     gates = W.rqc(n, depth, 2023)
     h = sv.sv_create(n)
     try:
-        c = sv.sv_circuit_create(h, gates, 5)
-        ci = sv.sv_circuit_create(h, W.inverse_circuit(gates), 5)
+        c = sv.sv_circuit_create(h, gates, F)
+        ci = sv.sv_circuit_create(h, W.inverse_circuit(gates), F)
+        assert (sv.sv_circuit_stats(c)["n_passes"] > 0) == (F <= 2)
         sv.sv_reset(h)
         sv.sv_circuit_run_device(h, c)
         # norm of the forward state from 2^20 sampled amplitudes (uniform indices)
@@ -125,7 +128,7 @@ def test_34q_d20_norm_and_inverse_roundtrip():
         assert abs(est - 1) < 0.01, est  # Porter-Thomas: relative std of the estimate ~ 2^-10
         sv.sv_circuit_run_device(h, ci)
         a0 = sv.sv_amplitudes(h, np.array([0], dtype=np.uint64))[0]
-        print(f"FULLSIZE 34q d20 F=5: norm estimate {est:.5f}, |<0|U^-1 U|0>|^2 - 1 = {abs(complex(a0)) ** 2 - 1:.3e}")
+        print(f"FULLSIZE 34q d20 F={F}: norm estimate {est:.5f}, |<0|U^-1 U|0>|^2 - 1 = {abs(complex(a0)) ** 2 - 1:.3e}")
         # two circuits of the north-star per-depth bound each
         assert abs(abs(complex(a0)) ** 2 - 1) <= 2e-5, a0
         sv.sv_circuit_destroy(c)
