@@ -11,7 +11,10 @@
  *     product) up to a "maximum of fused gates" (L98-104, Fig. 5);
  *   - gates on high qubits and on low qubits run in different kernels
  *     (L110-112, §2.3);
- *   - amplitudes can be read and measurement outcomes sampled (L131-132, §3).
+ *   - amplitudes can be read and measurement outcomes sampled (L131-132, §3);
+ *   - several fused gates can share one pass over the state (cache blocking,
+ *     related work [12], L221): the default for max_fused <= 2
+ *     (sv_set_blocking, sv_block_plan).
  *
  * Conventions (SURVEY.md §8c readings Q1/Q3):
  *   - qubit q is bit q of the basis index (little-endian, qubit 0 = stride 1);
