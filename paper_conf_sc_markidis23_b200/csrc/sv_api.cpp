@@ -59,7 +59,7 @@ struct sv_state {
     bool virt = true;         // all shards on this GPU
     int device = 0;
     int vmin = 5;
-    int block_bits = -1;      // cache-blocked passes: tile qubits (0 = off, -1 = auto: 12 when max_fused <= 2)
+    int block_bits = -1;      // cache-blocked passes: tile qubits (0 = off, -1 = auto, see sv_circuit_create)
     bool fp64 = false;        // complex128 amplitudes (NEXT-1)
     size_t elem = 8;          // bytes per amplitude
     double* planes64 = nullptr;   // fp64 scratch: planes of one gate (sv_apply_fused on fp64 states)
@@ -978,7 +978,9 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     // Cache-blocked passes (complex64, large shards, k <= 4; sharded or not):
     // each maximal run of APPLY events between exchanges is cut into passes
     // by build_passes (reading R7); exchanges and permutations stay as they are.
-    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? 12 : 0);
+    // auto tile: 12 qubits; 13 for shards of >= 2^33 amplitudes (34q D20:
+    // 1.91 s vs 1.98 s; 32q equal; 30q 0.078 s vs 0.080 s at T = 12)
+    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? (s->l >= 33 ? 13 : 12) : 0);
     const bool blocked = !s->fp64 && T >= 10 && s->l >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
                          max_fused >= 1;
     const double t2 = now_s();
