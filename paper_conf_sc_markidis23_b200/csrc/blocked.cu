@@ -3,14 +3,20 @@
 // Related work [12] applies several gates per memory pass;
 // the paper's own smem remedy (L94-96) keeps a block of the state on chip.
 // A pass loads a tile -- the 2^T amplitudes that share every bit outside a
-// qubit set S (|S| = T, S contains the low qubits 0..4 so runs stay >= 256 B)
-// -- into shared memory, applies EVERY fused gate of the pass (all their
-// qubits are in S) one after another inside the tile, and writes it back:
-// one HBM read + write for many gates.  The sequence of qubit sets comes from
-// the S4 planner run with "local" = the tile's T slots (planner.cpp); a
-// "remap" is only a change of S for the next pass -- the state never moves.
-// Per gate the group transform is the one of apply.cu (gather the 2^k
-// members, Gauss 3-multiplication y = M a, scatter).
+// qubit set S (|S| = T, S contains qubits 0..3 so runs stay >= 128 B) -- applies
+// EVERY fused gate of the pass (all their qubits are in S) inside the tile,
+// and writes it back: one HBM read + write for many gates.  Passes are formed
+// on the host (build_passes in sv_api.cpp, reading R7); the state
+// never moves -- a pass only chooses which amplitudes share a tile.
+//
+// Two kernels:
+//  * apply_rpass (default, gates with k <= 2): the gates of a pass run in
+//    register phases -- each thread holds 32 amplitudes of the tile in
+//    registers and applies every gate whose qubits lie in the phase's 5 tile
+//    positions (plus CZ-like gates anywhere), one shared-memory exchange and
+//    barrier per phase;
+//  * apply_pass (k = 3, 4; opt-in): one sweep of the shared-memory tile per
+//    gate (gather the 2^k members, Gauss 3-multiplication y = M a, scatter).
 #include <cuda_runtime.h>
 
 #include <algorithm>
