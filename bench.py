@@ -346,7 +346,11 @@ def run_ours(args):
     if dist is not None:
         dist.all_reduce(et, op=dist.ReduceOp.MAX)
     e2e_ms = float(et.item())
-    h2d = int(sum(8 * (1 << (2 * k)) * c for k, c in enumerate(cst["fused_hist"])))
+    # host -> device per e2e step: the step's input is the gate list (sv_gate
+    # records with fp64 matrices) the library fuses on the host; what crosses
+    # to the device is the fused matrices (kernel parameters / one upload),
+    # counted as complex64 2^k x 2^k per fused gate; the larger of the two
+    h2d = int(max(g_arr.nbytes, sum(8 * (1 << (2 * k)) * c for k, c in enumerate(cst["fused_hist"]))))
 
     peak, peak_src = load_peaks()
     launches_apply = n_high + n_low
