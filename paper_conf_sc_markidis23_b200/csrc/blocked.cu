@@ -270,6 +270,7 @@ struct alignas(16) RpassParams {
     // direct load: the first phase reads its registers straight from HBM
     // (same layout condition; one tile buffer only) instead of via the tile
     int dload;
+    int early;  // direct store: issue the next tile's load before the last phase's gates
     uint64_t lgoff[16];
     uint64_t lgtbw[10];
     RpPhase ph[kRpMaxPhases];
@@ -824,6 +825,16 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
 #pragma unroll
                 for (int j = 0; j < NA; ++j) a[j] = lds2(cur + (tb ^ P.roff[j]));
             }
+            const bool early = SVB_RP_STAGES == 1 && ph == p.nph - 1 && p.direct && !p.dload && p.early;
+            if (early) {
+                // the last phase keeps its amplitudes in registers and stores
+                // them straight to HBM: once every thread has gathered, the
+                // tile buffer is free -- start the next tile's load now so it
+                // overlaps this phase's gates
+                __syncthreads();
+                if (gnext) load(gnext, cur);
+                cp_async_commit();
+            }
             for (int gi = P.g0; gi < P.g1; ++gi) {
                 const uint32_t code = p.gcode[gi];
                 reg_gate_dispatch<M, F2>(code, a, p.mats + (code >> 8));
@@ -854,7 +865,7 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
         }
         if (!p.direct) store(const_cast<float2*>(gcur), cur);
         if constexpr (SVB_RP_STAGES == 1) {
-            if (!p.dload) {
+            if (!p.dload && !(p.direct && p.early)) {
                 __syncthreads();  // every thread is done with the tile buffer
                 if (gnext) load(gnext, cur);
                 cp_async_commit();
@@ -1212,6 +1223,12 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                 lenv = (e && e[0] == '1') ? 1 : 0;
             }
             p.dload = lenv && SVB_RP_STAGES == 1 && coalesced(fp);
+            static int eenv = -1;
+            if (eenv < 0) {
+                const char* e = getenv("SVB200_RPASS_EARLY");
+                eenv = (e && e[0] == '0') ? 0 : 1;
+            }
+            p.early = eenv;
             if (p.dload) {
                 for (int j = 0; j < (1 << (M - 1)); ++j) p.lgoff[j] = dep(deposit(2u * j, fp.R));
                 for (int b = 0; b < p.tbits; ++b) p.lgtbw[b] = dep(1ull << fp.lanes[b]);
