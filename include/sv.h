@@ -239,8 +239,7 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each);
  * register-blocked kernel (32 amplitudes per thread, gates applied in
  * registers); others in the shared-memory pass kernel.
  * tile_bits in [10,13]; 0 disables (one launch per fused gate); -1 (default)
- * = auto: 12 when max_fused <= 2 and the shard has >= 20 qubits (13 from 33
- * qubits on), else off.  Takes effect for
+ * = auto: 13 when max_fused <= 2 and the shard has >= 20 qubits, else off.  Takes effect for
  * circuits created afterwards.  Errors: SV_EINVAL for other values. */
 int sv_set_blocking(sv_state* s, int tile_bits);
 /* 1: record CUDA events around every launch and fill the *_dev_s stats. */

@@ -978,9 +978,9 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     // Cache-blocked passes (complex64, large shards, k <= 4; sharded or not):
     // each maximal run of APPLY events between exchanges is cut into passes
     // by build_passes (reading R7); exchanges and permutations stay as they are.
-    // auto tile: 12 qubits; 13 for shards of >= 2^33 amplitudes (34q D20:
-    // 1.91 s vs 1.98 s; 32q equal; 30q 0.078 s vs 0.080 s at T = 12)
-    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? (s->l >= 33 ? 13 : 12) : 0);
+    // auto tile: 13 qubits (with the early next-tile load of apply_rpass:
+    // 30q D14 F=1 0.0745 s vs 0.0775 s at 12; 32q D20 0.430 vs 0.462 s)
+    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? 13 : 0);
     const bool blocked = !s->fp64 && T >= 10 && s->l >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
                          max_fused >= 1;
     const double t2 = now_s();

@@ -75,7 +75,7 @@ def ref30():
 @pytest.mark.parametrize("F,kmax", [(1, 2), (2, 2), (4, 4), (5, 5), (6, 6)])
 def test_30q_d14_state_vs_oracle(ref30, F, kmax):
     """F = 1, 2: register-blocked passes (the library default for
-    max_fused <= 2, tile qubits 12); F >= 4: one launch per fused gate."""
+    max_fused <= 2, tile qubits 13); F >= 4: one launch per fused gate."""
     n, depth = 30, 14
     gates = W.rqc(n, depth, 2023)
     h, st = _run_prepared(n, gates, F)
