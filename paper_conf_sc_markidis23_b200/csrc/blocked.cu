@@ -271,6 +271,8 @@ struct alignas(16) RpassParams {
     // (same layout condition; one tile buffer only) instead of via the tile
     int dload;
     int early;  // direct store: issue the next tile's load before the last phase's gates
+    int zinit;  // the state is |0...0>: nothing is loaded, phase 0 starts from zeros
+    int zone;   // ... and this shard holds amplitude 0 (= 1, tile 0, thread 0, register 0)
     uint64_t lgoff[16];
     uint64_t lgtbw[10];
     RpPhase ph[kRpMaxPhases];
@@ -778,7 +780,7 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
     if (u < p.n_tiles) {
         gtile = p.psi + tbase(u);
         gcur = gtile + dthr;
-        if (!p.dload) load(gcur, s0);
+        if (!p.dload && !p.zinit) load(gcur, s0);
     }
     cp_async_commit();
     for (int it = 0; u < p.n_tiles; u += gridDim.x, ++it) {
@@ -806,7 +808,11 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             for (int i = 0; i < p.tbits; ++i)
                 if ((threadIdx.x >> i) & 1u) tb ^= P.tbw[i];
             float2 a[NA];
-            if (ph == 0 && p.dload) {
+            if (ph == 0 && p.zinit) {
+#pragma unroll
+                for (int j = 0; j < NA; ++j) a[j] = make_float2(0.f, 0.f);
+                if (p.zone && u == 0 && threadIdx.x == 0) a[0].x = 1.f;
+            } else if (ph == 0 && p.dload) {
                 const float2* g = gtile + lgthr;
 #pragma unroll
                 for (int j = 0; j < NA / 2; ++j) {
@@ -825,7 +831,7 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
 #pragma unroll
                 for (int j = 0; j < NA; ++j) a[j] = lds2(cur + (tb ^ P.roff[j]));
             }
-            const bool early = SVB_RP_STAGES == 1 && ph == p.nph - 1 && p.direct && !p.dload && p.early;
+            const bool early = SVB_RP_STAGES == 1 && ph == p.nph - 1 && p.direct && !p.dload && !p.zinit && p.early;
             if (early) {
                 // the last phase keeps its amplitudes in registers and stores
                 // them straight to HBM: once every thread has gathered, the
@@ -865,7 +871,7 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
         }
         if (!p.direct) store(const_cast<float2*>(gcur), cur);
         if constexpr (SVB_RP_STAGES == 1) {
-            if (!p.dload && !(p.direct && p.early)) {
+            if (!p.dload && !p.zinit && !(p.direct && p.early)) {
                 __syncthreads();  // every thread is done with the tile buffer
                 if (gnext) load(gnext, cur);
                 cp_async_commit();
@@ -1096,7 +1102,7 @@ int phase_conflicts(const RpPhaseHost& ph, int T, int M) {
 }
 
 template <int M, bool F2>
-cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st) {
+cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone) {
     const int T = (int)pd.S.size();
     const uint32_t nthr = 1u << (T - M);
     const size_t smem = SVB_RP_STAGES * ((size_t)8 << T);
@@ -1229,6 +1235,8 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                 eenv = (e && e[0] == '0') ? 0 : 1;
             }
             p.early = eenv;
+            p.zinit = zinit && g0 == 0;  // only the first launch of a split pass starts from |0...0>
+            p.zone = zone ? 1 : 0;
             if (p.dload) {
                 for (int j = 0; j < (1 << (M - 1)); ++j) p.lgoff[j] = dep(deposit(2u * j, fp.R));
                 for (int b = 0; b < p.tbits; ++b) p.lgtbw[b] = dep(1ull << fp.lanes[b]);
@@ -1287,15 +1295,15 @@ void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {
     if (worst_conflict) *worst_conflict = w;
 }
 
-cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st) {
+cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone) {
     static_assert(sizeof(RpassParams) <= 32764, "rpass params exceed the kernel parameter space");
     static int f2 = -1;
     if (f2 < 0) {
         const char* e = getenv("SVB200_RPASS_F2");
         f2 = (e && e[0] == '0') ? 0 : 1;
     }
-    if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st) : launch_rpass_m<5, false>(psi, n, pd, st);
-    return f2 ? launch_rpass_m<4, true>(psi, n, pd, st) : launch_rpass_m<4, false>(psi, n, pd, st);
+    if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st, zinit, zone) : launch_rpass_m<5, false>(psi, n, pd, st, zinit, zone);
+    return f2 ? launch_rpass_m<4, true>(psi, n, pd, st, zinit, zone) : launch_rpass_m<4, false>(psi, n, pd, st, zinit, zone);
 }
 
 }  // namespace svb

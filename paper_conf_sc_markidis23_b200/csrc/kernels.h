@@ -97,7 +97,10 @@ bool rpass_supported(const PassDesc& pd);
 // fp32 FMAs per amplitude the rpass kernel executes for this pass (dense
 // 2^k x 2^k: 4 * 2^k, diagonal: 4, CZ-like: 0)
 uint64_t rpass_fma_per_amp(const PassDesc& pd);
-cudaError_t launch_rpass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
+// zero_init: the tiles are |0...0> (not loaded); one_here: this shard holds
+// amplitude 0 (= 1)
+cudaError_t launch_rpass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st, bool zero_init = false,
+                         bool one_here = false);
 // Host model of the rpass phase plan (tests / tools): number of phases and
 // the worst bank-conflict degree of their gathers.
 void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict);

@@ -72,6 +72,10 @@ struct sv_state {
     void* alloc = nullptr;             // library-owned state allocation
     std::vector<int> pos;              // logical -> physical
     int sticky = SV_OK;
+    // |0...0> requested by sv_reset but not yet written (complex64): the next
+    // circuit whose first step is a register-blocked pass synthesises the
+    // zero tiles instead of loading them; any other access writes it first
+    bool zero_pending = false;
     // scratch
     uint64_t* bins = nullptr;          // world_local * n_bins
     uint64_t* scan_scratch = nullptr;
@@ -636,10 +640,28 @@ int sv_destroy(sv_state* s) {
     return SV_OK;
 }
 
+static int write_zero_state(sv_state* s);
+
 int sv_reset(sv_state* s) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
     if (s->sticky) return fail(SV_EBADSTATE, "state poisoned by an earlier device failure");
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
+    if (!s->fp64) {
+        s->zero_pending = true;  // written lazily (see sv_state::zero_pending)
+        return SV_OK;
+    }
+    return write_zero_state(s);
+}
+
+// materialise a pending |0...0> (every entry point that reads or writes the
+// state calls this first, except sv_circuit_run_device's fused path)
+static int materialize(sv_state* s) {
+    if (!s->zero_pending) return SV_OK;
+    s->zero_pending = false;
+    return write_zero_state(s);
+}
+
+static int write_zero_state(sv_state* s) {
     for (int d = 0; d < s->local_shards(); ++d) {
         const int shard = s->virt ? d : s->rank;
         float2* psi = s->shard[shard];
@@ -677,6 +699,10 @@ int sv_apply_fused_c128(sv_state* s, int k, const int32_t* qubits, const sv_c128
 }
 
 static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::vector<cd>& Min) {
+    {
+        const int rz = materialize(s);
+        if (rz) return rz;
+    }
     int rc = SV_OK;
     uint64_t mask = 0;
     for (int b = 0; b < k; ++b) {
@@ -748,6 +774,8 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
 int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k, const int32_t* targets,
                         const sv_c64* matrix) {
     int rc = check_state(s);
+    if (rc) return rc;
+    rc = materialize(s);
     if (rc) return rc;
     if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
     if (n_ctrl < 0 || n_ctrl > SV_MAX_FUSED) return fail(SV_EINVAL, "n_ctrl must be in [0, 6]");
@@ -1144,6 +1172,18 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     s->stats.t_upload_s = keep.t_upload_s;
     s->stats.n_fused = keep.n_fused;
     for (int k = 0; k < 7; ++k) s->stats.fused_hist[k] = keep.fused_hist[k];
+    // a pending |0...0> is synthesised inside the first pass when the circuit
+    // starts with a register-blocked pass (no reset write, no first-pass read)
+    bool zinit = false;
+    if (s->zero_pending) {
+        zinit = !c->small && !s->fp64 && !c->steps.empty() && c->steps[0].block && rpass_supported(c->steps[0].pass);
+        if (zinit) {
+            s->zero_pending = false;
+        } else {
+            rc = materialize(s);
+            if (rc) return rc;
+        }
+    }
     if (c->small) {
         if (c->n_small > 0) {
             rc = launch(s, LaunchClass::HIGH, [&] {
@@ -1173,9 +1213,11 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     for (auto& st : c->steps) {
         if (st.block) {
             for (int sh = 0; sh < s->local_shards(); ++sh) {
-                float2* psi = s->virt ? s->shard[sh] : s->shard[s->rank];
+                const int shard = s->virt ? sh : s->rank;
+                float2* psi = s->shard[shard];
+                const bool z = zinit && &st == &c->steps[0];
                 rc = launch(s, LaunchClass::HIGH, [&] {
-                    return rpass_supported(st.pass) ? launch_rpass(psi, s->l, st.pass, s->stream)
+                    return rpass_supported(st.pass) ? launch_rpass(psi, s->l, st.pass, s->stream, z, shard == 0)
                                                     : launch_pass(psi, s->l, st.pass, s->stream);
                 });
                 if (rc) return rc;
@@ -1241,6 +1283,10 @@ int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fu
 // ---- amplitudes ----------------------------------------------------------------
 // complex128 states (single shard): gather into double2, D2H
 static int amplitudes64(sv_state* s, const uint64_t* idx, size_t count, sv_c128* out) {
+    {
+        const int rz = materialize(s);
+        if (rz) return rz;
+    }
     const uint64_t dim = 1ull << s->n;
     for (size_t i = 0; i < count; ++i)
         if (idx[i] >= dim) return fail(SV_EINVAL, "amplitude index out of range");
@@ -1273,6 +1319,8 @@ int sv_amplitudes_c128(sv_state* s, const uint64_t* idx, size_t count, sv_c128* 
 
 int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
     int rc = check_state(s);
+    if (rc) return rc;
+    rc = materialize(s);
     if (rc) return rc;
     if (count == 0) return SV_OK;
     if (!idx || !out) return fail(SV_EINVAL, "idx/out is NULL");
@@ -1337,6 +1385,10 @@ int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
 
 // ---- sampling --------------------------------------------------------------------
 static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) {
+    {
+        const int rz = materialize(s);
+        if (rz) return rz;
+    }
     int rc = canonicalize(s);
     if (rc) return rc;
     const uint64_t La = s->local_amps();
@@ -1435,6 +1487,7 @@ int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out) {
 
 // ---- whole state ------------------------------------------------------------------
 static int set_state_bytes(sv_state* s, const void* host) {
+    s->zero_pending = false;  // every amplitude is overwritten
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
     const size_t sb = s->elem << s->l;
     for (int i = 0; i < s->local_shards(); ++i) {
@@ -1467,6 +1520,10 @@ int sv_set_state_c128(sv_state* s, const sv_c128* host, size_t count) {
 }
 
 static int get_state_bytes(sv_state* s, void* host) {
+    {
+        const int rz = materialize(s);
+        if (rz) return rz;
+    }
     int rc = canonicalize(s);
     if (rc) return rc;
     rc = barrier(s);
@@ -1512,6 +1569,11 @@ int sv_get_state_c128(sv_state* s, sv_c128* host, size_t count) {
 int sv_device_ptr(sv_state* s, int shard, void** out) {
     if (!s || !out) return fail(SV_EINVAL, "NULL argument");
     if (shard < 0 || shard >= s->world || !s->shard[shard]) return fail(SV_EINVAL, "shard not available here");
+    if (s->zero_pending) {  // the caller may read the memory: write |0...0> now
+        int rc = materialize(s);
+        if (rc == SV_OK) rc = sync(s);
+        if (rc) return rc;
+    }
     *out = s->shard[shard];
     return SV_OK;
 }

@@ -264,3 +264,40 @@ def test_virtual_shards_blocked_passes(world, F):
         sv.sv_destroy(h)
     assert st["n_exchanges"] >= 1 and st["n_passes"] >= 1
     _check(n, 14, got, ref_c.run(n, gates))
+
+
+def test_reset_is_exact_for_every_reader():
+    """sv_reset writes |0...0> lazily (complex64): every reader sees it --
+    get_state, amplitudes, sampling, a per-gate apply, and a circuit whose
+    first register-blocked pass synthesises the zero tiles."""
+    n = 20
+    rs = np.random.default_rng(3)
+    h = sv.sv_create(n)
+    try:
+        e0 = np.zeros(1 << n, dtype=np.complex64)
+        e0[0] = 1
+        sv.sv_set_state(h, W.random_state_c64(n, 2))
+        sv.sv_reset(h)
+        assert np.array_equal(sv.sv_get_state(h, n), e0)
+        sv.sv_set_state(h, W.random_state_c64(n, 2))
+        sv.sv_reset(h)
+        assert sv.sv_amplitudes(h, np.array([0, 1, 5], dtype=np.uint64)).tolist() == [1, 0, 0]
+        sv.sv_reset(h)
+        assert np.all(sv.sv_sample(h, 1, 100) == 0)
+        sv.sv_reset(h)
+        M = W.haar_unitary(2, rs).astype(np.complex64)
+        sv.sv_apply_fused(h, [7], M)
+        got = sv.sv_get_state(h, n)
+        assert abs(got[0] - M[0, 0]) < 1e-6 and abs(got[1 << 7] - M[1, 0]) < 1e-6
+        gates = W.rqc(n, 8)
+        sv.sv_set_state(h, W.random_state_c64(n, 4))
+        sv.sv_reset(h)
+        c = sv.sv_circuit_create(h, gates, 1)
+        assert sv.sv_circuit_stats(c)["n_passes"] > 0
+        sv.sv_circuit_run_device(h, c)
+        sv.sv_synchronize(h)
+        got = sv.sv_get_state(h, n)
+        sv.sv_circuit_destroy(c)
+    finally:
+        sv.sv_destroy(h)
+    _check(n, 8, got, ref_c.run(n, gates))
