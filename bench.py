@@ -356,7 +356,10 @@ def run_ours(args):
     launches_apply = n_high + n_low
     avg_launch = t_apply / max(launches_apply, 1)
     bytes_per_launch = 2 * elem * (1 << (n - (world.bit_length() - 1)))
-    achieved = bytes_per_launch / avg_launch / 1e9 if avg_launch > 0 else None
+    # algorithmic bytes the library counted for these launches (16 B per
+    # amplitude per pass; 8 B for a first pass that synthesises |0...0>)
+    achieved = (bytes_apply / t_apply / 1e9) if t_apply > 0 and bytes_apply else (
+        bytes_per_launch / avg_launch / 1e9 if avg_launch > 0 else None)
     frac = achieved / peak if achieved else None
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -410,6 +413,7 @@ def run_ours(args):
                          "peak_source": peak_src, "unit": "GB/s", "frac": frac,
                          "frac_of_8tbs": achieved / 8000.0 if achieved else None,
                          "algorithmic_bytes_per_launch": bytes_per_launch,
+                         "algorithmic_bytes_per_step": bytes_apply // max(args.steps, 1),
                          "traffic": load_traffic("rpass" if cst["n_passes"] else "apply"),
                          # the blocked passes are bound by HBM and the FP32 pipe
                          # together: the FMA-pipe share of the same launches

@@ -1222,7 +1222,8 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
                 });
                 if (rc) return rc;
             }
-            s->stats.bytes_apply += 16ull << s->l;
+            // algorithmic bytes: read + write, or write only when |0...0> is synthesised
+            s->stats.bytes_apply += ((zinit && &st == &c->steps[0]) ? 8ull : 16ull) << s->l;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
             s->stats.fma_apply += st.pass.fma_per_amp << s->l;
             s->stats.n_passes += 1;
