@@ -133,7 +133,10 @@ int sv_create(int n_qubits, sv_state** out);
 /* General form (sharded / caller-owned buffer / caller stream). */
 int sv_create_ex(const sv_config* cfg, sv_state** out);
 int sv_destroy(sv_state* s);
-/* |0...0> and the identity qubit map. Asynchronous. */
+/* |0...0> and the identity qubit map. Asynchronous.  On complex64 states the
+ * write is deferred: a circuit that starts with a register-blocked pass
+ * builds the zero tiles itself (no extra pass over HBM); every other call that
+ * reads or writes the state (or sv_device_ptr) writes |0...0> first. */
 int sv_reset(sv_state* s);
 
 /* ---- the hot path ----------------------------------------------------------- */
