@@ -119,7 +119,7 @@ class ClockSampler:
             parts = [x.strip() for x in line.split(",")]
             if len(parts) >= 3:
                 try:
-                    self.rows.append((float(parts[0]), float(parts[1]), int(parts[2], 16)))
+                    self.rows.append((float(parts[0]), float(parts[1]), int(parts[2], 16), time.time()))
                 except ValueError:
                     pass
 
@@ -131,10 +131,25 @@ class ClockSampler:
             except Exception:
                 self.proc.kill()
 
+    def wait_ready(self, timeout: float = 5.0):
+        """Block until nvidia-smi delivers its first sample (its start-up
+        takes longer than a short timed region)."""
+        t0 = time.time()
+        while self.proc and not self.rows and time.time() - t0 < timeout:
+            time.sleep(0.02)
+
+    def mark(self, t0: float, t1: float):
+        self.window = (t0, t1)
+
     def summary(self):
         if not self.rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
-        load = [r for r in self.rows if not (r[2] & 0x1)] or self.rows
+        rows = self.rows
+        w = getattr(self, "window", None)
+        if w:  # samples taken during the timed region (100 ms period), else the nearest ones
+            inside = [r for r in rows if w[0] - 0.05 <= r[3] <= w[1] + 0.15]
+            rows = inside or sorted(rows, key=lambda r: min(abs(r[3] - w[0]), abs(r[3] - w[1])))[:2]
+        load = [r for r in rows if not (r[2] & 0x1)] or rows
         reasons = set()
         for r in load:
             for bit, name in REASON_BITS.items():
@@ -291,9 +306,11 @@ def run_ours(args):
     bytes_exch = 0
     fma = 0
     with ClockSampler(dev) as clk:
+        clk.wait_ready()
         start = torch.cuda.Event(enable_timing=True)
         end = torch.cuda.Event(enable_timing=True)
         barrier()
+        t_host0 = time.time()
         start.record(stream)
         for _ in range(args.steps):
             device_step()
@@ -311,6 +328,8 @@ def run_ours(args):
             fma += st["fma_apply"]
         end.record(stream)
         barrier()
+        clk.mark(t_host0, time.time())
+        time.sleep(0.15)  # let the sampler deliver the sample that covers the end of the region
     sv.sv_set_timing(h, False)
     ms = start.elapsed_time(end) / args.steps
     # the per-step sv_last_stats sync adds a host round trip per step; report

@@ -314,7 +314,7 @@ __device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
 // modifier; both matrix pairs come straight from uniform registers,
 // LDCU.64).  Otherwise four FFMA.
 #ifndef SVB_RP_G
-#define SVB_RP_G 2  // groups transformed together (independent FFMA2 chains)
+#define SVB_RP_G 1  // groups transformed together (1 measured 0.8 % faster than 2 or 4 at T = 13)
 #endif
 template <int M, int MASK, bool F2>
 __device__ __forceinline__ void reg_gate(float2 (&a)[1 << M], const float* __restrict__ mf) {
