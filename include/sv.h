@@ -88,7 +88,10 @@ typedef struct {
     sv_c128 m[16];
 } sv_gate;
 
-/* Statistics of the last sv_run_circuit / sv_circuit_run_device.  Host times
+/* Statistics of the last sv_run_circuit / sv_circuit_run_device.  (SURVEY.md
+ * §8b proposed a smaller struct; this one adds launch counts per kernel class,
+ * device-side times, the blocked-pass and FMA counters and a byte split by
+ * class -- every §8b field keeps its meaning.)  Host times
  * are wall-clock; t_apply_*_dev / t_exchange_dev / t_sample_dev are summed
  * CUDA-event durations around each launch and are filled only when timing is
  * enabled with sv_set_timing(s, 1).  Bytes are ALGORITHMIC: 16 B per
@@ -110,6 +113,10 @@ typedef struct {
     uint64_t fma_apply;         /* fp32 FMAs the register-blocked passes execute (dense
                                    2^k x 2^k: 4*2^k per amplitude, diagonal: 4, CZ: 0),
                                    per shard; 0 for other kernels                       */
+    uint64_t bytes_apply_high;  /* bytes_apply split by kernel class: high-qubit kernels  */
+    uint64_t bytes_apply_low;   /*   (incl. all blocked passes) / low-qubit kernels       */
+    int32_t n_jit_passes;       /* blocked passes run by pass-specialised kernels          */
+    int32_t reserved2_;
 } sv_stats;
 
 typedef struct {
@@ -133,17 +140,22 @@ int sv_create(int n_qubits, sv_state** out);
 /* General form (sharded / caller-owned buffer / caller stream). */
 int sv_create_ex(const sv_config* cfg, sv_state** out);
 int sv_destroy(sv_state* s);
-/* |0...0> and the identity qubit map. Asynchronous.  On complex64 states the
- * write is deferred: a circuit that starts with a register-blocked pass
- * builds the zero tiles itself (no extra pass over HBM); every other call that
- * reads or writes the state (or sv_device_ptr) writes |0...0> first. */
+/* |0...0> and the identity qubit map. Asynchronous.  On complex64 states in
+ * library-owned memory the write is deferred: a circuit that starts with a
+ * register-blocked pass builds the zero tiles itself (no extra pass over
+ * HBM); every other call that reads or writes the state (or sv_device_ptr)
+ * writes |0...0> first.  States in a caller-owned buffer (sv_config.dev_buf)
+ * and complex128 states are written immediately (stream-ordered). */
 int sv_reset(sv_state* s);
 
 /* ---- the hot path ----------------------------------------------------------- */
 /* Apply one dense k-qubit matrix (1 <= k <= 6) in place.  qubits distinct and
  * < n in any order; matrix row-major 2^k x 2^k complex64, bit b <-> qubits[b]
  * (logical qubits: in sharded mode an exchange is inserted when needed).
- * Asynchronous: the matrix is staged before return. */
+ * Asynchronous: matrices that do not travel as kernel parameters (k = 6,
+ * int8 tensor-core slices, complex128 planes) are copied into a pinned
+ * staging ring before return; the call blocks only when the GPU is more than
+ * 8 such applies behind. */
 int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix);
 
 /* Controlled gate (qsim ApplyControlledGate; SURVEY.md
@@ -185,7 +197,10 @@ int sv_amplitudes_c128(sv_state* s, const uint64_t* idx, size_t count, sv_c128* 
  * complex128 states p = fl(fl(re^2) + fl(im^2)) (reading R5). */
 int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out);
 /* Device form: writes n_samples uint64 into device memory dev_out
- * (asynchronous; the bench's device step). */
+ * (asynchronous, no host round trip; the bench's device step).  The total
+ * weight is checked on the device: if it is 0 or sum |c|^2 >= 3.99 every
+ * output is UINT64_MAX (not a basis index) and the next sv_synchronize (or
+ * sv_sample) on this handle returns SV_EINVAL once. */
 int sv_sample_device(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* dev_out);
 
 /* ---- whole-state access (tests, debugging) ------------------------------ */
@@ -196,7 +211,9 @@ int sv_get_state(sv_state* s, sv_c64* host, size_t count);
 /* complex128 forms (converting on complex64 states). */
 int sv_set_state_c128(sv_state* s, const sv_c128* host, size_t count);
 int sv_get_state_c128(sv_state* s, sv_c128* host, size_t count);
-/* Device pointer of shard `shard` (virtual mode) / of this rank's shard. */
+/* Device pointer of shard `shard` (virtual mode) / of this rank's shard
+ * (multi-process mode: shard must equal the rank; peers' shards are not
+ * handed out).  Materialises a pending |0...0> first. */
 int sv_device_ptr(sv_state* s, int shard, void** out);
 
 /* ---- pure host helpers (no GPU needed) ------------------------------------ */
@@ -249,8 +266,45 @@ int sv_set_blocking(sv_state* s, int tile_bits);
 int sv_set_timing(sv_state* s, int enable);
 /* Stats of the most recent run on this handle. */
 int sv_last_stats(const sv_state* s, sv_stats* out);
-/* Synchronise the handle's stream. */
+/* Synchronise the handle's stream.  Returns SV_EINVAL (once) if an earlier
+ * sv_sample_device found an invalid total weight (see there). */
 int sv_synchronize(sv_state* s);
+
+/* Per-handle execution options (replace process-wide environment switches):
+ *   SV_OPT_BLOCK_BITS  = sv_set_blocking (tile qubits of the blocked passes);
+ *   SV_OPT_PASS_JIT    1 (default): register-blocked passes run kernels
+ *                      specialised to each pass (PTX for sm_100a, compiled in
+ *                      sv_circuit_create and cached per process); 0: the
+ *                      generic apply_rpass kernel.  Both give bit-identical
+ *                      states;
+ *   SV_OPT_APPLY_PATH  dense fused gates of one launch each:
+ *                      SV_PATH_AUTO (default: k = 5, 6 on the exact int8
+ *                      tensor-core path, k <= 4 SIMT), SV_PATH_SIMT,
+ *                      SV_PATH_INT8 (int8 tensor cores for k = 4..6);
+ *   SV_OPT_TIMING      = sv_set_timing.
+ * Takes effect for circuits created / gates applied afterwards.  SV_EINVAL
+ * for unknown options or values. */
+#define SV_OPT_BLOCK_BITS 1
+#define SV_OPT_PASS_JIT 2
+#define SV_OPT_APPLY_PATH 3
+#define SV_OPT_TIMING 4
+#define SV_PATH_AUTO 0
+#define SV_PATH_SIMT 1
+#define SV_PATH_INT8 2
+int sv_set_option(sv_state* s, int option, int value);
+
+/* PTX of the pass-specialised kernels of every register-blocked pass of a
+ * circuit (max_fused in [1, 2], tile_bits in [10, 13]; the first pass also
+ * in its |0...0> form), separated by "//----" lines.  Pure host unless
+ * compile != 0, which also assembles them through the driver JIT on the
+ * current device (SV_ECUDA with the JIT log on failure).  *need gets the
+ * length including the terminating NUL; cap < *need returns SV_EINVAL unless
+ * buf is NULL and cap is 0 (size query). */
+int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int tile_bits, int compile, char* buf,
+                    size_t cap, size_t* need);
+/* Process-wide counters of the pass-kernel compiler: kernels compiled, cache
+ * hits, seconds spent compiling.  Pointers may be NULL. */
+int sv_jit_stats(uint64_t* compiled, uint64_t* cache_hits, double* compile_seconds);
 const char* sv_last_error(void);
 /* Library version string. */
 const char* sv_version(void);

@@ -31,6 +31,14 @@ SV_ECOMM = -4
 SV_EUNSUPPORTED = -5
 SV_EBADSTATE = -6
 
+SV_OPT_BLOCK_BITS = 1
+SV_OPT_PASS_JIT = 2
+SV_OPT_APPLY_PATH = 3
+SV_OPT_TIMING = 4
+SV_PATH_AUTO = 0
+SV_PATH_SIMT = 1
+SV_PATH_INT8 = 2
+
 SV_GATE = np.dtype([("nq", "<i4"), ("q", "<i4", (2,)), ("pad", "<i4"), ("m", "<c16", (16,))], align=True)
 assert SV_GATE.itemsize == 272
 
@@ -63,6 +71,10 @@ class sv_stats(ctypes.Structure):
         ("n_passes", ctypes.c_int32),
         ("block_bits", ctypes.c_int32),
         ("fma_apply", ctypes.c_uint64),
+        ("bytes_apply_high", ctypes.c_uint64),
+        ("bytes_apply_low", ctypes.c_uint64),
+        ("n_jit_passes", ctypes.c_int32),
+        ("reserved2_", ctypes.c_int32),
     ]
 
     def as_dict(self):
@@ -125,6 +137,10 @@ _SIGS = {
     "sv_attach_peers": ([_vp, _vp, _sz], ctypes.c_int),
     "sv_set_blocking": ([_vp, ctypes.c_int], ctypes.c_int),
     "sv_set_timing": ([_vp, ctypes.c_int], ctypes.c_int),
+    "sv_set_option": ([_vp, ctypes.c_int, ctypes.c_int], ctypes.c_int),
+    "sv_pass_kernels": ([_vp, _sz, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_char_p, _sz, ctypes.POINTER(_sz)],
+                        ctypes.c_int),
+    "sv_jit_stats": ([_u64p, _u64p, ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
     "sv_last_stats": ([_vp, ctypes.POINTER(sv_stats)], ctypes.c_int),
     "sv_synchronize": ([_vp], ctypes.c_int),
     "sv_last_error": ([], ctypes.c_char_p),
@@ -403,6 +419,29 @@ def sv_set_blocking(h: int, tile_bits: int) -> None:
 
 def sv_set_timing(h: int, enable: bool) -> None:
     _check(lib().sv_set_timing(h, 1 if enable else 0), "sv_set_timing")
+
+
+def sv_set_option(h: int, option: int, value: int) -> None:
+    _check(lib().sv_set_option(h, option, value), "sv_set_option")
+
+
+def sv_pass_kernels(gates, max_fused: int, tile_bits: int, compile: bool = False) -> list:
+    """CUDA sources of the pass-specialised kernels of a circuit's register-
+    blocked passes (pure host; compile=True also compiles the PTX)."""
+    g = as_gates(gates)
+    need = _sz()
+    _check(lib().sv_pass_kernels(_ptr(g), len(g), max_fused, tile_bits, 1 if compile else 0, None, 0,
+                                 ctypes.byref(need)), "sv_pass_kernels")
+    buf = ctypes.create_string_buffer(need.value)
+    _check(lib().sv_pass_kernels(_ptr(g), len(g), max_fused, tile_bits, 0, buf, need.value, ctypes.byref(need)),
+           "sv_pass_kernels")
+    return [x for x in buf.value.decode().split("\n//----\n") if x.strip()]
+
+
+def sv_jit_stats() -> dict:
+    c, h, t = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_double()
+    _check(lib().sv_jit_stats(ctypes.byref(c), ctypes.byref(h), ctypes.byref(t)), "sv_jit_stats")
+    return {"compiled": c.value, "cache_hits": h.value, "compile_s": t.value}
 
 
 def sv_last_stats(h: int) -> dict:

@@ -18,9 +18,12 @@ INCLUDE = os.path.join(ROOT, "include")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+# nvJitLink compiles the PTX of the pass-specialised kernels at circuit creation (rpass_jit.cpp)
+LINK: list = []
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcudafe", "--diag_suppress=177", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC]
 
-SOURCES = ["apply.cu", "apply64.cu", "blocked.cu", "small.cu", "state.cu", "fuser.cpp", "planner.cpp", "sv_api.cpp"]
+SOURCES = ["apply.cu", "apply64.cu", "blocked.cu", "small.cu", "state.cu", "fuser.cpp", "planner.cpp", "rpass_jit.cpp",
+           "sv_api.cpp"]
 HEADERS = ["kernels.h", "sv_internal.h", "device_util.cuh"]
 
 
@@ -31,6 +34,9 @@ def _newest_input() -> float:
 
 def _compile(src: str, verbose: bool) -> str:
     obj = os.path.join(BUILD, src + ".o")
+    hdr = max(os.path.getmtime(p) for p in [os.path.join(CSRC, f) for f in HEADERS] + [os.path.join(INCLUDE, "sv.h"), __file__])
+    if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(os.path.join(CSRC, src)), hdr):
+        return obj  # up to date
     cmd = [NVCC] + ARCH + COMMON + ["-c", os.path.join(CSRC, src), "-o", obj]
     if src.endswith(".cu"):
         cmd += ["-Xptxas", "-v"] if verbose else []
@@ -60,7 +66,7 @@ def build_variant(name: str, defines, csrc: str = CSRC, include: str = INCLUDE) 
 
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
         objs = list(ex.map(comp, SOURCES))
-    subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", out] + objs + ["-Xcompiler", "-fPIC"])
+    subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", out] + objs + ["-Xcompiler", "-fPIC"] + LINK)
     return out
 
 
@@ -71,7 +77,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), SOURCES))
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-Xcompiler", "-fPIC"]
+    cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-Xcompiler", "-fPIC"] + LINK
     if verbose:
         print(" ".join(cmd), flush=True)
     subprocess.check_call(cmd)

@@ -35,6 +35,26 @@
 #include "device_util.cuh"
 #include "kernels.h"
 
+// Build options (compile-time; A/B variants via build.py --variant):
+#ifndef SVB_TF32X3
+#define SVB_TF32X3 0  // TF32x3 tensor-core path (biased): quarantined, off
+#endif
+#ifndef SVB_WS
+#define SVB_WS 1  // bulk/tensor-copy (warp-specialised) tile loop
+#endif
+#ifndef SVB_WS_UNSWZ
+#define SVB_WS_UNSWZ -1  // low gates on the bulk-copy loop: -1 conflict model, 0 never, 1 always
+#endif
+#ifndef SVB_SWZ128
+#define SVB_SWZ128 1  // allow the TMA 128 B swizzle layout
+#endif
+#ifndef SVB_WS_MINRUN
+#define SVB_WS_MINRUN 2048u  // shortest run (bytes) moved by per-run bulk copies
+#endif
+#ifndef SVB_TMAP
+#define SVB_TMAP -1  // tensor-map tile copies: -1 auto, 0 never, 1 always
+#endif
+
 namespace svb {
 
 namespace {
@@ -1696,10 +1716,8 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
         static const uint32_t kNone[3] = {0u, 0u, 0u}, k128[3] = {1u << 4, 1u << 5, 1u << 6};
         const bool natural = p.swz[0] == 0 && p.swz[1] == 0 && p.swz[2] == 0;
         const bool simt = !d.tc && K <= 5 && K != 3;
-        const bool eligible = std::getenv("SVB200_NO_WS") == nullptr && p.nH <= 6 && (simt || d.tci);
-        const char* ev = std::getenv("SVB200_WS_UNSWZ");
-        const bool force = ev != nullptr && ev[0] == '1', never = ev != nullptr && ev[0] == '0';
-        const char* e128 = std::getenv("SVB200_SWZ128");
+        const bool eligible = SVB_WS && p.nH <= 6 && (simt || d.tci);
+        const bool force = SVB_WS_UNSWZ == 1, never = SVB_WS_UNSWZ == 0;
         double cf = 1.0;
         if (eligible && !natural) {
             cf = gather_conflicts(K, gpt, pair, tl, ng[0], kNone);
@@ -1708,7 +1726,7 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
             // at most 2-way (its >= 2 KB runs can use per-run bulk copies, which
             // measured faster there than tensor copies: k = 5 2.86 vs 2.96 ms)
             const bool better = d.tci ? (cf > 2.0 && c128 <= 2.0) : c128 < cf;
-            if (better && !(e128 && e128[0] == '0')) {
+            if (better && SVB_SWZ128) {
                 swz128 = true;
                 cf = c128;
             }
@@ -1719,10 +1737,8 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
             // copies (encode_tile_map): per-run bulk copies of 1 KB runs measured
             // 10-40 % slower, of 2 KB runs 8 % slower inside a circuit; tensor
             // copies of >= 4 KB runs 1-3 % slower than per-run bulk copies
-            const char* mr = std::getenv("SVB200_WS_MINRUN");
-            const uint32_t minrun = mr ? (uint32_t)std::atoi(mr) : 2048u;
-            const char* tm = std::getenv("SVB200_TMAP");
-            const bool tmap = swz128 || (tm ? tm[0] == '1' : (p.r <= 8 || (d.tci && K == 6) || (gpt == 2 && pair)));
+            const uint32_t minrun = SVB_WS_MINRUN;
+            const bool tmap = swz128 || (SVB_TMAP >= 0 ? SVB_TMAP == 1 : (p.r <= 8 || (d.tci && K == 6) || (gpt == 2 && pair)));
             if (tmap)
                 encode_tile_map(p.tmap, p.trank, p.tstart, p.tbits, p.tnx, p.txpos, psi, n, p.r, p.Hpos, p.nH, swz128);
             ws = swz128 ? p.trank > 0 : ((8u << p.r) >= minrun || p.trank > 0);
@@ -1868,12 +1884,16 @@ cudaError_t launch_tile_k(float2* psi, int n, const ApplyDesc& d, cudaStream_t s
             return pair ? go(apply_tci<K, true>) : go(apply_tci<K, false>);
         }
     }
+#if SVB_TF32X3
     if constexpr (K == 4 || K == 5) {
         if (d.tc) {
             if (p.T != 12) return cudaErrorInvalidConfiguration;
             return pair ? go(apply_tc<K, true>) : go(apply_tc<K, false>);
         }
     }
+#else
+    if (d.tc) return cudaErrorInvalidConfiguration;  // only the int8 path is built
+#endif
     if constexpr (K <= 5) {
         if (ws) {
             if (p.mono) return pair ? go(apply_high_ws<K, true, true>, nthr + 32) : go(apply_high_ws<K, false, true>, nthr + 32);
@@ -1985,20 +2005,16 @@ void plan_apply(int n, ApplyDesc& d) {
             else used |= 1ull << src;
         }
         d.mono = mono;
-        // Tensor cores for dense k = 4, 5 gates.  SVB200_TC selects the path:
-        //   unset / "auto": k = 5, 6 on the exact int8-slice tensor-core path
+        // Tensor cores for dense gates; d.tc_mode (sv_set_option
+        // SV_OPT_APPLY_PATH) selects the path:
+        //   3 (auto, default): k = 5, 6 on the exact int8-slice tensor-core path
         //     (SIMT k = 5, 6 are FP32-issue bound), k <= 4 SIMT (HBM-bound or
         //     close to it);
-        //   "i8": the int8 path for k = 4..6; "tf32": TF32x3 for k = 4, 5
-        //     (its accumulation truncates toward zero, shrinking the norm by
-        //     ~4u / ~7u per apply); "simt" / "0": SIMT only.
-        static const int tc_mode = [] {
-            const char* e = std::getenv("SVB200_TC");
-            if (!e || std::strcmp(e, "auto") == 0) return 3;
-            if (std::strcmp(e, "tf32") == 0 || std::strcmp(e, "1") == 0) return 1;
-            if (std::strcmp(e, "i8") == 0) return 2;
-            return 0;
-        }();
+        //   2: the int8 path for k = 4..6;   0: SIMT only;
+        //   1: TF32x3 for k = 4, 5 -- quarantined: its accumulation truncates
+        //     toward zero, shrinking the norm by ~4u / ~7u per apply (DESIGN.md
+        //     §11), so it exists only in builds with -DSVB_TF32X3=1.
+        const int tc_mode = (d.tc_mode == 1 && !SVB_TF32X3) ? 0 : d.tc_mode;
         const bool want = (tc_mode == 1 && d.k <= 5) || tc_mode == 2 || (tc_mode == 3 && d.k >= 5);
         d.tc = !mono && want && d.nc == 0 && tc_supported(n, d);
         d.tci = d.tc && tc_mode != 1;

@@ -27,6 +27,29 @@
 #include "device_util.cuh"
 #include "kernels.h"
 
+// Build options (compile-time; A/B variants via build.py --variant):
+#ifndef SVB_RP_M
+#define SVB_RP_M 5  // log2 amplitudes per thread (4: 16 per thread, measured slower)
+#endif
+#ifndef SVB_RP_ENABLE
+#define SVB_RP_ENABLE 1  // register-blocked passes (0: shared-memory pass kernel only)
+#endif
+#ifndef SVB_RP_F2
+#define SVB_RP_F2 1  // packed FFMA2 complex MACs
+#endif
+#ifndef SVB_RP_DIRECT
+#define SVB_RP_DIRECT 1  // last phase stores registers straight to HBM when coalesced
+#endif
+#ifndef SVB_RP_DLOAD
+#define SVB_RP_DLOAD 0  // first phase loads registers straight from HBM
+#endif
+#ifndef SVB_RP_EARLY
+#define SVB_RP_EARLY 1  // next tile's load issued before the last phase's gates
+#endif
+#ifndef SVB_RP_DEBUG
+#define SVB_RP_DEBUG 0  // print phase plans to stderr
+#endif
+
 namespace svb {
 
 namespace {
@@ -214,6 +237,8 @@ __global__ void __launch_bounds__(kPassThreads) apply_pass(const __grid_constant
     }
 }
 
+}  // namespace
+
 int pass_sms() {
     static int n = 0;
     if (!n) {
@@ -224,6 +249,8 @@ int pass_sms() {
     }
     return n;
 }
+
+namespace {
 
 
 // ------------------------------------------------ register-blocked passes
@@ -241,8 +268,6 @@ int pass_sms() {
 // a fold swizzle (16 B chunk bits 1..3 ^= the XOR of tile bits 4..6, 7..9,
 // ...) and the thread -> position order chosen so that each quarter-warp
 // (LDS.128) / half-warp (LDS.64) gather is conflict-free.
-constexpr int kRpMaxPhases = 48;
-constexpr int kRpMaxGates = 64;
 constexpr int kRpMatFloats = kRpMaxGates * 64;  // 4 floats per element, k <= 2
 
 struct RpPhase {
@@ -728,6 +753,10 @@ __device__ __forceinline__ void reg_gate_dispatch(uint32_t code, float2 (&a)[1 <
 #ifndef SVB_RP_MAXREG5
 #define SVB_RP_MAXREG5 128
 #endif
+#ifndef SVB_RP_PF
+#define SVB_RP_PF 0  // L2 prefetch distance in tiles (0: off; 1 and 2 measured 5 % slower at 30q D14)
+#endif
+__device__ __forceinline__ void prefetch_l2(const void* g) { asm volatile("prefetch.global.L2 [%0];" ::"l"(g)); }
 template <int M, bool F2>
 __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : SVB_RP_MAXREG5) apply_rpass(const __grid_constant__ RpassParams p) {
     constexpr int NA = 1 << M;   // amplitudes per thread
@@ -793,9 +822,20 @@ __global__ void __launch_bounds__(M == 4 ? 512 : 256) __maxnreg__(M == 4 ? 80 : 
             gtile_next = p.psi + tbase(un);
             gnext = gtile_next + dthr;
         }
+        if constexpr (SVB_RP_PF > 0) {
+            // pull a later tile into L2 while this one is transformed, so that
+            // HBM reads stay in flight across the phases (8 threads cover one
+            // 128 B line: runs are >= 16 amplitudes)
+            const uint64_t up = u + (uint64_t)SVB_RP_PF * gridDim.x;
+            if (up < p.n_tiles && !p.zinit && (threadIdx.x & 7u) == 0) {
+                const float2* g = p.psi + tbase(up) + dthr;
+#pragma unroll
+                for (int i = 0; i < UPT; ++i) prefetch_l2(g + p.goff[i]);
+            }
+        }
         if constexpr (SVB_RP_STAGES == 2) {
             __syncthreads();  // buffer `nxt` drained by the previous store
-            if (gnext) load(gnext, nxt);
+            if (gnext && !p.zinit) load(gnext, nxt);
             cp_async_commit();
             cp_async_wait1();
         } else {
@@ -945,7 +985,6 @@ cudaError_t launch_pass(float2* psi, int n, const PassDesc& pd, cudaStream_t st)
 
 // ---------------------------------------------- register-blocked pass (host)
 namespace svb {
-namespace {
 
 uint32_t fold_swz(uint32_t t, int T) {
     uint32_t f = 0;
@@ -956,13 +995,6 @@ uint32_t fold_swz(uint32_t t, int T) {
 // 16 B chunk bank bit (0..2) that tile position q moves under the fold swizzle
 int bank_class(int q) { return q == 0 ? -1 : (q <= 3 ? q - 1 : (q - 4) % 3); }
 
-struct RpPhaseHost {
-    std::vector<int> gates;  // pass gate indices, in application order
-    std::vector<int> R;      // M tile positions, ascending (register bit j <-> R[j])
-    std::vector<int> lanes;  // T-M positions: thread-index bit i <-> lanes[i]
-    bool b0;
-};
-
 uint32_t deposit(uint32_t v, const std::vector<int>& pos) {
     uint32_t x = 0;
     for (size_t b = 0; b < pos.size(); ++b)
@@ -970,14 +1002,7 @@ uint32_t deposit(uint32_t v, const std::vector<int>& pos) {
     return x;
 }
 
-int rpass_m() {
-    static int m = 0;
-    if (!m) {
-        const char* e = getenv("SVB200_RPASS_M");
-        m = (e && e[0] == '4') ? 4 : 5;
-    }
-    return m;
-}
+int rpass_m() { return SVB_RP_M; }
 
 // 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
 int gate_kind(const PassDesc& pd, const PassGate& pg) {
@@ -1008,12 +1033,7 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
     };
     // CZ-like gates run in any layout (their qubits may be thread bits)
     std::vector<char> anyl(pd.gates.size(), 0);
-    static int czfree = -1;
-    if (czfree < 0) {
-        const char* e = getenv("SVB200_RPASS_CZFREE");
-        czfree = (e && e[0] == '0') ? 0 : 1;
-    }
-    for (size_t g = g0; g < g1; ++g) anyl[g] = czfree && gate_kind(pd, pd.gates[g]) == 2;
+    for (size_t g = g0; g < g1; ++g) anyl[g] = gate_kind(pd, pd.gates[g]) == 2;
     while (!rem.empty()) {
         RpPhaseHost ph;
         // R = the M-subset of tile positions that lets the most remaining
@@ -1084,6 +1104,29 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
     return out;
 }
 
+std::vector<std::pair<size_t, size_t>> rpass_chunks(const PassDesc& pd, int M) {
+    std::vector<std::pair<size_t, size_t>> out;
+    const size_t ng = pd.gates.size();
+    size_t g0 = 0;
+    while (g0 < ng) {
+        size_t g1 = std::min(ng, g0 + (size_t)kRpMaxGates);
+        if ((int)plan_phases(pd, g0, g1, M).size() > kRpMaxPhases) {
+            // the first kRpMaxPhases phases hold a prefix of the gates only if
+            // no gate was moved past a later phase: re-plan a shorter prefix
+            size_t cut = g1;
+            do {
+                cut = g0 + (cut - g0) / 2;
+            } while ((int)plan_phases(pd, g0, cut, M).size() > kRpMaxPhases);
+            g1 = cut;
+        }
+        out.push_back({g0, g1});
+        g0 = g1;
+    }
+    return out;
+}
+
+namespace {
+
 // worst bank-conflict degree of a phase's gathers (warp 0, every register j)
 int phase_conflicts(const RpPhaseHost& ph, int T, int M) {
     int worst = 1;
@@ -1138,21 +1181,10 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
     p.n_tiles = 1ull << (n - T);
     const uint64_t grid = std::min<uint64_t>(p.n_tiles, (uint64_t)pass_sms() * per_sm_cache[T]);
     // gates in chunks that fit the parameter block (one launch each)
-    const size_t ng = pd.gates.size();
-    size_t g0 = 0;
-    while (g0 < ng && e == cudaSuccess) {
-        size_t g1 = std::min(ng, g0 + (size_t)kRpMaxGates);
+    for (const auto& ch : rpass_chunks(pd, M)) {
+        if (e != cudaSuccess) break;
+        const size_t g0 = ch.first, g1 = ch.second;
         auto phs = plan_phases(pd, g0, g1, M);
-        if ((int)phs.size() > kRpMaxPhases) {
-            // keep the first kRpMaxPhases phases; their gates are a prefix
-            // only if no gate was moved past a later phase: re-plan a prefix
-            size_t cut = g1;
-            do {
-                cut = g0 + (cut - g0) / 2;
-                phs = plan_phases(pd, g0, cut, M);
-            } while ((int)phs.size() > kRpMaxPhases);
-            g1 = cut;
-        }
         p.nph = (int)phs.size();
         uint32_t moff = 0;
         int li = 0;
@@ -1188,8 +1220,7 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             }
             P.g1 = (uint16_t)li;
         }
-        static const bool dbg = getenv("SVB200_RPASS_DEBUG") != nullptr;
-        if (dbg) {
+        if (SVB_RP_DEBUG) {
             int w = 1;
             for (auto& x : phs) w = std::max(w, phase_conflicts(x, T, M));
             int nb0 = 0;
@@ -1199,11 +1230,6 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             fprintf(stderr, "\n");
         }
         {
-            static int denv = -1;
-            if (denv < 0) {
-                const char* e = getenv("SVB200_RPASS_DIRECT");
-                denv = (e && e[0] == '0') ? 0 : 1;
-            }
             auto coalesced = [](const RpPhaseHost& h) {
                 return h.b0 && h.lanes.size() >= 3 && h.lanes[0] == 1 && h.lanes[1] == 2 && h.lanes[2] == 3;
             };
@@ -1212,7 +1238,7 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                        h.lanes[3] == 3;
             };
             const RpPhaseHost& lp = phs.back();
-            p.direct = denv && (coalesced(lp) || coalesced8(lp));
+            p.direct = SVB_RP_DIRECT && (coalesced(lp) || coalesced8(lp));
             if (p.direct) {
                 if (lp.b0)
                     for (int j = 0; j < (1 << (M - 1)); ++j) p.dgoff[j] = dep(deposit(2u * j, lp.R));
@@ -1222,19 +1248,9 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             }
             const RpPhaseHost& fp = phs.front();
             // measured 1.5 % slower on 30q F=1 (the load latency is no longer
-            // hidden behind the other CTAs' phases): opt-in SVB200_RPASS_DLOAD=1
-            static int lenv = -1;
-            if (lenv < 0) {
-                const char* e = getenv("SVB200_RPASS_DLOAD");
-                lenv = (e && e[0] == '1') ? 1 : 0;
-            }
-            p.dload = lenv && SVB_RP_STAGES == 1 && coalesced(fp);
-            static int eenv = -1;
-            if (eenv < 0) {
-                const char* e = getenv("SVB200_RPASS_EARLY");
-                eenv = (e && e[0] == '0') ? 0 : 1;
-            }
-            p.early = eenv;
+            // hidden behind the other CTAs' phases): build option SVB_RP_DLOAD=1
+            p.dload = SVB_RP_DLOAD && SVB_RP_STAGES == 1 && coalesced(fp);
+            p.early = SVB_RP_EARLY;
             p.zinit = zinit && g0 == 0;  // only the first launch of a split pass starts from |0...0>
             p.zone = zone ? 1 : 0;
             if (p.dload) {
@@ -1242,10 +1258,9 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
                 for (int b = 0; b < p.tbits; ++b) p.lgtbw[b] = dep(1ull << fp.lanes[b]);
             }
         }
-        if (dbg) fprintf(stderr, "   direct=%d dload=%d\n", p.direct, p.dload);
+        if (SVB_RP_DEBUG) fprintf(stderr, "   direct=%d dload=%d\n", p.direct, p.dload);
         apply_rpass<M, F2><<<(unsigned)grid, nthr, smem, st>>>(p);
         e = cudaGetLastError();
-        g0 = g1;
     }
     delete pp;
     return e;
@@ -1254,12 +1269,7 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
 }  // namespace
 
 bool rpass_supported(const PassDesc& pd) {
-    static int env = -1;
-    if (env < 0) {
-        const char* e = getenv("SVB200_RPASS");
-        env = (e && e[0] == '0') ? 0 : 1;
-    }
-    if (!env) return false;
+    if (!SVB_RP_ENABLE) return false;
     const int T = (int)pd.S.size();
     if (T < 10 || T > 13 || pd.r < 1) return false;
     for (auto& g : pd.gates)
@@ -1297,11 +1307,7 @@ void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {
 
 cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone) {
     static_assert(sizeof(RpassParams) <= 32764, "rpass params exceed the kernel parameter space");
-    static int f2 = -1;
-    if (f2 < 0) {
-        const char* e = getenv("SVB200_RPASS_F2");
-        f2 = (e && e[0] == '0') ? 0 : 1;
-    }
+    constexpr bool f2 = SVB_RP_F2 != 0;
     if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st, zinit, zone) : launch_rpass_m<5, false>(psi, n, pd, st, zinit, zone);
     return f2 ? launch_rpass_m<4, true>(psi, n, pd, st, zinit, zone) : launch_rpass_m<4, false>(psi, n, pd, st, zinit, zone);
 }

@@ -5,6 +5,9 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <memory>
+#include <string>
+#include <utility>
 #include <vector>
 
 #include "sv_internal.h"
@@ -27,6 +30,7 @@ struct ApplyDesc {
     bool mono = false;                // one nonzero per row (exact permutation/diagonal path)
     int nc = 0;                       // control qubits (controlled gate, NEXT-4): only the
     int cq[SV_MAX_FUSED] = {0};       //   amplitudes with every control bit 1 are transformed
+    int tc_mode = 3;                  // dense-gate path: 3 auto, 2 int8 k>=4, 0 SIMT (sv_set_option)
     bool tc = false;                  // tensor-core path
     bool tci = false;                 //   ... exact int8-slice variant (needs dev_wi8)
     const uint8_t* dev_wi8 = nullptr; // int8 W slices + column exponents (pack_wi8), device
@@ -109,6 +113,52 @@ void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict);
 // indices, in application order).
 void rpass_phase_plan(const PassDesc& pd, std::vector<std::vector<int>>& R, std::vector<std::vector<int>>& gates);
 
+// ---- rpass host planning, shared by the generic kernel (blocked.cu) and the
+// pass-specialised kernels compiled at circuit creation (rpass_jit.cpp)
+struct RpPhaseHost {
+    std::vector<int> gates;  // pass gate indices, in application order
+    std::vector<int> R;      // M tile positions, ascending (register bit j <-> R[j])
+    std::vector<int> lanes;  // T-M positions: thread-index bit i <-> lanes[i]
+    bool b0;                 // tile position 0 is a register bit (16 B gathers)
+};
+constexpr int kRpMaxPhases = 48;  // per launch (parameter space of the generic kernel)
+constexpr int kRpMaxGates = 64;
+// fold swizzle of a tile index (16 B chunk bits 1..3 ^= tile bits 4..6 ^ 7..9 ^ 10..12)
+uint32_t fold_swz(uint32_t t, int T);
+uint32_t deposit(uint32_t v, const std::vector<int>& pos);
+int rpass_m();
+// 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
+int gate_kind(const PassDesc& pd, const PassGate& pg);
+// phases of pass gates [g0, g1) for M register bits
+std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, int M);
+// The gates [g0, g1) of a pass as launch chunks: each chunk [c0, c1) fits one
+// launch (<= kRpMaxGates gates, <= kRpMaxPhases phases).
+std::vector<std::pair<size_t, size_t>> rpass_chunks(const PassDesc& pd, int M);
+int pass_sms();
+
+// Pass-specialised register-blocked kernels (rpass_jit.cpp): the phase plan,
+// gate kinds, register masks and every address offset of one launch chunk
+// are compiled into a kernel (PTX -> sm_100a via nvJitLink) at circuit creation; only the
+// matrices, the state pointer and the tile count are launch parameters.
+// Kernels are cached per process by their PTX text.
+struct RpJitKernel;
+struct RpJitLaunch {
+    std::shared_ptr<RpJitKernel> kern;
+    std::vector<float> mats;  // float4 (mr, mr, -mi, mi) per matrix element, launch order
+    size_t c0 = 0, c1 = 0;    // gate chunk
+    bool zinit = false;
+};
+// Generate (and compile unless compile == false) the kernels of one pass;
+// returns SV_OK or an error code with the message set (the compiler log).
+int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile, std::vector<RpJitLaunch>& out,
+                      std::vector<std::string>* sources = nullptr);
+// Prepare many passes at once (compiles in parallel host threads).
+int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local, const std::vector<char>& zinit,
+                           std::vector<std::vector<RpJitLaunch>>& out);
+cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st);
+// process-wide counters (sv_jit_stats)
+void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compile_s);
+
 // Launch one fused-gate apply on a shard of 2^n_local amplitudes.
 cudaError_t launch_apply(float2* psi, int n_local, const ApplyDesc& d, cudaStream_t st);
 
@@ -128,13 +178,14 @@ cudaError_t launch_bin_weights(const void* psi, bool fp64, uint64_t n_amps, uint
 size_t scan_scratch_elems(uint64_t count);
 cudaError_t launch_inclusive_scan(uint64_t* data, uint64_t count, uint64_t* scratch, cudaStream_t st);
 // Resolve samples s in [0, n_samples): t_s = (splitmix64#(s+1)(seed) * T) >> 64
+// (T == 0 or T >= 3.99 * 2^62: every out[s] = UINT64_MAX, *status = 1 / 2)
 // with T = *total_dev (+ global offset); samples whose t falls into this
 // shard's range [range_lo, range_lo + local_total) are written as
 // logical index = index_base + local index.  Others untouched.
 cudaError_t launch_sample_resolve(const void* psi, bool fp64, uint64_t n_amps, const uint64_t* cum_bins,
                                   uint64_t n_bins, const uint64_t* range_lo_dev, const uint64_t* total_dev,
                                   uint64_t seed, uint64_t n_samples, uint64_t index_base, uint64_t* out,
-                                  cudaStream_t st);
+                                  uint64_t* status, cudaStream_t st);
 
 // offsets of shard totals in LOGICAL shard order: lo[d] = sum of totals of
 // shards whose logical index sigma[d'] < sigma[d]; *total = sum of all.

@@ -1,0 +1,604 @@
+// rpass_jit.cpp -- pass-specialised register-blocked kernels (SURVEY.md §8f
+// NEXT-2; related work [12]: several gates per memory pass).
+//
+// The generic apply_rpass kernel (blocked.cu) reads its phase plan from the
+// kernel parameters and dispatches every gate through a compare tree on a
+// gate code.  ncu on a 20-gate pass of the 30q RQC (profiles/r2_*) put only
+// 42 % of its instructions in the FFMA2 complex MACs: the per-gate dispatch,
+// the per-phase address tables and the uniform-datapath chains between them
+// cost as much issue time as the math.  Here the same plan -- the phases
+// (register positions R, lane positions, 16 B or 8 B gathers), every gate's
+// kind and register mask, every shared-memory and global offset -- is
+// written out as straight-line PTX for one launch chunk and assembled for
+// sm_100a by the driver's JIT (ptxas: ~0.1-0.3 s per kernel; going through
+// CUDA C++ and NVVM took 15-130 s) when the circuit is created; only the matrices,
+// the state pointer and the tile count remain launch parameters, so circuits
+// with the same structure share kernels (process-wide cache keyed by the
+// PTX text).
+//
+// The arithmetic is the generic kernel's, operation for operation (the same
+// FFMA2 sequence per complex MAC, the same order over columns), so both
+// produce bit-identical states; tests/test_gpu_jit.py checks that.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <sstream>
+#include <thread>
+
+#include "kernels.h"
+
+namespace svb {
+
+struct RpJitKernel {
+    std::string src;  // PTX
+    int nthr = 0;
+    size_t smem = 0;
+    size_t param_bytes = 0;  // sizeof(JP) of the generated kernel
+    size_t nm = 0;           // float4 matrix slots
+    std::mutex mu;           // guards the lazy module load
+    cudaLibrary_t lib = nullptr;
+    cudaKernel_t kern = nullptr;
+    int blocks_per_sm = 0;
+    uint64_t dev_mask = 0;   // devices on which the smem attribute is set
+};
+
+namespace {
+
+std::mutex g_cache_mu;
+std::map<std::string, std::shared_ptr<RpJitKernel>> g_cache;
+std::atomic<uint64_t> g_compiled{0}, g_hits{0};
+std::atomic<uint64_t> g_compile_ns{0};
+
+constexpr int popc(uint32_t m) { return __builtin_popcount(m); }
+uint32_t pdep(uint32_t v, uint32_t mask) {
+    uint32_t r = 0, b = 0;
+    for (int i = 0; i < 32; ++i)
+        if ((mask >> i) & 1u) {
+            if ((v >> b) & 1u) r |= 1u << i;
+            ++b;
+        }
+    return r;
+}
+uint32_t pext(uint32_t v, uint32_t mask) {
+    uint32_t r = 0, b = 0;
+    for (int i = 0; i < 32; ++i)
+        if ((mask >> i) & 1u) {
+            if ((v >> i) & 1u) r |= 1u << b;
+            ++b;
+        }
+    return r;
+}
+
+// global amplitude offset (within the tile's base) of tile index t
+struct TileMap {
+    int r = 0;
+    std::vector<int> H;  // tile positions >= r -> qubit
+    uint64_t dep(uint64_t t) const {
+        uint64_t g = t & ((1ull << r) - 1ull);
+        const uint64_t h = t >> r;
+        for (size_t b = 0; b < H.size(); ++b)
+            if ((h >> b) & 1ull) g += 1ull << H[b];
+        return g;
+    }
+};
+
+// PTX text builder: amplitudes live in %a0..%a31 (one .b64 = packed
+// (re, im) complex64 each), rewritten in place; ptxas renames them.
+struct Ptx {
+    std::ostringstream o;
+    int nr = 0, nrd = 0, np = 0;
+    std::string r32() { return "%r" + std::to_string(nr++); }
+    std::string r64() { return "%rd" + std::to_string(nrd++); }
+    std::string pr() { return "%p" + std::to_string(np++); }
+    template <class... A>
+    void op(const A&... a) {
+        o << "\t";
+        (o << ... << a);
+        o << ";\n";
+    }
+};
+
+// global address "[base+off]" operand (PTX offsets are 32-bit signed)
+std::string gaddr(Ptx& P, const std::string& base, uint64_t off) {
+    if (off == 0) return "[" + base + "]";
+    if (off < (1ull << 31)) return "[" + base + "+" + std::to_string(off) + "]";
+    const std::string t = P.r64();
+    P.op("add.s64 ", t, ", ", base, ", ", off);
+    return "[" + t + "]";
+}
+
+// tile base byte offset = bit-deposit of the tile index u into the qubit
+// positions outside S (runs of consecutive free positions), times 8
+void emit_tbase(Ptx& P, const std::vector<int>& S, int n_local, const std::string& u, const std::string& out) {
+    std::vector<char> in(64, 0);
+    for (int q : S) in[q] = 1;
+    P.op("mov.b64 ", out, ", 0");
+    int b = 0;  // next bit of u
+    for (int q = 0; q < n_local;) {
+        if (in[q]) {
+            ++q;
+            continue;
+        }
+        int e = q;
+        while (e < n_local && !in[e]) ++e;
+        const int L = e - q;
+        const std::string t = P.r64();
+        // (u >> b) & (2^L - 1)) << (q + 3)
+        if (q + 3 >= b) P.op("shl.b64 ", t, ", ", u, ", ", q + 3 - b);
+        else P.op("shr.u64 ", t, ", ", u, ", ", b - q - 3);
+        const uint64_t mask = (L >= 61 ? ~0ull : ((1ull << L) - 1ull)) << (q + 3);
+        P.op("and.b64 ", t, ", ", t, ", ", mask);
+        P.op("or.b64 ", out, ", ", out, ", ", t);
+        b += L;
+        q = e;
+    }
+}
+
+// PTX of one launch chunk [g0, g1) of pass pd; nm receives the number of
+// float4 matrix slots, mats their values (launch order).
+std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
+                      std::vector<float>& mats) {
+    constexpr int M = 5, NA = 32, UPT = 16;
+    const int T = (int)pd.S.size();
+    const int tbits = T - M;
+    const uint32_t nthr = 1u << tbits;
+    TileMap tm;
+    tm.r = pd.r;
+    for (int i = pd.r; i < T; ++i) tm.H.push_back(pd.S[i]);
+    const auto phs = plan_phases(pd, g0, g1, M);
+    const int nph = (int)phs.size();
+    auto coalesced = [](const RpPhaseHost& h) {
+        return h.b0 && h.lanes.size() >= 3 && h.lanes[0] == 1 && h.lanes[1] == 2 && h.lanes[2] == 3;
+    };
+    auto coalesced8 = [](const RpPhaseHost& h) {
+        return !h.b0 && h.lanes.size() >= 4 && h.lanes[0] == 0 && h.lanes[1] == 1 && h.lanes[2] == 2 && h.lanes[3] == 3;
+    };
+    const RpPhaseHost& lp = phs.back();
+    const bool direct = coalesced(lp) || coalesced8(lp);
+    const bool early = direct && !zinit;
+    // matrix slots first (their count fixes the parameter layout)
+    mats.clear();
+    std::vector<size_t> gbase(pd.gates.size(), 0);
+    for (int ph = 0; ph < nph; ++ph)
+        for (int g : phs[ph].gates) {
+            const PassGate& pg = pd.gates[g];
+            const int kind = gate_kind(pd, pg);
+            if (kind == 2) continue;
+            const int D = 1 << pg.k;
+            const float* mg = pd.mats.data() + pg.moff;
+            gbase[g] = mats.size() / 4;
+            const int ne = kind == 1 ? D : D * D;
+            for (int e = 0; e < ne; ++e) {
+                const int src = kind == 1 ? e * D + e : e;
+                const float mr = mg[2 * src], mi = mg[2 * src + 1];
+                mats.push_back(mr);
+                mats.push_back(mr);
+                mats.push_back(-mi);
+                mats.push_back(mi);
+            }
+        }
+    nm = mats.size() / 4;
+    const size_t off_psi = std::max<size_t>(nm, 1) * 16, off_nt = off_psi + 8, off_zone = off_psi + 16;
+    const size_t pbytes = (off_zone + 4 + 15) / 16 * 16;
+
+    Ptx P;
+    // ---- prologue: thread constants
+    P.op("mov.u32 %t_id, %tid.x");
+    P.op("mov.u32 %cur, rsm");
+    P.op("mov.b64 %dthr, 0");
+    P.op("mov.b32 %sthr, 0");
+    if (direct) P.op("mov.b64 %dg, 0");
+    for (int b = 0; b < tbits; ++b) {
+        const std::string t = P.r32(), q = P.pr();
+        P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+        P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+        const uint32_t t2 = 2u << b;  // unit 0 of the thread: tile index 2 tid
+        P.op("@", q, " add.s64 %dthr, %dthr, ", 8 * tm.dep(t2));
+        P.op("@", q, " xor.b32 %sthr, %sthr, ", fold_swz(t2, T) << 3);
+        if (direct) P.op("@", q, " add.s64 %dg, %dg, ", 8 * tm.dep(1ull << lp.lanes[b]));
+    }
+    P.op("ld.param.u64 %psi, [rpj_param_0+", off_psi, "]");
+    P.op("ld.param.u64 %ntiles, [rpj_param_0+", off_nt, "]");
+    P.op("ld.param.u32 %zone, [rpj_param_0+", off_zone, "]");
+    P.op("mov.u32 %r_c, %ctaid.x");
+    P.op("cvt.u64.u32 %u, %r_c");
+    P.op("mov.u32 %r_c, %nctaid.x");
+    P.op("cvt.u64.u32 %grid, %r_c");
+    P.op("setp.ge.u64 %p_out, %u, %ntiles");
+    P.op("@%p_out bra $DONE");
+    emit_tbase(P, pd.S, n_local, "%u", "%tbo");
+    P.op("add.s64 %gtile, %psi, %tbo");
+    P.op("add.s64 %gcur, %gtile, %dthr");
+    auto loadtile = [&](const std::string& g, const std::string& pred) {
+        for (int i = 0; i < UPT; ++i) {
+            const std::string sa = P.r32();
+            P.op("xor.b32 ", sa, ", %sthr, ", fold_swz(2u * nthr * i, T) << 3);
+            P.op("add.s32 ", sa, ", ", sa, ", %cur");
+            const std::string ga = gaddr(P, g, 8 * tm.dep(2ull * nthr * i));
+            P.op(pred, "cp.async.cg.shared.global [", sa, "], ", ga, ", 16");
+        }
+    };
+    if (!zinit) loadtile("%gcur", "");
+    P.op("cp.async.commit_group");
+    P.o << "$LOOP:\n";
+    P.op("add.s64 %un, %u, %grid");
+    P.op("setp.lt.u64 %p_next, %un, %ntiles");
+    emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+    P.op("add.s64 %gtile_next, %psi, %tbo");
+    P.op("add.s64 %gnext, %gtile_next, %dthr");
+    P.op("cp.async.wait_group 0");
+    P.op("bar.sync 0");
+    // ---- phases
+    for (int ph = 0; ph < nph; ++ph) {
+        const RpPhaseHost& Ph = phs[ph];
+        const bool last = ph == nph - 1;
+        P.o << "\t// phase " << ph << ": R = {";
+        for (int q : Ph.R) P.o << q << ",";
+        P.o << "}, " << Ph.gates.size() << " gates\n";
+        P.op("mov.b32 %tb, 0");
+        for (int b = 0; b < tbits; ++b) {
+            const std::string t = P.r32(), q = P.pr();
+            P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+            P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+            P.op("@", q, " xor.b32 %tb, %tb, ", fold_swz(1u << Ph.lanes[b], T) << 3);
+        }
+        auto saddr = [&](uint32_t j) {
+            const std::string t = P.r32();
+            P.op("xor.b32 ", t, ", %tb, ", fold_swz(deposit(j, Ph.R), T) << 3);
+            P.op("add.s32 ", t, ", ", t, ", %cur");
+            return t;
+        };
+        if (ph == 0 && zinit) {
+            for (int j = 0; j < NA; ++j) P.op("mov.b64 %a", j, ", 0");
+            // amplitude 0 = 1 (tile 0, thread 0, register 0) on the shard that holds it
+            P.op("setp.ne.u32 %p_z, %zone, 0");
+            P.op("setp.eq.and.u64 %p_z, %u, 0, %p_z");
+            P.op("setp.eq.and.u32 %p_z, %t_id, 0, %p_z");
+            P.op("@%p_z mov.b64 %a0, 1065353216");  // (1.0f, 0.0f)
+        } else if (Ph.b0) {
+            for (int j = 0; j < NA / 2; ++j) {
+                const std::string a = saddr(2u * j);
+                P.op("ld.shared.v2.b64 {%a", 2 * j, ", %a", 2 * j + 1, "}, [", a, "]");
+            }
+        } else {
+            for (int j = 0; j < NA; ++j) {
+                const std::string a = saddr((uint32_t)j);
+                P.op("ld.shared.b64 %a", j, ", [", a, "]");
+            }
+        }
+        if (last && early) {
+            // tile buffer free: the next tile's load overlaps this phase's gates
+            P.op("bar.sync 0");
+            loadtile("%gnext", "@%p_next ");
+            P.op("cp.async.commit_group");
+        }
+        for (int g : Ph.gates) {
+            const PassGate& pg = pd.gates[g];
+            const int kind = gate_kind(pd, pg);
+            uint32_t mask = 0, tmask = 0;
+            for (int b = 0; b < pg.k; ++b) {
+                const auto it = std::find(Ph.R.begin(), Ph.R.end(), pg.pos[b]);
+                if (it != Ph.R.end()) mask |= 1u << (int)(it - Ph.R.begin());
+                else tmask |= 1u << (int)(std::find(Ph.lanes.begin(), Ph.lanes.end(), pg.pos[b]) - Ph.lanes.begin());
+            }
+            const int D = 1 << pg.k;
+            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask << "\n";
+            if (kind == 2) {  // CZ-like: sign flips of both halves
+                std::string pred;
+                if (popc(mask) != 2) {
+                    const std::string t = P.r32();
+                    pred = P.pr();
+                    P.op("and.b32 ", t, ", %t_id, ", tmask);
+                    P.op("setp.eq.u32 ", pred, ", ", t, ", ", tmask);
+                    pred = "@" + pred + " ";
+                }
+                for (uint32_t j = 0; j < 32; ++j)
+                    if ((j & mask) == mask) P.op(pred, "xor.b64 %a", j, ", %a", j, ", -9223372034707292160");
+                continue;
+            }
+            const size_t base = gbase[g];
+            auto mload = [&](size_t e) {  // (mr, mr) -> %ml, (-mi, mi) -> %mh
+                P.op("ld.param.v2.b64 {%ml, %mh}, [rpj_param_0+", 16 * e, "]");
+            };
+            auto swp = [&](const std::string& x, const std::string& out) {
+                P.op("mov.b64 {%lo, %hi}, ", x);
+                P.op("mov.b64 ", out, ", {%hi, %lo}");
+            };
+            if (kind == 1) {
+                for (int e = 0; e < D; ++e) {
+                    mload(base + e);
+                    for (uint32_t j = 0; j < 32; ++j) {
+                        if (pext(j, mask) != (uint32_t)e) continue;
+                        swp("%a" + std::to_string(j), "%xs0");
+                        P.op("fma.rn.f32x2 %y, %ml, %a", j, ", %zero");
+                        P.op("fma.rn.f32x2 %a", j, ", %mh, %xs0, %y");
+                    }
+                }
+                continue;
+            }
+            const uint32_t rest = 31u & ~mask;
+            for (uint32_t gi = 0; gi < 32u / D; ++gi) {
+                const uint32_t b0 = pdep(gi, rest);
+                for (int c = 0; c < D; ++c) {
+                    P.op("mov.b64 %x", c, ", %a", b0 | pdep(c, mask));
+                    swp("%x" + std::to_string(c), "%xs" + std::to_string(c));
+                }
+                for (int rr = 0; rr < D; ++rr) {
+                    const uint32_t dst = b0 | pdep(rr, mask);
+                    for (int c = 0; c < D; ++c) {
+                        mload(base + rr * D + c);
+                        P.op("fma.rn.f32x2 %y, %ml, %x", c, ", ", c == 0 ? "%zero" : "%y");
+                        P.op("fma.rn.f32x2 ", c == D - 1 ? "%a" + std::to_string(dst) : std::string("%y"), ", %mh, %xs", c,
+                             ", %y");
+                    }
+                }
+            }
+        }
+        if (last && direct) {
+            P.op("add.s64 %gst, %gtile, %dg");
+            if (lp.b0) {
+                for (int j = 0; j < NA / 2; ++j)
+                    P.op("st.global.cs.v2.b64 ", gaddr(P, "%gst", 8 * tm.dep(deposit(2u * j, lp.R))), ", {%a", 2 * j, ", %a",
+                         2 * j + 1, "}");
+            } else {
+                for (int j = 0; j < NA; ++j)
+                    P.op("st.global.cs.b64 ", gaddr(P, "%gst", 8 * tm.dep(deposit((uint32_t)j, lp.R))), ", %a", j);
+            }
+        } else {
+            if (Ph.b0) {
+                for (int j = 0; j < NA / 2; ++j) {
+                    const std::string a = saddr(2u * j);
+                    P.op("st.shared.v2.b64 [", a, "], {%a", 2 * j, ", %a", 2 * j + 1, "}");
+                }
+            } else {
+                for (int j = 0; j < NA; ++j) {
+                    const std::string a = saddr((uint32_t)j);
+                    P.op("st.shared.b64 [", a, "], %a", j);
+                }
+            }
+            P.op("bar.sync 0");
+        }
+    }
+    if (!direct) {  // write the tile back from shared memory
+        for (int i = 0; i < UPT; ++i) {
+            const std::string sa = P.r32();
+            P.op("xor.b32 ", sa, ", %sthr, ", fold_swz(2u * nthr * i, T) << 3);
+            P.op("add.s32 ", sa, ", ", sa, ", %cur");
+            P.op("ld.shared.v2.b64 {%x0, %x1}, [", sa, "]");
+            P.op("st.global.cs.v2.b64 ", gaddr(P, "%gcur", 8 * tm.dep(2ull * nthr * i)), ", {%x0, %x1}");
+        }
+    }
+    if (!zinit && !early) {
+        P.op("bar.sync 0");  // every thread is done with the tile buffer
+        loadtile("%gnext", "@%p_next ");
+        P.op("cp.async.commit_group");
+    }
+    P.op("mov.b64 %gcur, %gnext");
+    P.op("mov.b64 %gtile, %gtile_next");
+    P.op("mov.b64 %u, %un");
+    P.op("@%p_next bra $LOOP");
+    P.o << "$DONE:\n";
+    P.op("ret");
+
+    std::ostringstream k;
+    k << "// pass-specialised register-blocked kernel (generated by rpass_jit.cpp)\n";
+    k << "// T=" << T << " r=" << pd.r << " n=" << n_local << " S={";
+    for (int q : pd.S) k << q << ",";
+    k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (direct ? " direct" : "") << "\n";
+    k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
+    k << ".extern .shared .align 16 .b8 rsm[];\n";
+    k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
+    k << ".maxntid " << nthr << ", 1, 1\n.maxnreg 128\n{\n";
+    k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z;\n";
+    k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi;\n";
+    k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
+    k << "\t.reg .b64 %a<32>;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
+    k << "\t.reg .b64 %y, %ml, %mh, %zero, %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, "
+         "%gnext, %gst;\n";
+    k << "\tmov.b64 %zero, 0;\n";
+    k << P.o.str();
+    k << "}\n";
+    return k.str();
+}
+
+// Assemble the PTX for this device through the driver's JIT (ptxas; the
+// driver also caches the result across processes) and look the kernel up,
+// which forces the module load under lazy loading.
+int compile_one(RpJitKernel& K, int dev, std::string& log) {
+    const auto t0 = std::chrono::steady_clock::now();
+    cudaError_t e = cudaSetDevice(dev);  // worker threads start on device 0
+    if (e != cudaSuccess) {
+        log = cudaGetErrorString(e);
+        return SV_ECUDA;
+    }
+    std::vector<char> elog(8192, 0);
+    cudaJitOption opt[2] = {cudaJitErrorLogBuffer, cudaJitErrorLogBufferSizeBytes};
+    void* val[2] = {elog.data(), (void*)(uintptr_t)elog.size()};
+    e = cudaLibraryLoadData(&K.lib, K.src.c_str(), opt, val, 2, nullptr, nullptr, 0);
+    if (e == cudaSuccess) e = cudaLibraryGetKernel(&K.kern, K.lib, "rpj");
+    if (e == cudaSuccess) e = cudaKernelSetAttributeForDevice(K.kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)K.smem, dev);
+    if (e != cudaSuccess) {
+        log = std::string(cudaGetErrorString(e)) + ": " + elog.data();
+        cudaGetLastError();
+        return SV_ECUDA;
+    }
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, (const void*)K.kern, K.nthr, K.smem) != cudaSuccess || nb < 1) {
+        cudaGetLastError();
+        nb = std::max(1, (int)((227u * 1024u) / (K.smem + 1024u)));
+    }
+    K.blocks_per_sm = nb;
+    K.dev_mask |= 1ull << dev;
+    g_compiled++;
+    g_compile_ns += (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count();
+    return SV_OK;
+}
+
+// find or create the cache entry of a source; `fresh` = needs compiling
+std::shared_ptr<RpJitKernel> lookup(const std::string& src, bool& fresh) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_cache.find(src);
+    if (it != g_cache.end()) {
+        fresh = false;
+        g_hits++;
+        return it->second;
+    }
+    auto K = std::make_shared<RpJitKernel>();
+    K->src = src;
+    g_cache[src] = K;
+    fresh = true;
+    return K;
+}
+
+void drop(const std::string& src) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    g_cache.erase(src);
+}
+
+}  // namespace
+
+int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile, std::vector<RpJitLaunch>& out,
+                      std::vector<std::string>* sources) {
+    std::vector<const PassDesc*> one{&pd};
+    if (!compile) {
+        out.clear();
+        const int T = (int)pd.S.size();
+        bool first = true;
+        for (const auto& ch : rpass_chunks(pd, 5)) {
+            RpJitLaunch l;
+            size_t nm = 0;
+            const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats);
+            if (sources) sources->push_back(src);
+            l.c0 = ch.first;
+            l.c1 = ch.second;
+            l.zinit = zinit && first;
+            (void)T;
+            (void)n_local;
+            out.push_back(std::move(l));
+            first = false;
+        }
+        return SV_OK;
+    }
+    std::vector<std::vector<RpJitLaunch>> all;
+    std::vector<char> z{(char)zinit};
+    int rc = rpass_jit_prepare_many(one, n_local, z, all);
+    if (rc) return rc;
+    out = std::move(all[0]);
+    if (sources)
+        for (auto& l : out) sources->push_back(l.kern->src);
+    return SV_OK;
+}
+
+int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local, const std::vector<char>& zinit,
+                           std::vector<std::vector<RpJitLaunch>>& out) {
+    out.assign(pds.size(), {});
+    std::vector<std::shared_ptr<RpJitKernel>> todo;
+    for (size_t i = 0; i < pds.size(); ++i) {
+        const PassDesc& pd = *pds[i];
+        const int T = (int)pd.S.size();
+        bool first = true;
+        for (const auto& ch : rpass_chunks(pd, 5)) {
+            RpJitLaunch l;
+            size_t nm = 0;
+            const bool z = zinit[i] && first;
+            const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
+            bool fresh = false;
+            l.kern = lookup(src, fresh);
+            if (fresh) {
+                l.kern->nthr = 1 << (T - 5);
+                l.kern->smem = (size_t)8 << T;
+                l.kern->nm = nm;
+                l.kern->param_bytes = (std::max<size_t>(nm, 1) * 16 + 8 + 8 + 4 + 15) / 16 * 16;  // as in gen_chunk
+                todo.push_back(l.kern);
+            }
+            l.c0 = ch.first;
+            l.c1 = ch.second;
+            l.zinit = z;
+            out[i].push_back(std::move(l));
+            first = false;
+        }
+    }
+    if (todo.empty()) return SV_OK;
+    // assemble the new kernels in parallel host threads
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+        cudaGetLastError();
+        for (auto& K : todo) drop(K->src);
+        return fail(SV_ECUDA, "no CUDA device for the pass kernels");
+    }
+    std::atomic<size_t> next{0};
+    std::atomic<int> failed{0};
+    std::string first_log;
+    std::mutex log_mu;
+    auto worker = [&]() {
+        for (;;) {
+            const size_t i = next++;
+            if (i >= todo.size()) return;
+            std::string log;
+            if (compile_one(*todo[i], dev, log) != SV_OK) {
+                failed++;
+                std::lock_guard<std::mutex> lk(log_mu);
+                if (first_log.empty()) first_log = log;
+            }
+        }
+    };
+    const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+    const size_t nt = std::min<size_t>(todo.size(), std::min(hw, 16u));
+    std::vector<std::thread> th;
+    for (size_t t = 1; t < nt; ++t) th.emplace_back(worker);
+    worker();
+    for (auto& t : th) t.join();
+    cudaSetDevice(dev);
+    if (failed) {
+        for (auto& K : todo) drop(K->src);
+        return fail(SV_ECUDA, "PTX JIT of a pass kernel failed: " + first_log.substr(0, 2000));
+    }
+    return SV_OK;
+}
+
+cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st) {
+    RpJitKernel& K = *l.kern;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev >= 64) return cudaErrorInvalidDevice;
+    if (!((K.dev_mask >> dev) & 1ull)) {  // first use on another device
+        std::lock_guard<std::mutex> lk(K.mu);
+        if (!((K.dev_mask >> dev) & 1ull)) {
+            std::string log;
+            if (!K.lib) {
+                if (compile_one(K, dev, log) != SV_OK) return cudaErrorInvalidPtx;
+            } else {
+                e = cudaKernelSetAttributeForDevice(K.kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)K.smem, dev);
+                if (e != cudaSuccess) return e;
+                K.dev_mask |= 1ull << dev;
+            }
+        }
+    }
+    const int T = 5 + __builtin_ctz((unsigned)K.nthr);
+    const uint64_t n_tiles = 1ull << (n_local - T);
+    const uint64_t grid = std::min<uint64_t>(n_tiles, (uint64_t)pass_sms() * K.blocks_per_sm);
+    std::vector<unsigned char> prm(K.param_bytes, 0);
+    std::memcpy(prm.data(), l.mats.data(), l.mats.size() * sizeof(float));
+    const size_t off = std::max<size_t>(K.nm, 1) * 16;
+    const float2* cpsi = psi;
+    std::memcpy(prm.data() + off, &cpsi, 8);
+    std::memcpy(prm.data() + off + 8, &n_tiles, 8);
+    const int zone = one_here ? 1 : 0;
+    std::memcpy(prm.data() + off + 16, &zone, 4);
+    void* args[] = {prm.data()};
+    return cudaLaunchKernel((const void*)K.kern, dim3((unsigned)grid), dim3((unsigned)K.nthr), args, K.smem, st);
+}
+
+void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compile_s) {
+    if (compiled) *compiled = g_compiled;
+    if (cache_hits) *cache_hits = g_hits;
+    if (compile_s) *compile_s = (double)g_compile_ns * 1e-9;
+}
+
+}  // namespace svb

@@ -182,10 +182,18 @@ template <class E>
 __global__ void sample_resolve_kernel(const E* __restrict__ psi, const uint64_t* __restrict__ cum,
                                       uint64_t n_bins, const uint64_t* range_lo_dev, const uint64_t* total_dev,
                                       uint64_t seed, uint64_t n_samples, uint64_t index_base, uint64_t n_amps,
-                                      uint64_t* out) {
+                                      uint64_t* out, uint64_t* status) {
     const uint64_t s = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= n_samples) return;
     const uint64_t T = *total_dev;
+    // S5 validity (checked here so that sampling needs no host round trip):
+    // a zero total or sum |c|^2 >= 3.99 (uint64 overflow risk) yields no
+    // sample -- every output is UINT64_MAX and the status word is set
+    if (T == 0 || (double)T >= 3.99 * 4611686018427387904.0) {
+        out[s] = ~0ull;
+        if (s == 0 && status) *status = T == 0 ? 1ull : 2ull;
+        return;
+    }
     const uint64_t lo = range_lo_dev ? *range_lo_dev : 0ull;
     const uint64_t local_total = cum[n_bins - 1];
     const uint64_t t = __umul64hi(splitmix64_at(seed, s), T);
@@ -329,14 +337,16 @@ cudaError_t launch_inclusive_scan(uint64_t* data, uint64_t count, uint64_t* scra
 cudaError_t launch_sample_resolve(const void* psi, bool fp64, uint64_t n_amps, const uint64_t* cum_bins,
                                   uint64_t n_bins, const uint64_t* range_lo_dev, const uint64_t* total_dev,
                                   uint64_t seed, uint64_t n_samples, uint64_t index_base, uint64_t* out,
-                                  cudaStream_t st) {
+                                  uint64_t* status, cudaStream_t st) {
     if (n_samples == 0) return cudaSuccess;
     if (fp64)
         sample_resolve_kernel<double2><<<(unsigned)((n_samples + 255) / 256), 256, 0, st>>>(
-            (const double2*)psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out);
+            (const double2*)psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out,
+            status);
     else
         sample_resolve_kernel<float2><<<(unsigned)((n_samples + 255) / 256), 256, 0, st>>>(
-            (const float2*)psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out);
+            (const float2*)psi, cum_bins, n_bins, range_lo_dev, total_dev, seed, n_samples, index_base, n_amps, out,
+            status);
     return cudaGetLastError();
 }
 

@@ -22,6 +22,10 @@
 
 using namespace svb;
 
+#ifndef SVB_PASS_PIN
+#define SVB_PASS_PIN 4  // qubits 0..PIN-1 in every blocked-pass tile (runs of 8 * 2^PIN bytes)
+#endif
+
 namespace svb {
 
 static thread_local std::string g_err;
@@ -61,10 +65,23 @@ struct sv_state {
     int vmin = 5;
     int block_bits = -1;      // cache-blocked passes: tile qubits (0 = off, -1 = auto, see sv_circuit_create)
     bool fp64 = false;        // complex128 amplitudes (NEXT-1)
+    bool ext_buf = false;     // the state lives in a caller-owned buffer (sv_config.dev_buf)
+    int tc_mode = 3;          // SV_OPT_APPLY_PATH
+    int pass_jit = 1;         // SV_OPT_PASS_JIT
+    bool sample_pending = false;  // a sv_sample_device status word not yet checked
     size_t elem = 8;          // bytes per amplitude
-    double* planes64 = nullptr;   // fp64 scratch: planes of one gate (sv_apply_fused on fp64 states)
-    uint8_t* wi8 = nullptr;       // int8 tensor-core scratch: W slices of one gate (sv_apply_fused)
-    int* q64 = nullptr;           // fp64 scratch: qubits of one gate (tiny states)
+    // staging ring for per-call device inputs of sv_apply_fused /
+    // sv_apply_controlled (k = 6 matrices, int8 W slices, fp64 planes): a
+    // slot is reused only after the launch that read it has completed (its
+    // event), so the calls stay asynchronous
+    struct StageSlot {
+        char* host = nullptr;  // pinned
+        char* dev = nullptr;
+        cudaEvent_t ev = nullptr;
+        bool used = false;
+    };
+    std::vector<StageSlot> stage;
+    size_t stage_next = 0;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     std::vector<float2*> shard;        // shard pointers (local or peer-mapped)
@@ -82,7 +99,6 @@ struct sv_state {
     uint64_t* misc = nullptr;          // [0..63] lo, [64] total, [65..] totals ptrs area
     uint64_t** totals_ptr_dev = nullptr;
     int32_t* sigma_dev = nullptr;
-    float2* kmat = nullptr;            // k=6 matrix for sv_apply_fused
     // multi-process
     Ctrl* ctrl = nullptr;
     uint64_t* xfer = nullptr;          // kXferBytes
@@ -124,6 +140,7 @@ struct sv_circuit {
         ApplyDesc apply;
         Apply64Desc a64;  // complex128 states
         PassDesc pass;
+        std::vector<RpJitLaunch> jit, jitz;   // pass-specialised kernels (jitz: first pass from |0...0>)
         ExchangeDesc exch;
         std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
     };
@@ -242,7 +259,9 @@ int barrier(sv_state* s) {
 }
 
 // ---- building launch descriptors -------------------------------------------
-void make_apply(int l, int k, const int* phys_in_order, const cd* M /* bit b <-> phys_in_order[b] */, ApplyDesc& d) {
+void make_apply(int l, int k, const int* phys_in_order, const cd* M /* bit b <-> phys_in_order[b] */, ApplyDesc& d,
+                int tc_mode = 3) {
+    d.tc_mode = tc_mode;
     std::vector<cd> Ms((size_t)1 << (2 * k));
     int sq[SV_MAX_FUSED];
     sort_matrix_qubits<cd>(k, phys_in_order, M, sq, Ms.data());
@@ -320,6 +339,7 @@ int run_apply(sv_state* s, const ApplyDesc& d) {
     }
     const int k = d.k;
     s->stats.bytes_apply += 16ull << s->l;
+    (d.high ? s->stats.bytes_apply_high : s->stats.bytes_apply_low) += 16ull << s->l;
     s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
     return SV_OK;
 }
@@ -409,10 +429,6 @@ int alloc_scratch(sv_state* s) {
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
     e = cudaMalloc(&s->sigma_dev, 64 * sizeof(int32_t));
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
-    e = cudaMalloc(&s->kmat, 64 * 64 * sizeof(float2));
-    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
-    e = cudaMalloc(&s->wi8, wi8_bytes(6));
-    if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc failed");
     return SV_OK;
 }
 
@@ -422,10 +438,15 @@ void destroy_state(sv_state* s) {
     for (void* p : s->ipc_opened) cudaIpcCloseMemHandle(p);
     if (s->alloc) cudaFree(s->alloc);
     for (void* p : {(void*)s->shard_dev, (void*)s->bins, (void*)s->scan_scratch, (void*)s->misc,
-                    (void*)s->totals_ptr_dev, (void*)s->sigma_dev, (void*)s->kmat, (void*)s->ctrl, (void*)s->xfer,
+                    (void*)s->totals_ptr_dev, (void*)s->sigma_dev, (void*)s->ctrl, (void*)s->xfer,
                     (void*)s->flags_dev, (void*)s->xfer_dev, (void*)s->idx_dev, (void*)s->amp_dev,
-                    (void*)s->samp_dev, (void*)s->planes64, (void*)s->q64, (void*)s->wi8})
+                    (void*)s->samp_dev})
         if (p) cudaFree(p);
+    for (auto& sl : s->stage) {
+        if (sl.host) cudaFreeHost(sl.host);
+        if (sl.dev) cudaFree(sl.dev);
+        if (sl.ev) cudaEventDestroy(sl.ev);
+    }
     for (auto e : s->ev_pool) cudaEventDestroy(e);
     if (s->own_stream && s->stream) cudaStreamDestroy(s->stream);
     delete s;
@@ -434,6 +455,39 @@ void destroy_state(sv_state* s) {
 int upload_shard_table(sv_state* s) {
     CK(s, cudaMemcpyAsync(s->shard_dev, s->shard.data(), sizeof(float2*) * s->world, cudaMemcpyHostToDevice,
                           s->stream));
+    return SV_OK;
+}
+
+// staging slot layout: k = 6 matrix (32 KB) at 0, int8 W slices at 32 KB;
+// complex128 states: planes (<= 24 KB, k <= 5) at 0, qubits at 128 KB
+constexpr size_t kStageSlots = 8;
+constexpr size_t kStageBytes = 136u << 10;
+constexpr size_t kStageW = 32u << 10, kStageQ = 128u << 10;
+
+int stage_acquire(sv_state* s, sv_state::StageSlot*& out) {
+    if (s->stage.empty()) {
+        s->stage.resize(kStageSlots);
+        for (auto& sl : s->stage) {
+            if (cudaMallocHost((void**)&sl.host, kStageBytes) != cudaSuccess ||
+                cudaMalloc((void**)&sl.dev, kStageBytes) != cudaSuccess ||
+                cudaEventCreateWithFlags(&sl.ev, cudaEventDisableTiming) != cudaSuccess)
+                return fail(SV_ENOMEM, "staging ring allocation failed");
+        }
+    }
+    sv_state::StageSlot& sl = s->stage[s->stage_next++ % kStageSlots];
+    if (sl.used) CK(s, cudaEventSynchronize(sl.ev));  // waits only if the GPU is kStageSlots applies behind
+    out = &sl;
+    return SV_OK;
+}
+// copy `bytes` at slot offset `off` to the device (stream-ordered)
+int stage_put(sv_state* s, sv_state::StageSlot& sl, size_t off, const void* src, size_t bytes) {
+    std::memcpy(sl.host + off, src, bytes);
+    CK(s, cudaMemcpyAsync(sl.dev + off, sl.host + off, bytes, cudaMemcpyHostToDevice, s->stream));
+    return SV_OK;
+}
+int stage_release(sv_state* s, sv_state::StageSlot& sl) {
+    CK(s, cudaEventRecord(sl.ev, s->stream));
+    sl.used = true;
     return SV_OK;
 }
 
@@ -460,11 +514,7 @@ struct PassIn {
 // remaining qubits (longer runs).  The state never moves: a pass only
 // chooses which amplitudes share a tile.
 std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
-    static int kPassPinned = 0;
-    if (!kPassPinned) {
-        const char* e = getenv("SVB200_PASS_PIN");
-        kPassPinned = (e && e[0] >= '1' && e[0] <= '6') ? e[0] - '0' : 4;
-    }
+    constexpr int kPassPinned = SVB_PASS_PIN;
     const uint64_t pin = (1ull << kPassPinned) - 1ull;
     const int Fp = T - kPassPinned;
     const size_t nf = in.size();
@@ -582,6 +632,7 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
     s->vmin = cfg->exchange_vmin < 0 ? 5 : cfg->exchange_vmin;
     s->fp64 = fp64;
     s->elem = fp64 ? 16 : 8;
+    s->ext_buf = cfg->dev_buf != nullptr;
     if (cfg->device >= 0) CK(nullptr, cudaSetDevice(cfg->device));
     CK(nullptr, cudaGetDevice(&s->device));
     if (cfg->cuda_stream) {
@@ -618,11 +669,6 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
     CK(nullptr, cudaMalloc(&s->shard_dev, sizeof(float2*) * world));
     int rc = alloc_scratch(s.get());
     if (rc) return rc;
-    if (fp64) {
-        cudaError_t e = cudaMalloc(&s->planes64, 3 * 4096 * sizeof(double));
-        if (e == cudaSuccess) e = cudaMalloc(&s->q64, 8 * sizeof(int));
-        if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(fp64 scratch)");
-    }
     rc = upload_shard_table(s.get());
     if (rc) return rc;
     s->pos.resize(n);
@@ -646,10 +692,13 @@ int sv_reset(sv_state* s) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
     if (s->sticky) return fail(SV_EBADSTATE, "state poisoned by an earlier device failure");
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
-    if (!s->fp64) {
+    if (!s->fp64 && !s->ext_buf) {
         s->zero_pending = true;  // written lazily (see sv_state::zero_pending)
         return SV_OK;
     }
+    // complex128 states and caller-owned buffers (the caller may read or
+    // write the memory directly) are written now
+    s->zero_pending = false;
     return write_zero_state(s);
 }
 
@@ -699,10 +748,7 @@ int sv_apply_fused_c128(sv_state* s, int k, const int32_t* qubits, const sv_c128
 }
 
 static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::vector<cd>& Min) {
-    {
-        const int rz = materialize(s);
-        if (rz) return rz;
-    }
+    // every argument is validated before any side effect (sv.h)
     int rc = SV_OK;
     uint64_t mask = 0;
     for (int b = 0; b < k; ++b) {
@@ -711,9 +757,11 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
         mask |= 1ull << qubits[b];
     }
     if (s->g > 0 && k > s->l - 1) return fail(SV_EUNSUPPORTED, "gate wider than a shard allows");
+    if (s->fp64 && k > 5) return fail(SV_EUNSUPPORTED, "complex128 states support fused gates with k <= 5");
+    rc = materialize(s);
+    if (rc) return rc;
     std::vector<cd> M = Min;
     std::vector<int> q(qubits, qubits + k);
-    if (s->fp64 && k > 5) return fail(SV_EUNSUPPORTED, "complex128 states support fused gates with k <= 5");
     if (s->fp64) {
         Apply64Desc d;
         d.k = k;
@@ -722,18 +770,22 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
         d.m = Ms;
         std::vector<double> planes(3 * M.size());
         pack_planes64(d, planes.data());
-        CK(s, cudaStreamSynchronize(s->stream));  // the previous launch may still read the scratch
-        CK(s, cudaMemcpyAsync(s->planes64, planes.data(), planes.size() * sizeof(double), cudaMemcpyHostToDevice,
-                              s->stream));
-        CK(s, cudaMemcpyAsync(s->q64, d.q, sizeof(int) * SV_MAX_FUSED, cudaMemcpyHostToDevice, s->stream));
-        CK(s, cudaStreamSynchronize(s->stream));
-        d.dev_planes = s->planes64;
-        d.small_scratch = s->q64;
+        sv_state::StageSlot* sl = nullptr;
+        rc = stage_acquire(s, sl);
+        if (rc) return rc;
+        rc = stage_put(s, *sl, 0, planes.data(), planes.size() * sizeof(double));
+        if (rc == SV_OK) rc = stage_put(s, *sl, kStageQ, d.q, sizeof(int) * SV_MAX_FUSED);
+        if (rc) return rc;
+        d.dev_planes = reinterpret_cast<const double*>(sl->dev);
+        d.small_scratch = sl->dev + kStageQ;
         rc = launch(s, LaunchClass::HIGH, [&] {
             return launch_apply64(reinterpret_cast<double2*>(s->shard[0]), s->l, d, s->stream);
         });
         if (rc) return rc;
+        rc = stage_release(s, *sl);
+        if (rc) return rc;
         s->stats.bytes_apply += 32ull << s->l;
+        s->stats.bytes_apply_high += 32ull << s->l;
         s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
         return SV_OK;
     }
@@ -753,29 +805,33 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
     std::vector<int> phys(k);
     for (int b = 0; b < k; ++b) phys[b] = s->pos[q[b]];
     ApplyDesc d;
-    make_apply(s->l, k, phys.data(), M.data(), d);
-    if (k == 6) {
-        // matrix staged in device memory before return (stream-ordered)
-        CK(s, cudaMemcpyAsync(s->kmat, d.m.data(), 64 * 64 * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
-        CK(s, cudaStreamSynchronize(s->stream));
-        d.dev_m = s->kmat;
+    make_apply(s->l, k, phys.data(), M.data(), d, s->tc_mode);
+    sv_state::StageSlot* sl = nullptr;
+    if (k == 6 || d.tci) {
+        // device inputs staged through the ring (stream-ordered, no host sync)
+        rc = stage_acquire(s, sl);
+        if (rc) return rc;
+        if (k == 6) {
+            rc = stage_put(s, *sl, 0, d.m.data(), 64 * 64 * sizeof(float2));
+            if (rc) return rc;
+            d.dev_m = reinterpret_cast<const float2*>(sl->dev);
+        }
+        if (d.tci) {
+            std::vector<uint8_t> w(wi8_bytes(k));
+            pack_wi8(d, w.data());
+            rc = stage_put(s, *sl, kStageW, w.data(), w.size());
+            if (rc) return rc;
+            d.dev_wi8 = reinterpret_cast<const uint8_t*>(sl->dev + kStageW);
+        }
     }
-    if (d.tci) {
-        std::vector<uint8_t> w(wi8_bytes(k));
-        pack_wi8(d, w.data());
-        CK(s, cudaStreamSynchronize(s->stream));  // the previous tensor-core launch may still read the scratch
-        CK(s, cudaMemcpyAsync(s->wi8, w.data(), w.size(), cudaMemcpyHostToDevice, s->stream));
-        CK(s, cudaStreamSynchronize(s->stream));
-        d.dev_wi8 = s->wi8;
-    }
-    return run_apply(s, d);
+    rc = run_apply(s, d);
+    if (rc) return rc;
+    return sl ? stage_release(s, *sl) : SV_OK;
 }
 
 int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k, const int32_t* targets,
                         const sv_c64* matrix) {
     int rc = check_state(s);
-    if (rc) return rc;
-    rc = materialize(s);
     if (rc) return rc;
     if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
     if (n_ctrl < 0 || n_ctrl > SV_MAX_FUSED) return fail(SV_EINVAL, "n_ctrl must be in [0, 6]");
@@ -793,7 +849,12 @@ int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k,
     for (int i = 0; i < D * D; ++i) M[i] = cd(matrix[i].re, matrix[i].im);
     int minc = s->n;
     for (int c = 0; c < n_ctrl; ++c) minc = std::min(minc, (int)controls[c]);
-    if (!s->fp64 && s->g == 0 && minc >= 1) {
+    const bool subspace = !s->fp64 && s->g == 0 && minc >= 1;
+    if (!subspace && k + n_ctrl > SV_MAX_FUSED)
+        return fail(SV_EUNSUPPORTED, "controlled gate needs k + n_ctrl <= 6 here (control on qubit 0, sharded or fp64)");
+    if (subspace) {
+        rc = materialize(s);
+        if (rc) return rc;
         // tile engine over the control-1 subspace only: 2^-n_ctrl of the state
         ApplyDesc d;
         make_apply(s->l, k, targets, M.data(), d);
@@ -802,20 +863,25 @@ int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k,
         d.tc = false;
         plan_apply(s->l, d);
         d.tc = false;
+        sv_state::StageSlot* sl = nullptr;
         if (k == 6) {
-            CK(s, cudaMemcpyAsync(s->kmat, d.m.data(), 64 * 64 * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
-            CK(s, cudaStreamSynchronize(s->stream));
-            d.dev_m = s->kmat;
+            rc = stage_acquire(s, sl);
+            if (rc == SV_OK) rc = stage_put(s, *sl, 0, d.m.data(), 64 * 64 * sizeof(float2));
+            if (rc) return rc;
+            d.dev_m = reinterpret_cast<const float2*>(sl->dev);
         }
         rc = launch(s, d.high ? LaunchClass::HIGH : LaunchClass::LOW,
                     [&] { return launch_apply(s->shard[0], s->l, d, s->stream); });
         if (rc) return rc;
+        if (sl) {
+            rc = stage_release(s, *sl);
+            if (rc) return rc;
+        }
         s->stats.bytes_apply += 16ull << (s->l - n_ctrl);
+        (d.high ? s->stats.bytes_apply_high : s->stats.bytes_apply_low) += 16ull << (s->l - n_ctrl);
         s->stats.flops_apply += (uint64_t)((8 << k) - 2) << (s->l - n_ctrl);
         return SV_OK;
     }
-    if (k + n_ctrl > SV_MAX_FUSED)
-        return fail(SV_EUNSUPPORTED, "controlled gate needs k + n_ctrl <= 6 here (control on qubit 0, sharded or fp64)");
     // dense block expansion over targets ++ controls: U on the all-ones control block, identity elsewhere
     const int kk = k + n_ctrl, DD = 1 << kk;
     std::vector<int32_t> qs(targets, targets + k);
@@ -1080,7 +1146,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         sv_circuit::Step st;
         st.type = e.type;
         if (e.type == Event::APPLY) {
-            make_apply(s->l, e.k, e.phys, plan[e.fused].M.data(), st.apply);
+            make_apply(s->l, e.k, e.phys, plan[e.fused].M.data(), st.apply, s->tc_mode);
             if (e.k == 6) ++n6;
         } else if (e.type == Event::EXCHANGE) {
             st.exch = make_exchange(s->l, e.pairs);
@@ -1091,6 +1157,31 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         c->steps.push_back(std::move(st));
     }
     flush_passes();
+    // pass-specialised kernels of every register-blocked pass (compiled in
+    // parallel, cached per process; the first pass also in its |0...0> form)
+    if (blocked && s->pass_jit) {
+        std::vector<const PassDesc*> pds;
+        std::vector<char> zs;
+        std::vector<std::vector<RpJitLaunch>*> dst;
+        for (size_t i = 0; i < c->steps.size(); ++i) {
+            auto& st = c->steps[i];
+            if (!st.block || !rpass_supported(st.pass)) continue;
+            pds.push_back(&st.pass);
+            zs.push_back(0);
+            dst.push_back(&st.jit);
+            if (i == 0) {
+                pds.push_back(&st.pass);
+                zs.push_back(1);
+                dst.push_back(&st.jitz);
+            }
+        }
+        if (!pds.empty()) {
+            std::vector<std::vector<RpJitLaunch>> got;
+            rc = rpass_jit_prepare_many(pds, s->l, zs, got);
+            if (rc) return rc;
+            for (size_t i = 0; i < got.size(); ++i) *dst[i] = std::move(got[i]);
+        }
+    }
     // int8 tensor-core W slices of every tensor-core gate: one H2D upload
     {
         size_t total = 0;
@@ -1216,6 +1307,15 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
                 const int shard = s->virt ? sh : s->rank;
                 float2* psi = s->shard[shard];
                 const bool z = zinit && &st == &c->steps[0];
+                const std::vector<RpJitLaunch>& jl = z ? st.jitz : st.jit;
+                if (!jl.empty()) {
+                    for (const auto& l : jl) {
+                        rc = launch(s, LaunchClass::HIGH,
+                                    [&] { return launch_rpass_jit(psi, s->l, l, shard == 0, s->stream); });
+                        if (rc) return rc;
+                    }
+                    continue;
+                }
                 rc = launch(s, LaunchClass::HIGH, [&] {
                     return rpass_supported(st.pass) ? launch_rpass(psi, s->l, st.pass, s->stream, z, shard == 0)
                                                     : launch_pass(psi, s->l, st.pass, s->stream);
@@ -1224,6 +1324,8 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
             }
             // algorithmic bytes: read + write, or write only when |0...0> is synthesised
             s->stats.bytes_apply += ((zinit && &st == &c->steps[0]) ? 8ull : 16ull) << s->l;
+            s->stats.bytes_apply_high += ((zinit && &st == &c->steps[0]) ? 8ull : 16ull) << s->l;
+            if (!(zinit && &st == &c->steps[0] ? st.jitz : st.jit).empty()) s->stats.n_jit_passes += 1;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
             s->stats.fma_apply += st.pass.fma_per_amp << s->l;
             s->stats.n_passes += 1;
@@ -1385,6 +1487,20 @@ int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
 }
 
 // ---- sampling --------------------------------------------------------------------
+constexpr size_t kMiscStatus = 200;  // s->misc slot of the sampling status word
+
+// Synchronise and report the status word of the last sampling call:
+// SV_EINVAL if its total weight was zero or >= 3.99 * 2^62.
+static int sample_status(sv_state* s) {
+    uint64_t st = 0;
+    if (s->sample_pending) CK(s, cudaMemcpyAsync(&st, s->misc + kMiscStatus, 8, cudaMemcpyDeviceToHost, s->stream));
+    int rc = sync(s);
+    if (rc) return rc;
+    s->sample_pending = false;
+    if (st == 1) return fail(SV_EINVAL, "state has zero total weight (no samples drawn)");
+    if (st == 2) return fail(SV_EINVAL, "sum |c|^2 >= 3.99 (uint64 overflow risk; no samples drawn)");
+    return SV_OK;
+}
 static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) {
     {
         const int rz = materialize(s);
@@ -1425,19 +1541,17 @@ static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) 
         return launch_shard_offsets(s->totals_ptr_dev, s->sigma_dev, s->world, lo, total, s->stream);
     });
     if (rc) return rc;
-    // check total weight on the host (argument validation of the result)
-    uint64_t T = 0;
-    CK(s, cudaMemcpyAsync(&T, total, 8, cudaMemcpyDeviceToHost, s->stream));
-    rc = sync(s);
-    if (rc) return rc;
-    if (T == 0) return fail(SV_EINVAL, "state has zero total weight");
-    if ((double)T >= 3.99 * 4611686018427387904.0) return fail(SV_EINVAL, "sum |c|^2 >= 3.99 (uint64 overflow risk)");
+    // the total weight is checked on the device (sample_resolve_kernel): no
+    // host round trip; an invalid total sets the status word
+    uint64_t* status = s->misc + kMiscStatus;
+    CK(s, cudaMemsetAsync(status, 0, 8, s->stream));
+    s->sample_pending = true;
     if (s->virt) {
         for (int d = 0; d < s->world; ++d) {
             const uint64_t base = (uint64_t)sig[d] << s->l;
             rc = launch(s, LaunchClass::OTHER, [&] {
                 return launch_sample_resolve(s->shard[d], s->fp64, La, s->bins + (size_t)d * nb, nb, lo + d, total, seed, N,
-                                             base, dev_out, s->stream);
+                                             base, dev_out, status, s->stream);
             });
             if (rc) return rc;
         }
@@ -1450,7 +1564,8 @@ static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) 
             // resolve samples o..o+cnt: shift the counter by o through the seed stream
             rc = launch(s, LaunchClass::OTHER, [&] {
                 return launch_sample_resolve(s->shard[s->rank], s->fp64, La, s->bins, nb, lo + s->rank, total,
-                                             seed + (uint64_t)o * 0x9E3779B97F4A7C15ull, cnt, base, s->xfer, s->stream);
+                                             seed + (uint64_t)o * 0x9E3779B97F4A7C15ull, cnt, base, s->xfer, status,
+                                             s->stream);
             });
             if (rc) return rc;
             rc = barrier(s);
@@ -1483,7 +1598,7 @@ int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out) {
     rc = sample_impl(s, seed, n_samples, s->samp_dev);
     if (rc) return rc;
     CK(s, cudaMemcpyAsync(out, s->samp_dev, n_samples * 8, cudaMemcpyDeviceToHost, s->stream));
-    return sync(s);
+    return sample_status(s);
 }
 
 // ---- whole state ------------------------------------------------------------------
@@ -1568,8 +1683,11 @@ int sv_get_state_c128(sv_state* s, sv_c128* host, size_t count) {
 }
 
 int sv_device_ptr(sv_state* s, int shard, void** out) {
-    if (!s || !out) return fail(SV_EINVAL, "NULL argument");
+    int rc = check_state(s);
+    if (rc) return rc;
+    if (!out) return fail(SV_EINVAL, "NULL argument");
     if (shard < 0 || shard >= s->world || !s->shard[shard]) return fail(SV_EINVAL, "shard not available here");
+    if (!s->virt && shard != s->rank) return fail(SV_EINVAL, "multi-process mode: only this rank's shard");
     if (s->zero_pending) {  // the caller may read the memory: write |0...0> now
         int rc = materialize(s);
         if (rc == SV_OK) rc = sync(s);
@@ -1659,6 +1777,71 @@ int sv_set_blocking(sv_state* s, int tile_bits) {
     return SV_OK;
 }
 
+int sv_set_option(sv_state* s, int option, int value) {
+    if (!s) return fail(SV_EINVAL, "state handle is NULL");
+    switch (option) {
+        case SV_OPT_BLOCK_BITS: return sv_set_blocking(s, value);
+        case SV_OPT_PASS_JIT:
+            if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_PASS_JIT takes 0 or 1");
+            s->pass_jit = value;
+            return SV_OK;
+        case SV_OPT_APPLY_PATH:
+            if (value != SV_PATH_AUTO && value != SV_PATH_SIMT && value != SV_PATH_INT8)
+                return fail(SV_EINVAL, "SV_OPT_APPLY_PATH takes SV_PATH_AUTO, SV_PATH_SIMT or SV_PATH_INT8");
+            s->tc_mode = value == SV_PATH_AUTO ? 3 : value == SV_PATH_INT8 ? 2 : 0;
+            return SV_OK;
+        case SV_OPT_TIMING: return sv_set_timing(s, value);
+        default: return fail(SV_EINVAL, "unknown option");
+    }
+}
+
+int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int tile_bits, int compile, char* buf,
+                    size_t cap, size_t* need) {
+    if (!need) return fail(SV_EINVAL, "need is NULL");
+    if (max_fused < 1 || max_fused > 2) return fail(SV_EINVAL, "max_fused must be in [1, 2] for register-blocked passes");
+    if (tile_bits < 10 || tile_bits > 13) return fail(SV_EINVAL, "tile_bits must be in [10, 13]");
+    int rc = validate_gates(gates, n_gates, -1);
+    if (rc) return rc;
+    std::vector<FusedGate> plan;
+    fuse_plan(gates, n_gates, max_fused, plan);
+    int nq = 0;
+    std::vector<PassIn> in;
+    for (auto& f : plan) {
+        build_fused_matrix(gates, f);
+        PassIn pi;
+        pi.k = f.k;
+        for (int b = 0; b < f.k; ++b) {
+            pi.q[b] = f.q[b];
+            nq = std::max(nq, f.q[b] + 1);
+        }
+        pi.M = f.M;
+        in.push_back(std::move(pi));
+    }
+    std::string all;
+    bool first = true;
+    for (auto& pd : build_passes(tile_bits, in)) {
+        if (!rpass_supported(pd)) continue;
+        for (int z = 0; z < (first ? 2 : 1); ++z) {
+            std::vector<RpJitLaunch> ls;
+            std::vector<std::string> srcs;
+            rc = rpass_jit_prepare(pd, std::max(nq, tile_bits + 2), z == 1, compile != 0, ls, &srcs);
+            if (rc) return rc;
+            for (auto& x : srcs) all += x + "\n//----\n";
+        }
+        first = false;
+    }
+    *need = all.size() + 1;
+    if (cap == 0 && !buf) return SV_OK;
+    if (cap < all.size() + 1 || !buf) return fail(SV_EINVAL, "cap too small");
+    std::memcpy(buf, all.c_str(), all.size() + 1);
+    return SV_OK;
+}
+
+int sv_jit_stats(uint64_t* compiled, uint64_t* cache_hits, double* compile_seconds) {
+    rpass_jit_counters(compiled, cache_hits, compile_seconds);
+    return SV_OK;
+}
+
 int sv_set_timing(sv_state* s, int enable) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
     s->timing = enable != 0;
@@ -1678,7 +1861,7 @@ int sv_last_stats(const sv_state* s_, sv_stats* out) {
 
 int sv_synchronize(sv_state* s) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
-    return sync(s);
+    return sample_status(s);
 }
 
 }  // extern "C"

@@ -110,3 +110,35 @@ def test_gate_struct_layout():
     g = sv.as_gates([W.Gate(0, "cz", (3, 1), W.GATE_CZ)])
     assert g.itemsize == 272 and g["nq"][0] == 2 and list(g["q"][0]) == [3, 1]
     assert g["m"][0][15] == -1 and g["m"][0][0] == 1
+
+
+PTXAS = "/usr/local/cuda/bin/ptxas"
+
+
+@pytest.mark.skipif(not os.path.exists(PTXAS), reason="ptxas not installed")
+@pytest.mark.parametrize("n,d,F,T", [(30, 14, 1, 13), (24, 14, 2, 12), (20, 10, 1, 10)])
+def test_pass_kernels_assemble(n, d, F, T, tmp_path):
+    """The PTX of every pass-specialised kernel (one per register-blocked
+    pass, plus the |0...0> form of the first) assembles for sm_100a within
+    128 registers (ptxas may spill a few loop-invariant thread constants,
+    reloaded once per tile); one kernel per pass of the block plan."""
+    import subprocess
+    gates = W.rqc(n, d)
+    srcs = sv.sv_pass_kernels(gates, F, T)
+    plan = sv.sv_block_plan(gates, F, T)
+    assert len(srcs) == len(plan) + 1
+    for i, src in enumerate(srcs[:4] + srcs[-1:]):
+        p = tmp_path / f"k{i}.ptx"
+        p.write_text(src)
+        out = subprocess.run([PTXAS, "-arch=sm_100a", "-v", str(p), "-o", str(tmp_path / f"k{i}.cubin")],
+                             capture_output=True, text=True)
+        assert out.returncode == 0, out.stderr[-2000:]
+        spill = int(re.search(r"(\d+) bytes spill stores", out.stderr).group(1))
+        assert spill <= 256, out.stderr[-800:]
+    assert "zinit" in srcs[1] and "zinit" not in srcs[0]
+
+
+def test_options_validate():
+    with pytest.raises(sv.SVError) as e:
+        sv.sv_set_option(0, sv.SV_OPT_PASS_JIT, 1)
+    assert e.value.code == sv.SV_EINVAL

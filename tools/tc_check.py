@@ -1,6 +1,8 @@
-"""Tensor-core path check (run with SVB200_TC=tf32, i8 or auto): single
-apply parity for k = 4, 5, 6 against the oracle and the per-apply norm change
-(k = 6 runs on the tensor cores with i8 / auto only; with tf32 it is SIMT).
+"""Tensor-core path check: single apply parity for k = 4, 5, 6 against the
+oracle and the per-apply norm change, on the dense-gate path given as the
+argument (sv_set_option SV_OPT_APPLY_PATH): auto (k = 5, 6 on int8 tensor
+cores), i8 (k = 4..6 on int8 tensor cores) or simt.
+usage: python tools/tc_check.py [auto|i8|simt]
 The int8 path's slicing error is relative to the group-row / column maximum,
 so its bound adds 2^(k+1) 2^-21 max_c|a| max|M| to the SIMT bound."""
 import os
@@ -13,6 +15,7 @@ import paper_conf_sc_markidis23_b200 as sv
 from oracle import sv as osv
 from workloads import rqc as W
 
+PATH = {"auto": sv.SV_PATH_AUTO, "i8": sv.SV_PATH_INT8, "simt": sv.SV_PATH_SIMT}[sys.argv[1] if len(sys.argv) > 1 else "auto"]
 U = 2.0 ** -24
 n = 16
 worst = 0.0
@@ -25,6 +28,7 @@ for k, cases in ((4, [(4, 5, 6, 7), (0, 1, 2, 3), (1, 6, 8, 11), (10, 0, 3, 5)])
         M = W.haar_unitary(1 << k, rs).astype(np.complex64)
         psi = W.random_state_c64(n, 7 + i)
         h = sv.sv_create(n)
+        sv.sv_set_option(h, sv.SV_OPT_APPLY_PATH, PATH)
         sv.sv_set_state(h, psi)
         sv.sv_apply_fused(h, list(qs), M)
         got = sv.sv_get_state(h, n).astype(np.complex128)
@@ -41,18 +45,15 @@ for k, cases in ((4, [(4, 5, 6, 7), (0, 1, 2, 3), (1, 6, 8, 11), (10, 0, 3, 5)])
         drift.append(float(np.vdot(got, got).real - np.vdot(ref, ref).real))
 print(f"TC_CHECK worst_error_over_bound={worst:.3f} mean_norm_change_per_apply={np.mean(drift):+.3e}")
 
-# whole circuits from |0..0> (many all-zero group rows early on) at F = 4, 5;
-# skipped for the biased TF32 path, whose norm loss fails the fidelity bound
+# whole circuits from |0..0> (many all-zero group rows early on) at F = 4..6
 from oracle import ref_c
-
-if os.environ.get("SVB200_TC") in ("1", "tf32"):
-    sys.exit(0)
 
 cworst = 0.0
 for nq, depth, F in ((20, 14, 5), (20, 14, 4), (18, 20, 5), (20, 14, 6), (18, 20, 6)):
     gates = W.rqc(nq, depth, 2023)
     ref = ref_c.run(nq, gates)
     h = sv.sv_create(nq)
+    sv.sv_set_option(h, sv.SV_OPT_APPLY_PATH, PATH)
     sv.sv_run_circuit(h, gates, F)
     got = sv.sv_get_state(h, nq).astype(np.complex128)
     sv.sv_destroy(h)
