@@ -91,6 +91,12 @@ struct PassDesc {
     std::vector<float> mats;  // per gate: 2^k x 2^k complex64, row-major (re, im pairs)
     uint64_t fma_per_amp = 0;  // rpass FMAs per amplitude (stats), set at circuit creation
     std::vector<int> src;      // index of each gate in the planner's input run (sv_block_plan)
+    // product-state start (first pass of a circuit run from |0...0>, pass-
+    // specialised kernels only): the first gate of every qubit, when it is a
+    // one-qubit gate, moved to time 0 (it commutes with every earlier gate),
+    // so the pass starts from prod_q v_q[bit q] with v_q = that gate's first
+    // column (identity: (1, 0)).  pinit_v: v of tile position p at [2p, 2p+1]
+    std::vector<std::complex<double>> pinit_v;
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
@@ -147,6 +153,11 @@ struct RpJitLaunch {
     std::vector<float> mats;  // float4 (mr, mr, -mi, mi) per matrix element, launch order
     size_t c0 = 0, c1 = 0;    // gate chunk
     bool zinit = false;
+    // product-state start: tile factor = tabA[u & (2^h1 - 1)] * tabB[u >> h1]
+    // (device tables owned by the circuit, complex64)
+    const float2* tabA = nullptr;
+    const float2* tabB = nullptr;
+    int h1 = 0;
 };
 // Generate (and compile unless compile == false) the kernels of one pass;
 // returns SV_OK or an error code with the message set (the compiler log).

@@ -182,9 +182,35 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 mats.push_back(mi);
             }
         }
+    // product-state start: register factors of phase 0 (32 slots) and the
+    // two vectors of every lane position (2 slots per thread bit)
+    const bool pinit = zinit && !pd.pinit_v.empty();
+    size_t reg0 = 0, lane0 = 0;
+    if (pinit) {
+        auto put = [&](std::complex<double> z) {
+            mats.push_back((float)z.real());
+            mats.push_back((float)z.real());
+            mats.push_back((float)-z.imag());
+            mats.push_back((float)z.imag());
+        };
+        const RpPhaseHost& P0 = phs[0];
+        reg0 = mats.size() / 4;
+        for (uint32_t j = 0; j < 32; ++j) {
+            std::complex<double> z = 1.0;
+            for (int b = 0; b < M; ++b) z *= pd.pinit_v[2 * P0.R[b] + ((j >> b) & 1u)];
+            put(z);
+        }
+        lane0 = mats.size() / 4;
+        for (int b = 0; b < tbits; ++b) {
+            put(pd.pinit_v[2 * P0.lanes[b]]);
+            put(pd.pinit_v[2 * P0.lanes[b] + 1]);
+        }
+    }
     nm = mats.size() / 4;
-    const size_t off_psi = std::max<size_t>(nm, 1) * 16, off_nt = off_psi + 8, off_zone = off_psi + 16;
-    const size_t pbytes = (off_zone + 4 + 15) / 16 * 16;
+    // parameter tail (rpj_jit_tail): psi, n_tiles, zone, h1, tabA, tabB
+    const size_t off_psi = std::max<size_t>(nm, 1) * 16, off_nt = off_psi + 8, off_zone = off_psi + 16,
+                 off_h1 = off_psi + 20, off_ta = off_psi + 24, off_tb = off_psi + 32;
+    const size_t pbytes = off_psi + 48;
 
     Ptx P;
     // ---- prologue: thread constants
@@ -201,6 +227,26 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         P.op("@", q, " add.s64 %dthr, %dthr, ", 8 * tm.dep(t2));
         P.op("@", q, " xor.b32 %sthr, %sthr, ", fold_swz(t2, T) << 3);
         if (direct) P.op("@", q, " add.s64 %dg, %dg, ", 8 * tm.dep(1ull << lp.lanes[b]));
+    }
+    if (pinit) {
+        // thread factor: product of the lane vectors selected by the thread index
+        P.op("mov.b64 %tf, 1065353216");  // (1.0f, 0.0f)
+        for (int b = 0; b < tbits; ++b) {
+            const std::string t = P.r32(), q = P.pr();
+            P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+            P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+            P.op("ld.param.v2.b64 {%ml, %mh}, [rpj_param_0+", 16 * (lane0 + 2 * b), "]");
+            P.op("ld.param.v2.b64 {%x0, %x1}, [rpj_param_0+", 16 * (lane0 + 2 * b + 1), "]");
+            P.op("selp.b64 %ml, %x0, %ml, ", q);
+            P.op("selp.b64 %mh, %x1, %mh, ", q);
+            P.op("mov.b64 {%lo, %hi}, %tf");
+            P.op("mov.b64 %xs0, {%hi, %lo}");
+            P.op("fma.rn.f32x2 %y, %ml, %tf, %zero");
+            P.op("fma.rn.f32x2 %tf, %mh, %xs0, %y");
+        }
+        P.op("ld.param.u32 %h1, [rpj_param_0+", off_h1, "]");
+        P.op("ld.param.u64 %tabA, [rpj_param_0+", off_ta, "]");
+        P.op("ld.param.u64 %tabB, [rpj_param_0+", off_tb, "]");
     }
     P.op("ld.param.u64 %psi, [rpj_param_0+", off_psi, "]");
     P.op("ld.param.u64 %ntiles, [rpj_param_0+", off_nt, "]");
@@ -253,7 +299,40 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("add.s32 ", t, ", ", t, ", %cur");
             return t;
         };
-        if (ph == 0 && zinit) {
+        if (ph == 0 && pinit) {
+            // tile factor from the two tables, times the thread factor
+            P.op("cvt.u64.u32 %rdA, %h1");
+            P.op("mov.b64 %rdB, 1");
+            P.op("shl.b64 %rdB, %rdB, %h1");
+            P.op("sub.s64 %rdB, %rdB, 1");
+            P.op("and.b64 %rdB, %u, %rdB");
+            P.op("shl.b64 %rdB, %rdB, 3");
+            P.op("add.s64 %rdB, %tabA, %rdB");
+            P.op("ld.global.nc.b64 %x0, [%rdB]");
+            P.op("shr.u64 %rdB, %u, %h1");
+            P.op("shl.b64 %rdB, %rdB, 3");
+            P.op("add.s64 %rdB, %tabB, %rdB");
+            P.op("ld.global.nc.b64 %x1, [%rdB]");
+            auto cmul = [&](const std::string& a, const std::string& b, const std::string& out) {  // out = a * b
+                P.op("mov.b64 {%lo, %hi}, ", b);
+                P.op("neg.f32 %nhi, %hi");
+                P.op("mov.b64 %ml, {%lo, %lo}");
+                P.op("mov.b64 %mh, {%nhi, %hi}");
+                P.op("mov.b64 {%lo, %hi}, ", a);
+                P.op("mov.b64 %xs0, {%hi, %lo}");
+                P.op("fma.rn.f32x2 %y, %ml, ", a, ", %zero");
+                P.op("fma.rn.f32x2 ", out, ", %mh, %xs0, %y");
+            };
+            cmul("%x0", "%x1", "%x2");
+            cmul("%x2", "%tf", "%x3");
+            P.op("mov.b64 {%lo, %hi}, %x3");
+            P.op("mov.b64 %xs1, {%hi, %lo}");
+            for (int j = 0; j < NA; ++j) {
+                P.op("ld.param.v2.b64 {%ml, %mh}, [rpj_param_0+", 16 * (reg0 + j), "]");
+                P.op("fma.rn.f32x2 %y, %ml, %x3, %zero");
+                P.op("fma.rn.f32x2 %a", j, ", %mh, %xs1, %y");
+            }
+        } else if (ph == 0 && zinit) {
             for (int j = 0; j < NA; ++j) P.op("mov.b64 %a", j, ", 0");
             // amplitude 0 = 1 (tile 0, thread 0, register 0) on the shard that holds it
             P.op("setp.ne.u32 %p_z, %zone, 0");
@@ -364,19 +443,24 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("bar.sync 0");
         }
     }
-    if (!direct) {  // write the tile back from shared memory
+    if (!direct) {
+        // write the tile back from shared memory: every unit into registers
+        // first, so that the next tile's load can be issued before the stores
+        // (the buffer is free once all threads have read it)
         for (int i = 0; i < UPT; ++i) {
             const std::string sa = P.r32();
             P.op("xor.b32 ", sa, ", %sthr, ", fold_swz(2u * nthr * i, T) << 3);
             P.op("add.s32 ", sa, ", ", sa, ", %cur");
-            P.op("ld.shared.v2.b64 {%x0, %x1}, [", sa, "]");
-            P.op("st.global.cs.v2.b64 ", gaddr(P, "%gcur", 8 * tm.dep(2ull * nthr * i)), ", {%x0, %x1}");
+            P.op("ld.shared.v2.b64 {%a", 2 * i, ", %a", 2 * i + 1, "}, [", sa, "]");
         }
-    }
-    if (!zinit && !early) {
-        P.op("bar.sync 0");  // every thread is done with the tile buffer
-        loadtile("%gnext", "@%p_next ");
-        P.op("cp.async.commit_group");
+        if (!zinit) {
+            P.op("bar.sync 0");  // every thread is done with the tile buffer
+            loadtile("%gnext", "@%p_next ");
+            P.op("cp.async.commit_group");
+        }
+        for (int i = 0; i < UPT; ++i)
+            P.op("st.global.cs.v2.b64 ", gaddr(P, "%gcur", 8 * tm.dep(2ull * nthr * i)), ", {%a", 2 * i, ", %a", 2 * i + 1,
+                 "}");
     }
     P.op("mov.b64 %gcur, %gnext");
     P.op("mov.b64 %gtile, %gtile_next");
@@ -389,17 +473,18 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << "// pass-specialised register-blocked kernel (generated by rpass_jit.cpp)\n";
     k << "// T=" << T << " r=" << pd.r << " n=" << n_local << " S={";
     for (int q : pd.S) k << q << ",";
-    k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (direct ? " direct" : "") << "\n";
+    k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (pinit ? " product-start" : "")
+      << (direct ? " direct" : "") << "\n";
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
     k << ".maxntid " << nthr << ", 1, 1\n.maxnreg 128\n{\n";
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z;\n";
-    k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi;\n";
+    k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
     k << "\t.reg .b64 %a<32>;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
     k << "\t.reg .b64 %y, %ml, %mh, %zero, %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, "
-         "%gnext, %gst;\n";
+         "%gnext, %gst, %tf, %tabA, %tabB, %rdA, %rdB;\n";
     k << "\tmov.b64 %zero, 0;\n";
     k << P.o.str();
     k << "}\n";
@@ -513,7 +598,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
                 l.kern->nthr = 1 << (T - 5);
                 l.kern->smem = (size_t)8 << T;
                 l.kern->nm = nm;
-                l.kern->param_bytes = (std::max<size_t>(nm, 1) * 16 + 8 + 8 + 4 + 15) / 16 * 16;  // as in gen_chunk
+                l.kern->param_bytes = std::max<size_t>(nm, 1) * 16 + 48;  // as in gen_chunk
                 todo.push_back(l.kern);
             }
             l.c0 = ch.first;
@@ -591,6 +676,9 @@ cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, boo
     std::memcpy(prm.data() + off + 8, &n_tiles, 8);
     const int zone = one_here ? 1 : 0;
     std::memcpy(prm.data() + off + 16, &zone, 4);
+    std::memcpy(prm.data() + off + 20, &l.h1, 4);
+    std::memcpy(prm.data() + off + 24, &l.tabA, 8);
+    std::memcpy(prm.data() + off + 32, &l.tabB, 8);
     void* args[] = {prm.data()};
     return cudaLaunchKernel((const void*)K.kern, dim3((unsigned)grid), dim3((unsigned)K.nthr), args, K.smem, st);
 }

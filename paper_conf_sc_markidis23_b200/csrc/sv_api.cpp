@@ -145,6 +145,12 @@ struct sv_circuit {
         std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
     };
     std::vector<Step> steps;
+    // the same circuit for runs that start from a pending |0...0>: the first
+    // gate of every qubit (a one-qubit gate) folded into a product-state
+    // first pass (PassDesc::pinit_v); empty when not applicable
+    std::vector<Step> steps_z;
+    sv_stats stats_z{};
+    float2* ptab = nullptr;  // its tile-factor tables (device, complex64)
     float2* dev_mats = nullptr;
     double* planes64 = nullptr;  // complex128 states: planes of every gate
     uint8_t* wi8 = nullptr;      // int8 tensor-core W slices of every tensor-core gate
@@ -1117,7 +1123,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     }
     // lower events to launch descriptors
     size_t n6 = 0;
-    std::vector<PassIn> run;
+    std::vector<PassIn> run, run_all;
     auto flush_passes = [&]() {
         if (run.empty()) return;
         for (auto& pd : build_passes(T, run)) {
@@ -1139,6 +1145,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             pi.k = e.k;
             pi.M.resize((size_t)1 << (2 * e.k));
             sort_matrix_qubits<cd>(e.k, e.phys, plan[e.fused].M.data(), pi.q, pi.M.data());
+            if (s->g == 0) run_all.push_back(pi);
             run.push_back(std::move(pi));
             continue;
         }
@@ -1157,22 +1164,69 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         c->steps.push_back(std::move(st));
     }
     flush_passes();
+    // product-state start (unsharded, pass-specialised kernels): the first
+    // gate of each qubit, if it is a one-qubit gate, commutes with every gate
+    // before it, so a run from |0...0> may apply all of them first -- i.e.
+    // start from the product state prod_q v_q[bit q] (v_q = that gate's first
+    // column) and skip them.  Built as a second step list (steps_z) used when
+    // the state is a pending |0...0> at run time.
+    std::vector<cd> pv;  // v_q, 2 per qubit
+    if (blocked && s->pass_jit && s->g == 0 && !run_all.empty()) {
+        pv.assign(2 * (size_t)s->n, cd(0));
+        for (int q = 0; q < s->n; ++q) pv[2 * q] = 1.0;
+        std::vector<char> seen(s->n, 0);
+        std::vector<PassIn> rest;
+        int nfold = 0;
+        for (auto& g : run_all) {
+            if (g.k == 1 && !seen[g.q[0]]) {
+                pv[2 * g.q[0]] = g.M[0];      // column 0 of the 2 x 2 matrix
+                pv[2 * g.q[0] + 1] = g.M[2];
+                ++nfold;
+            } else {
+                rest.push_back(g);
+            }
+            for (int b = 0; b < g.k; ++b) seen[g.q[b]] = 1;
+        }
+        std::vector<PassDesc> pz = (nfold && !rest.empty()) ? build_passes(T, rest) : std::vector<PassDesc>{};
+        if (!pz.empty() && rpass_supported(pz[0])) {
+            for (int p = 0; p < (int)pz[0].S.size(); ++p) {
+                pz[0].pinit_v.push_back(pv[2 * pz[0].S[p]]);
+                pz[0].pinit_v.push_back(pv[2 * pz[0].S[p] + 1]);
+            }
+            c->stats_z = c->stats;
+            c->stats_z.n_passes = 0;
+            c->stats_z.fma_apply = 0;
+            for (auto& pd : pz) {
+                pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
+                c->stats_z.fma_apply += pd.fma_per_amp << s->l;
+                c->stats_z.n_passes++;
+                sv_circuit::Step st;
+                st.type = Event::APPLY;
+                st.block = true;
+                st.pass = std::move(pd);
+                c->steps_z.push_back(std::move(st));
+            }
+        }
+    }
     // pass-specialised kernels of every register-blocked pass (compiled in
     // parallel, cached per process; the first pass also in its |0...0> form)
     if (blocked && s->pass_jit) {
         std::vector<const PassDesc*> pds;
         std::vector<char> zs;
         std::vector<std::vector<RpJitLaunch>*> dst;
-        for (size_t i = 0; i < c->steps.size(); ++i) {
-            auto& st = c->steps[i];
-            if (!st.block || !rpass_supported(st.pass)) continue;
-            pds.push_back(&st.pass);
-            zs.push_back(0);
-            dst.push_back(&st.jit);
-            if (i == 0) {
+        for (auto* list : {&c->steps, &c->steps_z}) {
+            for (size_t i = 0; i < list->size(); ++i) {
+                auto& st = (*list)[i];
+                if (!st.block || !rpass_supported(st.pass)) continue;
+                const bool z = list == &c->steps_z && i == 0;
                 pds.push_back(&st.pass);
-                zs.push_back(1);
-                dst.push_back(&st.jitz);
+                zs.push_back(z ? 1 : 0);
+                dst.push_back(z ? &st.jitz : &st.jit);
+                if (list == &c->steps && i == 0 && c->steps_z.empty()) {  // lazy |0...0> without the fold
+                    pds.push_back(&st.pass);
+                    zs.push_back(1);
+                    dst.push_back(&st.jitz);
+                }
             }
         }
         if (!pds.empty()) {
@@ -1180,6 +1234,35 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             rc = rpass_jit_prepare_many(pds, s->l, zs, got);
             if (rc) return rc;
             for (size_t i = 0; i < got.size(); ++i) *dst[i] = std::move(got[i]);
+        }
+        if (!c->steps_z.empty()) {
+            // tile-factor tables of the product-state pass: tile index bit i
+            // <-> the i-th qubit outside its tile (ascending); A over the low
+            // h1 bits, B over the rest; fp64 products rounded once
+            const PassDesc& p0 = c->steps_z[0].pass;
+            std::vector<int> out_q;
+            for (int q = 0; q < s->l; ++q)
+                if (std::find(p0.S.begin(), p0.S.end(), q) == p0.S.end()) out_q.push_back(q);
+            const int h = (int)out_q.size(), h1 = h / 2, h2 = h - h1;
+            std::vector<float2> tab(((size_t)1 << h1) + ((size_t)1 << h2));
+            for (int part = 0; part < 2; ++part) {
+                const int nb = part ? h2 : h1, b0 = part ? h1 : 0;
+                float2* t = tab.data() + (part ? ((size_t)1 << h1) : 0);
+                for (size_t x = 0; x < ((size_t)1 << nb); ++x) {
+                    cd z = 1.0;
+                    for (int i = 0; i < nb; ++i) z *= pv[2 * out_q[b0 + i] + ((x >> i) & 1)];
+                    t[x] = make_float2((float)z.real(), (float)z.imag());
+                }
+            }
+            cudaError_t e = cudaMalloc(&c->ptab, tab.size() * sizeof(float2));
+            if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(product-state tables)");
+            CK(s, cudaMemcpyAsync(c->ptab, tab.data(), tab.size() * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
+            CK(s, cudaStreamSynchronize(s->stream));
+            for (auto& l : c->steps_z[0].jitz) {
+                l.tabA = c->ptab;
+                l.tabB = c->ptab + ((size_t)1 << h1);
+                l.h1 = h1;
+            }
         }
     }
     // int8 tensor-core W slices of every tensor-core gate: one H2D upload
@@ -1266,8 +1349,12 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     // a pending |0...0> is synthesised inside the first pass when the circuit
     // starts with a register-blocked pass (no reset write, no first-pass read)
     bool zinit = false;
+    // a run from a pending |0...0> takes the product-state step list when
+    // the circuit has one (first gates folded into the first pass)
+    const bool use_z = s->zero_pending && !c->steps_z.empty();
+    const std::vector<sv_circuit::Step>& steps = use_z ? c->steps_z : c->steps;
     if (s->zero_pending) {
-        zinit = !c->small && !s->fp64 && !c->steps.empty() && c->steps[0].block && rpass_supported(c->steps[0].pass);
+        zinit = !c->small && !s->fp64 && !steps.empty() && steps[0].block && rpass_supported(steps[0].pass);
         if (zinit) {
             s->zero_pending = false;
         } else {
@@ -1301,12 +1388,12 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
         s->pos = c->pos_out;
         return SV_OK;
     }
-    for (auto& st : c->steps) {
+    for (auto& st : steps) {
         if (st.block) {
             for (int sh = 0; sh < s->local_shards(); ++sh) {
                 const int shard = s->virt ? sh : s->rank;
                 float2* psi = s->shard[shard];
-                const bool z = zinit && &st == &c->steps[0];
+                const bool z = zinit && &st == &steps[0];
                 const std::vector<RpJitLaunch>& jl = z ? st.jitz : st.jit;
                 if (!jl.empty()) {
                     for (const auto& l : jl) {
@@ -1323,9 +1410,9 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
                 if (rc) return rc;
             }
             // algorithmic bytes: read + write, or write only when |0...0> is synthesised
-            s->stats.bytes_apply += ((zinit && &st == &c->steps[0]) ? 8ull : 16ull) << s->l;
-            s->stats.bytes_apply_high += ((zinit && &st == &c->steps[0]) ? 8ull : 16ull) << s->l;
-            if (!(zinit && &st == &c->steps[0] ? st.jitz : st.jit).empty()) s->stats.n_jit_passes += 1;
+            s->stats.bytes_apply += ((zinit && &st == &steps[0]) ? 8ull : 16ull) << s->l;
+            s->stats.bytes_apply_high += ((zinit && &st == &steps[0]) ? 8ull : 16ull) << s->l;
+            if (!(zinit && &st == &steps[0] ? st.jitz : st.jit).empty()) s->stats.n_jit_passes += 1;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
             s->stats.fma_apply += st.pass.fma_per_amp << s->l;
             s->stats.n_passes += 1;
@@ -1356,8 +1443,9 @@ int sv_circuit_stats(const sv_circuit* c, sv_stats* st) {
 
 int sv_circuit_destroy(sv_circuit* c) {
     if (!c) return fail(SV_EINVAL, "circuit is NULL");
-    if (c->dev_mats || c->small_gates || c->small_mats || c->planes64 || c->q64 || c->wi8) {
+    if (c->dev_mats || c->small_gates || c->small_mats || c->planes64 || c->q64 || c->wi8 || c->ptab) {
         if (c->owner && c->owner->stream) cudaStreamSynchronize(c->owner->stream);
+        if (c->ptab) cudaFree(c->ptab);
         if (c->wi8) cudaFree(c->wi8);
         if (c->planes64) cudaFree(c->planes64);
         if (c->q64) cudaFree(c->q64);

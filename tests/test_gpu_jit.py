@@ -40,8 +40,8 @@ def _state(n, gates, F, bits, jit, world=1, lazy_zero=True):
 def test_jit_bit_identical_to_generic_rqc(bits, F):
     n, d = 21, 12
     gates = W.rqc(n, d, seed=bits + 10 * F)
-    a, sa = _state(n, gates, F, bits, jit=True)
-    b, sb = _state(n, gates, F, bits, jit=False)
+    a, sa = _state(n, gates, F, bits, jit=True, lazy_zero=False)
+    b, sb = _state(n, gates, F, bits, jit=False, lazy_zero=False)
     assert sa["n_jit_passes"] == sa["n_passes"] > 0
     assert sb["n_jit_passes"] == 0
     assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
@@ -54,22 +54,48 @@ def test_jit_mixed_kinds_vs_generic_and_oracle(bits, F):
     tile bit 0 in and out of the register set, both store paths."""
     n, m = 20, 200
     gates = _mixed_circuit(n, m, seed=7 * bits + F)
-    a, sa = _state(n, gates, F, bits, jit=True)
-    b, _ = _state(n, gates, F, bits, jit=False)
+    a, sa = _state(n, gates, F, bits, jit=True, lazy_zero=False)
+    b, _ = _state(n, gates, F, bits, jit=False, lazy_zero=False)
     assert sa["n_jit_passes"] > 0
     assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
     _check(n, layer_depth(gates), a, ref_c.run(n, gates))
 
 
-@pytest.mark.parametrize("lazy", [True, False])
-def test_jit_first_pass_zero_init_and_loaded(lazy):
-    """The first pass synthesises |0...0> (lazy reset) or loads it."""
+def test_jit_first_pass_loads_zero_state():
+    """A materialised |0...0>: the first pass loads it (bit-identical)."""
     n, d = 22, 14
     gates = W.rqc(n, d)
-    a, _ = _state(n, gates, 1, 13, jit=True, lazy_zero=lazy)
-    b, _ = _state(n, gates, 1, 13, jit=False, lazy_zero=lazy)
+    a, _ = _state(n, gates, 1, 13, jit=True, lazy_zero=False)
+    b, _ = _state(n, gates, 1, 13, jit=False, lazy_zero=False)
     assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
     _check(n, d, a, ref_c.run(n, gates))
+
+
+@pytest.mark.parametrize("n,d,F,bits", [(22, 14, 1, 13), (21, 12, 2, 12), (20, 10, 1, 10)])
+def test_jit_product_state_start_rqc(n, d, F, bits):
+    """A run from the lazy |0...0> folds the first one-qubit gate of every
+    qubit into a product-state first pass (R8): parity with the
+    oracle, and with the generic kernel (which applies every gate) within
+    the same tolerance."""
+    gates = W.rqc(n, d, seed=n)
+    a, sa = _state(n, gates, F, bits, jit=True, lazy_zero=True)
+    b, sb = _state(n, gates, F, bits, jit=False, lazy_zero=True)
+    assert sa["n_jit_passes"] == sa["n_passes"] > 0
+    assert sa["fma_apply"] < sb["fma_apply"]  # folded gates are not applied
+    ref = ref_c.run(n, gates)
+    _check(n, d, a, ref)
+    _check(n, d, b, ref)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_jit_product_state_start_mixed(seed):
+    """Mixed circuits: some qubits start with a two-qubit gate (not folded),
+    some with diagonal or permutation gates, some are never touched."""
+    n, m = 20, 120
+    gates = _mixed_circuit(n - 2, m, seed=seed)  # qubits 18, 19 untouched
+    a, sa = _state(n, gates, 1, 12, jit=True, lazy_zero=True)
+    assert sa["n_jit_passes"] > 0
+    _check(n, layer_depth(gates), a, ref_c.run(n, gates))
 
 
 @pytest.mark.parametrize("world", [2, 4])
@@ -103,19 +129,28 @@ def test_jit_kernel_cache_reuses_structure():
 
 
 def test_jit_30q_sampled_amplitudes_match_generic():
-    """Full size (30q D14, the bench workload): JIT and generic kernels give
-    the same amplitudes on a sample of 2^16 indices."""
+    """Full size (30q D14, the bench workload): from a materialised |0...0>
+    the JIT and generic kernels give bit-identical amplitudes (2^16 sampled
+    indices); from the lazy |0...0> (product-state start, the bench's step)
+    they agree within the north-star max-abs bound."""
     n, d = 30, 14
     gates = W.rqc(n, d)
     idx = np.random.default_rng(5).integers(0, 1 << n, size=1 << 16).astype(np.uint64)
-    out = []
+    out = {}
     for jit in (True, False):
-        h = sv.sv_create(n)
-        try:
-            sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, 1 if jit else 0)
-            st = sv.sv_run_circuit(h, gates, 1)
-            assert (st["n_jit_passes"] > 0) == jit
-            out.append(sv.sv_amplitudes(h, idx))
-        finally:
-            sv.sv_destroy(h)
-    assert np.array_equal(out[0].view(np.uint32), out[1].view(np.uint32))
+        for lazy in (True, False):
+            h = sv.sv_create(n)
+            try:
+                sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, 1 if jit else 0)
+                if not lazy:
+                    sv.sv_device_ptr(h)  # writes |0...0> now
+                st = sv.sv_run_circuit(h, gates, 1)
+                assert (st["n_jit_passes"] > 0) == jit
+                out[jit, lazy] = sv.sv_amplitudes(h, idx)
+            finally:
+                sv.sv_destroy(h)
+    assert np.array_equal(out[True, False].view(np.uint32), out[False, False].view(np.uint32))
+    assert np.array_equal(out[False, True].view(np.uint32), out[False, False].view(np.uint32))
+    err = np.abs(out[True, True].astype(np.complex128) - out[False, False].astype(np.complex128)).max()
+    bound = 1e-5 * 2.0 ** (-n / 2) * d
+    assert err <= bound, (err, bound)
