@@ -20,11 +20,16 @@ circuit, and drawing 10^6 samples.
             kernels) + sv_sample into host memory.
 
 N>1 (torchrun): the multi-process sharded mode (one shard per GPU, P2P
-exchanges), weak scaling with 2^30 amplitudes per GPU (n = 30 + log2 N)
-unless --qubits is given (e.g. --qubits 36 for the north star's 36q run).
+exchanges) on BASELINE configs[4]: 36 qubits at depth 20 over 4 or 8 GPUs
+(35 qubits over 2: 36 q needs 256 GiB per GPU there), strong scaling; the
+line adds "exchange" (exchange time, bytes each GPU sends, NVLink GB/s and
+fraction of 900 GB/s, and an s = 1..log2 N exchange microbenchmark).  --weak:
+2^30 amplitudes per GPU (n = 30 + log2 N) at depth 14.
 
 --impl reference: the CPU oracle (oracle/sv_ref.c, complex128, unfused,
-OpenMP on the host cores) on a bounded sample of the same workload.
+OpenMP on the host cores) on a bounded sample of the same workload: a step
+is one gate of the circuit; value = seconds per circuit from the per-gate
+means.  --cpu-full times the whole circuit on the oracle once.
 """
 from __future__ import annotations
 
@@ -59,18 +64,25 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--qubits", type=int, default=0)
-    ap.add_argument("--depth", type=int, default=14)
+    ap.add_argument("--qubits", type=int, default=0, help="0: the BASELINE config for this N (workload_size)")
+    ap.add_argument("--depth", type=int, default=0, help="0: 14 at N = 1, 20 for the sharded 35/36q runs")
+    ap.add_argument("--weak", action="store_true", help="N > 1: 2^30 amplitudes per GPU at depth 14 instead of 36q D20")
     ap.add_argument("--max-fused", type=int, default=-1,
-                    help="-1 (default): optimal over 1..6 from the fusion sweep (N=1; 4 for N>1)")
+                    help="-1 (default): optimal over 1..6 from the fusion sweep at N = 1; 1 for N > 1")
     ap.add_argument("--seed", type=int, default=2023)
+    ap.add_argument("--workload", default="rqc", choices=["rqc", "sycamore"],
+                    help="rqc: Boixo-v2 RQC (the paper's workload); sycamore: fSim + sqrt(X/Y/W) RQC (NEXT-4), "
+                         "depth = cycles")
     ap.add_argument("--samples", type=int, default=N_SAMPLES)
     ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
     ap.add_argument("--precision", type=int, default=32, choices=[32, 64], help="complex64 (32) or complex128 (64) state")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sweep", action="store_true",
                     help="skip the max_fused = 1..6 sweep (N = 1) that reports the optimal fusion")
-    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-exchange-micro", action="store_true", help="N > 1: skip the s = 1..g exchange microbenchmark")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample length of cpu_baseline")
+    ap.add_argument("--cpu-budget", type=float, default=150.0, help="--impl reference: stop after this many seconds")
+    ap.add_argument("--cpu-full", action="store_true", help="time the whole circuit on the oracle once and exit")
     return ap.parse_args()
 
 
@@ -160,53 +172,232 @@ class ClockSampler:
 
 
 # ----------------------------------------------------------------------------- CPU oracle
-def cpu_oracle_sample(n: int, gates, seconds: float):
-    """Time the oracle (unfused complex128 C simulator) on the first gates of
-    the workload circuit; extrapolate to seconds per circuit."""
+def host_info():
+    """Cores the oracle uses, CPU model and RAM of this host."""
     import psutil
 
     from oracle import ref_c
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"cores": ref_c.threads(), "cpu_model": model, "ram_gib": round(psutil.virtual_memory().total / 2 ** 30, 1),
+            "affinity": len(os.sched_getaffinity(0))}
+
+
+def cpu_oracle_small(reps: int = 5):
+    """BASELINE configs[0]: the whole 12q D14 circuit (121 gates, unfused),
+    timed `reps` times on the host cores (mean +- sigma)."""
+    from oracle import ref_c
+    gates = W.rqc(12, 14, 2023)
+    ref_c.run(12, gates)  # warm-up
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        ref_c.run(12, gates)
+        ts.append(time.perf_counter() - t0)
+    return {"workload": "rqc_12q_d14", "gates": len(gates), "value": statistics.mean(ts),
+            "std": statistics.stdev(ts) if len(ts) > 1 else 0.0, "reps": reps, "unit": "s", "kind": "oracle",
+            "sample": "measured: the whole circuit, every rep"}
+
+
+def stride_order(m: int, stride: int = 7):
+    """Gate order for a bounded sample whose every prefix is spread over the
+    whole circuit (all moments, all gate types): 0, 7, 14, ..., 1, 8, ..."""
+    return [i for o in range(stride) for i in range(o, m, stride)]
+
+
+class OracleSampler:
+    """The oracle (unfused complex128 C simulator, OpenMP on the host cores)
+    applying the workload circuit's gates one at a time on a 2^n state, in
+    stride order; per-gate times by gate size extrapolate to seconds per
+    circuit: sum over the circuit's gates of the mean time of their size."""
+
+    def __init__(self, n: int, gates):
+        from oracle import ref_c
+        from workloads.rqc import gate_arrays
+        self.n, self.gates = n, gates
+        self.L = ref_c
+        self.psi = ref_c.zero_state(n)  # first touch on all host threads
+        self.nq, self.qq, self.mat = gate_arrays(gates)
+        self.order = stride_order(len(gates))
+        self.pos = 0
+        self.t = {1: [], 2: []}
+
+    def step(self) -> float:
+        i = self.order[self.pos % len(self.order)]
+        self.pos += 1
+        k = int(self.nq[i])
+        q = np.ascontiguousarray(self.qq[i])
+        m = np.ascontiguousarray(self.mat[i])
+        t0 = time.perf_counter()
+        rc = self.L.lib().svref_apply(self.n, k, self.L._ip(q), self.L._dp(m), self.L._dp(self.psi.view(np.float64)))
+        dt = time.perf_counter() - t0
+        assert rc == 0
+        self.t[k].append(dt)
+        return dt
+
+    def circuit_seconds(self):
+        cnt = {1: int(np.sum(self.nq == 1)), 2: int(np.sum(self.nq == 2))}
+        mean = {k: (statistics.mean(v) if v else None) for k, v in self.t.items()}
+        if mean[1] is None or mean[2] is None:
+            allv = self.t[1] + self.t[2]
+            m = statistics.mean(allv)
+            return m * len(self.gates), cnt, mean
+        return cnt[1] * mean[1] + cnt[2] * mean[2], cnt, mean
+
+
+def cpu_oracle_sample(n: int, gates, seconds: float, make=None):
+    """cpu_baseline of the bench line: the oracle on the workload circuit for a
+    bounded time (gates in stride order), extrapolated to seconds per circuit
+    by gate size, next to the measured 12q D14 circuit (configs[0]) and the
+    committed full-circuit measurement of this workload, if any."""
+    import psutil
     n_eff = n
     avail = psutil.virtual_memory().available
     while n_eff > 20 and (16 << n_eff) > 0.6 * avail:
         n_eff -= 1
-    sub = W.rqc(n_eff, 14, 2023) if n_eff != n else gates
-    done, sec = ref_c.time_gates(n_eff, sub, max_seconds=seconds)
-    per_gate = sec / done
+    sub = (make(n_eff) if make else W.rqc(n_eff, 14, 2023)) if n_eff != n else gates
+    smp = OracleSampler(n_eff, sub)
+    t0 = time.perf_counter()
+    while time.perf_counter() - t0 < seconds and smp.pos < len(sub):
+        smp.step()
+    value, cnt, mean = smp.circuit_seconds()
     scale = 2.0 ** (n - n_eff)
-    value = per_gate * len(gates) * scale
-    sample = (f"first {done} of {len(sub)} unfused gates of the {n_eff}q depth-14 RQC in {sec:.1f} s "
-              f"({per_gate * 1e3:.1f} ms/gate), extrapolated x{len(gates)} gates"
+    value *= scale
+    sample = (f"{smp.pos} of {len(sub)} unfused gates of the {n_eff}q workload circuit (stride-7 order over the whole "
+              f"circuit: {len(smp.t[1])} one-qubit, {len(smp.t[2])} two-qubit) in {time.perf_counter() - t0:.1f} s; "
+              f"seconds per circuit = {cnt[1]} x {mean[1] and mean[1] * 1e3:.1f} ms + {cnt[2]} x "
+              f"{mean[2] and mean[2] * 1e3:.1f} ms (per-gate means by size)"
               + (f" x{scale:.0f} (2^{n - n_eff}: host RAM too small for 2^{n} complex128)" if scale > 1 else ""))
-    return {"value": value, "unit": "s", "cores": ref_c.threads(), "kind": "oracle", "sample": sample}
+    del smp
+    out = {"value": value, "unit": "s", "kind": "oracle", "sample": sample, "extrapolated": True}
+    out.update(host_info())
+    out["config0_12q_d14"] = cpu_oracle_small()
+    full = os.path.join(ROOT, "profiles", f"cpu_oracle_{n}q.json")
+    if os.path.exists(full):
+        out["full_circuit_measured"] = json.load(open(full))
+    return out
+
+
+def cpu_oracle_full(n: int, depth: int, seed: int):
+    """The whole circuit on the oracle, once (bench.py --cpu-full; minutes at 30 q)."""
+    from oracle import ref_c
+    gates = W.rqc(n, depth, seed)
+    psi = ref_c.zero_state(n)
+    t0 = time.perf_counter()
+    ref_c.run(n, gates, psi)
+    dt = time.perf_counter() - t0
+    out = {"workload": f"rqc_{n}q_d{depth}", "gates": len(gates), "value": dt, "unit": "s", "kind": "oracle",
+           "sample": "measured: the whole circuit once", "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime())}
+    out.update(host_info())
+    return out
 
 
 def run_reference(args):
+    """--impl reference: the oracle, as it stands, on the host cores.  A step
+    is ONE unfused gate of the workload circuit (stride order over the whole
+    circuit) on the 2^n complex128 state; value = seconds per circuit from the
+    per-gate means by gate size; ms_per_step is the measured time per step."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    n = args.qubits or (30 if args.gpus == 1 else 30 + (args.gpus.bit_length() - 1))
-    gates = W.rqc(n, args.depth, args.seed)
-    vals = []
-    last = None
+    import psutil
+    n, depth = workload_size(args, int(os.environ.get("WORLD_SIZE", "1")))
+    gates = make_gates(args, n, depth)
+    # the oracle state is complex128: shrink n until it fits the host RAM
+    # (the per-gate times then scale by 2^(n - n_eff): bandwidth-bound)
+    n_eff = n
+    while n_eff > 20 and (16 << n_eff) > 0.6 * psutil.virtual_memory().available:
+        n_eff -= 1
+    scale = 2.0 ** (n - n_eff)
+    smp = OracleSampler(n_eff, gates if n_eff == n else make_gates(args, n_eff, depth))
     for _ in range(args.warmup):
-        cpu_oracle_sample(n, gates, min(3.0, args.cpu_seconds))
-    for _ in range(args.steps):
-        last = cpu_oracle_sample(n, gates, args.cpu_seconds)
-        vals.append(last["value"])
-    v = statistics.mean(vals)
-    cfg = {"workload": f"rqc_{n}q_d{args.depth}", "n_qubits": n, "depth": args.depth,
-           "max_fused": "none (the oracle applies the gates unfused)", "seed": args.seed}
-    last["value"] = v
-    out = {"impl": "reference", "metric": f"rqc_circuit_time_{n}q_d{args.depth}", "value": v, "unit": "s",
-           "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": v * 1e3,
+        smp.step()
+    smp.t = {1: [], 2: []}
+    t0 = time.perf_counter()
+    steps = 0
+    while steps < args.steps:
+        smp.step()
+        steps += 1
+        if time.perf_counter() - t0 > args.cpu_budget:  # the run must end within minutes
+            break
+    wall = time.perf_counter() - t0
+    v, cnt, mean = smp.circuit_seconds()
+    v *= scale
+    cfg = {"workload": f"{args.workload}_{n}q_d{depth}", "n_qubits": n, "depth": depth,
+           "max_fused": "none (the oracle applies the gates unfused)", "seed": args.seed,
+           "step": "one unfused gate of the circuit on the 2^n complex128 state (stride-7 order)",
+           "steps_requested": args.steps}
+    cpu = {"value": v, "unit": "s", "kind": "oracle", "extrapolated": True,
+           "sample": f"{steps} gates in {wall:.1f} s ({len(smp.t[1])} one-qubit, {len(smp.t[2])} two-qubit); "
+                     f"{cnt[1]} x {mean[1] and mean[1] * 1e3:.1f} ms + {cnt[2]} x {mean[2] and mean[2] * 1e3:.1f} ms"
+                     + (f" on {n_eff} qubits x{scale:.0f} (2^{n - n_eff}: host RAM too small for 2^{n} complex128)"
+                        if scale > 1 else "")}
+    cpu.update(host_info())
+    out = {"impl": "reference", "metric": f"{args.workload}_circuit_time_{n}q_d{depth}", "value": v, "unit": "s",
+           "n_gpus": args.gpus, "steps": steps, "warmup": args.warmup, "ms_per_step": wall / steps * 1e3,
            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-           "data": "synthetic", "config": cfg, "cpu_baseline": last,
+           "data": "synthetic", "config": cfg, "cpu_baseline": cpu,
            "e2e": {"value": v, "unit": "s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
 
+def make_gates(args, n, depth):
+    return W.sycamore_rqc(n, depth, args.seed) if args.workload == "sycamore" else W.rqc(n, depth, args.seed)
+
+
+def workload_size(args, world: int):
+    """N = 1: BASELINE configs[1] (30q, depth 14).  N > 1: configs[4], 36q
+    depth 20 sharded over 4 / 8 GPUs and 35q at 2 GPUs (36 q needs 256 GiB
+    per GPU there); --weak: 2^30 amplitudes per GPU at depth 14."""
+    if args.qubits:
+        return args.qubits, args.depth or (14 if world == 1 else 20)
+    if world == 1:
+        return 30, args.depth or 14
+    if args.weak:
+        return 30 + (world.bit_length() - 1), args.depth or 14
+    return (35 if world == 2 else 36), args.depth or 20
+
+
 # ----------------------------------------------------------------------------- ours
+def exchange_micro(sv, h, n, world, cdev, reps=3):
+    """s = 1 .. log2(P) global qubits swapped with local ones: one
+    sv_apply_fused of an identity matrix on s currently-global logical qubits
+    triggers exactly one exchange of s pairs (then a local apply).  The
+    exchange kernel's own CUDA-event time (t_exchange_dev_s) gives GB/s sent
+    per GPU = (1 - 2^-s) * 8 * 2^(n - g) bytes / time."""
+    import torch
+    g = world.bit_length() - 1
+    l = n - g
+    out = {}
+    sv.sv_set_timing(h, True)
+    for s_ in range(1, g + 1):
+        ts = []
+        for _ in range(reps + 1):
+            pos = sv.sv_qubit_map(h, n)
+            glob = [q for q in range(n) if pos[q] >= l][:s_]
+            M = np.eye(1 << s_, dtype=np.complex64)
+            sv.sv_last_stats(h)
+            sv.sv_apply_fused(h, glob, M)
+            st = sv.sv_last_stats(h)
+            ts.append(st["t_exchange_dev_s"])
+        t = statistics.mean(ts[1:])
+        sent = (1 - 2.0 ** -s_) * 8 * 2 ** l
+        tt = torch.tensor([t], device=cdev)
+        import torch.distributed as dist
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t = float(tt.item())
+        out[str(s_)] = {"ms": t * 1e3, "bytes_sent_per_gpu": sent, "gbs": sent / t / 1e9,
+                        "nvlink_frac": sent / t / 900e9}
+    sv.sv_set_timing(h, False)
+    return out
+
+
 def run_ours(args):
     import torch
 
@@ -221,6 +412,7 @@ def run_ours(args):
     torch.cuda.set_device(dev)
     dist = None
     cdev = "cuda"  # device of the small tensors the collectives carry
+    shared = False
     if world > 1:
         import torch.distributed as dist
         shared = world > torch.cuda.device_count()
@@ -228,8 +420,8 @@ def run_ours(args):
         # traffic then; the data path is our own P2P kernel either way
         dist.init_process_group("gloo" if shared else "nccl", **({} if shared else {"device_id": torch.device("cuda", dev)}))
         cdev = "cpu" if shared else "cuda"
-    n = args.qubits or (30 if world == 1 else 30 + (world.bit_length() - 1))
-    gates = W.rqc(n, args.depth, args.seed)
+    n, depth = workload_size(args, world)
+    gates = make_gates(args, n, depth)
     stream = torch.cuda.Stream()
     fp64 = args.precision == 64
     elem = 16 if fp64 else 8
@@ -254,7 +446,7 @@ def run_ours(args):
     # CUDA events on the launching stream, 1 warm-up + 3 timed steps each;
     # the fastest max_fused becomes the timed configuration (max_fused = -1)
     sweep = None
-    if not fp64 and (args.max_fused < 0 or (world == 1 and not args.no_sweep)):
+    if not fp64 and world == 1 and not args.no_sweep:
         sweep = {}
         for f in range(1, 7):
             c = sv.sv_circuit_create(h, gates, f)
@@ -276,16 +468,20 @@ def run_ours(args):
             sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
             sv.sv_circuit_destroy(c)
     if args.max_fused < 0:
-        best = torch.tensor([int(min(sweep, key=sweep.get)) if sweep else 4], device=cdev)
-        if dist is not None:  # every rank runs rank 0's choice (collective calls)
-            dist.broadcast(best, 0)
-        args.max_fused = int(best.item())
-        fusion_choice = "optimal over max_fused 1..6 (fusion_sweep_s)" if sweep else "4 (complex128 default)"
+        if sweep:
+            args.max_fused = int(min(sweep, key=sweep.get))
+            fusion_choice = "optimal over max_fused 1..6 (fusion_sweep_s)"
+        else:
+            args.max_fused = 1 if not fp64 else 4
+            fusion_choice = ("1 (the single-GPU optimum: register-blocked passes between the exchanges)" if not fp64
+                             else "4 (complex128 default)")
     else:
         fusion_choice = "fixed by --max-fused"
 
     # ---- device step: fused circuit resident
+    t_c0 = time.time()
     circ = sv.sv_circuit_create(h, gates, args.max_fused)
+    t_create = time.time() - t_c0
     cst = sv.sv_circuit_stats(circ)
 
     def device_step():
@@ -299,12 +495,11 @@ def run_ours(args):
     barrier()
     sv.sv_set_timing(h, True)
     sv.sv_last_stats(h)  # drain
-    t_apply = t_high = t_low = t_exch = t_other = 0.0
-    n_high = n_low = n_other = 0
-    bytes_apply = 0
-    flops = 0
-    bytes_exch = 0
-    fma = 0
+    acc = {k: 0 for k in ("t_apply_high_dev_s", "t_apply_low_dev_s", "t_exchange_dev_s", "t_other_dev_s",
+                          "n_launch_high", "n_launch_low", "n_launch_other", "bytes_apply", "bytes_apply_high",
+                          "bytes_apply_low", "flops_apply", "bytes_exchange", "fma_apply", "n_exchanges")}
+    last = None
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     with ClockSampler(dev) as clk:
         clk.wait_ready()
         start = torch.cuda.Event(enable_timing=True)
@@ -312,33 +507,37 @@ def run_ours(args):
         barrier()
         t_host0 = time.time()
         start.record(stream)
-        for _ in range(args.steps):
+        for i in range(args.steps):
+            evs[i][0].record(stream)
             device_step()
-            st = sv.sv_last_stats(h)  # syncs + collects per-launch event times of this step
-            t_high += st["t_apply_high_dev_s"]
-            t_low += st["t_apply_low_dev_s"]
-            t_exch += st["t_exchange_dev_s"]
-            t_other += st["t_other_dev_s"]
-            n_high += st["n_launch_high"]
-            n_low += st["n_launch_low"]
-            n_other += st["n_launch_other"]
-            bytes_apply += st["bytes_apply"]
-            flops += st["flops_apply"]
-            bytes_exch += st["bytes_exchange"]
-            fma += st["fma_apply"]
+            evs[i][1].record(stream)
+            last = sv.sv_last_stats(h)  # syncs + collects per-launch event times of this step
+            for k in acc:
+                acc[k] += last[k]
         end.record(stream)
         barrier()
         clk.mark(t_host0, time.time())
         time.sleep(0.15)  # let the sampler deliver the sample that covers the end of the region
     sv.sv_set_timing(h, False)
     ms = start.elapsed_time(end) / args.steps
-    # the per-step sv_last_stats sync adds a host round trip per step; report
-    # the device-side sum of our launches as well
+    per_step = [a.elapsed_time(b) for a, b in evs]
+    t_high, t_low, t_exch = acc["t_apply_high_dev_s"], acc["t_apply_low_dev_s"], acc["t_exchange_dev_s"]
     t_apply = t_high + t_low
-    ms_t = torch.tensor([ms], device=cdev)
+    ms_t = torch.tensor([ms] + per_step, device=cdev)
     if dist is not None:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
-    ms = float(ms_t.item())
+    ms = float(ms_t[0].item())
+    per_step = [float(x) for x in ms_t[1:].tolist()]
+    ex_t = torch.tensor([t_exch], device=cdev)
+    if dist is not None:
+        dist.all_reduce(ex_t, op=dist.ReduceOp.MAX)
+    t_exch_max = float(ex_t.item())
+
+    # ---- exchange microbenchmark (N > 1)
+    micro = None
+    if world > 1 and not args.no_exchange_micro:
+        sv.sv_reset(h)
+        micro = exchange_micro(sv, h, n, world, cdev)
 
     # ---- end-to-end through the public API with host buffers
     host_samples = np.empty(args.samples, dtype=np.uint64)
@@ -372,84 +571,107 @@ def run_ours(args):
     h2d = int(max(g_arr.nbytes, sum(8 * (1 << (2 * k)) * c for k, c in enumerate(cst["fused_hist"]))))
 
     peak, peak_src = load_peaks()
-    launches_apply = n_high + n_low
-    avg_launch = t_apply / max(launches_apply, 1)
-    bytes_per_launch = 2 * elem * (1 << (n - (world.bit_length() - 1)))
+    steps = max(args.steps, 1)
+    launches_apply = acc["n_launch_high"] + acc["n_launch_low"]
+    g = world.bit_length() - 1
+    bytes_per_launch = 2 * elem * (1 << (n - g))
     # algorithmic bytes the library counted for these launches (16 B per
-    # amplitude per pass; 8 B for a first pass that synthesises |0...0>)
-    achieved = (bytes_apply / t_apply / 1e9) if t_apply > 0 and bytes_apply else (
-        bytes_per_launch / avg_launch / 1e9 if avg_launch > 0 else None)
+    # amplitude per pass; 8 B for a first pass that synthesises its tiles)
+    achieved = acc["bytes_apply"] / t_apply / 1e9 if t_apply > 0 and acc["bytes_apply"] else None
     frac = achieved / peak if achieved else None
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
-            cpu = cpu_oracle_sample(n, gates, args.cpu_seconds)
+            cpu = cpu_oracle_sample(n, gates, args.cpu_seconds, lambda m: make_gates(args, m, depth))
         except Exception as ex:  # host RAM / build issues must not kill the bench line
-            cpu = {"value": None, "unit": "s", "cores": os.cpu_count(), "kind": "oracle",
-                   "sample": f"failed: {ex}"}
+            cpu = {"value": None, "unit": "s", "cores": os.cpu_count(), "kind": "oracle", "sample": f"failed: {ex}"}
+    jit = sv.sv_jit_stats()
     if rank == 0:
         sv_fused = cst["n_fused"]
+        exch_bytes = acc["bytes_exchange"] / steps
+        fma = acc["fma_apply"]
+        smax = clk.summary().get("sm_max_mhz") or 1965
         out = {
-            "metric": f"rqc_circuit_time_{n}q_d{args.depth}" + ("_c128" if fp64 else ""),
+            "metric": f"{args.workload}_circuit_time_{n}q_d{depth}" + ("_c128" if fp64 else ""),
             "value": ms / 1e3,
             "unit": "s",
             "n_gpus": world,
             "steps": args.steps,
             "warmup": args.warmup,
             "ms_per_step": ms,
+            "value_std": statistics.stdev(per_step) / 1e3 if len(per_step) > 1 else 0.0,
+            "step_ms": per_step,
             "higher_is_better": False,
-            "scaling": "weak",
+            "scaling": "weak" if (world == 1 or args.weak) else "strong",
             "vs_baseline": None,
             "dtype": "f64" if fp64 else "f32",
             "data": "synthetic",
             "config": {
-                "workload": f"rqc_{n}q_d{args.depth}",
-                "n_qubits": n, "depth": args.depth, "max_fused": args.max_fused, "fusion": fusion_choice,
-                "execution": ("register-blocked passes (apply_rpass), tile qubits "
-                              f"{cst.get('block_bits', 12)}" if cst.get("n_passes", 0) else "one launch per fused gate"),
+                "workload": f"{args.workload}_{n}q_d{depth}",
+                "n_qubits": n, "depth": depth, "max_fused": args.max_fused, "fusion": fusion_choice,
+                "execution": ("register-blocked passes (pass-specialised kernels), tile qubits "
+                              f"{cst.get('block_bits', 13)}" if cst.get("n_passes", 0) else "one launch per fused gate"),
                 "seed": args.seed,
                 "gates": len(gates), "n_fused": sv_fused, "fused_hist": cst["fused_hist"],
                 "samples_per_step": args.samples,
-                "step": "sv_reset + all fused-gate applies + sv_sample_device(1e6)",
+                "step": "sv_reset + all fused-gate applies (+ exchanges) + sv_sample_device(1e6)",
                 "l2": f"inputs larger than L2 (state {elem << n >> 30} GiB per circuit)",
-                "parallelism": "single GPU" if world == 1 else f"sharded x{world} (P2P exchange)",
-                "apply_ms_per_step": 1e3 * t_apply / args.steps,
-                "apply_high_ms_per_step": 1e3 * t_high / args.steps,
-                "apply_low_ms_per_step": 1e3 * t_low / args.steps,
-                "exchange_ms_per_step": 1e3 * t_exch / args.steps,
-                "other_ms_per_step": 1e3 * t_other / args.steps,
-                "apply_gbs_high": bytes_per_launch * n_high / t_high / 1e9 if t_high else None,
-                "apply_gbs_low": bytes_per_launch * n_low / t_low / 1e9 if t_low else None,
-                "apply_tflops": flops / t_apply / 1e12 if t_apply else None,
+                "parallelism": "single GPU" if world == 1 else
+                               f"sharded x{world} by the top {g} physical qubits (P2P exchange kernel over CUDA-IPC"
+                               f"-mapped peer memory){' -- ranks SHARE GPUs: timing not meaningful' if shared else ''}",
+                "passes_per_step": last["n_passes"] if last else None,
+                "jit_passes_per_step": last["n_jit_passes"] if last else None,
+                "apply_ms_per_step": 1e3 * t_apply / steps,
+                "apply_high_ms_per_step": 1e3 * t_high / steps,
+                "apply_low_ms_per_step": 1e3 * t_low / steps,
+                "exchange_ms_per_step": 1e3 * t_exch_max / steps,
+                "other_ms_per_step": 1e3 * acc["t_other_dev_s"] / steps,
+                "apply_gbs_high": acc["bytes_apply_high"] / t_high / 1e9 if t_high else None,
+                "apply_gbs_low": acc["bytes_apply_low"] / t_low / 1e9 if t_low else None,
+                "apply_tflops": acc["flops_apply"] / t_apply / 1e12 if t_apply else None,
                 "fuse_plan_upload_s": cst["t_fuse_s"] + cst["t_plan_s"] + cst["t_upload_s"],
-                "apply_launches_per_step": launches_apply // max(args.steps, 1),
+                "circuit_create_s": t_create,
+                "pass_kernels_compiled": jit["compiled"], "pass_kernel_compile_s": jit["compile_s"],
+                "apply_launches_per_step": launches_apply // steps,
                 "block_bits": args.block_bits,
             },
             "roofline": {"bound": "hbm",
-                         "kernel": ("apply_rpass (register-blocked pass: all gates of a pass per HBM read+write)"
-                                    if cst["n_passes"] else "apply_high+apply_low (one launch per fused gate)"),
+                         "kernel": ("rpj (pass-specialised register-blocked pass: all gates of a pass per HBM "
+                                    "read + write)" if cst["n_passes"] else "apply_high+apply_low (one launch per fused gate)"),
                          "achieved": achieved, "peak": peak,
                          "peak_source": peak_src, "unit": "GB/s", "frac": frac,
                          "frac_of_8tbs": achieved / 8000.0 if achieved else None,
                          "algorithmic_bytes_per_launch": bytes_per_launch,
-                         "algorithmic_bytes_per_step": bytes_apply // max(args.steps, 1),
+                         "algorithmic_bytes_per_step": acc["bytes_apply"] // steps,
                          "traffic": load_traffic("rpass" if cst["n_passes"] else "apply"),
                          # the blocked passes are bound by HBM and the FP32 pipe
                          # together: the FMA-pipe share of the same launches
                          # (fp32 FMAs executed / (148 SMs x 128 FMA/clk x max clock))
                          "fma_pipe": ({"achieved_tfma_s": fma / t_apply / 1e12,
-                                       "peak_tfma_s": 148 * 128 * (clk.summary().get("sm_max_mhz") or 1965) * 1e6 / 1e12,
-                                       "frac": fma / t_apply / (148 * 128 * (clk.summary().get("sm_max_mhz") or 1965) * 1e6)}
+                                       "peak_tfma_s": 148 * 128 * smax * 1e6 / 1e12,
+                                       "frac": fma / t_apply / (148 * 128 * smax * 1e6)}
                                       if fma and t_apply else None)},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_ms / 1e3, "unit": "s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": 8 * args.samples},
-            "gpu_launches": (n_high + n_low + n_other),
+            "gpu_launches": (acc["n_launch_high"] + acc["n_launch_low"] + acc["n_launch_other"]),
             "fusion_sweep_s": sweep,
             "optimal_fusion": (None if not sweep else
                                {"max_fused": int(min(sweep, key=sweep.get)), "value": min(sweep.values()), "unit": "s"}),
             "clocks": clk.summary(),
         }
+        if world > 1:
+            # NVLink: bytes each GPU sends per step over its exchanges' time
+            # (kernel CUDA events, max over ranks) against 900 GB/s per direction
+            out["exchange"] = {
+                "exchanges_per_step": acc["n_exchanges"] / steps,
+                "bytes_exchange_per_step": exch_bytes,
+                "exchange_ms_per_step": 1e3 * t_exch_max / steps,
+                "nvlink_gbs": exch_bytes / (t_exch_max / steps) / 1e9 if t_exch_max else None,
+                "nvlink_frac": exch_bytes / (t_exch_max / steps) / 900e9 if t_exch_max else None,
+                "nvlink_peak_gbs": 900.0,
+                "micro": micro,
+            }
         print(json.dumps(out), flush=True)
     sv.sv_circuit_destroy(circ)
     sv.sv_destroy(h)
@@ -460,7 +682,10 @@ def run_ours(args):
 
 def main():
     args = parse()
-    if args.impl == "reference":
+    if args.cpu_full:
+        n, depth = workload_size(args, int(os.environ.get("WORLD_SIZE", "1")))
+        print(json.dumps(cpu_oracle_full(n, depth, args.seed)), flush=True)
+    elif args.impl == "reference":
         run_reference(args)
     else:
         run_ours(args)

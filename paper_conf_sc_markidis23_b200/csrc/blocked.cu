@@ -1026,11 +1026,10 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
     std::vector<RpPhaseHost> out;
     std::vector<int> rem;
     for (size_t g = g0; g < g1; ++g) rem.push_back((int)g);
-    auto gmask = [&](int g) {
-        uint32_t m = 0;
-        for (int b = 0; b < pd.gates[g].k; ++b) m |= 1u << pd.gates[g].pos[b];
-        return m;
-    };
+    std::vector<uint32_t> gm(pd.gates.size(), 0);
+    for (size_t g = g0; g < g1; ++g)
+        for (int b = 0; b < pd.gates[g].k; ++b) gm[g] |= 1u << pd.gates[g].pos[b];
+    auto gmask = [&](int g) { return gm[g]; };
     // CZ-like gates run in any layout (their qubits may be thread bits)
     std::vector<char> anyl(pd.gates.size(), 0);
     for (size_t g = g0; g < g1; ++g) anyl[g] = gate_kind(pd, pd.gates[g]) == 2;
@@ -1043,12 +1042,20 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
         // 0..2 = bits 1..3: direct-store layout)
         uint32_t used = 0;
         int best = -1;
+        // remaining gates as flat arrays (the subset loop below is the hot spot)
+        std::vector<uint32_t> rm(rem.size());
+        std::vector<char> ra(rem.size());
+        for (size_t i = 0; i < rem.size(); ++i) {
+            rm[i] = gm[rem[i]];
+            ra[i] = anyl[rem[i]];
+        }
+        const size_t nr = rem.size();
         for (uint32_t R = (1u << M) - 1u; R < (1u << T);) {
             int cnt = 0;
             uint32_t blocked = 0;
-            for (int g : rem) {
-                const uint32_t m = gmask(g);
-                if (!(m & blocked) && (anyl[g] || !(m & ~R))) ++cnt;
+            for (size_t i = 0; i < nr; ++i) {
+                const uint32_t m = rm[i];
+                if (!(m & blocked) && (ra[i] || !(m & ~R))) ++cnt;
                 else blocked |= m;
             }
             const int score = 4 * cnt + ((R & 1u) ? 2 : 0) + ((R & 0xEu) ? 0 : 1);

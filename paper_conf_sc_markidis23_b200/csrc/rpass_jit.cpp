@@ -35,6 +35,7 @@
 namespace svb {
 
 struct RpJitKernel {
+    std::string key;  // chunk_key (cache key)
     std::string src;  // PTX
     int nthr = 0;
     size_t smem = 0;
@@ -139,10 +140,34 @@ void emit_tbase(Ptx& P, const std::vector<int>& S, int n_local, const std::strin
     }
 }
 
+// Structural key of a launch chunk: everything the PTX text depends on
+// (tile, state size, flags and every gate's size, positions and kind).
+std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit) {
+    std::string k;
+    k.reserve(16 + 8 * (g1 - g0));
+    auto put = [&](int v) {
+        k += std::to_string(v);
+        k += ',';
+    };
+    put(n_local);
+    put(pd.r);
+    put(zinit ? 1 : 0);
+    put(zinit && !pd.pinit_v.empty() ? 1 : 0);
+    for (int q : pd.S) put(q);
+    k += '|';
+    for (size_t g = g0; g < g1; ++g) {
+        const PassGate& pg = pd.gates[g];
+        put(pg.k * 16 + gate_kind(pd, pg));
+        for (int b = 0; b < pg.k; ++b) put(pg.pos[b]);
+    }
+    return k;
+}
+
 // PTX of one launch chunk [g0, g1) of pass pd; nm receives the number of
-// float4 matrix slots, mats their values (launch order).
+// float4 matrix slots, mats their values (launch order).  emit == false:
+// only nm and mats (the PTX is cached under chunk_key).
 std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
-                      std::vector<float>& mats) {
+                      std::vector<float>& mats, bool emit = true) {
     constexpr int M = 5, NA = 32, UPT = 16;
     const int T = (int)pd.S.size();
     const int tbits = T - M;
@@ -211,6 +236,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     const size_t off_psi = std::max<size_t>(nm, 1) * 16, off_nt = off_psi + 8, off_zone = off_psi + 16,
                  off_h1 = off_psi + 20, off_ta = off_psi + 24, off_tb = off_psi + 32;
     const size_t pbytes = off_psi + 48;
+    if (!emit) return std::string();
 
     Ptx P;
     // ---- prologue: thread constants
@@ -524,25 +550,25 @@ int compile_one(RpJitKernel& K, int dev, std::string& log) {
     return SV_OK;
 }
 
-// find or create the cache entry of a source; `fresh` = needs compiling
-std::shared_ptr<RpJitKernel> lookup(const std::string& src, bool& fresh) {
+// find or create the cache entry of a chunk key; `fresh` = needs compiling
+std::shared_ptr<RpJitKernel> lookup(const std::string& key, bool& fresh) {
     std::lock_guard<std::mutex> lk(g_cache_mu);
-    auto it = g_cache.find(src);
+    auto it = g_cache.find(key);
     if (it != g_cache.end()) {
         fresh = false;
         g_hits++;
         return it->second;
     }
     auto K = std::make_shared<RpJitKernel>();
-    K->src = src;
-    g_cache[src] = K;
+    K->key = key;
+    g_cache[key] = K;
     fresh = true;
     return K;
 }
 
-void drop(const std::string& src) {
+void drop(const std::string& key) {
     std::lock_guard<std::mutex> lk(g_cache_mu);
-    g_cache.erase(src);
+    g_cache.erase(key);
 }
 
 }  // namespace
@@ -591,10 +617,11 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
             RpJitLaunch l;
             size_t nm = 0;
             const bool z = zinit[i] && first;
-            const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
             bool fresh = false;
-            l.kern = lookup(src, fresh);
+            l.kern = lookup(chunk_key(pd, n_local, ch.first, ch.second, z), fresh);
+            gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats, false);
             if (fresh) {
+                l.kern->src = gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
                 l.kern->nthr = 1 << (T - 5);
                 l.kern->smem = (size_t)8 << T;
                 l.kern->nm = nm;
@@ -613,7 +640,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) {
         cudaGetLastError();
-        for (auto& K : todo) drop(K->src);
+        for (auto& K : todo) drop(K->key);
         return fail(SV_ECUDA, "no CUDA device for the pass kernels");
     }
     std::atomic<size_t> next{0};
@@ -640,7 +667,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     for (auto& t : th) t.join();
     cudaSetDevice(dev);
     if (failed) {
-        for (auto& K : todo) drop(K->src);
+        for (auto& K : todo) drop(K->key);
         return fail(SV_ECUDA, "PTX JIT of a pass kernel failed: " + first_log.substr(0, 2000));
     }
     return SV_OK;

@@ -315,3 +315,24 @@ def test_reset_is_exact_for_every_reader():
     finally:
         sv.sv_destroy(h)
     _check(n, 8, got, ref_c.run(n, gates))
+
+
+# ------------------------------------------------ Sycamore-style RQC (NEXT-4)
+@pytest.mark.parametrize("F", range(7))
+def test_sycamore_all_fusion_sizes(F):
+    """fSim(pi/2, pi/6) + sqrt(X/Y/W) circuits: the default path for each
+    fusion size (register-blocked passes for F <= 2 at n >= 20)."""
+    n, cyc = 22, 12
+    gates = W.sycamore_rqc(n, cyc, seed=F)
+    got, st = _run(n, gates, F)
+    _check(n, 2 * cyc + 1, got, ref_c.run(n, gates))
+
+
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("F", [1, 4])
+def test_sycamore_virtual_shards(world, F):
+    n, cyc = 20, 10
+    gates = W.sycamore_rqc(n, cyc, seed=world)
+    got, st = _run(n, gates, F, world=world)
+    assert st["n_exchanges"] >= 1
+    _check(n, 2 * cyc + 1, got, ref_c.run(n, gates))

@@ -44,6 +44,8 @@ def _circuits():
     yield "rqc30", W.rqc(30, 14)
     yield "rqc36", W.rqc(36, 20)
     yield "rand", W.random_circuit(11, 200, 5, two_qubit_frac=0.4)
+    yield "syc30", W.sycamore_rqc(30, 14)
+    yield "syc36", W.sycamore_rqc(36, 20)
 
 
 @pytest.mark.parametrize("F", range(7))

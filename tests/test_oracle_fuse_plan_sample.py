@@ -35,6 +35,19 @@ def test_fused_equals_unfused_rqc(F):
     assert np.abs(_sim_fused(n, fuse.fuse(gates, F)) - ref).max() < 1e-12
 
 
+@pytest.mark.parametrize("F", range(7))
+def test_fused_equals_unfused_sycamore(F):
+    """NEXT-4 workload: fSim gates stand alone at F = 1 and absorb their
+    neighbours' single-qubit gates from F = 2 on."""
+    n = 10
+    gates = W.sycamore_rqc(n, 8, seed=3)
+    ref = sv.simulate(n, gates)
+    fz = fuse.fuse(gates, F)
+    assert np.abs(_sim_fused(n, fz) - ref).max() < 1e-12
+    if F == 1:
+        assert sum(len(Q) == 2 for Q, _, _ in fz) == sum(x.name == "fs" for x in gates)
+
+
 @pytest.mark.parametrize("F,seed", [(1, 0), (2, 1), (3, 2), (4, 3), (5, 4), (6, 5)])
 def test_fused_equals_unfused_random(F, seed):
     n = 9

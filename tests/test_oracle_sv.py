@@ -192,3 +192,41 @@ def test_appendix_c_rqc12_state():
     for i, (re, im) in g["psi"].items():
         assert abs(psi[int(i)] - complex(re, im)) < 1e-15
     assert abs((1 << g["n"]) * np.sum(np.abs(psi) ** 4) - g["two_n_sum_p2"]) < 1e-6
+
+
+# ------------------------------------------- Sycamore-style gates (NEXT-4)
+@pytest.mark.parametrize("name", ["hz_1_2", "fs"])
+def test_sycamore_gates_unitary(name):
+    g = W.GATE_TABLE[name]
+    assert np.abs(g.conj().T @ g - np.eye(g.shape[0])).max() < 1e-15
+
+
+def test_sycamore_gate_identities():
+    """sqrt(W)^2 = W with W = (X + Y)/sqrt(2) (so W^2 = I); the fSim closed
+    form: fSim(0, 0) = I, fSim(theta, phi) maps |01> -> cos|01> - i sin|10>,
+    |11> -> e^{-i phi}|11> and is symmetric in its two qubits."""
+    Wm = (W.GATE_X + W.GATE_Y) / math.sqrt(2)
+    assert np.abs(W.GATE_W - Wm).max() < 1e-15
+    assert np.abs(W.GATE_W @ W.GATE_W - np.eye(2)).max() < 1e-15
+    assert np.abs(W.GATE_SQRT_W @ W.GATE_SQRT_W - W.GATE_W).max() < 1e-15
+    assert np.abs(W.gate_fsim(0, 0) - np.eye(4)).max() == 0
+    th, ph = 0.7, 1.3
+    f = W.gate_fsim(th, ph)
+    e01 = np.array([0, 1, 0, 0], complex)
+    assert np.abs(f @ e01 - np.array([0, math.cos(th), -1j * math.sin(th), 0])).max() < 1e-15
+    assert abs(f[3, 3] - np.exp(-1j * ph)) < 1e-15
+    swap = W.GATE_SWAP
+    assert np.abs(swap @ f @ swap - f).max() < 1e-15
+    # the Sycamore gate: iSWAP-like exchange with a pi/6 conditional phase
+    syc = W.GATE_FSIM_SYC
+    assert abs(syc[1, 2] + 1j) < 1e-15 and abs(syc[1, 1]) < 1e-15 and abs(syc[3, 3] - np.exp(-1j * np.pi / 6)) < 1e-15
+
+
+def test_sycamore_circuit_brute_force():
+    """A 9-qubit, 6-cycle Sycamore-style circuit: oracle state = first column
+    of the brute-force circuit unitary; the C oracle agrees."""
+    gates = W.sycamore_rqc(9, 6, seed=4)
+    u = sv.full_circuit_unitary(9, gates)
+    psi = sv.simulate(9, gates)
+    assert np.abs(psi - u[:, 0]).max() < 1e-12
+    assert np.abs(ref_c.run(9, gates) - psi).max() < 1e-13

@@ -4,6 +4,7 @@ import json
 import os
 from collections import Counter
 
+import numpy as np
 import pytest
 
 from workloads import rqc as W
@@ -58,3 +59,42 @@ def test_qsim_text_roundtrip():
     gates = W.rqc(12, 14)
     n, back = W.from_qsim_text(W.to_qsim_text(12, gates))
     assert n == 12 and [(x.time, x.name, x.qubits) for x in back] == [(x.time, x.name, x.qubits) for x in gates]
+
+
+@pytest.mark.parametrize("n,cycles", [(12, 8), (30, 14), (36, 20)])
+def test_sycamore_structure(n, cycles):
+    """NEXT-4 generator rules: a single-qubit layer on every qubit each cycle
+    and at the end, never the same gate twice in a row on a qubit; fSim on
+    grid neighbours of pattern ABCDCDAB[cycle % 8], disjoint within a cycle."""
+    gates = W.sycamore_rqc(n, cycles)
+    sites = W.grid_sites(n)
+    last = {}
+    for t in range(2 * cycles + 1):
+        layer = [x for x in gates if x.time == t]
+        if t % 2 == 0:
+            assert sorted(x.qubits[0] for x in layer) == list(range(n))
+            for x in layer:
+                assert x.name in ("x_1_2", "y_1_2", "hz_1_2") and last.get(x.qubits[0]) != x.name
+                last[x.qubits[0]] = x.name
+        else:
+            letter = "ABCDCDAB"[(t // 2) % 8]
+            used = [q for x in layer for q in x.qubits]
+            assert len(used) == len(set(used))
+            assert [tuple(x.qubits) for x in layer] == W._syc_couplers(sites, letter)
+            for x in layer:
+                (r0, c0), (r1, c1) = sites[x.qubits[0]], sites[x.qubits[1]]
+                assert (r1 - r0, c1 - c0) == ((1, 0) if letter in "AB" else (0, 1))
+                assert x.name == "fs"
+
+
+def test_sycamore_patterns_cover_every_edge_once():
+    sites = W.grid_sites(30)
+    allp = [p for L in "ABCD" for p in W._syc_couplers(sites, L)]
+    assert len(allp) == len(set(allp)) == 5 * 5 + 4 * 6  # 5x6 grid: 25 horizontal, 24 vertical edges
+
+
+def test_sycamore_qsim_text_roundtrip():
+    gates = W.sycamore_rqc(12, 4)
+    n, back = W.from_qsim_text(W.to_qsim_text(12, gates))
+    assert n == 12 and [(x.name, x.qubits) for x in back] == [(x.name, x.qubits) for x in gates]
+    assert all(np.abs(a.matrix - b.matrix).max() < 1e-15 for a, b in zip(gates, back))

@@ -71,6 +71,26 @@ GATE_CX = np.array([[1, 0, 0, 0], [0, 0, 0, 1], [0, 0, 1, 0], [0, 1, 0, 0]], dty
 GATE_SWAP = np.array([[1, 0, 0, 0], [0, 0, 1, 0], [0, 1, 0, 0], [0, 0, 0, 1]], dtype=np.complex128)
 
 
+# Sycamore-style RQC gates (ref [3] of the paper, Arute
+# et al. 2019, cited at PAPER.md L145/L169 -- the gate set is [not in paper]):
+# sqrt(X), sqrt(Y), sqrt(W) with W = (X + Y)/sqrt(2), each P^(1/2) =
+# (1+i)/2 I + (1-i)/2 P for a Pauli-like P (P^2 = I); and fSim(theta, phi)
+# on |00>, |01>, |10>, |11>.
+GATE_SQRT_X = GATE_X_1_2
+GATE_SQRT_Y = GATE_Y_1_2
+GATE_W = np.array([[0, np.exp(-1j * np.pi / 4)], [np.exp(1j * np.pi / 4), 0]], dtype=np.complex128)
+GATE_SQRT_W = 0.5 * (1 + 1j) * np.eye(2, dtype=np.complex128) + 0.5 * (1 - 1j) * GATE_W
+
+
+def gate_fsim(theta: float, phi: float) -> np.ndarray:
+    c, s_ = math.cos(theta), math.sin(theta)
+    return np.array([[1, 0, 0, 0], [0, c, -1j * s_, 0], [0, -1j * s_, c, 0], [0, 0, 0, np.exp(-1j * phi)]],
+                    dtype=np.complex128)
+
+
+GATE_FSIM_SYC = gate_fsim(math.pi / 2, math.pi / 6)
+
+
 def gate_cp(phi: float) -> np.ndarray:
     """Controlled phase diag(1,1,1,e^{i phi})."""
     return np.diag([1, 1, 1, np.exp(1j * phi)]).astype(np.complex128)
@@ -88,6 +108,8 @@ GATE_TABLE = {
     "s": GATE_S,
     "cx": GATE_CX,
     "swap": GATE_SWAP,
+    "hz_1_2": GATE_SQRT_W,  # qsim's name of sqrt(W)
+    "fs": GATE_FSIM_SYC,    # fSim(pi/2, pi/6), the Sycamore two-qubit gate
 }
 
 
@@ -206,6 +228,59 @@ def rqc(n: int, depth: int, seed: int = 2023) -> List[Gate]:
     return gates
 
 
+# --------------------------------------------------------------------------
+# Sycamore-style RQC (reading R9)
+# --------------------------------------------------------------------------
+_SYC_PATTERN = "ABCDCDAB"
+
+
+def _syc_couplers(sites, letter: str):
+    """Coupler pattern on the square grid: A / B = vertical edges from even /
+    odd rows, C / D = horizontal edges from even / odd columns (four disjoint
+    matchings covering every edge, as Sycamore's four diagonal patterns do)."""
+    index = {s: i for i, s in enumerate(sites)}
+    pairs = []
+    for (r, c) in sites:
+        if letter in "AB" and r % 2 == (0 if letter == "A" else 1):
+            o = (r + 1, c)
+        elif letter in "CD" and c % 2 == (0 if letter == "C" else 1):
+            o = (r, c + 1)
+        else:
+            continue
+        if o in index:
+            pairs.append((index[(r, c)], index[o]))
+    pairs.sort()
+    return pairs
+
+
+def sycamore_rqc(n: int, cycles: int, seed: int = 2023) -> List[Gate]:
+    """Sycamore-style RQC on grid_sites(n): every cycle is a layer of random
+    single-qubit gates from {sqrt(X), sqrt(Y), sqrt(W)} on all qubits (never
+    the gate the qubit had in the previous cycle; choice = candidates[(r *
+    len) >> 64] with r the next splitmix64 output, qubits ascending), then
+    fSim(pi/2, pi/6) on the couplers of pattern ABCDCDAB[cycle % 8]; a final
+    single-qubit layer follows the last cycle."""
+    sites = grid_sites(n)
+    rng = SplitMix64(seed)
+    names = ["x_1_2", "y_1_2", "hz_1_2"]
+    prev = [""] * n
+    gates: List[Gate] = []
+
+    def one_qubit_layer(t):
+        for q in range(n):
+            cand = [x for x in names if x != prev[q]]
+            name = cand[(rng.next() * len(cand)) >> 64]
+            gates.append(Gate(t, name, (q,), GATE_TABLE[name]))
+            prev[q] = name
+
+    for cyc in range(cycles):
+        one_qubit_layer(2 * cyc)
+        for a, b in _syc_couplers(sites, _SYC_PATTERN[cyc % 8]):
+            gates.append(Gate(2 * cyc + 1, "fs", (a, b), GATE_FSIM_SYC))
+    one_qubit_layer(2 * cycles)
+    return gates
+
+
 def inverse_circuit(gates: Sequence[Gate]) -> List[Gate]:
     """C^dagger: reversed order, conjugate-transposed matrices (test input)."""
     out = []
@@ -217,10 +292,12 @@ def inverse_circuit(gates: Sequence[Gate]) -> List[Gate]:
 
 
 def to_qsim_text(n: int, gates: Sequence[Gate]) -> str:
-    """qsim circuit text format: first line n, then 'time name q...'."""
+    """qsim circuit text format: first line n, then 'time name q...' (fSim:
+    'time fs q0 q1 theta phi')."""
     lines = [str(n)]
     for g in gates:
-        lines.append(" ".join([str(g.time), g.name] + [str(q) for q in g.qubits]))
+        extra = [repr(math.pi / 2), repr(math.pi / 6)] if g.name == "fs" else []
+        lines.append(" ".join([str(g.time), g.name] + [str(q) for q in g.qubits] + extra))
     return "\n".join(lines) + "\n"
 
 
@@ -231,6 +308,10 @@ def from_qsim_text(text: str) -> Tuple[int, List[Gate]]:
     gates = []
     for tok in lines[1:]:
         t, name = int(tok[0]), tok[1]
+        if name == "fs":
+            qs = (int(tok[2]), int(tok[3]))
+            gates.append(Gate(t, name, qs, gate_fsim(float(tok[4]), float(tok[5]))))
+            continue
         qs = tuple(int(x) for x in tok[2:])
         gates.append(Gate(t, name, qs, GATE_TABLE[name]))
     return n, gates
