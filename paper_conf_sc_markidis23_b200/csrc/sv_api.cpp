@@ -17,6 +17,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges for nsys / ncu --nvtx
+
 #include "kernels.h"
 #include "sv_internal.h"
 
@@ -39,6 +41,15 @@ int fail(int code, const std::string& msg) {
 }  // namespace svb
 
 namespace {
+
+// NVTX range for the duration of a scope (host side: fuse, plan, pass
+// kernels, upload, apply / exchange / sample launches)
+struct Nvtx {
+    explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+    ~Nvtx() { nvtxRangePop(); }
+    Nvtx(const Nvtx&) = delete;
+    Nvtx& operator=(const Nvtx&) = delete;
+};
 
 double now_s() {
     return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
@@ -351,6 +362,7 @@ int run_apply(sv_state* s, const ApplyDesc& d) {
 }
 
 int run_exchange(sv_state* s, const ExchangeDesc& x) {
+    Nvtx nv("sv.exchange");
     int rc = barrier(s);
     if (rc) return rc;
     rc = launch(s, LaunchClass::EXCH,
@@ -732,6 +744,7 @@ static int write_zero_state(sv_state* s) {
 static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::vector<cd>& M);
 
 int sv_apply_fused(sv_state* s, int k, const int32_t* qubits, const sv_c64* matrix) {
+    Nvtx nv("sv.apply_fused");
     int rc = check_state(s);
     if (rc) return rc;
     if (k < 1 || k > SV_MAX_FUSED) return fail(SV_EINVAL, "k must be in [1, 6]");
@@ -1045,13 +1058,18 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     if (rc) return rc;
     if (s->g > 0 && std::max(max_fused, 2) > s->l - 1) return fail(SV_EUNSUPPORTED, "fused gates wider than a shard allows");
     if (s->fp64 && max_fused > 5) return fail(SV_EUNSUPPORTED, "complex128 states support max_fused <= 5");
+    Nvtx nv("sv.circuit_create");
     std::unique_ptr<sv_circuit> c(new sv_circuit());
     c->owner = s;
     const double t0 = now_s();
     std::vector<FusedGate> plan;
-    fuse_plan(gates, n_gates, max_fused, plan);
-    for (auto& f : plan) build_fused_matrix(gates, f);
+    {
+        Nvtx nf("sv.fuse");
+        fuse_plan(gates, n_gates, max_fused, plan);
+        for (auto& f : plan) build_fused_matrix(gates, f);
+    }
     const double t1 = now_s();
+    Nvtx np_("sv.plan");
     c->stats.t_fuse_s = t1 - t0;
     c->stats.n_fused = (int)plan.size();
     for (auto& f : plan) c->stats.fused_hist[f.k]++;
@@ -1230,6 +1248,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             }
         }
         if (!pds.empty()) {
+            Nvtx nk("sv.pass_kernels");
             std::vector<std::vector<RpJitLaunch>> got;
             rc = rpass_jit_prepare_many(pds, s->l, zs, got);
             if (rc) return rc;
@@ -1339,6 +1358,7 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     if (rc) return rc;
     if (!c || c->owner != s) return fail(SV_EINVAL, "circuit is NULL or belongs to another state");
     if (s->pos != c->pos_in) return fail(SV_EINVAL, "state qubit map differs from the circuit's (sv_reset first)");
+    Nvtx nv("sv.circuit_run");
     const sv_stats keep = c->stats;
     reset_stats(s);
     s->stats.t_fuse_s = keep.t_fuse_s;
@@ -1590,6 +1610,7 @@ static int sample_status(sv_state* s) {
     return SV_OK;
 }
 static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) {
+    Nvtx nv("sv.sample");
     {
         const int rz = materialize(s);
         if (rz) return rz;
