@@ -240,6 +240,19 @@ int sv_fused_matrix(const sv_gate* gates, size_t n_gates, int max_fused, size_t 
  * final_pos (n entries, may be NULL) receives logical -> physical positions. */
 int sv_shard_plan(const int32_t* fusion_stream, size_t len, int n_qubits, int log2_world, int vmin,
                   int32_t* buf, size_t cap, size_t* need, int32_t* final_pos);
+/* The same with the diagonal exchange skip (DESIGN.md
+ * reading R10): diag[i] = mask of the logical qubits fused gate i is
+ * block-diagonal in (sv_fusion_diag_masks); such a qubit, when global, does
+ * not force an exchange, and APPLY events may then list global physical
+ * positions (each shard runs the block its device bits select). */
+int sv_shard_plan_diag(const int32_t* fusion_stream, size_t len, const uint64_t* diag, int n_qubits, int log2_world,
+                       int vmin, int32_t* buf, size_t cap, size_t* need, int32_t* final_pos);
+/* Pure host: per fused gate of sv_fusion_plan's plan, the mask of logical
+ * qubits in which its fp64 fused matrix is block-diagonal (every entry
+ * between a row and a column that differ in that qubit's bit has |entry| <=
+ * 1e-10: fp64 rounding residue of exact zeros).
+ * *need = number of fused gates; cap < *need -> SV_EINVAL. */
+int sv_fusion_diag_masks(const sv_gate* gates, size_t n_gates, int max_fused, uint64_t* out, size_t cap, size_t* need);
 /* Current logical -> physical qubit map (n entries). */
 int sv_qubit_map(const sv_state* s, int32_t* pos);
 
@@ -281,13 +294,17 @@ int sv_synchronize(sv_state* s);
  *                      SV_PATH_AUTO (default: k = 5, 6 on the exact int8
  *                      tensor-core path, k <= 4 SIMT), SV_PATH_SIMT,
  *                      SV_PATH_INT8 (int8 tensor cores for k = 4..6);
- *   SV_OPT_TIMING      = sv_set_timing.
+ *   SV_OPT_TIMING      = sv_set_timing;
+ *   SV_OPT_DIAG_SKIP   1 (default): sharded circuits (sv_circuit_create) do
+ *                      not exchange a global qubit for a fused gate that is
+ *                      block-diagonal in it (sv_shard_plan_diag); 0: plain S4.
  * Takes effect for circuits created / gates applied afterwards.  SV_EINVAL
  * for unknown options or values. */
 #define SV_OPT_BLOCK_BITS 1
 #define SV_OPT_PASS_JIT 2
 #define SV_OPT_APPLY_PATH 3
 #define SV_OPT_TIMING 4
+#define SV_OPT_DIAG_SKIP 5  /* 1 (default): sharded circuits plan with the diagonal exchange skip */
 #define SV_PATH_AUTO 0
 #define SV_PATH_SIMT 1
 #define SV_PATH_INT8 2

@@ -7,6 +7,15 @@ gate that touches a global qubit, swaps global and local qubits.  The planning
 rule (Belady pairing with a victim floor vmin) is the reading of SURVEY.md
 §8c-S4, listed in DESIGN.md (Readings).
 
+Diagonal skip (reading R10): with ``diag``
+given, a fused gate only forces an exchange for its global qubits in which it
+is NOT block-diagonal.  A gate block-diagonal in qubit q (M[r][c] == 0
+whenever bit q of r and c differ -- it commutes with Z_q, like CZ or a
+control qubit) acts on the shard whose device bit for q is x as the block
+G_x over its other qubits, so a global q needs no exchange.  Next use counts
+only non-diagonal uses.  APPLY events then list global physical bits for
+such qubits.
+
 Events: ("X", [(P_j, p_j), ...])  -- exchange: swap physical bit P_j (global,
           >= l = n-g) with physical bit p_j (local, < l), all j at once;
         ("A", i, [pos[q] for q in sorted(Q_i)]) -- apply fused gate i on those
@@ -25,23 +34,43 @@ from .sv import apply_gate
 INF = math.inf
 
 
-def plan_sharded(fused_qubits: Sequence[Sequence[int]], n: int, g: int, vmin: int = 5):
-    """S4 exactly as SURVEY.md §8c-S4 states it.  Returns (events, pos)."""
+DIAG_TOL = 1e-10  # |entry| below this counts as zero (fp64 rounding residue of exact zeros)
+
+
+def diag_qubits(Q: Sequence[int], M: np.ndarray) -> set:
+    """Qubits of a fused gate (matrix M over sorted Q, bit b <-> Q[b]) in
+    which M is block-diagonal: every entry between a row and a column that
+    differ in bit b is zero (|entry| <= DIAG_TOL: products of the fp64 gate
+    table leave ~1e-17 where the exact product has 0; reading R10)."""
+    k = len(Q)
+    out = set()
+    for b in range(k):
+        r = np.arange(1 << k)
+        differ = ((r[:, None] ^ r[None, :]) >> b) & 1
+        if not np.any(np.abs(M[differ.astype(bool)]) > DIAG_TOL):
+            out.add(Q[b])
+    return out
+
+
+def plan_sharded(fused_qubits: Sequence[Sequence[int]], n: int, g: int, vmin: int = 5, diag=None):
+    """S4 exactly as SURVEY.md §8c-S4 states it (diag: per fused gate the set
+    of its block-diagonal qubits, or None).  Returns (events, pos)."""
     l = n - g
     pos = list(range(n))
     inv = list(range(n))
     nf = len(fused_qubits)
+    uses = [set(Q) - (set(diag[i]) if diag else set()) for i, Q in enumerate(fused_qubits)]
 
     def nu(q, i):
         for j in range(i, nf):
-            if q in fused_qubits[j]:
+            if q in uses[j]:
                 return j
         return INF
 
     events = []
     for i, Qi in enumerate(fused_qubits):
         Qs = set(Qi)
-        need = [q for q in Qi if pos[q] >= l]
+        need = [q for q in Qi if pos[q] >= l and q in uses[i]]
         if need:
             glob = [inv[p] for p in range(l, n)]
             glob.sort(key=lambda q: (nu(q, i), q))
@@ -138,8 +167,38 @@ def run_sharded(n: int, g: int, fused, events, psi0: np.ndarray | None = None, e
                 pos[a], pos[b] = p, P
         else:
             _, i, phys = ev
-            psi = apply_gate(psi, n, phys, fused[i][2])
+            if any(p >= l for p in phys):
+                # diagonal skip: shard d applies the block of M selected by its
+                # device bits at the global positions, on its local bits
+                shards = [psi[d << l:(d + 1) << l].copy() for d in range(1 << g)]
+                for d in range(1 << g):
+                    loc, sub = shard_block(fused[i][2], phys, l, d)
+                    if loc:
+                        shards[d] = apply_gate(shards[d], l, loc, sub)
+                    else:
+                        shards[d] = shards[d] * sub[0, 0]
+                psi = np.concatenate(shards)
+            else:
+                psi = apply_gate(psi, n, phys, fused[i][2])
     return to_logical(psi, n, pos), pos
+
+
+def shard_block(M: np.ndarray, phys: Sequence[int], l: int, d: int):
+    """Block of M (bit b <-> phys[b]) on shard d: rows/columns whose global
+    bits (phys[b] >= l) equal d's device bits; returns (local phys, block)."""
+    k = len(phys)
+    gb = [b for b in range(k) if phys[b] >= l]
+    lb = [b for b in range(k) if phys[b] < l]
+    x = 0
+    for b in gb:
+        x |= ((d >> (phys[b] - l)) & 1) << b
+    idx = []
+    for t in range(1 << len(lb)):
+        r = x
+        for j, b in enumerate(lb):
+            r |= ((t >> j) & 1) << b
+        idx.append(r)
+    return [phys[b] for b in lb], M[np.ix_(idx, idx)]
 
 
 def to_logical(psi_phys: np.ndarray, n: int, pos: Sequence[int]) -> np.ndarray:

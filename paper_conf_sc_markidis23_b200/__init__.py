@@ -35,6 +35,7 @@ SV_OPT_BLOCK_BITS = 1
 SV_OPT_PASS_JIT = 2
 SV_OPT_APPLY_PATH = 3
 SV_OPT_TIMING = 4
+SV_OPT_DIAG_SKIP = 5
 SV_PATH_AUTO = 0
 SV_PATH_SIMT = 1
 SV_PATH_INT8 = 2
@@ -132,6 +133,9 @@ _SIGS = {
     "sv_block_plan": ([_vp, _sz, ctypes.c_int, ctypes.c_int, _i32p, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_shard_plan": ([_i32p, _sz, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i32p, _sz, ctypes.POINTER(_sz), _i32p],
                       ctypes.c_int),
+    "sv_shard_plan_diag": ([_i32p, _sz, _u64p, ctypes.c_int, ctypes.c_int, ctypes.c_int, _i32p, _sz,
+                            ctypes.POINTER(_sz), _i32p], ctypes.c_int),
+    "sv_fusion_diag_masks": ([_vp, _sz, ctypes.c_int, _u64p, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_qubit_map": ([_vp, _i32p], ctypes.c_int),
     "sv_ipc_handle": ([_vp, _vp, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_attach_peers": ([_vp, _vp, _sz], ctypes.c_int),
@@ -387,6 +391,31 @@ def sv_shard_plan(fusion_stream, n_qubits: int, log2_world: int, vmin: int = 5):
     _check(lib().sv_shard_plan(fs.ctypes.data_as(_i32p), fs.size, n_qubits, log2_world, vmin,
                                buf.ctypes.data_as(_i32p), buf.size, ctypes.byref(need), pos.ctypes.data_as(_i32p)),
            "sv_shard_plan")
+    return buf[: need.value], pos
+
+
+def sv_fusion_diag_masks(gates, max_fused: int) -> np.ndarray:
+    """Per fused gate: mask of the logical qubits its fp64 matrix is block-diagonal in."""
+    g = as_gates(gates)
+    need = _sz()
+    lib().sv_fusion_diag_masks(_ptr(g), len(g), max_fused, None, 0, ctypes.byref(need))
+    out = np.zeros(max(need.value, 1), dtype=np.uint64)
+    _check(lib().sv_fusion_diag_masks(_ptr(g), len(g), max_fused, out.ctypes.data_as(_u64p), out.size,
+                                      ctypes.byref(need)), "sv_fusion_diag_masks")
+    return out[: need.value]
+
+
+def sv_shard_plan_diag(fusion_stream, diag_masks, n_qubits: int, log2_world: int, vmin: int = 5):
+    fs = np.ascontiguousarray(fusion_stream, dtype=np.int32)
+    dm = np.ascontiguousarray(diag_masks, dtype=np.uint64)
+    need = _sz()
+    pos = np.empty(n_qubits, dtype=np.int32)
+    lib().sv_shard_plan_diag(fs.ctypes.data_as(_i32p), fs.size, dm.ctypes.data_as(_u64p), n_qubits, log2_world, vmin,
+                             None, 0, ctypes.byref(need), None)
+    buf = np.empty(max(need.value, 1), dtype=np.int32)
+    _check(lib().sv_shard_plan_diag(fs.ctypes.data_as(_i32p), fs.size, dm.ctypes.data_as(_u64p), n_qubits, log2_world,
+                                    vmin, buf.ctypes.data_as(_i32p), buf.size, ctypes.byref(need),
+                                    pos.ctypes.data_as(_i32p)), "sv_shard_plan_diag")
     return buf[: need.value], pos
 
 

@@ -1006,6 +1006,7 @@ int rpass_m() { return SVB_RP_M; }
 
 // 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
 int gate_kind(const PassDesc& pd, const PassGate& pg) {
+    if (pg.kind >= 0) return pg.kind;
     const int D = 1 << pg.k;
     const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
     bool diag = true, cz = pg.k == 2;
@@ -1152,7 +1153,8 @@ int phase_conflicts(const RpPhaseHost& ph, int T, int M) {
 }
 
 template <int M, bool F2>
-cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone) {
+cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone, int slot) {
+    const float* mats = pd.mats_shard.empty() ? pd.mats.data() : pd.mats_shard[slot].data();
     const int T = (int)pd.S.size();
     const uint32_t nthr = 1u << (T - M);
     const size_t smem = SVB_RP_STAGES * ((size_t)8 << T);
@@ -1205,7 +1207,7 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
             for (int g : h.gates) {
                 const PassGate& pg = pd.gates[g];
                 const int D = 1 << pg.k;
-                const float* mg = pd.mats.data() + pg.moff;  // (re, im) row-major
+                const float* mg = mats + pg.moff;  // (re, im) row-major
                 const int kind = gate_kind(pd, pg);
                 const int ne = kind == 1 ? D : kind == 2 ? 0 : D * D;
                 for (int e2 = 0; e2 < ne; ++e2) {
@@ -1312,11 +1314,11 @@ void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {
     if (worst_conflict) *worst_conflict = w;
 }
 
-cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone) {
+cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone, int slot) {
     static_assert(sizeof(RpassParams) <= 32764, "rpass params exceed the kernel parameter space");
     constexpr bool f2 = SVB_RP_F2 != 0;
-    if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st, zinit, zone) : launch_rpass_m<5, false>(psi, n, pd, st, zinit, zone);
-    return f2 ? launch_rpass_m<4, true>(psi, n, pd, st, zinit, zone) : launch_rpass_m<4, false>(psi, n, pd, st, zinit, zone);
+    if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st, zinit, zone, slot) : launch_rpass_m<5, false>(psi, n, pd, st, zinit, zone, slot);
+    return f2 ? launch_rpass_m<4, true>(psi, n, pd, st, zinit, zone, slot) : launch_rpass_m<4, false>(psi, n, pd, st, zinit, zone, slot);
 }
 
 }  // namespace svb

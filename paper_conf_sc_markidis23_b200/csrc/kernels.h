@@ -82,6 +82,7 @@ struct PassGate {
     int pos[4];     // tile-local positions (rank of the qubit in sorted S), ascending
     uint32_t poff;  // offset (floats) of the gate's planes P, S, Q (3 x 4^k floats)
     uint32_t moff;  // offset (floats) of the gate's matrix in PassDesc::mats
+    int kind = -1;  // gate_kind override (shard-dependent gates: the kind that fits every shard)
 };
 struct PassDesc {
     std::vector<int> S;  // qubits of the tile
@@ -89,6 +90,10 @@ struct PassDesc {
     std::vector<PassGate> gates;
     std::vector<float> planes;
     std::vector<float> mats;  // per gate: 2^k x 2^k complex64, row-major (re, im pairs)
+    // sharded runs with the diagonal exchange skip: mats of every local shard
+    // slot (a gate block-diagonal in a global qubit has a block per shard);
+    // empty when every shard runs `mats`
+    std::vector<std::vector<float>> mats_shard;
     uint64_t fma_per_amp = 0;  // rpass FMAs per amplitude (stats), set at circuit creation
     std::vector<int> src;      // index of each gate in the planner's input run (sv_block_plan)
     // product-state start (first pass of a circuit run from |0...0>, pass-
@@ -110,7 +115,7 @@ uint64_t rpass_fma_per_amp(const PassDesc& pd);
 // zero_init: the tiles are |0...0> (not loaded); one_here: this shard holds
 // amplitude 0 (= 1)
 cudaError_t launch_rpass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st, bool zero_init = false,
-                         bool one_here = false);
+                         bool one_here = false, int slot = 0);
 // Host model of the rpass phase plan (tests / tools): number of phases and
 // the worst bank-conflict degree of their gathers.
 void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict);
@@ -151,6 +156,7 @@ struct RpJitKernel;
 struct RpJitLaunch {
     std::shared_ptr<RpJitKernel> kern;
     std::vector<float> mats;  // float4 (mr, mr, -mi, mi) per matrix element, launch order
+    std::vector<std::vector<float>> mats_shard;  // per local shard slot (PassDesc::mats_shard)
     size_t c0 = 0, c1 = 0;    // gate chunk
     bool zinit = false;
     // product-state start: tile factor = tabA[u & (2^h1 - 1)] * tabB[u >> h1]
@@ -166,7 +172,8 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
 // Prepare many passes at once (compiles in parallel host threads).
 int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local, const std::vector<char>& zinit,
                            std::vector<std::vector<RpJitLaunch>>& out);
-cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st);
+cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st,
+                             int slot = 0);
 // process-wide counters (sv_jit_stats)
 void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compile_s);
 

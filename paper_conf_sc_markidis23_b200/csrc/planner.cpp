@@ -8,7 +8,15 @@
 // that sits at a global position, an EXCHANGE swaps physical bits (P_j, p_j)
 // (global, local) for a batch of pairs chosen by Belady next-use order with
 // a victim floor vmin.  Must match oracle/plan.py bit for bit.
+//
+// Diagonal skip (diag != nullptr; reading R10, SURVEY.md §8f
+// NEXT-4): a fused gate forces an exchange only for its global qubits in
+// which it is not block-diagonal (diag[i] = logical-qubit mask of the
+// qubits it is block-diagonal in); next use counts non-diagonal uses only.
+// Such an APPLY lists global physical positions; the dispatcher runs the
+// block selected by each shard's device bits.
 #include <algorithm>
+#include <complex>
 #include <limits>
 
 #include "sv_internal.h"
@@ -16,7 +24,7 @@
 namespace svb {
 
 void plan_sharded(const std::vector<std::vector<int>>& fq, int n, int g, int vmin, std::vector<Event>& ev,
-                  std::vector<int>& pos) {
+                  std::vector<int>& pos, const std::vector<uint64_t>* diag) {
     const int l = n - g;
     const int nf = (int)fq.size();
     const int INF = std::numeric_limits<int>::max();
@@ -28,9 +36,11 @@ void plan_sharded(const std::vector<std::vector<int>>& fq, int n, int g, int vmi
     for (int q = 0; q < n; ++q) inv[pos[q]] = q;
     // next_use[i][q] = min{ j >= i : q in Q_j } (INF if none), built backwards
     std::vector<std::vector<int>> next_use(nf + 1, std::vector<int>(n, INF));
+    auto uses = [&](int i, int q) { return !diag || !(((*diag)[i] >> q) & 1ull); };
     for (int i = nf - 1; i >= 0; --i) {
         next_use[i] = next_use[i + 1];
-        for (int q : fq[i]) next_use[i][q] = i;
+        for (int q : fq[i])
+            if (uses(i, q)) next_use[i][q] = i;
     }
     ev.clear();
     for (int i = 0; i < nf; ++i) {
@@ -38,7 +48,7 @@ void plan_sharded(const std::vector<std::vector<int>>& fq, int n, int g, int vmi
         auto inQ = [&](int q) { return std::find(Qi.begin(), Qi.end(), q) != Qi.end(); };
         int need = 0;
         for (int q : Qi)
-            if (pos[q] >= l) ++need;
+            if (pos[q] >= l && uses(i, q)) ++need;
         const std::vector<int>& nu = next_use[i];
         if (need) {
             std::vector<int> glob;
@@ -119,6 +129,29 @@ void plan_canonicalize(int n, int g, std::vector<int>& pos, std::vector<Event>& 
         for (int p = 0; p < l; ++p) pos[inv[p]] = inv[p];
         ev.push_back(std::move(x));
     }
+}
+
+}  // namespace svb
+
+namespace svb {
+
+// block-diagonal in qubit b: every entry between a row and a column that
+// differ in bit b has |entry| <= 1e-10 (fp64 rounding residue of exact zeros;
+// the blocks drop them -- reading R10; oracle/plan.py DIAG_TOL)
+uint64_t diag_mask(const FusedGate& f) {
+    const int D = 1 << f.k;
+    uint64_t m = 0;
+    for (int b = 0; b < f.k; ++b) {
+        bool block = true;
+        for (int r = 0; r < D && block; ++r)
+            for (int c = 0; c < D; ++c)
+                if ((((r ^ c) >> b) & 1) && std::abs(f.M[(size_t)r * D + c]) > 1e-10) {
+                    block = false;
+                    break;
+                }
+        if (block) m |= 1ull << f.q[b];
+    }
+    return m;
 }
 
 }  // namespace svb

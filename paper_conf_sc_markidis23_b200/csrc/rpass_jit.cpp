@@ -167,7 +167,8 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
 // float4 matrix slots, mats their values (launch order).  emit == false:
 // only nm and mats (the PTX is cached under chunk_key).
 std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
-                      std::vector<float>& mats, bool emit = true) {
+                      std::vector<float>& mats, bool emit = true, const std::vector<float>* msrc = nullptr) {
+    const std::vector<float>& pmats = msrc ? *msrc : pd.mats;
     constexpr int M = 5, NA = 32, UPT = 16;
     const int T = (int)pd.S.size();
     const int tbits = T - M;
@@ -195,7 +196,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             const int kind = gate_kind(pd, pg);
             if (kind == 2) continue;
             const int D = 1 << pg.k;
-            const float* mg = pd.mats.data() + pg.moff;
+            const float* mg = pmats.data() + pg.moff;
             gbase[g] = mats.size() / 4;
             const int ne = kind == 1 ? D : D * D;
             for (int e = 0; e < ne; ++e) {
@@ -620,6 +621,10 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
             bool fresh = false;
             l.kern = lookup(chunk_key(pd, n_local, ch.first, ch.second, z), fresh);
             gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats, false);
+            for (const auto& ms : pd.mats_shard) {
+                l.mats_shard.emplace_back();
+                gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats_shard.back(), false, &ms);
+            }
             if (fresh) {
                 l.kern->src = gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
                 l.kern->nthr = 1 << (T - 5);
@@ -673,7 +678,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     return SV_OK;
 }
 
-cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st) {
+cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st, int slot) {
     RpJitKernel& K = *l.kern;
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -696,7 +701,8 @@ cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, boo
     const uint64_t n_tiles = 1ull << (n_local - T);
     const uint64_t grid = std::min<uint64_t>(n_tiles, (uint64_t)pass_sms() * K.blocks_per_sm);
     std::vector<unsigned char> prm(K.param_bytes, 0);
-    std::memcpy(prm.data(), l.mats.data(), l.mats.size() * sizeof(float));
+    const std::vector<float>& mats = l.mats_shard.empty() ? l.mats : l.mats_shard[slot];
+    std::memcpy(prm.data(), mats.data(), mats.size() * sizeof(float));
     const size_t off = std::max<size_t>(K.nm, 1) * 16;
     const float2* cpsi = psi;
     std::memcpy(prm.data() + off, &cpsi, 8);

@@ -79,6 +79,7 @@ struct sv_state {
     bool ext_buf = false;     // the state lives in a caller-owned buffer (sv_config.dev_buf)
     int tc_mode = 3;          // SV_OPT_APPLY_PATH
     int pass_jit = 1;         // SV_OPT_PASS_JIT
+    int diag_skip = 1;        // SV_OPT_DIAG_SKIP
     bool sample_pending = false;  // a sv_sample_device status word not yet checked
     size_t elem = 8;          // bytes per amplitude
     // staging ring for per-call device inputs of sv_apply_fused /
@@ -151,6 +152,7 @@ struct sv_circuit {
         ApplyDesc apply;
         Apply64Desc a64;  // complex128 states
         PassDesc pass;
+        std::vector<ApplyDesc> apply_shard;   // per local shard slot (diagonal exchange skip)
         std::vector<RpJitLaunch> jit, jitz;   // pass-specialised kernels (jitz: first pass from |0...0>)
         ExchangeDesc exch;
         std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
@@ -290,6 +292,36 @@ void make_apply(int l, int k, const int* phys_in_order, const cd* M /* bit b <->
     plan_apply(l, d);
 }
 
+// Block of a fused gate (matrix M over bits b <-> phys[b]) on the shard whose
+// device bits are d: rows/columns whose global bits (phys[b] >= l) equal d's
+// bits; locq receives the local positions.  A gate with no local position
+// becomes a phase on local bit 0 (diag(c, c)).  Mirrors oracle/plan.py
+// shard_block (reading R10).
+std::vector<cd> shard_block(int k, const int* phys, const std::vector<cd>& M, int l, int d, std::vector<int>& locq) {
+    std::vector<int> gb, lb;
+    for (int b = 0; b < k; ++b) (phys[b] >= l ? gb : lb).push_back(b);
+    int x = 0;
+    for (int b : gb) x |= ((d >> (phys[b] - l)) & 1) << b;
+    const int Dk = 1 << k, Dl = 1 << (int)lb.size();
+    std::vector<int> idx(Dl);
+    for (int t = 0; t < Dl; ++t) {
+        int r = x;
+        for (size_t j = 0; j < lb.size(); ++j) r |= ((t >> j) & 1) << lb[j];
+        idx[t] = r;
+    }
+    locq.clear();
+    for (int b : lb) locq.push_back(phys[b]);
+    if (lb.empty()) {
+        locq.push_back(0);
+        const cd c = M[(size_t)x * Dk + x];
+        return {c, cd(0), cd(0), c};
+    }
+    std::vector<cd> B((size_t)Dl * Dl);
+    for (int r = 0; r < Dl; ++r)
+        for (int c = 0; c < Dl; ++c) B[(size_t)r * Dl + c] = M[(size_t)idx[r] * Dk + idx[c]];
+    return B;
+}
+
 // PERMUTE (data at local bit b moves to bit perm[b]) as passes of disjoint
 // transpositions, <= 2 per pass (a 4-qubit permutation matrix carried in the
 // kernel parameters; the FMA chain of a 0/1 matrix is exact).
@@ -358,6 +390,22 @@ int run_apply(sv_state* s, const ApplyDesc& d) {
     s->stats.bytes_apply += 16ull << s->l;
     (d.high ? s->stats.bytes_apply_high : s->stats.bytes_apply_low) += 16ull << s->l;
     s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
+    return SV_OK;
+}
+
+// per-shard blocks of one fused gate (diagonal exchange skip)
+int run_apply_shards(sv_state* s, const std::vector<ApplyDesc>& ds) {
+    for (int sh = 0; sh < s->local_shards(); ++sh) {
+        float2* psi = s->virt ? s->shard[sh] : s->shard[s->rank];
+        const ApplyDesc& d = ds[sh];
+        int rc = launch(s, d.high ? LaunchClass::HIGH : LaunchClass::LOW,
+                        [&] { return launch_apply(psi, s->l, d, s->stream); });
+        if (rc) return rc;
+    }
+    const ApplyDesc& d = ds[0];
+    s->stats.bytes_apply += 16ull << s->l;
+    (d.high ? s->stats.bytes_apply_high : s->stats.bytes_apply_low) += 16ull << s->l;
+    s->stats.flops_apply += (uint64_t)((8 << d.k) - 2) << s->l;
     return SV_OK;
 }
 
@@ -520,7 +568,24 @@ struct PassIn {
     int k = 0;
     int q[SV_MAX_FUSED] = {0};
     std::vector<cd> M;
+    // shard-dependent gate (diagonal exchange skip): its block on every local
+    // shard slot over the same local qubits q (M = Mshard[0])
+    std::vector<std::vector<cd>> Mshard;
 };
+
+// rpass gate kind of a 2^k x 2^k matrix rounded to complex64 (as gate_kind):
+// 0 dense, 1 diagonal, 2 CZ-like diag(1, 1, 1, -1)
+int kind_of(const std::vector<cd>& M, int k) {
+    const int D = 1 << k;
+    bool diag = true, cz = k == 2;
+    for (int r = 0; r < D; ++r)
+        for (int c = 0; c < D; ++c) {
+            const float re = (float)M[(size_t)r * D + c].real(), im = (float)M[(size_t)r * D + c].imag();
+            if (r != c && (re != 0.f || im != 0.f)) diag = cz = false;
+            if (r == c && (im != 0.f || re != (r == D - 1 ? -1.f : 1.f))) cz = false;
+        }
+    return cz ? 2 : diag ? 1 : 0;
+}
 
 // Cache-blocked passes (reading R7).  Passes are formed like fused
 // gates (the S3 greedy, one level up): a pass starts at the first unplaced
@@ -595,6 +660,27 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
         for (size_t j : mem) {
             add_gate(cur, j);
             cur.src.push_back((int)j);
+        }
+        // shard-dependent gates: per-slot copies of the pass's matrices, and a
+        // gate kind that fits every slot (dense < diagonal < CZ-like)
+        size_t slots = 0;
+        for (size_t j : mem) slots = std::max(slots, in[j].Mshard.size());
+        if (slots) {
+            cur.mats_shard.assign(slots, cur.mats);
+            for (size_t t = 0; t < mem.size(); ++t) {
+                const PassIn& f = in[mem[t]];
+                if (f.Mshard.empty()) continue;
+                PassGate& pg = cur.gates[t];
+                int kind = 2;
+                for (size_t sl = 0; sl < slots; ++sl) {
+                    kind = std::min(kind, kind_of(f.Mshard[sl], f.k));
+                    for (size_t e = 0; e < f.Mshard[sl].size(); ++e) {
+                        cur.mats_shard[sl][pg.moff + 2 * e] = (float)f.Mshard[sl][e].real();
+                        cur.mats_shard[sl][pg.moff + 2 * e + 1] = (float)f.Mshard[sl][e].imag();
+                    }
+                }
+                pg.kind = kind;
+            }
         }
         passes.push_back(std::move(cur));
     }
@@ -1015,8 +1101,39 @@ static void write_events(const std::vector<Event>& ev, std::vector<int32_t>& o) 
     }
 }
 
+static int shard_plan_impl(const int32_t* fs, size_t len, const uint64_t* diag, int n, int g, int vmin, int32_t* buf,
+                           size_t cap, size_t* need, int32_t* final_pos);
+
 int sv_shard_plan(const int32_t* fs, size_t len, int n, int g, int vmin, int32_t* buf, size_t cap, size_t* need,
                   int32_t* final_pos) {
+    return shard_plan_impl(fs, len, nullptr, n, g, vmin, buf, cap, need, final_pos);
+}
+
+int sv_shard_plan_diag(const int32_t* fs, size_t len, const uint64_t* diag, int n, int g, int vmin, int32_t* buf,
+                       size_t cap, size_t* need, int32_t* final_pos) {
+    if (!diag && len) return fail(SV_EINVAL, "diag is NULL");
+    return shard_plan_impl(fs, len, diag, n, g, vmin, buf, cap, need, final_pos);
+}
+
+int sv_fusion_diag_masks(const sv_gate* gates, size_t n_gates, int max_fused, uint64_t* out, size_t cap, size_t* need) {
+    if (!need) return fail(SV_EINVAL, "need is NULL");
+    if (max_fused < 0 || max_fused > SV_MAX_FUSED) return fail(SV_EINVAL, "max_fused must be in [0, 6]");
+    int rc = validate_gates(gates, n_gates, -1);
+    if (rc) return rc;
+    std::vector<FusedGate> plan;
+    fuse_plan(gates, n_gates, max_fused, plan);
+    *need = plan.size();
+    if (cap < plan.size()) return fail(SV_EINVAL, "cap too small");
+    if (!plan.empty() && !out) return fail(SV_EINVAL, "out is NULL");
+    for (size_t i = 0; i < plan.size(); ++i) {
+        build_fused_matrix(gates, plan[i]);
+        out[i] = diag_mask(plan[i]);
+    }
+    return SV_OK;
+}
+
+static int shard_plan_impl(const int32_t* fs, size_t len, const uint64_t* diag, int n, int g, int vmin, int32_t* buf,
+                           size_t cap, size_t* need, int32_t* final_pos) {
     if (!need) return fail(SV_EINVAL, "need is NULL");
     if (n < 1 || n > SV_MAX_QUBITS || g < 0 || g >= n) return fail(SV_EINVAL, "bad n / log2_world");
     if (len && !fs) return fail(SV_EINVAL, "fusion stream is NULL");
@@ -1037,7 +1154,9 @@ int sv_shard_plan(const int32_t* fs, size_t len, int n, int g, int vmin, int32_t
     }
     std::vector<Event> ev;
     std::vector<int> pos;
-    plan_sharded(fq, n, g, vmin < 0 ? 5 : vmin, ev, pos);
+    std::vector<uint64_t> dm;
+    if (diag) dm.assign(diag, diag + fq.size());
+    plan_sharded(fq, n, g, vmin < 0 ? 5 : vmin, ev, pos, diag ? &dm : nullptr);
     std::vector<int32_t> outv;
     write_events(ev, outv);
     *need = outv.size();
@@ -1073,6 +1192,14 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     c->stats.t_fuse_s = t1 - t0;
     c->stats.n_fused = (int)plan.size();
     for (auto& f : plan) c->stats.fused_hist[f.k]++;
+    // Cache-blocked passes (complex64, large shards, k <= 4; sharded or not):
+    // each maximal run of APPLY events between exchanges is cut into passes
+    // by build_passes (reading R7); exchanges and permutations stay as they are.
+    // auto tile: 13 qubits (with the early next-tile load of apply_rpass:
+    // 30q D14 F=1 0.0745 s vs 0.0775 s at 12; 32q D20 0.430 vs 0.462 s)
+    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? 13 : 0);
+    const bool blocked = !s->fp64 && T >= 10 && s->l >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
+                         max_fused >= 1;
     // plan (sharded) or trivial apply list
     std::vector<Event> ev;
     c->pos_in = s->pos;
@@ -1080,7 +1207,13 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     if (s->g > 0) {
         std::vector<std::vector<int>> fq;
         for (auto& f : plan) fq.emplace_back(f.q, f.q + f.k);
-        plan_sharded(fq, s->n, s->g, s->vmin, ev, pos);
+        // diagonal exchange skip (reading R10): per-shard blocks run on the
+        // per-gate SIMT path or in register-blocked passes (k <= 2)
+        const bool skip = s->diag_skip && !s->fp64 && (!blocked || max_fused <= 2);
+        std::vector<uint64_t> dm;
+        if (skip)
+            for (auto& f : plan) dm.push_back(diag_mask(f));
+        plan_sharded(fq, s->n, s->g, s->vmin, ev, pos, skip ? &dm : nullptr);
         plan_canonicalize(s->n, s->g, pos, ev);
     } else {
         for (size_t i = 0; i < plan.size(); ++i) {
@@ -1093,14 +1226,6 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
     }
     c->pos_out = pos;
-    // Cache-blocked passes (complex64, large shards, k <= 4; sharded or not):
-    // each maximal run of APPLY events between exchanges is cut into passes
-    // by build_passes (reading R7); exchanges and permutations stay as they are.
-    // auto tile: 13 qubits (with the early next-tile load of apply_rpass:
-    // 30q D14 F=1 0.0745 s vs 0.0775 s at 12; 32q D20 0.430 vs 0.462 s)
-    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? 13 : 0);
-    const bool blocked = !s->fp64 && T >= 10 && s->l >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
-                         max_fused >= 1;
     const double t2 = now_s();
     c->stats.t_plan_s = t2 - t1;
     if (s->fp64) {
@@ -1158,11 +1283,33 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     };
     if (blocked) c->stats.block_bits = T;
     for (auto& e : ev) {
+        // APPLY on global positions (diagonal skip): the block of every local
+        // shard slot over the gate's local qubits
+        std::vector<int> locq;
+        std::vector<std::vector<cd>> blocks;
+        if (e.type == Event::APPLY && s->g > 0) {
+            bool gl = false;
+            for (int b = 0; b < e.k; ++b) gl |= e.phys[b] >= s->l;
+            if (gl) {
+                for (int sl = 0; sl < s->local_shards(); ++sl)
+                    blocks.push_back(shard_block(e.k, e.phys, plan[e.fused].M, s->l, s->virt ? sl : s->rank, locq));
+            }
+        }
         if (blocked && e.type == Event::APPLY) {
             PassIn pi;
-            pi.k = e.k;
-            pi.M.resize((size_t)1 << (2 * e.k));
-            sort_matrix_qubits<cd>(e.k, e.phys, plan[e.fused].M.data(), pi.q, pi.M.data());
+            if (!blocks.empty()) {
+                pi.k = (int)locq.size();
+                for (auto& B : blocks) {
+                    std::vector<cd> Ms(B.size());
+                    sort_matrix_qubits<cd>(pi.k, locq.data(), B.data(), pi.q, Ms.data());
+                    pi.Mshard.push_back(std::move(Ms));
+                }
+                pi.M = pi.Mshard[0];
+            } else {
+                pi.k = e.k;
+                pi.M.resize((size_t)1 << (2 * e.k));
+                sort_matrix_qubits<cd>(e.k, e.phys, plan[e.fused].M.data(), pi.q, pi.M.data());
+            }
             if (s->g == 0) run_all.push_back(pi);
             run.push_back(std::move(pi));
             continue;
@@ -1170,7 +1317,13 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         flush_passes();
         sv_circuit::Step st;
         st.type = e.type;
-        if (e.type == Event::APPLY) {
+        if (e.type == Event::APPLY && !blocks.empty()) {
+            for (auto& B : blocks) {  // SIMT: no per-shard int8 slices
+                st.apply_shard.emplace_back();
+                make_apply(s->l, (int)locq.size(), locq.data(), B.data(), st.apply_shard.back(), 0);
+            }
+            st.apply = st.apply_shard[0];
+        } else if (e.type == Event::APPLY) {
             make_apply(s->l, e.k, e.phys, plan[e.fused].M.data(), st.apply, s->tc_mode);
             if (e.k == 6) ++n6;
         } else if (e.type == Event::EXCHANGE) {
@@ -1418,13 +1571,13 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
                 if (!jl.empty()) {
                     for (const auto& l : jl) {
                         rc = launch(s, LaunchClass::HIGH,
-                                    [&] { return launch_rpass_jit(psi, s->l, l, shard == 0, s->stream); });
+                                    [&] { return launch_rpass_jit(psi, s->l, l, shard == 0, s->stream, sh); });
                         if (rc) return rc;
                     }
                     continue;
                 }
                 rc = launch(s, LaunchClass::HIGH, [&] {
-                    return rpass_supported(st.pass) ? launch_rpass(psi, s->l, st.pass, s->stream, z, shard == 0)
+                    return rpass_supported(st.pass) ? launch_rpass(psi, s->l, st.pass, s->stream, z, shard == 0, sh)
                                                     : launch_pass(psi, s->l, st.pass, s->stream);
                 });
                 if (rc) return rc;
@@ -1439,7 +1592,9 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
             s->stats.block_bits = (int)st.pass.S.size();
             continue;
         }
-        if (st.type == Event::APPLY) {
+        if (st.type == Event::APPLY && !st.apply_shard.empty()) {
+            rc = run_apply_shards(s, st.apply_shard);
+        } else if (st.type == Event::APPLY) {
             rc = run_apply(s, st.apply);
         } else if (st.type == Event::EXCHANGE) {
             rc = run_exchange(s, st.exch);
@@ -1900,6 +2055,10 @@ int sv_set_option(sv_state* s, int option, int value) {
             s->tc_mode = value == SV_PATH_AUTO ? 3 : value == SV_PATH_INT8 ? 2 : 0;
             return SV_OK;
         case SV_OPT_TIMING: return sv_set_timing(s, value);
+        case SV_OPT_DIAG_SKIP:
+            if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_DIAG_SKIP takes 0 or 1");
+            s->diag_skip = value;
+            return SV_OK;
         default: return fail(SV_EINVAL, "unknown option");
     }
 }

@@ -47,8 +47,13 @@ struct Event {
     std::vector<int> perm;                // PERMUTE: new local position of local bit b (size l)
 };
 // S4 exactly; events + final pos (logical -> physical).
+// diag (optional): per fused gate the mask of logical qubits it is
+// block-diagonal in (the diagonal exchange skip, reading R10).
 void plan_sharded(const std::vector<std::vector<int>>& fused_q, int n, int g, int vmin,
-                  std::vector<Event>& ev, std::vector<int>& pos);
+                  std::vector<Event>& ev, std::vector<int>& pos, const std::vector<uint64_t>* diag = nullptr);
+// Logical qubits of a fused gate in which its fp64 matrix is block-diagonal
+// (entries between rows and columns differing in that bit are exactly 0).
+uint64_t diag_mask(const FusedGate& f);
 // Canonicalisation events appended after a plan so that the final map is the
 // identity up to a relabelling of the global bits (Readings R9).
 void plan_canonicalize(int n, int g, std::vector<int>& pos, std::vector<Event>& ev);

@@ -336,3 +336,31 @@ def test_sycamore_virtual_shards(world, F):
     got, st = _run(n, gates, F, world=world)
     assert st["n_exchanges"] >= 1
     _check(n, 2 * cyc + 1, got, ref_c.run(n, gates))
+
+
+# ------------------------------------ diagonal exchange skip (NEXT-4, R10)
+@pytest.mark.parametrize("world", [2, 4, 8])
+@pytest.mark.parametrize("F,bits", [(1, 11), (2, 11), (1, 0), (4, 0)])
+def test_diag_skip_virtual_shards(world, F, bits):
+    """Fused gates block-diagonal in a global qubit (CZ-like at F = 1) run as
+    per-shard blocks without an exchange: fewer exchanges, same state as the
+    oracle, on register-blocked passes (bits 11) and per-gate launches."""
+    n, d = 18, 14
+    gates = W.rqc(n, d, seed=world + F)
+    ref = ref_c.run(n, gates)
+    out = {}
+    for skip in (1, 0):
+        h = sv.sv_create_ex(n, world=world, virtual_shards=True)
+        try:
+            sv.sv_set_option(h, sv.SV_OPT_DIAG_SKIP, skip)
+            sv.sv_set_blocking(h, bits)
+            st = sv.sv_run_circuit(h, gates, F)
+            got = sv.sv_get_state(h, n)
+        finally:
+            sv.sv_destroy(h)
+        _check(n, d, got, ref)
+        out[skip] = st["n_exchanges"]
+    # n_exchanges includes the final canonicalisation exchange (R3)
+    assert out[1] <= out[0]
+    if F == 1 and world >= 4:
+        assert out[1] < out[0], out

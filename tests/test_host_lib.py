@@ -81,6 +81,39 @@ def test_shard_plan_bit_exact(n, d, g, F, vmin):
     assert list(gpos) == list(pos)
 
 
+@pytest.mark.parametrize("F", [1, 2, 4])
+def test_diag_masks_match_oracle(F):
+    """The C++ block-diagonal test on the fp64 fused matrices equals
+    oracle/plan.diag_qubits on the oracle's fused matrices."""
+    for name, gates in [("rqc20", W.rqc(20, 14)), ("syc16", W.sycamore_rqc(16, 8)),
+                        ("mixed", W.random_circuit(10, 80, 3, two_qubit_frac=0.4))]:
+        got = sv.sv_fusion_diag_masks(gates, F)
+        ref = [sum(1 << q for q in oplan.diag_qubits(Q, M)) for Q, _, M in ofuse.fuse(gates, F)]
+        assert [int(x) for x in got] == ref, name
+
+
+@pytest.mark.parametrize("n,d,g,F", [(36, 20, 3, 1), (36, 20, 2, 1), (35, 20, 1, 1), (36, 20, 3, 2), (34, 20, 1, 4),
+                                     (20, 14, 2, 1), (16, 14, 3, 2)])
+def test_shard_plan_diag_skip_bit_exact(n, d, g, F):
+    """Diagonal exchange skip (reading R10): the C++ planner equals the
+    oracle's bit for bit; it never needs more exchanges than plain S4
+    (36q D20 F=1 at P=8: 7 -> 4)."""
+    gates = W.rqc(n, d)
+    fs = sv.sv_fusion_plan(gates, F)
+    fq = [Q for Q, _ in ofuse.fuse_plan([x.qubits for x in gates], F)]
+    dm = sv.sv_fusion_diag_masks(gates, F)
+    diag = [{q for q in range(n) if (int(m) >> q) & 1} for m in dm]
+    ev, pos = oplan.plan_sharded(fq, n, g, 5, diag=diag)
+    got, gpos = sv.sv_shard_plan_diag(fs, dm, n, g, 5)
+    assert np.array_equal(got, oplan.plan_stream(ev))
+    assert list(gpos) == list(pos)
+    ev0, _ = oplan.plan_sharded(fq, n, g, 5)
+    nx, nx0 = sum(e[0] == "X" for e in ev), sum(e[0] == "X" for e in ev0)
+    assert nx <= nx0
+    if (n, g, F) == (36, 3, 1):
+        assert (nx0, nx) == (7, 4)
+
+
 def test_error_codes():
     gates = W.rqc(12, 14)
     with pytest.raises(sv.SVError) as e:

@@ -218,3 +218,39 @@ def test_sampler_appendix_c():
     psi = sv.simulate(12, W.rqc(12, 14)).astype(np.complex64)
     out, T = sample.sample(psi, 1, 8)
     assert T == g["sampler_T"] and [int(x) for x in out] == g["sampler_seed1_first8"]
+
+
+# ------------------------------------------- diagonal exchange skip (NEXT-4)
+def test_diag_qubits_definition():
+    assert plan.diag_qubits((0, 1), W.GATE_CZ) == {0, 1}
+    assert plan.diag_qubits((3, 5), W.GATE_CX) == {3}  # control (bit 0) only
+    assert plan.diag_qubits((2,), W.GATE_T) == {2}
+    assert plan.diag_qubits((2,), W.GATE_H) == set()
+    assert plan.diag_qubits((0, 1), W.GATE_FSIM_SYC) == set()
+
+
+@pytest.mark.parametrize("n,g,F,seed", [(10, 1, 1, 0), (11, 2, 1, 1), (12, 3, 1, 2), (12, 3, 2, 3), (11, 2, 4, 4)])
+def test_sharded_diag_skip_equals_unsharded(n, g, F, seed):
+    """With the diagonal skip, global qubits a gate is block-diagonal in stay
+    global; the per-shard block emulation (shard_block) equals the plain
+    unsharded simulation, and the skip never adds exchanges."""
+    gates = W.rqc(n, 14, seed=seed)
+    fz = fuse.fuse(gates, F)
+    dq = [plan.diag_qubits(Q, M) for Q, _, M in fz]
+    ev, pos = plan.plan_sharded([Q for Q, _, _ in fz], n, g, 5, diag=dq)
+    ev0, _ = plan.plan_sharded([Q for Q, _, _ in fz], n, g, 5)
+    nx = sum(e[0] == "X" for e in ev)
+    assert nx <= sum(e[0] == "X" for e in ev0)
+    l = n - g
+    skipped = 0
+    for e in ev:
+        if e[0] == "A":
+            i, phys = e[1], e[2]
+            for q, p in zip(sorted(fz[i][0]), phys):
+                if p >= l:
+                    assert q in dq[i]
+                    skipped += 1
+    if F == 1:
+        assert skipped > 0  # CZ gates on global qubits run in place
+    out, _ = plan.run_sharded(n, g, fz, ev)
+    assert np.abs(out - sv.simulate(n, gates)).max() < 1e-12
