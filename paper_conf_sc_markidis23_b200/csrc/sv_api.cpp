@@ -1649,14 +1649,12 @@ int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fu
 // ---- amplitudes ----------------------------------------------------------------
 // complex128 states (single shard): gather into double2, D2H
 static int amplitudes64(sv_state* s, const uint64_t* idx, size_t count, sv_c128* out) {
-    {
-        const int rz = materialize(s);
-        if (rz) return rz;
-    }
     const uint64_t dim = 1ull << s->n;
     for (size_t i = 0; i < count; ++i)
         if (idx[i] >= dim) return fail(SV_EINVAL, "amplitude index out of range");
-    int rc = ensure(s, s->idx_dev, s->idx_cap, count);
+    int rc = materialize(s);
+    if (rc) return rc;
+    rc = ensure(s, s->idx_dev, s->idx_cap, count);
     if (rc) return rc;
     rc = ensure(s, s->amp_dev, s->amp_cap, 2 * count);
     if (rc) return rc;
@@ -1686,8 +1684,6 @@ int sv_amplitudes_c128(sv_state* s, const uint64_t* idx, size_t count, sv_c128* 
 int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
     int rc = check_state(s);
     if (rc) return rc;
-    rc = materialize(s);
-    if (rc) return rc;
     if (count == 0) return SV_OK;
     if (!idx || !out) return fail(SV_EINVAL, "idx/out is NULL");
     if (s->fp64) {
@@ -1706,6 +1702,8 @@ int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
         loc[i] = p & (s->local_amps() - 1);
         own[i] = (int32_t)(p >> s->l);
     }
+    rc = materialize(s);
+    if (rc) return rc;
     const size_t chunk = s->virt ? count : std::min<size_t>(count, kXferBytes / 8);
     for (size_t o = 0; o < count; o += chunk) {
         const size_t cnt = std::min(chunk, count - o);
