@@ -314,7 +314,8 @@ int sv_set_option(sv_state* s, int option, int value);
  * circuit (max_fused in [1, 2], tile_bits in [10, 13]; the first pass also
  * in its |0...0> form), separated by "//----" lines.  Pure host unless
  * compile != 0, which also assembles them through the driver JIT on the
- * current device (SV_ECUDA with the JIT log on failure).  *need gets the
+ * current device (SV_ECUDA with the JIT log on failure).  tile_bits < 0:
+ * the complex128 (wide) kernels for tiles of |tile_bits| qubits.  *need gets the
  * length including the terminating NUL; cap < *need returns SV_EINVAL unless
  * buf is NULL and cap is 0 (size query). */
 int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int tile_bits, int compile, char* buf,

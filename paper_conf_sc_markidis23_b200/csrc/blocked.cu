@@ -1022,7 +1022,7 @@ int gate_kind(const PassDesc& pd, const PassGate& pg) {
 // Phases of gates [g0, g1): each phase takes, in order, every remaining gate
 // whose positions fit in the phase's M-set and that does not touch a position
 // of a gate skipped before it (so it only moves past gates it commutes with).
-std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, int M) {
+std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, int M, bool wide) {
     const int T = (int)pd.S.size();
     std::vector<RpPhaseHost> out;
     std::vector<int> rem;
@@ -1059,7 +1059,9 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
                 if (!(m & blocked) && (ra[i] || !(m & ~R))) ++cnt;
                 else blocked |= m;
             }
-            const int score = 4 * cnt + ((R & 1u) ? 2 : 0) + ((R & 0xEu) ? 0 : 1);
+            // wide (16 B complex128 amplitudes): ties prefer R free of bits
+            // 0..2 (lanes 0..2 = bits 0..2: conflict-free, direct-store layout)
+            const int score = wide ? 4 * cnt + ((R & 0x7u) ? 0 : 1) : 4 * cnt + ((R & 1u) ? 2 : 0) + ((R & 0xEu) ? 0 : 1);
             if (score > best) {
                 best = score;
                 used = R;
@@ -1083,7 +1085,30 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
         }
         for (int q = 0; q < T; ++q)
             if ((used >> q) & 1u) ph.R.push_back(q);
-        ph.b0 = (used & 1u) != 0;
+        ph.b0 = !wide && (used & 1u) != 0;
+        if (wide) {
+            // 16 B per amplitude: the first 3 lanes (a quarter-warp of LDS.128)
+            // must move distinct chunk bits under the wide fold swizzle
+            // (class q % 3), lowest positions first
+            std::vector<int> rest, lanes;
+            for (int q = 0; q < T; ++q)
+                if (!((used >> q) & 1u)) rest.push_back(q);
+            int have = 0;
+            for (size_t i = 0; i < rest.size() && have != 7;) {
+                const int c = rest[i] % 3;
+                if (!((have >> c) & 1)) {
+                    have |= 1 << c;
+                    lanes.push_back(rest[i]);
+                    rest.erase(rest.begin() + (long)i);
+                } else {
+                    ++i;
+                }
+            }
+            lanes.insert(lanes.end(), rest.begin(), rest.end());
+            ph.lanes = lanes;
+            out.push_back(ph);
+            continue;
+        }
         // lanes: the first lanes of a quarter- (16 B) / half-warp (8 B) must
         // move distinct bank bits
         std::vector<int> rest;
@@ -1112,19 +1137,19 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
     return out;
 }
 
-std::vector<std::pair<size_t, size_t>> rpass_chunks(const PassDesc& pd, int M) {
+std::vector<std::pair<size_t, size_t>> rpass_chunks(const PassDesc& pd, int M, bool wide) {
     std::vector<std::pair<size_t, size_t>> out;
     const size_t ng = pd.gates.size();
     size_t g0 = 0;
     while (g0 < ng) {
         size_t g1 = std::min(ng, g0 + (size_t)kRpMaxGates);
-        if ((int)plan_phases(pd, g0, g1, M).size() > kRpMaxPhases) {
+        if ((int)plan_phases(pd, g0, g1, M, wide).size() > kRpMaxPhases) {
             // the first kRpMaxPhases phases hold a prefix of the gates only if
             // no gate was moved past a later phase: re-plan a shorter prefix
             size_t cut = g1;
             do {
                 cut = g0 + (cut - g0) / 2;
-            } while ((int)plan_phases(pd, g0, cut, M).size() > kRpMaxPhases);
+            } while ((int)plan_phases(pd, g0, cut, M, wide).size() > kRpMaxPhases);
             g1 = cut;
         }
         out.push_back({g0, g1});

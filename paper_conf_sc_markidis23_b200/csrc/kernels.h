@@ -102,6 +102,8 @@ struct PassDesc {
     // so the pass starts from prod_q v_q[bit q] with v_q = that gate's first
     // column (identity: (1, 0)).  pinit_v: v of tile position p at [2p, 2p+1]
     std::vector<std::complex<double>> pinit_v;
+    std::vector<double> mats64;  // complex128 states: the matrices in fp64 (same layout as mats)
+    bool wide = false;           // complex128 state: pass-specialised fp64 kernel, 16 amplitudes per thread
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
@@ -141,10 +143,12 @@ int rpass_m();
 // 0 dense, 1 diagonal, 2 CZ-like (diag(1, 1, 1, -1)), exact in fp32
 int gate_kind(const PassDesc& pd, const PassGate& pg);
 // phases of pass gates [g0, g1) for M register bits
-std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, int M);
+// wide: 16 B (complex128) amplitudes -- lanes for LDS.128 of single
+// amplitudes under the wide fold swizzle (amplitude bits 0..2 ^= 3..5 ^ 6..8 ...)
+std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, int M, bool wide = false);
 // The gates [g0, g1) of a pass as launch chunks: each chunk [c0, c1) fits one
 // launch (<= kRpMaxGates gates, <= kRpMaxPhases phases).
-std::vector<std::pair<size_t, size_t>> rpass_chunks(const PassDesc& pd, int M);
+std::vector<std::pair<size_t, size_t>> rpass_chunks(const PassDesc& pd, int M, bool wide = false);
 int pass_sms();
 
 // Pass-specialised register-blocked kernels (rpass_jit.cpp): the phase plan,
@@ -157,12 +161,14 @@ struct RpJitLaunch {
     std::shared_ptr<RpJitKernel> kern;
     std::vector<float> mats;  // float4 (mr, mr, -mi, mi) per matrix element, launch order
     std::vector<std::vector<float>> mats_shard;  // per local shard slot (PassDesc::mats_shard)
+    std::vector<double> mats64;  // complex128 kernels: (mr, mi) per matrix element
+    bool wide = false;
     size_t c0 = 0, c1 = 0;    // gate chunk
     bool zinit = false;
     // product-state start: tile factor = tabA[u & (2^h1 - 1)] * tabB[u >> h1]
     // (device tables owned by the circuit, complex64)
-    const float2* tabA = nullptr;
-    const float2* tabB = nullptr;
+    const void* tabA = nullptr;  // complex64 (complex128 for wide kernels)
+    const void* tabB = nullptr;
     int h1 = 0;
 };
 // Generate (and compile unless compile == false) the kernels of one pass;
@@ -172,7 +178,7 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
 // Prepare many passes at once (compiles in parallel host threads).
 int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local, const std::vector<char>& zinit,
                            std::vector<std::vector<RpJitLaunch>>& out);
-cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st,
+cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st,
                              int slot = 0);
 // process-wide counters (sv_jit_stats)
 void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compile_s);

@@ -149,6 +149,7 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         k += std::to_string(v);
         k += ',';
     };
+    if (pd.wide) k += "w,";
     put(n_local);
     put(pd.r);
     put(zinit ? 1 : 0);
@@ -521,6 +522,335 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
 // Assemble the PTX for this device through the driver's JIT (ptxas; the
 // driver also caches the result across processes) and look the kernel up,
 // which forces the module load under lazy loading.
+// ---------------------------------------------------------------------------
+// complex128 states (NEXT-1, Fig. 8): the same pass structure
+// with 16 B amplitudes -- 16 per thread (M = 4; 64 fp64 registers), one
+// LDS.128 / cp.async per amplitude, the wide fold swizzle (amplitude bits
+// 0..2 ^= bits 3..5 ^ 6..8 ^ ...: 8 consecutive lanes hit 8 distinct 16 B
+// bank groups), fp64 FMAs (4 per complex MAC).  Matrices travel as fp64.
+uint32_t fold64(uint32_t t, int T) {
+    uint32_t f = 0;
+    for (int q = 3; q < T; ++q)
+        if ((t >> q) & 1u) f ^= 1u << ((q - 3) % 3);
+    return t ^ f;
+}
+
+std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
+                        std::vector<double>& mats, bool emit = true) {
+    constexpr int M = 4, NA = 16, UPT = 16;
+    const int T = (int)pd.S.size();
+    const int tbits = T - M;
+    const uint32_t nthr = 1u << tbits;
+    TileMap tm;
+    tm.r = pd.r;
+    for (int i = pd.r; i < T; ++i) tm.H.push_back(pd.S[i]);
+    const auto phs = plan_phases(pd, g0, g1, M, true);
+    const int nph = (int)phs.size();
+    const RpPhaseHost& lp = phs.back();
+    const bool direct = lp.lanes.size() >= 3 && lp.lanes[0] == 0 && lp.lanes[1] == 1 && lp.lanes[2] == 2;
+    const bool early = direct && !zinit;
+    mats.clear();
+    std::vector<size_t> gbase(pd.gates.size(), 0);
+    for (int ph = 0; ph < nph; ++ph)
+        for (int g : phs[ph].gates) {
+            const PassGate& pg = pd.gates[g];
+            const int kind = gate_kind(pd, pg);
+            if (kind == 2) continue;
+            const int D = 1 << pg.k;
+            const double* mg = pd.mats64.data() + pg.moff;
+            gbase[g] = mats.size() / 2;
+            const int ne = kind == 1 ? D : D * D;
+            for (int e = 0; e < ne; ++e) {
+                const int src = kind == 1 ? e * D + e : e;
+                mats.push_back(mg[2 * src]);
+                mats.push_back(mg[2 * src + 1]);
+            }
+        }
+    const bool pinit = zinit && !pd.pinit_v.empty();
+    size_t reg0 = 0, lane0 = 0;
+    if (pinit) {
+        const RpPhaseHost& P0 = phs[0];
+        reg0 = mats.size() / 2;
+        for (uint32_t j = 0; j < NA; ++j) {
+            std::complex<double> z = 1.0;
+            for (int b = 0; b < M; ++b) z *= pd.pinit_v[2 * P0.R[b] + ((j >> b) & 1u)];
+            mats.push_back(z.real());
+            mats.push_back(z.imag());
+        }
+        lane0 = mats.size() / 2;
+        for (int b = 0; b < tbits; ++b)
+            for (int v = 0; v < 2; ++v) {
+                mats.push_back(pd.pinit_v[2 * P0.lanes[b] + v].real());
+                mats.push_back(pd.pinit_v[2 * P0.lanes[b] + v].imag());
+            }
+    }
+    nm = mats.size() / 2;
+    const size_t off_psi = std::max<size_t>(nm, 1) * 16, off_nt = off_psi + 8, off_zone = off_psi + 16,
+                 off_h1 = off_psi + 20, off_ta = off_psi + 24, off_tb = off_psi + 32;
+    const size_t pbytes = off_psi + 48;
+    if (!emit) return std::string();
+
+    Ptx P;
+    P.op("mov.u32 %t_id, %tid.x");
+    P.op("mov.u32 %cur, rsm");
+    P.op("mov.b64 %dthr, 0");
+    P.op("mov.b32 %sthr, 0");
+    if (direct) P.op("mov.b64 %dg, 0");
+    for (int b = 0; b < tbits; ++b) {
+        const std::string t = P.r32(), q = P.pr();
+        P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+        P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+        P.op("@", q, " add.s64 %dthr, %dthr, ", 16 * tm.dep(1ull << b));
+        P.op("@", q, " xor.b32 %sthr, %sthr, ", fold64(1u << b, T) << 4);
+        if (direct) P.op("@", q, " add.s64 %dg, %dg, ", 16 * tm.dep(1ull << lp.lanes[b]));
+    }
+    auto cmul = [&](const std::string& ar, const std::string& ai, const std::string& br, const std::string& bi,
+                    const std::string& orr, const std::string& oi) {  // (or, oi) = a * b
+        P.op("mul.rn.f64 %t0, ", ar, ", ", br);
+        P.op("mul.rn.f64 %t1, ", ar, ", ", bi);
+        P.op("neg.f64 %t2, ", ai);
+        P.op("fma.rn.f64 ", orr, ", %t2, ", bi, ", %t0");
+        P.op("fma.rn.f64 ", oi, ", ", ai, ", ", br, ", %t1");
+    };
+    if (pinit) {
+        P.op("mov.f64 %tfr, 0d3FF0000000000000");
+        P.op("mov.f64 %tfi, 0d0000000000000000");
+        for (int b = 0; b < tbits; ++b) {
+            const std::string t = P.r32(), q = P.pr();
+            P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+            P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+            P.op("ld.param.v2.f64 {%mr, %mi}, [rpj_param_0+", 16 * (lane0 + 2 * b), "]");
+            P.op("ld.param.v2.f64 {%yr, %yi}, [rpj_param_0+", 16 * (lane0 + 2 * b + 1), "]");
+            P.op("selp.f64 %mr, %yr, %mr, ", q);
+            P.op("selp.f64 %mi, %yi, %mi, ", q);
+            cmul("%tfr", "%tfi", "%mr", "%mi", "%tfr", "%tfi");
+        }
+        P.op("ld.param.u32 %h1, [rpj_param_0+", off_h1, "]");
+        P.op("ld.param.u64 %tabA, [rpj_param_0+", off_ta, "]");
+        P.op("ld.param.u64 %tabB, [rpj_param_0+", off_tb, "]");
+    }
+    P.op("ld.param.u64 %psi, [rpj_param_0+", off_psi, "]");
+    P.op("ld.param.u64 %ntiles, [rpj_param_0+", off_nt, "]");
+    P.op("ld.param.u32 %zone, [rpj_param_0+", off_zone, "]");
+    P.op("mov.u32 %r_c, %ctaid.x");
+    P.op("cvt.u64.u32 %u, %r_c");
+    P.op("mov.u32 %r_c, %nctaid.x");
+    P.op("cvt.u64.u32 %grid, %r_c");
+    P.op("setp.ge.u64 %p_out, %u, %ntiles");
+    P.op("@%p_out bra $DONE");
+    // tile base (bytes) = 2 x the 8 B deposit
+    emit_tbase(P, pd.S, n_local, "%u", "%tbo");
+    P.op("shl.b64 %tbo, %tbo, 1");
+    P.op("add.s64 %gtile, %psi, %tbo");
+    P.op("add.s64 %gcur, %gtile, %dthr");
+    auto loadtile = [&](const std::string& g, const std::string& pred) {
+        for (int i = 0; i < UPT; ++i) {
+            const std::string sa = P.r32();
+            P.op("xor.b32 ", sa, ", %sthr, ", fold64(nthr * i, T) << 4);
+            P.op("add.s32 ", sa, ", ", sa, ", %cur");
+            const std::string ga = gaddr(P, g, 16 * tm.dep((uint64_t)nthr * i));
+            P.op(pred, "cp.async.cg.shared.global [", sa, "], ", ga, ", 16");
+        }
+    };
+    if (!zinit) loadtile("%gcur", "");
+    P.op("cp.async.commit_group");
+    P.o << "$LOOP:\n";
+    P.op("add.s64 %un, %u, %grid");
+    P.op("setp.lt.u64 %p_next, %un, %ntiles");
+    emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+    P.op("shl.b64 %tbo, %tbo, 1");
+    P.op("add.s64 %gtile_next, %psi, %tbo");
+    P.op("add.s64 %gnext, %gtile_next, %dthr");
+    P.op("cp.async.wait_group 0");
+    P.op("bar.sync 0");
+    auto ar = [](int j) { return "%ar" + std::to_string(j); };
+    auto ai = [](int j) { return "%ai" + std::to_string(j); };
+    for (int ph = 0; ph < nph; ++ph) {
+        const RpPhaseHost& Ph = phs[ph];
+        const bool last = ph == nph - 1;
+        P.o << "\t// phase " << ph << ": R = {";
+        for (int q : Ph.R) P.o << q << ",";
+        P.o << "}, " << Ph.gates.size() << " gates\n";
+        P.op("mov.b32 %tb, 0");
+        for (int b = 0; b < tbits; ++b) {
+            const std::string t = P.r32(), q = P.pr();
+            P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+            P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+            P.op("@", q, " xor.b32 %tb, %tb, ", fold64(1u << Ph.lanes[b], T) << 4);
+        }
+        auto saddr = [&](uint32_t j) {
+            const std::string t = P.r32();
+            P.op("xor.b32 ", t, ", %tb, ", fold64(deposit(j, Ph.R), T) << 4);
+            P.op("add.s32 ", t, ", ", t, ", %cur");
+            return t;
+        };
+        if (ph == 0 && pinit) {
+            // tile factor (two table entries) x thread factor, then x the register factor
+            P.op("mov.b64 %rdB, 1");
+            P.op("shl.b64 %rdB, %rdB, %h1");
+            P.op("sub.s64 %rdB, %rdB, 1");
+            P.op("and.b64 %rdB, %u, %rdB");
+            P.op("shl.b64 %rdB, %rdB, 4");
+            P.op("add.s64 %rdB, %tabA, %rdB");
+            P.op("ld.global.nc.v2.f64 {%xr0, %xi0}, [%rdB]");
+            P.op("shr.u64 %rdB, %u, %h1");
+            P.op("shl.b64 %rdB, %rdB, 4");
+            P.op("add.s64 %rdB, %tabB, %rdB");
+            P.op("ld.global.nc.v2.f64 {%xr1, %xi1}, [%rdB]");
+            cmul("%xr0", "%xi0", "%xr1", "%xi1", "%xr2", "%xi2");
+            cmul("%xr2", "%xi2", "%tfr", "%tfi", "%xr3", "%xi3");
+            for (int j = 0; j < NA; ++j) {
+                P.op("ld.param.v2.f64 {%mr, %mi}, [rpj_param_0+", 16 * (reg0 + j), "]");
+                cmul("%mr", "%mi", "%xr3", "%xi3", ar(j), ai(j));
+            }
+        } else if (ph == 0 && zinit) {
+            for (int j = 0; j < NA; ++j) {
+                P.op("mov.f64 ", ar(j), ", 0d0000000000000000");
+                P.op("mov.f64 ", ai(j), ", 0d0000000000000000");
+            }
+            P.op("setp.ne.u32 %p_z, %zone, 0");
+            P.op("setp.eq.and.u64 %p_z, %u, 0, %p_z");
+            P.op("setp.eq.and.u32 %p_z, %t_id, 0, %p_z");
+            P.op("@%p_z mov.f64 %ar0, 0d3FF0000000000000");
+        } else {
+            for (int j = 0; j < NA; ++j) {
+                const std::string a = saddr((uint32_t)j);
+                P.op("ld.shared.v2.f64 {", ar(j), ", ", ai(j), "}, [", a, "]");
+            }
+        }
+        if (last && early) {
+            P.op("bar.sync 0");
+            loadtile("%gnext", "@%p_next ");
+            P.op("cp.async.commit_group");
+        }
+        for (int g : Ph.gates) {
+            const PassGate& pg = pd.gates[g];
+            const int kind = gate_kind(pd, pg);
+            uint32_t mask = 0, tmask = 0;
+            for (int b = 0; b < pg.k; ++b) {
+                const auto it = std::find(Ph.R.begin(), Ph.R.end(), pg.pos[b]);
+                if (it != Ph.R.end()) mask |= 1u << (int)(it - Ph.R.begin());
+                else tmask |= 1u << (int)(std::find(Ph.lanes.begin(), Ph.lanes.end(), pg.pos[b]) - Ph.lanes.begin());
+            }
+            const int D = 1 << pg.k;
+            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask << "\n";
+            if (kind == 2) {
+                std::string pred;
+                if (popc(mask) != 2) {
+                    const std::string t = P.r32();
+                    pred = P.pr();
+                    P.op("and.b32 ", t, ", %t_id, ", tmask);
+                    P.op("setp.eq.u32 ", pred, ", ", t, ", ", tmask);
+                    pred = "@" + pred + " ";
+                }
+                for (uint32_t j = 0; j < (uint32_t)NA; ++j)
+                    if ((j & mask) == mask) {
+                        P.op(pred, "neg.f64 ", ar(j), ", ", ar(j));
+                        P.op(pred, "neg.f64 ", ai(j), ", ", ai(j));
+                    }
+                continue;
+            }
+            const size_t base = gbase[g];
+            auto mload = [&](size_t e) {
+                P.op("ld.param.v2.f64 {%mr, %mi}, [rpj_param_0+", 16 * e, "]");
+                P.op("neg.f64 %nmi, %mi");
+            };
+            if (kind == 1) {
+                for (int e = 0; e < D; ++e) {
+                    mload(base + e);
+                    for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
+                        if (pext(j, mask) != (uint32_t)e) continue;
+                        P.op("mov.f64 %xr0, ", ar(j));
+                        P.op("mul.rn.f64 ", ar(j), ", %mr, %xr0");
+                        P.op("fma.rn.f64 ", ar(j), ", %nmi, ", ai(j), ", ", ar(j));
+                        P.op("mul.rn.f64 %yi, %mr, ", ai(j));
+                        P.op("fma.rn.f64 ", ai(j), ", %mi, %xr0, %yi");
+                    }
+                }
+                continue;
+            }
+            const uint32_t rest = ((1u << M) - 1u) & ~mask;
+            for (uint32_t gi = 0; gi < (uint32_t)NA / D; ++gi) {
+                const uint32_t b0 = pdep(gi, rest);
+                for (int c = 0; c < D; ++c) {
+                    P.op("mov.f64 %xr", c, ", ", ar(b0 | pdep(c, mask)));
+                    P.op("mov.f64 %xi", c, ", ", ai(b0 | pdep(c, mask)));
+                }
+                for (int rr = 0; rr < D; ++rr) {
+                    const uint32_t dst = b0 | pdep(rr, mask);
+                    for (int c = 0; c < D; ++c) {
+                        mload(base + rr * D + c);
+                        if (c == 0) {
+                            P.op("mul.rn.f64 %yr, %mr, %xr0");
+                            P.op("mul.rn.f64 %yi, %mr, %xi0");
+                        } else {
+                            P.op("fma.rn.f64 %yr, %mr, %xr", c, ", %yr");
+                            P.op("fma.rn.f64 %yi, %mr, %xi", c, ", %yi");
+                        }
+                        P.op("fma.rn.f64 %yr, %nmi, %xi", c, ", %yr");
+                        P.op("fma.rn.f64 %yi, %mi, %xr", c, ", %yi");
+                    }
+                    P.op("mov.f64 ", ar(dst), ", %yr");
+                    P.op("mov.f64 ", ai(dst), ", %yi");
+                }
+            }
+        }
+        if (last && direct) {
+            P.op("add.s64 %gst, %gtile, %dg");
+            for (int j = 0; j < NA; ++j)
+                P.op("st.global.cs.v2.f64 ", gaddr(P, "%gst", 16 * tm.dep(deposit((uint32_t)j, lp.R))), ", {", ar(j), ", ",
+                     ai(j), "}");
+        } else {
+            for (int j = 0; j < NA; ++j) {
+                const std::string a = saddr((uint32_t)j);
+                P.op("st.shared.v2.f64 [", a, "], {", ar(j), ", ", ai(j), "}");
+            }
+            P.op("bar.sync 0");
+        }
+    }
+    if (!direct) {
+        for (int i = 0; i < UPT; ++i) {
+            const std::string sa = P.r32();
+            P.op("xor.b32 ", sa, ", %sthr, ", fold64(nthr * i, T) << 4);
+            P.op("add.s32 ", sa, ", ", sa, ", %cur");
+            P.op("ld.shared.v2.f64 {", ar(i), ", ", ai(i), "}, [", sa, "]");
+        }
+        if (!zinit) {
+            P.op("bar.sync 0");
+            loadtile("%gnext", "@%p_next ");
+            P.op("cp.async.commit_group");
+        }
+        for (int i = 0; i < UPT; ++i)
+            P.op("st.global.cs.v2.f64 ", gaddr(P, "%gcur", 16 * tm.dep((uint64_t)nthr * i)), ", {", ar(i), ", ", ai(i), "}");
+    }
+    P.op("mov.b64 %gcur, %gnext");
+    P.op("mov.b64 %gtile, %gtile_next");
+    P.op("mov.b64 %u, %un");
+    P.op("@%p_next bra $LOOP");
+    P.o << "$DONE:\n";
+    P.op("ret");
+
+    std::ostringstream k;
+    k << "// pass-specialised register-blocked kernel, complex128 (generated by rpass_jit.cpp)\n";
+    k << "// T=" << T << " r=" << pd.r << " n=" << n_local << " S={";
+    for (int q : pd.S) k << q << ",";
+    k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (pinit ? " product-start" : "")
+      << (direct ? " direct" : "") << "\n";
+    k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
+    k << ".extern .shared .align 16 .b8 rsm[];\n";
+    k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
+    k << ".maxntid " << nthr << ", 1, 1\n.maxnreg 128\n{\n";
+    k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z;\n";
+    k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %h1;\n";
+    k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
+    k << "\t.reg .f64 %ar<16>, %ai<16>, %xr<4>, %xi<4>, %yr, %yi, %mr, %mi, %nmi, %t0, %t1, %t2, %tfr, %tfi;\n";
+    k << "\t.reg .b64 %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, %gnext, %gst, "
+         "%tabA, %tabB, %rdB;\n";
+    k << P.o.str();
+    k << "}\n";
+    return k.str();
+}
+
 int compile_one(RpJitKernel& K, int dev, std::string& log) {
     const auto t0 = std::chrono::steady_clock::now();
     cudaError_t e = cudaSetDevice(dev);  // worker threads start on device 0
@@ -613,22 +943,28 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     for (size_t i = 0; i < pds.size(); ++i) {
         const PassDesc& pd = *pds[i];
         const int T = (int)pd.S.size();
+        const int M = pd.wide ? 4 : 5;
         bool first = true;
-        for (const auto& ch : rpass_chunks(pd, 5)) {
+        for (const auto& ch : rpass_chunks(pd, M, pd.wide)) {
             RpJitLaunch l;
             size_t nm = 0;
             const bool z = zinit[i] && first;
             bool fresh = false;
             l.kern = lookup(chunk_key(pd, n_local, ch.first, ch.second, z), fresh);
-            gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats, false);
-            for (const auto& ms : pd.mats_shard) {
-                l.mats_shard.emplace_back();
-                gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats_shard.back(), false, &ms);
+            if (pd.wide) {
+                gen_chunk64(pd, n_local, ch.first, ch.second, z, nm, l.mats64, false);
+            } else {
+                gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats, false);
+                for (const auto& ms : pd.mats_shard) {
+                    l.mats_shard.emplace_back();
+                    gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats_shard.back(), false, &ms);
+                }
             }
             if (fresh) {
-                l.kern->src = gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
-                l.kern->nthr = 1 << (T - 5);
-                l.kern->smem = (size_t)8 << T;
+                l.kern->src = pd.wide ? gen_chunk64(pd, n_local, ch.first, ch.second, z, nm, l.mats64)
+                                      : gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
+                l.kern->nthr = 1 << (T - M);
+                l.kern->smem = (size_t)(pd.wide ? 16 : 8) << T;
                 l.kern->nm = nm;
                 l.kern->param_bytes = std::max<size_t>(nm, 1) * 16 + 48;  // as in gen_chunk
                 todo.push_back(l.kern);
@@ -636,6 +972,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
             l.c0 = ch.first;
             l.c1 = ch.second;
             l.zinit = z;
+            l.wide = pd.wide;
             out[i].push_back(std::move(l));
             first = false;
         }
@@ -678,7 +1015,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     return SV_OK;
 }
 
-cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st, int slot) {
+cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st, int slot) {
     RpJitKernel& K = *l.kern;
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -697,14 +1034,18 @@ cudaError_t launch_rpass_jit(float2* psi, int n_local, const RpJitLaunch& l, boo
             }
         }
     }
-    const int T = 5 + __builtin_ctz((unsigned)K.nthr);
+    const int T = __builtin_ctz((unsigned)(K.smem / (l.wide ? 16 : 8)));
     const uint64_t n_tiles = 1ull << (n_local - T);
     const uint64_t grid = std::min<uint64_t>(n_tiles, (uint64_t)pass_sms() * K.blocks_per_sm);
     std::vector<unsigned char> prm(K.param_bytes, 0);
-    const std::vector<float>& mats = l.mats_shard.empty() ? l.mats : l.mats_shard[slot];
-    std::memcpy(prm.data(), mats.data(), mats.size() * sizeof(float));
+    if (l.wide) {
+        std::memcpy(prm.data(), l.mats64.data(), l.mats64.size() * sizeof(double));
+    } else {
+        const std::vector<float>& mats = l.mats_shard.empty() ? l.mats : l.mats_shard[slot];
+        std::memcpy(prm.data(), mats.data(), mats.size() * sizeof(float));
+    }
     const size_t off = std::max<size_t>(K.nm, 1) * 16;
-    const float2* cpsi = psi;
+    const void* cpsi = psi;
     std::memcpy(prm.data() + off, &cpsi, 8);
     std::memcpy(prm.data() + off + 8, &n_tiles, 8);
     const int zone = one_here ? 1 : 0;

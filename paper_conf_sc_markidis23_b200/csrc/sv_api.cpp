@@ -163,7 +163,7 @@ struct sv_circuit {
     // first pass (PassDesc::pinit_v); empty when not applicable
     std::vector<Step> steps_z;
     sv_stats stats_z{};
-    float2* ptab = nullptr;  // its tile-factor tables (device, complex64)
+    void* ptab = nullptr;  // its tile-factor tables (device, complex64 / complex128)
     float2* dev_mats = nullptr;
     double* planes64 = nullptr;  // complex128 states: planes of every gate
     uint8_t* wi8 = nullptr;      // int8 tensor-core W slices of every tensor-core gate
@@ -617,6 +617,8 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
         for (int e = 0; e < D * D; ++e) {
             cur.mats.push_back((float)f.M[e].real());
             cur.mats.push_back((float)f.M[e].imag());
+            cur.mats64.push_back(f.M[e].real());
+            cur.mats64.push_back(f.M[e].imag());
         }
         std::vector<float> Pp(D * D), Sp(D * D), Qp(D * D);
         for (int e = 0; e < D * D; ++e) {
@@ -796,12 +798,12 @@ int sv_reset(sv_state* s) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
     if (s->sticky) return fail(SV_EBADSTATE, "state poisoned by an earlier device failure");
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
-    if (!s->fp64 && !s->ext_buf) {
+    if (!s->ext_buf) {
         s->zero_pending = true;  // written lazily (see sv_state::zero_pending)
         return SV_OK;
     }
-    // complex128 states and caller-owned buffers (the caller may read or
-    // write the memory directly) are written now
+    // caller-owned buffers (the caller may read or write the memory
+    // directly) are written now
     s->zero_pending = false;
     return write_zero_state(s);
 }
@@ -1197,9 +1199,11 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     // by build_passes (reading R7); exchanges and permutations stay as they are.
     // auto tile: 13 qubits (with the early next-tile load of apply_rpass:
     // 30q D14 F=1 0.0745 s vs 0.0775 s at 12; 32q D20 0.430 vs 0.462 s)
-    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? 13 : 0);
-    const bool blocked = !s->fp64 && T >= 10 && s->l >= T + 2 && s->n > kSmallCircuitMaxQubits && max_fused <= 4 &&
-                         max_fused >= 1;
+    // complex128 states: pass-specialised fp64 kernels (16 amplitudes per
+    // thread, auto tile 12 qubits = 64 KB) for max_fused <= 2
+    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? (s->fp64 ? 12 : 13) : 0);
+    const bool blocked = (!s->fp64 || (s->pass_jit && max_fused <= 2)) && T >= 10 && s->l >= T + 2 &&
+                         s->n > kSmallCircuitMaxQubits && max_fused <= 4 && max_fused >= 1;
     // plan (sharded) or trivial apply list
     std::vector<Event> ev;
     c->pos_in = s->pos;
@@ -1228,7 +1232,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     c->pos_out = pos;
     const double t2 = now_s();
     c->stats.t_plan_s = t2 - t1;
-    if (s->fp64) {
+    if (s->fp64 && !blocked) {
         // complex128: one apply64 launch per fused gate; all planes and qubit
         // lists uploaded once (row a4)
         std::vector<double> planes;
@@ -1270,6 +1274,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     auto flush_passes = [&]() {
         if (run.empty()) return;
         for (auto& pd : build_passes(T, run)) {
+            pd.wide = s->fp64;
             pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
             c->stats.fma_apply += pd.fma_per_amp << s->l;
             c->stats.n_passes++;
@@ -1368,6 +1373,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             c->stats_z.n_passes = 0;
             c->stats_z.fma_apply = 0;
             for (auto& pd : pz) {
+                pd.wide = s->fp64;
                 pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
                 c->stats_z.fma_apply += pd.fma_per_amp << s->l;
                 c->stats_z.n_passes++;
@@ -1416,23 +1422,29 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             for (int q = 0; q < s->l; ++q)
                 if (std::find(p0.S.begin(), p0.S.end(), q) == p0.S.end()) out_q.push_back(q);
             const int h = (int)out_q.size(), h1 = h / 2, h2 = h - h1;
-            std::vector<float2> tab(((size_t)1 << h1) + ((size_t)1 << h2));
+            const size_t nA = (size_t)1 << h1, nB = (size_t)1 << h2;
+            std::vector<cd> tab(nA + nB);
             for (int part = 0; part < 2; ++part) {
                 const int nb = part ? h2 : h1, b0 = part ? h1 : 0;
-                float2* t = tab.data() + (part ? ((size_t)1 << h1) : 0);
+                cd* t = tab.data() + (part ? nA : 0);
                 for (size_t x = 0; x < ((size_t)1 << nb); ++x) {
                     cd z = 1.0;
                     for (int i = 0; i < nb; ++i) z *= pv[2 * out_q[b0 + i] + ((x >> i) & 1)];
-                    t[x] = make_float2((float)z.real(), (float)z.imag());
+                    t[x] = z;
                 }
             }
-            cudaError_t e = cudaMalloc(&c->ptab, tab.size() * sizeof(float2));
+            // complex64 tables (rounded once) or complex128 ones (fp64 states)
+            std::vector<float2> tab32;
+            for (const cd& z : tab) tab32.push_back(make_float2((float)z.real(), (float)z.imag()));
+            const size_t esz = s->fp64 ? sizeof(cd) : sizeof(float2);
+            const void* host = s->fp64 ? (const void*)tab.data() : (const void*)tab32.data();
+            cudaError_t e = cudaMalloc(&c->ptab, tab.size() * esz);
             if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(product-state tables)");
-            CK(s, cudaMemcpyAsync(c->ptab, tab.data(), tab.size() * sizeof(float2), cudaMemcpyHostToDevice, s->stream));
+            CK(s, cudaMemcpyAsync(c->ptab, host, tab.size() * esz, cudaMemcpyHostToDevice, s->stream));
             CK(s, cudaStreamSynchronize(s->stream));
             for (auto& l : c->steps_z[0].jitz) {
                 l.tabA = c->ptab;
-                l.tabB = c->ptab + ((size_t)1 << h1);
+                l.tabB = (const char*)c->ptab + nA * esz;
                 l.h1 = h1;
             }
         }
@@ -1527,7 +1539,8 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     const bool use_z = s->zero_pending && !c->steps_z.empty();
     const std::vector<sv_circuit::Step>& steps = use_z ? c->steps_z : c->steps;
     if (s->zero_pending) {
-        zinit = !c->small && !s->fp64 && !steps.empty() && steps[0].block && rpass_supported(steps[0].pass);
+        zinit = !c->small && !steps.empty() && steps[0].block && rpass_supported(steps[0].pass) &&
+                (!s->fp64 || !steps[0].jitz.empty());
         if (zinit) {
             s->zero_pending = false;
         } else {
@@ -1549,7 +1562,7 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
         s->pos = c->pos_out;
         return SV_OK;
     }
-    if (s->fp64) {
+    if (s->fp64 && !(steps.empty() || steps[0].block)) {
         for (auto& st : c->steps) {
             rc = launch(s, LaunchClass::HIGH, [&] {
                 return launch_apply64(reinterpret_cast<double2*>(s->shard[0]), s->l, st.a64, s->stream);
@@ -1583,8 +1596,9 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
                 if (rc) return rc;
             }
             // algorithmic bytes: read + write, or write only when |0...0> is synthesised
-            s->stats.bytes_apply += ((zinit && &st == &steps[0]) ? 8ull : 16ull) << s->l;
-            s->stats.bytes_apply_high += ((zinit && &st == &steps[0]) ? 8ull : 16ull) << s->l;
+            const uint64_t pass_bytes = ((zinit && &st == &steps[0]) ? 1ull : 2ull) * s->elem << s->l;
+            s->stats.bytes_apply += pass_bytes;
+            s->stats.bytes_apply_high += pass_bytes;
             if (!(zinit && &st == &steps[0] ? st.jitz : st.jit).empty()) s->stats.n_jit_passes += 1;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
             s->stats.fma_apply += st.pass.fma_per_amp << s->l;
@@ -2065,7 +2079,9 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
                     size_t cap, size_t* need) {
     if (!need) return fail(SV_EINVAL, "need is NULL");
     if (max_fused < 1 || max_fused > 2) return fail(SV_EINVAL, "max_fused must be in [1, 2] for register-blocked passes");
-    if (tile_bits < 10 || tile_bits > 13) return fail(SV_EINVAL, "tile_bits must be in [10, 13]");
+    const bool wide = tile_bits < 0;  // complex128 kernels
+    if (wide) tile_bits = -tile_bits;
+    if (tile_bits < 10 || tile_bits > 13) return fail(SV_EINVAL, "tile_bits must be in [10, 13] (or -13..-10)");
     int rc = validate_gates(gates, n_gates, -1);
     if (rc) return rc;
     std::vector<FusedGate> plan;
@@ -2086,6 +2102,7 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
     std::string all;
     bool first = true;
     for (auto& pd : build_passes(tile_bits, in)) {
+        pd.wide = wide;
         if (!rpass_supported(pd)) continue;
         for (int z = 0; z < (first ? 2 : 1); ++z) {
             std::vector<RpJitLaunch> ls;

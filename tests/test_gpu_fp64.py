@@ -99,3 +99,27 @@ def test_fp64_limits():
         assert e.value.code == sv.SV_EUNSUPPORTED
     finally:
         sv.sv_destroy(h)
+
+
+@pytest.mark.parametrize("n,F,bits", [(20, 1, 12), (20, 2, 12), (21, 1, 10), (22, 2, 11), (20, 1, 13)])
+@pytest.mark.parametrize("lazy", [True, False])
+def test_fp64_register_blocked_passes(n, F, bits, lazy):
+    """complex128 pass-specialised kernels (16 amplitudes per thread, wide
+    fold swizzle, fp64 FMAs): from the lazy |0...0> (product-state start) and
+    from a written one, against the complex128 oracle at fp64 tolerance."""
+    from test_gpu_circuit import _mixed_circuit, layer_depth
+    for gates, d in ((W.rqc(n, 14, seed=n + F), 14), (_mixed_circuit(n, 120, seed=n), None)):
+        d = d or layer_depth(gates)
+        ref = ref_c.run(n, gates)
+        h = sv.sv_create_ex(n, precision=1)
+        try:
+            sv.sv_set_blocking(h, bits)
+            if not lazy:
+                sv.sv_device_ptr(h)
+            st = sv.sv_run_circuit(h, gates, F)
+            got = sv.sv_get_state_c128(h, n)
+        finally:
+            sv.sv_destroy(h)
+        assert st["n_passes"] > 0 and st["n_jit_passes"] == st["n_passes"], st
+        assert osv.fidelity(got, ref) >= 1 - 1e-12
+        assert np.abs(got - ref).max() <= 1e-12 * 2.0 ** (-n / 2) * d
