@@ -104,6 +104,7 @@ struct PassDesc {
     std::vector<std::complex<double>> pinit_v;
     std::vector<double> mats64;  // complex128 states: the matrices in fp64 (same layout as mats)
     bool wide = false;           // complex128 state: pass-specialised fp64 kernel, 16 amplitudes per thread
+    bool bins = false;           // last pass of an unsharded complex64 circuit: also write the sampler's bins
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
@@ -178,8 +179,10 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
 // Prepare many passes at once (compiles in parallel host threads).
 int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local, const std::vector<char>& zinit,
                            std::vector<std::vector<RpJitLaunch>>& out);
+// bins: the sampler's bin array (kernels of a pass with PassDesc::bins write
+// the 16-amplitude S5 bin weights of the final state there)
 cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st,
-                             int slot = 0);
+                             int slot = 0, uint64_t* bins = nullptr);
 // process-wide counters (sv_jit_stats)
 void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compile_s);
 
@@ -195,8 +198,9 @@ cudaError_t launch_gather(const float2* psi, const uint64_t* phys, const int32_t
                           uint64_t count, float2* out, cudaStream_t st);
 
 // ---- sampling (S5) ----------------------------------------------------------
-constexpr int kSampleBinBits = 5;  // 32 amplitudes per fine bin
-// bins[b] = sum over the 32 amplitudes of bin b of floor(p * 2^62)
+constexpr int kSampleBinBits = 4;  // 16 amplitudes per fine bin (= the 128 B runs of a blocked pass, whose
+                                   // last pass can write the bin weights itself)
+// bins[b] = sum over the 16 amplitudes of bin b of floor(p * 2^62)
 cudaError_t launch_bin_weights(const void* psi, bool fp64, uint64_t n_amps, uint64_t* bins, cudaStream_t st);
 // inclusive prefix sum in place over `count` uint64 (scratch: >= scan_scratch_elems(count))
 size_t scan_scratch_elems(uint64_t count);

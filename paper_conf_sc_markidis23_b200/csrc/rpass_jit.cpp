@@ -32,6 +32,10 @@
 
 #include "kernels.h"
 
+#ifndef SVB_JIT_PF
+#define SVB_JIT_PF 0  // L2 bulk prefetch of the next tile at the top of each tile (pass kernels)
+#endif
+
 namespace svb {
 
 struct RpJitKernel {
@@ -154,6 +158,7 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     put(pd.r);
     put(zinit ? 1 : 0);
     put(zinit && !pd.pinit_v.empty() ? 1 : 0);
+    put(pd.bins && g1 == pd.gates.size() ? 1 : 0);
     for (int q : pd.S) put(q);
     k += '|';
     for (size_t g = g0; g < g1; ++g) {
@@ -188,6 +193,9 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     const RpPhaseHost& lp = phs.back();
     const bool direct = coalesced(lp) || coalesced8(lp);
     const bool early = direct && !zinit;
+    // sampling bin weights (the last launch of a circuit's last pass): 16-
+    // amplitude bins = tile bits 0..3, reduced over the lanes that hold them
+    const bool bins = pd.bins && g1 == pd.gates.size();
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
     std::vector<size_t> gbase(pd.gates.size(), 0);
@@ -236,11 +244,48 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     nm = mats.size() / 4;
     // parameter tail (rpj_jit_tail): psi, n_tiles, zone, h1, tabA, tabB
     const size_t off_psi = std::max<size_t>(nm, 1) * 16, off_nt = off_psi + 8, off_zone = off_psi + 16,
-                 off_h1 = off_psi + 20, off_ta = off_psi + 24, off_tb = off_psi + 32;
+                 off_h1 = off_psi + 20, off_ta = off_psi + 24, off_tb = off_psi + 32, off_bins = off_psi + 40;
     const size_t pbytes = off_psi + 48;
     if (!emit) return std::string();
 
     Ptx P;
+    // S5 weight floor(fl(re^2 + im^2) 2^62) of the packed amplitude a (the
+    // products are exact in fp64, so the FMA form equals state.cu weight()),
+    // into acc (first: set, else add)
+    auto wadd = [&](const std::string& a, bool first) {
+        P.op("mov.b64 {%lo, %hi}, ", a);
+        P.op("cvt.f64.f32 %dre, %lo");
+        P.op("cvt.f64.f32 %dim, %hi");
+        P.op("mul.rn.f64 %dp, %dim, %dim");
+        P.op("fma.rn.f64 %dp, %dre, %dre, %dp");
+        P.op("mul.rn.f64 %dp, %dp, 0d43D0000000000000");  // 2^62
+        if (first) {
+            P.op("cvt.rzi.u64.f64 %w, %dp");
+        } else {
+            P.op("cvt.rzi.u64.f64 %wt, %dp");
+            P.op("add.u64 %w, %w, %wt");
+        }
+    };
+    // sum over the low `steps` lane bits (exact uint64 butterfly), then the
+    // lane whose low bits are 0 stores the bin of the slot at address `addr`
+    auto wstore = [&](int steps, const std::string& addr) {
+        for (int st = 0; st < steps; ++st) {
+            P.op("mov.b64 {%wl, %wh}, %w");
+            P.op("shfl.sync.bfly.b32 %wl2, %wl, ", 1 << st, ", 31, -1");
+            P.op("shfl.sync.bfly.b32 %wh2, %wh, ", 1 << st, ", 31, -1");
+            P.op("mov.b64 %wt, {%wl2, %wh2}");
+            P.op("add.u64 %w, %w, %wt");
+        }
+        P.op("sub.s64 %bo, ", addr, ", %psi");
+        P.op("shr.u64 %bo, %bo, 4");
+        P.op("add.s64 %bo, %bo, %bins");
+        P.op("@%p_bw st.global.u64 [%bo], %w");
+    };
+    auto gaddr_reg = [&](const std::string& base, uint64_t off) {  // base + off into a register
+        const std::string t = P.r64();
+        P.op("add.s64 ", t, ", ", base, ", ", off);
+        return t;
+    };
     // ---- prologue: thread constants
     P.op("mov.u32 %t_id, %tid.x");
     P.op("mov.u32 %cur, rsm");
@@ -279,6 +324,12 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     P.op("ld.param.u64 %psi, [rpj_param_0+", off_psi, "]");
     P.op("ld.param.u64 %ntiles, [rpj_param_0+", off_nt, "]");
     P.op("ld.param.u32 %zone, [rpj_param_0+", off_zone, "]");
+    if (bins) {
+        P.op("ld.param.u64 %bins, [rpj_param_0+", off_bins, "]");
+        const bool b8 = direct && !lp.b0;  // coalesced8: tile bits 0..3 on lanes 0..3
+        P.op("and.b32 %r_c, %t_id, ", b8 ? 15 : 7);
+        P.op("setp.eq.u32 %p_bw, %r_c, 0");
+    }
     P.op("mov.u32 %r_c, %ctaid.x");
     P.op("cvt.u64.u32 %u, %r_c");
     P.op("mov.u32 %r_c, %nctaid.x");
@@ -305,6 +356,30 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     emit_tbase(P, pd.S, n_local, "%un", "%tbo");
     P.op("add.s64 %gtile_next, %psi, %tbo");
     P.op("add.s64 %gnext, %gtile_next, %dthr");
+    if (SVB_JIT_PF && !zinit) {
+        // pull the next tile's runs into L2 now (one bulk prefetch per run,
+        // spread over the threads), so the cp.async of the early load finds
+        // them there instead of waiting for HBM
+        const int runs = 1 << (T - pd.r);
+        const uint32_t rb = 8u << pd.r;
+        for (int i = 0; i < (runs + (int)nthr - 1) / (int)nthr; ++i) {
+            const std::string t = P.r32(), q = P.pr(), a = P.r64(), o = P.r64();
+            // run index j = tid + nthr * i -> tile index j << r
+            P.op("add.u32 ", t, ", %t_id, ", nthr * i);
+            P.op("setp.lt.u32 ", q, ", ", t, ", ", runs);
+            P.op("and.pred ", q, ", ", q, ", %p_next");
+            // offset: deposit of the run index into H (the tile's positions >= r)
+            P.op("mov.b64 ", o, ", 0");
+            for (size_t b = 0; b < tm.H.size(); ++b) {
+                const std::string tt = P.r32(), qq = P.pr();
+                P.op("and.b32 ", tt, ", ", t, ", ", 1u << b);
+                P.op("setp.ne.u32 ", qq, ", ", tt, ", 0");
+                P.op("@", qq, " add.s64 ", o, ", ", o, ", ", 8ull << tm.H[b]);
+            }
+            P.op("add.s64 ", a, ", %gtile_next, ", o);
+            P.op("@", q, " cp.async.bulk.prefetch.L2.global [", a, "], ", rb);
+        }
+    }
     P.op("cp.async.wait_group 0");
     P.op("bar.sync 0");
     // ---- phases
@@ -452,9 +527,20 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 for (int j = 0; j < NA / 2; ++j)
                     P.op("st.global.cs.v2.b64 ", gaddr(P, "%gst", 8 * tm.dep(deposit(2u * j, lp.R))), ", {%a", 2 * j, ", %a",
                          2 * j + 1, "}");
+                if (bins)
+                    for (int j = 0; j < NA / 2; ++j) {
+                        wadd("%a" + std::to_string(2 * j), true);
+                        wadd("%a" + std::to_string(2 * j + 1), false);
+                        wstore(3, gaddr_reg("%gst", 8 * tm.dep(deposit(2u * j, lp.R))));
+                    }
             } else {
                 for (int j = 0; j < NA; ++j)
                     P.op("st.global.cs.b64 ", gaddr(P, "%gst", 8 * tm.dep(deposit((uint32_t)j, lp.R))), ", %a", j);
+                if (bins)
+                    for (int j = 0; j < NA; ++j) {
+                        wadd("%a" + std::to_string(j), true);
+                        wstore(4, gaddr_reg("%gst", 8 * tm.dep(deposit((uint32_t)j, lp.R))));
+                    }
             }
         } else {
             if (Ph.b0) {
@@ -489,6 +575,12 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         for (int i = 0; i < UPT; ++i)
             P.op("st.global.cs.v2.b64 ", gaddr(P, "%gcur", 8 * tm.dep(2ull * nthr * i)), ", {%a", 2 * i, ", %a", 2 * i + 1,
                  "}");
+        if (bins)  // unit i: tile bit 0 = the pair, bits 1..3 = lane bits 0..2
+            for (int i = 0; i < UPT; ++i) {
+                wadd("%a" + std::to_string(2 * i), true);
+                wadd("%a" + std::to_string(2 * i + 1), false);
+                wstore(3, gaddr_reg("%gcur", 8 * tm.dep(2ull * nthr * i)));
+            }
     }
     P.op("mov.b64 %gcur, %gnext");
     P.op("mov.b64 %gtile, %gtile_next");
@@ -502,12 +594,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << "// T=" << T << " r=" << pd.r << " n=" << n_local << " S={";
     for (int q : pd.S) k << q << ",";
     k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (pinit ? " product-start" : "")
-      << (direct ? " direct" : "") << "\n";
+      << (direct ? " direct" : "") << (bins ? " bins" : "") << "\n";
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
     k << ".maxntid " << nthr << ", 1, 1\n.maxnreg 128\n{\n";
-    k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z;\n";
+    k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw;\n";
+    k << "\t.reg .f64 %dre, %dim, %dp;\n\t.reg .b64 %w, %wt, %bo, %bins;\n\t.reg .b32 %wl, %wh, %wl2, %wh2;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
     k << "\t.reg .b64 %a<32>;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
@@ -1015,7 +1108,8 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     return SV_OK;
 }
 
-cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st, int slot) {
+cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st, int slot,
+                             uint64_t* bins) {
     RpJitKernel& K = *l.kern;
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -1053,6 +1147,7 @@ cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool 
     std::memcpy(prm.data() + off + 20, &l.h1, 4);
     std::memcpy(prm.data() + off + 24, &l.tabA, 8);
     std::memcpy(prm.data() + off + 32, &l.tabB, 8);
+    std::memcpy(prm.data() + off + 40, &bins, 8);
     void* args[] = {prm.data()};
     return cudaLaunchKernel((const void*)K.kern, dim3((unsigned)grid), dim3((unsigned)K.nthr), args, K.smem, st);
 }

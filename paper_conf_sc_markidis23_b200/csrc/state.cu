@@ -64,15 +64,13 @@ __device__ __forceinline__ uint64_t weight(double2 a) {
     return __double2ull_rz(p * 0x1p62);
 }
 
-__device__ __forceinline__ void load4w(const float2* psi, uint64_t i0, uint64_t& w) {
+// kAmpsPerLane = 2 consecutive amplitudes per lane (8 lanes per 16-amplitude bin)
+__device__ __forceinline__ void load_lane_w(const float2* psi, uint64_t i0, uint64_t& w) {
     const float4 u = __ldcs(reinterpret_cast<const float4*>(psi + i0));
-    const float4 v = __ldcs(reinterpret_cast<const float4*>(psi + i0 + 2));
-    w = weight(make_float2(u.x, u.y)) + weight(make_float2(u.z, u.w)) + weight(make_float2(v.x, v.y)) +
-        weight(make_float2(v.z, v.w));
+    w = weight(make_float2(u.x, u.y)) + weight(make_float2(u.z, u.w));
 }
-__device__ __forceinline__ void load4w(const double2* psi, uint64_t i0, uint64_t& w) {
-    w = weight(__ldcs(psi + i0)) + weight(__ldcs(psi + i0 + 1)) + weight(__ldcs(psi + i0 + 2)) +
-        weight(__ldcs(psi + i0 + 3));
+__device__ __forceinline__ void load_lane_w(const double2* psi, uint64_t i0, uint64_t& w) {
+    w = weight(__ldcs(psi + i0)) + weight(__ldcs(psi + i0 + 1));
 }
 
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
@@ -81,23 +79,25 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
     return v;
 }
 
-// 8 lanes per 32-amplitude bin, 4 amplitudes per lane.
+// 8 lanes per 16-amplitude bin, 2 amplitudes per lane.
+constexpr int kAmpsPerLane = (1 << kSampleBinBits) / 8;
+static_assert(kAmpsPerLane == 2, "bin_weights_kernel loads 2 amplitudes per lane");
 template <class E>
 __global__ void bin_weights_kernel(const E* __restrict__ psi, uint64_t n_amps, uint64_t* __restrict__ bins,
                                    uint64_t n_bins) {
     const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;  // multiple of 32
     const int sub = threadIdx.x & 7;
-    const uint64_t full_bins = n_amps >> kSampleBinBits;  // bins with all 32 amplitudes
+    const uint64_t full_bins = n_amps >> kSampleBinBits;  // bins with all 16 amplitudes
     // warp-uniform loop (4 bins per warp per trip) so the shuffles see all lanes
     for (uint64_t b0 = (tid >> 5) << 2; b0 < n_bins; b0 += (nthr >> 5) << 2) {
         const uint64_t b = b0 + ((threadIdx.x & 31) >> 3);
         uint64_t w = 0;
-        const uint64_t i0 = (b << kSampleBinBits) + 4 * sub;
+        const uint64_t i0 = (b << kSampleBinBits) + kAmpsPerLane * sub;
         if (b < full_bins) {
-            load4w(psi, i0, w);
+            load_lane_w(psi, i0, w);
         } else if (b < n_bins) {
-            for (int j = 0; j < 4; ++j)
+            for (int j = 0; j < kAmpsPerLane; ++j)
                 if (i0 + j < n_amps) w += weight(psi[i0 + j]);
         }
         w += __shfl_xor_sync(0xffffffffu, w, 1);

@@ -24,6 +24,9 @@
 
 using namespace svb;
 
+#ifndef SVB_FUSED_BINS
+#define SVB_FUSED_BINS 1  // the last register-blocked pass writes the sampler's bin weights
+#endif
 #ifndef SVB_PASS_PIN
 #define SVB_PASS_PIN 4  // qubits 0..PIN-1 in every blocked-pass tile (runs of 8 * 2^PIN bytes)
 #endif
@@ -81,6 +84,9 @@ struct sv_state {
     int pass_jit = 1;         // SV_OPT_PASS_JIT
     int diag_skip = 1;        // SV_OPT_DIAG_SKIP
     bool sample_pending = false;  // a sv_sample_device status word not yet checked
+    // the sampler's bins hold the current state's S5 weights (written by the
+    // last register-blocked pass of the last circuit); any state change clears it
+    bool bins_valid = false;
     size_t elem = 8;          // bytes per amplitude
     // staging ring for per-call device inputs of sv_apply_fused /
     // sv_apply_controlled (k = 6 matrices, int8 W slices, fp64 planes): a
@@ -483,7 +489,7 @@ uint64_t phys_of(const sv_state* s, uint64_t i) {
 }
 
 int alloc_scratch(sv_state* s) {
-    const uint64_t nb_local = (s->local_amps() + 31) >> 5;
+    const uint64_t nb_local = (s->local_amps() + (1u << kSampleBinBits) - 1) >> kSampleBinBits;
     const uint64_t nb = nb_local * s->local_shards();
     cudaError_t e = cudaMalloc(&s->bins, nb * sizeof(uint64_t));
     if (e != cudaSuccess) return fail(SV_ENOMEM, "cudaMalloc(bins) failed");
@@ -753,7 +759,8 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
     } else {
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
-        if (need_bytes + (need_bytes >> 5) + (64ull << 20) > free_b)
+        const size_t bins_bytes = 8 * ((((size_t)1 << l) >> kSampleBinBits) + 1) * (virt ? world : 1);
+        if (need_bytes + bins_bytes + (64ull << 20) > free_b)
             return fail(SV_ENOMEM, "state does not fit in free device memory");
         cudaError_t e = cudaMalloc(&s->alloc, need_bytes);
         if (e != cudaSuccess) return fail(SV_ENOMEM, std::string("cudaMalloc(state): ") + cudaGetErrorString(e));
@@ -798,6 +805,7 @@ int sv_reset(sv_state* s) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
     if (s->sticky) return fail(SV_EBADSTATE, "state poisoned by an earlier device failure");
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
+    s->bins_valid = false;
     if (!s->ext_buf) {
         s->zero_pending = true;  // written lazily (see sv_state::zero_pending)
         return SV_OK;
@@ -817,6 +825,7 @@ static int materialize(sv_state* s) {
 }
 
 static int write_zero_state(sv_state* s) {
+    s->bins_valid = false;
     for (int d = 0; d < s->local_shards(); ++d) {
         const int shard = s->virt ? d : s->rank;
         float2* psi = s->shard[shard];
@@ -867,6 +876,7 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
     if (s->fp64 && k > 5) return fail(SV_EUNSUPPORTED, "complex128 states support fused gates with k <= 5");
     rc = materialize(s);
     if (rc) return rc;
+    s->bins_valid = false;
     std::vector<cd> M = Min;
     std::vector<int> q(qubits, qubits + k);
     if (s->fp64) {
@@ -962,6 +972,7 @@ int sv_apply_controlled(sv_state* s, int n_ctrl, const int32_t* controls, int k,
     if (subspace) {
         rc = materialize(s);
         if (rc) return rc;
+        s->bins_valid = false;
         // tile engine over the control-1 subspace only: 2^-n_ctrl of the state
         ApplyDesc d;
         make_apply(s->l, k, targets, M.data(), d);
@@ -1385,6 +1396,11 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             }
         }
     }
+    // the last pass of an unsharded complex64 circuit also writes the
+    // sampler's bin weights (sv_sample then skips its read of the state)
+    if (SVB_FUSED_BINS && blocked && s->pass_jit && s->g == 0 && !s->fp64)
+        for (auto* list : {&c->steps, &c->steps_z})
+            if (!list->empty() && list->back().block && rpass_supported(list->back().pass)) list->back().pass.bins = true;
     // pass-specialised kernels of every register-blocked pass (compiled in
     // parallel, cached per process; the first pass also in its |0...0> form)
     if (blocked && s->pass_jit) {
@@ -1524,6 +1540,7 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     if (!c || c->owner != s) return fail(SV_EINVAL, "circuit is NULL or belongs to another state");
     if (s->pos != c->pos_in) return fail(SV_EINVAL, "state qubit map differs from the circuit's (sv_reset first)");
     Nvtx nv("sv.circuit_run");
+    s->bins_valid = false;
     const sv_stats keep = c->stats;
     reset_stats(s);
     s->stats.t_fuse_s = keep.t_fuse_s;
@@ -1583,8 +1600,10 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
                 const std::vector<RpJitLaunch>& jl = z ? st.jitz : st.jit;
                 if (!jl.empty()) {
                     for (const auto& l : jl) {
-                        rc = launch(s, LaunchClass::HIGH,
-                                    [&] { return launch_rpass_jit(psi, s->l, l, shard == 0, s->stream, sh); });
+                        rc = launch(s, LaunchClass::HIGH, [&] {
+                            return launch_rpass_jit(psi, s->l, l, shard == 0, s->stream, sh,
+                                                    st.pass.bins ? s->bins : nullptr);
+                        });
                         if (rc) return rc;
                     }
                     continue;
@@ -1621,6 +1640,9 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
         if (rc) return rc;
     }
     s->pos = c->pos_out;
+    // the last pass wrote the final state's sampling bins
+    s->bins_valid = s->g == 0 && !s->fp64 && !steps.empty() && steps.back().block && steps.back().pass.bins &&
+                    !(zinit && steps.size() == 1 ? steps.back().jitz : steps.back().jit).empty();
     return SV_OK;
 }
 
@@ -1785,18 +1807,21 @@ static int sample_impl(sv_state* s, uint64_t seed, size_t N, uint64_t* dev_out) 
     int rc = canonicalize(s);
     if (rc) return rc;
     const uint64_t La = s->local_amps();
-    const uint64_t nb = (La + 31) >> 5;
+    const uint64_t nb = (La + (1u << kSampleBinBits) - 1) >> kSampleBinBits;
     const int nloc = s->local_shards();
     // per local shard: bin weights + inclusive scan
     for (int i = 0; i < nloc; ++i) {
         const int d = s->virt ? i : s->rank;
         uint64_t* bins = s->bins + (size_t)i * nb;
-        rc = launch(s, LaunchClass::OTHER,
-                    [&] { return launch_bin_weights(s->shard[d], s->fp64, La, bins, s->stream); });
-        if (rc) return rc;
+        if (!s->bins_valid) {  // else the circuit's last pass wrote them
+            rc = launch(s, LaunchClass::OTHER,
+                        [&] { return launch_bin_weights(s->shard[d], s->fp64, La, bins, s->stream); });
+            if (rc) return rc;
+        }
         rc = launch(s, LaunchClass::OTHER, [&] { return launch_inclusive_scan(bins, nb, s->scan_scratch, s->stream); });
         if (rc) return rc;
     }
+    s->bins_valid = false;  // the scan ran in place: the weights are consumed
     // totals pointers (shard d's total = last element of its prefix) and sigma
     std::vector<const uint64_t*> tp(s->world);
     std::vector<int32_t> sig(s->world);
@@ -1880,6 +1905,7 @@ int sv_sample(sv_state* s, uint64_t seed, size_t n_samples, uint64_t* out) {
 // ---- whole state ------------------------------------------------------------------
 static int set_state_bytes(sv_state* s, const void* host) {
     s->zero_pending = false;  // every amplitude is overwritten
+    s->bins_valid = false;
     for (int q = 0; q < s->n; ++q) s->pos[q] = q;
     const size_t sb = s->elem << s->l;
     for (int i = 0; i < s->local_shards(); ++i) {
@@ -1964,6 +1990,7 @@ int sv_device_ptr(sv_state* s, int shard, void** out) {
     if (!out) return fail(SV_EINVAL, "NULL argument");
     if (shard < 0 || shard >= s->world || !s->shard[shard]) return fail(SV_EINVAL, "shard not available here");
     if (!s->virt && shard != s->rank) return fail(SV_EINVAL, "multi-process mode: only this rank's shard");
+    s->bins_valid = false;  // the caller may write the memory
     if (s->zero_pending) {  // the caller may read the memory: write |0...0> now
         int rc = materialize(s);
         if (rc == SV_OK) rc = sync(s);
@@ -2101,7 +2128,9 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
     }
     std::string all;
     bool first = true;
-    for (auto& pd : build_passes(tile_bits, in)) {
+    auto passes = build_passes(tile_bits, in);
+    if (!wide && !passes.empty() && rpass_supported(passes.back())) passes.back().bins = true;  // as sv_circuit_create
+    for (auto& pd : passes) {
         pd.wide = wide;
         if (!rpass_supported(pd)) continue;
         for (int z = 0; z < (first ? 2 : 1); ++z) {

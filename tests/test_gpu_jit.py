@@ -154,3 +154,33 @@ def test_jit_30q_sampled_amplitudes_match_generic():
     err = np.abs(out[True, True].astype(np.complex128) - out[False, False].astype(np.complex128)).max()
     bound = 1e-5 * 2.0 ** (-n / 2) * d
     assert err <= bound, (err, bound)
+
+
+@pytest.mark.parametrize("bits", [10, 11, 12, 13])
+@pytest.mark.parametrize("F", [1, 2])
+def test_fused_sampling_bins_bit_exact(bits, F):
+    """The circuit's last pass writes the sampler's 16-amplitude S5 bin
+    weights (no separate read of the state): samples are bit-identical to
+    the oracle sampler on the GPU's final complex64 state, also for a second
+    draw (bins recomputed) and after a state change.  RQC and mixed circuits
+    cover the three store layouts of the last pass."""
+    from oracle import sample as osample
+    n = 21
+    for gates in (W.rqc(n, 12, seed=bits + F), _mixed_circuit(n, 150, seed=3 * bits + F)):
+        h = sv.sv_create(n)
+        try:
+            sv.sv_set_blocking(h, bits)
+            c = sv.sv_circuit_create(h, gates, F)
+            sv.sv_circuit_run_device(h, c)
+            got1 = sv.sv_sample(h, 11, 4000)
+            got2 = sv.sv_sample(h, 12, 4000)
+            psi = sv.sv_get_state(h, n)
+            sv.sv_apply_fused(h, [5], W.GATE_H.astype(np.complex64))
+            got3 = sv.sv_sample(h, 13, 4000)
+            psi3 = sv.sv_get_state(h, n)
+            sv.sv_circuit_destroy(c)
+        finally:
+            sv.sv_destroy(h)
+        assert np.array_equal(got1, osample.sample(psi, 11, 4000)[0])
+        assert np.array_equal(got2, osample.sample(psi, 12, 4000)[0])
+        assert np.array_equal(got3, osample.sample(psi3, 13, 4000)[0])

@@ -171,6 +171,7 @@ def test_pass_kernels_assemble(n, d, F, T, tmp_path):
         spill = int(re.search(r"(\d+) bytes spill stores", out.stderr).group(1))
         assert spill <= 256, out.stderr[-800:]
     assert "zinit" in srcs[1] and "zinit" not in srcs[0]
+    assert " bins" in srcs[-1].split("\n")[1]  # the last pass writes the sampler bins
 
 
 def test_options_validate():

@@ -1,0 +1,23 @@
+import json, os, subprocess, sys
+CHILD = r'''
+import sys, time, json
+sys.path.insert(0, "/root/repo")
+import torch
+import paper_conf_sc_markidis23_b200 as sv
+from workloads import rqc as W
+n=30; h=sv.sv_create(n); c=sv.sv_circuit_create(h, W.rqc(n,14), 1)
+out=torch.empty(1000000, dtype=torch.int64, device="cuda")
+def step():
+    sv.sv_reset(h); sv.sv_circuit_run_device(h,c); sv.sv_sample_device(h,1,1000000,out.data_ptr())
+for _ in range(3): step()
+sv.sv_synchronize(h)
+t0=time.perf_counter()
+for _ in range(10): step()
+sv.sv_synchronize(h)
+print(json.dumps({"step_ms": (time.perf_counter()-t0)/10*1e3}))
+'''
+libs = sys.argv[2:]
+for r in range(int(sys.argv[1])):
+    for lib in libs:
+        o = subprocess.run([sys.executable, "-c", CHILD], env=dict(os.environ, SVB200_LIB=lib), capture_output=True, text=True)
+        print(os.path.basename(lib), o.stdout.strip()[-60:] or o.stderr[-300:], flush=True)

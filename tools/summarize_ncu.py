@@ -19,7 +19,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def kclass(name: str) -> str:
-    if "apply_rpass" in name or "apply_pass" in name:
+    if "apply_rpass" in name or "apply_pass" in name or name.startswith("rpj"):
         return "rpass"
     if "apply_tci" in name or "apply_tc" in name:
         return "apply_tc"
