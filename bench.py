@@ -446,9 +446,15 @@ def run_ours(args):
     # CUDA events on the launching stream, 1 warm-up + 3 timed steps each;
     # the fastest max_fused becomes the timed configuration (max_fused = -1)
     sweep = None
+    pin_sweep = None
+    pass_pin = 4
     if not fp64 and world == 1 and not args.no_sweep:
         sweep = {}
-        for f in range(1, 7):
+        pin_sweep = {}
+        # max_fused 1..6 at the default pass runs (128 B), and F <= 2 (the
+        # register-blocked passes) also with 64 B runs (SV_OPT_PASS_PIN 3)
+        for f, pin in [(f, 4) for f in range(1, 7)] + [(1, 3), (2, 3)]:
+            sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pin)
             c = sv.sv_circuit_create(h, gates, f)
 
             def st_f():
@@ -465,12 +471,16 @@ def run_ours(args):
                 st_f()
             a1.record(stream)
             barrier()
-            sweep[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
+            (sweep if pin == 4 else pin_sweep)[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
             sv.sv_circuit_destroy(c)
+        sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, 4)
     if args.max_fused < 0:
         if sweep:
-            args.max_fused = int(min(sweep, key=sweep.get))
-            fusion_choice = "optimal over max_fused 1..6 (fusion_sweep_s)"
+            best = min([(v, int(f), 4) for f, v in sweep.items()] + [(v, int(f), 3) for f, v in pin_sweep.items()])
+            args.max_fused, pass_pin = best[1], best[2]
+            sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pass_pin)
+            fusion_choice = ("optimal over max_fused 1..6 (fusion_sweep_s) and, for the register-blocked passes "
+                             "(F <= 2), 128 B or 64 B tile runs (pass_pin_sweep_s)")
         else:
             args.max_fused = 1 if not fp64 else 4
             fusion_choice = ("1 (the single-GPU optimum: register-blocked passes between the exchanges)" if not fp64
@@ -610,7 +620,8 @@ def run_ours(args):
                 "workload": f"{args.workload}_{n}q_d{depth}",
                 "n_qubits": n, "depth": depth, "max_fused": args.max_fused, "fusion": fusion_choice,
                 "execution": ("register-blocked passes (pass-specialised kernels), tile qubits "
-                              f"{cst.get('block_bits', 13)}" if cst.get("n_passes", 0) else "one launch per fused gate"),
+                              f"{cst.get('block_bits', 13)}, runs of {8 << pass_pin} B (SV_OPT_PASS_PIN {pass_pin})"
+                              if cst.get("n_passes", 0) else "one launch per fused gate"),
                 "seed": args.seed,
                 "gates": len(gates), "n_fused": sv_fused, "fused_hist": cst["fused_hist"],
                 "samples_per_step": args.samples,
@@ -656,6 +667,7 @@ def run_ours(args):
                     "d2h_bytes_per_step": 8 * args.samples},
             "gpu_launches": (acc["n_launch_high"] + acc["n_launch_low"] + acc["n_launch_other"]),
             "fusion_sweep_s": sweep,
+            "pass_pin_sweep_s": pin_sweep,
             "optimal_fusion": (None if not sweep else
                                {"max_fused": int(min(sweep, key=sweep.get)), "value": min(sweep.values()), "unit": "s"}),
             "clocks": clk.summary(),

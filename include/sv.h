@@ -295,6 +295,11 @@ int sv_synchronize(sv_state* s);
  *                      tensor-core path, k <= 4 SIMT), SV_PATH_SIMT,
  *                      SV_PATH_INT8 (int8 tensor cores for k = 4..6);
  *   SV_OPT_TIMING      = sv_set_timing;
+ *   SV_OPT_PASS_PIN    v in {3, 4, 5}: every blocked-pass tile holds qubits
+ *                      0..v-1 (contiguous runs of 8 * 2^v bytes; default 4 =
+ *                      128 B).  64 B runs leave one more tile slot per pass
+ *                      (fewer passes) at some DRAM efficiency: which wins
+ *                      depends on the circuit (30q D14: 3, 32q D20: 4);
  *   SV_OPT_DIAG_SKIP   1 (default): sharded circuits (sv_circuit_create) do
  *                      not exchange a global qubit for a fused gate that is
  *                      block-diagonal in it (sv_shard_plan_diag); 0: plain S4.
@@ -305,6 +310,7 @@ int sv_synchronize(sv_state* s);
 #define SV_OPT_APPLY_PATH 3
 #define SV_OPT_TIMING 4
 #define SV_OPT_DIAG_SKIP 5  /* 1 (default): sharded circuits plan with the diagonal exchange skip */
+#define SV_OPT_PASS_PIN 6   /* qubits 0..v-1 in every blocked-pass tile (runs of 8*2^v bytes): 3, 4 (default), 5 */
 #define SV_PATH_AUTO 0
 #define SV_PATH_SIMT 1
 #define SV_PATH_INT8 2

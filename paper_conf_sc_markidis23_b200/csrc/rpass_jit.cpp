@@ -195,7 +195,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     const bool early = direct && !zinit;
     // sampling bin weights (the last launch of a circuit's last pass): 16-
     // amplitude bins = tile bits 0..3, reduced over the lanes that hold them
-    const bool bins = pd.bins && g1 == pd.gates.size();
+    const bool bins = pd.bins && g1 == pd.gates.size() && pd.r >= kSampleBinBits;
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
     std::vector<size_t> gbase(pd.gates.size(), 0);

@@ -83,6 +83,7 @@ struct sv_state {
     int tc_mode = 3;          // SV_OPT_APPLY_PATH
     int pass_jit = 1;         // SV_OPT_PASS_JIT
     int diag_skip = 1;        // SV_OPT_DIAG_SKIP
+    int pass_pin = SVB_PASS_PIN;  // SV_OPT_PASS_PIN: qubits 0..pin-1 in every blocked-pass tile
     bool sample_pending = false;  // a sv_sample_device status word not yet checked
     // the sampler's bins hold the current state's S5 weights (written by the
     // last register-blocked pass of the last circuit); any state change clears it
@@ -602,8 +603,7 @@ int kind_of(const std::vector<cd>& M, int k) {
 // tile set S is the pinned qubits, the pass's qubits, then the lowest
 // remaining qubits (longer runs).  The state never moves: a pass only
 // chooses which amplitudes share a tile.
-std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in) {
-    constexpr int kPassPinned = SVB_PASS_PIN;
+std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPassPinned = SVB_PASS_PIN) {
     const uint64_t pin = (1ull << kPassPinned) - 1ull;
     const int Fp = T - kPassPinned;
     const size_t nf = in.size();
@@ -1284,7 +1284,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     std::vector<PassIn> run, run_all;
     auto flush_passes = [&]() {
         if (run.empty()) return;
-        for (auto& pd : build_passes(T, run)) {
+        for (auto& pd : build_passes(T, run, s->pass_pin)) {
             pd.wide = s->fp64;
             pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
             c->stats.fma_apply += pd.fma_per_amp << s->l;
@@ -1374,7 +1374,7 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             }
             for (int b = 0; b < g.k; ++b) seen[g.q[b]] = 1;
         }
-        std::vector<PassDesc> pz = (nfold && !rest.empty()) ? build_passes(T, rest) : std::vector<PassDesc>{};
+        std::vector<PassDesc> pz = (nfold && !rest.empty()) ? build_passes(T, rest, s->pass_pin) : std::vector<PassDesc>{};
         if (!pz.empty() && rpass_supported(pz[0])) {
             for (int p = 0; p < (int)pz[0].S.size(); ++p) {
                 pz[0].pinit_v.push_back(pv[2 * pz[0].S[p]]);
@@ -1400,7 +1400,9 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
     // sampler's bin weights (sv_sample then skips its read of the state)
     if (SVB_FUSED_BINS && blocked && s->pass_jit && s->g == 0 && !s->fp64)
         for (auto* list : {&c->steps, &c->steps_z})
-            if (!list->empty() && list->back().block && rpass_supported(list->back().pass)) list->back().pass.bins = true;
+            if (!list->empty() && list->back().block && rpass_supported(list->back().pass) &&
+                list->back().pass.r >= kSampleBinBits)  // bins = 16 consecutive amplitudes = tile bits 0..3
+                list->back().pass.bins = true;
     // pass-specialised kernels of every register-blocked pass (compiled in
     // parallel, cached per process; the first pass also in its |0...0> form)
     if (blocked && s->pass_jit) {
@@ -2094,6 +2096,10 @@ int sv_set_option(sv_state* s, int option, int value) {
             s->tc_mode = value == SV_PATH_AUTO ? 3 : value == SV_PATH_INT8 ? 2 : 0;
             return SV_OK;
         case SV_OPT_TIMING: return sv_set_timing(s, value);
+        case SV_OPT_PASS_PIN:
+            if (value < 3 || value > 5) return fail(SV_EINVAL, "SV_OPT_PASS_PIN takes 3, 4 or 5");
+            s->pass_pin = value;
+            return SV_OK;
         case SV_OPT_DIAG_SKIP:
             if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_DIAG_SKIP takes 0 or 1");
             s->diag_skip = value;
@@ -2129,7 +2135,8 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
     std::string all;
     bool first = true;
     auto passes = build_passes(tile_bits, in);
-    if (!wide && !passes.empty() && rpass_supported(passes.back())) passes.back().bins = true;  // as sv_circuit_create
+    if (!wide && !passes.empty() && rpass_supported(passes.back()) && passes.back().r >= kSampleBinBits)
+        passes.back().bins = true;  // as sv_circuit_create
     for (auto& pd : passes) {
         pd.wide = wide;
         if (!rpass_supported(pd)) continue;

@@ -184,3 +184,34 @@ def test_fused_sampling_bins_bit_exact(bits, F):
         assert np.array_equal(got1, osample.sample(psi, 11, 4000)[0])
         assert np.array_equal(got2, osample.sample(psi, 12, 4000)[0])
         assert np.array_equal(got3, osample.sample(psi3, 13, 4000)[0])
+
+
+@pytest.mark.parametrize("pin", [3, 5])
+@pytest.mark.parametrize("F", [1, 2])
+def test_pass_pin_option(pin, F):
+    """SV_OPT_PASS_PIN: tiles pinned to qubits 0..pin-1 (64 B / 256 B runs):
+    JIT == generic bit for bit from a written |0...0>, oracle parity from the
+    lazy one, and sampling bit-exact whether or not the last pass can write
+    the 16-amplitude bins (it needs tile bits 0..3 = qubits 0..3)."""
+    from oracle import sample as osample
+    n, d = 21, 12
+    gates = W.rqc(n, d, seed=pin + F)
+    out = {}
+    for jit, lazy in ((1, False), (0, False), (1, True)):
+        h = sv.sv_create(n)
+        try:
+            sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pin)
+            sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, jit)
+            sv.sv_set_blocking(h, 12)
+            if not lazy:
+                sv.sv_device_ptr(h)
+            st = sv.sv_run_circuit(h, gates, F)
+            smp = sv.sv_sample(h, 3, 3000)
+            psi = sv.sv_get_state(h, n)
+        finally:
+            sv.sv_destroy(h)
+        assert st["n_passes"] > 0
+        assert np.array_equal(smp, osample.sample(psi, 3, 3000)[0])
+        out[jit, lazy] = psi
+    assert np.array_equal(out[1, False].view(np.uint32), out[0, False].view(np.uint32))
+    _check(n, d, out[1, True], ref_c.run(n, gates))
