@@ -75,6 +75,7 @@ def parse():
                          "depth = cycles")
     ap.add_argument("--samples", type=int, default=N_SAMPLES)
     ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
+    ap.add_argument("--pass-pin", type=int, default=0, help="fix SV_OPT_PASS_PIN (3: 64 B runs, 4: 128 B) instead of sweeping")
     ap.add_argument("--precision", type=int, default=32, choices=[32, 64], help="complex64 (32) or complex128 (64) state")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sweep", action="store_true",
@@ -435,6 +436,8 @@ def run_ours(args):
         sv.sv_attach_peers(h, blobs)
     if args.block_bits >= 0:
         sv.sv_set_blocking(h, args.block_bits)
+    if args.pass_pin:
+        sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, args.pass_pin)
     samples_dev = torch.empty(args.samples, dtype=torch.int64, device="cuda")
 
     def barrier():
@@ -447,7 +450,7 @@ def run_ours(args):
     # the fastest max_fused becomes the timed configuration (max_fused = -1)
     sweep = None
     pin_sweep = None
-    pass_pin = 4
+    pass_pin = args.pass_pin or 4
     if not fp64 and world == 1 and not args.no_sweep:
         sweep = {}
         pin_sweep = {}
@@ -473,7 +476,7 @@ def run_ours(args):
             barrier()
             (sweep if pin == 4 else pin_sweep)[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
             sv.sv_circuit_destroy(c)
-        sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, 4)
+        sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pass_pin)
     if args.max_fused < 0:
         if sweep:
             best = min([(v, int(f), 4) for f, v in sweep.items()] + [(v, int(f), 3) for f, v in pin_sweep.items()])

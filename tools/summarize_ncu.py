@@ -109,8 +109,9 @@ def main():
     caps = [c for one in fp.split(",") for c in captures(one)]
     if caps:
         summary["full_capture"] = caps
-        for c in caps:
-            summary["traffic_per_launch"].setdefault(kclass(c["kernel"]), c["traffic_bytes"])
+        for c in caps:  # a full (read + write) pass: the largest capture of the class
+            k = kclass(c["kernel"])
+            summary["traffic_per_launch"][k] = max(summary["traffic_per_launch"].get(k, 0), c["traffic_bytes"])
     old = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if os.path.exists(old):  # keep per-class traffic of kernels not captured this time
         for k, v in json.load(open(old)).get("traffic_per_launch", {}).items():
