@@ -32,6 +32,12 @@
 
 #include "kernels.h"
 
+#ifndef SVB_JIT_SECTOR_DIRECT
+#define SVB_JIT_SECTOR_DIRECT 1  // direct stores also for 32 B-sector layouts of the last phase
+#endif
+#ifndef SVB_JIT_RING
+#define SVB_JIT_RING 0  // two warp groups over three tile buffers per CTA (loads 1.5 tiles ahead)
+#endif
 #ifndef SVB_JIT_PF
 #define SVB_JIT_PF 0  // L2 bulk prefetch of the next tile at the top of each tile (pass kernels)
 #endif
@@ -42,6 +48,7 @@ struct RpJitKernel {
     std::string key;  // chunk_key (cache key)
     std::string src;  // PTX
     int nthr = 0;
+    int T = 0;
     size_t smem = 0;
     size_t param_bytes = 0;  // sizeof(JP) of the generated kernel
     size_t nm = 0;           // float4 matrix slots
@@ -191,11 +198,25 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         return !h.b0 && h.lanes.size() >= 4 && h.lanes[0] == 0 && h.lanes[1] == 1 && h.lanes[2] == 2 && h.lanes[3] == 3;
     };
     const RpPhaseHost& lp = phs.back();
-    const bool direct = coalesced(lp) || coalesced8(lp);
+    // direct store of the last phase's registers: full 128 B runs per quarter-
+    // (16 B) / half-warp (8 B), or -- SVB_JIT_SECTOR_DIRECT -- full 32 B
+    // sectors per lane pair / quad (the L2 merges the sectors of a line before
+    // write-back; the whole tile is written by this CTA)
+    auto sector = [](const RpPhaseHost& h) {
+        return h.b0 ? (h.lanes.size() >= 1 && h.lanes[0] == 1)
+                    : (h.lanes.size() >= 2 && h.lanes[0] == 0 && h.lanes[1] == 1);
+    };
+    const bool direct = coalesced(lp) || coalesced8(lp) || (SVB_JIT_SECTOR_DIRECT && sector(lp));
     const bool early = direct && !zinit;
     // sampling bin weights (the last launch of a circuit's last pass): 16-
     // amplitude bins = tile bits 0..3, reduced over the lanes that hold them
     const bool bins = pd.bins && g1 == pd.gates.size() && pd.r >= kSampleBinBits;
+    // ring (SVB_JIT_RING): two warp groups per CTA, each on its own tiles,
+    // over three tile buffers; the group that releases buffer b (its last
+    // read of tile k) loads tile k + 3 (the other group's) into it, tracked by
+    // an mbarrier -- loads are issued one and a half tiles ahead
+    const bool ring = SVB_JIT_RING != 0;
+    const uint32_t tile_bytes = 8u << T;
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
     std::vector<size_t> gbase(pd.gates.size(), 0);
@@ -266,13 +287,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("add.u64 %w, %w, %wt");
         }
     };
-    // sum over the low `steps` lane bits (exact uint64 butterfly), then the
-    // lane whose low bits are 0 stores the bin of the slot at address `addr`
-    auto wstore = [&](int steps, const std::string& addr) {
-        for (int st = 0; st < steps; ++st) {
+    // sum over the lane bits `lbits` (exact uint64 butterfly), then the lane
+    // whose bits there are 0 (%p_bw) stores the bin of the slot at `addr`
+    auto wstore = [&](const std::vector<int>& lbits, const std::string& addr) {
+        for (int b : lbits) {
             P.op("mov.b64 {%wl, %wh}, %w");
-            P.op("shfl.sync.bfly.b32 %wl2, %wl, ", 1 << st, ", 31, -1");
-            P.op("shfl.sync.bfly.b32 %wh2, %wh, ", 1 << st, ", 31, -1");
+            P.op("shfl.sync.bfly.b32 %wl2, %wl, ", 1 << b, ", 31, -1");
+            P.op("shfl.sync.bfly.b32 %wh2, %wh, ", 1 << b, ", 31, -1");
             P.op("mov.b64 %wt, {%wl2, %wh2}");
             P.op("add.u64 %w, %w, %wt");
         }
@@ -288,7 +309,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     };
     // ---- prologue: thread constants
     P.op("mov.u32 %t_id, %tid.x");
+    P.op("mov.u32 %rsm0, rsm");
     P.op("mov.u32 %cur, rsm");
+    if (ring) {
+        P.op("shr.u32 %grp, %t_id, ", tbits);
+        P.op("and.b32 %t_id, %t_id, ", nthr - 1);  // thread index within the group
+        P.op("add.u32 %bid, %grp, 1");
+    }
     P.op("mov.b64 %dthr, 0");
     P.op("mov.b32 %sthr, 0");
     if (direct) P.op("mov.b64 %dg, 0");
@@ -324,21 +351,30 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     P.op("ld.param.u64 %psi, [rpj_param_0+", off_psi, "]");
     P.op("ld.param.u64 %ntiles, [rpj_param_0+", off_nt, "]");
     P.op("ld.param.u32 %zone, [rpj_param_0+", off_zone, "]");
+    // bin layout: the last phase's register / lane bits that hold tile bits
+    // 0..3 (direct store), or the write-back units (tile bit 0 = the pair,
+    // bits 1..3 = lane bits 0..2)
+    uint32_t bin_regs = 0;
+    std::vector<int> bin_lanes;
+    if (direct) {
+        for (int j = 0; j < M; ++j)
+            if (lp.R[j] < 4) bin_regs |= 1u << j;
+        for (int b = 0; b < tbits; ++b)
+            if (lp.lanes[b] < 4) bin_lanes.push_back(b);
+    } else {
+        bin_lanes = {0, 1, 2};
+    }
     if (bins) {
         P.op("ld.param.u64 %bins, [rpj_param_0+", off_bins, "]");
-        const bool b8 = direct && !lp.b0;  // coalesced8: tile bits 0..3 on lanes 0..3
-        P.op("and.b32 %r_c, %t_id, ", b8 ? 15 : 7);
+        uint32_t lm = 0;
+        for (int b : bin_lanes) lm |= 1u << b;
+        P.op("and.b32 %r_c, %t_id, ", lm);
         P.op("setp.eq.u32 %p_bw, %r_c, 0");
     }
     P.op("mov.u32 %r_c, %ctaid.x");
     P.op("cvt.u64.u32 %u, %r_c");
     P.op("mov.u32 %r_c, %nctaid.x");
     P.op("cvt.u64.u32 %grid, %r_c");
-    P.op("setp.ge.u64 %p_out, %u, %ntiles");
-    P.op("@%p_out bra $DONE");
-    emit_tbase(P, pd.S, n_local, "%u", "%tbo");
-    P.op("add.s64 %gtile, %psi, %tbo");
-    P.op("add.s64 %gcur, %gtile, %dthr");
     auto loadtile = [&](const std::string& g, const std::string& pred) {
         for (int i = 0; i < UPT; ++i) {
             const std::string sa = P.r32();
@@ -348,14 +384,91 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op(pred, "cp.async.cg.shared.global [", sa, "], ", ga, ", 16");
         }
     };
-    if (!zinit) loadtile("%gcur", "");
-    P.op("cp.async.commit_group");
+    const std::string gbar = ring ? "bar.sync %bid, " + std::to_string(nthr) : std::string("bar.sync 0");
+    if (ring) {
+        // mbarriers full[0..2] after the three buffers; initial loads: group 0
+        // tiles 0 and 2, group 1 tile 1 (tile k of this CTA -> buffer k mod 3)
+        P.op("add.u32 %mb0, %rsm0, ", 3 * tile_bytes);
+        P.op("setp.eq.u32 %p_z, %t_id, 0");
+        P.op("setp.eq.and.u32 %p_z, %grp, 0, %p_z");
+        for (int b = 0; b < 3; ++b) {
+            P.op("add.u32 %fb, %mb0, ", 8 * b);
+            P.op("@%p_z mbarrier.init.shared.b64 [%fb], ", nthr);
+        }
+        P.op("fence.mbarrier_init.release.cluster");
+        P.op("bar.sync 0");
+        if (!zinit)
+            for (int k0 = 0; k0 < 3; ++k0) {
+                const std::string q = P.pr();
+                P.op("add.s64 %un, %u, ", 0);
+                for (int t = 0; t < k0; ++t) P.op("add.s64 %un, %un, %grid");
+                P.op("setp.lt.u64 ", q, ", %un, %ntiles");
+                P.op("setp.eq.and.u32 ", q, ", %grp, ", k0 % 2, ", ", q);
+                P.op("@!", q, " bra $INIT", k0);
+                emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+                P.op("add.s64 %gnext, %psi, %tbo");
+                P.op("add.s64 %gnext, %gnext, %dthr");
+                P.op("add.u32 %cur, %rsm0, ", k0 * tile_bytes);
+                loadtile("%gnext", "");
+                P.op("add.u32 %fb, %mb0, ", 8 * k0);
+                P.op("cp.async.mbarrier.arrive.noinc.shared.b64 [%fb]");
+                P.o << "$INIT" << k0 << ":\n";
+            }
+        // this group's first tile: k = grp
+        P.op("cvt.u64.u32 %rdk, %grp");
+        P.op("mul.lo.u64 %rdk, %rdk, %grid");
+        P.op("add.s64 %u, %u, %rdk");
+        P.op("mov.u32 %kk, %grp");
+        P.op("mov.u32 %bb, %grp");
+        P.op("setp.ge.u64 %p_out, %u, %ntiles");
+        P.op("@%p_out bra $DONE");
+    } else {
+        P.op("setp.ge.u64 %p_out, %u, %ntiles");
+        P.op("@%p_out bra $DONE");
+        emit_tbase(P, pd.S, n_local, "%u", "%tbo");
+        P.op("add.s64 %gtile, %psi, %tbo");
+        P.op("add.s64 %gcur, %gtile, %dthr");
+        if (!zinit) loadtile("%gcur", "");
+        P.op("cp.async.commit_group");
+    }
     P.o << "$LOOP:\n";
-    P.op("add.s64 %un, %u, %grid");
-    P.op("setp.lt.u64 %p_next, %un, %ntiles");
-    emit_tbase(P, pd.S, n_local, "%un", "%tbo");
-    P.op("add.s64 %gtile_next, %psi, %tbo");
-    P.op("add.s64 %gnext, %gtile_next, %dthr");
+    if (ring) {
+        // this tile: buffer bb, full[bb]; the tile 3 ahead (other group) goes
+        // into the same buffer once this group is done reading it
+        P.op("mul.lo.u32 %r_c, %bb, ", tile_bytes);
+        P.op("add.u32 %cur, %rsm0, %r_c");
+        P.op("shl.b32 %r_c, %bb, 3");
+        P.op("add.u32 %fb, %mb0, %r_c");
+        emit_tbase(P, pd.S, n_local, "%u", "%tbo");
+        P.op("add.s64 %gtile, %psi, %tbo");
+        P.op("add.s64 %gcur, %gtile, %dthr");
+        P.op("add.s64 %un, %u, %grid");
+        P.op("add.s64 %un, %un, %grid");
+        P.op("add.s64 %un, %un, %grid");  // u + 3 grid
+        P.op("setp.lt.u64 %p_next, %un, %ntiles");
+        emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+        P.op("add.s64 %gtile_next, %psi, %tbo");
+        P.op("add.s64 %gnext, %gtile_next, %dthr");
+        // wait for this tile: load mode phase (k / 3) & 1; zinit: buffer free
+        // (released by tile k - 3) for k >= 3
+        P.op("div.u32 %r_c, %kk, 3");
+        if (zinit) {
+            P.op("setp.ge.u32 %p_w, %kk, 3");
+            P.op("@!%p_w bra $READY");
+            P.op("sub.u32 %r_c, %r_c, 1");
+        }
+        P.op("and.b32 %par, %r_c, 1");
+        P.o << "$WAIT:\n";
+        P.op("mbarrier.try_wait.parity.shared.b64 %p_w, [%fb], %par");
+        P.op("@!%p_w bra $WAIT");
+        P.o << "$READY:\n";
+    } else {
+        P.op("add.s64 %un, %u, %grid");
+        P.op("setp.lt.u64 %p_next, %un, %ntiles");
+        emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+        P.op("add.s64 %gtile_next, %psi, %tbo");
+        P.op("add.s64 %gnext, %gtile_next, %dthr");
+    }
     if (SVB_JIT_PF && !zinit) {
         // pull the next tile's runs into L2 now (one bulk prefetch per run,
         // spread over the threads), so the cp.async of the early load finds
@@ -380,8 +493,21 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("@", q, " cp.async.bulk.prefetch.L2.global [", a, "], ", rb);
         }
     }
-    P.op("cp.async.wait_group 0");
-    P.op("bar.sync 0");
+    if (!ring) {
+        P.op("cp.async.wait_group 0");
+        P.op("bar.sync 0");
+    }
+    // ring: release buffer bb (this group is done reading it): load the tile
+    // three ahead into it, or in zinit mode just mark it free
+    auto release = [&]() {
+        P.op(gbar);
+        if (zinit) {
+            P.op("mbarrier.arrive.shared.b64 %rdk, [%fb]");
+        } else {
+            loadtile("%gnext", "@%p_next ");
+            P.op("@%p_next cp.async.mbarrier.arrive.noinc.shared.b64 [%fb]");
+        }
+    };
     // ---- phases
     for (int ph = 0; ph < nph; ++ph) {
         const RpPhaseHost& Ph = phs[ph];
@@ -453,7 +579,9 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 P.op("ld.shared.b64 %a", j, ", [", a, "]");
             }
         }
-        if (last && early) {
+        if (ring && last && direct) {
+            release();
+        } else if (last && early) {
             // tile buffer free: the next tile's load overlaps this phase's gates
             P.op("bar.sync 0");
             loadtile("%gnext", "@%p_next ");
@@ -527,21 +655,22 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 for (int j = 0; j < NA / 2; ++j)
                     P.op("st.global.cs.v2.b64 ", gaddr(P, "%gst", 8 * tm.dep(deposit(2u * j, lp.R))), ", {%a", 2 * j, ", %a",
                          2 * j + 1, "}");
-                if (bins)
-                    for (int j = 0; j < NA / 2; ++j) {
-                        wadd("%a" + std::to_string(2 * j), true);
-                        wadd("%a" + std::to_string(2 * j + 1), false);
-                        wstore(3, gaddr_reg("%gst", 8 * tm.dep(deposit(2u * j, lp.R))));
-                    }
+
             } else {
                 for (int j = 0; j < NA; ++j)
                     P.op("st.global.cs.b64 ", gaddr(P, "%gst", 8 * tm.dep(deposit((uint32_t)j, lp.R))), ", %a", j);
-                if (bins)
-                    for (int j = 0; j < NA; ++j) {
-                        wadd("%a" + std::to_string(j), true);
-                        wstore(4, gaddr_reg("%gst", 8 * tm.dep(deposit((uint32_t)j, lp.R))));
-                    }
             }
+            if (bins)  // per bin slot: its registers, then the lanes holding bin bits
+                for (uint32_t j0 = 0; j0 < (uint32_t)NA; ++j0) {
+                    if (j0 & bin_regs) continue;
+                    bool first = true;
+                    for (uint32_t sub = 0; sub < (uint32_t)NA; ++sub)
+                        if ((sub & ~bin_regs) == 0) {
+                            wadd("%a" + std::to_string(j0 | sub), first);
+                            first = false;
+                        }
+                    wstore(bin_lanes, gaddr_reg("%gst", 8 * tm.dep(deposit(j0, lp.R))));
+                }
         } else {
             if (Ph.b0) {
                 for (int j = 0; j < NA / 2; ++j) {
@@ -554,7 +683,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                     P.op("st.shared.b64 [", a, "], %a", j);
                 }
             }
-            P.op("bar.sync 0");
+            P.op(gbar);
         }
     }
     if (!direct) {
@@ -567,7 +696,9 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("add.s32 ", sa, ", ", sa, ", %cur");
             P.op("ld.shared.v2.b64 {%a", 2 * i, ", %a", 2 * i + 1, "}, [", sa, "]");
         }
-        if (!zinit) {
+        if (ring) {
+            release();
+        } else if (!zinit) {
             P.op("bar.sync 0");  // every thread is done with the tile buffer
             loadtile("%gnext", "@%p_next ");
             P.op("cp.async.commit_group");
@@ -579,14 +710,27 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             for (int i = 0; i < UPT; ++i) {
                 wadd("%a" + std::to_string(2 * i), true);
                 wadd("%a" + std::to_string(2 * i + 1), false);
-                wstore(3, gaddr_reg("%gcur", 8 * tm.dep(2ull * nthr * i)));
+                wstore(bin_lanes, gaddr_reg("%gcur", 8 * tm.dep(2ull * nthr * i)));
             }
     }
-    P.op("mov.b64 %gcur, %gnext");
-    P.op("mov.b64 %gtile, %gtile_next");
-    P.op("mov.b64 %u, %un");
-    P.op("@%p_next bra $LOOP");
+    if (ring) {
+        // next tile of this group: k + 2 (buffer (bb + 2) mod 3)
+        P.op("add.s64 %u, %u, %grid");
+        P.op("add.s64 %u, %u, %grid");
+        P.op("add.u32 %kk, %kk, 2");
+        P.op("add.u32 %bb, %bb, 2");
+        P.op("setp.ge.u32 %p_w, %bb, 3");
+        P.op("@%p_w sub.u32 %bb, %bb, 3");
+        P.op("setp.lt.u64 %p_w, %u, %ntiles");
+        P.op("@%p_w bra $LOOP");
+    } else {
+        P.op("mov.b64 %gcur, %gnext");
+        P.op("mov.b64 %gtile, %gtile_next");
+        P.op("mov.b64 %u, %un");
+        P.op("@%p_next bra $LOOP");
+    }
     P.o << "$DONE:\n";
+    if (ring) P.op("bar.sync 0");  // both groups: every load either group issued has been consumed
     P.op("ret");
 
     std::ostringstream k;
@@ -594,12 +738,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << "// T=" << T << " r=" << pd.r << " n=" << n_local << " S={";
     for (int q : pd.S) k << q << ",";
     k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (pinit ? " product-start" : "")
-      << (direct ? " direct" : "") << (bins ? " bins" : "") << "\n";
+      << (direct ? " direct" : "") << (bins ? " bins" : "") << (ring ? " ring" : "") << "\n";
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
-    k << ".maxntid " << nthr << ", 1, 1\n.maxnreg 128\n{\n";
-    k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw;\n";
+    k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg 128\n{\n";
+    k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw, %p_w;\n";
+    k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par;\n\t.reg .b64 %rdk;\n";
     k << "\t.reg .f64 %dre, %dim, %dp;\n\t.reg .b64 %w, %wt, %bo, %bins;\n\t.reg .b32 %wl, %wh, %wl2, %wh2;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
@@ -1056,8 +1201,10 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
             if (fresh) {
                 l.kern->src = pd.wide ? gen_chunk64(pd, n_local, ch.first, ch.second, z, nm, l.mats64)
                                       : gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
-                l.kern->nthr = 1 << (T - M);
-                l.kern->smem = (size_t)(pd.wide ? 16 : 8) << T;
+                const bool ring = SVB_JIT_RING && !pd.wide;
+                l.kern->nthr = (1 << (T - M)) * (ring ? 2 : 1);
+                l.kern->smem = ((size_t)(pd.wide ? 16 : 8) << T) * (ring ? 3 : 1) + (ring ? 64 : 0);
+                l.kern->T = T;
                 l.kern->nm = nm;
                 l.kern->param_bytes = std::max<size_t>(nm, 1) * 16 + 48;  // as in gen_chunk
                 todo.push_back(l.kern);
@@ -1128,7 +1275,7 @@ cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool 
             }
         }
     }
-    const int T = __builtin_ctz((unsigned)(K.smem / (l.wide ? 16 : 8)));
+    const int T = K.T;
     const uint64_t n_tiles = 1ull << (n_local - T);
     const uint64_t grid = std::min<uint64_t>(n_tiles, (uint64_t)pass_sms() * K.blocks_per_sm);
     std::vector<unsigned char> prm(K.param_bytes, 0);

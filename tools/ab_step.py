@@ -1,3 +1,6 @@
+"""Interleaved A/B of the bench step (reset + circuit + 10^6 samples; host wall time, mean of 10)
+across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3] python tools/ab_step.py <rounds> <lib.so> ...
+"""
 import json, os, subprocess, sys
 CHILD = r'''
 import sys, time, json
@@ -5,7 +8,11 @@ sys.path.insert(0, "/root/repo")
 import torch
 import paper_conf_sc_markidis23_b200 as sv
 from workloads import rqc as W
-n=30; h=sv.sv_create(n); c=sv.sv_circuit_create(h, W.rqc(n,14), 1)
+import os
+n=int(os.environ.get("AB_N", "30")); d=int(os.environ.get("AB_D", "14"))
+h=sv.sv_create(n)
+if os.environ.get("AB_PIN"): sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, int(os.environ["AB_PIN"]))
+c=sv.sv_circuit_create(h, W.rqc(n,d), 1)
 out=torch.empty(1000000, dtype=torch.int64, device="cuda")
 def step():
     sv.sv_reset(h); sv.sv_circuit_run_device(h,c); sv.sv_sample_device(h,1,1000000,out.data_ptr())
