@@ -672,7 +672,8 @@ def run_ours(args):
             "fusion_sweep_s": sweep,
             "pass_pin_sweep_s": pin_sweep,
             "optimal_fusion": (None if not sweep else
-                               {"max_fused": int(min(sweep, key=sweep.get)), "value": min(sweep.values()), "unit": "s"}),
+                               {"max_fused": args.max_fused, "pass_pin": pass_pin,
+                                "value": min(list(sweep.values()) + list((pin_sweep or {}).values())), "unit": "s"}),
             "clocks": clk.summary(),
         }
         if world > 1:

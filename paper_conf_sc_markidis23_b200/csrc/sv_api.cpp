@@ -24,6 +24,9 @@
 
 using namespace svb;
 
+#ifndef SVB_PASS_LOOKAHEAD
+#define SVB_PASS_LOOKAHEAD 1  // pass qubit sets chosen by lookahead (0: first-come greedy)
+#endif
 #ifndef SVB_FUSED_BINS
 #define SVB_FUSED_BINS 1  // the last register-blocked pass writes the sampler's bin weights
 #endif
@@ -643,20 +646,77 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
         std::vector<size_t> mem{i};
         placed[i] = 1;
         uint64_t Q = fm[i], B = 0;
-        size_t planes = 3ull << (2 * in[i].k);
-        for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
-            if (placed[j]) continue;
-            const uint64_t Sj = fm[j];
-            const size_t pj = 3ull << (2 * in[j].k);
-            if (Sj & B) {
-                B |= Sj;
-            } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
-                Q |= Sj;
-                planes += pj;
-                mem.push_back(j);
-                placed[j] = 1;
-            } else {
-                B |= Sj;
+        if (SVB_PASS_LOOKAHEAD) {
+            // choose the pass's free qubits by lookahead (reading R7): the
+            // gates a qubit set Q absorbs are fixed (every later unplaced gate
+            // inside Q | pinned that touches no qubit of an earlier gate left
+            // out); grow Q, starting from gate i's qubits, by the qubit set of
+            // a left-out gate that absorbs the most gates, until nothing helps
+            placed[i] = 0;
+            auto absorb = [&](uint64_t Qc, std::vector<size_t>* out) {
+                uint64_t Bl = 0;
+                size_t cnt = 0, planes = 0;
+                for (size_t j = i; j < nf; ++j) {
+                    if (placed[j]) continue;
+                    const uint64_t Sj = fm[j];
+                    const size_t pj = 3ull << (2 * in[j].k);
+                    if (!(Sj & Bl) && !(Sj & ~(Qc | pin)) && cnt < (size_t)kPassMaxGates &&
+                        planes + pj <= (size_t)kPassPlaneFloats) {
+                        ++cnt;
+                        planes += pj;
+                        if (out) out->push_back(j);
+                    } else {
+                        Bl |= Sj;
+                    }
+                }
+                return cnt;
+            };
+            Q = fm[i] & ~pin;
+            for (;;) {
+                std::vector<size_t> cur;
+                const size_t have = absorb(Q, &cur);
+                std::vector<char> in_cur(nf, 0);
+                for (size_t j : cur) in_cur[j] = 1;
+                std::vector<uint64_t> cands;
+                for (size_t j = i; j < nf && cands.size() < 40; ++j) {
+                    if (placed[j] || in_cur[j]) continue;
+                    const uint64_t add = fm[j] & ~pin & ~Q;
+                    if (!add || __builtin_popcountll(Q | add) > Fp) continue;
+                    if (std::find(cands.begin(), cands.end(), add) == cands.end()) cands.push_back(add);
+                }
+                uint64_t best = 0;
+                size_t bestc = have;
+                for (uint64_t add : cands) {
+                    const size_t c = absorb(Q | add, nullptr);
+                    if (c > bestc || (best && c == bestc && __builtin_popcountll(add) < __builtin_popcountll(best))) {
+                        best = add;
+                        bestc = c;
+                    }
+                }
+                if (!best) break;
+                Q |= best;
+            }
+            mem.clear();
+            absorb(Q, &mem);
+            for (size_t j : mem) placed[j] = 1;
+            Q = 0;
+            for (size_t j : mem) Q |= fm[j];
+        } else {
+            size_t planes = 3ull << (2 * in[i].k);
+            for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
+                if (placed[j]) continue;
+                const uint64_t Sj = fm[j];
+                const size_t pj = 3ull << (2 * in[j].k);
+                if (Sj & B) {
+                    B |= Sj;
+                } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
+                    Q |= Sj;
+                    planes += pj;
+                    mem.push_back(j);
+                    placed[j] = 1;
+                } else {
+                    B |= Sj;
+                }
             }
         }
         uint64_t tile = Q | pin;
