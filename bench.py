@@ -532,6 +532,7 @@ def run_ours(args):
         clk.mark(t_host0, time.time())
         time.sleep(0.15)  # let the sampler deliver the sample that covers the end of the region
     sv.sv_set_timing(h, False)
+    pass_bytes, pass_fma = sv.sv_last_pass_costs(h)  # per pass of the last timed step
     ms = start.elapsed_time(end) / args.steps
     per_step = [a.elapsed_time(b) for a, b in evs]
     t_high, t_low, t_exch = acc["t_apply_high_dev_s"], acc["t_apply_low_dev_s"], acc["t_exchange_dev_s"]
@@ -604,6 +605,16 @@ def run_ours(args):
         exch_bytes = acc["bytes_exchange"] / steps
         fma = acc["fma_apply"]
         smax = clk.summary().get("sm_max_mhz") or 1965
+        # FP32 ALU peak: 148 SMs x 128 FP32 lanes x 2 flop x max SM clock; the pass kernels'
+        # fp32 work is FMAs (FFMA2 = 2 FMAs at half the issue rate)
+        alu_peak_tflops = 148 * 128 * 2 * smax * 1e6 / 1e12
+        alu_ach = 2 * fma / t_apply / 1e12 if fma and t_apply else None
+        alu_frac = alu_ach / alu_peak_tflops if alu_ach else None
+        # per-pass roofline floor: every pass bound by max(HBM bytes / HBM peak, FMAs / FMA peak)
+        floor = sum(max(float(b) / (peak * 1e9), float(f) / (alu_peak_tflops * 1e12 / 2))
+                    for b, f in zip(pass_bytes, pass_fma))
+        apply_step = t_apply / steps
+        alu_bound = alu_frac is not None and frac is not None and alu_frac > frac
         out = {
             "metric": f"{args.workload}_circuit_time_{n}q_d{depth}" + ("_c128" if fp64 else ""),
             "value": ms / 1e3,
@@ -649,22 +660,26 @@ def run_ours(args):
                 "apply_launches_per_step": launches_apply // steps,
                 "block_bits": args.block_bits,
             },
-            "roofline": {"bound": "hbm",
+            "roofline": {"bound": "alu" if alu_bound else "hbm",
                          "kernel": ("rpj (pass-specialised register-blocked pass: all gates of a pass per HBM "
                                     "read + write)" if cst["n_passes"] else "apply_high+apply_low (one launch per fused gate)"),
-                         "achieved": achieved, "peak": peak,
-                         "peak_source": peak_src, "unit": "GB/s", "frac": frac,
-                         "frac_of_8tbs": achieved / 8000.0 if achieved else None,
+                         "achieved": alu_ach if alu_bound else achieved,
+                         "peak": alu_peak_tflops if alu_bound else peak,
+                         "peak_source": ("148 SMs x 128 FP32 lanes x 2 flop x max SM clock (FMA pipe)" if alu_bound
+                                         else peak_src),
+                         "unit": "TFLOP/s" if alu_bound else "GB/s",
+                         "frac": alu_frac if alu_bound else frac,
+                         "hbm": {"achieved": achieved, "peak": peak, "unit": "GB/s", "frac": frac,
+                                 "frac_of_8tbs": achieved / 8000.0 if achieved else None},
+                         "alu": {"achieved": alu_ach, "peak": alu_peak_tflops, "unit": "TFLOP/s", "frac": alu_frac},
+                         "pass_floor": ({"passes": len(pass_bytes), "floor_ms": floor * 1e3,
+                                         "apply_ms": apply_step * 1e3,
+                                         "frac": floor / apply_step if apply_step else None,
+                                         "rule": "sum over passes of max(HBM bytes / HBM peak, FMAs / FMA peak)"}
+                                        if len(pass_bytes) else None),
                          "algorithmic_bytes_per_launch": bytes_per_launch,
                          "algorithmic_bytes_per_step": acc["bytes_apply"] // steps,
-                         "traffic": load_traffic("rpass" if cst["n_passes"] else "apply"),
-                         # the blocked passes are bound by HBM and the FP32 pipe
-                         # together: the FMA-pipe share of the same launches
-                         # (fp32 FMAs executed / (148 SMs x 128 FMA/clk x max clock))
-                         "fma_pipe": ({"achieved_tfma_s": fma / t_apply / 1e12,
-                                       "peak_tfma_s": 148 * 128 * smax * 1e6 / 1e12,
-                                       "frac": fma / t_apply / (148 * 128 * smax * 1e6)}
-                                      if fma and t_apply else None)},
+                         "traffic": load_traffic("rpass" if cst["n_passes"] else "apply")},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_ms / 1e3, "unit": "s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": 8 * args.samples},

@@ -277,6 +277,12 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each);
 int sv_set_blocking(sv_state* s, int tile_bits);
 /* 1: record CUDA events around every launch and fill the *_dev_s stats. */
 int sv_set_timing(sv_state* s, int enable);
+/* Per register-blocked pass of the most recent circuit run (per shard): the
+ * algorithmic HBM bytes (16 B per amplitude; 8 B for a first pass that builds
+ * its tiles) and the fp32 FMAs it executed -- the inputs of a per-pass
+ * roofline floor max(bytes / HBM peak, FMAs / FMA peak).  *need = passes;
+ * cap < *need -> SV_EINVAL. */
+int sv_last_pass_costs(const sv_state* s, uint64_t* bytes, uint64_t* fmas, size_t cap, size_t* need);
 /* Stats of the most recent run on this handle. */
 int sv_last_stats(const sv_state* s, sv_stats* out);
 /* Synchronise the handle's stream.  Returns SV_EINVAL (once) if an earlier

@@ -147,6 +147,7 @@ _SIGS = {
                         ctypes.c_int),
     "sv_jit_stats": ([_u64p, _u64p, ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
     "sv_last_stats": ([_vp, ctypes.POINTER(sv_stats)], ctypes.c_int),
+    "sv_last_pass_costs": ([_vp, _u64p, _u64p, _sz, ctypes.POINTER(_sz)], ctypes.c_int),
     "sv_synchronize": ([_vp], ctypes.c_int),
     "sv_last_error": ([], ctypes.c_char_p),
     "sv_version": ([], ctypes.c_char_p),
@@ -478,6 +479,17 @@ def sv_last_stats(h: int) -> dict:
     st = sv_stats()
     _check(lib().sv_last_stats(h, ctypes.byref(st)), "sv_last_stats")
     return st.as_dict()
+
+
+def sv_last_pass_costs(h: int):
+    """(bytes, fmas) per register-blocked pass of the last circuit run."""
+    need = _sz()
+    lib().sv_last_pass_costs(h, None, None, 0, ctypes.byref(need))
+    b = np.zeros(max(need.value, 1), dtype=np.uint64)
+    f = np.zeros(max(need.value, 1), dtype=np.uint64)
+    _check(lib().sv_last_pass_costs(h, b.ctypes.data_as(_u64p), f.ctypes.data_as(_u64p), b.size, ctypes.byref(need)),
+           "sv_last_pass_costs")
+    return b[: need.value], f[: need.value]
 
 
 def sv_synchronize(h: int) -> None:

@@ -139,6 +139,7 @@ struct sv_state {
     };
     std::vector<Rec> recs;
     std::vector<cudaEvent_t> ev_pool;
+    std::vector<uint64_t> pass_bytes, pass_fma;  // per blocked pass of the last run (per shard)
     size_t ev_used = 0;
     sv_stats stats{};
     // reusable device buffers
@@ -1603,6 +1604,8 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     if (s->pos != c->pos_in) return fail(SV_EINVAL, "state qubit map differs from the circuit's (sv_reset first)");
     Nvtx nv("sv.circuit_run");
     s->bins_valid = false;
+    s->pass_bytes.clear();
+    s->pass_fma.clear();
     const sv_stats keep = c->stats;
     reset_stats(s);
     s->stats.t_fuse_s = keep.t_fuse_s;
@@ -1683,6 +1686,8 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
             if (!(zinit && &st == &steps[0] ? st.jitz : st.jit).empty()) s->stats.n_jit_passes += 1;
             for (auto& g : st.pass.gates) s->stats.flops_apply += (uint64_t)((8 << g.k) - 2) << s->l;
             s->stats.fma_apply += st.pass.fma_per_amp << s->l;
+            s->pass_bytes.push_back(pass_bytes);
+            s->pass_fma.push_back(st.pass.fma_per_amp << s->l);
             s->stats.n_passes += 1;
             s->stats.block_bits = (int)st.pass.S.size();
             continue;
@@ -2224,6 +2229,18 @@ int sv_jit_stats(uint64_t* compiled, uint64_t* cache_hits, double* compile_secon
 int sv_set_timing(sv_state* s, int enable) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
     s->timing = enable != 0;
+    return SV_OK;
+}
+
+int sv_last_pass_costs(const sv_state* s, uint64_t* bytes, uint64_t* fmas, size_t cap, size_t* need) {
+    if (!s || !need) return fail(SV_EINVAL, "NULL argument");
+    *need = s->pass_bytes.size();
+    if (cap < *need) return fail(SV_EINVAL, "cap too small");
+    if (*need && (!bytes || !fmas)) return fail(SV_EINVAL, "bytes/fmas is NULL");
+    for (size_t i = 0; i < *need; ++i) {
+        bytes[i] = s->pass_bytes[i];
+        fmas[i] = s->pass_fma[i];
+    }
     return SV_OK;
 }
 
