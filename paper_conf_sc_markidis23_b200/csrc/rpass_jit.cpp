@@ -35,6 +35,9 @@
 #ifndef SVB_JIT_SECTOR_DIRECT
 #define SVB_JIT_SECTOR_DIRECT 1  // direct stores also for 32 B-sector layouts of the last phase
 #endif
+#ifndef SVB_JIT_M
+#define SVB_JIT_M 5  // log2 amplitudes per thread of the complex64 pass kernels (4: 16 per thread, 64 registers)
+#endif
 #ifndef SVB_JIT_RING
 #define SVB_JIT_RING 0  // two warp groups over three tile buffers per CTA (loads 1.5 tiles ahead)
 #endif
@@ -182,7 +185,7 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
 std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
                       std::vector<float>& mats, bool emit = true, const std::vector<float>* msrc = nullptr) {
     const std::vector<float>& pmats = msrc ? *msrc : pd.mats;
-    constexpr int M = 5, NA = 32, UPT = 16;
+    constexpr int M = SVB_JIT_M, NA = 1 << M, UPT = 1 << (M - 1);
     const int T = (int)pd.S.size();
     const int tbits = T - M;
     const uint32_t nthr = 1u << tbits;
@@ -251,7 +254,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         };
         const RpPhaseHost& P0 = phs[0];
         reg0 = mats.size() / 4;
-        for (uint32_t j = 0; j < 32; ++j) {
+        for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
             std::complex<double> z = 1.0;
             for (int b = 0; b < M; ++b) z *= pd.pinit_v[2 * P0.R[b] + ((j >> b) & 1u)];
             put(z);
@@ -607,7 +610,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                     P.op("setp.eq.u32 ", pred, ", ", t, ", ", tmask);
                     pred = "@" + pred + " ";
                 }
-                for (uint32_t j = 0; j < 32; ++j)
+                for (uint32_t j = 0; j < (uint32_t)NA; ++j)
                     if ((j & mask) == mask) P.op(pred, "xor.b64 %a", j, ", %a", j, ", -9223372034707292160");
                 continue;
             }
@@ -622,7 +625,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             if (kind == 1) {
                 for (int e = 0; e < D; ++e) {
                     mload(base + e);
-                    for (uint32_t j = 0; j < 32; ++j) {
+                    for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
                         if (pext(j, mask) != (uint32_t)e) continue;
                         swp("%a" + std::to_string(j), "%xs0");
                         P.op("fma.rn.f32x2 %y, %ml, %a", j, ", %zero");
@@ -631,8 +634,8 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 }
                 continue;
             }
-            const uint32_t rest = 31u & ~mask;
-            for (uint32_t gi = 0; gi < 32u / D; ++gi) {
+            const uint32_t rest = ((1u << M) - 1u) & ~mask;
+            for (uint32_t gi = 0; gi < (uint32_t)NA / D; ++gi) {
                 const uint32_t b0 = pdep(gi, rest);
                 for (int c = 0; c < D; ++c) {
                     P.op("mov.b64 %x", c, ", %a", b0 | pdep(c, mask));
@@ -742,7 +745,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
-    k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg 128\n{\n";
+    k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg " << (M == 5 ? 128 : 64) << "\n{\n";
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw, %p_w;\n";
     k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par;\n\t.reg .b64 %rdk;\n";
     k << "\t.reg .f64 %dre, %dim, %dp;\n\t.reg .b64 %w, %wt, %bo, %bins;\n\t.reg .b32 %wl, %wh, %wl2, %wh2;\n";
@@ -1149,7 +1152,7 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
         out.clear();
         const int T = (int)pd.S.size();
         bool first = true;
-        for (const auto& ch : rpass_chunks(pd, 5)) {
+        for (const auto& ch : rpass_chunks(pd, pd.wide ? 4 : SVB_JIT_M, pd.wide)) {
             RpJitLaunch l;
             size_t nm = 0;
             const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats);
@@ -1181,7 +1184,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     for (size_t i = 0; i < pds.size(); ++i) {
         const PassDesc& pd = *pds[i];
         const int T = (int)pd.S.size();
-        const int M = pd.wide ? 4 : 5;
+        const int M = pd.wide ? 4 : SVB_JIT_M;
         bool first = true;
         for (const auto& ch : rpass_chunks(pd, M, pd.wide)) {
             RpJitLaunch l;
