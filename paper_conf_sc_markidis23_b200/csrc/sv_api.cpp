@@ -174,6 +174,7 @@ struct sv_circuit {
     // first pass (PassDesc::pinit_v); empty when not applicable
     std::vector<Step> steps_z;
     sv_stats stats_z{};
+    bool zero_only = false;  // only steps_z was built (a one-shot run from the pending |0...0>)
     void* ptab = nullptr;  // its tile-factor tables (device, complex64 / complex128)
     float2* dev_mats = nullptr;
     double* planes64 = nullptr;  // complex128 states: planes of every gate
@@ -1242,7 +1243,15 @@ static int shard_plan_impl(const int32_t* fs, size_t len, const uint64_t* diag, 
     return SV_OK;
 }
 
+static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out,
+                               bool zero_only);
+
 int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out) {
+    return circuit_create_impl(s, gates, n_gates, max_fused, out, false);
+}
+
+static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_circuit** out,
+                               bool zero_only) {
     int rc = check_state(s);
     if (rc) return rc;
     if (!out) return fail(SV_EINVAL, "out is NULL");
@@ -1411,7 +1420,6 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
         }
         c->steps.push_back(std::move(st));
     }
-    flush_passes();
     // product-state start (unsharded, pass-specialised kernels): the first
     // gate of each qubit, if it is a one-qubit gate, commutes with every gate
     // before it, so a run from |0...0> may apply all of them first -- i.e.
@@ -1457,6 +1465,15 @@ int sv_circuit_create(sv_state* s, const sv_gate* gates, size_t n_gates, int max
             }
         }
     }
+    // a circuit created for one run from the pending |0...0> (sv_run_circuit)
+    // needs only the product-state steps: skip planning the others
+    if (zero_only && !c->steps_z.empty()) {
+        run.clear();
+        c->zero_only = true;
+        c->stats.n_passes = c->stats_z.n_passes;
+        c->stats.fma_apply = c->stats_z.fma_apply;
+    }
+    flush_passes();
     // the last pass of an unsharded complex64 circuit also writes the
     // sampler's bin weights (sv_sample then skips its read of the state)
     if (SVB_FUSED_BINS && blocked && s->pass_jit && s->g == 0 && !s->fp64)
@@ -1602,6 +1619,7 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
     if (rc) return rc;
     if (!c || c->owner != s) return fail(SV_EINVAL, "circuit is NULL or belongs to another state");
     if (s->pos != c->pos_in) return fail(SV_EINVAL, "state qubit map differs from the circuit's (sv_reset first)");
+    if (c->zero_only && !s->zero_pending) return fail(SV_EINVAL, "circuit was built for a run from |0...0> only");
     Nvtx nv("sv.circuit_run");
     s->bins_valid = false;
     s->pass_bytes.clear();
@@ -1738,7 +1756,9 @@ int sv_circuit_destroy(sv_circuit* c) {
 int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fused, sv_stats* stats) {
     const double t0 = now_s();
     sv_circuit* c = nullptr;
-    int rc = sv_circuit_create(s, gates, n_gates, max_fused, &c);
+    int rc = check_state(s);
+    if (rc) return rc;
+    rc = circuit_create_impl(s, gates, n_gates, max_fused, &c, s->zero_pending);
     if (rc) return rc;
     rc = sv_circuit_run_device(s, c);
     if (rc == SV_OK) rc = sync(s);
