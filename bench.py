@@ -607,7 +607,7 @@ def run_ours(args):
         smax = clk.summary().get("sm_max_mhz") or 1965
         # FP32 ALU peak: 148 SMs x 128 FP32 lanes x 2 flop x max SM clock; the pass kernels'
         # fp32 work is FMAs (FFMA2 = 2 FMAs at half the issue rate)
-        alu_peak_tflops = 148 * 128 * 2 * smax * 1e6 / 1e12
+        alu_peak_tflops = 148 * 128 * 2 * smax * 1e6 / 1e12 / (2 if fp64 else 1)  # fp64 FMA at half rate
         alu_ach = 2 * fma / t_apply / 1e12 if fma and t_apply else None
         alu_frac = alu_ach / alu_peak_tflops if alu_ach else None
         # per-pass roofline floor: every pass bound by max(HBM bytes / HBM peak, FMAs / FMA peak)
@@ -665,7 +665,8 @@ def run_ours(args):
                                     "read + write)" if cst["n_passes"] else "apply_high+apply_low (one launch per fused gate)"),
                          "achieved": alu_ach if alu_bound else achieved,
                          "peak": alu_peak_tflops if alu_bound else peak,
-                         "peak_source": ("148 SMs x 128 FP32 lanes x 2 flop x max SM clock (FMA pipe)" if alu_bound
+                         "peak_source": ("148 SMs x 128 FP32 lanes x 2 flop x max SM clock (FMA pipe; fp64: half)"
+                                         if alu_bound
                                          else peak_src),
                          "unit": "TFLOP/s" if alu_bound else "GB/s",
                          "frac": alu_frac if alu_bound else frac,
