@@ -295,7 +295,7 @@ int sv_synchronize(sv_state* s);
  *                      specialised to each pass (PTX for sm_100a, compiled in
  *                      sv_circuit_create and cached per process); 0: the
  *                      generic apply_rpass kernel.  Both give bit-identical
- *                      states;
+ *                      states when SV_OPT_PASS_SPEC is 0;
  *   SV_OPT_APPLY_PATH  dense fused gates of one launch each:
  *                      SV_PATH_AUTO (default: k = 5, 6 on the exact int8
  *                      tensor-core path, k <= 4 SIMT), SV_PATH_SIMT,
@@ -308,7 +308,14 @@ int sv_synchronize(sv_state* s);
  *                      depends on the circuit (30q D14: 3, 32q D20: 4);
  *   SV_OPT_DIAG_SKIP   1 (default): sharded circuits (sv_circuit_create) do
  *                      not exchange a global qubit for a fused gate that is
- *                      block-diagonal in it (sv_shard_plan_diag); 0: plain S4.
+ *                      block-diagonal in it (sv_shard_plan_diag); 0: plain S4;
+ *   SV_OPT_PASS_SPEC   1 (default): the pass-specialised kernels apply
+ *                      structured one-qubit gates (rows or columns multiples
+ *                      of (1, i^p), diagonals; H, sqrt(X), sqrt(Y), T and
+ *                      their products) as fp32 additions with the gates'
+ *                      scalar factors multiplied in once per pass (DESIGN.md
+ *                      R11): same result up to fp32 rounding order, fewer
+ *                      operations; 0: every gate as a dense complex matrix.
  * Takes effect for circuits created / gates applied afterwards.  SV_EINVAL
  * for unknown options or values. */
 #define SV_OPT_BLOCK_BITS 1
@@ -317,6 +324,7 @@ int sv_synchronize(sv_state* s);
 #define SV_OPT_TIMING 4
 #define SV_OPT_DIAG_SKIP 5  /* 1 (default): sharded circuits plan with the diagonal exchange skip */
 #define SV_OPT_PASS_PIN 6   /* qubits 0..v-1 in every blocked-pass tile (runs of 8*2^v bytes): 3, 4 (default), 5 */
+#define SV_OPT_PASS_SPEC 7  /* 1 (default): structured one-qubit gates as additions in the pass kernels */
 #define SV_PATH_AUTO 0
 #define SV_PATH_SIMT 1
 #define SV_PATH_INT8 2

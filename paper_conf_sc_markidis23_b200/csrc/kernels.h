@@ -105,6 +105,11 @@ struct PassDesc {
     std::vector<double> mats64;  // complex128 states: the matrices in fp64 (same layout as mats)
     bool wide = false;           // complex128 state: pass-specialised fp64 kernel, 16 amplitudes per thread
     bool bins = false;           // last pass of an unsharded complex64 circuit: also write the sampler's bins
+    // structured one-qubit gates (pass-specialised complex64 kernels, reading
+    // R11): a one-qubit gate c * B with B's rows (or columns) of the form
+    // (1, i^p) runs as additions; the scalars c of the pass are multiplied
+    // out once per pass.  Only when every shard runs `mats` (no mats_shard).
+    bool spec = false;
 };
 void plan_pass_tile(PassDesc& pd);
 cudaError_t launch_pass(float2* psi, int n_local, const PassDesc& pd, cudaStream_t st);
@@ -183,6 +188,11 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
 // the 16-amplitude S5 bin weights of the final state there)
 cudaError_t launch_rpass_jit(void* psi, int n_local, const RpJitLaunch& l, bool one_here, cudaStream_t st,
                              int slot = 0, uint64_t* bins = nullptr);
+// fp32 pipe operations per amplitude of the pass-specialised kernels of this
+// pass (zinit: the |0...0>-start variant): as rpass_fma_per_amp for generic
+// gates, fewer for the structured gates of PassDesc::spec (one FADD, FMUL or
+// FFMA = 1)
+uint64_t rpass_jit_ops_per_amp(const PassDesc& pd, bool zinit);
 // process-wide counters (sv_jit_stats)
 void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compile_s);
 

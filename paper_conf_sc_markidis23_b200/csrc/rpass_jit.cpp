@@ -102,6 +102,130 @@ struct TileMap {
     }
 };
 
+// ---------------------------------------------------------------------------
+// Structured one-qubit gates (reading R11).  A one-qubit matrix U
+// whose rows are multiples of (1, i^p) -- U = diag(u00, u10) [[1, i^p0],
+// [1, i^p1]], the "row form" of H, sqrt(X), sqrt(Y), T sqrt(X), T sqrt(Y) --
+// or whose columns are multiples of (1, i^k) -- U = [[1, 1], [i^k0, i^k1]]
+// diag(u00, u01), the "column form" of H T -- or a diagonal one, runs as c B
+// with c = u00 taken out: B's products with 1 and i^p are sign and re/im
+// choices in fp32 additions (2 FADDs per output amplitude where a dense 2 x 2
+// takes 8 FMAs), its other factors complex multiplies (4 operations).  The
+// product C of the c's of a pass is multiplied in once by the pass's first
+// chunk: into the start state (|0...0> start), a generic gate's matrix, the
+// multipliers of a row-form gate, or explicitly.  Exact in real arithmetic;
+// in fp32 only the rounding differs from the dense product.
+using cd = std::complex<double>;
+struct GSpec {
+    int cls = 0;                  // 0 generic, 1 row form, 2 column form, 3 one-qubit diagonal
+    int p[2] = {0, 0};            // row: out_r = s_r (a0 + i^p[r] a1); column: out1 = i^p[0] a0 + i^p[1] mu a1
+    int q[2] = {0, 0};            // s_r = i^q[r] when unit[r]
+    bool unit[2] = {true, true};  // diagonal: s_r multiplies the amplitudes with the gate bit = r
+    cd s[2] = {1.0, 1.0};         // the non-unit s_r
+    cd mu = 1.0;                  // column form: out0 = a0 + mu a1
+    cd c = 1.0;                   // the scalar taken out
+};
+cd ipow(int q) {
+    static const cd u[4] = {cd(1, 0), cd(0, 1), cd(-1, 0), cd(0, -1)};
+    return u[q & 3];
+}
+bool unit_exp(cd z, int& e) {
+    static const cd u[4] = {cd(1, 0), cd(0, 1), cd(-1, 0), cd(0, -1)};
+    for (int k = 0; k < 4; ++k)
+        if (std::abs(z - u[k]) <= 1e-9) {
+            e = k;
+            return true;
+        }
+    return false;
+}
+GSpec classify(const PassDesc& pd, const PassGate& pg) {
+    GSpec g;
+    if (!pd.spec || pd.wide || pg.k != 1 || pd.mats64.size() < pg.moff + 8) return g;
+    const int kind = gate_kind(pd, pg);
+    const double* m = pd.mats64.data() + pg.moff;
+    const cd u00(m[0], m[1]), u01(m[2], m[3]), u10(m[4], m[5]), u11(m[6], m[7]);
+    const double big = std::max(std::max(std::abs(u00), std::abs(u01)), std::max(std::abs(u10), std::abs(u11)));
+    const double tiny = 1e-9 * big;
+    if (kind == 1) {
+        if (std::abs(u00) <= tiny) return g;
+        g.cls = 3;
+        g.c = u00;
+        if (!unit_exp(u11 / u00, g.q[1])) {
+            g.unit[1] = false;
+            g.s[1] = u11 / u00;
+        }
+        return g;
+    }
+    if (kind != 0) return g;
+    if (std::abs(u00) > tiny && std::abs(u10) > tiny && unit_exp(u01 / u00, g.p[0]) && unit_exp(u11 / u10, g.p[1])) {
+        g.cls = 1;
+        g.c = u00;
+        if (!unit_exp(u10 / u00, g.q[1])) {
+            g.unit[1] = false;
+            g.s[1] = u10 / u00;
+        }
+        return g;
+    }
+    GSpec h;
+    if (std::abs(u00) > tiny && std::abs(u01) > tiny && unit_exp(u10 / u00, h.p[0]) && unit_exp(u11 / u01, h.p[1])) {
+        h.cls = 2;
+        h.c = u00;
+        h.mu = u01 / u00;
+        return h;
+    }
+    return GSpec{};
+}
+// The gates of a pass classified, and how the launch chunk [g0, g1) applies
+// the pass scalar C (chunk 0 only): mode 1 start state, 2 folded into the
+// generic gate `fold`, 3 into the multipliers of the structured gate `fold`,
+// 4 explicit multiply after the chunk's last phase.
+struct ChunkSpec {
+    std::vector<GSpec> g;
+    cd C = 1.0;
+    int mode = 0;
+    int fold = -1;
+};
+ChunkSpec chunk_spec(const PassDesc& pd, size_t g0, size_t g1, bool zinit) {
+    ChunkSpec cs;
+    cs.g.resize(pd.gates.size());
+    if (!pd.spec || pd.wide) return cs;
+    bool any = false;
+    for (size_t i = 0; i < pd.gates.size(); ++i) {
+        cs.g[i] = classify(pd, pd.gates[i]);
+        cs.C *= cs.g[i].c;
+        any = any || cs.g[i].cls != 0;
+    }
+    if (g0 != 0 || !any) return cs;
+    if (zinit) {
+        cs.mode = 1;
+        return cs;
+    }
+    for (size_t i = g0; i < g1; ++i)
+        if (cs.g[i].cls == 0 && gate_kind(pd, pd.gates[i]) != 2) {
+            cs.mode = 2;
+            cs.fold = (int)i;
+            return cs;
+        }
+    // a row-form gate: +1 operation per amplitude when its row 1 already
+    // has a multiplier, +2 otherwise; a diagonal with one: +2
+    for (int pass = 0; pass < 3; ++pass)
+        for (size_t i = g0; i < g1; ++i) {
+            GSpec& x = cs.g[i];
+            const bool ok = pass == 0 ? x.cls == 1 && !x.unit[1] : pass == 1 ? x.cls == 1 : x.cls == 3 && !x.unit[1];
+            if (!ok) continue;
+            for (int r = 0; r < 2; ++r) {
+                if (x.unit[r]) x.s[r] = ipow(x.q[r]);
+                x.s[r] *= cs.C;
+                x.unit[r] = false;
+            }
+            cs.mode = 3;
+            cs.fold = (int)i;
+            return cs;
+        }
+    cs.mode = 4;
+    return cs;
+}
+
 // PTX text builder: amplitudes live in %a0..%a31 (one .b64 = packed
 // (re, im) complex64 each), rewritten in place; ptxas renames them.
 struct Ptx {
@@ -171,10 +295,20 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     put(pd.bins && g1 == pd.gates.size() ? 1 : 0);
     for (int q : pd.S) put(q);
     k += '|';
+    const ChunkSpec cs = chunk_spec(pd, g0, g1, zinit);
     for (size_t g = g0; g < g1; ++g) {
         const PassGate& pg = pd.gates[g];
         put(pg.k * 16 + gate_kind(pd, pg));
         for (int b = 0; b < pg.k; ++b) put(pg.pos[b]);
+        const GSpec& x = cs.g[g];
+        if (x.cls) k += 's';
+        if (x.cls) put(64 * x.cls + 16 * x.p[0] + 4 * x.p[1] + x.q[0] * 256 + x.q[1] * 1024 + (x.unit[0] ? 4096 : 0) +
+                       (x.unit[1] ? 8192 : 0));
+    }
+    if (cs.mode) {
+        k += 'm';
+        put(cs.mode);
+        put(cs.fold);
     }
     return k;
 }
@@ -222,25 +356,56 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     const uint32_t tile_bytes = 8u << T;
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
+    const ChunkSpec cs = chunk_spec(pd, g0, g1, zinit);
+    // structured-gate multiplier slot: (sr, si, -si, 0)
+    auto put_s = [&](cd z) {
+        mats.push_back((float)z.real());
+        mats.push_back((float)z.imag());
+        mats.push_back((float)-z.imag());
+        mats.push_back(0.f);
+    };
     std::vector<size_t> gbase(pd.gates.size(), 0);
     for (int ph = 0; ph < nph; ++ph)
         for (int g : phs[ph].gates) {
             const PassGate& pg = pd.gates[g];
             const int kind = gate_kind(pd, pg);
+            const GSpec& x = cs.g[g];
+            gbase[g] = mats.size() / 4;
+            if (x.cls == 2) {
+                put_s(x.mu);
+                continue;
+            }
+            if (x.cls) {
+                for (int r = 0; r < 2; ++r)
+                    if (!x.unit[r]) put_s(x.s[r]);
+                continue;
+            }
             if (kind == 2) continue;
             const int D = 1 << pg.k;
             const float* mg = pmats.data() + pg.moff;
-            gbase[g] = mats.size() / 4;
+            const cd f = cs.mode == 2 && g == cs.fold ? cs.C : cd(1.0);
             const int ne = kind == 1 ? D : D * D;
             for (int e = 0; e < ne; ++e) {
                 const int src = kind == 1 ? e * D + e : e;
-                const float mr = mg[2 * src], mi = mg[2 * src + 1];
+                float mr = mg[2 * src], mi = mg[2 * src + 1];
+                if (f != cd(1.0)) {
+                    const cd z = cd(mr, mi) * f;
+                    mr = (float)z.real();
+                    mi = (float)z.imag();
+                }
                 mats.push_back(mr);
                 mats.push_back(mr);
                 mats.push_back(-mi);
                 mats.push_back(mi);
             }
         }
+    // the pass scalar as the start amplitude (|0...0> start without the
+    // product state) or for the explicit multiply
+    size_t cslot = 0;
+    if ((cs.mode == 1 && pd.pinit_v.empty()) || cs.mode == 4) {
+        cslot = mats.size() / 4;
+        put_s(cs.C);
+    }
     // product-state start: register factors of phase 0 (32 slots) and the
     // two vectors of every lane position (2 slots per thread bit)
     const bool pinit = zinit && !pd.pinit_v.empty();
@@ -255,7 +420,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         const RpPhaseHost& P0 = phs[0];
         reg0 = mats.size() / 4;
         for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
-            std::complex<double> z = 1.0;
+            std::complex<double> z = cs.mode == 1 ? cs.C : cd(1.0);
             for (int b = 0; b < M; ++b) z *= pd.pinit_v[2 * P0.R[b] + ((j >> b) & 1u)];
             put(z);
         }
@@ -309,6 +474,98 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         const std::string t = P.r64();
         P.op("add.s64 ", t, ", ", base, ", ", off);
         return t;
+    };
+    // ---- structured gates (GSpec): fp32 scalar arithmetic on the halves of
+    // the packed amplitudes (%fe0..3 inputs, %fo0..3 outputs)
+    // d = eA A + eB B (eA, eB = +-1)
+    auto fsum = [&](const std::string& d, int eA, const std::string& A, int eB, const std::string& B) {
+        if (eA > 0 && eB > 0) P.op("add.rn.f32 ", d, ", ", A, ", ", B);
+        else if (eA > 0) P.op("sub.rn.f32 ", d, ", ", A, ", ", B);
+        else if (eB > 0) P.op("sub.rn.f32 ", d, ", ", B, ", ", A);
+        else {
+            P.op("neg.f32 %fn, ", A);
+            P.op("sub.rn.f32 ", d, ", %fn, ", B);
+        }
+    };
+    // (dr, di) = i^q (A + i^p B)
+    auto flin = [&](const std::string& dr, const std::string& di, int q, int p, const std::string& Ar,
+                    const std::string& Ai, const std::string& Br, const std::string& Bi) {
+        int er, ei;  // i^p B = (er * xr, ei * xi)
+        std::string xr, xi;
+        switch (p & 3) {
+            case 0: er = 1, xr = Br, ei = 1, xi = Bi; break;
+            case 1: er = -1, xr = Bi, ei = 1, xi = Br; break;
+            case 2: er = -1, xr = Br, ei = -1, xi = Bi; break;
+            default: er = 1, xr = Bi, ei = -1, xi = Br; break;
+        }
+        // t = A + i^p B; i^q t: q=0 (t.re, t.im), 1 (-t.im, t.re), 2 (-t.re, -t.im), 3 (t.im, -t.re)
+        auto part = [&](const std::string& d, int sg, bool im) {
+            fsum(d, sg, im ? Ai : Ar, sg * (im ? ei : er), im ? xi : xr);
+        };
+        switch (q & 3) {
+            case 0: part(dr, 1, false), part(di, 1, true); break;
+            case 1: part(dr, -1, true), part(di, 1, false); break;
+            case 2: part(dr, -1, false), part(di, -1, true); break;
+            default: part(dr, 1, true), part(di, -1, false); break;
+        }
+    };
+    // (dr, di) = s (xr, xi), s from slot (sr, si, -si, 0); d must not alias x
+    auto fmul = [&](const std::string& dr, const std::string& di, const std::string& xr, const std::string& xi,
+                    size_t slot) {
+        P.op("ld.param.v4.f32 {%fsr, %fsi, %fsn, %fsz}, [rpj_param_0+", 16 * slot, "]");
+        P.op("mul.rn.f32 %fu0, ", xi, ", %fsn");
+        P.op("mul.rn.f32 %fu1, ", xi, ", %fsr");
+        P.op("fma.rn.f32 ", dr, ", ", xr, ", %fsr, %fu0");
+        P.op("fma.rn.f32 ", di, ", ", xr, ", %fsi, %fu1");
+    };
+    auto emit_spec = [&](const GSpec& x, uint32_t mask, size_t base) {
+        size_t sl[2] = {base, base};
+        if (!x.unit[0]) sl[1] = base + 1;
+        if (x.cls == 3) {  // diagonal: s_r on the amplitudes whose gate bit is r
+            for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
+                const int r = (j & mask) ? 1 : 0;
+                const std::string a = "%a" + std::to_string(j);
+                if (!x.unit[r]) {
+                    P.op("mov.b64 {%fe0, %fe1}, ", a);
+                    fmul("%fo0", "%fo1", "%fe0", "%fe1", sl[r]);
+                    P.op("mov.b64 ", a, ", {%fo0, %fo1}");
+                } else if (x.q[r] == 2) {
+                    P.op("xor.b64 ", a, ", ", a, ", -9223372034707292160");
+                } else if (x.q[r] == 1) {  // (re, im) -> (-im, re)
+                    P.op("mov.b64 {%fe0, %fe1}, ", a);
+                    P.op("neg.f32 %fn, %fe1");
+                    P.op("mov.b64 ", a, ", {%fn, %fe0}");
+                } else if (x.q[r] == 3) {  // (im, -re)
+                    P.op("mov.b64 {%fe0, %fe1}, ", a);
+                    P.op("neg.f32 %fn, %fe0");
+                    P.op("mov.b64 ", a, ", {%fe1, %fn}");
+                }
+            }
+            return;
+        }
+        for (uint32_t j0 = 0; j0 < (uint32_t)NA; ++j0) {
+            if (j0 & mask) continue;
+            const uint32_t j1 = j0 | mask;
+            P.op("mov.b64 {%fe0, %fe1}, %a", j0);
+            P.op("mov.b64 {%fe2, %fe3}, %a", j1);
+            if (x.cls == 2) {  // out0 = a0 + mu a1, out1 = i^p0 (a0 + i^(p1-p0) mu a1)
+                fmul("%ft0", "%ft1", "%fe2", "%fe3", sl[0]);
+                flin("%fo0", "%fo1", 0, 0, "%fe0", "%fe1", "%ft0", "%ft1");
+                flin("%fo2", "%fo3", x.p[0], (x.p[1] - x.p[0]) & 3, "%fe0", "%fe1", "%ft0", "%ft1");
+            } else {  // row form: out_r = s_r (a0 + i^p_r a1)
+                for (int r = 0; r < 2; ++r) {
+                    const std::string dr = "%fo" + std::to_string(2 * r), di = "%fo" + std::to_string(2 * r + 1);
+                    if (x.unit[r]) {
+                        flin(dr, di, x.q[r], x.p[r], "%fe0", "%fe1", "%fe2", "%fe3");
+                    } else {
+                        flin("%ft0", "%ft1", 0, x.p[r], "%fe0", "%fe1", "%fe2", "%fe3");
+                        fmul(dr, di, "%ft0", "%ft1", sl[r]);
+                    }
+                }
+            }
+            P.op("mov.b64 %a", j0, ", {%fo0, %fo1}");
+            P.op("mov.b64 %a", j1, ", {%fo2, %fo3}");
+        }
     };
     // ---- prologue: thread constants
     P.op("mov.u32 %t_id, %tid.x");
@@ -570,7 +827,10 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("setp.ne.u32 %p_z, %zone, 0");
             P.op("setp.eq.and.u64 %p_z, %u, 0, %p_z");
             P.op("setp.eq.and.u32 %p_z, %t_id, 0, %p_z");
-            P.op("@%p_z mov.b64 %a0, 1065353216");  // (1.0f, 0.0f)
+            if (cs.mode == 1)  // (C re, C im)
+                P.op("@%p_z ld.param.b64 %a0, [rpj_param_0+", 16 * cslot, "]");
+            else
+                P.op("@%p_z mov.b64 %a0, 1065353216");  // (1.0f, 0.0f)
         } else if (Ph.b0) {
             for (int j = 0; j < NA / 2; ++j) {
                 const std::string a = saddr(2u * j);
@@ -600,7 +860,12 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 else tmask |= 1u << (int)(std::find(Ph.lanes.begin(), Ph.lanes.end(), pg.pos[b]) - Ph.lanes.begin());
             }
             const int D = 1 << pg.k;
-            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask << "\n";
+            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask
+                << " cls=" << cs.g[g].cls << "\n";
+            if (cs.g[g].cls) {
+                emit_spec(cs.g[g], mask, gbase[g]);
+                continue;
+            }
             if (kind == 2) {  // CZ-like: sign flips of both halves
                 std::string pred;
                 if (popc(mask) != 2) {
@@ -652,6 +917,12 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 }
             }
         }
+        if (last && cs.mode == 4)  // the pass scalar, explicitly
+            for (int j = 0; j < NA; ++j) {
+                P.op("mov.b64 {%fe0, %fe1}, %a", j);
+                fmul("%fo0", "%fo1", "%fe0", "%fe1", cslot);
+                P.op("mov.b64 %a", j, ", {%fo0, %fo1}");
+            }
         if (last && direct) {
             P.op("add.s64 %gst, %gtile, %dg");
             if (lp.b0) {
@@ -752,6 +1023,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
     k << "\t.reg .b64 %a<32>;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
+    k << "\t.reg .f32 %fe<4>, %fo<4>, %ft<2>, %fu<2>, %fn, %fsr, %fsi, %fsn, %fsz;\n";
     k << "\t.reg .b64 %y, %ml, %mh, %zero, %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, "
          "%gnext, %gst, %tf, %tabA, %tabB, %rdA, %rdB;\n";
     k << "\tmov.b64 %zero, 0;\n";
@@ -1306,6 +1578,29 @@ void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compil
     if (compiled) *compiled = g_compiled;
     if (cache_hits) *cache_hits = g_hits;
     if (compile_s) *compile_s = (double)g_compile_ns * 1e-9;
+}
+
+uint64_t rpass_jit_ops_per_amp(const PassDesc& pd, bool zinit) {
+    if (!pd.spec || pd.wide) return rpass_fma_per_amp(pd);
+    uint64_t f = 0;
+    bool first = true;
+    for (const auto& ch : rpass_chunks(pd, SVB_JIT_M, false)) {
+        const ChunkSpec cs = chunk_spec(pd, ch.first, ch.second, zinit && first);
+        for (size_t g = ch.first; g < ch.second; ++g) {
+            const GSpec& x = cs.g[g];
+            const int kind = gate_kind(pd, pd.gates[g]);
+            const uint64_t nu = (x.unit[0] ? 0 : 2) + (x.unit[1] ? 0 : 2);
+            switch (x.cls) {
+                case 1: f += 2 + nu; break;  // 2 FADDs per output, 4 ops per multiplier (per pair)
+                case 2: f += 4; break;
+                case 3: f += nu; break;
+                default: f += kind == 0 ? 4ull << pd.gates[g].k : kind == 1 ? 4 : 0;
+            }
+        }
+        if (cs.mode == 4) f += 4;
+        first = false;
+    }
+    return f;
 }
 
 }  // namespace svb

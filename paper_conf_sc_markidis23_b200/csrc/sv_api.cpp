@@ -87,6 +87,7 @@ struct sv_state {
     int pass_jit = 1;         // SV_OPT_PASS_JIT
     int diag_skip = 1;        // SV_OPT_DIAG_SKIP
     int pass_pin = SVB_PASS_PIN;  // SV_OPT_PASS_PIN: qubits 0..pin-1 in every blocked-pass tile
+    int pass_spec = 1;            // SV_OPT_PASS_SPEC: structured one-qubit gates as additions (reading R11)
     bool sample_pending = false;  // a sv_sample_device status word not yet checked
     // the sampler's bins hold the current state's S5 weights (written by the
     // last register-blocked pass of the last circuit); any state change clears it
@@ -587,6 +588,11 @@ struct PassIn {
 
 // rpass gate kind of a 2^k x 2^k matrix rounded to complex64 (as gate_kind):
 // 0 dense, 1 diagonal, 2 CZ-like diag(1, 1, 1, -1)
+// fp32 operations per amplitude of a pass's kernels (stats, roofline)
+uint64_t pass_ops(const PassDesc& pd, bool zinit) {
+    return pd.spec ? rpass_jit_ops_per_amp(pd, zinit) : rpass_fma_per_amp(pd);
+}
+
 int kind_of(const std::vector<cd>& M, int k) {
     const int D = 1 << k;
     bool diag = true, cz = k == 2;
@@ -1356,7 +1362,8 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
         if (run.empty()) return;
         for (auto& pd : build_passes(T, run, s->pass_pin)) {
             pd.wide = s->fp64;
-            pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
+            pd.spec = s->pass_spec && s->pass_jit && !s->fp64 && pd.mats_shard.empty();
+            pd.fma_per_amp = rpass_supported(pd) ? pass_ops(pd, false) : 0;
             c->stats.fma_apply += pd.fma_per_amp << s->l;
             c->stats.n_passes++;
             sv_circuit::Step st;
@@ -1454,7 +1461,8 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
             c->stats_z.fma_apply = 0;
             for (auto& pd : pz) {
                 pd.wide = s->fp64;
-                pd.fma_per_amp = rpass_supported(pd) ? rpass_fma_per_amp(pd) : 0;
+                pd.spec = s->pass_spec && !s->fp64 && pd.mats_shard.empty();
+                pd.fma_per_amp = rpass_supported(pd) ? pass_ops(pd, &pd == &pz[0]) : 0;
                 c->stats_z.fma_apply += pd.fma_per_amp << s->l;
                 c->stats_z.n_passes++;
                 sv_circuit::Step st;
@@ -2189,6 +2197,10 @@ int sv_set_option(sv_state* s, int option, int value) {
             if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_DIAG_SKIP takes 0 or 1");
             s->diag_skip = value;
             return SV_OK;
+        case SV_OPT_PASS_SPEC:
+            if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_PASS_SPEC takes 0 or 1");
+            s->pass_spec = value;
+            return SV_OK;
         default: return fail(SV_EINVAL, "unknown option");
     }
 }
@@ -2224,6 +2236,7 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
         passes.back().bins = true;  // as sv_circuit_create
     for (auto& pd : passes) {
         pd.wide = wide;
+        pd.spec = !wide;  // as sv_circuit_create with the default SV_OPT_PASS_SPEC
         if (!rpass_supported(pd)) continue;
         for (int z = 0; z < (first ? 2 : 1); ++z) {
             std::vector<RpJitLaunch> ls;

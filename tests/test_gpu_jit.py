@@ -2,8 +2,9 @@
 generic apply_rpass kernel and the oracle.
 
 Both kernels run the same phase plan with the same FFMA2 sequence per complex
-MAC, so their states must be bit-identical; the JIT path is also checked
-against the oracle with the north star's tolerances.
+MAC, so with SV_OPT_PASS_SPEC = 0 their states must be bit-identical; the
+JIT path (with and without the structured-gate arithmetic, R11) is
+also checked against the oracle with the north star's tolerances.
 """
 import numpy as np
 import pytest
@@ -17,10 +18,11 @@ from test_gpu_circuit import _check, _mixed_circuit, layer_depth
 pytestmark = pytest.mark.gpu
 
 
-def _state(n, gates, F, bits, jit, world=1, lazy_zero=True):
+def _state(n, gates, F, bits, jit, world=1, lazy_zero=True, spec=0):
     h = sv.sv_create_ex(n, world=world, virtual_shards=True) if world > 1 else sv.sv_create(n)
     try:
         sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, 1 if jit else 0)
+        sv.sv_set_option(h, sv.SV_OPT_PASS_SPEC, spec)
         sv.sv_set_blocking(h, bits)
         c = sv.sv_circuit_create(h, gates, F)
         if not lazy_zero:
@@ -80,11 +82,14 @@ def test_jit_product_state_start_rqc(n, d, F, bits):
     gates = W.rqc(n, d, seed=n)
     a, sa = _state(n, gates, F, bits, jit=True, lazy_zero=True)
     b, sb = _state(n, gates, F, bits, jit=False, lazy_zero=True)
+    c, sc = _state(n, gates, F, bits, jit=True, lazy_zero=True, spec=1)
     assert sa["n_jit_passes"] == sa["n_passes"] > 0
     assert sa["fma_apply"] < sb["fma_apply"]  # folded gates are not applied
+    assert sc["fma_apply"] <= sa["fma_apply"]
     ref = ref_c.run(n, gates)
     _check(n, d, a, ref)
     _check(n, d, b, ref)
+    _check(n, d, c, ref)
 
 
 @pytest.mark.parametrize("seed", [1, 2, 3])
@@ -142,6 +147,7 @@ def test_jit_30q_sampled_amplitudes_match_generic():
             h = sv.sv_create(n)
             try:
                 sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, 1 if jit else 0)
+                sv.sv_set_option(h, sv.SV_OPT_PASS_SPEC, 0)
                 if not lazy:
                     sv.sv_device_ptr(h)  # writes |0...0> now
                 st = sv.sv_run_circuit(h, gates, 1)
@@ -202,6 +208,7 @@ def test_pass_pin_option(pin, F):
         try:
             sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pin)
             sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, jit)
+            sv.sv_set_option(h, sv.SV_OPT_PASS_SPEC, 0)
             sv.sv_set_blocking(h, 12)
             if not lazy:
                 sv.sv_device_ptr(h)
@@ -215,3 +222,111 @@ def test_pass_pin_option(pin, F):
         out[jit, lazy] = psi
     assert np.array_equal(out[1, False].view(np.uint32), out[0, False].view(np.uint32))
     _check(n, d, out[1, True], ref_c.run(n, gates))
+
+
+# ---------------------------------------------------------------------------
+# Structured one-qubit gates (SV_OPT_PASS_SPEC, R11)
+
+def _structured_circuit(n, m, seed):
+    """Every one-qubit class the pass kernels specialise -- row form (H,
+    sqrt(X), sqrt(Y), with unit and non-unit row-1 factors, T sqrt(X)),
+    column form (H T), diagonals with unit (Z, S, S^dag) and non-unit (T)
+    ratios -- next to generic one-qubit gates (X, Y: zero diagonal; Haar) and CZ / dense two-qubit gates, with gates applied to
+    the same qubit back to back (fused at F = 1) and across tile / thread
+    bits."""
+    rng = np.random.default_rng(seed)
+    w = np.exp(1j * np.pi / 4)
+    pool = [W.GATE_H, W.GATE_X_1_2, W.GATE_Y_1_2, W.GATE_T, W.GATE_Z, W.GATE_S, np.conj(W.GATE_S),
+            W.GATE_T @ W.GATE_X_1_2, W.GATE_H @ W.GATE_T, W.GATE_X, W.GATE_Y, np.diag([1j, np.exp(0.3j)]),
+            np.array([[1, 1j], [1j * w, w]]) / np.sqrt(2), W.haar_unitary(2, rng)]
+    gates = []
+    for t in range(m):
+        r = rng.random()
+        if r < 0.7:
+            q = int(rng.integers(n if rng.random() < 0.5 else 6))
+            M = pool[int(rng.integers(len(pool)))] * np.exp(1j * rng.uniform(0, 2 * np.pi))
+            gates.append(W.Gate(t, "u", (q,), np.asarray(M, dtype=np.complex128)))
+        elif r < 0.9:
+            a, b = (int(x) for x in rng.choice(n, 2, replace=False))
+            gates.append(W.Gate(t, "cz", (a, b), W.GATE_CZ))
+        else:
+            a, b = (int(x) for x in rng.choice(n, 2, replace=False))
+            gates.append(W.Gate(t, "u2", (a, b), W.haar_unitary(4, rng)))
+    return gates
+
+
+@pytest.mark.parametrize("bits", [10, 12, 13])
+@pytest.mark.parametrize("lazy", [True, False])
+def test_spec_structured_gates_vs_oracle(bits, lazy):
+    """Structured-gate arithmetic (additions, one scalar per pass applied
+    into the start state, a generic gate, a row-form gate or explicitly)
+    against the oracle; with SV_OPT_PASS_SPEC = 0 the same circuit runs as
+    dense matrices: both within the bound, the structured one with fewer
+    operations."""
+    n, m = 20, 260
+    gates = _structured_circuit(n, m, seed=bits + 7 * lazy)
+    ref = ref_c.run(n, gates)
+    a, sa = _state(n, gates, 1, bits, jit=True, lazy_zero=lazy, spec=1)
+    b, sb = _state(n, gates, 1, bits, jit=True, lazy_zero=lazy, spec=0)
+    assert sa["n_jit_passes"] > 0
+    assert sa["fma_apply"] < sb["fma_apply"]
+    _check(n, layer_depth(gates), a, ref)
+    _check(n, layer_depth(gates), b, ref)
+
+
+@pytest.mark.parametrize("n,d,bits", [(22, 14, 13), (20, 20, 11), (21, 12, 10)])
+def test_spec_rqc_vs_oracle(n, d, bits):
+    """The RQC (H, sqrt(X), sqrt(Y), T, CZ) through the structured path,
+    from the lazy |0...0> (product start) and a written one; the depth-20
+    case has more passes than the pass scalar can hide (explicit multiply)."""
+    gates = W.rqc(n, d, seed=3 * n + d)
+    ref = ref_c.run(n, gates)
+    for lazy in (True, False):
+        a, sa = _state(n, gates, 1, bits, jit=True, lazy_zero=lazy, spec=1)
+        _check(n, d, a, ref)
+
+
+def test_spec_virtual_shards_and_sampling():
+    """Sharded runs (passes with per-shard matrices stay dense) and the
+    fused sampling bins on a structured final state: samples bit-exact to
+    the oracle sampler on the GPU's final state."""
+    from oracle import sample as osample
+    n, d = 20, 14
+    gates = W.rqc(n, d, seed=11)
+    ref = ref_c.run(n, gates)
+    for world in (1, 2, 4):
+        a, sa = _state(n, gates, 1, 11, jit=True, world=world, spec=1)
+        _check(n, d, a, ref)
+    h = sv.sv_create(n)
+    try:
+        sv.sv_set_blocking(h, 12)
+        sv.sv_run_circuit(h, gates, 1)
+        got = sv.sv_sample(h, 21, 3000)
+        psi = sv.sv_get_state(h, n)
+    finally:
+        sv.sv_destroy(h)
+    assert np.array_equal(got, osample.sample(psi, 21, 3000)[0])
+    _check(n, d, psi, ref)
+
+
+def test_spec_30q_sampled_amplitudes():
+    """Full size (30q D14, the bench step): the structured path within the
+    north-star max-abs bound of the dense-matrix path on 2^16 sampled
+    amplitudes, and with fewer fp32 operations."""
+    n, d = 30, 14
+    gates = W.rqc(n, d)
+    idx = np.random.default_rng(6).integers(0, 1 << n, size=1 << 16).astype(np.uint64)
+    out, ops = {}, {}
+    for spec in (1, 0):
+        h = sv.sv_create(n)
+        try:
+            sv.sv_set_option(h, sv.SV_OPT_PASS_SPEC, spec)
+            st = sv.sv_run_circuit(h, gates, 1)
+            out[spec] = sv.sv_amplitudes(h, idx)
+            ops[spec] = st["fma_apply"]
+        finally:
+            sv.sv_destroy(h)
+    err = np.abs(out[1].astype(np.complex128) - out[0].astype(np.complex128)).max()
+    bound = 1e-5 * 2.0 ** (-n / 2) * d
+    assert err <= bound, (err, bound)
+    assert ops[1] < 0.6 * ops[0], ops
