@@ -24,6 +24,9 @@
 
 using namespace svb;
 
+#ifndef SVB_PASS_COMMUTE
+#define SVB_PASS_COMMUTE 1  // pass formation: a left-out diagonal gate blocks only non-diagonal gates on its qubits
+#endif
 #ifndef SVB_PASS_LOOKAHEAD
 #define SVB_PASS_LOOKAHEAD 1  // pass qubit sets chosen by lookahead (0: first-come greedy)
 #endif
@@ -621,6 +624,11 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
     std::vector<uint64_t> fm(nf, 0);
     for (size_t i = 0; i < nf; ++i)
         for (int b = 0; b < in[i].k; ++b) fm[i] |= 1ull << in[i].q[b];
+    // diagonal gates commute with each other: a left-out diagonal gate only
+    // blocks the non-diagonal gates on its qubits
+    std::vector<char> dg(nf, 0);
+    if (SVB_PASS_COMMUTE)
+        for (size_t i = 0; i < nf; ++i) dg[i] = kind_of(in[i].M, in[i].k) >= 1;
     std::vector<char> placed(nf, 0);
     std::vector<PassDesc> passes;
     auto add_gate = [&](PassDesc& cur, size_t i) {
@@ -662,17 +670,19 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
             // a left-out gate that absorbs the most gates, until nothing helps
             placed[i] = 0;
             auto absorb = [&](uint64_t Qc, std::vector<size_t>* out) {
-                uint64_t Bl = 0;
+                uint64_t Bl = 0, Bd = 0;  // qubits of left-out gates: non-diagonal / diagonal
                 size_t cnt = 0, planes = 0;
                 for (size_t j = i; j < nf; ++j) {
                     if (placed[j]) continue;
                     const uint64_t Sj = fm[j];
                     const size_t pj = 3ull << (2 * in[j].k);
-                    if (!(Sj & Bl) && !(Sj & ~(Qc | pin)) && cnt < (size_t)kPassMaxGates &&
+                    if (!(Sj & (dg[j] ? Bl : Bl | Bd)) && !(Sj & ~(Qc | pin)) && cnt < (size_t)kPassMaxGates &&
                         planes + pj <= (size_t)kPassPlaneFloats) {
                         ++cnt;
                         planes += pj;
                         if (out) out->push_back(j);
+                    } else if (dg[j]) {
+                        Bd |= Sj;
                     } else {
                         Bl |= Sj;
                     }
