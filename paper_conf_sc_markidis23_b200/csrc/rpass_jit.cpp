@@ -357,12 +357,12 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
     const ChunkSpec cs = chunk_spec(pd, g0, g1, zinit);
-    // structured-gate multiplier slot: (sr, si, -si, 0)
+    // structured-gate multiplier slot: (sr, sr, si, si)
     auto put_s = [&](cd z) {
         mats.push_back((float)z.real());
+        mats.push_back((float)z.real());
         mats.push_back((float)z.imag());
-        mats.push_back((float)-z.imag());
-        mats.push_back(0.f);
+        mats.push_back((float)z.imag());
     };
     std::vector<size_t> gbase(pd.gates.size(), 0);
     for (int ph = 0; ph < nph; ++ph)
@@ -402,7 +402,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     // the pass scalar as the start amplitude (|0...0> start without the
     // product state) or for the explicit multiply
     size_t cslot = 0;
-    if ((cs.mode == 1 && pd.pinit_v.empty()) || cs.mode == 4) {
+    if (cs.mode == 1 && pd.pinit_v.empty()) {  // (C re, C im, 0, 0): the start amplitude
+        cslot = mats.size() / 4;
+        mats.push_back((float)cs.C.real());
+        mats.push_back((float)cs.C.imag());
+        mats.push_back(0.f);
+        mats.push_back(0.f);
+    } else if (cs.mode == 4) {
         cslot = mats.size() / 4;
         put_s(cs.C);
     }
@@ -475,48 +481,40 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         P.op("add.s64 ", t, ", ", base, ", ", off);
         return t;
     };
-    // ---- structured gates (GSpec): fp32 scalar arithmetic on the halves of
-    // the packed amplitudes (%fe0..3 inputs, %fo0..3 outputs)
-    // d = eA A + eB B (eA, eB = +-1)
-    auto fsum = [&](const std::string& d, int eA, const std::string& A, int eB, const std::string& B) {
-        if (eA > 0 && eB > 0) P.op("add.rn.f32 ", d, ", ", A, ", ", B);
-        else if (eA > 0) P.op("sub.rn.f32 ", d, ", ", A, ", ", B);
-        else if (eB > 0) P.op("sub.rn.f32 ", d, ", ", B, ", ", A);
-        else {
-            P.op("neg.f32 %fn, ", A);
-            P.op("sub.rn.f32 ", d, ", %fn, ", B);
+    // ---- structured gates (GSpec), on packed amplitudes: i^k X is a swap
+    // and per-lane negations that ptxas folds into the FADD2 / FFMA2 operand
+    // modifiers (.LO_HI, .NP, -), so out = i^q (a0 + i^p a1) is one FADD2 and
+    // a complex multiply s t = sr t + si (i t) one FMUL2 + one FFMA2
+    int nrot = 0;
+    auto rot = [&](const std::string& X, int k) -> std::string {
+        k &= 3;
+        if (k == 0) return X;
+        const std::string t = "%rt" + std::to_string(nrot++ % 8);
+        P.op("mov.b64 {%rlo, %rhi}, ", X);
+        if (k == 1) {
+            P.op("neg.f32 %rnh, %rhi");
+            P.op("mov.b64 ", t, ", {%rnh, %rlo}");
+        } else if (k == 2) {
+            P.op("neg.f32 %rnl, %rlo");
+            P.op("neg.f32 %rnh, %rhi");
+            P.op("mov.b64 ", t, ", {%rnl, %rnh}");
+        } else {
+            P.op("neg.f32 %rnl, %rlo");
+            P.op("mov.b64 ", t, ", {%rhi, %rnl}");
         }
+        return t;
     };
-    // (dr, di) = i^q (A + i^p B)
-    auto flin = [&](const std::string& dr, const std::string& di, int q, int p, const std::string& Ar,
-                    const std::string& Ai, const std::string& Br, const std::string& Bi) {
-        int er, ei;  // i^p B = (er * xr, ei * xi)
-        std::string xr, xi;
-        switch (p & 3) {
-            case 0: er = 1, xr = Br, ei = 1, xi = Bi; break;
-            case 1: er = -1, xr = Bi, ei = 1, xi = Br; break;
-            case 2: er = -1, xr = Br, ei = -1, xi = Bi; break;
-            default: er = 1, xr = Bi, ei = -1, xi = Br; break;
-        }
-        // t = A + i^p B; i^q t: q=0 (t.re, t.im), 1 (-t.im, t.re), 2 (-t.re, -t.im), 3 (t.im, -t.re)
-        auto part = [&](const std::string& d, int sg, bool im) {
-            fsum(d, sg, im ? Ai : Ar, sg * (im ? ei : er), im ? xi : xr);
-        };
-        switch (q & 3) {
-            case 0: part(dr, 1, false), part(di, 1, true); break;
-            case 1: part(dr, -1, true), part(di, 1, false); break;
-            case 2: part(dr, -1, false), part(di, -1, true); break;
-            default: part(dr, 1, true), part(di, -1, false); break;
-        }
+    // d = i^q (A + i^p B)
+    auto plin = [&](const std::string& d, int q, int p, const std::string& A, const std::string& B) {
+        const std::string x = rot(A, q), y = rot(B, p + q);
+        P.op("add.rn.f32x2 ", d, ", ", x, ", ", y);
     };
-    // (dr, di) = s (xr, xi), s from slot (sr, si, -si, 0); d must not alias x
-    auto fmul = [&](const std::string& dr, const std::string& di, const std::string& xr, const std::string& xi,
-                    size_t slot) {
-        P.op("ld.param.v4.f32 {%fsr, %fsi, %fsn, %fsz}, [rpj_param_0+", 16 * slot, "]");
-        P.op("mul.rn.f32 %fu0, ", xi, ", %fsn");
-        P.op("mul.rn.f32 %fu1, ", xi, ", %fsr");
-        P.op("fma.rn.f32 ", dr, ", ", xr, ", %fsr, %fu0");
-        P.op("fma.rn.f32 ", di, ", ", xr, ", %fsi, %fu1");
+    // d = s t, s from slot (sr, sr, si, si); d may alias t
+    auto pmul = [&](const std::string& d, const std::string& t, size_t slot) {
+        P.op("ld.param.v2.b64 {%qsr, %qsi}, [rpj_param_0+", 16 * slot, "]");
+        P.op("mul.rn.f32x2 %py, ", t, ", %qsr");
+        const std::string it = rot(t, 1);
+        P.op("fma.rn.f32x2 ", d, ", ", it, ", %qsi, %py");
     };
     auto emit_spec = [&](const GSpec& x, uint32_t mask, size_t base) {
         size_t sl[2] = {base, base};
@@ -526,19 +524,10 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 const int r = (j & mask) ? 1 : 0;
                 const std::string a = "%a" + std::to_string(j);
                 if (!x.unit[r]) {
-                    P.op("mov.b64 {%fe0, %fe1}, ", a);
-                    fmul("%fo0", "%fo1", "%fe0", "%fe1", sl[r]);
-                    P.op("mov.b64 ", a, ", {%fo0, %fo1}");
-                } else if (x.q[r] == 2) {
-                    P.op("xor.b64 ", a, ", ", a, ", -9223372034707292160");
-                } else if (x.q[r] == 1) {  // (re, im) -> (-im, re)
-                    P.op("mov.b64 {%fe0, %fe1}, ", a);
-                    P.op("neg.f32 %fn, %fe1");
-                    P.op("mov.b64 ", a, ", {%fn, %fe0}");
-                } else if (x.q[r] == 3) {  // (im, -re)
-                    P.op("mov.b64 {%fe0, %fe1}, ", a);
-                    P.op("neg.f32 %fn, %fe0");
-                    P.op("mov.b64 ", a, ", {%fe1, %fn}");
+                    pmul(a, a, sl[r]);
+                } else if (x.q[r]) {  // i^q a (one FMUL2 by 1 carries the rotation)
+                    const std::string t = rot(a, x.q[r]);
+                    P.op("mul.rn.f32x2 ", a, ", ", t, ", %pone");
                 }
             }
             return;
@@ -546,25 +535,25 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         for (uint32_t j0 = 0; j0 < (uint32_t)NA; ++j0) {
             if (j0 & mask) continue;
             const uint32_t j1 = j0 | mask;
-            P.op("mov.b64 {%fe0, %fe1}, %a", j0);
-            P.op("mov.b64 {%fe2, %fe3}, %a", j1);
-            if (x.cls == 2) {  // out0 = a0 + mu a1, out1 = i^p0 (a0 + i^(p1-p0) mu a1)
-                fmul("%ft0", "%ft1", "%fe2", "%fe3", sl[0]);
-                flin("%fo0", "%fo1", 0, 0, "%fe0", "%fe1", "%ft0", "%ft1");
-                flin("%fo2", "%fo3", x.p[0], (x.p[1] - x.p[0]) & 3, "%fe0", "%fe1", "%ft0", "%ft1");
+            const std::string a0 = "%a" + std::to_string(j0), a1 = "%a" + std::to_string(j1);
+            if (x.cls == 2) {  // out0 = a0 + mu a1, out1 = i^p0 a0 + i^p1 (mu a1)
+                pmul("%pt", a1, sl[0]);
+                plin("%po0", 0, 0, a0, "%pt");
+                const std::string u = rot(a0, x.p[0]), v = rot("%pt", x.p[1]);
+                P.op("add.rn.f32x2 %po1, ", u, ", ", v);
             } else {  // row form: out_r = s_r (a0 + i^p_r a1)
                 for (int r = 0; r < 2; ++r) {
-                    const std::string dr = "%fo" + std::to_string(2 * r), di = "%fo" + std::to_string(2 * r + 1);
+                    const std::string d = "%po" + std::to_string(r);
                     if (x.unit[r]) {
-                        flin(dr, di, x.q[r], x.p[r], "%fe0", "%fe1", "%fe2", "%fe3");
+                        plin(d, x.q[r], x.p[r], a0, a1);
                     } else {
-                        flin("%ft0", "%ft1", 0, x.p[r], "%fe0", "%fe1", "%fe2", "%fe3");
-                        fmul(dr, di, "%ft0", "%ft1", sl[r]);
+                        plin("%pt", 0, x.p[r], a0, a1);
+                        pmul(d, "%pt", sl[r]);
                     }
                 }
             }
-            P.op("mov.b64 %a", j0, ", {%fo0, %fo1}");
-            P.op("mov.b64 %a", j1, ", {%fo2, %fo3}");
+            P.op("mov.b64 ", a0, ", %po0");
+            P.op("mov.b64 ", a1, ", %po1");
         }
     };
     // ---- prologue: thread constants
@@ -827,7 +816,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("setp.ne.u32 %p_z, %zone, 0");
             P.op("setp.eq.and.u64 %p_z, %u, 0, %p_z");
             P.op("setp.eq.and.u32 %p_z, %t_id, 0, %p_z");
-            if (cs.mode == 1)  // (C re, C im)
+            if (cs.mode == 1 && !pinit)  // (C re, C im)
                 P.op("@%p_z ld.param.b64 %a0, [rpj_param_0+", 16 * cslot, "]");
             else
                 P.op("@%p_z mov.b64 %a0, 1065353216");  // (1.0f, 0.0f)
@@ -867,16 +856,18 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 continue;
             }
             if (kind == 2) {  // CZ-like: sign flips of both halves
-                std::string pred;
+                // one FMUL2 per flipped amplitude (2 LOP3s as an xor), by -1
+                // or, when a qubit is a thread bit, by this thread's sign
+                std::string sg = "%mneg1";
                 if (popc(mask) != 2) {
-                    const std::string t = P.r32();
-                    pred = P.pr();
+                    const std::string t = P.r32(), q = P.pr();
                     P.op("and.b32 ", t, ", %t_id, ", tmask);
-                    P.op("setp.eq.u32 ", pred, ", ", t, ", ", tmask);
-                    pred = "@" + pred + " ";
+                    P.op("setp.eq.u32 ", q, ", ", t, ", ", tmask);
+                    P.op("selp.b64 %csg, %mneg1, %pone, ", q);
+                    sg = "%csg";
                 }
                 for (uint32_t j = 0; j < (uint32_t)NA; ++j)
-                    if ((j & mask) == mask) P.op(pred, "xor.b64 %a", j, ", %a", j, ", -9223372034707292160");
+                    if ((j & mask) == mask) P.op("mul.rn.f32x2 %a", j, ", %a", j, ", ", sg);
                 continue;
             }
             const size_t base = gbase[g];
@@ -918,11 +909,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             }
         }
         if (last && cs.mode == 4)  // the pass scalar, explicitly
-            for (int j = 0; j < NA; ++j) {
-                P.op("mov.b64 {%fe0, %fe1}, %a", j);
-                fmul("%fo0", "%fo1", "%fe0", "%fe1", cslot);
-                P.op("mov.b64 %a", j, ", {%fo0, %fo1}");
-            }
+            for (int j = 0; j < NA; ++j) pmul("%a" + std::to_string(j), "%a" + std::to_string(j), cslot);
         if (last && direct) {
             P.op("add.s64 %gst, %gtile, %dg");
             if (lp.b0) {
@@ -1023,10 +1010,10 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
     k << "\t.reg .b64 %a<32>;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
-    k << "\t.reg .f32 %fe<4>, %fo<4>, %ft<2>, %fu<2>, %fn, %fsr, %fsi, %fsn, %fsz;\n";
+    k << "\t.reg .f32 %rlo, %rhi, %rnl, %rnh;\n\t.reg .b64 %rt<8>, %po0, %po1, %pt, %py, %qsr, %qsi, %pone, %mneg1, %csg;\n";
     k << "\t.reg .b64 %y, %ml, %mh, %zero, %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, "
          "%gnext, %gst, %tf, %tabA, %tabB, %rdA, %rdB;\n";
-    k << "\tmov.b64 %zero, 0;\n";
+    k << "\tmov.b64 %zero, 0;\n\tmov.b64 %pone, 4575657222473777152;\n\tmov.b64 %mneg1, -4647714812233515008;\n";  // (1, 1), (-1, -1)
     k << P.o.str();
     k << "}\n";
     return k.str();
