@@ -223,7 +223,7 @@ int sv_device_ptr(sv_state* s, int shard, void** out);
  * writes nothing to buf.  (SURVEY.md §8b / §8c-S3.) */
 int sv_fusion_plan(const sv_gate* gates, size_t n_gates, int max_fused, int32_t* buf, size_t cap, size_t* need);
 /* Cache-blocked pass plan (pure host; reading R7, §7) of the fusion
- * plan for max_fused in [1,4] and tile_bits in [10,13], as a flat int32 stream:
+ * plan for max_fused in [1,4] and tile_bits in [10,14], as a flat int32 stream:
  * per pass  T, S_0..S_{T-1} (tile qubits, ascending), n, f_0..f_{n-1} (fused-
  * gate indices of sv_fusion_plan, in pass order), n_phases, then per phase of
  * the register-blocked kernel (0 phases when the pass has a gate with k > 2)
@@ -271,8 +271,12 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each);
  * ONE HBM read + write of the state.  Passes of gates with k <= 2 run in the
  * register-blocked kernel (32 amplitudes per thread, gates applied in
  * registers); others in the shared-memory pass kernel.
- * tile_bits in [10,13]; 0 disables (one launch per fused gate); -1 (default)
- * = auto: 13 when max_fused <= 2 and the shard has >= 20 qubits, else off.  Takes effect for
+ * tile_bits in [10,14]; 0 disables (one launch per fused gate); -1 (default)
+ * = auto: when max_fused <= 2 and the shard has >= 20 qubits, 14 (complex64
+ * with SV_OPT_PASS_JIT), 13 (generic kernel), 12 (complex128), else off.
+ * 14-qubit tiles (512 threads, 128 KB of shared memory per pass CTA) exist
+ * only as pass-specialised complex64 kernels: a circuit created with 14 and
+ * SV_OPT_PASS_JIT 0, complex128 or max_fused > 2 uses 13.  Takes effect for
  * circuits created afterwards.  Errors: SV_EINVAL for other values. */
 int sv_set_blocking(sv_state* s, int tile_bits);
 /* 1: record CUDA events around every launch and fill the *_dev_s stats. */
@@ -331,7 +335,7 @@ int sv_synchronize(sv_state* s);
 int sv_set_option(sv_state* s, int option, int value);
 
 /* PTX of the pass-specialised kernels of every register-blocked pass of a
- * circuit (max_fused in [1, 2], tile_bits in [10, 13]; the first pass also
+ * circuit (max_fused in [1, 2], tile_bits in [10, 14]; the first pass also
  * in its |0...0> form), separated by "//----" lines.  Pure host unless
  * compile != 0, which also assembles them through the driver JIT on the
  * current device (SV_ECUDA with the JIT log on failure).  tile_bits < 0:

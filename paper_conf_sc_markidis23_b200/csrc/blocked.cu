@@ -1305,7 +1305,7 @@ cudaError_t launch_rpass_m(float2* psi, int n, const PassDesc& pd, cudaStream_t 
 bool rpass_supported(const PassDesc& pd) {
     if (!SVB_RP_ENABLE) return false;
     const int T = (int)pd.S.size();
-    if (T < 10 || T > 13 || pd.r < 1) return false;
+    if (T < 10 || T > 14 || pd.r < 1) return false;  // 14: pass-specialised kernels only
     for (auto& g : pd.gates)
         if (g.k > 2) return false;
     return true;
@@ -1342,6 +1342,7 @@ void rpass_plan_stats(const PassDesc& pd, int* n_phases, int* worst_conflict) {
 cudaError_t launch_rpass(float2* psi, int n, const PassDesc& pd, cudaStream_t st, bool zinit, bool zone, int slot) {
     static_assert(sizeof(RpassParams) <= 32764, "rpass params exceed the kernel parameter space");
     constexpr bool f2 = SVB_RP_F2 != 0;
+    if (pd.S.size() > 13) return cudaErrorInvalidValue;  // 14-qubit tiles: pass-specialised kernels only
     if (rpass_m() == 5) return f2 ? launch_rpass_m<5, true>(psi, n, pd, st, zinit, zone, slot) : launch_rpass_m<5, false>(psi, n, pd, st, zinit, zone, slot);
     return f2 ? launch_rpass_m<4, true>(psi, n, pd, st, zinit, zone, slot) : launch_rpass_m<4, false>(psi, n, pd, st, zinit, zone, slot);
 }

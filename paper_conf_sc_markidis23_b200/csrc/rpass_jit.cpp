@@ -41,6 +41,9 @@
 #ifndef SVB_JIT_RING
 #define SVB_JIT_RING 0  // two warp groups over three tile buffers per CTA (loads 1.5 tiles ahead)
 #endif
+#ifndef SVB_JIT_DB
+#define SVB_JIT_DB 0  // two tile buffers per CTA: the next tile loads during the whole current tile
+#endif
 #ifndef SVB_JIT_PF
 #define SVB_JIT_PF 0  // L2 bulk prefetch of the next tile at the top of each tile (pass kernels)
 #endif
@@ -353,6 +356,10 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     // read of tile k) loads tile k + 3 (the other group's) into it, tracked by
     // an mbarrier -- loads are issued one and a half tiles ahead
     const bool ring = SVB_JIT_RING != 0;
+    // double buffering (SVB_JIT_DB): tile u computes in buffer %cur while
+    // tile u + grid loads into %alt; the last phase frees %cur and loads
+    // tile u + 2 grid into it
+    const bool db = SVB_JIT_DB && !ring && !zinit;
     const uint32_t tile_bytes = 8u << T;
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
@@ -624,11 +631,11 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     P.op("cvt.u64.u32 %u, %r_c");
     P.op("mov.u32 %r_c, %nctaid.x");
     P.op("cvt.u64.u32 %grid, %r_c");
-    auto loadtile = [&](const std::string& g, const std::string& pred) {
+    auto loadtile = [&](const std::string& g, const std::string& pred, const std::string& base = "%cur") {
         for (int i = 0; i < UPT; ++i) {
             const std::string sa = P.r32();
             P.op("xor.b32 ", sa, ", %sthr, ", fold_swz(2u * nthr * i, T) << 3);
-            P.op("add.s32 ", sa, ", ", sa, ", %cur");
+            P.op("add.s32 ", sa, ", ", sa, ", ", base);
             const std::string ga = gaddr(P, g, 8 * tm.dep(2ull * nthr * i));
             P.op(pred, "cp.async.cg.shared.global [", sa, "], ", ga, ", 16");
         }
@@ -679,6 +686,16 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         P.op("add.s64 %gcur, %gtile, %dthr");
         if (!zinit) loadtile("%gcur", "");
         P.op("cp.async.commit_group");
+        if (db) {  // the second tile into the other buffer
+            P.op("add.u32 %alt, %rsm0, ", tile_bytes);
+            P.op("add.s64 %un, %u, %grid");
+            P.op("setp.lt.u64 %p_next, %un, %ntiles");
+            emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+            P.op("add.s64 %gnext, %psi, %tbo");
+            P.op("add.s64 %gnext, %gnext, %dthr");
+            loadtile("%gnext", "@%p_next ", "%alt");
+            P.op("cp.async.commit_group");
+        }
     }
     P.o << "$LOOP:\n";
     if (ring) {
@@ -711,6 +728,18 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         P.op("mbarrier.try_wait.parity.shared.b64 %p_w, [%fb], %par");
         P.op("@!%p_w bra $WAIT");
         P.o << "$READY:\n";
+    } else if (db) {
+        // this tile's addresses, and the tile two ahead (loaded into %cur
+        // once this tile's last phase has read it)
+        emit_tbase(P, pd.S, n_local, "%u", "%tbo");
+        P.op("add.s64 %gtile, %psi, %tbo");
+        P.op("add.s64 %gcur, %gtile, %dthr");
+        P.op("add.s64 %un, %u, %grid");
+        P.op("add.s64 %un, %un, %grid");
+        P.op("setp.lt.u64 %p_next, %un, %ntiles");
+        emit_tbase(P, pd.S, n_local, "%un", "%tbo");
+        P.op("add.s64 %gnext, %psi, %tbo");
+        P.op("add.s64 %gnext, %gnext, %dthr");
     } else {
         P.op("add.s64 %un, %u, %grid");
         P.op("setp.lt.u64 %p_next, %un, %ntiles");
@@ -743,7 +772,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         }
     }
     if (!ring) {
-        P.op("cp.async.wait_group 0");
+        P.op(db ? "cp.async.wait_group 1" : "cp.async.wait_group 0");  // db: the newest group is the next tile
         P.op("bar.sync 0");
     }
     // ring: release buffer bb (this group is done reading it): load the tile
@@ -984,6 +1013,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         P.op("@%p_w sub.u32 %bb, %bb, 3");
         P.op("setp.lt.u64 %p_w, %u, %ntiles");
         P.op("@%p_w bra $LOOP");
+    } else if (db) {
+        P.op("mov.u32 %r_c, %cur");
+        P.op("mov.u32 %cur, %alt");
+        P.op("mov.u32 %alt, %r_c");
+        P.op("add.s64 %u, %u, %grid");
+        P.op("setp.lt.u64 %p_w, %u, %ntiles");
+        P.op("@%p_w bra $LOOP");
     } else {
         P.op("mov.b64 %gcur, %gnext");
         P.op("mov.b64 %gtile, %gtile_next");
@@ -1005,7 +1041,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
     k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg " << (M == 5 ? 128 : 64) << "\n{\n";
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw, %p_w;\n";
-    k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par;\n\t.reg .b64 %rdk;\n";
+    k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par, %alt;\n\t.reg .b64 %rdk;\n";
     k << "\t.reg .f64 %dre, %dim, %dp;\n\t.reg .b64 %w, %wt, %bo, %bins;\n\t.reg .b32 %wl, %wh, %wl2, %wh2;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
@@ -1465,7 +1501,8 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
                                       : gen_chunk(pd, n_local, ch.first, ch.second, z, nm, l.mats);
                 const bool ring = SVB_JIT_RING && !pd.wide;
                 l.kern->nthr = (1 << (T - M)) * (ring ? 2 : 1);
-                l.kern->smem = ((size_t)(pd.wide ? 16 : 8) << T) * (ring ? 3 : 1) + (ring ? 64 : 0);
+                const bool db = SVB_JIT_DB && !ring && !z && !pd.wide;  // as gen_chunk
+                l.kern->smem = ((size_t)(pd.wide ? 16 : 8) << T) * (ring ? 3 : db ? 2 : 1) + (ring ? 64 : 0);
                 l.kern->T = T;
                 l.kern->nm = nm;
                 l.kern->param_bytes = std::max<size_t>(nm, 1) * 16 + 48;  // as in gen_chunk

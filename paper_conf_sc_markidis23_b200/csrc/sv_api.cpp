@@ -1120,7 +1120,7 @@ int sv_block_plan(const sv_gate* gates, size_t n_gates, int max_fused, int tile_
                   size_t* need) {
     if (!need) return fail(SV_EINVAL, "need is NULL");
     if (max_fused < 1 || max_fused > 4) return fail(SV_EINVAL, "max_fused must be in [1, 4] for blocked passes");
-    if (tile_bits < 10 || tile_bits > 13) return fail(SV_EINVAL, "tile_bits must be in [10, 13]");
+    if (tile_bits < 10 || tile_bits > 14) return fail(SV_EINVAL, "tile_bits must be in [10, 14]");
     int rc = validate_gates(gates, n_gates, -1);
     if (rc) return rc;
     std::vector<FusedGate> plan;
@@ -1294,11 +1294,14 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
     // Cache-blocked passes (complex64, large shards, k <= 4; sharded or not):
     // each maximal run of APPLY events between exchanges is cut into passes
     // by build_passes (reading R7); exchanges and permutations stay as they are.
-    // auto tile: 13 qubits (with the early next-tile load of apply_rpass:
-    // 30q D14 F=1 0.0745 s vs 0.0775 s at 12; 32q D20 0.430 vs 0.462 s)
     // complex128 states: pass-specialised fp64 kernels (16 amplitudes per
-    // thread, auto tile 12 qubits = 64 KB) for max_fused <= 2
-    const int T = s->block_bits >= 0 ? s->block_bits : (max_fused <= 2 && s->l >= 20 ? (s->fp64 ? 12 : 13) : 0);
+    // thread, auto tile 12 qubits = 64 KB) for max_fused <= 2.
+    // auto tile: 14 qubits for the complex64 pass kernels (512 threads, 128 KB;
+    // 30q D14 F=1 24.7 ms vs 26.1 at 13, 32q D20 145 vs 166 ms: fewer passes
+    // for the same runs), 13 for the generic kernel, 12 for complex128
+    int T = s->block_bits >= 0 ? s->block_bits
+                               : (max_fused <= 2 && s->l >= 20 ? (s->fp64 ? 12 : s->pass_jit ? 14 : 13) : 0);
+    if (T == 14 && (s->fp64 || !s->pass_jit || max_fused > 2)) T = 13;  // 14-qubit tiles: complex64 pass kernels only
     const bool blocked = (!s->fp64 || (s->pass_jit && max_fused <= 2)) && T >= 10 && s->l >= T + 2 &&
                          s->n > kSmallCircuitMaxQubits && max_fused <= 4 && max_fused >= 1;
     // plan (sharded) or trivial apply list
@@ -2179,8 +2182,8 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each) {
 
 int sv_set_blocking(sv_state* s, int tile_bits) {
     if (!s) return fail(SV_EINVAL, "state handle is NULL");
-    if (tile_bits != 0 && tile_bits != -1 && (tile_bits < 10 || tile_bits > 13))
-        return fail(SV_EINVAL, "tile_bits must be 0 (off), -1 (auto) or in [10, 13]");
+    if (tile_bits != 0 && tile_bits != -1 && (tile_bits < 10 || tile_bits > 14))
+        return fail(SV_EINVAL, "tile_bits must be 0 (off), -1 (auto) or in [10, 14]");
     s->block_bits = tile_bits;
     return SV_OK;
 }
@@ -2221,7 +2224,8 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
     if (max_fused < 1 || max_fused > 2) return fail(SV_EINVAL, "max_fused must be in [1, 2] for register-blocked passes");
     const bool wide = tile_bits < 0;  // complex128 kernels
     if (wide) tile_bits = -tile_bits;
-    if (tile_bits < 10 || tile_bits > 13) return fail(SV_EINVAL, "tile_bits must be in [10, 13] (or -13..-10)");
+    if (tile_bits < 10 || tile_bits > (wide ? 13 : 14))
+        return fail(SV_EINVAL, "tile_bits must be in [10, 14] (complex128: -13..-10)");
     int rc = validate_gates(gates, n_gates, -1);
     if (rc) return rc;
     std::vector<FusedGate> plan;

@@ -148,6 +148,7 @@ def test_jit_30q_sampled_amplitudes_match_generic():
             try:
                 sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, 1 if jit else 0)
                 sv.sv_set_option(h, sv.SV_OPT_PASS_SPEC, 0)
+                sv.sv_set_blocking(h, 13)  # the generic kernel's largest tile
                 if not lazy:
                     sv.sv_device_ptr(h)  # writes |0...0> now
                 st = sv.sv_run_circuit(h, gates, 1)
@@ -162,7 +163,7 @@ def test_jit_30q_sampled_amplitudes_match_generic():
     assert err <= bound, (err, bound)
 
 
-@pytest.mark.parametrize("bits", [10, 11, 12, 13])
+@pytest.mark.parametrize("bits", [10, 11, 12, 13, 14])
 @pytest.mark.parametrize("F", [1, 2])
 def test_fused_sampling_bins_bit_exact(bits, F):
     """The circuit's last pass writes the sampler's 16-amplitude S5 bin
@@ -255,7 +256,7 @@ def _structured_circuit(n, m, seed):
     return gates
 
 
-@pytest.mark.parametrize("bits", [10, 12, 13])
+@pytest.mark.parametrize("bits", [10, 12, 13, 14])
 @pytest.mark.parametrize("lazy", [True, False])
 def test_spec_structured_gates_vs_oracle(bits, lazy):
     """Structured-gate arithmetic (additions, one scalar per pass applied
@@ -274,7 +275,7 @@ def test_spec_structured_gates_vs_oracle(bits, lazy):
     _check(n, layer_depth(gates), b, ref)
 
 
-@pytest.mark.parametrize("n,d,bits", [(22, 14, 13), (20, 20, 11), (21, 12, 10)])
+@pytest.mark.parametrize("n,d,bits", [(22, 14, 13), (20, 20, 11), (21, 12, 10), (22, 16, 14)])
 def test_spec_rqc_vs_oracle(n, d, bits):
     """The RQC (H, sqrt(X), sqrt(Y), T, CZ) through the structured path,
     from the lazy |0...0> (product start) and a written one; the depth-20
@@ -330,3 +331,36 @@ def test_spec_30q_sampled_amplitudes():
     bound = 1e-5 * 2.0 ** (-n / 2) * d
     assert err <= bound, (err, bound)
     assert ops[1] < 0.6 * ops[0], ops
+
+
+@pytest.mark.parametrize("pin", [4, 5])
+@pytest.mark.parametrize("F", [1, 2])
+def test_tile14_vs_oracle(pin, F):
+    """14-qubit tiles (512 threads, 128 KB of shared memory; pass-specialised
+    kernels only): RQC and mixed circuits from the lazy and a written
+    |0...0>, with 128 B and 256 B runs, against the oracle; the generic
+    kernel refuses them (sv_set_blocking(14) with SV_OPT_PASS_JIT 0 runs 13)."""
+    n, d = 21, 14
+    for gates in (W.rqc(n, d, seed=pin + F), _mixed_circuit(n, 160, seed=9 * pin + F)):
+        ref = ref_c.run(n, gates)
+        for lazy in (True, False):
+            h = sv.sv_create(n)
+            try:
+                sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pin)
+                sv.sv_set_blocking(h, 14)
+                if not lazy:
+                    sv.sv_device_ptr(h)
+                st = sv.sv_run_circuit(h, gates, F)
+                psi = sv.sv_get_state(h, n)
+            finally:
+                sv.sv_destroy(h)
+            assert st["block_bits"] == 14 and st["n_jit_passes"] == st["n_passes"] > 0, st
+            _check(n, layer_depth(gates), psi, ref)
+    h = sv.sv_create(n)
+    try:
+        sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, 0)
+        sv.sv_set_blocking(h, 14)
+        st = sv.sv_run_circuit(h, W.rqc(n, d), 1)
+        assert st["block_bits"] == 13, st
+    finally:
+        sv.sv_destroy(h)

@@ -1,5 +1,5 @@
 """Interleaved A/B of the bench step (reset + circuit + 10^6 samples; host wall time, mean of 10)
-across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3] python tools/ab_step.py <rounds> <lib.so> ...
+across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3 AB_T=12] python tools/ab_step.py <rounds> <lib.so> ...
 """
 import json, os, subprocess, sys
 CHILD = r'''
@@ -12,6 +12,7 @@ import os
 n=int(os.environ.get("AB_N", "30")); d=int(os.environ.get("AB_D", "14"))
 h=sv.sv_create(n)
 if os.environ.get("AB_PIN"): sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, int(os.environ["AB_PIN"]))
+if os.environ.get("AB_T"): sv.sv_set_blocking(h, int(os.environ["AB_T"]))
 c=sv.sv_circuit_create(h, W.rqc(n,d), 1)
 out=torch.empty(1000000, dtype=torch.int64, device="cuda")
 def step():
