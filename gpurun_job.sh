@@ -1,3 +1,18 @@
-mkdir -p gpurun_out/t14
-timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/t14/pytest.log 2>&1; tail -15 gpurun_out/t14/pytest.log
-timeout 900 python bench.py > gpurun_out/t14/bench.json 2> gpurun_out/t14/bench.err; tail -1 gpurun_out/t14/bench.json | cut -c1-600
+#!/bin/bash
+# One validation job on a B200 box: GPU suite, bench, configs, ncu launch list
+# and full captures of every pass of the 30q D14 F=1 circuit.
+# usage: gpurun -- 'bash gpurun_job.sh <tag>'
+T=${1:-job}
+O=gpurun_out/$T
+mkdir -p $O
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.total --format=csv > $O/gpu.txt 2>&1
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
+timeout 2400 python -m pytest tests -m gpu -q -x > $O/pytest.log 2>&1; tail -5 $O/pytest.log
+timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; tail -1 $O/bench.json | cut -c1-400
+if [ "${NO_CONFIGS:-0}" = 0 ]; then bash tools/run_configs.sh $O/configs.jsonl; fi
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 400 --csv \
+  --log-file $O/launches.csv python bench.py --steps 2 --warmup 1 --no-sweep --no-cpu-baseline > $O/ncu_bench.log 2>&1
+timeout 1200 ncu --set full --clock-control none --import-source on -k regex:rpj -c 12 \
+  -o $O/rpj_full python tools/prof_circuit.py 30 14 1 1 > $O/ncu_full.log 2>&1
+ncu -i $O/rpj_full.ncu-rep --page raw --csv > $O/rpj_full_raw.csv 2>/dev/null
+echo done

@@ -273,7 +273,7 @@ int sv_attach_peers(sv_state* s, const void* handles, size_t each);
  * registers); others in the shared-memory pass kernel.
  * tile_bits in [10,14]; 0 disables (one launch per fused gate); -1 (default)
  * = auto: when max_fused <= 2 and the shard has >= 20 qubits, 14 (complex64
- * with SV_OPT_PASS_JIT), 13 (generic kernel), 12 (complex128), else off.
+ * with SV_OPT_PASS_JIT), 13 (generic kernel or complex128), else off.
  * 14-qubit tiles (512 threads, 128 KB of shared memory per pass CTA) exist
  * only as pass-specialised complex64 kernels: a circuit created with 14 and
  * SV_OPT_PASS_JIT 0, complex128 or max_fused > 2 uses 13.  Takes effect for

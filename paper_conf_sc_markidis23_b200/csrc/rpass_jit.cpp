@@ -44,6 +44,12 @@
 #ifndef SVB_JIT_DB
 #define SVB_JIT_DB 0  // two tile buffers per CTA: the next tile loads during the whole current tile
 #endif
+#ifndef SVB_JIT_PL
+#define SVB_JIT_PL 0  // three quarters of the next tile land in a spare buffer during the whole current tile
+#endif
+#ifndef SVB_JIT_L2PF
+#define SVB_JIT_L2PF 0  // tile loads with an L2 prefetch-size hint: 1 = 128 B, 2 = 256 B (the neighbouring tile's run)
+#endif
 #ifndef SVB_JIT_PF
 #define SVB_JIT_PF 0  // L2 bulk prefetch of the next tile at the top of each tile (pass kernels)
 #endif
@@ -143,7 +149,7 @@ bool unit_exp(cd z, int& e) {
 }
 GSpec classify(const PassDesc& pd, const PassGate& pg) {
     GSpec g;
-    if (!pd.spec || pd.wide || pg.k != 1 || pd.mats64.size() < pg.moff + 8) return g;
+    if (!pd.spec || pg.k != 1 || pd.mats64.size() < pg.moff + 8) return g;
     const int kind = gate_kind(pd, pg);
     const double* m = pd.mats64.data() + pg.moff;
     const cd u00(m[0], m[1]), u01(m[2], m[3]), u10(m[4], m[5]), u11(m[6], m[7]);
@@ -191,7 +197,7 @@ struct ChunkSpec {
 ChunkSpec chunk_spec(const PassDesc& pd, size_t g0, size_t g1, bool zinit) {
     ChunkSpec cs;
     cs.g.resize(pd.gates.size());
-    if (!pd.spec || pd.wide) return cs;
+    if (!pd.spec) return cs;
     bool any = false;
     for (size_t i = 0; i < pd.gates.size(); ++i) {
         cs.g[i] = classify(pd, pd.gates[i]);
@@ -360,6 +366,14 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     // tile u + grid loads into %alt; the last phase frees %cur and loads
     // tile u + 2 grid into it
     const bool db = SVB_JIT_DB && !ring && !zinit;
+    // pre-landing (SVB_JIT_PL): the tile buffer is only free between the
+    // last phase's gather and the next tile's first gather, so a single
+    // buffer leaves HBM idle during all earlier phases.  A spare buffer of
+    // 3/4 tile takes quarters 0..2 (top two tile bits) of the next tile,
+    // issued right after this tile's first gather; quarter 3 lands in the
+    // tile buffer once the last phase has read it.  The first gather of a
+    // tile reads quarters 0..2 from the spare buffer (same swizzle).
+    const bool pl = SVB_JIT_PL && !ring && !db && !zinit && M >= 3;
     const uint32_t tile_bytes = 8u << T;
     // matrix slots first (their count fixes the parameter layout)
     mats.clear();
@@ -631,13 +645,20 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     P.op("cvt.u64.u32 %u, %r_c");
     P.op("mov.u32 %r_c, %nctaid.x");
     P.op("cvt.u64.u32 %grid, %r_c");
-    auto loadtile = [&](const std::string& g, const std::string& pred, const std::string& base = "%cur") {
+    // quarters: bit q of `qmask` loads the units whose top two tile bits
+    // are q (unit i: tile index 2 (tid + nthr i), top bits = i >> (M - 3));
+    // with pre-landing quarters 0..2 go to the spare buffer
+    auto loadtile = [&](const std::string& g, const std::string& pred, const std::string& base = "%cur",
+                        unsigned qmask = 15u) {
         for (int i = 0; i < UPT; ++i) {
+            const int quarter = i >> (M - 3);
+            if (!((qmask >> quarter) & 1u)) continue;
             const std::string sa = P.r32();
             P.op("xor.b32 ", sa, ", %sthr, ", fold_swz(2u * nthr * i, T) << 3);
-            P.op("add.s32 ", sa, ", ", sa, ", ", base);
+            P.op("add.s32 ", sa, ", ", sa, ", ", pl && quarter < 3 ? std::string("%spr") : base);
             const std::string ga = gaddr(P, g, 8 * tm.dep(2ull * nthr * i));
-            P.op(pred, "cp.async.cg.shared.global [", sa, "], ", ga, ", 16");
+            P.op(pred, "cp.async.cg.shared.global", SVB_JIT_L2PF == 1 ? ".L2::128B" : SVB_JIT_L2PF == 2 ? ".L2::256B" : "",
+                 " [", sa, "], ", ga, ", 16");
         }
     };
     const std::string gbar = ring ? "bar.sync %bid, " + std::to_string(nthr) : std::string("bar.sync 0");
@@ -684,6 +705,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         emit_tbase(P, pd.S, n_local, "%u", "%tbo");
         P.op("add.s64 %gtile, %psi, %tbo");
         P.op("add.s64 %gcur, %gtile, %dthr");
+        if (pl) P.op("add.u32 %spr, %rsm0, ", tile_bytes);
         if (!zinit) loadtile("%gcur", "");
         P.op("cp.async.commit_group");
         if (db) {  // the second tile into the other buffer
@@ -800,10 +822,42 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             P.op("setp.ne.u32 ", q, ", ", t, ", 0");
             P.op("@", q, " xor.b32 %tb, %tb, ", fold_swz(1u << Ph.lanes[b], T) << 3);
         }
-        auto saddr = [&](uint32_t j) {
+        // pre-landed first gather: the base of an amplitude depends on its
+        // quarter = (lane part of the top tile bits) | (register part);
+        // one base per register part, chosen per thread
+        const bool plg = pl && ph == 0;
+        uint32_t qreg_mask = 0;  // register bits (of j) that are top tile bits -> quarter bit
+        if (plg) {
+            P.op("mov.b32 %qt, 0");
+            for (int b = 0; b < tbits; ++b)
+                if (Ph.lanes[b] >= T - 2) {
+                    const std::string t = P.r32(), q = P.pr();
+                    P.op("and.b32 ", t, ", %t_id, ", 1u << b);
+                    P.op("setp.ne.u32 ", q, ", ", t, ", 0");
+                    P.op("@", q, " or.b32 %qt, %qt, ", 1u << (Ph.lanes[b] - (T - 2)));
+                }
+            for (int v = 0; v < 4; ++v) {
+                bool ok = true;  // v must be reachable from register bits
+                for (int qb = 0; qb < 2; ++qb)
+                    if (((v >> qb) & 1) && std::find(Ph.R.begin(), Ph.R.end(), T - 2 + qb) == Ph.R.end()) ok = false;
+                if (!ok) continue;
+                const std::string t = P.r32(), q = P.pr();
+                P.op("or.b32 ", t, ", %qt, ", v);
+                P.op("setp.eq.u32 ", q, ", ", t, ", 3");
+                P.op("selp.b32 %pb", v, ", %cur, %spr, ", q);
+            }
+            for (int b = 0; b < M; ++b)
+                if (Ph.R[b] >= T - 2) qreg_mask |= 1u << b;
+        }
+        auto saddr = [&](uint32_t j, bool gather = false) {
             const std::string t = P.r32();
             P.op("xor.b32 ", t, ", %tb, ", fold_swz(deposit(j, Ph.R), T) << 3);
-            P.op("add.s32 ", t, ", ", t, ", %cur");
+            if (plg && gather) {
+                const uint32_t v = deposit(j & qreg_mask, Ph.R) >> (T - 2);
+                P.op("add.s32 ", t, ", ", t, ", %pb", v);
+            } else {
+                P.op("add.s32 ", t, ", ", t, ", %cur");
+            }
             return t;
         };
         if (ph == 0 && pinit) {
@@ -851,21 +905,29 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 P.op("@%p_z mov.b64 %a0, 1065353216");  // (1.0f, 0.0f)
         } else if (Ph.b0) {
             for (int j = 0; j < NA / 2; ++j) {
-                const std::string a = saddr(2u * j);
+                const std::string a = saddr(2u * j, true);
                 P.op("ld.shared.v2.b64 {%a", 2 * j, ", %a", 2 * j + 1, "}, [", a, "]");
             }
         } else {
             for (int j = 0; j < NA; ++j) {
-                const std::string a = saddr((uint32_t)j);
+                const std::string a = saddr((uint32_t)j, true);
                 P.op("ld.shared.b64 %a", j, ", [", a, "]");
             }
+        }
+        if (plg) {
+            // every thread has read the spare buffer (and quarter 3 of the
+            // tile buffer, which this phase's scatter overwrites): quarters
+            // 0..2 of the next tile land during the rest of this tile
+            P.op("bar.sync 0");
+            loadtile("%gnext", "@%p_next ", "%cur", 7u);
+            P.op("cp.async.commit_group");
         }
         if (ring && last && direct) {
             release();
         } else if (last && early) {
             // tile buffer free: the next tile's load overlaps this phase's gates
-            P.op("bar.sync 0");
-            loadtile("%gnext", "@%p_next ");
+            if (!plg) P.op("bar.sync 0");
+            loadtile("%gnext", "@%p_next ", "%cur", pl ? 8u : 15u);
             P.op("cp.async.commit_group");
         }
         for (int g : Ph.gates) {
@@ -990,7 +1052,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             release();
         } else if (!zinit) {
             P.op("bar.sync 0");  // every thread is done with the tile buffer
-            loadtile("%gnext", "@%p_next ");
+            loadtile("%gnext", "@%p_next ", "%cur", pl ? 8u : 15u);
             P.op("cp.async.commit_group");
         }
         for (int i = 0; i < UPT; ++i)
@@ -1035,13 +1097,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << "// T=" << T << " r=" << pd.r << " n=" << n_local << " S={";
     for (int q : pd.S) k << q << ",";
     k << "} gates " << g0 << ".." << g1 << " phases " << nph << (zinit ? " zinit" : "") << (pinit ? " product-start" : "")
-      << (direct ? " direct" : "") << (bins ? " bins" : "") << (ring ? " ring" : "") << "\n";
+      << (direct ? " direct" : "") << (bins ? " bins" : "") << (ring ? " ring" : "") << (pl ? " prelanded" : "") << "\n";
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
     k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg " << (M == 5 ? 128 : 64) << "\n{\n";
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw, %p_w;\n";
-    k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par, %alt;\n\t.reg .b64 %rdk;\n";
+    k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par, %alt, %spr, %qt, %pb<4>;\n\t.reg .b64 %rdk;\n";
     k << "\t.reg .f64 %dre, %dim, %dp;\n\t.reg .b64 %w, %wt, %bo, %bins;\n\t.reg .b32 %wl, %wh, %wl2, %wh2;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
@@ -1086,29 +1148,54 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
     const bool direct = lp.lanes.size() >= 3 && lp.lanes[0] == 0 && lp.lanes[1] == 1 && lp.lanes[2] == 2;
     const bool early = direct && !zinit;
     mats.clear();
+    // structured one-qubit gates (R11) as in gen_chunk: fp64 additions on
+    // (re, im) register pairs, complex multipliers (s re, s im) per slot
+    const ChunkSpec cs = chunk_spec(pd, g0, g1, zinit);
+    auto put_s = [&](cd z) {
+        mats.push_back(z.real());
+        mats.push_back(z.imag());
+    };
     std::vector<size_t> gbase(pd.gates.size(), 0);
     for (int ph = 0; ph < nph; ++ph)
         for (int g : phs[ph].gates) {
             const PassGate& pg = pd.gates[g];
             const int kind = gate_kind(pd, pg);
+            const GSpec& x = cs.g[g];
+            gbase[g] = mats.size() / 2;
+            if (x.cls == 2) {
+                put_s(x.mu);
+                continue;
+            }
+            if (x.cls) {
+                for (int r = 0; r < 2; ++r)
+                    if (!x.unit[r]) put_s(x.s[r]);
+                continue;
+            }
             if (kind == 2) continue;
             const int D = 1 << pg.k;
             const double* mg = pd.mats64.data() + pg.moff;
-            gbase[g] = mats.size() / 2;
+            const cd f = cs.mode == 2 && g == cs.fold ? cs.C : cd(1.0);
             const int ne = kind == 1 ? D : D * D;
             for (int e = 0; e < ne; ++e) {
                 const int src = kind == 1 ? e * D + e : e;
-                mats.push_back(mg[2 * src]);
-                mats.push_back(mg[2 * src + 1]);
+                put_s(cd(mg[2 * src], mg[2 * src + 1]) * f);
             }
         }
+    size_t cslot = 0;
+    if (cs.mode == 1 && pd.pinit_v.empty()) {  // the start amplitude
+        cslot = mats.size() / 2;
+        put_s(cs.C);
+    } else if (cs.mode == 4) {
+        cslot = mats.size() / 2;
+        put_s(cs.C);
+    }
     const bool pinit = zinit && !pd.pinit_v.empty();
     size_t reg0 = 0, lane0 = 0;
     if (pinit) {
         const RpPhaseHost& P0 = phs[0];
         reg0 = mats.size() / 2;
         for (uint32_t j = 0; j < NA; ++j) {
-            std::complex<double> z = 1.0;
+            std::complex<double> z = cs.mode == 1 ? cs.C : cd(1.0);
             for (int b = 0; b < M; ++b) z *= pd.pinit_v[2 * P0.R[b] + ((j >> b) & 1u)];
             mats.push_back(z.real());
             mats.push_back(z.imag());
@@ -1147,6 +1234,88 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
         P.op("neg.f64 %t2, ", ai);
         P.op("fma.rn.f64 ", orr, ", %t2, ", bi, ", %t0");
         P.op("fma.rn.f64 ", oi, ", ", ai, ", ", br, ", %t1");
+    };
+    // ---- structured gates (GSpec) on (re, im) pairs: i^k (x + i y) is a
+    // choice of components and signs, so out = i^q (a0 + i^p a1) is two
+    // DADDs; a multiplier s t is a complex multiply (2 DMUL + 2 DFMA)
+    struct SV {  // signed component references of a complex value
+        std::string r, i;
+        bool nr, ni;
+    };
+    auto rotv = [](const std::string& xr, const std::string& xi, int k) -> SV {
+        switch (k & 3) {
+            case 0: return {xr, xi, false, false};
+            case 1: return {xi, xr, true, false};   // i (x + i y) = -y + i x
+            case 2: return {xr, xi, true, true};
+            default: return {xi, xr, false, true};  // -i (x + i y) = y - i x
+        }
+    };
+    auto sadd = [&](const std::string& d, const std::string& a, bool na, const std::string& b, bool nb) {
+        if (!na && !nb) {
+            P.op("add.rn.f64 ", d, ", ", a, ", ", b);
+        } else if (!na) {
+            P.op("sub.rn.f64 ", d, ", ", a, ", ", b);
+        } else if (!nb) {
+            P.op("sub.rn.f64 ", d, ", ", b, ", ", a);
+        } else {
+            P.op("neg.f64 %t2, ", a);
+            P.op("sub.rn.f64 ", d, ", %t2, ", b);
+        }
+    };
+    auto vadd = [&](const std::string& dr, const std::string& di, const SV& u, const SV& v) {
+        sadd(dr, u.r, u.nr, v.r, v.nr);
+        sadd(di, u.i, u.ni, v.i, v.ni);
+    };
+    auto smul = [&](const std::string& dr, const std::string& di, const std::string& tr, const std::string& ti,
+                    size_t slot) {  // (dr, di) = s (tr, ti); d may alias t
+        P.op("ld.param.v2.f64 {%mr, %mi}, [rpj_param_0+", 16 * slot, "]");
+        cmul("%mr", "%mi", tr, ti, "%zr", "%zi");
+        P.op("mov.f64 ", dr, ", %zr");
+        P.op("mov.f64 ", di, ", %zi");
+    };
+    auto emit_spec64 = [&](const GSpec& x, uint32_t mask, size_t base) {
+        size_t sl[2] = {base, base};
+        if (!x.unit[0]) sl[1] = base + 1;
+        auto AR = [](uint32_t j) { return "%ar" + std::to_string(j); };
+        auto AI = [](uint32_t j) { return "%ai" + std::to_string(j); };
+        if (x.cls == 3) {
+            for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
+                const int r = (j & mask) ? 1 : 0;
+                if (!x.unit[r]) {
+                    smul(AR(j), AI(j), AR(j), AI(j), sl[r]);
+                } else if (x.q[r] & 3) {
+                    const SV v = rotv(AR(j), AI(j), x.q[r]);
+                    P.op(v.nr ? "neg.f64 %zr, " : "mov.f64 %zr, ", v.r);
+                    P.op(v.ni ? "neg.f64 %zi, " : "mov.f64 %zi, ", v.i);
+                    P.op("mov.f64 ", AR(j), ", %zr");
+                    P.op("mov.f64 ", AI(j), ", %zi");
+                }
+            }
+            return;
+        }
+        for (uint32_t j0 = 0; j0 < (uint32_t)NA; ++j0) {
+            if (j0 & mask) continue;
+            const uint32_t j1 = j0 | mask;
+            if (x.cls == 2) {  // out0 = a0 + mu a1, out1 = i^p0 a0 + i^p1 (mu a1)
+                smul("%ptr", "%pti", AR(j1), AI(j1), sl[0]);
+                vadd("%por0", "%poi0", rotv(AR(j0), AI(j0), 0), rotv("%ptr", "%pti", 0));
+                vadd("%por1", "%poi1", rotv(AR(j0), AI(j0), x.p[0]), rotv("%ptr", "%pti", x.p[1]));
+            } else {  // row form: out_r = s_r (a0 + i^p_r a1)
+                for (int r = 0; r < 2; ++r) {
+                    const std::string dr = "%por" + std::to_string(r), di = "%poi" + std::to_string(r);
+                    if (x.unit[r]) {
+                        vadd(dr, di, rotv(AR(j0), AI(j0), x.q[r]), rotv(AR(j1), AI(j1), x.p[r] + x.q[r]));
+                    } else {
+                        vadd("%ptr", "%pti", rotv(AR(j0), AI(j0), 0), rotv(AR(j1), AI(j1), x.p[r]));
+                        smul(dr, di, "%ptr", "%pti", sl[r]);
+                    }
+                }
+            }
+            P.op("mov.f64 ", AR(j0), ", %por0");
+            P.op("mov.f64 ", AI(j0), ", %poi0");
+            P.op("mov.f64 ", AR(j1), ", %por1");
+            P.op("mov.f64 ", AI(j1), ", %poi1");
+        }
     };
     if (pinit) {
         P.op("mov.f64 %tfr, 0d3FF0000000000000");
@@ -1247,7 +1416,10 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
             P.op("setp.ne.u32 %p_z, %zone, 0");
             P.op("setp.eq.and.u64 %p_z, %u, 0, %p_z");
             P.op("setp.eq.and.u32 %p_z, %t_id, 0, %p_z");
-            P.op("@%p_z mov.f64 %ar0, 0d3FF0000000000000");
+            if (cs.mode == 1 && !pinit)  // the pass scalar C as the start amplitude
+                P.op("@%p_z ld.param.v2.f64 {%ar0, %ai0}, [rpj_param_0+", 16 * cslot, "]");
+            else
+                P.op("@%p_z mov.f64 %ar0, 0d3FF0000000000000");
         } else {
             for (int j = 0; j < NA; ++j) {
                 const std::string a = saddr((uint32_t)j);
@@ -1269,7 +1441,12 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
                 else tmask |= 1u << (int)(std::find(Ph.lanes.begin(), Ph.lanes.end(), pg.pos[b]) - Ph.lanes.begin());
             }
             const int D = 1 << pg.k;
-            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask << "\n";
+            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask
+                << " cls=" << cs.g[g].cls << "\n";
+            if (cs.g[g].cls) {
+                emit_spec64(cs.g[g], mask, gbase[g]);
+                continue;
+            }
             if (kind == 2) {
                 std::string pred;
                 if (popc(mask) != 2) {
@@ -1331,6 +1508,8 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
                 }
             }
         }
+        if (last && cs.mode == 4)  // the pass scalar, explicitly
+            for (int j = 0; j < NA; ++j) smul(ar(j), ai(j), ar(j), ai(j), cslot);
         if (last && direct) {
             P.op("add.s64 %gst, %gtile, %dg");
             for (int j = 0; j < NA; ++j)
@@ -1379,7 +1558,8 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
-    k << "\t.reg .f64 %ar<16>, %ai<16>, %xr<4>, %xi<4>, %yr, %yi, %mr, %mi, %nmi, %t0, %t1, %t2, %tfr, %tfi;\n";
+    k << "\t.reg .f64 %ar<16>, %ai<16>, %xr<4>, %xi<4>, %yr, %yi, %mr, %mi, %nmi, %t0, %t1, %t2, %tfr, %tfi, %zr, %zi, "
+         "%ptr, %pti, %por<2>, %poi<2>;\n";
     k << "\t.reg .b64 %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, %gnext, %gst, "
          "%tabA, %tabB, %rdB;\n";
     k << P.o.str();
@@ -1502,7 +1682,9 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
                 const bool ring = SVB_JIT_RING && !pd.wide;
                 l.kern->nthr = (1 << (T - M)) * (ring ? 2 : 1);
                 const bool db = SVB_JIT_DB && !ring && !z && !pd.wide;  // as gen_chunk
-                l.kern->smem = ((size_t)(pd.wide ? 16 : 8) << T) * (ring ? 3 : db ? 2 : 1) + (ring ? 64 : 0);
+                const bool pl = SVB_JIT_PL && !ring && !db && !z && !pd.wide && M >= 3;
+                l.kern->smem = ((size_t)(pd.wide ? 16 : 8) << T) * (ring ? 3 : db ? 2 : 1) + (ring ? 64 : 0) +
+                               (pl ? ((size_t)6 << T) : 0);  // 3/4 tile spare buffer
                 l.kern->T = T;
                 l.kern->nm = nm;
                 l.kern->param_bytes = std::max<size_t>(nm, 1) * 16 + 48;  // as in gen_chunk
@@ -1605,10 +1787,10 @@ void rpass_jit_counters(uint64_t* compiled, uint64_t* cache_hits, double* compil
 }
 
 uint64_t rpass_jit_ops_per_amp(const PassDesc& pd, bool zinit) {
-    if (!pd.spec || pd.wide) return rpass_fma_per_amp(pd);
+    if (!pd.spec) return rpass_fma_per_amp(pd);
     uint64_t f = 0;
     bool first = true;
-    for (const auto& ch : rpass_chunks(pd, SVB_JIT_M, false)) {
+    for (const auto& ch : rpass_chunks(pd, pd.wide ? 4 : SVB_JIT_M, pd.wide)) {
         const ChunkSpec cs = chunk_spec(pd, ch.first, ch.second, zinit && first);
         for (size_t g = ch.first; g < ch.second; ++g) {
             const GSpec& x = cs.g[g];

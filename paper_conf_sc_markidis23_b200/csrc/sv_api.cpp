@@ -1295,12 +1295,14 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
     // each maximal run of APPLY events between exchanges is cut into passes
     // by build_passes (reading R7); exchanges and permutations stay as they are.
     // complex128 states: pass-specialised fp64 kernels (16 amplitudes per
-    // thread, auto tile 12 qubits = 64 KB) for max_fused <= 2.
+    // thread) for max_fused <= 2.
     // auto tile: 14 qubits for the complex64 pass kernels (512 threads, 128 KB;
     // 30q D14 F=1 24.7 ms vs 26.1 at 13, 32q D20 145 vs 166 ms: fewer passes
-    // for the same runs), 13 for the generic kernel, 12 for complex128
+    // for the same runs), 13 for the generic kernel, 13 for complex128 (512
+    // threads, 128 KB; with the structured gates 30q D14 F=1 57.6 ms, 7
+    // passes, vs 61.6 ms, 9 passes, at 12)
     int T = s->block_bits >= 0 ? s->block_bits
-                               : (max_fused <= 2 && s->l >= 20 ? (s->fp64 ? 12 : s->pass_jit ? 14 : 13) : 0);
+                               : (max_fused <= 2 && s->l >= 20 ? (s->fp64 ? 13 : s->pass_jit ? 14 : 13) : 0);
     if (T == 14 && (s->fp64 || !s->pass_jit || max_fused > 2)) T = 13;  // 14-qubit tiles: complex64 pass kernels only
     const bool blocked = (!s->fp64 || (s->pass_jit && max_fused <= 2)) && T >= 10 && s->l >= T + 2 &&
                          s->n > kSmallCircuitMaxQubits && max_fused <= 4 && max_fused >= 1;
@@ -1375,7 +1377,7 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
         if (run.empty()) return;
         for (auto& pd : build_passes(T, run, s->pass_pin)) {
             pd.wide = s->fp64;
-            pd.spec = s->pass_spec && s->pass_jit && !s->fp64 && pd.mats_shard.empty();
+            pd.spec = s->pass_spec && s->pass_jit && pd.mats_shard.empty();
             pd.fma_per_amp = rpass_supported(pd) ? pass_ops(pd, false) : 0;
             c->stats.fma_apply += pd.fma_per_amp << s->l;
             c->stats.n_passes++;
@@ -1474,7 +1476,7 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
             c->stats_z.fma_apply = 0;
             for (auto& pd : pz) {
                 pd.wide = s->fp64;
-                pd.spec = s->pass_spec && !s->fp64 && pd.mats_shard.empty();
+                pd.spec = s->pass_spec && s->pass_jit && pd.mats_shard.empty();
                 pd.fma_per_amp = rpass_supported(pd) ? pass_ops(pd, &pd == &pz[0]) : 0;
                 c->stats_z.fma_apply += pd.fma_per_amp << s->l;
                 c->stats_z.n_passes++;
@@ -2250,7 +2252,7 @@ int sv_pass_kernels(const sv_gate* gates, size_t n_gates, int max_fused, int til
         passes.back().bins = true;  // as sv_circuit_create
     for (auto& pd : passes) {
         pd.wide = wide;
-        pd.spec = !wide;  // as sv_circuit_create with the default SV_OPT_PASS_SPEC
+        pd.spec = true;  // as sv_circuit_create with the default SV_OPT_PASS_SPEC
         if (!rpass_supported(pd)) continue;
         for (int z = 0; z < (first ? 2 : 1); ++z) {
             std::vector<RpJitLaunch> ls;

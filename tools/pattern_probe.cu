@@ -38,7 +38,7 @@ __device__ __forceinline__ float4 ld256(const float4* p) {
 // prefetch-size hint; 2: each CTA takes 2 consecutive tiles back to back
 // (L2::256B); 3: 4 consecutive tiles (L2::256B)
 template <int UPT, int mode>
-__global__ void __launch_bounds__(256) probe(float4* psi, unsigned long long ntiles, int r) {
+__global__ void __launch_bounds__(512) probe(float4* psi, unsigned long long ntiles, int r) {
     // unit = 16 B = 2 amplitudes; tile = 256 threads * UPT units
     constexpr int gsh = mode == 2 ? 1 : mode == 3 ? 2 : 0;
     int lg = 0;
@@ -59,7 +59,7 @@ __global__ void __launch_bounds__(256) probe(float4* psi, unsigned long long nti
         float4 v[UPT];
 #pragma unroll
         for (int i = 0; i < UPT; ++i) {
-            const unsigned t = 2u * (threadIdx.x + 256u * i);  // tile index (amplitudes)
+            const unsigned t = 2u * (threadIdx.x + blockDim.x * i);  // tile index (amplitudes)
             unsigned long long g = t & ((1u << r) - 1u);
             const unsigned hi = t >> r;
             for (int b = 0; b < cm.nh; ++b)
@@ -69,7 +69,7 @@ __global__ void __launch_bounds__(256) probe(float4* psi, unsigned long long nti
         }
 #pragma unroll
         for (int i = 0; i < UPT; ++i) {
-            const unsigned t = 2u * (threadIdx.x + 256u * i);
+            const unsigned t = 2u * (threadIdx.x + blockDim.x * i);
             unsigned long long g = t & ((1u << r) - 1u);
             const unsigned hi = t >> r;
             for (int b = 0; b < cm.nh; ++b)
@@ -143,7 +143,7 @@ int main(int argc, char** argv) {
             for (int rep = 0; rep < 4; ++rep) {
                 cudaEventRecord(e0);
                 auto k = mode == 0 ? probe<16, 0> : mode == 1 ? probe<16, 4> : mode == 2 ? probe<16, 5> : probe<16, 1>;
-                k<<<sms * occ, 256>>>(psi, ntiles, r);
+                k<<<sms * (T >= 14 ? 1 : occ), 1u << (T - 5)>>>(psi, ntiles, r);
                 cudaEventRecord(e1);
                 cudaEventSynchronize(e1);
                 float ms; cudaEventElapsedTime(&ms, e0, e1);
