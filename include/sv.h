@@ -130,7 +130,7 @@ typedef struct {
     size_t buf_bytes;        /* size of dev_buf: >= 8 * 2^n / (world if multi-process)    */
     void* cuda_stream;       /* optional cudaStream_t; NULL = library-owned stream        */
     int32_t precision;       /* 0: complex64 (fp32, default); 1: complex128 (fp64, NEXT-1;
-                                PAPER.md L191 Fig. 8) -- single shard, fused k <= 5      */
+                                PAPER.md L191 Fig. 8) -- sharded as complex64, fused k <= 6 */
     int32_t reserved_;
 } sv_config;
 

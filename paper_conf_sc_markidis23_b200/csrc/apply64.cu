@@ -12,7 +12,11 @@
 // memory (per-gate XOR swizzle of amplitude bits 0..2 keeps the 8-lane LDS.128
 // phases conflict-free), transformed with the Gauss 3-multiplication form in
 // fp64 and scattered back.  Matrix planes travel in the kernel parameters.
-// k <= 5 (a k = 6 group would need 256 registers of fp64 inputs).
+// k = 6 (apply64_k6_kernel): a group's 64 inputs do not fit in registers, so
+// the 8 warps of a CTA split the 64 output rows (8 each) of the 32 groups of
+// a 2^11-amplitude tile (lane = group), read the inputs from the shared-memory
+// tile and the (transposed) planes from shared memory (warp-wide broadcasts),
+// and write the outputs to a second tile buffer that is then stored.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -169,6 +173,74 @@ __global__ void __launch_bounds__(256) apply64_kernel(const __grid_constant__ Ti
     }
 }
 
+__global__ void __launch_bounds__(256) apply64_k6_kernel(const __grid_constant__ Tile64Params<6> p) {
+    extern __shared__ double2 dsm64[];
+    const uint32_t tile_bytes = 16u << p.T;
+    const uint32_t s_in = smem_addr(dsm64), s_out = s_in + tile_bytes;
+    // planes transposed: pl[(plane * 64 + c) * 64 + r]
+    double* pl = reinterpret_cast<double*>(reinterpret_cast<char*>(dsm64) + 2 * tile_bytes);
+    for (int i = threadIdx.x; i < 3 * 4096; i += blockDim.x) {
+        const int plane = i >> 12, r = (i >> 6) & 63, c = i & 63;
+        pl[(plane * 64 + c) * 64 + r] = p.M.dev[i];
+    }
+    __syncthreads();
+    const uint32_t t0 = threadIdx.x;
+    const uint32_t rmask = (1u << p.r) - 1u;
+    uint64_t dthr = t0 & rmask;
+    {
+        const uint32_t h = t0 >> p.r;
+        for (int b = 0; b < p.nH; ++b)
+            if ((h >> b) & 1u) dthr += 1ull << p.Hpos[b];
+    }
+    const uint32_t sthr = swz64(t0, p.swz);
+    const uint32_t g = threadIdx.x & 31u, r0 = (threadIdx.x >> 5) * 8u;  // lane = group, warp = 8 rows
+    const uint32_t pb = swz64((uint32_t)insert_zeros(g, p.ztpos, p.nzt), p.swz);
+    uint64_t u = blockIdx.x;
+    if (u < p.n_tiles) {
+        const double2* gp = p.psi + insert_zeros(u << p.r, p.Hpos, p.nH) + dthr;
+        for (int i = 0; i < p.upt; ++i) cp_async16(s_in + ((sthr ^ p.soff[i]) << 4), gp + p.goff[i]);
+    }
+    cp_async_commit();
+    for (; u < p.n_tiles; u += gridDim.x) {
+        cp_async_wait0();
+        __syncthreads();
+        double A[8], B[8], C[8];
+#pragma unroll
+        for (int rr = 0; rr < 8; ++rr) A[rr] = B[rr] = C[rr] = 0.0;
+#pragma unroll 2
+        for (int c = 0; c < 64; ++c) {
+            const double2 a = ldsd(s_in + ((pb ^ p.loc[c]) << 4));
+            const double sc = a.x + a.y;
+            const double2* P = reinterpret_cast<const double2*>(pl + (0 * 64 + c) * 64 + r0);
+            const double2* S = reinterpret_cast<const double2*>(pl + (1 * 64 + c) * 64 + r0);
+            const double2* Q = reinterpret_cast<const double2*>(pl + (2 * 64 + c) * 64 + r0);
+#pragma unroll
+            for (int h = 0; h < 4; ++h) {
+                const double2 pp = P[h], ss = S[h], qq = Q[h];
+                A[2 * h] = fma(pp.x, sc, A[2 * h]);
+                A[2 * h + 1] = fma(pp.y, sc, A[2 * h + 1]);
+                B[2 * h] = fma(ss.x, a.y, B[2 * h]);
+                B[2 * h + 1] = fma(ss.y, a.y, B[2 * h + 1]);
+                C[2 * h] = fma(qq.x, a.x, C[2 * h]);
+                C[2 * h + 1] = fma(qq.y, a.x, C[2 * h + 1]);
+            }
+        }
+#pragma unroll
+        for (int rr = 0; rr < 8; ++rr)
+            stsd(s_out + ((pb ^ p.loc[r0 + rr]) << 4), make_double2(A[rr] - B[rr], A[rr] + C[rr]));
+        __syncthreads();  // the input tile is free, the output tile complete
+        const uint64_t un = u + gridDim.x;
+        if (un < p.n_tiles) {
+            const double2* gp = p.psi + insert_zeros(un << p.r, p.Hpos, p.nH) + dthr;
+            for (int i = 0; i < p.upt; ++i) cp_async16(s_in + ((sthr ^ p.soff[i]) << 4), gp + p.goff[i]);
+        }
+        cp_async_commit();
+        double2* gs = p.psi + insert_zeros(u << p.r, p.Hpos, p.nH) + dthr;
+        for (int i = 0; i < p.upt; ++i) stgd(gs + p.goff[i], ldsd(s_out + ((sthr ^ p.soff[i]) << 4)));
+    }
+    cp_async_wait0();
+}
+
 // Tiny states: one thread per group, direct global accesses.
 __global__ void apply64_small_kernel(double2* psi, int n, int k, const int* q_dev, const double* planes) {
     const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -177,8 +249,8 @@ __global__ void apply64_small_kernel(double2* psi, int n, int k, const int* q_de
     int q[SV_MAX_FUSED];
     for (int b = 0; b < k; ++b) q[b] = q_dev[b];
     const uint64_t base = insert_zeros(g, q, k);
-    double2 a[32];
-    uint64_t off[32];
+    double2 a[64];
+    uint64_t off[64];
     for (int c = 0; c < D; ++c) {
         uint64_t o = 0;
         for (int b = 0; b < k; ++b)
@@ -186,7 +258,7 @@ __global__ void apply64_small_kernel(double2* psi, int n, int k, const int* q_de
         off[c] = base | o;
         a[c] = psi[off[c]];
     }
-    double2 y[32];
+    double2 y[64];
     for (int r = 0; r < D; ++r) {
         double A = 0.0, B = 0.0, C = 0.0;
         for (int c = 0; c < D; ++c) {
@@ -282,21 +354,30 @@ cudaError_t launch64_k(double2* psi, int n, const Apply64Desc& d, cudaStream_t s
     }
     const uint32_t units = 1u << p.T;
     const uint32_t ngroups = 1u << (p.T - K);
-    const uint32_t nthr = std::min<uint32_t>(256, ngroups);
-    if (nthr < 32 || units / nthr > 64) return cudaErrorNotSupported;  // caller uses the small kernel
+    // k = 6: 256 threads (8 warps x 8 output rows, lane = group) on 32 groups
+    const uint32_t nthr = K == 6 ? 256u : std::min<uint32_t>(256, ngroups);
+    if (K == 6 ? ngroups != 32 : (nthr < 32 || units / nthr > 64)) return cudaErrorNotSupported;  // small kernel
     p.upt = (int)(units / nthr);
     for (int i = 0; i < p.upt; ++i) {
         p.goff[i] = dep((uint64_t)nthr * i);
         p.soff[i] = sw(nthr * (uint32_t)i);
     }
     p.n_tiles = 1ull << (n - p.T);
-    const int stages = (K == 6) ? 1 : 2;
-    size_t smem = (size_t)stages * ((size_t)16 << p.T) + (K == 6 ? 3 * 4096 * 8 : 0);
-    cudaError_t e = cudaFuncSetAttribute(apply64_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    // two tile buffers: double-buffered input (k <= 5) or input + output (k = 6)
+    size_t smem = 2 * ((size_t)16 << p.T) + (K == 6 ? 3 * 4096 * 8 : 0);
+    const void* kern = nullptr;
+    if constexpr (K == 6)
+        kern = (const void*)apply64_k6_kernel;
+    else
+        kern = (const void*)apply64_kernel<K>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     const int per_sm = std::max(1, (int)((227 * 1024) / (smem + 1024)));
     const uint64_t grid = std::min<uint64_t>(p.n_tiles, (uint64_t)sms64() * per_sm);
-    apply64_kernel<K><<<(unsigned)grid, nthr, smem, st>>>(p);
+    if constexpr (K == 6)
+        apply64_k6_kernel<<<(unsigned)grid, nthr, smem, st>>>(p);
+    else
+        apply64_kernel<K><<<(unsigned)grid, nthr, smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -304,6 +385,22 @@ __global__ void reset64_kernel(double2* psi, uint64_t n, int one) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
         psi[i] = make_double2((one && i == 0) ? 1.0 : 0.0, 0.0);
+}
+
+// exact in-place swap of local index bits a < b (pure moves): the element
+// with bit a = 1, bit b = 0 trades places with its partner (a = 0, b = 1)
+__global__ void swap_bits64_kernel(double2* psi, uint64_t n_pairs, int a, int b) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < n_pairs; w += stride) {
+        // insert a 0 at a and at b, then set bit a
+        uint64_t i = w;
+        i = ((i >> a) << (a + 1)) | (i & ((1ull << a) - 1ull));
+        i = ((i >> b) << (b + 1)) | (i & ((1ull << b) - 1ull));
+        const uint64_t x = i | (1ull << a), y = i | (1ull << b);
+        const double2 vx = psi[x], vy = psi[y];
+        psi[x] = vy;
+        psi[y] = vx;
+    }
 }
 
 __global__ void gather64_kernel(const double2* psi, const uint64_t* phys, uint64_t count, double2* out) {
@@ -330,6 +427,10 @@ cudaError_t launch_apply64(double2* psi, int n, const Apply64Desc& d, cudaStream
         case 3: e = launch64_k<3>(psi, n, d, st); break;
         case 4: e = launch64_k<4>(psi, n, d, st); break;
         case 5: e = launch64_k<5>(psi, n, d, st); break;
+        case 6:
+            if (!d.dev_planes) return cudaErrorInvalidValue;
+            e = launch64_k<6>(psi, n, d, st);
+            break;
     }
     if (e != cudaErrorNotSupported) return e;
     // small states: per-group kernel with planes and qubits in device scratch
@@ -343,6 +444,15 @@ cudaError_t launch_apply64(double2* psi, int n, const Apply64Desc& d, cudaStream
 cudaError_t launch_reset64(double2* psi, uint64_t n_amps, bool one, cudaStream_t st) {
     const uint64_t blocks = std::min<uint64_t>((n_amps + 255) / 256, (uint64_t)sms64() * 16);
     reset64_kernel<<<(unsigned)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(psi, n_amps, one ? 1 : 0);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_swap_bits64(double2* psi, int l, int a, int b, cudaStream_t st) {
+    if (a == b) return cudaSuccess;
+    if (a > b) std::swap(a, b);
+    const uint64_t n_pairs = 1ull << (l - 2);
+    const uint64_t blocks = std::min<uint64_t>((n_pairs + 255) / 256, (uint64_t)sms64() * 16);
+    swap_bits64_kernel<<<(unsigned)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(psi, n_pairs, a, b);
     return cudaGetLastError();
 }
 

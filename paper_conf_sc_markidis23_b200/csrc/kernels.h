@@ -61,6 +61,8 @@ void pack_planes64(const Apply64Desc& d, double* out);  // 3 * 4^k doubles
 cudaError_t launch_apply64(double2* psi, int n, const Apply64Desc& d, cudaStream_t st);
 cudaError_t launch_reset64(double2* psi, uint64_t n_amps, bool one, cudaStream_t st);
 cudaError_t launch_gather64(const double2* psi, const uint64_t* phys, uint64_t count, double2* out, cudaStream_t st);
+// exact in-place swap of local index bits a and b of a complex128 shard (2^l amplitudes)
+cudaError_t launch_swap_bits64(double2* psi, int l, int a, int b, cudaStream_t st);
 
 // Whole circuit in one CTA with the state in shared memory (n <= 13).
 constexpr int kSmallCircuitMaxQubits = 13;

@@ -38,6 +38,12 @@
 #ifndef SVB_JIT_M
 #define SVB_JIT_M 5  // log2 amplitudes per thread of the complex64 pass kernels (4: 16 per thread, 64 registers)
 #endif
+#ifndef SVB_JIT_M14
+#define SVB_JIT_M14 6  // ... for 14-qubit tiles: 64 per thread (256 threads, <= 255 registers, 8 warps per SM)
+#endif
+#ifndef SVB_JIT_M14_RUN
+#define SVB_JIT_M14_RUN 4  // ... when the tile's runs are >= 2^this amplitudes
+#endif
 #ifndef SVB_JIT_RING
 #define SVB_JIT_RING 0  // two warp groups over three tile buffers per CTA (loads 1.5 tiles ahead)
 #endif
@@ -72,6 +78,21 @@ struct RpJitKernel {
 };
 
 namespace {
+// log2 amplitudes per thread of a pass kernel: 16 (complex128); 64 for
+// 14-qubit complex64 tiles without dense two-qubit gates (fewer phases per
+// pass: 30q D14 24.8 -> 23.7 ms; with dense 4 x 4 matvecs, e.g. fSim, the
+// 8 warps of such a CTA stall on the FFMA2 chains: Sycamore 30q 0.114 ->
+// 0.156 s); else 32 (the generic kernel's, so the two stay bit-identical)
+// The 64-amplitude form only for tiles of runs >= 2^SVB_JIT_M14_RUN
+// amplitudes (A/B, round 2: 30q D14 with 128 B runs 24.8 -> 23.7 ms; 32q
+// D20 with 64 B runs 137.5 -> 142.5 ms, with 128 B runs unchanged)
+int jit_m(const PassDesc& pd) {
+    if (pd.wide) return 4;
+    if (pd.S.size() < 14 || pd.r < SVB_JIT_M14_RUN) return SVB_JIT_M;
+    for (const auto& g : pd.gates)
+        if (g.k == 2 && gate_kind(pd, g) == 0) return SVB_JIT_M;
+    return SVB_JIT_M14;
+}
 
 std::mutex g_cache_mu;
 std::map<std::string, std::shared_ptr<RpJitKernel>> g_cache;
@@ -297,6 +318,7 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         k += ',';
     };
     if (pd.wide) k += "w,";
+    put(jit_m(pd));
     put(n_local);
     put(pd.r);
     put(zinit ? 1 : 0);
@@ -328,7 +350,7 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
 std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
                       std::vector<float>& mats, bool emit = true, const std::vector<float>* msrc = nullptr) {
     const std::vector<float>& pmats = msrc ? *msrc : pd.mats;
-    constexpr int M = SVB_JIT_M, NA = 1 << M, UPT = 1 << (M - 1);
+    const int M = jit_m(pd), NA = 1 << M, UPT = 1 << (M - 1);
     const int T = (int)pd.S.size();
     const int tbits = T - M;
     const uint32_t nthr = 1u << tbits;
@@ -1101,13 +1123,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
-    k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg " << (M == 5 ? 128 : 64) << "\n{\n";
+    k << ".maxntid " << (ring ? 2 * nthr : nthr) << ", 1, 1\n.maxnreg " << (M >= 6 ? 255 : M == 5 ? 128 : 64) << "\n{\n";
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z, %p_bw, %p_w;\n";
     k << "\t.reg .b32 %rsm0, %grp, %bid, %mb0, %fb, %kk, %bb, %par, %alt, %spr, %qt, %pb<4>;\n\t.reg .b64 %rdk;\n";
     k << "\t.reg .f64 %dre, %dim, %dp;\n\t.reg .b64 %w, %wt, %bo, %bins;\n\t.reg .b32 %wl, %wh, %wl2, %wh2;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %lo, %hi, %nhi, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
-    k << "\t.reg .b64 %a<32>;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
+    k << "\t.reg .b64 %a<" << NA << ">;\n\t.reg .b64 %x<4>;\n\t.reg .b64 %xs<4>;\n";
     k << "\t.reg .f32 %rlo, %rhi, %rnl, %rnh;\n\t.reg .b64 %rt<8>, %po0, %po1, %pt, %py, %qsr, %qsi, %pone, %mneg1, %csg;\n";
     k << "\t.reg .b64 %y, %ml, %mh, %zero, %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, "
          "%gnext, %gst, %tf, %tabA, %tabB, %rdA, %rdB;\n";
@@ -1627,7 +1649,7 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
         out.clear();
         const int T = (int)pd.S.size();
         bool first = true;
-        for (const auto& ch : rpass_chunks(pd, pd.wide ? 4 : SVB_JIT_M, pd.wide)) {
+        for (const auto& ch : rpass_chunks(pd, jit_m(pd), pd.wide)) {
             RpJitLaunch l;
             size_t nm = 0;
             const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats);
@@ -1659,7 +1681,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
     for (size_t i = 0; i < pds.size(); ++i) {
         const PassDesc& pd = *pds[i];
         const int T = (int)pd.S.size();
-        const int M = pd.wide ? 4 : SVB_JIT_M;
+        const int M = jit_m(pd);
         bool first = true;
         for (const auto& ch : rpass_chunks(pd, M, pd.wide)) {
             RpJitLaunch l;
@@ -1790,7 +1812,7 @@ uint64_t rpass_jit_ops_per_amp(const PassDesc& pd, bool zinit) {
     if (!pd.spec) return rpass_fma_per_amp(pd);
     uint64_t f = 0;
     bool first = true;
-    for (const auto& ch : rpass_chunks(pd, pd.wide ? 4 : SVB_JIT_M, pd.wide)) {
+    for (const auto& ch : rpass_chunks(pd, jit_m(pd), pd.wide)) {
         const ChunkSpec cs = chunk_spec(pd, ch.first, ch.second, zinit && first);
         for (size_t g = ch.first; g < ch.second; ++g) {
             const GSpec& x = cs.g[g];

@@ -171,7 +171,9 @@ struct sv_circuit {
         std::vector<RpJitLaunch> jit, jitz;   // pass-specialised kernels (jitz: first pass from |0...0>)
         ExchangeDesc exch;
         std::vector<ApplyDesc> perm_applies;  // PERMUTE lowered to SWAP passes
+        std::vector<int> perm;                // PERMUTE (complex128: exact bit swaps)
     };
+    bool a64 = false;  // complex128, one apply64 launch per fused gate (not register-blocked)
     std::vector<Step> steps;
     // the same circuit for runs that start from a pending |0...0>: the first
     // gate of every qubit (a one-qubit gate) folded into a product-state
@@ -341,8 +343,8 @@ std::vector<cd> shard_block(int k, const int* phys, const std::vector<cd>& M, in
 // PERMUTE (data at local bit b moves to bit perm[b]) as passes of disjoint
 // transpositions, <= 2 per pass (a 4-qubit permutation matrix carried in the
 // kernel parameters; the FMA chain of a 0/1 matrix is exact).
-void lower_permute(int l, const std::vector<int>& perm, std::vector<ApplyDesc>& out) {
-    // current[b] = which original bit's data sits at bit b; target: bit perm[b] holds original b
+// the bit swaps (in order) that move original bit b's data to bit perm[b]
+std::vector<std::pair<int, int>> permute_swaps(int l, const std::vector<int>& perm) {
     std::vector<int> where(l);  // where[orig] = current position of orig's data
     for (int b = 0; b < l; ++b) where[b] = b;
     std::vector<std::pair<int, int>> swaps;
@@ -359,6 +361,11 @@ void lower_permute(int l, const std::vector<int>& perm, std::vector<ApplyDesc>& 
         where[b] = dst;
         where[other] = cur;
     }
+    return swaps;
+}
+
+void lower_permute(int l, const std::vector<int>& perm, std::vector<ApplyDesc>& out) {
+    const std::vector<std::pair<int, int>> swaps = permute_swaps(l, perm);
     size_t i = 0;
     while (i < swaps.size()) {
         std::vector<std::pair<int, int>> pass;
@@ -425,14 +432,24 @@ int run_apply_shards(sv_state* s, const std::vector<ApplyDesc>& ds) {
     return SV_OK;
 }
 
-int run_exchange(sv_state* s, const ExchangeDesc& x) {
+int run_exchange(sv_state* s, const ExchangeDesc& x0) {
     Nvtx nv("sv.exchange");
+    // complex128 shards: the same chunk swap over 8 B units (an amplitude is
+    // units 2i, 2i + 1), i.e. every local and global position one higher
+    ExchangeDesc x = x0;
+    if (s->fp64) {
+        x.l += 1;
+        for (int j = 0; j < x.s; ++j) {
+            x.P[j] += 1;
+            x.p[j] += 1;
+        }
+    }
     int rc = barrier(s);
     if (rc) return rc;
     rc = launch(s, LaunchClass::EXCH,
                 [&] { return launch_exchange(s->shard_dev, s->world, s->virt ? -1 : s->rank, x, s->stream); });
     if (rc) return rc;
-    s->stats.bytes_exchange += (uint64_t)((1.0 - 1.0 / (1 << x.s)) * 8.0 * (double)(1ull << s->l));
+    s->stats.bytes_exchange += (uint64_t)((1.0 - 1.0 / (1 << x.s)) * (double)s->elem * (double)(1ull << s->l));
     s->stats.n_exchanges++;
     return barrier(s);
 }
@@ -460,6 +477,19 @@ ExchangeDesc make_exchange(int l, const std::vector<std::pair<int, int>>& pairs)
     return x;
 }
 
+// local qubit permutation of complex128 shards: exact bit swaps (moves only)
+int run_permute64(sv_state* s, const std::vector<int>& perm) {
+    for (const auto& sw : permute_swaps(s->l, perm))
+        for (int i = 0; i < s->local_shards(); ++i) {
+            const int d = s->virt ? i : s->rank;
+            int rc = launch(s, LaunchClass::OTHER, [&] {
+                return launch_swap_bits64(reinterpret_cast<double2*>(s->shard[d]), s->l, sw.first, sw.second, s->stream);
+            });
+            if (rc) return rc;
+        }
+    return SV_OK;
+}
+
 // Bring the state to a canonical map (local part identity) -- needed before
 // sampling / whole-state reads in sharded mode.
 int canonicalize(sv_state* s) {
@@ -472,6 +502,9 @@ int canonicalize(sv_state* s) {
             int rc = run_exchange(s, make_exchange(s->l, e.pairs));
             if (rc) return rc;
             apply_event_pairs(s, e.pairs);
+        } else if (e.type == Event::PERMUTE && s->fp64) {
+            int rc = run_permute64(s, e.perm);
+            if (rc) return rc;
         } else if (e.type == Event::PERMUTE) {
             std::vector<ApplyDesc> passes;
             lower_permute(s->l, e.perm, passes);
@@ -806,7 +839,6 @@ int sv_create_ex(const sv_config* cfg, sv_state** out) {
     if (!virt && (cfg->rank < 0 || cfg->rank >= world)) return fail(SV_EINVAL, "rank out of range");
     if (cfg->precision != 0 && cfg->precision != 1) return fail(SV_EINVAL, "precision must be 0 (complex64) or 1 (complex128)");
     const bool fp64 = cfg->precision == 1;
-    if (fp64 && world > 1) return fail(SV_EUNSUPPORTED, "complex128 states are single-shard in this version");
     const size_t shard_bytes = (size_t)(fp64 ? 16 : 8) << l;
     const size_t need_bytes = shard_bytes * (virt ? world : 1);
     if (cfg->dev_buf && cfg->buf_bytes < need_bytes) return fail(SV_EINVAL, "buf_bytes too small for the state");
@@ -951,39 +983,11 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
         mask |= 1ull << qubits[b];
     }
     if (s->g > 0 && k > s->l - 1) return fail(SV_EUNSUPPORTED, "gate wider than a shard allows");
-    if (s->fp64 && k > 5) return fail(SV_EUNSUPPORTED, "complex128 states support fused gates with k <= 5");
     rc = materialize(s);
     if (rc) return rc;
     s->bins_valid = false;
     std::vector<cd> M = Min;
     std::vector<int> q(qubits, qubits + k);
-    if (s->fp64) {
-        Apply64Desc d;
-        d.k = k;
-        std::vector<cd> Ms(M.size());
-        sort_matrix_qubits<cd>(k, q.data(), M.data(), d.q, Ms.data());
-        d.m = Ms;
-        std::vector<double> planes(3 * M.size());
-        pack_planes64(d, planes.data());
-        sv_state::StageSlot* sl = nullptr;
-        rc = stage_acquire(s, sl);
-        if (rc) return rc;
-        rc = stage_put(s, *sl, 0, planes.data(), planes.size() * sizeof(double));
-        if (rc == SV_OK) rc = stage_put(s, *sl, kStageQ, d.q, sizeof(int) * SV_MAX_FUSED);
-        if (rc) return rc;
-        d.dev_planes = reinterpret_cast<const double*>(sl->dev);
-        d.small_scratch = sl->dev + kStageQ;
-        rc = launch(s, LaunchClass::HIGH, [&] {
-            return launch_apply64(reinterpret_cast<double2*>(s->shard[0]), s->l, d, s->stream);
-        });
-        if (rc) return rc;
-        rc = stage_release(s, *sl);
-        if (rc) return rc;
-        s->stats.bytes_apply += 32ull << s->l;
-        s->stats.bytes_apply_high += 32ull << s->l;
-        s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
-        return SV_OK;
-    }
     // sharded: bring global qubits local (one S4 step for this gate alone)
     if (s->g > 0) {
         std::vector<std::vector<int>> fq(1, q);
@@ -999,6 +1003,36 @@ static int apply_matrix(sv_state* s, int k, const int32_t* qubits, const std::ve
     }
     std::vector<int> phys(k);
     for (int b = 0; b < k; ++b) phys[b] = s->pos[q[b]];
+    if (s->fp64) {
+        Apply64Desc d;
+        d.k = k;
+        std::vector<cd> Ms(M.size());
+        sort_matrix_qubits<cd>(k, phys.data(), M.data(), d.q, Ms.data());
+        d.m = Ms;
+        std::vector<double> planes(3 * M.size());
+        pack_planes64(d, planes.data());
+        sv_state::StageSlot* sl = nullptr;
+        rc = stage_acquire(s, sl);
+        if (rc) return rc;
+        rc = stage_put(s, *sl, 0, planes.data(), planes.size() * sizeof(double));
+        if (rc == SV_OK) rc = stage_put(s, *sl, kStageQ, d.q, sizeof(int) * SV_MAX_FUSED);
+        if (rc) return rc;
+        d.dev_planes = reinterpret_cast<const double*>(sl->dev);
+        d.small_scratch = sl->dev + kStageQ;
+        for (int i = 0; i < s->local_shards(); ++i) {
+            const int sh = s->virt ? i : s->rank;
+            rc = launch(s, LaunchClass::HIGH, [&] {
+                return launch_apply64(reinterpret_cast<double2*>(s->shard[sh]), s->l, d, s->stream);
+            });
+            if (rc) return rc;
+        }
+        rc = stage_release(s, *sl);
+        if (rc) return rc;
+        s->stats.bytes_apply += 32ull << s->l;
+        s->stats.bytes_apply_high += 32ull << s->l;
+        s->stats.flops_apply += (uint64_t)((8 << k) - 2) << s->l;
+        return SV_OK;
+    }
     ApplyDesc d;
     make_apply(s->l, k, phys.data(), M.data(), d, s->tc_mode);
     sv_state::StageSlot* sl = nullptr;
@@ -1275,7 +1309,6 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
     rc = validate_gates(gates, n_gates, s->n);
     if (rc) return rc;
     if (s->g > 0 && std::max(max_fused, 2) > s->l - 1) return fail(SV_EUNSUPPORTED, "fused gates wider than a shard allows");
-    if (s->fp64 && max_fused > 5) return fail(SV_EUNSUPPORTED, "complex128 states support max_fused <= 5");
     Nvtx nv("sv.circuit_create");
     std::unique_ptr<sv_circuit> c(new sv_circuit());
     c->owner = s;
@@ -1335,21 +1368,31 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
     const double t2 = now_s();
     c->stats.t_plan_s = t2 - t1;
     if (s->fp64 && !blocked) {
-        // complex128: one apply64 launch per fused gate; all planes and qubit
-        // lists uploaded once (row a4)
+        // complex128: one apply64 launch per fused gate (per local shard, on
+        // its physical positions) and the plan's exchanges; all planes and
+        // qubit lists uploaded once (row a4)
+        c->a64 = true;
         std::vector<double> planes;
         std::vector<int> qs;
         std::vector<size_t> poff;
         for (auto& e : ev) {
             sv_circuit::Step st;
-            st.type = Event::APPLY;
-            const FusedGate& f = plan[e.fused];
-            st.a64.k = f.k;
-            for (int b = 0; b < f.k; ++b) st.a64.q[b] = f.q[b];
-            st.a64.m = f.M;  // fp64, ascending qubits: no rounding to complex64
+            st.type = e.type;
             poff.push_back(planes.size());
-            planes.resize(planes.size() + 3 * f.M.size());
-            pack_planes64(st.a64, planes.data() + poff.back());
+            if (e.type == Event::EXCHANGE) {
+                st.exch = make_exchange(s->l, e.pairs);
+                c->stats.n_exchanges++;
+            } else if (e.type == Event::PERMUTE) {
+                st.perm = e.perm;
+            } else {
+                const FusedGate& f = plan[e.fused];
+                st.a64.k = f.k;
+                st.a64.m.resize(f.M.size());
+                // fp64, ascending physical qubits: no rounding to complex64
+                sort_matrix_qubits<cd>(f.k, e.phys, f.M.data(), st.a64.q, st.a64.m.data());
+                planes.resize(planes.size() + 3 * f.M.size());
+                pack_planes64(st.a64, planes.data() + poff.back());
+            }
             for (int b = 0; b < SV_MAX_FUSED; ++b) qs.push_back(st.a64.q[b]);
             c->steps.push_back(std::move(st));
         }
@@ -1437,6 +1480,8 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
         } else if (e.type == Event::EXCHANGE) {
             st.exch = make_exchange(s->l, e.pairs);
             c->stats.n_exchanges++;
+        } else if (s->fp64) {
+            st.perm = e.perm;
         } else {
             lower_permute(s->l, e.perm, st.perm_applies);
         }
@@ -1685,14 +1730,23 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
         s->pos = c->pos_out;
         return SV_OK;
     }
-    if (s->fp64 && !(steps.empty() || steps[0].block)) {
+    if (c->a64) {
         for (auto& st : c->steps) {
-            rc = launch(s, LaunchClass::HIGH, [&] {
-                return launch_apply64(reinterpret_cast<double2*>(s->shard[0]), s->l, st.a64, s->stream);
-            });
+            if (st.type == Event::EXCHANGE) {
+                rc = run_exchange(s, st.exch);
+            } else if (st.type == Event::PERMUTE) {
+                rc = run_permute64(s, st.perm);
+            } else {
+                for (int i = 0; i < s->local_shards() && !rc; ++i) {
+                    const int sh = s->virt ? i : s->rank;
+                    rc = launch(s, LaunchClass::HIGH, [&] {
+                        return launch_apply64(reinterpret_cast<double2*>(s->shard[sh]), s->l, st.a64, s->stream);
+                    });
+                }
+                s->stats.bytes_apply += 32ull << s->l;
+                s->stats.flops_apply += (uint64_t)((8 << st.a64.k) - 2) << s->l;
+            }
             if (rc) return rc;
-            s->stats.bytes_apply += 32ull << s->l;
-            s->stats.flops_apply += (uint64_t)((8 << st.a64.k) - 2) << s->l;
         }
         s->pos = c->pos_out;
         return SV_OK;
@@ -1739,6 +1793,8 @@ int sv_circuit_run_device(sv_state* s, const sv_circuit* c) {
             rc = run_apply(s, st.apply);
         } else if (st.type == Event::EXCHANGE) {
             rc = run_exchange(s, st.exch);
+        } else if (s->fp64) {
+            rc = run_permute64(s, st.perm);
         } else {
             for (auto& d : st.perm_applies) {
                 rc = run_apply(s, d);
@@ -1793,6 +1849,7 @@ int sv_run_circuit(sv_state* s, const sv_gate* gates, size_t n_gates, int max_fu
 }
 
 // ---- amplitudes ----------------------------------------------------------------
+static int gather_units(sv_state* s, const std::vector<uint64_t>& loc, const std::vector<int32_t>& own, void* out_host);
 // complex128 states (single shard): gather into double2, D2H
 static int amplitudes64(sv_state* s, const uint64_t* idx, size_t count, sv_c128* out) {
     const uint64_t dim = 1ull << s->n;
@@ -1800,6 +1857,17 @@ static int amplitudes64(sv_state* s, const uint64_t* idx, size_t count, sv_c128*
         if (idx[i] >= dim) return fail(SV_EINVAL, "amplitude index out of range");
     int rc = materialize(s);
     if (rc) return rc;
+    if (s->g > 0) {  // sharded: the two 8 B units of every amplitude
+        std::vector<uint64_t> loc(2 * count);
+        std::vector<int32_t> own(2 * count);
+        for (size_t i = 0; i < count; ++i) {
+            const uint64_t p = phys_of(s, idx[i]);
+            loc[2 * i] = 2 * (p & (s->local_amps() - 1));
+            loc[2 * i + 1] = loc[2 * i] + 1;
+            own[2 * i] = own[2 * i + 1] = (int32_t)(p >> s->l);
+        }
+        return gather_units(s, loc, own, out);
+    }
     rc = ensure(s, s->idx_dev, s->idx_cap, count);
     if (rc) return rc;
     rc = ensure(s, s->amp_dev, s->amp_cap, 2 * count);
@@ -1850,6 +1918,16 @@ int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
     }
     rc = materialize(s);
     if (rc) return rc;
+    return gather_units(s, loc, own, out);
+}
+
+// Gather 8 B units (unit loc[i] of shard own[i]) of a sharded state into
+// host memory (virtual shards: every shard's kernel writes its own units;
+// multi-process: through the xfer areas, min-merged over ~0 fills)
+static int gather_units(sv_state* s, const std::vector<uint64_t>& loc, const std::vector<int32_t>& own, void* out_host) {
+    int rc = SV_OK;
+    const size_t count = loc.size();
+    char* out = (char*)out_host;
     const size_t chunk = s->virt ? count : std::min<size_t>(count, kXferBytes / 8);
     for (size_t o = 0; o < count; o += chunk) {
         const size_t cnt = std::min(chunk, count - o);
@@ -1886,7 +1964,7 @@ int sv_amplitudes(sv_state* s, const uint64_t* idx, size_t count, sv_c64* out) {
             rc = barrier(s);
             if (rc) return rc;
         }
-        CK(s, cudaMemcpyAsync(out + o, s->amp_dev, cnt * 8, cudaMemcpyDeviceToHost, s->stream));
+        CK(s, cudaMemcpyAsync(out + 8 * o, s->amp_dev, cnt * 8, cudaMemcpyDeviceToHost, s->stream));
         rc = sync(s);
         if (rc) return rc;
     }

@@ -1,5 +1,5 @@
 """Interleaved A/B of the bench step (reset + circuit + 10^6 samples; host wall time, mean of 10)
-across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3 AB_T=12] python tools/ab_step.py <rounds> <lib.so> ...
+across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3 AB_T=12 AB_F=1 AB_WL=rqc|sycamore] python tools/ab_step.py <rounds> <lib.so> ...
 """
 import json, os, subprocess, sys
 CHILD = r'''
@@ -13,7 +13,9 @@ n=int(os.environ.get("AB_N", "30")); d=int(os.environ.get("AB_D", "14"))
 h=sv.sv_create(n)
 if os.environ.get("AB_PIN"): sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, int(os.environ["AB_PIN"]))
 if os.environ.get("AB_T"): sv.sv_set_blocking(h, int(os.environ["AB_T"]))
-c=sv.sv_circuit_create(h, W.rqc(n,d), 1)
+F=int(os.environ.get("AB_F", "1"))
+gates=W.sycamore_rqc(n,d) if os.environ.get("AB_WL")=="sycamore" else W.rqc(n,d)
+c=sv.sv_circuit_create(h, gates, F)
 out=torch.empty(1000000, dtype=torch.int64, device="cuda")
 def step():
     sv.sv_reset(h); sv.sv_circuit_run_device(h,c); sv.sv_sample_device(h,1,1000000,out.data_ptr())

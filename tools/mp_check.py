@@ -91,6 +91,34 @@ def main():
     if np.abs(got - exp).max() > 1e-6:
         ok = False
         msgs.append(f"apply with global qubit err={np.abs(got - exp).max()}")
+    # 5. complex128 shards (NEXT-1): per-gate fp64 applies and fp64 passes
+    #    between exchanges of 16 B amplitudes, amplitudes, sampling
+    h64 = sv.sv_create_ex(n, world=world, rank=rank, virtual_shards=False, device=dev, precision=1)
+    blobs64 = [None] * world
+    dist.all_gather_object(blobs64, sv.sv_ipc_handle(h64))
+    sv.sv_attach_peers(h64, blobs64)
+    for F, bits in ((4, -1), (1, 10)):
+        sv.sv_set_blocking(h64, bits)
+        sv.sv_reset(h64)
+        st64 = sv.sv_run_circuit(h64, gates, F)
+        p64 = sv.sv_get_state_c128(h64, n)
+        f64 = osv.fidelity(p64, ref)
+        e64 = float(np.abs(p64 - ref).max())
+        if not (f64 >= 1 - 1e-12 and e64 <= 1e-12 * 2.0 ** (-n / 2) * 14 and st64["n_exchanges"] >= 1):
+            ok = False
+            msgs.append(f"complex128 F={F} fid={f64} err={e64} exch={st64['n_exchanges']}")
+    a64 = sv.sv_amplitudes_c128(h64, idx)
+    if not np.array_equal(a64, p64[idx.astype(np.int64)]):
+        ok = False
+        msgs.append("complex128 amplitudes mismatch")
+    s1 = s0.astype(np.complex128)
+    sv.sv_set_state_c128(h64, s1)
+    got64 = sv.sv_sample(h64, 42, 4000)
+    exp64, _ = osample.sample(s1, 42, 4000)
+    if not np.array_equal(got64, exp64):
+        ok = False
+        msgs.append("complex128 sampling mismatch")
+    sv.sv_destroy(h64)
     flags = [None] * world
     dist.all_gather_object(flags, (ok, msgs))
     sv.sv_destroy(h)

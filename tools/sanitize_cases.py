@@ -9,7 +9,8 @@
 * per-gate applies k = 1..6 on high, low and qubit-0 sets: SIMT tile loops
   (16 B cp.async and bulk/tensor-copy), int8 tensor-core (tcgen05) k = 5, 6;
 * controlled gates; virtual shards P = 4 (exchange kernel) with per-gate and
-  blocked passes; sampling (bins, scan, resolve); complex128 applies.
+  blocked passes; sampling (bins, scan, resolve); complex128 applies (k = 6,
+  virtual shards with 16 B exchanges and bit-swap permutations); 14-qubit tiles.
 Each result is checked against the oracle so a silent corruption also fails.
 """
 import os
@@ -93,4 +94,25 @@ h = sv.sv_create_ex(n, precision=1)
 sv.sv_run_circuit(h, gates, 4)
 check("complex128 F=4", sv.sv_get_state_c128(h, n), ref, 10)
 sv.sv_destroy(h)
+# 14-qubit tiles (64 amplitudes per thread), complex128 k = 6 (row-split tile
+# kernel), sharded complex128 (16 B exchanges, exact bit-swap permutations)
+for lazy in (True, False):
+    h = sv.sv_create(n)
+    sv.sv_set_blocking(h, 14)
+    if not lazy:
+        sv.sv_device_ptr(h)
+    sv.sv_run_circuit(h, gates, 1)
+    check(f"blocked T=14 F=1 lazy={lazy}", sv.sv_get_state(h, n), ref, 10)
+    sv.sv_destroy(h)
+h = sv.sv_create_ex(n, precision=1)
+sv.sv_run_circuit(h, gates, 6)
+check("complex128 F=6", sv.sv_get_state_c128(h, n), ref, 10)
+sv.sv_destroy(h)
+for F, T in ((4, -1), (1, 10)):
+    h = sv.sv_create_ex(n, world=4, virtual_shards=True, precision=1)
+    sv.sv_set_blocking(h, T)
+    sv.sv_run_circuit(h, gates, F)
+    sv.sv_sample(h, 3, 2000)
+    check(f"complex128 virtual shards P=4 F={F}", sv.sv_get_state_c128(h, n), ref, 10)
+    sv.sv_destroy(h)
 print("SANITIZE_CASES", "FAIL " + str(bad) if bad else "OK", flush=True)
