@@ -450,14 +450,20 @@ def run_ours(args):
     # the fastest max_fused becomes the timed configuration (max_fused = -1)
     sweep = None
     pin_sweep = None
+    beam_sweep = None
     pass_pin = args.pass_pin or 4
+    pass_beam = 5
     if not fp64 and world == 1 and not args.no_sweep:
         sweep = {}
         pin_sweep = {}
         # max_fused 1..6 at the default pass runs (128 B), and F <= 2 (the
         # register-blocked passes) also with 64 B runs (SV_OPT_PASS_PIN 3)
-        for f, pin in [(f, 4) for f in range(1, 7)] + [(1, 3), (2, 3)]:
+        # and with the greedy pass formation (SV_OPT_PASS_SEARCH 1)
+        beam_sweep = {}
+        for f, pin, beam in ([(f, 4, 5) for f in range(1, 7)] + [(1, 3, 5), (2, 3, 5)] +
+                             [(f, p, 1) for f in (1, 2) for p in (4, 3)]):
             sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pin)
+            sv.sv_set_option(h, sv.SV_OPT_PASS_SEARCH, beam)
             c = sv.sv_circuit_create(h, gates, f)
 
             def st_f():
@@ -474,16 +480,24 @@ def run_ours(args):
                 st_f()
             a1.record(stream)
             barrier()
-            (sweep if pin == 4 else pin_sweep)[str(f)] = a0.elapsed_time(a1) / 3 / 1e3
+            t_f = a0.elapsed_time(a1) / 3 / 1e3
+            if beam == 1:
+                beam_sweep[f"{f},{pin}"] = t_f
+            else:
+                (sweep if pin == 4 else pin_sweep)[str(f)] = t_f
             sv.sv_circuit_destroy(c)
         sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pass_pin)
+        sv.sv_set_option(h, sv.SV_OPT_PASS_SEARCH, 5)
     if args.max_fused < 0:
         if sweep:
-            best = min([(v, int(f), 4) for f, v in sweep.items()] + [(v, int(f), 3) for f, v in pin_sweep.items()])
-            args.max_fused, pass_pin = best[1], best[2]
+            best = min([(v, int(f), 4, 5) for f, v in sweep.items()] + [(v, int(f), 3, 5) for f, v in pin_sweep.items()] +
+                       [(v, int(k.split(",")[0]), int(k.split(",")[1]), 1) for k, v in beam_sweep.items()])
+            args.max_fused, pass_pin, pass_beam = best[1], best[2], best[3]
             sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, pass_pin)
+            sv.sv_set_option(h, sv.SV_OPT_PASS_SEARCH, pass_beam)
             fusion_choice = ("optimal over max_fused 1..6 (fusion_sweep_s) and, for the register-blocked passes "
-                             "(F <= 2), 128 B or 64 B tile runs (pass_pin_sweep_s)")
+                             "(F <= 2), 128 B or 64 B tile runs (pass_pin_sweep_s) and greedy vs searched pass "
+                             "formation (pass_search_sweep_s, SV_OPT_PASS_SEARCH 1 vs 5)")
         else:
             args.max_fused = 1 if not fp64 else 4
             fusion_choice = ("1 (the single-GPU optimum: register-blocked passes between the exchanges)" if not fp64
@@ -634,7 +648,8 @@ def run_ours(args):
                 "workload": f"{args.workload}_{n}q_d{depth}",
                 "n_qubits": n, "depth": depth, "max_fused": args.max_fused, "fusion": fusion_choice,
                 "execution": ("register-blocked passes (pass-specialised kernels), tile qubits "
-                              f"{cst.get('block_bits', 13)}, runs of {8 << pass_pin} B (SV_OPT_PASS_PIN {pass_pin})"
+                              f"{cst.get('block_bits', 13)}, runs of {8 << pass_pin} B (SV_OPT_PASS_PIN {pass_pin}), "
+                              f"pass formation {'greedy' if pass_beam == 1 else 'searched'} (SV_OPT_PASS_SEARCH {pass_beam})"
                               if cst.get("n_passes", 0) else "one launch per fused gate"),
                 "seed": args.seed,
                 "gates": len(gates), "n_fused": sv_fused, "fused_hist": cst["fused_hist"],
@@ -687,6 +702,7 @@ def run_ours(args):
             "gpu_launches": (acc["n_launch_high"] + acc["n_launch_low"] + acc["n_launch_other"]),
             "fusion_sweep_s": sweep,
             "pass_pin_sweep_s": pin_sweep,
+            "pass_search_sweep_s": beam_sweep,
             "optimal_fusion": (None if not sweep else
                                {"max_fused": args.max_fused, "pass_pin": pass_pin,
                                 "value": min(list(sweep.values()) + list((pin_sweep or {}).values())), "unit": "s"}),

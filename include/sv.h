@@ -319,7 +319,13 @@ int sv_synchronize(sv_state* s);
  *                      their products) as fp32 additions with the gates'
  *                      scalar factors multiplied in once per pass (DESIGN.md
  *                      R11): same result up to fp32 rounding order, fewer
- *                      operations; 0: every gate as a dense complex matrix.
+ *                      operations; 0: every gate as a dense complex matrix;
+ *   SV_OPT_PASS_SEARCH v in [1, 8], default 5: width of the pass-formation
+ *                      search (R7): 1 = the greedy lookahead alone;
+ *                      v > 1 keeps the v best qubit-set additions per growth
+ *                      step and takes the set whose greedy completion needs
+ *                      the fewest passes (34q D20: 10 -> 8 passes); which
+ *                      width runs faster depends on the circuit.
  * Takes effect for circuits created / gates applied afterwards.  SV_EINVAL
  * for unknown options or values. */
 #define SV_OPT_BLOCK_BITS 1
@@ -329,6 +335,7 @@ int sv_synchronize(sv_state* s);
 #define SV_OPT_DIAG_SKIP 5  /* 1 (default): sharded circuits plan with the diagonal exchange skip */
 #define SV_OPT_PASS_PIN 6   /* qubits 0..v-1 in every blocked-pass tile (runs of 8*2^v bytes): 3, 4 (default), 5 */
 #define SV_OPT_PASS_SPEC 7  /* 1 (default): structured one-qubit gates as additions in the pass kernels */
+#define SV_OPT_PASS_SEARCH 8 /* pass-formation search width 1..8 (default 5) */
 #define SV_PATH_AUTO 0
 #define SV_PATH_SIMT 1
 #define SV_PATH_INT8 2

@@ -38,6 +38,7 @@ SV_OPT_TIMING = 4
 SV_OPT_DIAG_SKIP = 5
 SV_OPT_PASS_PIN = 6
 SV_OPT_PASS_SPEC = 7
+SV_OPT_PASS_SEARCH = 8
 SV_PATH_AUTO = 0
 SV_PATH_SIMT = 1
 SV_PATH_INT8 = 2

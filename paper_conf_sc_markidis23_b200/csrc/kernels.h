@@ -79,6 +79,10 @@ cudaError_t launch_small_circuit(float2* psi, int n, int ngates, const SmallGate
 // (|S| = tile bits, contains 0..r-1); one HBM read + write per pass.
 constexpr int kPassMaxGates = 64;
 constexpr int kPassPlaneFloats = 6144;
+// 14-qubit tiles exist only as pass-specialised kernels, whose matrices are
+// launch parameters (<= 32 KB) rather than a fixed parameter struct: a pass
+// of such tiles may hold up to kJitPassMaxGates gates per launch
+constexpr int kJitPassMaxGates = 256;
 struct PassGate {
     int k;          // 1..4
     int pos[4];     // tile-local positions (rank of the qubit in sorted S), ascending

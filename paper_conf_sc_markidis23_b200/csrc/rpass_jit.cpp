@@ -86,11 +86,37 @@ namespace {
 // The 64-amplitude form only for tiles of runs >= 2^SVB_JIT_M14_RUN
 // amplitudes (A/B, round 2: 30q D14 with 128 B runs 24.8 -> 23.7 ms; 32q
 // D20 with 64 B runs 137.5 -> 142.5 ms, with 128 B runs unchanged)
+// A two-qubit gate with exactly one nonzero per row and column (e.g.
+// fSim(pi/2, phi), iSWAP, SWAP with phases): out_r = m_r a_perm[r] (reading
+// R11, two-qubit monomial form).  complex64 pass kernels with SV_OPT_PASS_SPEC.
+bool monomial2(const PassDesc& pd, const PassGate& pg, int perm[4], std::complex<double> m[4]) {
+    if (!pd.spec || pd.wide || pg.k != 2 || gate_kind(pd, pg) != 0 || pd.mats64.size() < pg.moff + 32) return false;
+    const double* M = pd.mats64.data() + pg.moff;
+    double big = 0;
+    for (int e = 0; e < 16; ++e) big = std::max(big, std::abs(std::complex<double>(M[2 * e], M[2 * e + 1])));
+    const double tiny = 1e-9 * big;
+    int used = 0;
+    for (int r = 0; r < 4; ++r) {
+        int c0 = -1;
+        for (int c = 0; c < 4; ++c)
+            if (std::abs(std::complex<double>(M[2 * (4 * r + c)], M[2 * (4 * r + c) + 1])) > tiny) {
+                if (c0 >= 0) return false;
+                c0 = c;
+            }
+        if (c0 < 0 || ((used >> c0) & 1)) return false;
+        used |= 1 << c0;
+        perm[r] = c0;
+        m[r] = std::complex<double>(M[2 * (4 * r + c0)], M[2 * (4 * r + c0) + 1]);
+    }
+    return true;
+}
 int jit_m(const PassDesc& pd) {
     if (pd.wide) return 4;
     if (pd.S.size() < 14 || pd.r < SVB_JIT_M14_RUN) return SVB_JIT_M;
+    int perm[4];
+    std::complex<double> m[4];
     for (const auto& g : pd.gates)
-        if (g.k == 2 && gate_kind(pd, g) == 0) return SVB_JIT_M;
+        if (g.k == 2 && gate_kind(pd, g) == 0 && !monomial2(pd, g, perm, m)) return SVB_JIT_M;
     return SVB_JIT_M14;
 }
 
@@ -147,13 +173,17 @@ struct TileMap {
 // in fp32 only the rounding differs from the dense product.
 using cd = std::complex<double>;
 struct GSpec {
-    int cls = 0;                  // 0 generic, 1 row form, 2 column form, 3 one-qubit diagonal
+    int cls = 0;                  // 0 generic, 1 row form, 2 column form, 3 one-qubit diagonal, 4 two-qubit monomial
     int p[2] = {0, 0};            // row: out_r = s_r (a0 + i^p[r] a1); column: out1 = i^p[0] a0 + i^p[1] mu a1
     int q[2] = {0, 0};            // s_r = i^q[r] when unit[r]
     bool unit[2] = {true, true};  // diagonal: s_r multiplies the amplitudes with the gate bit = r
     cd s[2] = {1.0, 1.0};         // the non-unit s_r
     cd mu = 1.0;                  // column form: out0 = a0 + mu a1
     cd c = 1.0;                   // the scalar taken out
+    int perm[4] = {0, 1, 2, 3};   // monomial: out_r = m_r a_perm[r], m_r = i^mq[r] when munit[r]
+    int mq[4] = {0, 0, 0, 0};
+    bool munit[4] = {true, true, true, true};
+    cd ms[4] = {1.0, 1.0, 1.0, 1.0};
 };
 cd ipow(int q) {
     static const cd u[4] = {cd(1, 0), cd(0, 1), cd(-1, 0), cd(0, -1)};
@@ -170,6 +200,17 @@ bool unit_exp(cd z, int& e) {
 }
 GSpec classify(const PassDesc& pd, const PassGate& pg) {
     GSpec g;
+    if (pg.k == 2) {
+        cd m[4];
+        if (!monomial2(pd, pg, g.perm, m)) return g;
+        g.cls = 4;
+        for (int r = 0; r < 4; ++r)
+            if (!unit_exp(m[r], g.mq[r])) {
+                g.munit[r] = false;
+                g.ms[r] = m[r];
+            }
+        return g;
+    }
     if (!pd.spec || pg.k != 1 || pd.mats64.size() < pg.moff + 8) return g;
     const int kind = gate_kind(pd, pg);
     const double* m = pd.mats64.data() + pg.moff;
@@ -256,6 +297,30 @@ ChunkSpec chunk_spec(const PassDesc& pd, size_t g0, size_t g1, bool zinit) {
     return cs;
 }
 
+// Launch chunks of a pass: tiles up to 13 qubits as the generic kernel's
+// (rpass_chunks: <= 64 gates, <= 48 phases; bit-identical states), 14-qubit
+// tiles up to kJitPassMaxGates gates and 96 phases with at most 1800 matrix
+// slots of 16 B (the parameter space, 32 KB)
+std::vector<std::pair<size_t, size_t>> jit_chunks(const PassDesc& pd) {
+    const int M = jit_m(pd);
+    if (pd.S.size() < 14) return rpass_chunks(pd, M, pd.wide);
+    std::vector<std::pair<size_t, size_t>> out;
+    const size_t ng = pd.gates.size();
+    auto slots = [&](size_t g) {
+        const int kind = gate_kind(pd, pd.gates[g]), k = pd.gates[g].k;
+        return kind == 2 ? 0u : kind == 1 ? (1u << k) : (1u << (2 * k));
+    };
+    size_t g0 = 0;
+    while (g0 < ng) {
+        size_t g1 = g0, sl = 0;
+        while (g1 < ng && g1 - g0 < (size_t)kJitPassMaxGates && sl + slots(g1) <= 1800) sl += slots(g1++);
+        while ((int)plan_phases(pd, g0, g1, M, pd.wide).size() > 96) g1 = g0 + (g1 - g0) / 2;
+        out.push_back({g0, g1});
+        g0 = g1;
+    }
+    return out;
+}
+
 // PTX text builder: amplitudes live in %a0..%a31 (one .b64 = packed
 // (re, im) complex64 each), rewritten in place; ptxas renames them.
 struct Ptx {
@@ -333,6 +398,8 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         for (int b = 0; b < pg.k; ++b) put(pg.pos[b]);
         const GSpec& x = cs.g[g];
         if (x.cls) k += 's';
+        if (x.cls == 4)
+            for (int r = 0; r < 4; ++r) put(x.perm[r] + 4 * x.mq[r] + (x.munit[r] ? 16 : 0));
         if (x.cls) put(64 * x.cls + 16 * x.p[0] + 4 * x.p[1] + x.q[0] * 256 + x.q[1] * 1024 + (x.unit[0] ? 4096 : 0) +
                        (x.unit[1] ? 8192 : 0));
     }
@@ -416,6 +483,11 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             gbase[g] = mats.size() / 4;
             if (x.cls == 2) {
                 put_s(x.mu);
+                continue;
+            }
+            if (x.cls == 4) {
+                for (int r = 0; r < 4; ++r)
+                    if (!x.munit[r]) put_s(x.ms[r]);
                 continue;
             }
             if (x.cls) {
@@ -560,6 +632,29 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         P.op("fma.rn.f32x2 ", d, ", ", it, ", %qsi, %py");
     };
     auto emit_spec = [&](const GSpec& x, uint32_t mask, size_t base) {
+        if (x.cls == 4) {  // two-qubit monomial: out_r = m_r a_perm[r] (copies, rotations, multiplies)
+            size_t slr[4];
+            size_t nxt = base;
+            for (int r = 0; r < 4; ++r) slr[r] = x.munit[r] ? 0 : nxt++;
+            const uint32_t rest = ((1u << M) - 1u) & ~mask;
+            for (uint32_t gi = 0; gi < (uint32_t)NA / 4; ++gi) {
+                const uint32_t b0 = pdep(gi, rest);
+                for (int c = 0; c < 4; ++c) P.op("mov.b64 %x", c, ", %a", b0 | pdep(c, mask));
+                for (int r = 0; r < 4; ++r) {
+                    const std::string d = "%a" + std::to_string(b0 | pdep(r, mask));
+                    const std::string src = "%x" + std::to_string(x.perm[r]);
+                    if (!x.munit[r]) {
+                        pmul(d, src, slr[r]);
+                    } else if (x.mq[r] & 3) {
+                        const std::string t = rot(src, x.mq[r]);
+                        P.op("mul.rn.f32x2 ", d, ", ", t, ", %pone");
+                    } else {
+                        P.op("mov.b64 ", d, ", ", src);
+                    }
+                }
+            }
+            return;
+        }
         size_t sl[2] = {base, base};
         if (!x.unit[0]) sl[1] = base + 1;
         if (x.cls == 3) {  // diagonal: s_r on the amplitudes whose gate bit is r
@@ -1649,7 +1744,7 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
         out.clear();
         const int T = (int)pd.S.size();
         bool first = true;
-        for (const auto& ch : rpass_chunks(pd, jit_m(pd), pd.wide)) {
+        for (const auto& ch : jit_chunks(pd)) {
             RpJitLaunch l;
             size_t nm = 0;
             const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats);
@@ -1683,7 +1778,7 @@ int rpass_jit_prepare_many(const std::vector<const PassDesc*>& pds, int n_local,
         const int T = (int)pd.S.size();
         const int M = jit_m(pd);
         bool first = true;
-        for (const auto& ch : rpass_chunks(pd, M, pd.wide)) {
+        for (const auto& ch : jit_chunks(pd)) {
             RpJitLaunch l;
             size_t nm = 0;
             const bool z = zinit[i] && first;
@@ -1812,13 +1907,16 @@ uint64_t rpass_jit_ops_per_amp(const PassDesc& pd, bool zinit) {
     if (!pd.spec) return rpass_fma_per_amp(pd);
     uint64_t f = 0;
     bool first = true;
-    for (const auto& ch : rpass_chunks(pd, jit_m(pd), pd.wide)) {
+    for (const auto& ch : jit_chunks(pd)) {
         const ChunkSpec cs = chunk_spec(pd, ch.first, ch.second, zinit && first);
         for (size_t g = ch.first; g < ch.second; ++g) {
             const GSpec& x = cs.g[g];
             const int kind = gate_kind(pd, pd.gates[g]);
             const uint64_t nu = (x.unit[0] ? 0 : 2) + (x.unit[1] ? 0 : 2);
+            uint64_t mono = 0;  // monomial: per 4 amplitudes 2 per rotation, 4 per multiply
+            for (int r = 0; r < 4; ++r) mono += !x.munit[r] ? 4 : (x.mq[r] & 3) ? 2 : 0;
             switch (x.cls) {
+                case 4: f += (mono + 3) / 4; break;
                 case 1: f += 2 + nu; break;  // 2 FADDs per output, 4 ops per multiplier (per pair)
                 case 2: f += 4; break;
                 case 3: f += nu; break;

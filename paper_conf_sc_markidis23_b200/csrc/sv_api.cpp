@@ -13,7 +13,9 @@
 #include <algorithm>
 #include <chrono>
 #include <cstring>
+#include <map>
 #include <memory>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -32,6 +34,9 @@ using namespace svb;
 #endif
 #ifndef SVB_FUSED_BINS
 #define SVB_FUSED_BINS 1  // the last register-blocked pass writes the sampler's bin weights
+#endif
+#ifndef SVB_PASS_BEAM
+#define SVB_PASS_BEAM 5  // pass formation search width (reading R7): 1 = the greedy lookahead alone
 #endif
 #ifndef SVB_PASS_PIN
 #define SVB_PASS_PIN 4  // qubits 0..PIN-1 in every blocked-pass tile (runs of 8 * 2^PIN bytes)
@@ -91,6 +96,7 @@ struct sv_state {
     int diag_skip = 1;        // SV_OPT_DIAG_SKIP
     int pass_pin = SVB_PASS_PIN;  // SV_OPT_PASS_PIN: qubits 0..pin-1 in every blocked-pass tile
     int pass_spec = 1;            // SV_OPT_PASS_SPEC: structured one-qubit gates as additions (reading R11)
+    int pass_beam = SVB_PASS_BEAM;  // SV_OPT_PASS_SEARCH: pass-formation search width (reading R7)
     bool sample_pending = false;  // a sv_sample_device status word not yet checked
     // the sampler's bins hold the current state's S5 weights (written by the
     // last register-blocked pass of the last circuit); any state change clears it
@@ -650,8 +656,19 @@ int kind_of(const std::vector<cd>& M, int k) {
 // tile set S is the pinned qubits, the pass's qubits, then the lowest
 // remaining qubits (longer runs).  The state never moves: a pass only
 // chooses which amplitudes share a tile.
-std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPassPinned = SVB_PASS_PIN) {
+// Pass qubit sets chosen for a fused-gate structure (masks, diagonal flags,
+// tile, pinning, search width): the formation depends on nothing else, so
+// circuits of the same structure reuse it (process-wide cache)
+std::mutex g_form_mu;
+std::map<std::string, std::vector<uint64_t>> g_form_cache;
+
+std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPassPinned = SVB_PASS_PIN,
+                                   int beam = SVB_PASS_BEAM) {
     const uint64_t pin = (1ull << kPassPinned) - 1ull;
+    // gates per pass: one launch of the generic kernel's parameter struct, or
+    // (14-qubit tiles: pass-specialised kernels only) a larger JIT launch
+    const size_t kMaxGates = T >= 14 ? (size_t)kJitPassMaxGates : (size_t)kPassMaxGates;
+    const size_t kMaxPlanes = T >= 14 ? (size_t)kJitPassMaxGates * 48 : (size_t)kPassPlaneFloats;
     const int Fp = T - kPassPinned;
     const size_t nf = in.size();
     std::vector<uint64_t> fm(nf, 0);
@@ -690,77 +707,159 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
         cur.planes.insert(cur.planes.end(), Qp.begin(), Qp.end());
         cur.gates.push_back(pg);
     };
+    // ---- pass formation (reading R7): the qubit set Q of each pass.  A set
+    // absorbs every later unplaced gate inside Q | pinned that touches no
+    // qubit of an earlier gate left out (diagonal gates only block
+    // non-diagonal ones, R12).  Greedy lookahead: grow Q from the first
+    // unplaced gate's qubits by the qubit set of a left-out gate (among the
+    // next 40 distinct ones) that absorbs the most gates, until none helps.
+    // Search (beam > 1): keep the `beam` best additions at every growth step
+    // (at most beam^2 partial sets), and take the final set whose greedy
+    // completion of the rest of the circuit needs the fewest passes (ties:
+    // the set absorbing more gates now).  30q D14: 6 -> 5 passes, 34q D20:
+    // 10 -> 8 (profiles/r2_ab.md).
+    auto absorb = [&](size_t i0, uint64_t Qc, const std::vector<char>& pl, std::vector<size_t>* out) {
+        uint64_t Bl = 0, Bd = 0;  // qubits of left-out gates: non-diagonal / diagonal
+        size_t cnt = 0, planes = 0;
+        for (size_t j = i0; j < nf; ++j) {
+            if (pl[j]) continue;
+            const uint64_t Sj = fm[j];
+            const size_t pj = 3ull << (2 * in[j].k);
+            if (!(Sj & (dg[j] ? Bl : Bl | Bd)) && !(Sj & ~(Qc | pin)) && cnt < kMaxGates && planes + pj <= kMaxPlanes) {
+                ++cnt;
+                planes += pj;
+                if (out) out->push_back(j);
+            } else if (dg[j]) {
+                Bd |= Sj;
+            } else {
+                Bl |= Sj;
+            }
+        }
+        return cnt;
+    };
+    auto grow = [&](size_t i0, const std::vector<char>& pl, int B, std::vector<uint64_t>& finals) {
+        std::vector<uint64_t> states{fm[i0] & ~pin};
+        std::vector<char> in_cur(nf, 0);
+        while (!states.empty()) {
+            std::vector<uint64_t> nxt;
+            for (uint64_t Qs : states) {
+                std::vector<size_t> cur;
+                const size_t have = absorb(i0, Qs, pl, &cur);
+                for (size_t j : cur) in_cur[j] = 1;
+                std::vector<uint64_t> cands;
+                for (size_t j = i0; j < nf && cands.size() < 40; ++j) {
+                    if (pl[j] || in_cur[j]) continue;
+                    const uint64_t add = fm[j] & ~pin & ~Qs;
+                    if (!add || __builtin_popcountll(Qs | add) > Fp) continue;
+                    if (std::find(cands.begin(), cands.end(), add) == cands.end()) cands.push_back(add);
+                }
+                for (size_t j : cur) in_cur[j] = 0;
+                struct Sc { size_t c; int bits; size_t ord; uint64_t add; };
+                std::vector<Sc> sc;
+                for (size_t o = 0; o < cands.size(); ++o) {
+                    const size_t c = absorb(i0, Qs | cands[o], pl, nullptr);
+                    if (c > have) sc.push_back({c, __builtin_popcountll(cands[o]), o, cands[o]});
+                }
+                std::sort(sc.begin(), sc.end(), [](const Sc& a, const Sc& b) {
+                    return a.c != b.c ? a.c > b.c : a.bits != b.bits ? a.bits < b.bits : a.ord < b.ord;
+                });
+                if (sc.empty()) {
+                    if (std::find(finals.begin(), finals.end(), Qs) == finals.end()) finals.push_back(Qs);
+                    continue;
+                }
+                for (size_t t = 0; t < sc.size() && t < (size_t)B; ++t) {
+                    const uint64_t Qn = Qs | sc[t].add;
+                    if (std::find(nxt.begin(), nxt.end(), Qn) == nxt.end()) nxt.push_back(Qn);
+                }
+            }
+            if (nxt.size() > (size_t)(B * B)) nxt.resize((size_t)(B * B));
+            states.swap(nxt);
+        }
+    };
+    auto greedy_rest = [&](std::vector<char> pl) {
+        int n = 0;
+        for (size_t i0 = 0; i0 < nf; ++i0) {
+            if (pl[i0]) continue;
+            std::vector<uint64_t> f;
+            grow(i0, pl, 1, f);
+            std::vector<size_t> m;
+            absorb(i0, f[0], pl, &m);
+            for (size_t j : m) pl[j] = 1;
+            ++n;
+        }
+        return n;
+    };
+    std::vector<uint64_t> forms;  // Q of every pass
+    if (SVB_PASS_LOOKAHEAD) {
+        std::string key;
+        key.reserve(16 * nf + 32);
+        key += std::to_string(T) + "," + std::to_string(kPassPinned) + "," + std::to_string(beam) + ",";
+        for (size_t i = 0; i < nf; ++i) key += std::to_string(fm[i]) + (dg[i] ? "d" : "") + ",";
+        bool hit = false;
+        {
+            std::lock_guard<std::mutex> lk(g_form_mu);
+            auto it = g_form_cache.find(key);
+            if (it != g_form_cache.end()) {
+                forms = it->second;
+                hit = true;
+            }
+        }
+        if (!hit) {
+            std::vector<char> pl(nf, 0);
+            for (size_t i0 = 0; i0 < nf; ++i0) {
+                if (pl[i0]) continue;
+                std::vector<uint64_t> finals;
+                grow(i0, pl, std::max(1, beam), finals);
+                uint64_t Qb = finals[0];
+                if (finals.size() > 1) {
+                    int best_n = 1 << 30;
+                    size_t best_c = 0;
+                    for (uint64_t Qf : finals) {
+                        std::vector<char> p2 = pl;
+                        std::vector<size_t> m;
+                        const size_t c = absorb(i0, Qf, p2, &m);
+                        for (size_t j : m) p2[j] = 1;
+                        const int nrest = greedy_rest(p2);
+                        if (nrest < best_n || (nrest == best_n && c > best_c)) {
+                            best_n = nrest;
+                            best_c = c;
+                            Qb = Qf;
+                        }
+                    }
+                }
+                std::vector<size_t> m;
+                absorb(i0, Qb, pl, &m);
+                for (size_t j : m) pl[j] = 1;
+                forms.push_back(Qb);
+            }
+            std::lock_guard<std::mutex> lk(g_form_mu);
+            if (g_form_cache.size() > 256) g_form_cache.clear();
+            g_form_cache[key] = forms;
+        }
+    }
+    size_t npass = 0;
     for (size_t i = 0; i < nf; ++i) {
         if (placed[i]) continue;
         std::vector<size_t> mem{i};
         placed[i] = 1;
         uint64_t Q = fm[i], B = 0;
         if (SVB_PASS_LOOKAHEAD) {
-            // choose the pass's free qubits by lookahead (reading R7): the
-            // gates a qubit set Q absorbs are fixed (every later unplaced gate
-            // inside Q | pinned that touches no qubit of an earlier gate left
-            // out); grow Q, starting from gate i's qubits, by the qubit set of
-            // a left-out gate that absorbs the most gates, until nothing helps
             placed[i] = 0;
-            auto absorb = [&](uint64_t Qc, std::vector<size_t>* out) {
-                uint64_t Bl = 0, Bd = 0;  // qubits of left-out gates: non-diagonal / diagonal
-                size_t cnt = 0, planes = 0;
-                for (size_t j = i; j < nf; ++j) {
-                    if (placed[j]) continue;
-                    const uint64_t Sj = fm[j];
-                    const size_t pj = 3ull << (2 * in[j].k);
-                    if (!(Sj & (dg[j] ? Bl : Bl | Bd)) && !(Sj & ~(Qc | pin)) && cnt < (size_t)kPassMaxGates &&
-                        planes + pj <= (size_t)kPassPlaneFloats) {
-                        ++cnt;
-                        planes += pj;
-                        if (out) out->push_back(j);
-                    } else if (dg[j]) {
-                        Bd |= Sj;
-                    } else {
-                        Bl |= Sj;
-                    }
-                }
-                return cnt;
-            };
-            Q = fm[i] & ~pin;
-            for (;;) {
-                std::vector<size_t> cur;
-                const size_t have = absorb(Q, &cur);
-                std::vector<char> in_cur(nf, 0);
-                for (size_t j : cur) in_cur[j] = 1;
-                std::vector<uint64_t> cands;
-                for (size_t j = i; j < nf && cands.size() < 40; ++j) {
-                    if (placed[j] || in_cur[j]) continue;
-                    const uint64_t add = fm[j] & ~pin & ~Q;
-                    if (!add || __builtin_popcountll(Q | add) > Fp) continue;
-                    if (std::find(cands.begin(), cands.end(), add) == cands.end()) cands.push_back(add);
-                }
-                uint64_t best = 0;
-                size_t bestc = have;
-                for (uint64_t add : cands) {
-                    const size_t c = absorb(Q | add, nullptr);
-                    if (c > bestc || (best && c == bestc && __builtin_popcountll(add) < __builtin_popcountll(best))) {
-                        best = add;
-                        bestc = c;
-                    }
-                }
-                if (!best) break;
-                Q |= best;
-            }
+            Q = forms[npass++];
             mem.clear();
-            absorb(Q, &mem);
+            absorb(i, Q, placed, &mem);
             for (size_t j : mem) placed[j] = 1;
             Q = 0;
             for (size_t j : mem) Q |= fm[j];
         } else {
             size_t planes = 3ull << (2 * in[i].k);
-            for (size_t j = i + 1; j < nf && mem.size() < (size_t)kPassMaxGates; ++j) {
+            for (size_t j = i + 1; j < nf && mem.size() < kMaxGates; ++j) {
                 if (placed[j]) continue;
                 const uint64_t Sj = fm[j];
                 const size_t pj = 3ull << (2 * in[j].k);
                 if (Sj & B) {
                     B |= Sj;
-                } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= (size_t)kPassPlaneFloats) {
+                } else if (__builtin_popcountll((Q | Sj) & ~pin) <= Fp && planes + pj <= kMaxPlanes) {
                     Q |= Sj;
                     planes += pj;
                     mem.push_back(j);
@@ -1418,7 +1517,7 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
     std::vector<PassIn> run, run_all;
     auto flush_passes = [&]() {
         if (run.empty()) return;
-        for (auto& pd : build_passes(T, run, s->pass_pin)) {
+        for (auto& pd : build_passes(T, run, s->pass_pin, s->pass_beam)) {
             pd.wide = s->fp64;
             pd.spec = s->pass_spec && s->pass_jit && pd.mats_shard.empty();
             pd.fma_per_amp = rpass_supported(pd) ? pass_ops(pd, false) : 0;
@@ -1510,7 +1609,7 @@ static int circuit_create_impl(sv_state* s, const sv_gate* gates, size_t n_gates
             }
             for (int b = 0; b < g.k; ++b) seen[g.q[b]] = 1;
         }
-        std::vector<PassDesc> pz = (nfold && !rest.empty()) ? build_passes(T, rest, s->pass_pin) : std::vector<PassDesc>{};
+        std::vector<PassDesc> pz = (nfold && !rest.empty()) ? build_passes(T, rest, s->pass_pin, s->pass_beam) : std::vector<PassDesc>{};
         if (!pz.empty() && rpass_supported(pz[0])) {
             for (int p = 0; p < (int)pz[0].S.size(); ++p) {
                 pz[0].pinit_v.push_back(pv[2 * pz[0].S[p]]);
@@ -2289,6 +2388,10 @@ int sv_set_option(sv_state* s, int option, int value) {
         case SV_OPT_DIAG_SKIP:
             if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_DIAG_SKIP takes 0 or 1");
             s->diag_skip = value;
+            return SV_OK;
+        case SV_OPT_PASS_SEARCH:
+            if (value < 1 || value > 8) return fail(SV_EINVAL, "SV_OPT_PASS_SEARCH takes 1..8");
+            s->pass_beam = value;
             return SV_OK;
         case SV_OPT_PASS_SPEC:
             if (value != 0 && value != 1) return fail(SV_EINVAL, "SV_OPT_PASS_SPEC takes 0 or 1");

@@ -47,6 +47,8 @@ def test_invalid_calls_launch_nothing():
         _expect(sv.SV_EINVAL, sv.sv_amplitudes, h, np.array([1 << n], dtype=np.uint64))
         _expect(sv.SV_EINVAL, sv.sv_run_circuit, h, W.rqc(n, 4), 7)    # max_fused > 6
         _expect(sv.SV_EINVAL, sv.sv_set_option, h, 99, 1)
+        _expect(sv.SV_EINVAL, sv.sv_set_option, h, sv.SV_OPT_PASS_SEARCH, 0)
+        _expect(sv.SV_EINVAL, sv.sv_set_option, h, sv.SV_OPT_PASS_SEARCH, 9)
         _expect(sv.SV_EINVAL, sv.sv_set_blocking, h, 9)
         _expect(sv.SV_EINVAL, sv.sv_set_state, h, np.zeros(5, np.complex64))
         assert _launches(h) == base

@@ -275,6 +275,54 @@ def test_spec_structured_gates_vs_oracle(bits, lazy):
     _check(n, layer_depth(gates), b, ref)
 
 
+def _monomial_circuit(n, m, seed):
+    """Two-qubit monomial gates (one nonzero per row and column: fSim(pi/2,
+    phi), iSWAP, SWAP, random permutations with unit (i^k) and non-unit
+    phases) among structured and dense one-qubit gates and dense two-qubit
+    gates, on register and tile bits in every order."""
+    rng = np.random.default_rng(seed)
+    iswap = np.array([[1, 0, 0, 0], [0, 0, 1j, 0], [0, 1j, 0, 0], [0, 0, 0, 1]])
+    swap = np.array([[1, 0, 0, 0], [0, 0, 1, 0], [0, 1, 0, 0], [0, 0, 0, 1]])
+    gates = []
+    for t in range(m):
+        r = rng.random()
+        a, b = (int(x) for x in rng.choice(n if rng.random() < 0.5 else 7, 2, replace=False))
+        if r < 0.45:
+            kind = int(rng.integers(4))
+            if kind == 0:
+                M = W.gate_fsim(np.pi / 2, rng.uniform(0, 2 * np.pi))
+            elif kind == 1:
+                M = iswap
+            elif kind == 2:
+                M = swap
+            else:
+                P = np.eye(4)[rng.permutation(4)]
+                ph = np.where(rng.random(4) < 0.5, 1j ** rng.integers(4, size=4), np.exp(1j * rng.uniform(0, 6.3, 4)))
+                M = np.diag(ph) @ P
+            gates.append(W.Gate(t, "mono", (a, b), np.asarray(M, dtype=np.complex128)))
+        elif r < 0.55:
+            gates.append(W.Gate(t, "u2", (a, b), W.haar_unitary(4, rng)))
+        else:
+            M = [W.GATE_H, W.GATE_X_1_2, W.GATE_T, W.haar_unitary(2, rng)][int(rng.integers(4))]
+            gates.append(W.Gate(t, "u", (a,), np.asarray(M, dtype=np.complex128)))
+    return gates
+
+
+@pytest.mark.parametrize("bits", [11, 13, 14])
+@pytest.mark.parametrize("lazy", [True, False])
+def test_spec_monomial_two_qubit_gates_vs_oracle(bits, lazy):
+    """Two-qubit monomial gates as copies, rotations and multiplies (reading
+    R11) against the oracle, and fewer operations than the dense form."""
+    n, m = 20, 220
+    gates = _monomial_circuit(n, m, seed=bits + 3 * lazy)
+    ref = ref_c.run(n, gates)
+    a, sa = _state(n, gates, 1, bits, jit=True, lazy_zero=lazy, spec=1)
+    b, sb = _state(n, gates, 1, bits, jit=True, lazy_zero=lazy, spec=0)
+    assert sa["n_jit_passes"] > 0 and sa["fma_apply"] < sb["fma_apply"]
+    _check(n, layer_depth(gates), a, ref)
+    _check(n, layer_depth(gates), b, ref)
+
+
 @pytest.mark.parametrize("n,d,bits", [(22, 14, 13), (20, 20, 11), (21, 12, 10), (22, 16, 14)])
 def test_spec_rqc_vs_oracle(n, d, bits):
     """The RQC (H, sqrt(X), sqrt(Y), T, CZ) through the structured path,
