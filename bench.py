@@ -76,6 +76,7 @@ def parse():
     ap.add_argument("--samples", type=int, default=N_SAMPLES)
     ap.add_argument("--block-bits", type=int, default=-1, help="cache-blocked passes: tile qubits (0 = off; -1 = library default)")
     ap.add_argument("--pass-pin", type=int, default=0, help="fix SV_OPT_PASS_PIN (3: 64 B runs, 4: 128 B) instead of sweeping")
+    ap.add_argument("--pass-search", type=int, default=0, help="fix SV_OPT_PASS_SEARCH (1: greedy, 5: searched) instead of sweeping")
     ap.add_argument("--precision", type=int, default=32, choices=[32, 64], help="complex64 (32) or complex128 (64) state")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sweep", action="store_true",
@@ -438,6 +439,8 @@ def run_ours(args):
         sv.sv_set_blocking(h, args.block_bits)
     if args.pass_pin:
         sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, args.pass_pin)
+    if args.pass_search:
+        sv.sv_set_option(h, sv.SV_OPT_PASS_SEARCH, args.pass_search)
     samples_dev = torch.empty(args.samples, dtype=torch.int64, device="cuda")
 
     def barrier():
@@ -452,7 +455,7 @@ def run_ours(args):
     pin_sweep = None
     beam_sweep = None
     pass_pin = args.pass_pin or 4
-    pass_beam = 5
+    pass_beam = args.pass_search or 5
     if not fp64 and world == 1 and not args.no_sweep:
         sweep = {}
         pin_sweep = {}

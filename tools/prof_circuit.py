@@ -1,6 +1,6 @@
 """Run a prepared RQC circuit a few times (for ncu captures of single passes).
 
-usage: python tools/prof_circuit.py <n> <depth> <max_fused> [reps] [pass_pin] [jit]
+usage: python tools/prof_circuit.py <n> <depth> <max_fused> [reps] [pass_pin] [jit] [pass_search]
 The first run starts from the lazily reset |0...0> (its first pass
 synthesises the zero tiles); later runs reset in between the same way."""
 import os
@@ -17,6 +17,8 @@ if len(sys.argv) > 5:
     sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, int(sys.argv[5]))
 if len(sys.argv) > 6:
     sv.sv_set_option(h, sv.SV_OPT_PASS_JIT, int(sys.argv[6]))
+if len(sys.argv) > 7:
+    sv.sv_set_option(h, sv.SV_OPT_PASS_SEARCH, int(sys.argv[7]))
 c = sv.sv_circuit_create(h, W.rqc(n, d), F)
 for _ in range(reps):
     sv.sv_reset(h)

@@ -11,3 +11,4 @@ run --qubits 34 --depth 20 --max-fused 1 --steps 2 --warmup 2 --no-cpu-baseline 
 run --qubits 30 --depth 14 --workload sycamore --steps 5 --warmup 3 --no-cpu-baseline
 run --qubits 30 --depth 14 --precision 64 --max-fused 1 --steps 3 --warmup 2 --no-cpu-baseline --no-sweep
 run --qubits 30 --depth 14 --precision 64 --max-fused 4 --steps 3 --warmup 2 --no-cpu-baseline --no-sweep
+run --qubits 30 --depth 14 --precision 64 --max-fused 1 --steps 3 --warmup 2 --no-cpu-baseline --no-sweep --pass-search 1
