@@ -301,6 +301,7 @@ ChunkSpec chunk_spec(const PassDesc& pd, size_t g0, size_t g1, bool zinit) {
 // (rpass_chunks: <= 64 gates, <= 48 phases; bit-identical states), 14-qubit
 // tiles up to kJitPassMaxGates gates and 96 phases with at most 1800 matrix
 // slots of 16 B (the parameter space, 32 KB)
+std::vector<RpPhaseHost> phases_cached(const PassDesc& pd, size_t g0, size_t g1, int M, bool wide);
 std::vector<std::pair<size_t, size_t>> jit_chunks(const PassDesc& pd) {
     const int M = jit_m(pd);
     if (pd.S.size() < 14) return rpass_chunks(pd, M, pd.wide);
@@ -314,7 +315,7 @@ std::vector<std::pair<size_t, size_t>> jit_chunks(const PassDesc& pd) {
     while (g0 < ng) {
         size_t g1 = g0, sl = 0;
         while (g1 < ng && g1 - g0 < (size_t)kJitPassMaxGates && sl + slots(g1) <= 1800) sl += slots(g1++);
-        while ((int)plan_phases(pd, g0, g1, M, pd.wide).size() > 96) g1 = g0 + (g1 - g0) / 2;
+        while ((int)phases_cached(pd, g0, g1, M, pd.wide).size() > 96) g1 = g0 + (g1 - g0) / 2;
         out.push_back({g0, g1});
         g0 = g1;
     }
@@ -411,6 +412,25 @@ std::string chunk_key(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     return k;
 }
 
+// Phase plans by chunk structure (plan_phases searches every M-subset of
+// the tile positions per phase: the dominant host cost of creating a
+// circuit; circuits of the same structure reuse the plan)
+std::mutex g_phase_mu;
+std::map<std::string, std::vector<RpPhaseHost>> g_phase_cache;
+std::vector<RpPhaseHost> phases_cached(const PassDesc& pd, size_t g0, size_t g1, int M, bool wide) {
+    const std::string key = chunk_key(pd, 0, g0, g1, false) + "#" + std::to_string(M) + (wide ? "w" : "");
+    {
+        std::lock_guard<std::mutex> lk(g_phase_mu);
+        auto it = g_phase_cache.find(key);
+        if (it != g_phase_cache.end()) return it->second;
+    }
+    std::vector<RpPhaseHost> ph = plan_phases(pd, g0, g1, M, wide);
+    std::lock_guard<std::mutex> lk(g_phase_mu);
+    if (g_phase_cache.size() > 4096) g_phase_cache.clear();
+    g_phase_cache[key] = ph;
+    return ph;
+}
+
 // PTX of one launch chunk [g0, g1) of pass pd; nm receives the number of
 // float4 matrix slots, mats their values (launch order).  emit == false:
 // only nm and mats (the PTX is cached under chunk_key).
@@ -424,7 +444,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     TileMap tm;
     tm.r = pd.r;
     for (int i = pd.r; i < T; ++i) tm.H.push_back(pd.S[i]);
-    const auto phs = plan_phases(pd, g0, g1, M);
+    const auto phs = phases_cached(pd, g0, g1, M, false);
     const int nph = (int)phs.size();
     auto coalesced = [](const RpPhaseHost& h) {
         return h.b0 && h.lanes.size() >= 3 && h.lanes[0] == 1 && h.lanes[1] == 2 && h.lanes[2] == 3;
@@ -1259,7 +1279,7 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
     TileMap tm;
     tm.r = pd.r;
     for (int i = pd.r; i < T; ++i) tm.H.push_back(pd.S[i]);
-    const auto phs = plan_phases(pd, g0, g1, M, true);
+    const auto phs = phases_cached(pd, g0, g1, M, true);
     const int nph = (int)phs.size();
     const RpPhaseHost& lp = phs.back();
     const bool direct = lp.lanes.size() >= 3 && lp.lanes[0] == 0 && lp.lanes[1] == 1 && lp.lanes[2] == 2;
