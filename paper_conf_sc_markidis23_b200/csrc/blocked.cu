@@ -40,6 +40,9 @@
 #ifndef SVB_RP_DIRECT
 #define SVB_RP_DIRECT 1  // last phase stores registers straight to HBM when coalesced
 #endif
+#ifndef SVB_RP_CZBONUS
+#define SVB_RP_CZBONUS 1  // phase planning: prefer register sets holding both qubits of CZ-like gates
+#endif
 #ifndef SVB_RP_DLOAD
 #define SVB_RP_DLOAD 0  // first phase loads registers straight from HBM
 #endif
@@ -1052,16 +1055,25 @@ std::vector<RpPhaseHost> plan_phases(const PassDesc& pd, size_t g0, size_t g1, i
         }
         const size_t nr = rem.size();
         for (uint32_t R = (1u << M) - 1u; R < (1u << T);) {
-            int cnt = 0;
+            int cnt = 0, czin = 0;
             uint32_t blocked = 0;
             for (size_t i = 0; i < nr; ++i) {
                 const uint32_t m = rm[i];
-                if (!(m & blocked) && (ra[i] || !(m & ~R))) ++cnt;
-                else blocked |= m;
+                if (!(m & blocked) && (ra[i] || !(m & ~R))) {
+                    ++cnt;
+                    czin += ra[i] && !(m & ~R);
+                } else {
+                    blocked |= m;
+                }
             }
             // wide (16 B complex128 amplitudes): ties prefer R free of bits
-            // 0..2 (lanes 0..2 = bits 0..2: conflict-free, direct-store layout)
-            const int score = wide ? 4 * cnt + ((R & 0x7u) ? 0 : 1) : 4 * cnt + ((R & 1u) ? 2 : 0) + ((R & 0xEu) ? 0 : 1);
+            // 0..2 (lanes 0..2 = bits 0..2: conflict-free, direct-store layout).
+            // complex64: ties prefer more CZ-like gates with both qubits in R
+            // (sign bookkeeping in the pass kernels instead of FMUL2s by a
+            // per-thread sign), then tile bit 0 in R, then the direct layout
+            const int score = wide ? 4 * cnt + ((R & 0x7u) ? 0 : 1)
+                                   : 64 * cnt + 4 * std::min(czin, 15) * SVB_RP_CZBONUS + ((R & 1u) ? 2 : 0) +
+                                         ((R & 0xEu) ? 0 : 1);
             if (score > best) {
                 best = score;
                 used = R;

@@ -50,6 +50,9 @@
 #ifndef SVB_JIT_DB
 #define SVB_JIT_DB 0  // two tile buffers per CTA: the next tile loads during the whole current tile
 #endif
+#ifndef SVB_JIT_CZFOLD
+#define SVB_JIT_CZFOLD 1  // CZ sign flips on register bits as pending signs: 1 materialised at the phase end; 2 also folded into each register's last write (no change on the RQC: no sign is pending at a phase end)
+#endif
 #ifndef SVB_JIT_PL
 #define SVB_JIT_PL 0  // three quarters of the next tile land in a spare buffer during the whole current tile
 #endif
@@ -620,6 +623,37 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     // and per-lane negations that ptxas folds into the FADD2 / FFMA2 operand
     // modifiers (.LO_HI, .NP, -), so out = i^q (a0 + i^p a1) is one FADD2 and
     // a complex multiply s t = sr t + si (i t) one FMUL2 + one FFMA2
+    // pending signs (SVB_JIT_CZFOLD): register j holds sgn[j] ? -a_j : a_j.
+    // A CZ on two register bits only flips them; structured gates take the
+    // sign difference of their inputs into the rotation exponent (i^2 = -1)
+    // and pass the first input's sign on; dense gates whose inputs disagree
+    // materialise them first; every register is materialised at the end of
+    // the phase (FMUL2 by -1 where still pending).
+    std::vector<int> sgn(NA, 0);
+    auto materialize = [&](uint32_t j) {
+        if (!sgn[j]) return;
+        P.op("mul.rn.f32x2 %a", j, ", %a", j, ", %mneg1");
+        sgn[j] = 0;
+    };
+    // SVB_JIT_CZFOLD 2: a dry run of the phase records each register's last
+    // write (write events numbered in emission order) and its final pending
+    // sign; the real run negates that write instead (a rotation by i^2 in the
+    // operand modifiers: no extra instruction) when the sign would be pending
+    bool dry = false;
+    int wev = 0;
+    std::vector<int> lastw(NA, -1), need(NA, 0);
+    auto fold_out = [&](uint32_t j) -> bool {  // a foldable write of register j
+        const int e = wev++;
+        if (dry || SVB_JIT_CZFOLD < 2) {
+            lastw[j] = e;
+            return false;
+        }
+        return e == lastw[j] && need[j];
+    };
+    auto note_write = [&](uint32_t j) {  // a write that cannot take the sign
+        const int e = wev++;
+        if (dry) lastw[j] = e;
+    };
     int nrot = 0;
     auto rot = [&](const std::string& X, int k) -> std::string {
         k &= 3;
@@ -644,11 +678,11 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         const std::string x = rot(A, q), y = rot(B, p + q);
         P.op("add.rn.f32x2 ", d, ", ", x, ", ", y);
     };
-    // d = s t, s from slot (sr, sr, si, si); d may alias t
-    auto pmul = [&](const std::string& d, const std::string& t, size_t slot) {
+    // d = s t (neg: -s t), s from slot (sr, sr, si, si); d may alias t
+    auto pmul = [&](const std::string& d, const std::string& t, size_t slot, bool neg = false) {
         P.op("ld.param.v2.b64 {%qsr, %qsi}, [rpj_param_0+", 16 * slot, "]");
-        P.op("mul.rn.f32x2 %py, ", t, ", %qsr");
-        const std::string it = rot(t, 1);
+        P.op("mul.rn.f32x2 %py, ", rot(t, neg ? 2 : 0), ", %qsr");
+        const std::string it = rot(t, neg ? 3 : 1);
         P.op("fma.rn.f32x2 ", d, ", ", it, ", %qsi, %py");
     };
     auto emit_spec = [&](const GSpec& x, uint32_t mask, size_t base) {
@@ -659,14 +693,20 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             const uint32_t rest = ((1u << M) - 1u) & ~mask;
             for (uint32_t gi = 0; gi < (uint32_t)NA / 4; ++gi) {
                 const uint32_t b0 = pdep(gi, rest);
+                int s_in[4];
+                for (int c = 0; c < 4; ++c) s_in[c] = sgn[b0 | pdep(c, mask)];
+                for (int r = 0; r < 4; ++r) sgn[b0 | pdep(r, mask)] = s_in[x.perm[r]];
                 for (int c = 0; c < 4; ++c) P.op("mov.b64 %x", c, ", %a", b0 | pdep(c, mask));
                 for (int r = 0; r < 4; ++r) {
-                    const std::string d = "%a" + std::to_string(b0 | pdep(r, mask));
+                    const uint32_t jr = b0 | pdep(r, mask);
+                    const std::string d = "%a" + std::to_string(jr);
                     const std::string src = "%x" + std::to_string(x.perm[r]);
+                    const bool ng = fold_out(jr);
+                    if (ng) sgn[jr] ^= 1;
                     if (!x.munit[r]) {
-                        pmul(d, src, slr[r]);
-                    } else if (x.mq[r] & 3) {
-                        const std::string t = rot(src, x.mq[r]);
+                        pmul(d, src, slr[r], ng);
+                    } else if ((x.mq[r] + (ng ? 2 : 0)) & 3) {
+                        const std::string t = rot(src, x.mq[r] + (ng ? 2 : 0));
                         P.op("mul.rn.f32x2 ", d, ", ", t, ", %pone");
                     } else {
                         P.op("mov.b64 ", d, ", ", src);
@@ -682,9 +722,13 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                 const int r = (j & mask) ? 1 : 0;
                 const std::string a = "%a" + std::to_string(j);
                 if (!x.unit[r]) {
-                    pmul(a, a, sl[r]);
+                    const bool ng = fold_out(j);
+                    if (ng) sgn[j] ^= 1;
+                    pmul(a, a, sl[r], ng);
                 } else if (x.q[r]) {  // i^q a (one FMUL2 by 1 carries the rotation)
-                    const std::string t = rot(a, x.q[r]);
+                    const bool ng = fold_out(j);
+                    if (ng) sgn[j] ^= 1;
+                    const std::string t = rot(a, x.q[r] + (ng ? 2 : 0));
                     P.op("mul.rn.f32x2 ", a, ", ", t, ", %pone");
                 }
             }
@@ -694,19 +738,26 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             if (j0 & mask) continue;
             const uint32_t j1 = j0 | mask;
             const std::string a0 = "%a" + std::to_string(j0), a1 = "%a" + std::to_string(j1);
+            // stored a1 = (-1)^(sgn1 - sgn0) relative to a0: a rotation by i^2
+            const int dz = (sgn[j0] ^ sgn[j1]) ? 2 : 0;
+            sgn[j1] = sgn[j0];  // both outputs carry the first input's sign
+            const bool n0 = fold_out(j0), n1 = fold_out(j1);
+            if (n0) sgn[j0] ^= 1;
+            if (n1) sgn[j1] ^= 1;
+            const int z[2] = {n0 ? 2 : 0, n1 ? 2 : 0};
             if (x.cls == 2) {  // out0 = a0 + mu a1, out1 = i^p0 a0 + i^p1 (mu a1)
                 pmul("%pt", a1, sl[0]);
-                plin("%po0", 0, 0, a0, "%pt");
-                const std::string u = rot(a0, x.p[0]), v = rot("%pt", x.p[1]);
+                plin("%po0", z[0], dz, a0, "%pt");
+                const std::string u = rot(a0, x.p[0] + z[1]), v = rot("%pt", x.p[1] + dz + z[1]);
                 P.op("add.rn.f32x2 %po1, ", u, ", ", v);
             } else {  // row form: out_r = s_r (a0 + i^p_r a1)
                 for (int r = 0; r < 2; ++r) {
                     const std::string d = "%po" + std::to_string(r);
                     if (x.unit[r]) {
-                        plin(d, x.q[r], x.p[r], a0, a1);
+                        plin(d, x.q[r] + z[r], x.p[r] + dz, a0, a1);
                     } else {
-                        plin("%pt", 0, x.p[r], a0, a1);
-                        pmul(d, "%pt", sl[r]);
+                        plin("%pt", 0, x.p[r] + dz, a0, a1);
+                        pmul(d, "%pt", sl[r], z[r] != 0);
                     }
                 }
             }
@@ -1067,77 +1118,119 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
             loadtile("%gnext", "@%p_next ", "%cur", pl ? 8u : 15u);
             P.op("cp.async.commit_group");
         }
+        auto gates_body = [&]() {
         for (int g : Ph.gates) {
-            const PassGate& pg = pd.gates[g];
-            const int kind = gate_kind(pd, pg);
-            uint32_t mask = 0, tmask = 0;
-            for (int b = 0; b < pg.k; ++b) {
-                const auto it = std::find(Ph.R.begin(), Ph.R.end(), pg.pos[b]);
-                if (it != Ph.R.end()) mask |= 1u << (int)(it - Ph.R.begin());
-                else tmask |= 1u << (int)(std::find(Ph.lanes.begin(), Ph.lanes.end(), pg.pos[b]) - Ph.lanes.begin());
-            }
-            const int D = 1 << pg.k;
-            P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask
-                << " cls=" << cs.g[g].cls << "\n";
-            if (cs.g[g].cls) {
-                emit_spec(cs.g[g], mask, gbase[g]);
-                continue;
-            }
-            if (kind == 2) {  // CZ-like: sign flips of both halves
-                // one FMUL2 per flipped amplitude (2 LOP3s as an xor), by -1
-                // or, when a qubit is a thread bit, by this thread's sign
-                std::string sg = "%mneg1";
-                if (popc(mask) != 2) {
-                    const std::string t = P.r32(), q = P.pr();
-                    P.op("and.b32 ", t, ", %t_id, ", tmask);
-                    P.op("setp.eq.u32 ", q, ", ", t, ", ", tmask);
-                    P.op("selp.b64 %csg, %mneg1, %pone, ", q);
-                    sg = "%csg";
+                const PassGate& pg = pd.gates[g];
+                const int kind = gate_kind(pd, pg);
+                uint32_t mask = 0, tmask = 0;
+                for (int b = 0; b < pg.k; ++b) {
+                    const auto it = std::find(Ph.R.begin(), Ph.R.end(), pg.pos[b]);
+                    if (it != Ph.R.end()) mask |= 1u << (int)(it - Ph.R.begin());
+                    else tmask |= 1u << (int)(std::find(Ph.lanes.begin(), Ph.lanes.end(), pg.pos[b]) - Ph.lanes.begin());
                 }
-                for (uint32_t j = 0; j < (uint32_t)NA; ++j)
-                    if ((j & mask) == mask) P.op("mul.rn.f32x2 %a", j, ", %a", j, ", ", sg);
-                continue;
-            }
-            const size_t base = gbase[g];
-            auto mload = [&](size_t e) {  // (mr, mr) -> %ml, (-mi, mi) -> %mh
-                P.op("ld.param.v2.b64 {%ml, %mh}, [rpj_param_0+", 16 * e, "]");
-            };
-            auto swp = [&](const std::string& x, const std::string& out) {
-                P.op("mov.b64 {%lo, %hi}, ", x);
-                P.op("mov.b64 ", out, ", {%hi, %lo}");
-            };
-            if (kind == 1) {
-                for (int e = 0; e < D; ++e) {
-                    mload(base + e);
-                    for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
-                        if (pext(j, mask) != (uint32_t)e) continue;
-                        swp("%a" + std::to_string(j), "%xs0");
-                        P.op("fma.rn.f32x2 %y, %ml, %a", j, ", %zero");
-                        P.op("fma.rn.f32x2 %a", j, ", %mh, %xs0, %y");
+                const int D = 1 << pg.k;
+                P.o << "\t// gate " << g << ": k=" << pg.k << " kind=" << kind << " mask=" << mask << " tmask=" << tmask
+                    << " cls=" << cs.g[g].cls << "\n";
+                if (cs.g[g].cls) {
+                    emit_spec(cs.g[g], mask, gbase[g]);
+                    continue;
+                }
+                if (kind == 2) {  // CZ-like: sign flips of both halves
+                    // one FMUL2 per flipped amplitude (2 LOP3s as an xor), by -1
+                    // or, when a qubit is a thread bit, by this thread's sign
+                    std::string sg = "%mneg1";
+                    if (popc(mask) != 2) {
+                        const std::string t = P.r32(), q = P.pr();
+                        P.op("and.b32 ", t, ", %t_id, ", tmask);
+                        P.op("setp.eq.u32 ", q, ", ", t, ", ", tmask);
+                        P.op("selp.b64 %csg, %mneg1, %pone, ", q);
+                        sg = "%csg";
                     }
+                    for (uint32_t j = 0; j < (uint32_t)NA; ++j)
+                        if ((j & mask) == mask) {
+                            if (SVB_JIT_CZFOLD && popc(mask) == 2) {
+                                sgn[j] ^= 1;
+                            } else {
+                                const bool ng = fold_out(j);
+                                if (ng) sgn[j] ^= 1;
+                                const std::string a = "%a" + std::to_string(j);
+                                P.op("mul.rn.f32x2 ", a, ", ", ng ? rot(a, 2) : a, ", ", sg);
+                            }
+                        }
+                    continue;
                 }
-                continue;
-            }
-            const uint32_t rest = ((1u << M) - 1u) & ~mask;
-            for (uint32_t gi = 0; gi < (uint32_t)NA / D; ++gi) {
-                const uint32_t b0 = pdep(gi, rest);
-                for (int c = 0; c < D; ++c) {
-                    P.op("mov.b64 %x", c, ", %a", b0 | pdep(c, mask));
-                    swp("%x" + std::to_string(c), "%xs" + std::to_string(c));
+                const size_t base = gbase[g];
+                auto mload = [&](size_t e) {  // (mr, mr) -> %ml, (-mi, mi) -> %mh
+                    P.op("ld.param.v2.b64 {%ml, %mh}, [rpj_param_0+", 16 * e, "]");
+                };
+                auto swp = [&](const std::string& x, const std::string& out) {
+                    P.op("mov.b64 {%lo, %hi}, ", x);
+                    P.op("mov.b64 ", out, ", {%hi, %lo}");
+                };
+                if (kind == 1) {
+                    for (int e = 0; e < D; ++e) {
+                        mload(base + e);
+                        for (uint32_t j = 0; j < (uint32_t)NA; ++j) {
+                            if (pext(j, mask) != (uint32_t)e) continue;
+                            swp("%a" + std::to_string(j), "%xs0");
+                            P.op("fma.rn.f32x2 %y, %ml, %a", j, ", %zero");
+                            P.op("fma.rn.f32x2 %a", j, ", %mh, %xs0, %y");
+                            note_write(j);
+                        }
+                    }
+                    continue;
                 }
-                for (int rr = 0; rr < D; ++rr) {
-                    const uint32_t dst = b0 | pdep(rr, mask);
+                const uint32_t rest = ((1u << M) - 1u) & ~mask;
+                for (uint32_t gi = 0; gi < (uint32_t)NA / D; ++gi) {
+                    const uint32_t b0 = pdep(gi, rest);
+                    // a common input sign passes to the outputs; mixed signs are materialised
+                    bool same = true;
+                    for (int c = 1; c < D; ++c) same = same && sgn[b0 | pdep(c, mask)] == sgn[b0];
+                    if (!same)
+                        for (int c = 0; c < D; ++c) materialize(b0 | pdep(c, mask));
                     for (int c = 0; c < D; ++c) {
-                        mload(base + rr * D + c);
-                        P.op("fma.rn.f32x2 %y, %ml, %x", c, ", ", c == 0 ? "%zero" : "%y");
-                        P.op("fma.rn.f32x2 ", c == D - 1 ? "%a" + std::to_string(dst) : std::string("%y"), ", %mh, %xs", c,
-                             ", %y");
+                        P.op("mov.b64 %x", c, ", %a", b0 | pdep(c, mask));
+                        swp("%x" + std::to_string(c), "%xs" + std::to_string(c));
+                    }
+                    for (int rr = 0; rr < D; ++rr) {
+                        const uint32_t dst = b0 | pdep(rr, mask);
+                        note_write(dst);
+                        for (int c = 0; c < D; ++c) {
+                            mload(base + rr * D + c);
+                            P.op("fma.rn.f32x2 %y, %ml, %x", c, ", ", c == 0 ? "%zero" : "%y");
+                            P.op("fma.rn.f32x2 ", c == D - 1 ? "%a" + std::to_string(dst) : std::string("%y"), ", %mh, %xs", c,
+                                 ", %y");
+                        }
                     }
                 }
             }
+            if (last && cs.mode == 4)  // the pass scalar, explicitly
+                for (int j = 0; j < NA; ++j) {
+                    const bool ng = fold_out((uint32_t)j);
+                    if (ng) sgn[j] ^= 1;
+                    pmul("%a" + std::to_string(j), "%a" + std::to_string(j), cslot, ng);
+                }
+        };
+        if (SVB_JIT_CZFOLD >= 2) {  // dry run: last writes and final signs
+            const std::string saved = P.o.str();
+            const int snr = P.nr, snrd = P.nrd, snp = P.np, srot = nrot;
+            dry = true;
+            wev = 0;
+            std::fill(lastw.begin(), lastw.end(), -1);
+            gates_body();
+            need = sgn;
+            P.o.str(saved);
+            P.o.seekp(0, std::ios_base::end);
+            P.nr = snr;
+            P.nrd = snrd;
+            P.np = snp;
+            nrot = srot;
+            dry = false;
+            wev = 0;
+            std::fill(sgn.begin(), sgn.end(), 0);
         }
-        if (last && cs.mode == 4)  // the pass scalar, explicitly
-            for (int j = 0; j < NA; ++j) pmul("%a" + std::to_string(j), "%a" + std::to_string(j), cslot);
+        gates_body();
+        for (int j = 0; j < NA; ++j) materialize((uint32_t)j);  // the phase's stores see true values
         if (last && direct) {
             P.op("add.s64 %gst, %gtile, %dg");
             if (lp.b0) {
