@@ -623,7 +623,9 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
     // and per-lane negations that ptxas folds into the FADD2 / FFMA2 operand
     // modifiers (.LO_HI, .NP, -), so out = i^q (a0 + i^p a1) is one FADD2 and
     // a complex multiply s t = sr t + si (i t) one FMUL2 + one FFMA2
-    // pending signs (SVB_JIT_CZFOLD): register j holds sgn[j] ? -a_j : a_j.
+    // pending signs (SVB_JIT_CZFOLD, structured path only: with
+    // SV_OPT_PASS_SPEC 0 the kernels stay bit-identical to the generic one,
+    // which a negated zero would break): register j holds sgn[j] ? -a_j : a_j.
     // A CZ on two register bits only flips them; structured gates take the
     // sign difference of their inputs into the rotation exponent (i^2 = -1)
     // and pass the first input's sign on; dense gates whose inputs disagree
@@ -1148,7 +1150,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
                     }
                     for (uint32_t j = 0; j < (uint32_t)NA; ++j)
                         if ((j & mask) == mask) {
-                            if (SVB_JIT_CZFOLD && popc(mask) == 2) {
+                            if (SVB_JIT_CZFOLD && pd.spec && popc(mask) == 2) {
                                 sgn[j] ^= 1;
                             } else {
                                 const bool ng = fold_out(j);
