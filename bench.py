@@ -337,7 +337,9 @@ def run_reference(args):
            "steps_requested": args.steps}
     cpu = {"value": v, "unit": "s", "kind": "oracle", "extrapolated": True,
            "sample": f"{steps} gates in {wall:.1f} s ({len(smp.t[1])} one-qubit, {len(smp.t[2])} two-qubit); "
-                     f"{cnt[1]} x {mean[1] and mean[1] * 1e3:.1f} ms + {cnt[2]} x {mean[2] and mean[2] * 1e3:.1f} ms"
+                     + (f"{cnt[1]} x {mean[1] * 1e3:.1f} ms + {cnt[2]} x {mean[2] * 1e3:.1f} ms"
+                        if mean[1] is not None and mean[2] is not None else
+                        f"{cnt[1] + cnt[2]} gates x {v / scale / max(1, cnt[1] + cnt[2]) * 1e3:.1f} ms (mean over both sizes)")
                      + (f" on {n_eff} qubits x{scale:.0f} (2^{n - n_eff}: host RAM too small for 2^{n} complex128)"
                         if scale > 1 else "")}
     cpu.update(host_info())
