@@ -1,4 +1,6 @@
-O=gpurun_out/mr; mkdir -p $O
-timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29655 bench.py --gpus 2 --qubits 28 --depth 14 --steps 2 --warmup 1 > $O/b2.json 2> $O/b2.err; tail -1 $O/b2.json | cut -c1-700; tail -3 $O/b2.err
-timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 4 --master-addr 127.0.0.1 --master-port 29656 bench.py --gpus 4 --qubits 28 --depth 20 --steps 2 --warmup 1 > $O/b4.json 2> $O/b4.err; tail -1 $O/b4.json | cut -c1-700; tail -3 $O/b4.err
-timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29657 bench.py --impl reference --gpus 2 --steps 3 --warmup 1 > $O/r2.json 2> $O/r2.err; tail -1 $O/r2.json | cut -c1-300
+O=gpurun_out/anyd; mkdir -p $O
+V=paper_conf_sc_markidis23_b200/_variants
+timeout 600 python tools/ab_step.py 3 $V/libsvb200_cur.so $V/libsvb200_anyd.so > $O/ab30.txt 2>&1; cat $O/ab30.txt
+AB_N=32 AB_D=20 timeout 900 python tools/ab_step.py 2 $V/libsvb200_cur.so $V/libsvb200_anyd.so > $O/ab32.txt 2>&1; cat $O/ab32.txt
+AB_PIN=3 timeout 600 python tools/ab_step.py 1 $V/libsvb200_cur.so $V/libsvb200_anyd.so > $O/ab30p3.txt 2>&1; cat $O/ab30p3.txt
+SVB200_LIB=$PWD/$V/libsvb200_anyd.so timeout 900 python -m pytest tests/test_gpu_jit.py -q -k "oracle or spec or tile14 or bins" > $O/pytest.log 2>&1; tail -3 $O/pytest.log

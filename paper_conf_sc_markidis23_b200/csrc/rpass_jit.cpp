@@ -35,6 +35,9 @@
 #ifndef SVB_JIT_SECTOR_DIRECT
 #define SVB_JIT_SECTOR_DIRECT 1  // direct stores also for 32 B-sector layouts of the last phase
 #endif
+#ifndef SVB_JIT_ANY_DIRECT
+#define SVB_JIT_ANY_DIRECT 0  // the last phase always stores straight to HBM, any layout (measured: 30q 23.5 -> 27.2 ms: scattered 8/16 B stores)
+#endif
 #ifndef SVB_JIT_M
 #define SVB_JIT_M 5  // log2 amplitudes per thread of the complex64 pass kernels (4: 16 per thread, 64 registers)
 #endif
@@ -464,7 +467,7 @@ std::string gen_chunk(const PassDesc& pd, int n_local, size_t g0, size_t g1, boo
         return h.b0 ? (h.lanes.size() >= 1 && h.lanes[0] == 1)
                     : (h.lanes.size() >= 2 && h.lanes[0] == 0 && h.lanes[1] == 1);
     };
-    const bool direct = coalesced(lp) || coalesced8(lp) || (SVB_JIT_SECTOR_DIRECT && sector(lp));
+    const bool direct = coalesced(lp) || coalesced8(lp) || (SVB_JIT_SECTOR_DIRECT && sector(lp)) || SVB_JIT_ANY_DIRECT;
     const bool early = direct && !zinit;
     // sampling bin weights (the last launch of a circuit's last pass): 16-
     // amplitude bins = tile bits 0..3, reduced over the lanes that hold them
