@@ -41,6 +41,10 @@
 #ifndef SVB_JIT_M
 #define SVB_JIT_M 5  // log2 amplitudes per thread of the complex64 pass kernels (4: 16 per thread, 64 registers)
 #endif
+#ifndef SVB_JIT_M64
+#define SVB_JIT_M64 5  // log2 amplitudes per thread of the complex128 pass kernels for 13-qubit tiles (32: 256 threads,
+                       // <= 255 registers; 30q D14 59.3 -> 54.4 ms); 12-qubit and smaller tiles keep 16 per thread
+#endif
 #ifndef SVB_JIT_M14
 #define SVB_JIT_M14 6  // ... for 14-qubit tiles: 64 per thread (256 threads, <= 255 registers, 8 warps per SM)
 #endif
@@ -117,7 +121,7 @@ bool monomial2(const PassDesc& pd, const PassGate& pg, int perm[4], std::complex
     return true;
 }
 int jit_m(const PassDesc& pd) {
-    if (pd.wide) return 4;
+    if (pd.wide) return pd.S.size() >= 13 ? SVB_JIT_M64 : 4;
     if (pd.S.size() < 14 || pd.r < SVB_JIT_M14_RUN) return SVB_JIT_M;
     int perm[4];
     std::complex<double> m[4];
@@ -1370,7 +1374,7 @@ uint32_t fold64(uint32_t t, int T) {
 
 std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, bool zinit, size_t& nm,
                         std::vector<double>& mats, bool emit = true) {
-    constexpr int M = 4, NA = 16, UPT = 16;
+    const int M = jit_m(pd), NA = 1 << M, UPT = NA;
     const int T = (int)pd.S.size();
     const int tbits = T - M;
     const uint32_t nthr = 1u << tbits;
@@ -1789,11 +1793,11 @@ std::string gen_chunk64(const PassDesc& pd, int n_local, size_t g0, size_t g1, b
     k << ".version 8.8\n.target sm_100a\n.address_size 64\n";
     k << ".extern .shared .align 16 .b8 rsm[];\n";
     k << ".visible .entry rpj(.param .align 16 .b8 rpj_param_0[" << pbytes << "])\n";
-    k << ".maxntid " << nthr << ", 1, 1\n.maxnreg 128\n{\n";
+    k << ".maxntid " << nthr << ", 1, 1\n.maxnreg " << (M >= 5 ? 255 : 128) << "\n{\n";
     k << "\t.reg .pred %p<" << std::max(P.np, 1) << ">;\n\t.reg .pred %p_out, %p_next, %p_z;\n";
     k << "\t.reg .b32 %r<" << std::max(P.nr, 1) << ">;\n\t.reg .b32 %t_id, %cur, %sthr, %tb, %zone, %r_c, %h1;\n";
     k << "\t.reg .b64 %rd<" << std::max(P.nrd, 1) << ">;\n";
-    k << "\t.reg .f64 %ar<16>, %ai<16>, %xr<4>, %xi<4>, %yr, %yi, %mr, %mi, %nmi, %t0, %t1, %t2, %tfr, %tfi, %zr, %zi, "
+    k << "\t.reg .f64 %ar<" << NA << ">, %ai<" << NA << ">, %xr<4>, %xi<4>, %yr, %yi, %mr, %mi, %nmi, %t0, %t1, %t2, %tfr, %tfi, %zr, %zi, "
          "%ptr, %pti, %por<2>, %poi<2>;\n";
     k << "\t.reg .b64 %dthr, %dg, %psi, %ntiles, %u, %un, %grid, %tbo, %gtile, %gcur, %gtile_next, %gnext, %gst, "
          "%tabA, %tabB, %rdB;\n";
@@ -1865,7 +1869,8 @@ int rpass_jit_prepare(const PassDesc& pd, int n_local, bool zinit, bool compile,
         for (const auto& ch : jit_chunks(pd)) {
             RpJitLaunch l;
             size_t nm = 0;
-            const std::string src = gen_chunk(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats);
+            const std::string src = pd.wide ? gen_chunk64(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats64)
+                                            : gen_chunk(pd, n_local, ch.first, ch.second, zinit && first, nm, l.mats);
             if (sources) sources->push_back(src);
             l.c0 = ch.first;
             l.c1 = ch.second;
