@@ -573,14 +573,14 @@ def run_ours(args):
         micro = exchange_micro(sv, h, n, world, cdev)
 
     # ---- end-to-end through the public API with host buffers
-    host_samples = np.empty(args.samples, dtype=np.uint64)
+    # the step's result lands in pinned host memory (the D2H of the e2e step)
+    host_samples = torch.empty(args.samples, dtype=torch.int64, pin_memory=True).numpy().view(np.uint64)
     g_arr = sv.as_gates(gates)
 
     def e2e_step():
         sv.sv_reset(h)
         sv.sv_run_circuit(h, g_arr, args.max_fused)
-        out = sv.sv_sample(h, 1, args.samples)
-        host_samples[:] = out
+        sv.sv_sample(h, 1, args.samples, out=host_samples)
 
     e2e_step()
     barrier()

@@ -292,8 +292,14 @@ def sv_amplitudes_c128(h: int, idx) -> np.ndarray:
     return out
 
 
-def sv_sample(h: int, seed: int, n_samples: int) -> np.ndarray:
-    out = np.empty(n_samples, dtype=np.uint64)
+def sv_sample(h: int, seed: int, n_samples: int, out=None) -> np.ndarray:
+    """n_samples logical bitstrings; `out` (optional): a caller-owned contiguous
+    uint64 array of at least n_samples entries (e.g. pinned host memory) to
+    receive them."""
+    if out is None:
+        out = np.empty(n_samples, dtype=np.uint64)
+    elif out.dtype != np.uint64 or not out.flags["C_CONTIGUOUS"] or out.size < n_samples:
+        raise ValueError("out must be a contiguous uint64 array of at least n_samples entries")
     _check(lib().sv_sample(h, seed, n_samples, out.ctypes.data_as(_u64p)), "sv_sample")
     return out
 

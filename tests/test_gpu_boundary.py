@@ -122,3 +122,21 @@ def test_async_staging_ring(k, qs):
     for M in Ms:
         ref = osv.apply_gate(ref, n, list(qs), M.astype(np.complex128))
     assert osv.fidelity(got, ref) >= 1 - 1e-5 and np.abs(got - ref).max() < 1e-5
+
+
+def test_sample_into_caller_buffer():
+    """sv_sample writes into a caller-owned (here pinned) host buffer: the same
+    bitstrings as into a fresh array; a short buffer is rejected."""
+    import torch
+    n = 14
+    h = sv.sv_create(n)
+    try:
+        sv.sv_set_state(h, W.random_state_c64(n, 5))
+        ref = sv.sv_sample(h, 9, 5000)
+        buf = torch.empty(5000, dtype=torch.int64, pin_memory=True).numpy().view(np.uint64)
+        got = sv.sv_sample(h, 9, 5000, out=buf)
+        assert got is buf and np.array_equal(buf, ref)
+        with pytest.raises(ValueError):
+            sv.sv_sample(h, 9, 5000, out=np.empty(10, dtype=np.uint64))
+    finally:
+        sv.sv_destroy(h)
