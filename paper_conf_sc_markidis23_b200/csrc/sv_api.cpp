@@ -737,7 +737,10 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
         }
         return cnt;
     };
-    auto grow = [&](size_t i0, const std::vector<char>& pl, int B, std::vector<uint64_t>& finals) {
+    // ties between additions that absorb as many gates with as many qubits:
+    // the earlier candidate (value_ties false) or the smaller qubit mask
+    auto grow = [&](size_t i0, const std::vector<char>& pl, int B, std::vector<uint64_t>& finals,
+                    bool value_ties = false) {
         std::vector<uint64_t> states{fm[i0] & ~pin};
         std::vector<char> in_cur(nf, 0);
         while (!states.empty()) {
@@ -760,8 +763,10 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
                     const size_t c = absorb(i0, Qs | cands[o], pl, nullptr);
                     if (c > have) sc.push_back({c, __builtin_popcountll(cands[o]), o, cands[o]});
                 }
-                std::sort(sc.begin(), sc.end(), [](const Sc& a, const Sc& b) {
-                    return a.c != b.c ? a.c > b.c : a.bits != b.bits ? a.bits < b.bits : a.ord < b.ord;
+                std::sort(sc.begin(), sc.end(), [&](const Sc& a, const Sc& b) {
+                    if (a.c != b.c) return a.c > b.c;
+                    if (a.bits != b.bits) return a.bits < b.bits;
+                    return value_ties ? a.add < b.add : a.ord < b.ord;
                 });
                 if (sc.empty()) {
                     if (std::find(finals.begin(), finals.end(), Qs) == finals.end()) finals.push_back(Qs);
@@ -776,12 +781,12 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
             states.swap(nxt);
         }
     };
-    auto greedy_rest = [&](std::vector<char> pl) {
+    auto greedy_rest = [&](std::vector<char> pl, bool value_ties) {
         int n = 0;
         for (size_t i0 = 0; i0 < nf; ++i0) {
             if (pl[i0]) continue;
             std::vector<uint64_t> f;
-            grow(i0, pl, 1, f);
+            grow(i0, pl, 1, f, value_ties);
             std::vector<size_t> m;
             absorb(i0, f[0], pl, &m);
             for (size_t j : m) pl[j] = 1;
@@ -805,33 +810,51 @@ std::vector<PassDesc> build_passes(int T, const std::vector<PassIn>& in, int kPa
             }
         }
         if (!hit) {
-            std::vector<char> pl(nf, 0);
-            for (size_t i0 = 0; i0 < nf; ++i0) {
-                if (pl[i0]) continue;
-                std::vector<uint64_t> finals;
-                grow(i0, pl, std::max(1, beam), finals);
-                uint64_t Qb = finals[0];
-                if (finals.size() > 1) {
-                    int best_n = 1 << 30;
-                    size_t best_c = 0;
-                    for (uint64_t Qf : finals) {
-                        std::vector<char> p2 = pl;
-                        std::vector<size_t> m;
-                        const size_t c = absorb(i0, Qf, p2, &m);
-                        for (size_t j : m) p2[j] = 1;
-                        const int nrest = greedy_rest(p2);
-                        if (nrest < best_n || (nrest == best_n && c > best_c)) {
-                            best_n = nrest;
-                            best_c = c;
-                            Qb = Qf;
+            // one formation per tie policy (policy 2: both tie orders'
+            // candidates, optimistic rollouts); the plan with the fewest passes
+            // wins (ties: the earlier policy).  The search is sensitive to
+            // ties: 30q D14 from |0...0> gives 6 passes with one order, 5 with
+            // the other.
+            auto formation = [&](int policy) {
+                std::vector<uint64_t> fs;
+                std::vector<char> pl(nf, 0);
+                const bool vt = policy == 1;
+                for (size_t i0 = 0; i0 < nf; ++i0) {
+                    if (pl[i0]) continue;
+                    std::vector<uint64_t> finals;
+                    grow(i0, pl, std::max(1, beam), finals, vt);
+                    if (beam > 1 && policy == 2) grow(i0, pl, beam, finals, true);
+                    uint64_t Qb = finals[0];
+                    if (finals.size() > 1) {
+                        int best_n = 1 << 30;
+                        size_t best_c = 0;
+                        for (uint64_t Qf : finals) {
+                            std::vector<char> p2 = pl;
+                            std::vector<size_t> m;
+                            const size_t c = absorb(i0, Qf, p2, &m);
+                            for (size_t j : m) p2[j] = 1;
+                            const int nrest = policy == 2 ? std::min(greedy_rest(p2, false), greedy_rest(p2, true))
+                                                          : greedy_rest(p2, vt);
+                            if (nrest < best_n || (nrest == best_n && c > best_c)) {
+                                best_n = nrest;
+                                best_c = c;
+                                Qb = Qf;
+                            }
                         }
                     }
+                    std::vector<size_t> m;
+                    absorb(i0, Qb, pl, &m);
+                    for (size_t j : m) pl[j] = 1;
+                    fs.push_back(Qb);
                 }
-                std::vector<size_t> m;
-                absorb(i0, Qb, pl, &m);
-                for (size_t j : m) pl[j] = 1;
-                forms.push_back(Qb);
-            }
+                return fs;
+            };
+            forms = formation(0);
+            if (beam > 1)
+                for (int policy = 1; policy <= 2; ++policy) {
+                    std::vector<uint64_t> f2 = formation(policy);
+                    if (f2.size() < forms.size()) forms.swap(f2);
+                }
             std::lock_guard<std::mutex> lk(g_form_mu);
             if (g_form_cache.size() > 256) g_form_cache.clear();
             g_form_cache[key] = forms;

@@ -1,5 +1,5 @@
 """Interleaved A/B of the bench step (reset + circuit + 10^6 samples; host wall time, mean of 10)
-across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3 AB_T=12 AB_F=1 AB_WL=rqc|sycamore] python tools/ab_step.py <rounds> <lib.so> ...
+across library builds.  usage: [AB_N=30 AB_D=14 AB_PIN=3 AB_T=12 AB_F=1 AB_WL=rqc|sycamore AB_BEAM=1..8] python tools/ab_step.py <rounds> <lib.so> ...
 """
 import json, os, subprocess, sys
 CHILD = r'''
@@ -13,6 +13,7 @@ n=int(os.environ.get("AB_N", "30")); d=int(os.environ.get("AB_D", "14"))
 h=sv.sv_create(n)
 if os.environ.get("AB_PIN"): sv.sv_set_option(h, sv.SV_OPT_PASS_PIN, int(os.environ["AB_PIN"]))
 if os.environ.get("AB_T"): sv.sv_set_blocking(h, int(os.environ["AB_T"]))
+if os.environ.get("AB_BEAM"): sv.sv_set_option(h, sv.SV_OPT_PASS_SEARCH, int(os.environ["AB_BEAM"]))
 F=int(os.environ.get("AB_F", "1"))
 gates=W.sycamore_rqc(n,d) if os.environ.get("AB_WL")=="sycamore" else W.rqc(n,d)
 c=sv.sv_circuit_create(h, gates, F)
@@ -24,7 +25,7 @@ sv.sv_synchronize(h)
 t0=time.perf_counter()
 for _ in range(10): step()
 sv.sv_synchronize(h)
-print(json.dumps({"step_ms": (time.perf_counter()-t0)/10*1e3}))
+print(json.dumps({"step_ms": (time.perf_counter()-t0)/10*1e3, "passes": sv.sv_last_stats(h)["n_passes"]}))
 '''
 libs = sys.argv[2:]
 for r in range(int(sys.argv[1])):
