@@ -1,3 +1,4 @@
-O=gpurun_out/p0b; mkdir -p $O
-timeout 1500 python -m pytest tests/test_gpu_jit.py tests/test_gpu_circuit.py tests/test_gpu_fullsize.py -x -q > $O/pytest.log 2>&1; tail -2 $O/pytest.log
-timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; tail -1 $O/bench.json | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['value'], d['e2e']['value'], d['roofline']['frac'], d['roofline']['alu']['frac'], d['roofline']['pass_floor']['frac'], d['config']['execution'][-45:])"
+O=gpurun_out/bm5; mkdir -p $O
+V=paper_conf_sc_markidis23_b200/_variants
+timeout 600 python tools/ab_step.py 3 $V/libsvb200_cur.so $V/libsvb200_bm5.so > $O/ab30.txt 2>&1; cat $O/ab30.txt
+AB_N=32 AB_D=20 timeout 900 python tools/ab_step.py 1 $V/libsvb200_cur.so $V/libsvb200_bm5.so > $O/ab32.txt 2>&1; cat $O/ab32.txt

@@ -51,6 +51,9 @@
 #ifndef SVB_JIT_P0_M
 #define SVB_JIT_P0_M 5  // the compute-bound product-state first pass keeps 32 per thread (16 warps per SM: 30q 21.52 -> 21.0 ms)
 #endif
+#ifndef SVB_JIT_BINS_M
+#define SVB_JIT_BINS_M 0  // nonzero: log2 amplitudes per thread of the circuit's last pass (it writes the bins)
+#endif
 #ifndef SVB_JIT_M14_RUN
 #define SVB_JIT_M14_RUN 4  // ... when the tile's runs are >= 2^this amplitudes
 #endif
@@ -131,6 +134,7 @@ int jit_m(const PassDesc& pd) {
     for (const auto& g : pd.gates)
         if (g.k == 2 && gate_kind(pd, g) == 0 && !monomial2(pd, g, perm, m)) return SVB_JIT_M;
     if (SVB_JIT_P0_M && !pd.pinit_v.empty()) return SVB_JIT_P0_M;  // product-state first pass
+    if (SVB_JIT_BINS_M && pd.bins) return SVB_JIT_BINS_M;  // the last pass (sampler bins)
     return SVB_JIT_M14;
 }
 
